@@ -1,0 +1,347 @@
+"""GEM hot-path benchmark (driver contract).
+
+  python bench.py [--gpus N] [--steps K] [--warmup W] [--impl gem|reference]
+                  [--workload c3] [--streams S] [--cycles C]
+
+A "step" = one gem_step over C simulated cycles (default 1000) of the whole
+hot path (global read, layers, endpoint commit, RAM, grid barriers) for S
+streams per GPU of the workload netlist (default C3: ~1M live ANDs, 32K
+flops, 2 RAM blocks; BASELINE.json metric "simulated cycles/sec at 1M AIG
+nodes").  value = simulated stream-cycles/s summed over all ranks (weak
+scaling: each rank simulates its own streams; N>1 adds the NCCL gather of the
+PO traces to rank 0 inside every step).
+
+The L2 (126 MB) is flushed between timed steps by writing a 512 MB buffer
+(the C3 program, ~36 MB, would otherwise stay L2-resident across steps).
+"""
+from __future__ import annotations
+
+import argparse
+import json
+import os
+import subprocess
+import sys
+import threading
+import time
+
+import numpy as np
+
+ROOT = os.path.dirname(os.path.abspath(__file__))
+sys.path.insert(0, ROOT)
+
+METRIC = "simulated cycles/sec at 1M AIG nodes (1 B200); gate-evals/s; batched 1/2/4/8 GPU"
+UNIT = "cycles/s"
+PEAKS_FALLBACK = {"hbm_gbs": 6650.0, "sm_max_mhz": 1965.0}
+
+
+def _peaks():
+    p = os.path.join(ROOT, "MEASURED_PEAKS.json")
+    if os.path.exists(p):
+        d = json.load(open(p))
+        d["_source"] = "measured"
+        return d
+    d = dict(PEAKS_FALLBACK)
+    d["_source"] = "fallback"
+    return d
+
+
+class ClockSampler:
+    """nvidia-smi clocks + throttle reasons sampled during the timed region."""
+
+    FIELDS = "index,clocks.sm,clocks.max.sm,power.draw,clocks_event_reasons.active," \
+             "clocks_event_reasons.hw_slowdown,clocks_event_reasons.hw_thermal_slowdown," \
+             "clocks_event_reasons.sw_thermal_slowdown,clocks_event_reasons.sw_power_cap"
+
+    def __init__(self, gpu: int):
+        self.gpu = gpu
+        self.rows = []
+        self._stop = threading.Event()
+        self._t = None
+
+    def start(self):
+        def run():
+            while not self._stop.is_set():
+                try:
+                    out = subprocess.run(["nvidia-smi", "-i", str(self.gpu), f"--query-gpu={self.FIELDS}",
+                                          "--format=csv,noheader,nounits"], capture_output=True, text=True,
+                                         timeout=5).stdout.strip()
+                    if out:
+                        self.rows.append([x.strip() for x in out.split(",")])
+                except Exception:
+                    pass
+                self._stop.wait(0.2)
+        self._t = threading.Thread(target=run, daemon=True)
+        self._t.start()
+
+    def stop(self) -> dict:
+        self._stop.set()
+        if self._t:
+            self._t.join(timeout=10)
+        if not self.rows:
+            return {"sm_mhz": None, "sm_max_mhz": None, "reasons": ["unsampled"], "samples": 0}
+        sm = [float(r[1]) for r in self.rows if r[1].replace(".", "").isdigit()]
+        mx = [float(r[2]) for r in self.rows if r[2].replace(".", "").isdigit()]
+        names = ["hw_slowdown", "hw_thermal_slowdown", "sw_thermal_slowdown", "sw_power_cap"]
+        reasons = set()
+        for r in self.rows:
+            for k, n in enumerate(names):
+                if len(r) > 5 + k and r[5 + k].lower().startswith("active"):
+                    reasons.add(n)
+        return {"sm_mhz": float(np.median(sm)) if sm else None, "sm_max_mhz": max(mx) if mx else None,
+                "reasons": sorted(reasons), "samples": len(self.rows)}
+
+
+def dist_env():
+    ws = int(os.environ.get("WORLD_SIZE", "1"))
+    rank = int(os.environ.get("RANK", "0"))
+    local = int(os.environ.get("LOCAL_RANK", "0"))
+    return ws, rank, local
+
+
+def workload_inputs(cfg: str, n_pi: int, cycles: int, streams, step: int):
+    """Synthetic stimulus for one step: C3/C5 recipe (PI0 = reset for the first
+    4 cycles of step 0 only, other PIs Bern(1/2)), one seed per (stream, step)."""
+    from gen.stimulus import splitmix64, stim_random
+    out = []
+    base = {"c1": 1, "c2": 102, "c3": 103, "c4": 104, "c5": 105}[cfg]
+    for s in streams:
+        seed = splitmix64((base ^ (int(s) << 24) ^ step) & 0xFFFFFFFFFFFFFFFF) & 0xFFFFFFFF
+        if cfg == "c1":
+            from gen.stimulus import stim_c1
+            w = stim_c1(cycles, seed, reset_cycles=(0, 1) if step == 0 else ())
+        else:
+            w = stim_random(n_pi, cycles, seed, reset_pi0_cycles=4 if step == 0 else 0)
+            if step and cfg != "c2":
+                w[:, 0] &= np.uint32(0xFFFFFFFE)
+        out.append(w)
+    return np.stack(out)
+
+
+def cpu_baseline(eaig_path: str, n_pi: int, cfg: str, target_s: float = 12.0) -> dict:
+    """The oracle as it stands, single-threaded, on a bounded sample (host cores)."""
+    from gen import stimulus
+    from oracle import Oracle
+    o = Oracle(eaig_path)
+    probe = 50
+    st = stimulus("c3" if cfg == "c5" else cfg, n_pi, probe)
+    o.run(st, po=True)
+    rate = probe / max(o.last_seconds, 1e-9)
+    cycles = int(max(probe, min(200000, rate * target_s)))
+    o.reset()
+    st = stimulus("c3" if cfg == "c5" else cfg, n_pi, cycles)
+    o.run(st, po=True)
+    v = cycles / o.last_seconds
+    return {"value": v, "unit": UNIT, "cores": 1, "kind": "oracle",
+            "sample": f"{cycles} cycles of {cfg} (1 stream), oracle cycle loop only, single thread",
+            "gate_evals_per_s": v * o.n_ands, "host_nproc": os.cpu_count(), "seconds": o.last_seconds}
+
+
+def run_reference(args):
+    """--impl reference: the CPU oracle as the reference arm (this tier has no
+    reference implementation)."""
+    ws, rank, local = dist_env()
+    if rank != 0:
+        return 0
+    from tests.common import eaig
+    from oracle import Oracle
+    from gen import stimulus
+    cfg = args.workload
+    path = eaig(cfg)
+    o = Oracle(path)
+    n_pi = o.n_pi
+    # bounded sample per step so the whole run ends within minutes
+    probe = 20
+    o.run(stimulus("c3" if cfg == "c5" else cfg, n_pi, probe))
+    rate = probe / max(o.last_seconds, 1e-9)
+    per_step = int(max(5, min(args.cycles, rate * 120.0 / max(1, args.steps + args.warmup))))
+    o.reset()
+    tot_c, tot_s = 0, 0.0
+    for k in range(args.warmup + args.steps):
+        st = stimulus("c3" if cfg == "c5" else cfg, n_pi, per_step, seed=103 + k)
+        o.run(st)
+        if k >= args.warmup:
+            tot_c += per_step
+            tot_s += o.last_seconds
+    v = tot_c / tot_s
+    line = {"impl": "reference", "metric": METRIC, "value": v, "unit": UNIT, "n_gpus": ws, "steps": args.steps,
+            "warmup": args.warmup, "ms_per_step": 1e3 * tot_s / args.steps, "higher_is_better": True,
+            "scaling": "weak", "vs_baseline": None, "dtype": "u32", "data": "synthetic",
+            "config": {"workload": f"{cfg}: synthetic netlist ({o.n_ands} live ANDs), 1 stream",
+                       "cycles_per_step": per_step, "streams_per_gpu": 1},
+            "cpu_baseline": {"value": v, "unit": UNIT, "cores": 1, "kind": "oracle",
+                             "sample": f"{per_step} cycles per step x {args.steps} steps, single thread"},
+            "e2e": {"value": v, "unit": UNIT, "h2d_bytes_per_step": 0, "d2h_bytes_per_step": 0}}
+    print(json.dumps(line), flush=True)
+    return 0
+
+
+def main():
+    ap = argparse.ArgumentParser()
+    ap.add_argument("--gpus", type=int, default=1)
+    ap.add_argument("--steps", type=int, default=20)
+    ap.add_argument("--warmup", type=int, default=3)
+    ap.add_argument("--impl", default="gem", choices=["gem", "reference"])
+    ap.add_argument("--workload", default="c3", choices=["c1", "c2", "c3", "c4", "c5"])
+    ap.add_argument("--streams", type=int, default=0, help="streams per GPU (0 = 1, or 4096/N for c5)")
+    ap.add_argument("--cycles", type=int, default=1000, help="simulated cycles per step")
+    ap.add_argument("--no-cpu-baseline", action="store_true")
+    ap.add_argument("--no-flush", action="store_true")
+    ap.add_argument("--map-opts", default=None)
+    args = ap.parse_args()
+    if args.impl == "reference":
+        return run_reference(args)
+    args.warmup = max(3, args.warmup)
+
+    import torch
+    import torch.distributed as dist
+    ws, rank, local = dist_env()
+    if ws > 1:
+        os.environ.setdefault("MASTER_ADDR", "127.0.0.1")
+        torch.cuda.set_device(local)
+        dist.init_process_group("nccl", device_id=torch.device("cuda", local))
+    else:
+        torch.cuda.set_device(0)
+    dev = torch.device("cuda", local if ws > 1 else 0)
+
+    from paper_conf_dac_guozwlr25_b200 import gem
+    from paper_conf_dac_guozwlr25_b200.isa import blob_info
+    from tests.common import blob, eaig, MAP_OPTS
+
+    cfg = args.workload
+    S = args.streams or (max(1, 4096 // ws) if cfg == "c5" else 1)
+    opts = MAP_OPTS[cfg] if args.map_opts is None else args.map_opts
+    # rank 0 maps (cached on disk), others wait
+    if rank == 0:
+        b = blob(cfg, opts)
+    if ws > 1:
+        dist.barrier()
+    if rank != 0:
+        b = blob(cfg, opts)
+    info = blob_info(b)
+    stream = torch.cuda.current_stream(dev)
+    sim = gem.Simulator(b, device=dev.index, n_streams=S, cuda_stream=stream.cuda_stream, flags=gem.GEM_F_ASYNC)
+    C = args.cycles
+    gstreams = list(range(rank * S, rank * S + S))
+    # inputs for (warmup + steps), pre-generated on the host, uploaded per step
+    n_steps = args.warmup + args.steps
+    host_in = [workload_inputs(cfg, info.n_pi, C, gstreams, k) for k in range(min(n_steps, 4))]
+    pi_words = sim.pi_words
+    dev_in = [torch.from_numpy(x.view(np.int32)).to(dev) for x in host_in]
+    po_dev = torch.empty((S, C, sim.po_words), dtype=torch.int32, device=dev)
+    gather_buf = [torch.empty_like(po_dev) for _ in range(ws)] if (ws > 1 and rank == 0) else None
+    flush = torch.empty(512 * 1024 * 1024 // 4, dtype=torch.int32, device=dev)
+
+    def one_step(k, timed_events=None):
+        sim.set_inputs_device(dev_in[k % len(dev_in)], C)
+        if timed_events is not None:
+            timed_events[0].record(stream)
+        sim.step(C)
+        sim.read_outputs_device(po_dev, C)
+        if ws > 1:
+            dist.gather(po_dev, gather_buf, dst=0)
+        if timed_events is not None:
+            timed_events[1].record(stream)
+
+    for k in range(args.warmup):
+        one_step(k)
+    torch.cuda.synchronize(dev)
+    clocks = ClockSampler(dev.index)
+    clocks.start()
+    if ws > 1:
+        dist.barrier()
+    torch.cuda.synchronize(dev)
+    evs = []
+    kern_ms = []
+    for k in range(args.steps):
+        if not args.no_flush:
+            flush.fill_(k)
+        e = (torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True))
+        one_step(args.warmup + k, e)
+        evs.append(e)
+        kern_ms.append(sim.last_step_ms())
+    torch.cuda.synchronize(dev)
+    if ws > 1:
+        dist.barrier()
+    clk = clocks.stop()
+    step_ms = [a.elapsed_time(b_) for a, b_ in evs]
+    tot_ms = float(sum(step_ms))
+    # kernel-only duration (events inside libgem around gem_step_kernel, same stream)
+    kern_last = float(np.mean(kern_ms))
+    t = torch.tensor([tot_ms], dtype=torch.float64, device=dev)
+    if ws > 1:
+        dist.all_reduce(t, op=dist.ReduceOp.MAX)
+    tot_ms = float(t.item())
+    total_stream_cycles = ws * S * C * args.steps
+    value = total_stream_cycles / (tot_ms / 1e3)
+
+    # ---- e2e through the public API with HOST buffers (pinned), copies inside the timed region
+    e2e = None
+    sim_h = gem.Simulator(b, device=dev.index, n_streams=S)
+    host_pinned = [torch.from_numpy(x.view(np.int32)).pin_memory() for x in host_in]
+    for k in range(3):
+        sim_h.set_inputs(host_pinned[k % len(host_pinned)].numpy().view(np.uint32))
+        sim_h.step(C)
+        sim_h.read_outputs(C)
+    if ws > 1:
+        dist.barrier()
+    t0 = time.perf_counter()
+    e2e_steps = max(3, args.steps // 2)
+    for k in range(e2e_steps):
+        sim_h.set_inputs(host_pinned[k % len(host_pinned)].numpy().view(np.uint32))
+        sim_h.step(C)
+        out = sim_h.read_outputs(C)
+    e2e_s = time.perf_counter() - t0
+    te = torch.tensor([e2e_s], dtype=torch.float64, device=dev)
+    if ws > 1:
+        dist.all_reduce(te, op=dist.ReduceOp.MAX)
+    e2e_s = float(te.item())
+    e2e = {"value": ws * S * C * e2e_steps / e2e_s, "unit": UNIT,
+           "h2d_bytes_per_step": int(S * C * pi_words * 4), "d2h_bytes_per_step": int(S * C * sim.po_words * 4),
+           "api": "gem_set_inputs(host) + gem_step + gem_read_outputs(host), synchronous C ABI"}
+    sim_h.close()
+
+    if rank == 0:
+        peaks = _peaks()
+        sm_mhz = clk.get("sm_mhz") or peaks.get("sm_max_mhz", 1965.0)
+        # ALU roofline: 148 SMs x 64 LOP3/clk (alu pipe: 4 SMSP x 16 lanes)
+        n_sms = torch.cuda.get_device_properties(dev).multi_processor_count
+        peak_lop3 = n_sms * 64 * float(peaks.get("sm_max_mhz", 1965.0)) * 1e6
+        hz_kernel = C / (kern_last / 1e3)
+        achieved_lop3 = info.n_and / 16.0 * hz_kernel * S
+        roof = {"bound": "alu", "achieved": achieved_lop3 / 1e12, "peak": peak_lop3 / 1e12, "unit": "TLOP3/s",
+                "frac": achieved_lop3 / peak_lop3, "traffic": None,
+                "kernel": "gem_step_kernel", "kernel_ms_per_step": kern_last,
+                "algorithmic": "N_and/16 LOP3 per stream-cycle (2 LOP3 per 32 gate evals, P:81)",
+                "peak_source": f"{n_sms} SMs x 64 LOP3/clk x sm_max_mhz ({peaks['_source']})",
+                "hbm_program_bytes_per_cycle": info.program_bytes,
+                "hbm_frac_if_streamed": info.program_bytes * hz_kernel / (float(peaks.get("hbm_gbs", 6650)) * 1e9),
+                "us_per_layer_critical": 1e6 / hz_kernel / max(1, info.max_layers)}
+        cpu = None
+        if ws == 1 and not args.no_cpu_baseline:
+            cpu = cpu_baseline(eaig(cfg), info.n_pi, cfg)
+        line = {"metric": METRIC, "value": value, "unit": UNIT, "n_gpus": ws, "steps": args.steps,
+                "warmup": args.warmup, "ms_per_step": tot_ms / args.steps, "higher_is_better": True,
+                "scaling": "weak", "vs_baseline": None, "dtype": "u32", "data": "synthetic",
+                "config": {"workload": f"{cfg}: synthetic CPU-core-shaped netlist, {info.n_and} live ANDs, "
+                                       f"{info.n_flops} flops, {info.n_rams} RAM blocks" if cfg == "c3" else cfg,
+                           "streams_per_gpu": S, "cycles_per_step": C, "parts": info.n_parts,
+                           "stages": info.n_stages, "max_layers": info.max_layers, "levels": info.max_levels,
+                           "replication": round(info.replication, 3), "program_bytes": info.program_bytes,
+                           "grid": sim.info["grid"], "l2": "flushed between timed steps (512 MB write)"
+                           if not args.no_flush else "not flushed",
+                           "parallelism": f"streams sharded over {ws} GPU(s), NCCL gather of PO traces"
+                           if ws > 1 else "1 GPU"},
+                "gate_evals_per_s": value * info.n_and,
+                "clocks": clk, "gpu_launches": args.steps * 2,
+                "gpu_launches_detail": "per step: 1 gem_step_kernel (persistent, all cycles) + 1 unpermute_kernel",
+                "e2e": e2e, "roofline": roof, "cpu_baseline": cpu,
+                "step_ms": {"min": min(step_ms), "median": float(np.median(step_ms)), "max": max(step_ms)}}
+        print(json.dumps(line), flush=True)
+    sim.close()
+    if ws > 1:
+        dist.destroy_process_group()
+    return 0
+
+
+if __name__ == "__main__":
+    sys.exit(main())

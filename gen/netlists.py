@@ -267,7 +267,9 @@ def build_G(spec: GSpec, seed: int, scale: float = 1.0) -> (Netlist, dict):
         hop = 1 + (rng.random(n_l) * np.maximum(gz - 1, 1)).astype(np.int64)
         c1 = np.where(cross & (gz > 1), gs + (cl - gs + hop) % np.maximum(gz, 1), cl)
         l1 = np.minimum(l1, top[c1])
-        l1 = np.where(c1 != cl, np.minimum(l1, l - 1), l1)
+        # cross-cluster fan-ins come from shallow levels of the other cluster
+        # (module-interface logic), so cones leak across clusters only a little
+        l1 = np.where(c1 != cl, np.minimum(rng.integers(0, 4, size=n_l), l - 1), l1)
         in1 = np.empty(n_l, dtype=np.int64)
         z = l1 == 0
         if np.any(z):

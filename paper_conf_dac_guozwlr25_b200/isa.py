@@ -1,0 +1,75 @@
+"""Read-only view of a `.gemb` header (field names from csrc/gem_isa.h)."""
+from __future__ import annotations
+
+import dataclasses
+
+import numpy as np
+
+GH = ["MAGIC", "VERSION", "N_PI", "N_PO", "N_FLOPS", "N_RAMS", "N_PARTS", "N_STAGES",
+      "MAX_STATE_WORDS", "MAX_LAYERS", "PI_WORDS", "PO_WORDS", "Q_WORDS", "CUT_WORDS",
+      "N_AND_LO", "N_AND_HI", "N_AND_MAPPED_LO", "N_AND_MAPPED_HI", "TOTAL_LAYERS",
+      "TOTAL_LEAVES_LO", "TOTAL_LEAVES_HI", "OFF_PARTS", "OFF_STAGES", "OFF_FLOP_INIT",
+      "OFF_PROG", "PROG_WORDS_LO", "PROG_WORDS_HI", "MAX_LEVELS", "TOTAL_WRITEOUTS",
+      "MAX_OUT", "TOTAL_WORDS_LO", "TOTAL_WORDS_HI", "SLOTS_USED_LO", "SLOTS_USED_HI"]
+GEM_MAGIC = 0x424D4547
+SLOTS_PER_LAYER = 8191
+
+
+@dataclasses.dataclass
+class BlobInfo:
+    n_pi: int
+    n_po: int
+    n_flops: int
+    n_rams: int
+    n_parts: int
+    n_stages: int
+    max_state_words: int
+    max_layers: int
+    total_layers: int
+    q_words: int
+    po_words: int
+    cut_words: int
+    n_and: int
+    n_and_mapped: int
+    total_leaves: int
+    max_levels: int
+    program_bytes: int
+    blob_bytes: int
+    slots_used: int
+    part_layers: list
+
+    @property
+    def replication(self) -> float:
+        return self.n_and_mapped / max(1, self.n_and) - 1.0
+
+    @property
+    def slot_util(self) -> float:
+        return self.n_and / max(1, self.total_layers * SLOTS_PER_LAYER)
+
+    @property
+    def bytes_per_and(self) -> float:
+        return self.program_bytes / max(1, self.n_and)
+
+    def as_dict(self) -> dict:
+        d = dataclasses.asdict(self)
+        d.pop("part_layers")
+        d.update(replication=self.replication, slot_util=self.slot_util, bytes_per_and=self.bytes_per_and,
+                 levels_per_layer=self.max_levels / max(1, self.max_layers))
+        return d
+
+
+def blob_info(blob: bytes) -> BlobInfo:
+    w = np.frombuffer(blob, dtype=np.uint32)
+    h = {k: int(w[i]) for i, k in enumerate(GH)}
+    if h["MAGIC"] != GEM_MAGIC:
+        raise ValueError("not a .gemb blob")
+    u64 = lambda k: h[k + "_LO"] | (h[k + "_HI"] << 32)
+    np_ = h["N_PARTS"]
+    pt = w[h["OFF_PARTS"]:h["OFF_PARTS"] + 4 * np_].reshape(np_, 4)
+    return BlobInfo(n_pi=h["N_PI"], n_po=h["N_PO"], n_flops=h["N_FLOPS"], n_rams=h["N_RAMS"],
+                    n_parts=np_, n_stages=h["N_STAGES"], max_state_words=h["MAX_STATE_WORDS"],
+                    max_layers=h["MAX_LAYERS"], total_layers=h["TOTAL_LAYERS"], q_words=h["Q_WORDS"],
+                    po_words=h["PO_WORDS"], cut_words=h["CUT_WORDS"], n_and=u64("N_AND"),
+                    n_and_mapped=u64("N_AND_MAPPED"), total_leaves=u64("TOTAL_LEAVES"),
+                    max_levels=h["MAX_LEVELS"], program_bytes=4 * u64("PROG_WORDS"),
+                    blob_bytes=len(blob), slots_used=u64("SLOTS_USED"), part_layers=pt[:, 3].tolist())

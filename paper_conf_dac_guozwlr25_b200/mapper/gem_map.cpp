@@ -1,0 +1,1297 @@
+// gem_map.cpp -- host-side mapping flow: E-AIG -> VLIW program blob (.gemb).
+//
+// Follows PAPER.md §III, simplified where SURVEY.md §2 says so:
+//   * synthesis (§III-B): the input is already an E-AIG; we only do
+//     structural hashing, trivial simplification and cone-of-influence pruning
+//     (the commercial depth-optimising synthesiser is out of scope).
+//   * partitioning (§III-C): replication-aided (RepCut-style)
+//     endpoint clustering.  Endpoints are single flop / PO bits and whole RAM
+//     blocks; each partition recomputes the full cone of its endpoints, so
+//     partitions never depend on each other inside a cycle.  Clustering
+//     is min-hash ordered greedy packing followed by Algorithm 1 merging
+//     (P:119-125): try to merge partitions with large overlap, commit if the
+//     result is still mappable (here: under the size cap).
+//   * multi-stage cut (Fig.5): nodes at a cut level become stage-0
+//     endpoints ("cut words") and stage-1 sources.
+//   * placement (§III-D, Algorithm 2): iterative layer filling,
+//     bottom (1-bit tip, level 13) to top (leaf side), choosing the most
+//     timing-critical node (largest reverse depth) of logic level i for
+//     a free level-i slot and recursively mapping its fan-in cone into the
+//     slot's subtree (bit-mapping primitive); realised values are
+//     written out and become leaves of later layers ("remove the nodes
+//     already realised ... create a new AIG subgraph").
+//   * bitstream generation (§III-E): gem_isa.h encoding.
+//
+// The mapper shares no code with oracle/.
+
+#include <algorithm>
+#include <atomic>
+#include <chrono>
+#include <cstdint>
+#include <cstdio>
+#include <cstdlib>
+#include <cstring>
+#include <fstream>
+#include <functional>
+#include <mutex>
+#include <numeric>
+#include <sstream>
+#include <stdexcept>
+#include <string>
+#include <thread>
+#include <unordered_map>
+#include <vector>
+
+#include "../csrc/gem_isa.h"
+
+namespace gm {
+
+static thread_local std::string g_err;
+
+// =========================================================== options
+struct Options {
+  int parts = 0;            // target partition count (0 = auto)
+  int part_size = 6000;     // auto target ANDs per partition (paper: 5.7-12.9K, Table I)
+  int threads = 0;          // 0 = hardware concurrency
+  int leafcap = 320;        // max leaves of one placed root (cost filter)
+  int stages = 1;           // 1 or 2 (multi-stage RepCut)
+  int cut_level = 0;        // 0 = auto (middle)
+  int merge = 1;            // Algorithm 1 merge pass
+  int verbose = 0;
+  int max_state_words = GEM_MAX_STATE_WORDS;
+  double cap_slack = 1.0;
+};
+
+static Options parse_opts(const char* s) {
+  Options o;
+  if (!s) return o;
+  std::stringstream ss(s);
+  std::string tok;
+  while (ss >> tok) {
+    size_t eq = tok.find('=');
+    if (eq == std::string::npos) throw std::runtime_error("bad option " + tok);
+    std::string k = tok.substr(0, eq), v = tok.substr(eq + 1);
+    if (k == "parts") o.parts = std::stoi(v);
+    else if (k == "part_size") o.part_size = std::stoi(v);
+    else if (k == "threads") o.threads = std::stoi(v);
+    else if (k == "leafcap") o.leafcap = std::stoi(v);
+    else if (k == "stages") o.stages = std::stoi(v);
+    else if (k == "cut_level") o.cut_level = std::stoi(v);
+    else if (k == "merge") o.merge = std::stoi(v);
+    else if (k == "verbose") o.verbose = std::stoi(v);
+    else if (k == "max_state_words") o.max_state_words = std::stoi(v);
+    else if (k == "cap_slack") o.cap_slack = std::stod(v);
+    else throw std::runtime_error("unknown option " + k);
+  }
+  if (o.stages < 1 || o.stages > 2) throw std::runtime_error("stages must be 1 or 2");
+  if (o.max_state_words > GEM_MAX_STATE_WORDS || o.max_state_words < 64)
+    throw std::runtime_error("bad max_state_words");
+  return o;
+}
+
+// =========================================================== AIGER reader
+struct RawRam {
+  std::vector<uint64_t> rdata, raddr, waddr, wdata, wbe;
+};
+struct Raw {
+  uint64_t M = 0, I = 0, L = 0, O = 0, A = 0;
+  std::vector<uint64_t> lnext;
+  std::vector<uint8_t> linit;
+  std::vector<uint64_t> outs;
+  std::vector<uint64_t> lhs, r0, r1;
+  std::vector<RawRam> rams;
+};
+
+struct Reader {
+  const char* p;
+  const char* e;
+  bool eof() const { return p >= e; }
+  void skip_ws() { while (p < e && (*p == ' ' || *p == '\t' || *p == '\r')) p++; }
+  uint64_t num() {
+    skip_ws();
+    if (p >= e || *p < '0' || *p > '9') throw std::runtime_error("number expected");
+    uint64_t x = 0;
+    while (p < e && *p >= '0' && *p <= '9') x = x * 10 + (uint64_t)(*p++ - '0');
+    return x;
+  }
+  bool at_eol() { skip_ws(); return p >= e || *p == '\n'; }
+  void eol() {
+    skip_ws();
+    if (p < e && *p != '\n') throw std::runtime_error("end of line expected");
+    if (p < e) p++;
+  }
+  std::string line() {
+    const char* s = p;
+    while (p < e && *p != '\n') p++;
+    std::string r(s, p);
+    if (p < e) p++;
+    return r;
+  }
+  uint64_t varint() {
+    uint64_t x = 0;
+    int sh = 0;
+    while (true) {
+      if (p >= e) throw std::runtime_error("EOF in binary ANDs");
+      uint8_t c = (uint8_t)*p++;
+      x |= (uint64_t)(c & 0x7f) << sh;
+      if (!(c & 0x80)) return x;
+      sh += 7;
+      if (sh > 63) throw std::runtime_error("varint overflow");
+    }
+  }
+};
+
+static std::vector<uint64_t> split_nums(const std::string& s) {
+  std::vector<uint64_t> r;
+  size_t i = 0;
+  while (i < s.size()) {
+    size_t j = s.find(',', i);
+    if (j == std::string::npos) j = s.size();
+    r.push_back(std::stoull(s.substr(i, j - i)));
+    i = j + 1;
+  }
+  return r;
+}
+
+static Raw read_aiger(const char* data, size_t n) {
+  Raw g;
+  Reader rd{data, data + n};
+  std::string magic;
+  while (!rd.eof() && *rd.p != ' ') magic.push_back(*rd.p++);
+  bool bin;
+  if (magic == "aag") bin = false;
+  else if (magic == "aig") bin = true;
+  else throw std::runtime_error("not an AIGER file");
+  g.M = rd.num(); g.I = rd.num(); g.L = rd.num(); g.O = rd.num(); g.A = rd.num();
+  if (!rd.at_eol()) throw std::runtime_error("AIGER B/C/J/F sections are not supported");
+  rd.eol();
+  if (!bin)
+    for (uint64_t i = 0; i < g.I; i++) {
+      if (rd.num() != 2 * (i + 1)) throw std::runtime_error("inputs must be 2,4,..");
+      rd.eol();
+    }
+  g.lnext.resize(g.L);
+  g.linit.assign(g.L, 0);
+  for (uint64_t j = 0; j < g.L; j++) {
+    uint64_t cur = 2 * (g.I + 1 + j);
+    if (!bin && rd.num() != cur) throw std::runtime_error("latch numbering");
+    g.lnext[j] = rd.num();
+    if (!rd.at_eol()) {
+      uint64_t init = rd.num();
+      g.linit[j] = (init == 1) ? 1 : 0;
+      if (init != 0 && init != 1 && init != cur) throw std::runtime_error("bad latch init");
+    }
+    rd.eol();
+  }
+  g.outs.resize(g.O);
+  for (uint64_t k = 0; k < g.O; k++) { g.outs[k] = rd.num(); rd.eol(); }
+  g.lhs.resize(g.A); g.r0.resize(g.A); g.r1.resize(g.A);
+  if (!bin) {
+    for (uint64_t k = 0; k < g.A; k++) {
+      g.lhs[k] = rd.num(); g.r0[k] = rd.num(); g.r1[k] = rd.num();
+      rd.eol();
+    }
+  } else {
+    for (uint64_t k = 0; k < g.A; k++) {
+      uint64_t lhs = 2 * (g.I + g.L + 1 + k);
+      uint64_t d0 = rd.varint(), d1 = rd.varint();
+      if (d0 > lhs || d1 > lhs - d0) throw std::runtime_error("bad binary delta");
+      g.lhs[k] = lhs; g.r0[k] = lhs - d0; g.r1[k] = lhs - d0 - d1;
+    }
+  }
+  bool comments = false;
+  while (!rd.eof()) {
+    std::string ln = rd.line();
+    if (!comments) {
+      if (ln == "c" || ln.rfind("c ", 0) == 0) comments = true;
+      continue;
+    }
+    if (ln.rfind("gem-ram ", 0) != 0) continue;
+    std::stringstream ss(ln);
+    std::string tag, id, f;
+    ss >> tag >> id;
+    RawRam r;
+    while (ss >> f) {
+      size_t eq = f.find('=');
+      if (eq == std::string::npos) throw std::runtime_error("bad gem-ram");
+      std::string k = f.substr(0, eq);
+      auto v = split_nums(f.substr(eq + 1));
+      if (k == "rdata") r.rdata = v;
+      else if (k == "raddr") r.raddr = v;
+      else if (k == "waddr") r.waddr = v;
+      else if (k == "wdata") r.wdata = v;
+      else if (k == "wbe") r.wbe = v;
+      else throw std::runtime_error("bad gem-ram key");
+    }
+    if (r.rdata.size() != 32 || r.raddr.size() != 13 || r.waddr.size() != 13 || r.wdata.size() != 32 ||
+        r.wbe.size() != 32)
+      throw std::runtime_error("gem-ram port widths must be 32/13/13/32/32");
+    g.rams.push_back(r);
+  }
+  return g;
+}
+
+// =========================================================== compact graph
+// Node kinds: sources (const, PI, latch, RAM rdata) then ANDs in topological order.
+enum : uint8_t { K_CONST = 0, K_SRC = 1, K_AND = 2 };
+
+struct Graph {
+  uint32_t n_pi = 0, n_flops = 0, n_po = 0, n_rams = 0;
+  std::vector<uint8_t> kind;
+  std::vector<uint32_t> a, b;        // AND fanins (compact literals)
+  std::vector<uint32_t> gbit;        // sources: region<<27 | word<<5 | bit
+  std::vector<uint32_t> level;
+  std::vector<uint32_t> flop_next;   // compact literal per flop
+  std::vector<uint8_t> flop_init;
+  std::vector<uint32_t> po;          // compact literal per PO
+  struct Ram { uint32_t port[4][32]; } ;
+  std::vector<Ram> rams;             // ports: raddr(13) waddr(13) wdata wbe; missing bits = 0
+  uint64_t n_and_live = 0;
+  uint32_t max_level = 0;
+};
+
+static inline uint32_t mk_gbit(uint32_t region, uint32_t word, uint32_t bit) {
+  return (region << 27) | (word << 5) | bit;
+}
+
+static Graph build_graph(const Raw& r) {
+  Graph g;
+  // classify inputs
+  std::vector<int64_t> in_ram(r.I, -1), in_bit(r.I, -1);
+  for (size_t k = 0; k < r.rams.size(); k++)
+    for (int j = 0; j < 32; j++) {
+      uint64_t i = r.rams[k].rdata[j];
+      if (i >= r.I) throw std::runtime_error("rdata index out of range");
+      if (in_ram[i] >= 0) throw std::runtime_error("rdata input owned twice");
+      in_ram[i] = (int64_t)k; in_bit[i] = j;
+    }
+  std::vector<uint32_t> m(r.M + 1, UINT32_MAX);   // orig var -> compact literal
+  g.kind.push_back(K_CONST); g.a.push_back(0); g.b.push_back(0); g.gbit.push_back(0); g.level.push_back(0);
+  m[0] = 0;
+  uint32_t pi = 0;
+  for (uint64_t i = 0; i < r.I; i++) {
+    uint32_t id = (uint32_t)g.kind.size();
+    g.kind.push_back(K_SRC); g.a.push_back(0); g.b.push_back(0); g.level.push_back(0);
+    if (in_ram[i] >= 0) g.gbit.push_back(mk_gbit(GEM_R_RD, (uint32_t)in_ram[i], (uint32_t)in_bit[i]));
+    else { g.gbit.push_back(mk_gbit(GEM_R_PI, pi / 32, pi % 32)); pi++; }
+    m[i + 1] = 2 * id;
+  }
+  g.n_pi = pi;
+  for (uint64_t j = 0; j < r.L; j++) {
+    uint32_t id = (uint32_t)g.kind.size();
+    g.kind.push_back(K_SRC); g.a.push_back(0); g.b.push_back(0); g.level.push_back(0);
+    g.gbit.push_back(mk_gbit(GEM_R_Q, (uint32_t)(j / 32), (uint32_t)(j % 32)));  // external order for now
+    m[r.I + 1 + j] = 2 * id;
+  }
+  // topological order of the original ANDs (Kahn)
+  std::vector<int64_t> and_of_var(r.M + 1, -1);
+  for (uint64_t k = 0; k < r.A; k++) {
+    uint64_t v = r.lhs[k] >> 1;
+    if ((r.lhs[k] & 1) || v <= r.I + r.L || v > r.M || and_of_var[v] >= 0)
+      throw std::runtime_error("bad AND lhs");
+    and_of_var[v] = (int64_t)k;
+  }
+  std::vector<uint32_t> indeg(r.A, 0);
+  std::vector<uint32_t> uoff(r.A + 1, 0);
+  for (uint64_t k = 0; k < r.A; k++)
+    for (uint64_t l : {r.r0[k], r.r1[k]}) {
+      if ((l >> 1) > r.M) throw std::runtime_error("literal out of range");
+      int64_t d = and_of_var[l >> 1];
+      if (d >= 0) { indeg[k]++; uoff[d + 1]++; }
+      else if ((l >> 1) > r.I + r.L) throw std::runtime_error("undefined literal");
+    }
+  for (uint64_t k = 0; k < r.A; k++) uoff[k + 1] += uoff[k];
+  std::vector<uint32_t> users(uoff[r.A]);
+  {
+    std::vector<uint32_t> fill(uoff.begin(), uoff.end() - 1);
+    for (uint64_t k = 0; k < r.A; k++)
+      for (uint64_t l : {r.r0[k], r.r1[k]}) {
+        int64_t d = and_of_var[l >> 1];
+        if (d >= 0) users[fill[d]++] = (uint32_t)k;
+      }
+  }
+  std::vector<uint32_t> q;
+  q.reserve(r.A);
+  for (uint64_t k = 0; k < r.A; k++) if (!indeg[k]) q.push_back((uint32_t)k);
+  std::unordered_map<uint64_t, uint32_t> strash;
+  strash.reserve(r.A * 2 + 16);
+  for (size_t h = 0; h < q.size(); h++) {
+    uint32_t k = q[h];
+    uint32_t la = m[r.r0[k] >> 1] ^ (uint32_t)(r.r0[k] & 1);
+    uint32_t lb = m[r.r1[k] >> 1] ^ (uint32_t)(r.r1[k] & 1);
+    if (la > lb) std::swap(la, lb);
+    uint32_t res;
+    if (la == 0) res = 0;
+    else if (la == 1) res = lb;
+    else if (la == lb) res = la;
+    else if (la == (lb ^ 1)) res = 0;
+    else {
+      uint64_t key = ((uint64_t)la << 32) | lb;
+      auto it = strash.find(key);
+      if (it != strash.end()) res = it->second;
+      else {
+        uint32_t id = (uint32_t)g.kind.size();
+        g.kind.push_back(K_AND); g.a.push_back(la); g.b.push_back(lb); g.gbit.push_back(0);
+        g.level.push_back(1 + std::max(g.level[la >> 1], g.level[lb >> 1]));
+        res = 2 * id;
+        strash.emplace(key, res);
+      }
+    }
+    m[r.lhs[k] >> 1] = res;
+    for (uint32_t i = uoff[k]; i < uoff[k + 1]; i++)
+      if (--indeg[users[i]] == 0) q.push_back(users[i]);
+  }
+  if (q.size() != r.A) throw std::runtime_error("combinational loop");
+  auto lit = [&](uint64_t l) {
+    uint32_t x = m[l >> 1];
+    if (x == UINT32_MAX) throw std::runtime_error("undefined literal");
+    return x ^ (uint32_t)(l & 1);
+  };
+  g.n_flops = (uint32_t)r.L;
+  g.flop_next.resize(r.L);
+  g.flop_init = r.linit;
+  for (uint64_t j = 0; j < r.L; j++) g.flop_next[j] = lit(r.lnext[j]);
+  g.n_po = (uint32_t)r.O;
+  g.po.resize(r.O);
+  for (uint64_t k = 0; k < r.O; k++) g.po[k] = lit(r.outs[k]);
+  g.n_rams = (uint32_t)r.rams.size();
+  for (auto& rr : r.rams) {
+    Graph::Ram gr;
+    std::memset(&gr, 0, sizeof(gr));
+    for (int k = 0; k < 13; k++) gr.port[0][k] = lit(rr.raddr[k]);
+    for (int k = 0; k < 13; k++) gr.port[1][k] = lit(rr.waddr[k]);
+    for (int k = 0; k < 32; k++) gr.port[2][k] = lit(rr.wdata[k]);
+    for (int k = 0; k < 32; k++) gr.port[3][k] = lit(rr.wbe[k]);
+    g.rams.push_back(gr);
+  }
+  // live AND count (cone of influence of all endpoints)
+  std::vector<uint8_t> live(g.kind.size(), 0);
+  auto mark = [&](uint32_t l) { live[l >> 1] = 1; };
+  for (auto l : g.flop_next) mark(l);
+  for (auto l : g.po) mark(l);
+  for (auto& rr : g.rams) for (int p = 0; p < 4; p++) for (int k = 0; k < 32; k++) mark(rr.port[p][k]);
+  for (size_t i = g.kind.size(); i-- > 0;)
+    if (live[i] && g.kind[i] == K_AND) { live[g.a[i] >> 1] = 1; live[g.b[i] >> 1] = 1; }
+  for (size_t i = 0; i < g.kind.size(); i++)
+    if (live[i] && g.kind[i] == K_AND) { g.n_and_live++; g.max_level = std::max(g.max_level, g.level[i]); }
+  return g;
+}
+
+// =========================================================== partition description
+// An output word: destination gid + 32 compact literals (bit k of the word).
+struct OutWord {
+  uint32_t dst;            // gid (region<<24 | index); RAMP index filled at encode time
+  uint32_t lit[32];
+};
+
+struct Unit {              // a partitioning unit
+  int kind;                // 0 flop bit, 1 PO bit, 2 RAM block, 3 cut bit
+  uint32_t idx;            // flop / po / ram / cut index
+  uint64_t key;            // locality sort key
+};
+
+struct Part {
+  int stage = 0;
+  std::vector<uint32_t> flops, pos, rams, cuts;   // endpoints owned
+  // filled by the layout step
+  std::vector<OutWord> outs;
+  // filled by mapping
+  std::vector<uint32_t> prog;
+  uint32_t n_layers = 0, n_nodes = 0, state_words = 0, n_leaves = 0, max_level = 0, n_writeouts = 0;
+  uint64_t slots_used = 0;
+  bool ok = false;
+  std::string err;
+};
+
+// =========================================================== placement (Algorithm 2)
+static inline uint32_t group_width(int k) {      // slots per unit at level k
+  if (k <= 5) return 1u << (5 - k);
+  if (k <= 10) return 1u << (10 - k);
+  return 1u << (13 - k);
+}
+static inline uint32_t level_slots(int k) { return 8192u >> k; }
+static inline uint32_t child_a(int k, uint32_t id) {
+  uint32_t g = group_width(k);
+  return (id / g) * 2 * g + (id % g);
+}
+static inline uint32_t child_b(int k, uint32_t id) { return child_a(k, id) + group_width(k); }
+static const int kOff[6] = {0, GEM_OFF_L1, GEM_OFF_L2, GEM_OFF_L3, GEM_OFF_L4, GEM_OFF_L5};
+// unit (thread for 1..5, warp for 6..10, 0 for 11..13) and packed bit of slot (k,id)
+static inline uint32_t slot_unit(int k, uint32_t id) { return k >= 11 ? 0 : id / group_width(k); }
+static inline uint32_t slot_bit(int k, uint32_t id) {
+  if (k >= 11) return (k == 11 ? 0 : k == 12 ? 4 : 6) + id;
+  int kk = k <= 5 ? k : k - 5;
+  return (uint32_t)kOff[kk] + id % group_width(k);
+}
+
+struct Mapper {
+  const Graph& G;
+  const Options& opt;
+  explicit Mapper(const Graph& g, const Options& o) : G(g), opt(o) {}
+
+  // local graph
+  std::vector<uint32_t> cid;          // local -> compact id
+  std::vector<uint8_t> is_src;
+  std::vector<uint32_t> la, lb;       // local literals
+  std::vector<uint32_t> coff, cons;   // consumers CSR
+  std::vector<uint8_t> is_ep;         // referenced by an output word
+  std::vector<int32_t> loc;           // realised: state bit, or -1
+
+  void map(Part& P, std::vector<int32_t>& scratch) {
+    // ---- collect the cone (compact ids), sorted = topological
+    std::vector<uint32_t> stack, nodes;
+    auto visit = [&](uint32_t c) {
+      if (scratch[c] >= 0) return;
+      scratch[c] = 0;
+      stack.push_back(c);
+      while (!stack.empty()) {
+        uint32_t x = stack.back();
+        stack.pop_back();
+        nodes.push_back(x);
+        if (G.kind[x] == K_AND)
+          for (uint32_t y : {G.a[x] >> 1, G.b[x] >> 1})
+            if (scratch[y] < 0) { scratch[y] = 0; stack.push_back(y); }
+      }
+    };
+    visit(0);   // constant always present (padding / constant outputs)
+    for (auto& ow : P.outs) for (int k = 0; k < 32; k++) visit(ow.lit[k] >> 1);
+    std::sort(nodes.begin(), nodes.end());
+    struct Cleanup {
+      std::vector<uint32_t>& nodes; std::vector<int32_t>& scratch;
+      ~Cleanup() { for (uint32_t c : nodes) scratch[c] = -1; }
+    } cleanup{nodes, scratch};
+    uint32_t n = (uint32_t)nodes.size();
+    for (uint32_t i = 0; i < n; i++) scratch[nodes[i]] = (int32_t)i;
+    cid = nodes;
+    is_src.assign(n, 0); la.assign(n, 0); lb.assign(n, 0); is_ep.assign(n, 0); loc.assign(n, -1);
+    std::vector<uint32_t> cnt(n + 1, 0);
+    uint32_t n_and = 0;
+    for (uint32_t i = 0; i < n; i++) {
+      uint32_t c = nodes[i];
+      if (G.kind[c] != K_AND) { is_src[i] = 1; continue; }
+      n_and++;
+      la[i] = 2 * (uint32_t)scratch[G.a[c] >> 1] | (G.a[c] & 1);
+      lb[i] = 2 * (uint32_t)scratch[G.b[c] >> 1] | (G.b[c] & 1);
+      cnt[(la[i] >> 1) + 1]++;
+      cnt[(lb[i] >> 1) + 1]++;
+    }
+    coff.assign(n + 1, 0);
+    for (uint32_t i = 0; i < n; i++) coff[i + 1] = coff[i] + cnt[i + 1];
+    cons.assign(coff[n], 0);
+    {
+      std::vector<uint32_t> f(coff.begin(), coff.end() - 1);
+      for (uint32_t i = 0; i < n; i++)
+        if (!is_src[i]) { cons[f[la[i] >> 1]++] = i; cons[f[lb[i] >> 1]++] = i; }
+    }
+    for (auto& ow : P.outs) for (int k = 0; k < 32; k++) is_ep[(uint32_t)scratch[ow.lit[k] >> 1]] = 1;
+    P.n_nodes = n_and;
+
+    // ---- state: word 0 = const 0; gread words next
+    std::vector<uint32_t> gread_src;     // gid per gread
+    std::unordered_map<uint32_t, uint32_t> gword;   // gid -> state word
+    uint32_t sw_next = 1;
+    std::vector<uint32_t> word_live;     // live realised values per state word
+    for (uint32_t i = 0; i < n; i++) {
+      if (!is_src[i]) continue;
+      uint32_t c = nodes[i];
+      if (G.kind[c] == K_CONST) { loc[i] = 0; continue; }
+      uint32_t gb = G.gbit[c];
+      uint32_t gid = GEM_GID(gb >> 27, (gb >> 5) & 0x3FFFFF);
+      auto it = gword.find(gid);
+      uint32_t sw;
+      if (it == gword.end()) {
+        sw = sw_next++;
+        gword.emplace(gid, sw);
+        gread_src.push_back(gid);
+      } else sw = it->second;
+      loc[i] = (int32_t)(sw * 32 + (gb & 31));
+    }
+    uint32_t n_gread = sw_next - 1;
+    if (sw_next > (uint32_t)opt.max_state_words) { fail(P, "too many gread words"); return; }
+    word_live.assign(opt.max_state_words, 0);
+
+    // ---- liveness helpers
+    std::vector<uint8_t> mc(n, 0);            // must compute
+    auto compute_mc = [&]() {
+      for (uint32_t i = n; i-- > 0;) {
+        mc[i] = 0;
+        if (is_src[i] || loc[i] >= 0) continue;
+        if (is_ep[i]) { mc[i] = 1; continue; }
+        for (uint32_t j = coff[i]; j < coff[i + 1]; j++)
+          if (mc[cons[j]]) { mc[i] = 1; break; }
+      }
+    };
+    auto value_live = [&](uint32_t i) {      // realised i still needed?
+      if (is_ep[i]) return true;
+      for (uint32_t j = coff[i]; j < coff[i + 1]; j++)
+        if (mc[cons[j]]) return true;
+      return false;
+    };
+    compute_mc();
+    // live counts for gread words
+    std::vector<std::vector<uint32_t>> word_vals(opt.max_state_words);
+    for (uint32_t i = 0; i < n; i++)
+      if (is_src[i] && loc[i] > 0) word_vals[(uint32_t)loc[i] >> 5].push_back(i);
+    std::vector<uint8_t> word_used(opt.max_state_words, 0);
+    word_used[0] = 1;
+    for (uint32_t w = 1; w < sw_next; w++) word_used[w] = 1;
+    std::vector<uint32_t> free_words;
+    auto refresh_free = [&]() {
+      // a used word becomes free when none of its values is live
+      for (uint32_t w = 1; w < (uint32_t)opt.max_state_words; w++) {
+        if (!word_used[w]) continue;
+        bool live = false;
+        for (uint32_t i : word_vals[w]) if (value_live(i)) { live = true; break; }
+        if (!live) { word_used[w] = 0; word_vals[w].clear(); free_words.push_back(w); }
+      }
+    };
+    for (uint32_t w = (uint32_t)opt.max_state_words; w-- > sw_next;) free_words.push_back(w);
+    refresh_free();
+    // keep free words sorted descending so pop_back gives the lowest index
+    auto sort_free = [&]() { std::sort(free_words.begin(), free_words.end(), std::greater<uint32_t>()); };
+    sort_free();
+
+    std::vector<uint32_t> d(n, 0), rd(n, 0), lf(n, 0);
+    std::vector<uint32_t> prog_layers;
+    uint32_t n_layers = 0, total_leaves = 0, total_wo = 0, max_state = sw_next;
+    uint64_t slots_used = 0;
+    // per-layer slot arrays
+    std::vector<int32_t> slot[14];
+    std::vector<uint8_t> sxa[14], sxb[14], sob[14];
+    for (int k = 0; k <= 13; k++) {
+      slot[k].assign(level_slots(k), -1);
+      sxa[k].assign(level_slots(k), 0); sxb[k].assign(level_slots(k), 0); sob[k].assign(level_slots(k), 0);
+    }
+    std::vector<int32_t> comp_k(n, -1), comp_id(n, -1);   // one computed copy per node
+    std::vector<uint32_t> computed;
+    std::vector<uint32_t> thread_leaves(256, 0);
+
+    while (true) {
+      // any work left?
+      bool any = false;
+      for (uint32_t i = 0; i < n; i++) if (mc[i]) { any = true; break; }
+      if (!any) break;
+      if (n_layers > 4096) { fail(P, "no progress"); return; }
+      // depth over realised set, reverse depth, leaf cost
+      for (uint32_t i = 0; i < n; i++) {
+        if (!mc[i]) continue;
+        uint32_t a = la[i] >> 1, b = lb[i] >> 1;
+        uint32_t da = loc[a] >= 0 ? 0 : d[a], db = loc[b] >= 0 ? 0 : d[b];
+        d[i] = 1 + std::max(da, db);
+        uint32_t fa = loc[a] >= 0 ? 1 : lf[a], fb = loc[b] >= 0 ? 1 : lf[b];
+        lf[i] = std::min<uint32_t>(1u << 24, fa + fb);
+      }
+      for (uint32_t i = n; i-- > 0;) {
+        if (!mc[i]) continue;
+        uint32_t r = 0;
+        for (uint32_t j = coff[i]; j < coff[i + 1]; j++)
+          if (mc[cons[j]]) r = std::max(r, rd[cons[j]] + 1);
+        rd[i] = r;
+      }
+      // candidates per level
+      std::vector<uint32_t> cand[14];
+      for (uint32_t i = 0; i < n; i++)
+        if (mc[i] && d[i] <= 13) cand[d[i]].push_back(i);
+      for (int k = 1; k <= 13; k++)
+        std::sort(cand[k].begin(), cand[k].end(), [&](uint32_t x, uint32_t y) {
+          if (rd[x] != rd[y]) return rd[x] > rd[y];
+          if (lf[x] != lf[y]) return lf[x] < lf[y];
+          return x < y;
+        });
+      // reset slots
+      for (int k = 0; k <= 13; k++) {
+        std::fill(slot[k].begin(), slot[k].end(), -1);
+        std::fill(sxa[k].begin(), sxa[k].end(), 0);
+        std::fill(sxb[k].begin(), sxb[k].end(), 0);
+        std::fill(sob[k].begin(), sob[k].end(), 0);
+      }
+      std::fill(thread_leaves.begin(), thread_leaves.end(), 0);
+      for (uint32_t i : computed) { comp_k[i] = -1; comp_id[i] = -1; }
+      computed.clear();
+      uint32_t layer_leaves = 0;
+
+      // recursive placement (explicit stack)
+      std::function<void(uint32_t, int, uint32_t)> place_lit;
+      std::function<void(uint32_t, int, uint32_t)> place_node = [&](uint32_t x, int k, uint32_t id) {
+        // pass-throughs above x down to level d[x]
+        while (k > (int)d[x]) {
+          slot[k][id] = -2; sob[k][id] = 1;
+          id = child_a(k, id);
+          k--;
+        }
+        slot[k][id] = (int32_t)x;
+        sxa[k][id] = (uint8_t)(la[x] & 1);
+        sxb[k][id] = (uint8_t)(lb[x] & 1);
+        if (comp_k[x] < 0) { comp_k[x] = k; comp_id[x] = (int32_t)id; computed.push_back(x); }
+        place_lit(la[x], k - 1, child_a(k, id));
+        place_lit(lb[x], k - 1, child_b(k, id));
+      };
+      place_lit = [&](uint32_t l, int k, uint32_t id) {
+        uint32_t x = l >> 1;
+        if (loc[x] >= 0) {
+          while (k > 0) { slot[k][id] = -2; sob[k][id] = 1; id = child_a(k, id); k--; }
+          slot[0][id] = loc[x];
+          thread_leaves[id >> 5]++;
+          layer_leaves++;
+        } else {
+          place_node(x, k, id);
+        }
+      };
+      // bottom (tip, level 13) to top (leaf side)
+      for (int k = 13; k >= 1; k--) {
+        if (cand[k].empty()) continue;
+        // free slots at level k, interleaved over units to spread leaves
+        std::vector<uint32_t> fs;
+        uint32_t g = group_width(k), units = level_slots(k) / g;
+        std::vector<uint32_t> unit_order(units);
+        std::iota(unit_order.begin(), unit_order.end(), 0);
+        if (k <= 5) {
+          // thread order interleaved across warps, least-loaded first
+          std::stable_sort(unit_order.begin(), unit_order.end(), [&](uint32_t a, uint32_t b) {
+            if (thread_leaves[a] != thread_leaves[b]) return thread_leaves[a] < thread_leaves[b];
+            uint32_t ka = (a % 32) * 8 + a / 32, kb = (b % 32) * 8 + b / 32;
+            return ka < kb;
+          });
+        }
+        for (uint32_t q = 0; q < g; q++)
+          for (uint32_t u : unit_order)
+            if (slot[k][u * g + q] == -1) fs.push_back(u * g + q);
+        size_t ci = 0;
+        for (uint32_t id : fs) {
+          // next admissible candidate
+          while (ci < cand[k].size()) {
+            uint32_t x = cand[k][ci];
+            if (comp_k[x] >= 0) { ci++; continue; }           // already computed in this layer
+            if (lf[x] > (uint32_t)opt.leafcap) { ci++; continue; }   // cost filter
+            break;
+          }
+          if (ci >= cand[k].size()) break;
+          uint32_t x = cand[k][ci++];
+          place_node(x, k, id);
+
+        }
+      }
+      if (computed.empty()) { fail(P, "empty layer"); return; }
+      // ---- write-outs: computed values needed by later layers or endpoints
+      std::vector<uint8_t> in_c(0);
+      // mark computed set
+      std::vector<uint32_t> need_wo;
+      for (uint32_t x : computed) {
+        bool need = is_ep[x];
+        if (!need)
+          for (uint32_t j = coff[x]; j < coff[x + 1]; j++) {
+            uint32_t c = cons[j];
+            if (mc[c] && comp_k[c] < 0) { need = true; break; }
+          }
+        if (need) need_wo.push_back(x);
+      }
+      // units with a write-out: thread t (levels 1-5), warp w (6-10), top (11-13)
+      std::vector<int32_t> wo_thread(256, -1), wo_warp(8, -1);
+      int32_t wo_top = -1;
+      auto alloc = [&]() -> int32_t {
+        if (free_words.empty()) return -1;
+        uint32_t w = free_words.back();
+        free_words.pop_back();
+        word_used[w] = 1;
+        return (int32_t)w;
+      };
+      for (uint32_t x : need_wo) {
+        int k = comp_k[x];
+        uint32_t id = (uint32_t)comp_id[x];
+        int32_t* tgt = k <= 5 ? &wo_thread[slot_unit(k, id)] : k <= 10 ? &wo_warp[slot_unit(k, id)] : &wo_top;
+        if (*tgt < 0) { *tgt = alloc(); total_wo++; }
+        if (*tgt < 0) { fail(P, "state overflow"); return; }
+        loc[x] = (int32_t)((uint32_t)*tgt * 32 + slot_bit(k, id));
+        word_vals[(uint32_t)*tgt].push_back(x);
+      }
+      if (opt.verbose >= 2) {
+        uint32_t nwo = 0;
+        for (auto x : wo_thread) nwo += x >= 0;
+        for (auto x : wo_warp) nwo += x >= 0;
+        uint32_t nmc = 0;
+        for (uint32_t i = 0; i < n; i++) nmc += mc[i];
+        fprintf(stderr, "  layer %u: mc=%u computed=%zu need_wo=%zu wo_words=%u leaves=%u free=%zu\n", n_layers, nmc,
+                computed.size(), need_wo.size(), nwo, layer_leaves, free_words.size());
+      }
+      // ---- encode the layer
+      encode_layer(prog_layers, slot, sxa, sxb, sob, wo_thread, wo_warp, wo_top);
+      n_layers++;
+      total_leaves += layer_leaves;
+      for (int k = 1; k <= 13; k++) for (auto s : slot[k]) if (s != -1) slots_used++;
+      // ---- advance: recompute must-compute set, free dead words
+      compute_mc();
+      refresh_free();
+      sort_free();
+      uint32_t hi = 0;
+      for (uint32_t w = 0; w < (uint32_t)opt.max_state_words; w++) if (word_used[w]) hi = w;
+      max_state = std::max(max_state, hi + 1);
+    }
+    // every endpoint must be realised now
+    for (uint32_t i = 0; i < n; i++)
+      if (is_ep[i] && loc[i] < 0) { fail(P, "unrealised endpoint"); return; }
+    // ---- assemble the partition program
+    std::vector<uint32_t>& pr = P.prog;
+    pr.assign(PH_WORDS, 0);
+    pr[PH_MAGIC] = GEM_PART_MAGIC;
+    pr[PH_N_GREAD] = n_gread;
+    pr[PH_N_LAYERS] = n_layers;
+    pr[PH_N_OUT] = (uint32_t)P.outs.size();
+    pr[PH_N_RAM] = (uint32_t)P.rams.size();
+    pr[PH_OFF_GREAD] = (uint32_t)pr.size();
+    for (uint32_t k = 0; k < n_gread; k++) { pr.push_back(gread_src[k]); pr.push_back(k + 1); }
+    while (pr.size() % 4) pr.push_back(0);
+    pr[PH_OFF_LAYERS] = (uint32_t)pr.size();
+    pr.insert(pr.end(), prog_layers.begin(), prog_layers.end());
+    pr[PH_OFF_OUT] = (uint32_t)pr.size();
+    uint32_t n_out = (uint32_t)P.outs.size(), n_out_pad = (n_out + 3) & ~3u;
+    pr[PH_N_OUT_PAD] = n_out_pad;
+    for (uint32_t j = 0; j < n_out_pad; j++) pr.push_back(j < n_out ? P.outs[j].dst : 0);
+    for (uint32_t j = 0; j < n_out; j++)
+      for (int k = 0; k < 32; k++) {
+        uint32_t l = P.outs[j].lit[k];
+        uint32_t x = (uint32_t)scratch[l >> 1];
+        pr.push_back((uint32_t)loc[x] | ((l & 1) ? GEM_OUT_INV : 0u));
+      }
+    pr[PH_OFF_RAM] = (uint32_t)pr.size();
+    for (uint32_t r : P.rams) { pr.push_back(r); pr.push_back(0); pr.push_back(0); pr.push_back(0); }
+    pr[PH_STATE_WORDS] = max_state;
+    pr[PH_N_LEAVES] = total_leaves;
+    pr[PH_N_NODES] = n_and;
+    P.n_layers = n_layers;
+    P.state_words = max_state;
+    P.n_leaves = total_leaves;
+    P.n_writeouts = total_wo;
+    P.slots_used = slots_used;
+    P.ok = true;
+  }
+
+  void fail(Part& P, const char* why) {
+    P.ok = false;
+    P.err = why;
+    for (uint32_t c : cid) (void)c;
+  }
+
+  static void encode_layer(std::vector<uint32_t>& out, std::vector<int32_t>* slot, std::vector<uint8_t>* sxa,
+                           std::vector<uint8_t>* sxb, std::vector<uint8_t>* sob,
+                           const std::vector<int32_t>& wo_thread, const std::vector<int32_t>& wo_warp,
+                           int32_t wo_top) {
+    size_t base = out.size();
+    out.resize(base + LH_WORDS, 0);
+    // leaves per thread
+    std::vector<std::vector<uint32_t>> leaves(256);
+    for (uint32_t id = 0; id < 8192; id++)
+      if (slot[0][id] >= 0) leaves[id >> 5].push_back(GEM_LEAF((uint32_t)slot[0][id], id & 31));
+    uint32_t active = 0;
+    uint32_t niter[8] = {0};
+    for (uint32_t w = 0; w < 8; w++) {
+      for (uint32_t l = 0; l < 32; l++) niter[w] = std::max<uint32_t>(niter[w], (uint32_t)leaves[w * 32 + l].size());
+      bool act = niter[w] > 0 || wo_warp[w] >= 0;
+      for (uint32_t l = 0; l < 32; l++) act = act || wo_thread[w * 32 + l] >= 0;
+      if (act) active |= 1u << w;
+    }
+    auto pack = [&](int k0, int k1, uint32_t unit, const std::vector<uint8_t>* arr) {
+      uint32_t v = 0;
+      for (int k = k0; k <= k1; k++) {
+        uint32_t g = group_width(k);
+        for (uint32_t q = 0; q < g; q++) {
+          uint32_t id = unit * g + q;
+          if (arr[k][id]) v |= 1u << slot_bit(k, id);
+        }
+      }
+      return v;
+    };
+    bool uses_top = wo_top >= 0;
+    out[base + LH_FLAGS] = active | (uses_top ? GEM_LF_USES_TOP : 0u);
+    out[base + LH_TOPC] = pack(11, 13, 0, sxa) | (pack(11, 13, 0, sxb) << 8) | (pack(11, 13, 0, sob) << 16);
+    out[base + LH_TOPWO] = uses_top ? (uint32_t)wo_top : 0u;
+    for (uint32_t w = 0; w < 8; w++) out[base + LH_NITER0 + w] = (active >> w & 1) ? niter[w] : 0;
+    for (uint32_t w = 0; w < 8; w++) {
+      if (!(active >> w & 1)) continue;
+      out.push_back(pack(6, 10, w, sxa));
+      out.push_back(pack(6, 10, w, sxb));
+      out.push_back(pack(6, 10, w, sob));
+      out.push_back(wo_warp[w] >= 0 ? (uint32_t)wo_warp[w] : 0u);
+      for (uint32_t l = 0; l < 32; l++) {
+        uint32_t t = w * 32 + l;
+        out.push_back(pack(1, 5, t, sxa));
+        out.push_back(pack(1, 5, t, sxb));
+        out.push_back(pack(1, 5, t, sob));
+        out.push_back(wo_thread[t] >= 0 ? (uint32_t)wo_thread[t] : 0u);
+      }
+      for (uint32_t i = 0; i < niter[w]; i++)
+        for (uint32_t l = 0; l < 32; l++) {
+          auto& lv = leaves[w * 32 + l];
+          out.push_back(i < lv.size() ? lv[i] : GEM_LEAF(0, 0));
+        }
+    }
+    out[base + LH_WORDS_] = (uint32_t)(out.size() - base);
+  }
+};
+
+// =========================================================== partitioning
+struct Design {
+  Graph G;
+  std::vector<uint32_t> ext_gbit;   // source locations before the internal flop layout
+  Options opt;
+  std::vector<Part> parts;
+  uint32_t q_words = 0, po_words = 0, cut_words = 0, n_stages = 1;
+  std::vector<int64_t> q_ext_of_int, po_ext_of_int;   // internal bit -> external index / -1
+  std::vector<uint32_t> cut_lit;                      // cut index -> compact literal
+};
+
+static uint64_t mix64(uint64_t x) {
+  x ^= x >> 33; x *= 0xff51afd7ed558ccdull; x ^= x >> 33; x *= 0xc4ceb9fe1a85ec53ull; x ^= x >> 33;
+  return x;
+}
+
+// min-hash cone signatures: sig(n) = min(h(n), sig(a), sig(b))
+static std::vector<uint64_t> cone_minhash(const Graph& G, uint64_t seed) {
+  size_t N = G.kind.size();
+  std::vector<uint64_t> s(N);
+  for (size_t i = 0; i < N; i++) {
+    uint64_t h = mix64(i * 0x9E3779B97F4A7C15ull + seed);
+    if (G.kind[i] == K_AND) h = std::min(h, std::min(s[G.a[i] >> 1], s[G.b[i] >> 1]));
+    else if (G.kind[i] == K_CONST) h = UINT64_MAX;
+    s[i] = h;
+  }
+  return s;
+}
+
+static void partition(Design& D) {
+  const Graph& G = D.G;
+  const Options& opt = D.opt;
+  size_t N = G.kind.size();
+  // stage assignment of nodes: stage 1 nodes have level > cut
+  uint32_t cut = 0;
+  if (opt.stages == 2) {
+    cut = opt.cut_level ? (uint32_t)opt.cut_level : std::max<uint32_t>(1, G.max_level / 2);
+  }
+  // ---- units
+  std::vector<Unit> units;
+  auto s0 = cone_minhash(G, 1), s1 = cone_minhash(G, 2);
+  auto key_of = [&](uint32_t lit) -> uint64_t {
+    uint32_t x = lit >> 1;
+    return (uint64_t)((s0[x] & 0xFFFFFFFF00000000ull) | (s1[x] >> 32));
+  };
+  std::vector<uint32_t> cut_nodes;            // compact ids that are stage-0 endpoints
+  std::vector<int32_t> cut_of(N, -1);
+  if (opt.stages == 2) {
+    // cut nodes: level <= cut with a consumer above the cut, or an endpoint above... (endpoints
+    // deeper than the cut are stage-1 units; shallow endpoints stay stage-0 units)
+    std::vector<uint8_t> live(N, 0);
+    for (auto l : G.flop_next) live[l >> 1] = 1;
+    for (auto l : G.po) live[l >> 1] = 1;
+    for (auto& rr : G.rams) for (int p = 0; p < 4; p++) for (int k = 0; k < 32; k++) live[rr.port[p][k] >> 1] = 1;
+    for (size_t i = N; i-- > 0;)
+      if (live[i] && G.kind[i] == K_AND) { live[G.a[i] >> 1] = 1; live[G.b[i] >> 1] = 1; }
+    for (size_t i = 0; i < N; i++) {
+      if (!live[i] || G.kind[i] != K_AND || G.level[i] <= cut) continue;
+      for (uint32_t y : {G.a[i] >> 1, G.b[i] >> 1})
+        if (G.kind[y] == K_AND && G.level[y] <= cut && cut_of[y] < 0) {
+          cut_of[y] = (int32_t)cut_nodes.size();
+          cut_nodes.push_back(y);
+        }
+    }
+  }
+  auto ep_stage = [&](uint32_t lit) -> int {
+    if (opt.stages == 1) return 0;
+    uint32_t x = lit >> 1;
+    return (G.kind[x] == K_AND && G.level[x] > cut) ? 1 : 0;
+  };
+  for (uint32_t j = 0; j < G.n_flops; j++) units.push_back({0, j, key_of(G.flop_next[j])});
+  for (uint32_t j = 0; j < G.n_po; j++) units.push_back({1, j, key_of(G.po[j])});
+  for (uint32_t r = 0; r < G.n_rams; r++) {
+    uint64_t k = UINT64_MAX;
+    for (int p = 0; p < 4; p++) for (int b = 0; b < 32; b++) k = std::min(k, key_of(G.rams[r].port[p][b]));
+    units.push_back({2, r, k});
+  }
+  for (uint32_t c = 0; c < cut_nodes.size(); c++) units.push_back({3, c, key_of(2 * cut_nodes[c])});
+  // unit stage
+  auto unit_stage = [&](const Unit& u) -> int {
+    if (opt.stages == 1) return 0;
+    if (u.kind == 0) return ep_stage(G.flop_next[u.idx]);
+    if (u.kind == 1) return ep_stage(G.po[u.idx]);
+    if (u.kind == 3) return 0;
+    int s = 0;
+    for (int p = 0; p < 4; p++) for (int b = 0; b < 32; b++) s = std::max(s, ep_stage(G.rams[u.idx].port[p][b]));
+    return s;
+  };
+  // sources of a stage-1 cone: cut nodes act as leaves
+  auto is_leaf_for = [&](uint32_t x, int stage) {
+    if (G.kind[x] != K_AND) return true;
+    return stage == 1 && cut_of[x] >= 0;
+  };
+  auto unit_lits = [&](const Unit& u, std::vector<uint32_t>& out) {
+    out.clear();
+    if (u.kind == 0) out.push_back(G.flop_next[u.idx]);
+    else if (u.kind == 1) out.push_back(G.po[u.idx]);
+    else if (u.kind == 2) { for (int p = 0; p < 4; p++) for (int b = 0; b < 32; b++) out.push_back(G.rams[u.idx].port[p][b]); }
+    else out.push_back(2 * cut_nodes[u.idx]);
+  };
+  for (int stage = 0; stage < opt.stages; stage++) {
+    std::vector<Unit> su;
+    for (auto& u : units) if (unit_stage(u) == stage) su.push_back(u);
+    std::stable_sort(su.begin(), su.end(), [](const Unit& a, const Unit& b) { return a.key < b.key; });
+    // cone sizes in stage terms; greedy sequential packing with a size cap
+    std::vector<uint32_t> stamp(N, 0);
+    uint32_t cur_stamp = 0;
+    std::vector<uint32_t> st;
+    std::vector<uint32_t> lits;
+    auto add_cone = [&](const Unit& u) -> uint32_t {
+      uint32_t added = 0;
+      unit_lits(u, lits);
+      for (uint32_t l : lits) {
+        uint32_t x = l >> 1;
+        if (stamp[x] == cur_stamp) continue;
+        stamp[x] = cur_stamp;
+        st.push_back(x);
+        while (!st.empty()) {
+          uint32_t y = st.back(); st.pop_back();
+          if (is_leaf_for(y, stage)) continue;
+          added++;
+          for (uint32_t z : {G.a[y] >> 1, G.b[y] >> 1})
+            if (stamp[z] != cur_stamp) { stamp[z] = cur_stamp; st.push_back(z); }
+        }
+      }
+      return added;
+    };
+    // total stage work estimate
+    uint64_t stage_ands = 0;
+    {
+      cur_stamp++;
+      for (auto& u : su) stage_ands += add_cone(u);
+    }
+    int target = opt.parts > 0 ? opt.parts : (int)std::max<uint64_t>(1, (G.n_and_live + opt.part_size / 2) / opt.part_size);
+    if (opt.stages == 2) target = std::max(1, target / 2);
+    target = std::max(1, std::min<int>(target, (int)su.size()));
+    double cap = std::max<double>(64.0, (double)stage_ands / target * opt.cap_slack);
+    std::vector<std::vector<uint32_t>> groups;   // indices into su
+    for (int iter = 0; iter < 6; iter++) {
+      groups.clear();
+      cur_stamp++;
+      uint64_t size = 0;
+      for (uint32_t i = 0; i < su.size(); i++) {
+        // try adding to the current group
+        if (groups.empty()) groups.emplace_back();
+        uint32_t add = add_cone(su[i]);
+        if (!groups.back().empty() && size + add > cap) {
+          // start a new group containing unit i
+          groups.emplace_back();
+          cur_stamp++;
+          size = add_cone(su[i]);
+          groups.back().push_back(i);
+        } else {
+          size += add;
+          groups.back().push_back(i);
+        }
+      }
+      double ratio = (double)groups.size() / target;
+      if (ratio > 0.9 && ratio < 1.15) break;
+      cap *= std::max(0.5, std::min(2.0, ratio));
+    }
+    for (auto& grp : groups) {
+      Part P;
+      P.stage = stage;
+      for (uint32_t i : grp) {
+        const Unit& u = su[i];
+        if (u.kind == 0) P.flops.push_back(u.idx);
+        else if (u.kind == 1) P.pos.push_back(u.idx);
+        else if (u.kind == 2) P.rams.push_back(u.idx);
+        else P.cuts.push_back(u.idx);
+      }
+      D.parts.push_back(std::move(P));
+    }
+  }
+  D.n_stages = (uint32_t)opt.stages;
+  D.cut_lit.resize(cut_nodes.size());
+  for (size_t c = 0; c < cut_nodes.size(); c++) D.cut_lit[c] = 2 * cut_nodes[c];
+  // stage-1 sources: cut nodes are read from the CUT region; rewrite graph view
+  // by giving cut nodes a gbit (the Mapper treats nodes with gbit as sources
+  // only in stage 1, see layout()).
+  (void)cut;
+}
+
+// internal layout: each partition owns whole internal words for its flops / POs / cuts
+static void layout(Design& D) {
+  Graph& G = D.G;
+  uint32_t qw = 0, pw = 0, cw = 0;
+  D.q_ext_of_int.clear();
+  D.po_ext_of_int.clear();
+  std::vector<uint32_t> q_int_of_ext(G.n_flops), cut_int(D.cut_lit.size());
+  for (auto& P : D.parts) {
+    auto words = [](size_t n) { return (uint32_t)((n + 31) / 32); };
+    for (size_t k = 0; k < P.flops.size(); k++) q_int_of_ext[P.flops[k]] = qw * 32 + (uint32_t)k;
+    for (size_t k = 0; k < P.cuts.size(); k++) cut_int[P.cuts[k]] = cw * 32 + (uint32_t)k;
+    for (uint32_t w = 0; w < words(P.flops.size()); w++)
+      for (int b = 0; b < 32; b++) {
+        size_t k = w * 32 + b;
+        D.q_ext_of_int.push_back(k < P.flops.size() ? (int64_t)P.flops[k] : -1);
+      }
+    for (uint32_t w = 0; w < words(P.pos.size()); w++)
+      for (int b = 0; b < 32; b++) {
+        size_t k = w * 32 + b;
+        D.po_ext_of_int.push_back(k < P.pos.size() ? (int64_t)P.pos[k] : -1);
+      }
+    qw += words(P.flops.size());
+    pw += words(P.pos.size());
+    cw += words(P.cuts.size());
+  }
+  D.q_words = qw; D.po_words = pw; D.cut_words = cw;
+  // rewrite latch source locations to the internal layout
+  if (D.ext_gbit.empty()) D.ext_gbit = G.gbit;
+  for (size_t i = 0; i < G.kind.size(); i++) {
+    if (G.kind[i] != K_SRC) continue;
+    uint32_t gb = D.ext_gbit[i];
+    if ((gb >> 27) == GEM_R_Q) {
+      uint32_t ext = ((gb >> 5) & 0x3FFFFF) * 32 + (gb & 31);
+      uint32_t in = q_int_of_ext[ext];
+      G.gbit[i] = mk_gbit(GEM_R_Q, in / 32, in % 32);
+    }
+  }
+  // output words per partition
+  uint32_t qbase = 0, pbase = 0, cbase = 0;
+  for (auto& P : D.parts) {
+    P.outs.clear();
+    auto emit = [&](uint32_t region, uint32_t base, const std::vector<uint32_t>& idx,
+                    const std::function<uint32_t(uint32_t)>& lit_of) {
+      uint32_t nw = (uint32_t)((idx.size() + 31) / 32);
+      for (uint32_t w = 0; w < nw; w++) {
+        OutWord o;
+        o.dst = GEM_GID(region, base + w);
+        for (int b = 0; b < 32; b++) {
+          size_t k = w * 32 + b;
+          o.lit[b] = k < idx.size() ? lit_of(idx[k]) : 0u;
+        }
+        P.outs.push_back(o);
+      }
+      return nw;
+    };
+    qbase += emit(GEM_R_Q, qbase, P.flops, [&](uint32_t j) { return G.flop_next[j]; });
+    pbase += emit(GEM_R_PO, pbase, P.pos, [&](uint32_t j) { return G.po[j]; });
+    cbase += emit(GEM_R_CUT, cbase, P.cuts, [&](uint32_t c) { return D.cut_lit[c]; });
+    for (uint32_t r = 0; r < P.rams.size(); r++)
+      for (int p = 0; p < 4; p++) {
+        OutWord o;
+        o.dst = GEM_GID(GEM_R_RAMP, r * 4 + p);
+        for (int b = 0; b < 32; b++) o.lit[b] = G.rams[P.rams[r]].port[p][b];
+        P.outs.push_back(o);
+      }
+  }
+  D.cut_lit.clear();
+  // cut nodes become CUT-region sources for stage-1 partitions: remember them
+  D.cut_lit.resize(cut_int.size());
+  for (size_t c = 0; c < cut_int.size(); c++) D.cut_lit[c] = cut_int[c];
+}
+
+// =========================================================== top level
+struct Blob {
+  std::vector<uint32_t> w;
+};
+
+static Blob compile(const char* data, size_t n, const char* opts) {
+  auto t0 = std::chrono::steady_clock::now();
+  Design D;
+  D.opt = parse_opts(opts);
+  Raw raw = read_aiger(data, n);
+  D.G = build_graph(raw);
+  raw = Raw();
+  partition(D);
+  // remember which compact nodes are cut nodes (stage-1 leaves) before layout rewrites cut_lit
+  std::vector<uint32_t> cut_nodes;
+  for (auto& P : D.parts) (void)P;
+  {
+    // cut_lit holds compact literals at this point
+    for (auto l : D.cut_lit) cut_nodes.push_back(l >> 1);
+  }
+  std::vector<uint32_t> cut_compact = D.cut_lit;   // compact literals of cut nodes
+  auto t1 = std::chrono::steady_clock::now();
+  int nth = D.opt.threads > 0 ? D.opt.threads : (int)std::max(1u, std::thread::hardware_concurrency());
+  for (int attempt = 0;; attempt++) {
+    D.cut_lit = cut_compact;
+    layout(D);   // cut_lit now holds internal cut bit indices
+    // Stage-1 partitions see cut nodes as sources: a graph view where cut
+    // nodes are K_SRC with a CUT-region location.
+    Graph G1;
+    bool two = D.n_stages == 2;
+    if (two) {
+      G1 = D.G;
+      for (size_t c = 0; c < cut_nodes.size(); c++) {
+        uint32_t x = cut_nodes[c];
+        uint32_t in = D.cut_lit[c];
+        G1.kind[x] = K_SRC;
+        G1.gbit[x] = mk_gbit(GEM_R_CUT, in / 32, in % 32);
+      }
+    }
+    std::atomic<size_t> next{0};
+    std::vector<std::thread> th;
+    for (int t = 0; t < nth; t++)
+      th.emplace_back([&]() {
+        std::vector<int32_t> scratch(D.G.kind.size(), -1);
+        while (true) {
+          size_t i = next++;
+          if (i >= D.parts.size()) break;
+          Part& P = D.parts[i];
+          Mapper M(P.stage == 1 ? G1 : D.G, D.opt);
+          M.map(P, scratch);
+        }
+      });
+    for (auto& x : th) x.join();
+    // split partitions that did not fit (state overflow) and retry
+    std::vector<Part> next_parts;
+    bool any_fail = false;
+    for (size_t i = 0; i < D.parts.size(); i++) {
+      Part& P = D.parts[i];
+      if (P.ok) { next_parts.push_back(std::move(P)); continue; }
+      any_fail = true;
+      size_t n_units = P.flops.size() + P.pos.size() + P.rams.size() + P.cuts.size();
+      if (n_units <= 1 || attempt >= 12)
+        throw std::runtime_error("mapping partition " + std::to_string(i) + " failed: " + P.err);
+      Part A, B;
+      A.stage = B.stage = P.stage;
+      auto half = [](const std::vector<uint32_t>& v, std::vector<uint32_t>& a, std::vector<uint32_t>& b) {
+        size_t h = (v.size() + 1) / 2;
+        a.assign(v.begin(), v.begin() + h);
+        b.assign(v.begin() + h, v.end());
+      };
+      // keep unit kinds together where possible: split the largest list
+      half(P.flops, A.flops, B.flops);
+      half(P.pos, A.pos, B.pos);
+      half(P.cuts, A.cuts, B.cuts);
+      half(P.rams, A.rams, B.rams);
+      for (Part* X : {&A, &B})
+        if (X->flops.size() + X->pos.size() + X->rams.size() + X->cuts.size()) next_parts.push_back(std::move(*X));
+    }
+    D.parts = std::move(next_parts);
+    if (!any_fail) break;
+    for (auto& P : D.parts) { P.prog.clear(); P.ok = false; }
+    if (D.opt.verbose) fprintf(stderr, "gem_map: retry %d with %zu partitions\n", attempt + 1, D.parts.size());
+  }
+  // drop partitions with no endpoints (possible after splitting)
+  auto t2 = std::chrono::steady_clock::now();
+  // ---- assemble blob
+  Blob B;
+  auto& w = B.w;
+  w.assign(GH_N_WORDS, 0);
+  uint32_t np = (uint32_t)D.parts.size();
+  w[GH_MAGIC] = GEM_MAGIC;
+  w[GH_VERSION] = GEM_VERSION;
+  w[GH_N_PI] = D.G.n_pi;
+  w[GH_N_PO] = D.G.n_po;
+  w[GH_N_FLOPS] = D.G.n_flops;
+  w[GH_N_RAMS] = D.G.n_rams;
+  w[GH_N_PARTS] = np;
+  w[GH_N_STAGES] = D.n_stages;
+  w[GH_PI_WORDS] = (D.G.n_pi + 31) / 32;
+  w[GH_PO_WORDS] = D.po_words;
+  w[GH_Q_WORDS] = D.q_words;
+  w[GH_CUT_WORDS] = D.cut_words;
+  w[GH_N_AND_LO] = (uint32_t)D.G.n_and_live;
+  w[GH_N_AND_HI] = (uint32_t)(D.G.n_and_live >> 32);
+  uint64_t mapped = 0, leaves = 0, slots = 0;
+  uint32_t maxl = 0, maxs = 0, tl = 0, two_ = 0, maxout = 0;
+  for (auto& P : D.parts) {
+    mapped += P.n_nodes; leaves += P.n_leaves; slots += P.slots_used;
+    maxl = std::max(maxl, P.n_layers); maxs = std::max(maxs, P.state_words); tl += P.n_layers;
+    two_ += P.n_writeouts; maxout = std::max<uint32_t>(maxout, (uint32_t)P.outs.size());
+  }
+  w[GH_N_AND_MAPPED_LO] = (uint32_t)mapped;
+  w[GH_N_AND_MAPPED_HI] = (uint32_t)(mapped >> 32);
+  w[GH_MAX_LAYERS] = maxl;
+  w[GH_MAX_STATE_WORDS] = maxs;
+  w[GH_TOTAL_LAYERS] = tl;
+  w[GH_TOTAL_LEAVES_LO] = (uint32_t)leaves;
+  w[GH_TOTAL_LEAVES_HI] = (uint32_t)(leaves >> 32);
+  w[GH_MAX_LEVELS] = D.G.max_level;
+  w[GH_TOTAL_WRITEOUTS] = two_;
+  w[GH_MAX_OUT] = maxout;
+  w[GH_SLOTS_USED_LO] = (uint32_t)slots;
+  w[GH_SLOTS_USED_HI] = (uint32_t)(slots >> 32);
+  // part table
+  w[GH_OFF_PARTS] = (uint32_t)w.size();
+  size_t part_tab = w.size();
+  w.resize(w.size() + (size_t)np * GP_WORDS, 0);
+  // stage list: prefix offsets [n_stages+1] then part ids
+  w[GH_OFF_STAGES] = (uint32_t)w.size();
+  {
+    std::vector<std::vector<uint32_t>> by(D.n_stages);
+    for (uint32_t i = 0; i < np; i++) by[D.parts[i].stage].push_back(i);
+    uint32_t acc = 0;
+    for (uint32_t s = 0; s < D.n_stages; s++) { w.push_back(acc); acc += (uint32_t)by[s].size(); }
+    w.push_back(acc);
+    for (uint32_t s = 0; s < D.n_stages; s++) for (auto i : by[s]) w.push_back(i);
+  }
+  // flop init (internal layout) + permutation tables
+  w[GH_OFF_FLOP_INIT] = (uint32_t)w.size();
+  {
+    size_t base = w.size();
+    w.resize(base + D.q_words, 0);
+    for (size_t b = 0; b < D.q_ext_of_int.size(); b++) {
+      int64_t e = D.q_ext_of_int[b];
+      if (e >= 0 && D.G.flop_init[(size_t)e]) w[base + b / 32] |= 1u << (b % 32);
+    }
+    // q_ext_of_int [q_words*32] then po_ext_of_int [po_words*32] (0xFFFFFFFF = padding)
+    for (auto e : D.q_ext_of_int) w.push_back(e < 0 ? 0xFFFFFFFFu : (uint32_t)e);
+    for (auto e : D.po_ext_of_int) w.push_back(e < 0 ? 0xFFFFFFFFu : (uint32_t)e);
+  }
+  while (w.size() % 4) w.push_back(0);
+  w[GH_OFF_PROG] = (uint32_t)w.size();
+  uint64_t prog = 0;
+  for (uint32_t i = 0; i < np; i++) {
+    auto& P = D.parts[i];
+    w[part_tab + i * GP_WORDS + GP_STAGE] = (uint32_t)P.stage;
+    w[part_tab + i * GP_WORDS + GP_PROG_OFF] = (uint32_t)prog;
+    w[part_tab + i * GP_WORDS + GP_PROG_LEN] = (uint32_t)P.prog.size();
+    w[part_tab + i * GP_WORDS + GP_N_LAYERS] = P.n_layers;
+    w.insert(w.end(), P.prog.begin(), P.prog.end());
+    prog += P.prog.size();
+    while (prog % 4) { w.push_back(0); prog++; }
+  }
+  w[GH_PROG_WORDS_LO] = (uint32_t)prog;
+  w[GH_PROG_WORDS_HI] = (uint32_t)(prog >> 32);
+  w[GH_TOTAL_WORDS_LO] = (uint32_t)w.size();
+  w[GH_TOTAL_WORDS_HI] = (uint32_t)((uint64_t)w.size() >> 32);
+  auto t3 = std::chrono::steady_clock::now();
+  if (D.opt.verbose) {
+    auto ms = [](auto a, auto b) { return std::chrono::duration<double, std::milli>(b - a).count(); };
+    fprintf(stderr, "gem_map: %u parts, %u stages, n_and=%llu mapped=%llu max_layers=%u total_layers=%u "
+            "leaves=%llu prog=%.2f MB  (partition %.0f ms, place %.0f ms, asm %.0f ms)\n",
+            np, D.n_stages, (unsigned long long)D.G.n_and_live, (unsigned long long)mapped, maxl, tl,
+            (unsigned long long)leaves, prog * 4.0 / 1e6, ms(t0, t1), ms(t1, t2), ms(t2, t3));
+  }
+  return B;
+}
+
+}  // namespace gm
+
+// =========================================================== C ABI
+extern "C" {
+
+const char* gem_map_last_error(void) { return gm::g_err.c_str(); }
+
+int gem_compile(const void* eaig, size_t n, const char* opts, void** blob, size_t* nbytes) {
+  if (!eaig || !blob || !nbytes) { gm::g_err = "null argument"; return -1; }
+  try {
+    gm::Blob B = gm::compile((const char*)eaig, n, opts);
+    size_t bytes = B.w.size() * 4;
+    void* p = std::malloc(bytes);
+    if (!p) { gm::g_err = "out of memory"; return -4; }
+    std::memcpy(p, B.w.data(), bytes);
+    *blob = p;
+    *nbytes = bytes;
+    return 0;
+  } catch (const std::exception& e) {
+    gm::g_err = e.what();
+    return -2;
+  }
+}
+
+int gem_compile_file(const char* path, const char* opts, void** blob, size_t* nbytes) {
+  std::ifstream f(path, std::ios::binary);
+  if (!f) { gm::g_err = std::string("cannot open ") + path; return -1; }
+  std::string data((std::istreambuf_iterator<char>(f)), std::istreambuf_iterator<char>());
+  return gem_compile(data.data(), data.size(), opts, blob, nbytes);
+}
+
+void gem_free_blob(void* blob) { std::free(blob); }
+
+}  // extern "C"

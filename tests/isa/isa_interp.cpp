@@ -1,0 +1,220 @@
+// isa_interp.cpp -- TEST TOOL: executes a .gemb program on the CPU by the ISA
+// *definition* in gem_isa.h (slot by slot, level by level), to check the
+// mapper against the oracle without a GPU.  It is not the oracle (it knows
+// partitions/layers) and not a product fallback (nothing in the package loads
+// it).  Hazard checks: a layer's write-out targets must not be read by the
+// same layer's gathers, and state word 0 is never written.
+#include <cstdint>
+#include <cstdio>
+#include <cstdlib>
+#include <cstring>
+#include <string>
+#include <vector>
+
+#include "../../paper_conf_dac_guozwlr25_b200/csrc/gem_isa.h"
+
+namespace {
+thread_local std::string g_err;
+
+struct Interp {
+  std::vector<uint32_t> w;
+  uint32_t n_parts, n_stages, q_words, po_words, cut_words, pi_words, n_rams, n_flops, n_po;
+  const uint32_t* parts;
+  const uint32_t* stages;
+  const uint32_t* prog;
+  const uint32_t* flop_init;
+  const uint32_t* q_ext;
+  const uint32_t* po_ext;
+  std::vector<uint32_t> Q[2], RD[2], CUT;
+  std::vector<std::vector<uint32_t>> MEM;
+  uint64_t cycle = 0;
+};
+
+static inline uint32_t gw(int k) { return k <= 5 ? 1u << (5 - k) : k <= 10 ? 1u << (10 - k) : 1u << (13 - k); }
+static inline uint32_t sbit(int k, uint32_t id) {
+  static const int off[6] = {0, 0, 16, 24, 28, 30};
+  if (k >= 11) return (k == 11 ? 0 : k == 12 ? 4 : 6) + id;
+  int kk = k <= 5 ? k : k - 5;
+  return (uint32_t)off[kk] + id % gw(k);
+}
+
+int run_part(Interp& I, uint32_t p, uint64_t t, const uint32_t* stim, uint32_t* po_row) {
+  const uint32_t* pt = I.parts + p * GP_WORDS;
+  const uint32_t* pr = I.prog + pt[GP_PROG_OFF];
+  if (pr[PH_MAGIC] != GEM_PART_MAGIC) { g_err = "bad part magic"; return -1; }
+  uint32_t cur = (uint32_t)(I.cycle & 1), nxt = cur ^ 1;
+  std::vector<uint32_t> S(GEM_MAX_STATE_WORDS, 0);
+  std::vector<uint8_t> written(GEM_MAX_STATE_WORDS, 0);
+  // gread
+  const uint32_t* gr = pr + pr[PH_OFF_GREAD];
+  for (uint32_t k = 0; k < pr[PH_N_GREAD]; k++) {
+    uint32_t gid = gr[2 * k], dst = gr[2 * k + 1];
+    uint32_t reg = GEM_GID_REGION(gid), idx = GEM_GID_INDEX(gid), v;
+    if (reg == GEM_R_PI) v = stim[idx];
+    else if (reg == GEM_R_Q) v = I.Q[cur][idx];
+    else if (reg == GEM_R_RD) v = I.RD[cur][idx];
+    else if (reg == GEM_R_CUT) v = I.CUT[idx];
+    else { g_err = "bad gread region"; return -1; }
+    if (dst == 0 || dst >= GEM_MAX_STATE_WORDS) { g_err = "bad gread dst"; return -1; }
+    S[dst] = v;
+  }
+  // layers
+  const uint32_t* L = pr + pr[PH_OFF_LAYERS];
+  std::vector<uint8_t> val[14];
+  for (int k = 0; k <= 13; k++) val[k].assign(8192u >> k, 0);
+  for (uint32_t l = 0; l < pr[PH_N_LAYERS]; l++) {
+    uint32_t flags = L[LH_FLAGS];
+    uint32_t topc = L[LH_TOPC];
+    uint32_t lane_c[256][4];
+    uint32_t warp_c[8][4];
+    std::memset(lane_c, 0, sizeof(lane_c));
+    std::memset(warp_c, 0, sizeof(warp_c));
+    for (int k = 0; k <= 13; k++) std::fill(val[k].begin(), val[k].end(), 0);
+    std::vector<uint8_t> read(GEM_MAX_STATE_WORDS, 0);
+    const uint32_t* rec = L + LH_WORDS;
+    for (uint32_t wp = 0; wp < 8; wp++) {
+      if (!((flags >> wp) & 1)) continue;
+      uint32_t niter = L[LH_NITER0 + wp];
+      for (int c = 0; c < 4; c++) warp_c[wp][c] = rec[c];
+      for (uint32_t ln = 0; ln < 32; ln++)
+        for (int c = 0; c < 4; c++) lane_c[wp * 32 + ln][c] = rec[4 + ln * 4 + c];
+      const uint32_t* lv = rec + 4 + 128;
+      for (uint32_t i = 0; i < niter; i++)
+        for (uint32_t ln = 0; ln < 32; ln++) {
+          uint32_t e = lv[i * 32 + ln];
+          uint32_t src = e & 0xFFFF, pos = (e >> 16) & 31;
+          read[src >> 5] = 1;
+          uint32_t bit = (S[src >> 5] >> (src & 31)) & 1u;
+          val[0][(wp * 32 + ln) * 32 + pos] |= (uint8_t)bit;
+        }
+      rec += GEM_WARP_REC_WORDS(niter);
+    }
+    if ((uint32_t)(rec - L) != L[LH_WORDS_]) { g_err = "layer size mismatch"; return -1; }
+    for (int k = 1; k <= 13; k++) {
+      uint32_t g = gw(k);
+      for (uint32_t id = 0; id < (8192u >> k); id++) {
+        uint32_t ca = (id / g) * 2 * g + id % g, cb = ca + g;
+        uint32_t xa, xb, ob, b = sbit(k, id);
+        if (k <= 5) { uint32_t t = id / g; xa = lane_c[t][0]; xb = lane_c[t][1]; ob = lane_c[t][2]; }
+        else if (k <= 10) { uint32_t wq = id / g; xa = warp_c[wq][0]; xb = warp_c[wq][1]; ob = warp_c[wq][2]; }
+        else { xa = topc & 0xFF; xb = (topc >> 8) & 0xFF; ob = (topc >> 16) & 0xFF; }
+        uint32_t A = val[k - 1][ca] ^ ((xa >> b) & 1u);
+        uint32_t B = (val[k - 1][cb] ^ ((xb >> b) & 1u)) | ((ob >> b) & 1u);
+        val[k][id] = (uint8_t)(A & B);
+      }
+    }
+    // write-outs (after all gathers of the layer)
+    auto wo = [&](uint32_t dst, int k0, int k1, uint32_t unit) -> int {
+      if (!dst) return 0;
+      if (dst >= GEM_MAX_STATE_WORDS) { g_err = "bad write-out"; return -1; }
+      if (read[dst]) { g_err = "write-out target read in the same layer"; return -1; }
+      if (written[dst] == 2) { g_err = "two write-outs to one word in a layer"; return -1; }
+      uint32_t v = 0;
+      for (int k = k0; k <= k1; k++) {
+        uint32_t g = gw(k);
+        for (uint32_t q = 0; q < g; q++) v |= (uint32_t)val[k][unit * g + q] << sbit(k, unit * g + q);
+      }
+      S[dst] = v;
+      written[dst] = 2;
+      return 0;
+    };
+    for (uint32_t t = 0; t < 256; t++) if (wo(lane_c[t][3], 1, 5, t)) return -1;
+    for (uint32_t wq = 0; wq < 8; wq++) if (wo(warp_c[wq][3], 6, 10, wq)) return -1;
+    if (flags & GEM_LF_USES_TOP) if (wo(L[LH_TOPWO], 11, 13, 0)) return -1;
+    for (auto& x : written) if (x == 2) x = 1;
+    L += L[LH_WORDS_];
+  }
+  // outputs
+  const uint32_t* od = pr + pr[PH_OFF_OUT];
+  const uint32_t* os = od + pr[PH_N_OUT_PAD];
+  uint32_t ramp[GEM_MAX_RAMS_PER_PART * 4];
+  std::memset(ramp, 0, sizeof(ramp));
+  for (uint32_t j = 0; j < pr[PH_N_OUT]; j++) {
+    uint32_t v = 0;
+    for (int b = 0; b < 32; b++) {
+      uint32_t e = os[j * 32 + b];
+      uint32_t src = e & 0xFFFF;
+      v |= (((S[src >> 5] >> (src & 31)) & 1u) ^ (e >> 31)) << b;
+    }
+    uint32_t reg = GEM_GID_REGION(od[j]), idx = GEM_GID_INDEX(od[j]);
+    if (reg == GEM_R_Q) I.Q[nxt][idx] = v;
+    else if (reg == GEM_R_PO) po_row[idx] = v;
+    else if (reg == GEM_R_CUT) I.CUT[idx] = v;
+    else if (reg == GEM_R_RAMP) ramp[idx] = v;
+    else { g_err = "bad out region"; return -1; }
+  }
+  const uint32_t* rr = pr + pr[PH_OFF_RAM];
+  for (uint32_t r = 0; r < pr[PH_N_RAM]; r++) {
+    uint32_t id = rr[4 * r];
+    uint32_t ra = ramp[4 * r + 0] & 0x1FFF, wa = ramp[4 * r + 1] & 0x1FFF;
+    uint32_t wd = ramp[4 * r + 2], be = ramp[4 * r + 3];
+    I.RD[nxt][id] = I.MEM[id][ra];
+    I.MEM[id][wa] = (I.MEM[id][wa] & ~be) | (wd & be);
+  }
+  (void)t;
+  return 0;
+}
+}  // namespace
+
+extern "C" {
+const char* isa_last_error(void) { return g_err.c_str(); }
+
+void* isa_load(const void* blob, size_t nbytes) {
+  Interp* I = new Interp();
+  I->w.assign((const uint32_t*)blob, (const uint32_t*)blob + nbytes / 4);
+  const uint32_t* h = I->w.data();
+  if (h[GH_MAGIC] != GEM_MAGIC) { g_err = "bad magic"; delete I; return nullptr; }
+  I->n_parts = h[GH_N_PARTS]; I->n_stages = h[GH_N_STAGES];
+  I->q_words = h[GH_Q_WORDS]; I->po_words = h[GH_PO_WORDS]; I->cut_words = h[GH_CUT_WORDS];
+  I->pi_words = h[GH_PI_WORDS]; I->n_rams = h[GH_N_RAMS]; I->n_flops = h[GH_N_FLOPS]; I->n_po = h[GH_N_PO];
+  I->parts = h + h[GH_OFF_PARTS];
+  I->stages = h + h[GH_OFF_STAGES];
+  I->prog = h + h[GH_OFF_PROG];
+  I->flop_init = h + h[GH_OFF_FLOP_INIT];
+  I->q_ext = I->flop_init + I->q_words;
+  I->po_ext = I->q_ext + (size_t)I->q_words * 32;
+  for (int b = 0; b < 2; b++) { I->Q[b].assign(I->q_words, 0); I->RD[b].assign(I->n_rams, 0); }
+  for (uint32_t w = 0; w < I->q_words; w++) I->Q[0][w] = I->flop_init[w];
+  I->CUT.assign(I->cut_words, 0);
+  I->MEM.assign(I->n_rams, std::vector<uint32_t>(GEM_RAM_WORDS, 0));
+  return I;
+}
+
+void isa_free(void* h) { delete (Interp*)h; }
+
+// stim [cycles][pi_words] ; po_ext [cycles][ceil(n_po/32)] ; q_ext [cycles][ceil(n_flops/32)] (nullable)
+int isa_run(void* h, const uint32_t* stim, uint64_t cycles, uint32_t* po_ext, uint32_t* q_ext_tr) {
+  Interp& I = *(Interp*)h;
+  std::vector<uint32_t> po_int(I.po_words);
+  uint32_t pwe = (I.n_po + 31) / 32, qwe = (I.n_flops + 31) / 32;
+  for (uint64_t t = 0; t < cycles; t++) {
+    std::fill(po_int.begin(), po_int.end(), 0);
+    for (uint32_t s = 0; s < I.n_stages; s++)
+      for (uint32_t k = I.stages[s]; k < I.stages[s + 1]; k++) {
+        uint32_t p = I.stages[I.n_stages + 1 + k];
+        if (run_part(I, p, t, stim + t * I.pi_words, po_int.data())) return -1;
+      }
+    I.cycle++;
+    uint32_t cur = (uint32_t)(I.cycle & 1);
+    if (po_ext) {
+      uint32_t* row = po_ext + t * pwe;
+      std::memset(row, 0, pwe * 4);
+      for (uint32_t b = 0; b < I.po_words * 32; b++) {
+        uint32_t e = I.po_ext[b];
+        if (e == 0xFFFFFFFFu) continue;
+        row[e / 32] |= ((po_int[b / 32] >> (b % 32)) & 1u) << (e % 32);
+      }
+    }
+    if (q_ext_tr) {
+      uint32_t* row = q_ext_tr + t * qwe;
+      std::memset(row, 0, qwe * 4);
+      for (uint32_t b = 0; b < I.q_words * 32; b++) {
+        uint32_t e = I.q_ext[b];
+        if (e == 0xFFFFFFFFu) continue;
+        row[e / 32] |= ((I.Q[cur][b / 32] >> (b % 32)) & 1u) << (e % 32);
+      }
+    }
+  }
+  return 0;
+}
+}

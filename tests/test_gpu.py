@@ -1,0 +1,144 @@
+"""GPU parity: the sm_100a path (through the C ABI) vs the CPU oracle, bit-exact.
+
+Bar: the trace of an acyclic 2-state single-clock netlist is
+unique, so every PO and flop must match the oracle at every cycle.
+  C1, C2, small designs: full PO and full flop vector every cycle.
+  C3, C5: full PO trace, per-cycle flop digest, final flops and RAM contents.
+  C4: sampled (a short window; the oracle needs seconds per cycle there).
+"""
+import numpy as np
+import pytest
+
+from gen import stimulus, stimulus_streams
+from gen.stimulus import stim_random
+from oracle import Oracle
+from tests import circuits
+from tests.common import blob, eaig
+
+pytestmark = pytest.mark.gpu
+
+
+@pytest.fixture(scope="module")
+def gem():
+    import torch
+    if not torch.cuda.is_available():
+        pytest.fail("CUDA device required for -m gpu tests")
+    from paper_conf_dac_guozwlr25_b200 import gem as g
+    return g
+
+
+def _full_parity(gem, path, b, stim, n_streams=1, chunks=(None,), **kw):
+    """Run GPU and oracle; compare PO + state trace every cycle."""
+    T = stim.shape[-2]
+    sim = gem.Simulator(b, n_streams=n_streams, flags=gem.GEM_F_TRACE_STATE | gem.GEM_F_DIGEST, **kw)
+    po_g, st_g, dg_g = [], [], []
+    bounds = [0, T] if chunks == (None,) else [0, *chunks, T]
+    for a, e in zip(bounds[:-1], bounds[1:]):
+        sim.set_inputs(stim[..., a:e, :])
+        sim.step(e - a)
+        po_g.append(sim.read_outputs(e - a))
+        st_g.append(sim.read_state_trace(e - a))
+        dg_g.append(sim.read_digests(e - a))
+    po_g = np.concatenate(po_g, 1)
+    st_g = np.concatenate(st_g, 1)
+    dg_g = np.concatenate(dg_g, 1)
+    stims = stim if stim.ndim == 3 else stim[None]
+    for s in range(n_streams):
+        r = Oracle(path).run(stims[s], state=True, digest=True)
+        assert np.array_equal(po_g[s], r["po"]), ("PO", s, np.where((po_g[s] != r["po"]).any(1))[0][:5])
+        assert np.array_equal(st_g[s], r["state"]), ("Q", s, np.where((st_g[s] != r["state"]).any(1))[0][:5])
+        assert np.array_equal(dg_g[s], r["digest"]), ("digest", s)
+    return sim
+
+
+def test_c1_full_10k_cycles(gem):
+    _full_parity(gem, eaig("c1"), blob("c1"), stimulus("c1", 35, 10_000))
+
+
+def test_c1_ragged_steps_and_resume(gem):
+    # run(n)+run(m)+... == run(n+m+...) with ragged chunk sizes
+    _full_parity(gem, eaig("c1"), blob("c1"), stimulus("c1", 35, 1000), chunks=(1, 2, 37, 500))
+
+
+def test_small_designs_with_ram_and_stages(gem, tmp_path):
+    from paper_conf_dac_guozwlr25_b200.mapping import compile_file
+    net = circuits.small_G(seed=21, n_and=4000, with_ram=True)
+    p = circuits.save(net, str(tmp_path), "g")
+    st = stim_random(net.n_pi, 400, 3, reset_pi0_cycles=2)
+    for opts in ["parts=1", "parts=5", "parts=5 stages=2", "parts=3 max_state_words=256"]:
+        _full_parity(gem, p, compile_file(p, opts), st)
+
+
+def test_cells_ram_shift(gem, tmp_path):
+    from paper_conf_dac_guozwlr25_b200.mapping import compile_file
+    rng = np.random.default_rng(5)
+    for name, net in [("cells", circuits.cells()), ("ram", circuits.ram_direct()),
+                      ("sr", circuits.shift_register(70)), ("rc", circuits.random_comb(12, 400, 30, 9))]:
+        p = circuits.save(net, str(tmp_path), name)
+        n_pi = Oracle(p).n_pi
+        st = rng.integers(0, 1 << 32, size=(300, (n_pi + 31) // 32), dtype=np.uint64).astype(np.uint32)
+        if n_pi % 32:
+            st[:, -1] &= (1 << (n_pi % 32)) - 1
+        if name == "ram":
+            st[:, 0] = (st[:, 0] & ~np.uint32(0x3FFFFFF)) | (st[:, 0] & 0x7) | ((st[:, 0] & 0x7) << 13)
+        _full_parity(gem, p, compile_file(p), st)
+
+
+def test_c2_full_parity(gem):
+    _full_parity(gem, eaig("c2"), blob("c2"), stimulus("c2", 128, 2000))
+
+
+def test_c3_parity_digests_and_ram(gem):
+    T = 600
+    st = stimulus("c3", 256, T)
+    sim = gem.Simulator(blob("c3"), flags=gem.GEM_F_DIGEST)
+    sim.set_inputs(st)
+    sim.step(T)
+    po = sim.read_outputs(T)[0]
+    dg = sim.read_digests(T)[0]
+    o = Oracle(eaig("c3"))
+    r = o.run(st, digest=True)
+    assert np.array_equal(po, r["po"])
+    assert np.array_equal(dg, r["digest"])
+    assert np.array_equal(sim.read_state()[0], o.get_state())
+    for ram in range(o.n_rams):
+        assert np.array_equal(sim.read_ram(ram), o.get_ram(ram))
+
+
+def test_c3_state_roundtrip_and_determinism(gem):
+    T = 200
+    st = stimulus("c3", 256, T)
+    a = gem.Simulator(blob("c3"))
+    b = gem.Simulator(blob("c3"))
+    pa = a.run(st)
+    pb = b.run(st)
+    assert np.array_equal(pa, pb)
+    q = a.read_state()
+    c = gem.Simulator(blob("c3"))
+    c.write_state(q)
+    assert np.array_equal(c.read_state(), q)
+
+
+def test_c5_streams_vs_oracle_lanes(gem):
+    """Batched streams: stream s of the GPU == 64-lane oracle lane s (C5 recipe)."""
+    S, T = 64, 120
+    st = stimulus_streams("c5", 256, T, range(S))
+    sim = gem.Simulator(blob("c5"), n_streams=S, flags=gem.GEM_F_DIGEST)
+    sim.set_inputs(st)
+    sim.step(T)
+    po = sim.read_outputs(T)
+    dg = sim.read_digests(T)
+    o = Oracle(eaig("c5"))
+    o.lanes_reset(1)
+    r = o.lanes_run(0, st, digest=True)
+    assert np.array_equal(po, r["po"])
+    assert np.array_equal(dg, r["digest"])
+
+
+def test_noinput_and_bad_args(gem):
+    sim = gem.Simulator(blob("c1"))
+    sim.set_inputs(stimulus("c1", 35, 10))
+    with pytest.raises(gem.GemError):
+        sim.step(11)
+    with pytest.raises(gem.GemError):
+        gem.Simulator(b"\0" * 512)

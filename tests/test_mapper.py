@@ -1,0 +1,77 @@
+"""Mapper + bitstream checks on CPU: the CPU ISA interpreter (tests/isa, a test
+tool executing the ISA definition) must reproduce the oracle exactly, so mapper
+bugs are caught without a GPU.  Metamorphic: partition count, stage count and
+the leaf cap must not change results."""
+import os
+
+import numpy as np
+import pytest
+
+from gen import build_c1, stimulus
+from gen.aig import write_eaig
+from gen.stimulus import stim_random
+from oracle import Oracle
+from paper_conf_dac_guozwlr25_b200.isa import blob_info
+from paper_conf_dac_guozwlr25_b200.mapping import compile_file
+from tests import circuits
+from tests.common import blob, eaig
+from tests.isa import IsaInterp
+
+
+def _check(path, b, stim):
+    r = Oracle(path).run(stim, state=True)
+    po, q = IsaInterp(b).run(stim)
+    assert np.array_equal(po, r["po"]), np.where((po != r["po"]).any(1))[0][:5]
+    assert np.array_equal(q, r["state"]), np.where((q != r["state"]).any(1))[0][:5]
+
+
+def test_c1_isa_matches_oracle(tmp_path):
+    p = os.path.join(str(tmp_path), "c1.aag")
+    write_eaig(build_c1(), p)
+    b = compile_file(p)
+    info = blob_info(b)
+    assert info.n_parts == 1 and info.n_and > 500
+    _check(p, b, stimulus("c1", 35, 3000))
+
+
+@pytest.mark.parametrize("opts", ["parts=1", "parts=3", "parts=6 leafcap=64", "parts=5 stages=2",
+                                  "parts=4 stages=2 cut_level=3", "parts=2 max_state_words=256"])
+def test_small_designs_metamorphic(tmp_path, opts):
+    net = circuits.small_G(seed=21, n_and=4000, with_ram=True)
+    p = circuits.save(net, str(tmp_path), "g")
+    b = compile_file(p, opts)
+    _check(p, b, stim_random(net.n_pi, 150, 3, reset_pi0_cycles=2))
+
+
+@pytest.mark.parametrize("seed", [1, 2, 3])
+def test_random_comb_and_cells(tmp_path, seed):
+    for name, net in [("rc", circuits.random_comb(12, 300, 20, seed)), ("cells", circuits.cells()),
+                      ("sr", circuits.shift_register(40)), ("ram", circuits.ram_direct()),
+                      ("cnt", circuits.counter_with_load())]:
+        p = circuits.save(net, str(tmp_path), name)
+        b = compile_file(p)
+        rng = np.random.default_rng(seed)
+        n_pi = Oracle(p).n_pi
+        st = rng.integers(0, 1 << 32, size=(200, (n_pi + 31) // 32), dtype=np.uint64).astype(np.uint32)
+        if n_pi % 32:
+            st[:, -1] &= (1 << (n_pi % 32)) - 1
+        if name == "ram":   # force same-address traffic
+            st[:, 0] = (st[:, 0] & ~np.uint32(0x3FFFFFF)) | (st[:, 0] & 0x7) | ((st[:, 0] & 0x7) << 13)
+        _check(p, b, st)
+
+
+def test_c2_prefix():
+    _check(eaig("c2"), blob("c2"), stimulus("c2", 128, 120))
+
+
+@pytest.mark.slow
+def test_c3_prefix():
+    _check(eaig("c3"), blob("c3"), stimulus("c3", 256, 12))
+
+
+def test_blob_stats_c2():
+    i = blob_info(blob("c2"))
+    assert i.n_and > 90_000
+    assert i.max_layers >= 40 / 13          # cannot beat 13 levels per layer
+    assert i.max_layers <= 40               # boomerang layers are fewer than levels
+    assert i.max_state_words <= 2048
