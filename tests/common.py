@@ -2,6 +2,7 @@
 from __future__ import annotations
 
 import functools
+import zlib
 import os
 
 import numpy as np
@@ -24,7 +25,7 @@ def eaig(cfg: str) -> str:
 def blob(cfg: str, opts: str = None) -> bytes:
     from paper_conf_dac_guozwlr25_b200.mapping import compile_file
     o = MAP_OPTS[cfg] if opts is None else opts
-    key = f"{cfg}_{abs(hash(o)) % (1 << 32):08x}"
+    key = f"{cfg}_{zlib.crc32(o.encode()):08x}"
     p = os.path.join(CACHE, key + ".gemb")
     src = eaig(cfg)
     if os.path.exists(p) and os.path.getmtime(p) > os.path.getmtime(src):
