@@ -47,6 +47,7 @@ extern "C" {
 #define GEM_F_TRACE_STATE 0x1u  /* record Q(t+1) every cycle (gem_read_state_trace) */
 #define GEM_F_DIGEST 0x2u       /* record the per-cycle flop digest d_t              */
 #define GEM_F_ASYNC 0x4u        /* gem_step returns without synchronising            */
+#define GEM_F_PROFILE 0x8u      /* record per-CTA clock64 phase stamps (first 256 cycles) */
 
 typedef struct gem_sim gem_sim; /* opaque, owned by the library */
 
@@ -62,6 +63,8 @@ typedef struct {
   uint32_t n_pi, n_po, n_flops, n_rams, n_parts, n_stages, max_layers, total_layers;
   uint32_t pi_words, po_words, q_words;   /* external word counts per cycle/stream */
   uint32_t grid, blocks_per_sm, smem_bytes, n_streams;
+  uint32_t resident;     /* 1 = every CTA's programs live in its shared memory */
+  uint32_t ring_slots;   /* else: TMA ring depth used to stream program chunks */
   uint64_t n_and;                          /* live 2-input ANDs (gate evals/cycle) */
   uint64_t n_and_mapped;                   /* with RepCut replication              */
   uint64_t program_bytes;
@@ -106,6 +109,13 @@ int gem_write_ram(gem_sim* sim, uint32_t ram_id, uint32_t stream, const uint32_t
 
 /* Device time (CUDA events on the launch stream) of the last gem_step kernel. */
 int gem_last_step_ms(gem_sim* sim, float* ms);
+
+/* Needs GEM_F_PROFILE: per-cycle, per-CTA SM clock64 stamps of the last step,
+ * uint64 [n_cycles][grid][8]: 0 cycle start, 1 input ports read, 2 layers done,
+ * 3 endpoints+RAM committed (first work item), 4 stage-0 items done,
+ * 5 after the last grid barrier, 6 = layer count of the first item.
+ * Call with dst = NULL to query n_cycles / grid. */
+int gem_read_profile(gem_sim* sim, uint64_t* dst, uint32_t* n_cycles, uint32_t* grid);
 
 void gem_free(gem_sim* sim);
 const char* gem_last_error(void);

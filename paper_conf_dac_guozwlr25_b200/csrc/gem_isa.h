@@ -44,7 +44,7 @@
 #define GEM_WARPS 8
 #define GEM_LEAVES 8192         /* 8,192 bits per boomerang layer */
 #define GEM_LEVELS 13
-#define GEM_MAX_STATE_WORDS 2048  /* 64 Kbit state (16-bit leaf indices) */
+#define GEM_MAX_STATE_WORDS 8192  /* 256 Kbit state (32 KB of shared memory) */
 #define GEM_RAM_ABITS 13
 #define GEM_RAM_WORDS 8192
 #define GEM_MAX_RAMS_PER_PART 32
@@ -69,8 +69,17 @@
 /* output-gather source entry: bit index into S, bit 31 = invert */
 #define GEM_OUT_INV 0x80000000u
 
-/* leaf entry: bits [0,16) = state bit index, bits [16,21) = leaf position */
-#define GEM_LEAF(src, pos) ((uint32_t)(src) | ((uint32_t)(pos) << 16))
+/* leaf entry (gather of one state bit b of word w into leaf position p):
+ *   bits [0,5)   rot = (p - b) mod 32   -> rotl(S[w], rot) puts bit b at p
+ *   bits [5,20)  byte offset of S[w] (w*4; S sits at shared-memory offset 0)
+ *   bits [24,29) p (SPARSE warps only; DENSE warps use entry index = p)
+ * Padding entries are 0: they read S[0] == 0.                                  */
+#define GEM_LEAF(word, bit, pos) \
+  ((((uint32_t)(pos) - (uint32_t)(bit)) & 31u) | ((uint32_t)(word) << 7) | ((uint32_t)(pos) << 24))
+#define GEM_LEAF_DENSE(word, bit, pos) ((((uint32_t)(pos) - (uint32_t)(bit)) & 31u) | ((uint32_t)(word) << 7))
+#define GEM_LEAF_WORD(e) (((e) >> 7) & 0x1FFFu)
+#define GEM_LEAF_ROT(e) ((e) & 31u)
+#define GEM_LEAF_POS(e) (((e) >> 24) & 31u)
 
 /* packed slot-word bit offsets for levels 1..5 of a group */
 #define GEM_OFF_L1 0
@@ -87,29 +96,52 @@ enum {
   GH_TOTAL_LEAVES_LO, GH_TOTAL_LEAVES_HI, GH_OFF_PARTS, GH_OFF_STAGES, GH_OFF_FLOP_INIT,
   GH_OFF_PROG, GH_PROG_WORDS_LO, GH_PROG_WORDS_HI, GH_MAX_LEVELS, GH_TOTAL_WRITEOUTS,
   GH_MAX_OUT, GH_TOTAL_WORDS_LO, GH_TOTAL_WORDS_HI, GH_SLOTS_USED_LO, GH_SLOTS_USED_HI,
+  GH_MAX_CHUNK_WORDS, GH_MAX_PROG_WORDS,
   GH_N_WORDS = 64
 };
 
-/* part table entry (4 words) */
-enum { GP_STAGE = 0, GP_PROG_OFF, GP_PROG_LEN, GP_N_LAYERS, GP_WORDS = 4 };
+/* part table entry (8 words) */
+enum {
+  GP_STAGE = 0, GP_PROG_OFF, GP_PROG_LEN, GP_N_LAYERS, GP_CHUNK0, GP_MAX_CHUNK, GP_CHUNK1, GP_CHUNK2,
+  GP_COST, GP_R9, GP_R10, GP_R11, GP_WORDS = 12
+};
+/* GP_COST: mapper's estimate of one cycle of the partition in SM clocks (used by
+ * the runtime's longest-processing-time work-list scheduling). */
+/* GP_CHUNK1/2: sizes of chunks 1 and 2 (0 if absent) so the first three chunks of
+ * the next work item can be prefetched before its chunk table has arrived. */
 
+/* A partition program is a sequence of "chunks" streamed into shared memory by
+ * TMA bulk copies (cp.async.bulk, 16-byte granules): chunk 0 = header + chunk
+ * table + gread list, chunks 1..n_layers = one layer record each, chunk
+ * n_layers+1 = output + RAM sections.  The chunk table (PH_OFF_CHUNKS) holds
+ * the word size of every chunk (all multiples of 4 words).                  */
 /* partition program header (16 words) */
 enum {
   PH_MAGIC = 0, PH_N_GREAD, PH_N_LAYERS, PH_N_OUT, PH_N_RAM, PH_STATE_WORDS, PH_OFF_GREAD,
-  PH_OFF_LAYERS, PH_OFF_OUT, PH_OFF_RAM, PH_N_LEAVES, PH_N_NODES, PH_N_OUT_PAD, PH_R13,
-  PH_R14, PH_R15, PH_WORDS = 16
+  PH_OFF_LAYERS, PH_OFF_OUT, PH_OFF_RAM, PH_N_LEAVES, PH_N_NODES, PH_N_OUT_PAD, PH_OFF_CHUNKS,
+  PH_N_CHUNKS, PH_R15, PH_WORDS = 16
 };
 #define GEM_PART_MAGIC 0x54524150u  /* "PART" */
 
 /* layer header (16 words) followed by one record per active warp:
- *   wconst[4] = {wxa, wxb, wob, wwo}
- *   lane[32][4] = {xa, xb, ob, wo}         (uint4 per lane)
- *   leaves[n_iter][32]                      (lane-minor, coalesced)       */
+ *   [LH_WORDS_] layer size in words, [LH_FLAGS] active-warp mask | USES_TOP,
+ *   [LH_TOPC] top constants, [LH_TOPWO] top write-out word,
+ *   [LH_WOFF0 + w] word offset of warp w's record from the layer start (0 = inactive)
+ * warp record:
+ *   [0..3]  wxa, wxb, wob, wwo           (levels 6-10 constants, write-out)
+ *   [4]     mode (GEM_WM_DENSE / GEM_WM_SPARSE) | n4 << 8   (n4 = uint4 leaf groups per lane)
+ *   [5..7]  reserved
+ *   [8..136) lane constants: uint4 {xa, xb, ob, wo} per lane (levels 1-5)
+ *   [136..) leaves: [n4][32 lanes] x uint4 (4 entries per lane per group)
+ * DENSE warps have n4 = 8 and entry j of a lane fills leaf position j.        */
 enum {
-  LH_WORDS_ = 0, LH_FLAGS, LH_TOPC, LH_TOPWO, LH_NITER0 /* ..LH_NITER0+7 */, LH_WORDS = 16
+  LH_WORDS_ = 0, LH_FLAGS, LH_TOPC, LH_TOPWO, LH_WOFF0 /* ..LH_WOFF0+7 */, LH_WORDS = 16
 };
 #define GEM_LF_USES_TOP 0x100u   /* flags bit 8; bits [0,8) = active warp mask */
-#define GEM_WARP_REC_WORDS(n_iter) (4 + 32 * 4 + 32 * (n_iter))
+#define GEM_WM_SPARSE 0u
+#define GEM_WM_DENSE 1u
+#define GEM_WREC_HDR 8
+#define GEM_WARP_REC_WORDS(n4) (GEM_WREC_HDR + 32 * 4 + 128 * (n4))
 
 /* output section: dst gid [n_out_pad] then src [n_out][32]
  * RAM section: per owned RAM 4 words {ram_id, 0, 0, 0}; its ports are staged by

@@ -53,7 +53,17 @@ struct KParams {
   uint32_t n_stages, n_streams, state_words;
   uint32_t pi_words, po_words, q_words, cut_words, n_rams, n_flops, q_ext_words;
   uint32_t flags;
+  uint32_t area_words, slot_words, ring_slots, allow_resident;
+  unsigned long long* prof;   // GEM_F_PROFILE: [prof_cycles][grid][8] clock64 stamps
+  uint32_t prof_cycles;
+  const uint32_t* __restrict__ wl_off;   // [n_stages][grid+1] CSR offsets into wl_items
+  const uint2* __restrict__ wl_items;    // {partition, stream} per work item
 };
+#define PROF(slot_)                                                                          \
+  do {                                                                                       \
+    if (prof_on && threadIdx.x == 0)                                                         \
+      kp.prof[((size_t)c * gridDim.x + blockIdx.x) * 8 + (slot_)] = (unsigned long long)clock64(); \
+  } while (0)
 
 __device__ __forceinline__ unsigned long long ld_acquire_u64(const unsigned long long* p) {
   unsigned long long v;
@@ -114,21 +124,250 @@ __device__ __forceinline__ uint32_t fold3(uint32_t v, uint32_t xa, uint32_t xb, 
 
 __device__ __forceinline__ uint32_t rd_global(const uint32_t* p) { return __ldcg(p); }
 
-__device__ void run_partition(const KParams& kp, uint32_t* S, uint32_t* ramp, uint32_t* topb, uint32_t p,
-                              uint32_t st, uint32_t c, uint32_t cur, uint32_t nxt) {
+// ---------------------------------------------------------------- TMA / mbarrier
+__device__ __forceinline__ uint32_t smem_u32(const void* p) {
+  return (uint32_t)__cvta_generic_to_shared(p);
+}
+__device__ __forceinline__ void mbar_init(uint64_t* bar, uint32_t count) {
+  asm volatile("mbarrier.init.shared::cta.b64 [%0], %1;" ::"r"(smem_u32(bar)), "r"(count) : "memory");
+}
+__device__ __forceinline__ void mbar_expect_tx(uint64_t* bar, uint32_t bytes) {
+  asm volatile("mbarrier.arrive.expect_tx.shared::cta.b64 _, [%0], %1;" ::"r"(smem_u32(bar)), "r"(bytes)
+               : "memory");
+}
+__device__ __forceinline__ void mbar_wait(uint64_t* bar, uint32_t parity) {
+  uint32_t done = 0;
+  while (!done) {
+    asm volatile(
+        "{\n .reg .pred p;\n mbarrier.try_wait.parity.shared::cta.b64 p, [%1], %2;\n selp.u32 %0, 1, 0, p;\n}\n"
+        : "=r"(done)
+        : "r"(smem_u32(bar)), "r"(parity)
+        : "memory");
+  }
+}
+// 1-D bulk copy global -> shared (TMA engine), completion signalled on `bar`.
+// bytes must be a multiple of 16 and both addresses 16-byte aligned.
+__device__ __forceinline__ void tma_load_1d(void* dst, const void* src, uint32_t bytes, uint64_t* bar) {
+  asm volatile(
+      "cp.async.bulk.shared::cluster.global.mbarrier::complete_tx::bytes [%0], [%1], %2, [%3];" ::"r"(
+          smem_u32(dst)),
+      "l"(src), "r"(bytes), "r"(smem_u32(bar))
+      : "memory");
+}
+__device__ __forceinline__ void fence_mbar_init() {
+  asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
+}
+
+#define GEM_RING_MAX 4
+#define GEM_MAX_CHUNKS 256
+#define GEM_MAX_RESIDENT 16
+
+// Shared-memory program source: either every program of this CTA resident
+// (copied once per launch) or a ring of R slots fed chunk by chunk by TMA.
+struct ProgSrc {
+  uint64_t* mbar;        // [GEM_RING_MAX + 1]; last one = residency barrier
+  uint32_t* area;        // resident programs or ring slots
+  uint32_t* ctab;        // chunk table copy (streamed mode)
+  uint32_t slot_words, R;
+  uint32_t seq_issue, seq_wait, seq_free;   // chunk sequence numbers (uniform across the CTA)
+  bool resident;
+  uint32_t n_res;
+  const uint32_t* res_p;   // smem [GEM_MAX_RESIDENT] partition ids
+  const uint32_t* res_off; // smem [GEM_MAX_RESIDENT] word offsets into area
+};
+
+__device__ __forceinline__ uint32_t* ring_slot(const ProgSrc& ps, uint32_t seq) {
+  return ps.area + (size_t)(seq % ps.R) * ps.slot_words;
+}
+// All threads call this (uniformly); thread 0 issues the copy.
+__device__ __forceinline__ void ring_issue(ProgSrc& ps, const uint32_t* g, uint32_t words) {
+  const uint32_t seq = ps.seq_issue++;
+  if (threadIdx.x == 0) {
+    uint64_t* bar = ps.mbar + seq % ps.R;
+    mbar_expect_tx(bar, words * 4);
+    tma_load_1d(ring_slot(ps, seq), g, words * 4, bar);
+  }
+}
+__device__ __forceinline__ const uint32_t* ring_wait(ProgSrc& ps) {
+  const uint32_t seq = ps.seq_wait++;
+  mbar_wait(ps.mbar + seq % ps.R, (seq / ps.R) & 1u);
+  return ring_slot(ps, seq);
+}
+
+// Prologue of a work item in streamed mode: its first min(R, 3, n_chunks)
+// chunks, sized from the partition table (issued before the item starts,
+// e.g. while the CTA waits at the grid barrier).
+__device__ __forceinline__ uint32_t prologue_count(const KParams& kp, const ProgSrc& ps, uint32_t p) {
+  const uint32_t nch = __ldg(kp.parts + p * GP_WORDS + GP_N_LAYERS) + 2;
+  return min(min(ps.R, 3u), nch);
+}
+__device__ __forceinline__ void issue_prologue(const KParams& kp, ProgSrc& ps, uint32_t p) {
+  const uint32_t* g = kp.prog + __ldg(kp.parts + p * GP_WORDS + GP_PROG_OFF);
+  const uint32_t k = prologue_count(kp, ps, p);
+  const uint32_t sz[3] = {__ldg(kp.parts + p * GP_WORDS + GP_CHUNK0), __ldg(kp.parts + p * GP_WORDS + GP_CHUNK1),
+                          __ldg(kp.parts + p * GP_WORDS + GP_CHUNK2)};
+  uint32_t off = 0;
+  for (uint32_t i = 0; i < k; i++) {
+    ring_issue(ps, g + off, sz[i]);
+    off += sz[i];
+  }
+}
+
+// Explicit shared-window accesses (32-bit addresses): avoids generic->shared
+// conversions in the hot loops.
+__device__ __forceinline__ uint32_t lds(uint32_t addr) {
+  uint32_t v;
+  asm volatile("ld.shared.u32 %0, [%1];" : "=r"(v) : "r"(addr));
+  return v;
+}
+__device__ __forceinline__ void sts(uint32_t addr, uint32_t v) {
+  asm volatile("st.shared.u32 [%0], %1;" ::"r"(addr), "r"(v) : "memory");
+}
+
+// Gather of one leaf entry: rotate the source state word so bit b lands on
+// leaf position p (gem_isa.h).  S sits at the start of dynamic shared memory,
+// so the entry's byte-offset field plus the window base addresses it.
+__device__ __forceinline__ uint32_t leaf_rot(uint32_t s_base, uint32_t e, uint32_t byte_mask) {
+  const uint32_t s = lds(s_base + ((e >> 5) & byte_mask));
+  return __funnelshift_l(s, s, e);   // rotl(s, e & 31)
+}
+template <int N4>
+__device__ __forceinline__ uint32_t gather_sparse(uint32_t s_base, const uint4* e) {
+  uint32_t v = 0;
+#pragma unroll
+  for (int g = 0; g < N4; g++) {
+    v |= leaf_rot(s_base, e[g].x, 0x7FFFu) & (1u << GEM_LEAF_POS(e[g].x));
+    v |= leaf_rot(s_base, e[g].y, 0x7FFFu) & (1u << GEM_LEAF_POS(e[g].y));
+    v |= leaf_rot(s_base, e[g].z, 0x7FFFu) & (1u << GEM_LEAF_POS(e[g].z));
+    v |= leaf_rot(s_base, e[g].w, 0x7FFFu) & (1u << GEM_LEAF_POS(e[g].w));
+  }
+  return v;
+}
+
+// Per-thread registers of one layer record: everything that does not depend
+// on the state, so it can be loaded before the barrier of the previous layer.
+struct LayerRegs {
+  uint4 e[8];
+  uint4 lc, wc;
+  uint32_t mode, flags, topc, topwo;
+};
+
+__device__ __forceinline__ void load_layer(const uint32_t* L, LayerRegs& R) {
+  const uint32_t lane = threadIdx.x & 31, warp = threadIdx.x >> 5;
+  const uint4 lh0 = *reinterpret_cast<const uint4*>(L);
+  R.flags = lh0.y;
+  R.topc = lh0.z;
+  R.topwo = lh0.w;
+  if ((R.flags >> warp) & 1u) {
+    const uint32_t* rec = L + L[LH_WOFF0 + warp];
+    R.wc = *reinterpret_cast<const uint4*>(rec);
+    R.mode = rec[4];
+    R.lc = *(reinterpret_cast<const uint4*>(rec + GEM_WREC_HDR) + lane);
+    const uint4* lv = reinterpret_cast<const uint4*>(rec + GEM_WREC_HDR + 128) + lane;
+    const uint32_t n4 = R.mode >> 8;
+#pragma unroll
+    for (uint32_t g = 0; g < 8; g++) R.e[g] = g < n4 ? lv[g * 32] : make_uint4(0u, 0u, 0u, 0u);
+  }
+}
+
+// Rows a3-a5 of one layer with pre-loaded records: gather (bit permutation),
+// 13-level boomerang fold, write-outs.  No trailing barrier.
+__device__ __forceinline__ void exec_layer(const LayerRegs& R, uint32_t s_base, uint32_t* topb) {
+  const uint32_t lane = threadIdx.x & 31, warp = threadIdx.x >> 5;
+  const bool uses_top = (R.flags & GEM_LF_USES_TOP) != 0;
+  if ((R.flags >> warp) & 1u) {
+    uint32_t v = 0;
+    const uint32_t n4 = R.mode >> 8;
+    if ((R.mode & 0xFFu) == GEM_WM_DENSE) {
+      // entry j of the lane fills leaf position j: rotate + LOP3 with an immediate mask
+#pragma unroll
+      for (uint32_t g = 0; g < 8; g++) {
+        v |= leaf_rot(s_base, R.e[g].x, 0xFFFFFFFFu) & (1u << (4 * g + 0));
+        v |= leaf_rot(s_base, R.e[g].y, 0xFFFFFFFFu) & (1u << (4 * g + 1));
+        v |= leaf_rot(s_base, R.e[g].z, 0xFFFFFFFFu) & (1u << (4 * g + 2));
+        v |= leaf_rot(s_base, R.e[g].w, 0xFFFFFFFFu) & (1u << (4 * g + 3));
+      }
+    } else if (n4 <= 1) {
+      v = gather_sparse<1>(s_base, R.e);
+    } else if (n4 <= 2) {
+      v = gather_sparse<2>(s_base, R.e);
+    } else if (n4 <= 4) {
+      v = gather_sparse<4>(s_base, R.e);
+    } else {
+      v = gather_sparse<8>(s_base, R.e);
+    }
+    const uint32_t P = fold5(v, R.lc.x, R.lc.y, R.lc.z);
+    if (R.lc.w) sts(s_base + 4 * R.lc.w, P);
+    const uint32_t u = __ballot_sync(0xFFFFFFFFu, (P >> 30) & 1u);
+    const uint32_t Pw = fold5(u, R.wc.x, R.wc.y, R.wc.z);
+    if (lane == 0) {
+      if (R.wc.w) sts(s_base + 4 * R.wc.w, Pw);
+      if (uses_top) topb[warp] = (Pw >> 30) & 1u;
+    }
+  } else if (uses_top && lane == 0) {
+    topb[warp] = 0u;
+  }
+}
+
+__device__ __forceinline__ void exec_top(uint32_t flags, uint32_t topc, uint32_t topwo, uint32_t* S,
+                                         const uint32_t* topb) {
+  if (flags & GEM_LF_USES_TOP) {
+    __syncthreads();
+    if (threadIdx.x == 0) {
+      uint32_t t8 = 0;
+#pragma unroll
+      for (uint32_t w = 0; w < GEM_WARPS; w++) t8 |= topb[w] << w;
+      S[topwo] = fold3(t8, topc & 0xFFu, (topc >> 8) & 0xFFu, (topc >> 16) & 0xFFu);
+    }
+  }
+}
+
+// One work item = one partition for one stream in one cycle.  In streamed
+// mode the caller has already issued the item's prologue chunks.
+__device__ void run_partition(const KParams& kp, ProgSrc& ps, uint32_t* S, uint32_t* ramp, uint32_t* topb,
+                              uint32_t p, uint32_t st, uint32_t c, uint32_t cur, uint32_t nxt, bool prof_on) {
   const uint32_t tid = threadIdx.x, lane = tid & 31, warp = tid >> 5;
-  const uint32_t* pr = kp.prog + __ldg(kp.parts + p * GP_WORDS + GP_PROG_OFF);
-  const uint4 h0 = __ldg(reinterpret_cast<const uint4*>(pr));
-  const uint4 h1 = __ldg(reinterpret_cast<const uint4*>(pr) + 1);
-  const uint4 h2 = __ldg(reinterpret_cast<const uint4*>(pr) + 2);
-  const uint4 h3 = __ldg(reinterpret_cast<const uint4*>(pr) + 3);
+  const uint32_t s_base = smem_u32(S);
+  const uint32_t* gprog = kp.prog + __ldg(kp.parts + p * GP_WORDS + GP_PROG_OFF);
+  const uint32_t* C0;
+  const uint32_t* ctab;
+  uint32_t next_chunk = 0, next_off = 0;
+  if (ps.resident) {
+    uint32_t off = 0;
+    for (uint32_t k = 0; k < ps.n_res; k++) if (ps.res_p[k] == p) off = ps.res_off[k];
+    C0 = ps.area + off;
+    ctab = C0 + C0[PH_OFF_CHUNKS];
+  } else {
+    next_chunk = prologue_count(kp, ps, p);
+    next_off = __ldg(kp.parts + p * GP_WORDS + GP_CHUNK0);
+    if (next_chunk > 1) next_off += __ldg(kp.parts + p * GP_WORDS + GP_CHUNK1);
+    if (next_chunk > 2) next_off += __ldg(kp.parts + p * GP_WORDS + GP_CHUNK2);
+    C0 = ring_wait(ps);
+    // keep the chunk table: chunk 0's slot is recycled
+    const uint32_t nch = C0[PH_N_CHUNKS];
+    for (uint32_t k = tid; k < nch; k += GEM_THREADS) ps.ctab[k] = C0[C0[PH_OFF_CHUNKS] + k];
+    ctab = C0 + C0[PH_OFF_CHUNKS];
+  }
+  const uint4 h0 = *reinterpret_cast<const uint4*>(C0);
+  const uint4 h1 = *(reinterpret_cast<const uint4*>(C0) + 1);
+  const uint4 h2 = *(reinterpret_cast<const uint4*>(C0) + 2);
+  const uint4 h3 = *(reinterpret_cast<const uint4*>(C0) + 3);
   const uint32_t n_gread = h0.y, n_layers = h0.z, n_out = h0.w;
   const uint32_t n_ram = h1.x, off_gread = h1.z, off_layers = h1.w;
-  const uint32_t off_out = h2.x, off_ram = h2.y, n_out_pad = h3.x;
+  const uint32_t off_out = h2.x, off_ram = h2.y, n_out_pad = h3.x, n_chunks = h3.z;
+  auto refill = [&]() {   // issue chunks into free ring slots
+    if (!ps.resident)
+      while (next_chunk < n_chunks && ps.seq_issue - ps.seq_free < ps.R) {
+        const uint32_t words = ps.ctab[next_chunk];
+        ring_issue(ps, gprog + next_off, words);
+        next_off += words;
+        next_chunk++;
+      }
+  };
   // ---- a2: global read of input ports (once per cycle)
-  const uint32_t* gr = pr + off_gread;
+  const uint32_t* gr = C0 + off_gread;
   for (uint32_t k = tid; k < n_gread; k += GEM_THREADS) {
-    const uint2 e = __ldg(reinterpret_cast<const uint2*>(gr) + k);
+    const uint2 e = *(reinterpret_cast<const uint2*>(gr) + k);
     const uint32_t reg = GEM_GID_REGION(e.x), idx = GEM_GID_INDEX(e.x);
     uint32_t v;
     if (reg == GEM_R_PI) v = __ldg(kp.pi + ((size_t)st * kp.in_cap + kp.in_base + c) * kp.pi_words + idx);
@@ -138,71 +377,46 @@ __device__ void run_partition(const KParams& kp, uint32_t* S, uint32_t* ramp, ui
     S[e.y] = v;
   }
   if (tid == 0) S[0] = 0u;
-  __syncthreads();
-  // ---- a3-a5: layers
-  const uint32_t* L = pr + off_layers;
-  for (uint32_t l = 0; l < n_layers; l++) {
-    const uint4 lh0 = __ldg(reinterpret_cast<const uint4*>(L));
-    const uint4 n03 = __ldg(reinterpret_cast<const uint4*>(L) + 1);
-    const uint4 n47 = __ldg(reinterpret_cast<const uint4*>(L) + 2);
-    const uint32_t flags = lh0.y, topc = lh0.z, topwo = lh0.w;
-    const uint32_t niter_all[8] = {n03.x, n03.y, n03.z, n03.w, n47.x, n47.y, n47.z, n47.w};
-    const bool uses_top = (flags & GEM_LF_USES_TOP) != 0;
-    if ((flags >> warp) & 1u) {
-      uint32_t off = LH_WORDS;
-#pragma unroll
-      for (uint32_t w = 0; w < GEM_WARPS; w++)
-        if (w < warp && ((flags >> w) & 1u)) off += GEM_WARP_REC_WORDS(niter_all[w]);
-      const uint32_t* rec = L + off;
-      uint32_t niter = 0;
-#pragma unroll
-      for (uint32_t w = 0; w < GEM_WARPS; w++) if (w == warp) niter = niter_all[w];
-      const uint4 wc = __ldg(reinterpret_cast<const uint4*>(rec));
-      const uint4 lc = __ldg(reinterpret_cast<const uint4*>(rec + 4) + lane);
-      // gather (bit permutation)
-      const uint32_t* lv = rec + 4 + 128 + lane;
-      uint32_t v = 0;
-#pragma unroll 4
-      for (uint32_t i = 0; i < niter; i++) {
-        const uint32_t e = __ldg(lv + i * 32);
-        const uint32_t s = S[(e & 0xFFFFu) >> 5];
-        v |= ((s >> (e & 31u)) & 1u) << ((e >> 16) & 31u);
-      }
-      // fold levels 1-5 in-thread
-      const uint32_t P = fold5(v, lc.x, lc.y, lc.z);
-      if (lc.w) S[lc.w] = P;
-      // levels 6-10 in-warp
-      const uint32_t u = __ballot_sync(0xFFFFFFFFu, (P >> 30) & 1u);
-      const uint32_t Pw = fold5(u, wc.x, wc.y, wc.z);
-      if (lane == 0) {
-        if (wc.w) S[wc.w] = Pw;
-        if (uses_top) topb[warp] = (Pw >> 30) & 1u;
-      }
-    } else if (uses_top && lane == 0) {
-      topb[warp] = 0u;
-    }
-    if (uses_top) {
-      __syncthreads();
-      if (tid == 0) {
-        uint32_t t8 = 0;
-#pragma unroll
-        for (uint32_t w = 0; w < GEM_WARPS; w++) t8 |= topb[w] << w;
-        S[topwo] = fold3(t8, topc & 0xFFu, (topc >> 8) & 0xFFu, (topc >> 16) & 0xFFu);
-      }
-    }
-    __syncthreads();
-    L += lh0.x;
+  // first layer's records (independent of S) before the barrier
+  LayerRegs R;
+  const uint32_t* Lres = C0 + off_layers;
+  if (n_layers) {
+    const uint32_t* L;
+    if (ps.resident) { L = Lres; Lres += ctab[1]; }
+    else L = ring_wait(ps);
+    load_layer(L, R);
   }
+  __syncthreads();   // S ready; chunk 0 and layer 0's chunk consumed
+  if (!ps.resident) ps.seq_free += n_layers ? 2 : 1;
+  PROF(1);
+  refill();
+  // ---- a3-a5: layers, software-pipelined: layer l+1's records are loaded
+  // into registers before the barrier that ends layer l
+  for (uint32_t l = 0; l < n_layers; l++) {
+    exec_layer(R, s_base, topb);
+    const uint32_t flags = R.flags, topc = R.topc, topwo = R.topwo;
+    if (l + 1 < n_layers) {
+      const uint32_t* L;
+      if (ps.resident) { L = Lres; Lres += ctab[2 + l]; }
+      else L = ring_wait(ps);
+      load_layer(L, R);
+    }
+    exec_top(flags, topc, topwo, S, topb);
+    __syncthreads();
+    if (!ps.resident && l + 1 < n_layers) ps.seq_free++;
+    refill();
+  }
+  PROF(2);
   // ---- a6: endpoint commit (warp ballot-gather per output word)
-  const uint32_t* od = pr + off_out;
+  const uint32_t* od = ps.resident ? (C0 + off_out) : ring_wait(ps);
   const uint32_t* os = od + n_out_pad;
   for (uint32_t j = warp; j < n_out; j += GEM_WARPS) {
-    const uint32_t e = __ldg(os + j * 32 + lane);
-    const uint32_t src = e & 0xFFFFu;
+    const uint32_t e = os[j * 32 + lane];
+    const uint32_t src = e & 0x7FFFFFFFu;
     const uint32_t bit = ((S[src >> 5] >> (src & 31u)) & 1u) ^ (e >> 31);
     const uint32_t v = __ballot_sync(0xFFFFFFFFu, bit);
     if (lane == 0) {
-      const uint32_t dst = __ldg(od + j);
+      const uint32_t dst = od[j];
       const uint32_t reg = GEM_GID_REGION(dst), idx = GEM_GID_INDEX(dst);
       if (reg == GEM_R_Q) __stcg(kp.q + ((size_t)nxt * kp.n_streams + st) * kp.q_words + idx, v);
       else if (reg == GEM_R_PO) __stcg(kp.po + ((size_t)st * kp.out_cap + c) * kp.po_words + idx, v);
@@ -213,9 +427,9 @@ __device__ void run_partition(const KParams& kp, uint32_t* S, uint32_t* ramp, ui
   // ---- a7: RAM blocks (read-first, then per-bit write; readings U7-U10)
   if (n_ram) {
     __syncthreads();
-    const uint32_t* rr = pr + off_ram;
+    const uint32_t* rr = od + (off_ram - off_out);
     for (uint32_t r = tid; r < n_ram; r += GEM_THREADS) {
-      const uint32_t id = __ldg(rr + 4 * r);
+      const uint32_t id = rr[4 * r];
       const uint32_t ra = ramp[4 * r + GEM_PORT_RADDR] & (GEM_RAM_WORDS - 1);
       const uint32_t wa = ramp[4 * r + GEM_PORT_WADDR] & (GEM_RAM_WORDS - 1);
       const uint32_t wd = ramp[4 * r + GEM_PORT_WDATA], be = ramp[4 * r + GEM_PORT_WBE];
@@ -226,7 +440,10 @@ __device__ void run_partition(const KParams& kp, uint32_t* S, uint32_t* ramp, ui
       __stcg(kp.rd + ((size_t)nxt * kp.n_streams + st) * kp.n_rams + id, old);
     }
   }
-  __syncthreads();  // S / ramp reused by the next work item
+  __syncthreads();  // S / ramp / ring slots reused by the next work item
+  if (!ps.resident) ps.seq_free = ps.seq_issue;   // every chunk of this item consumed
+  PROF(3);
+  if (prof_on && tid == 0) kp.prof[((size_t)c * gridDim.x + blockIdx.x) * 8 + 6] = n_layers;
 }
 
 // Parity instruments: trace / digest of Q(t+1) in external (AIGER) order.
@@ -253,26 +470,108 @@ __device__ void record_state(const KParams& kp, uint32_t c, uint32_t buf) {
 }
 
 __global__ void __launch_bounds__(GEM_THREADS, 2) gem_step_kernel(const KParams kp) {
-  extern __shared__ uint32_t smem[];
+  extern __shared__ __align__(16) uint32_t smem[];
+  // layout (words): S[state_words] | area[area_words] | ctab[256] | ramp[128] | topb[16] |
+  //                 res_p[16] | res_off[16] | res_n[16] | mbar[8 x u64]
+  // S must stay at offset 0 (leaf entries carry byte offsets into it).
   uint32_t* S = smem;
-  uint32_t* ramp = smem + kp.state_words;
+  uint32_t* area = S + kp.state_words;
+  uint32_t* ctab = area + kp.area_words;
+  uint32_t* ramp = ctab + GEM_MAX_CHUNKS;
   uint32_t* topb = ramp + 4 * GEM_MAX_RAMS_PER_PART;
+  uint32_t* res_p = topb + 16;
+  uint32_t* res_off = res_p + GEM_MAX_RESIDENT;
+  uint32_t* res_n = res_off + GEM_MAX_RESIDENT;      // [0] = n_res, [1] = resident flag
+  uint64_t* mbar = reinterpret_cast<uint64_t*>(res_n + 16);
+  const uint32_t tid = threadIdx.x;
+  const uint32_t G = gridDim.x, B = blockIdx.x;
+  auto wl_begin = [&](uint32_t s) { return __ldg(kp.wl_off + s * (G + 1) + B); };
+  auto wl_end = [&](uint32_t s) { return __ldg(kp.wl_off + s * (G + 1) + B + 1); };
+  if (tid == 0) {
+    for (uint32_t k = 0; k <= GEM_RING_MAX; k++) mbar_init(mbar + k, 1);
+    fence_mbar_init();
+    // residency: the distinct partitions of this CTA's work lists (fixed for the launch)
+    uint32_t n = 0, words = 0;
+    bool ok = kp.allow_resident != 0;
+    for (uint32_t s = 0; s < kp.n_stages && ok; s++) {
+      for (uint32_t k = wl_begin(s); k < wl_end(s); k++) {
+        const uint32_t p = __ldg(&kp.wl_items[k].x);
+        bool seen = false;
+        for (uint32_t j = 0; j < n; j++) seen |= res_p[j] == p;
+        if (seen) continue;
+        const uint32_t len = (__ldg(kp.parts + p * GP_WORDS + GP_PROG_LEN) + 3u) & ~3u;
+        if (n == GEM_MAX_RESIDENT || words + len > kp.area_words) { ok = false; break; }
+        res_p[n] = p;
+        res_off[n] = words;
+        words += len;
+        n++;
+      }
+    }
+    res_n[0] = n;
+    res_n[1] = ok ? 1u : 0u;
+    if (ok && words) {
+      mbar_expect_tx(mbar + GEM_RING_MAX, words * 4);
+      for (uint32_t k = 0; k < n; k++) {
+        const uint32_t p = res_p[k];
+        const uint32_t len = (__ldg(kp.parts + p * GP_WORDS + GP_PROG_LEN) + 3u) & ~3u;
+        tma_load_1d(area + res_off[k], kp.prog + __ldg(kp.parts + p * GP_WORDS + GP_PROG_OFF), len * 4,
+                    mbar + GEM_RING_MAX);
+      }
+    }
+  }
+  __syncthreads();
+  ProgSrc ps;
+  ps.mbar = mbar;
+  ps.area = area;
+  ps.ctab = ctab;
+  ps.resident = res_n[1] != 0;
+  ps.n_res = res_n[0];
+  ps.res_p = res_p;
+  ps.res_off = res_off;
+  ps.slot_words = kp.slot_words;
+  ps.R = kp.ring_slots;
+  ps.seq_issue = 0;
+  ps.seq_wait = 0;
+  ps.seq_free = 0;
+  if (ps.resident && ps.n_res) mbar_wait(mbar + GEM_RING_MAX, 0);
+  // first work item of this CTA in a cycle (index into wl_items), or ~0u
+  auto first_item = [&]() -> uint32_t {
+    for (uint32_t s = 0; s < kp.n_stages; s++)
+      if (wl_begin(s) < wl_end(s)) return wl_begin(s);
+    return ~0u;
+  };
+  if (!ps.resident && kp.ncycles) {
+    const uint32_t k0 = first_item();
+    if (k0 != ~0u) issue_prologue(kp, ps, __ldg(&kp.wl_items[k0].x));
+  }
+
   unsigned long long bar_target = 0;
   const bool instr = (kp.flags & (GEM_F_TRACE_STATE | GEM_F_DIGEST)) != 0;
   for (uint32_t c = 0; c < kp.ncycles; c++) {
     const uint64_t t = kp.t0 + c;
     const uint32_t cur = (uint32_t)(t & 1u), nxt = cur ^ 1u;
     if (instr && c > 0) record_state(kp, c - 1, cur);
+    const bool prof_on = kp.prof && c < kp.prof_cycles;
+    PROF(0);
     for (uint32_t s = 0; s < kp.n_stages; s++) {
-      const uint32_t pb = __ldg(kp.stage_list + s), pe = __ldg(kp.stage_list + s + 1);
-      const uint32_t np = pe - pb;
-      const uint32_t n_items = np * kp.n_streams;
-      for (uint32_t item = blockIdx.x; item < n_items; item += gridDim.x) {
-        const uint32_t p = __ldg(kp.stage_list + kp.n_stages + 1 + pb + item % np);
-        run_partition(kp, S, ramp, topb, p, item / np, c, cur, nxt);
+      const uint32_t kb = wl_begin(s), ke = wl_end(s);
+      for (uint32_t k = kb; k < ke; k++) {
+        const uint2 it = __ldg(&kp.wl_items[k]);
+        run_partition(kp, ps, S, ramp, topb, it.x, it.y, c, cur, nxt, prof_on && k == kb && s == 0);
+        if (!ps.resident) {
+          // prefetch the next work item's prologue (overlaps the grid barrier)
+          uint32_t nk = ~0u;
+          if (k + 1 < ke) nk = k + 1;
+          for (uint32_t s2 = s + 1; nk == ~0u && s2 < kp.n_stages; s2++)
+            if (wl_begin(s2) < wl_end(s2)) nk = wl_begin(s2);
+          if (nk == ~0u && c + 1 < kp.ncycles) nk = first_item();
+          if (nk != ~0u) issue_prologue(kp, ps, __ldg(&kp.wl_items[nk].x));
+        }
       }
+      if (s == 0) PROF(4);
       grid_sync(kp, bar_target);
     }
+    PROF(5);
   }
   if (instr) record_state(kp, kp.ncycles - 1, (uint32_t)((kp.t0 + kp.ncycles) & 1u));
 }
@@ -335,12 +634,16 @@ struct gem_sim {
   uint32_t po_words_ext = 0, q_words_ext = 0;
   uint64_t n_and = 0, n_and_mapped = 0, program_bytes = 0;
   uint32_t max_items = 0;
+  uint32_t area_words = 0, slot_words = 0, ring_slots = 0, resident = 0;
+  std::vector<uint32_t> h_parts, h_stage;
   // device buffers
   uint32_t *d_prog = nullptr, *d_parts = nullptr, *d_stage = nullptr;
   uint32_t *d_q_int_of_ext = nullptr, *d_q_ext_of_int = nullptr, *d_po_int_of_ext = nullptr;
   uint32_t *d_q = nullptr, *d_rd = nullptr, *d_cut = nullptr, *d_mem = nullptr;
-  uint32_t *d_pi = nullptr, *d_po = nullptr, *d_qtrace = nullptr, *d_scratch = nullptr;
-  unsigned long long *d_digest = nullptr, *d_bar = nullptr;
+  uint32_t *d_pi = nullptr, *d_po = nullptr, *d_qtrace = nullptr, *d_scratch = nullptr, *d_wl_off = nullptr;
+  uint2* d_wl_items = nullptr;
+  unsigned long long *d_digest = nullptr, *d_bar = nullptr, *d_prof = nullptr;
+  uint32_t prof_cycles = 0;
   int* d_err = nullptr;
   uint32_t in_cap = 0, in_queued = 0, in_head = 0, out_cap = 0, last_cycles = 0;
   size_t scratch_bytes = 0;
@@ -398,6 +701,135 @@ static int check(const gem_sim* sim) {
   if (!sim) return fail(GEM_E_INVAL, "null handle");
   if (sim->poisoned) return fail(GEM_E_CUDA, "handle poisoned by an earlier CUDA error");
   return 0;
+}
+
+// Longest-processing-time-first work lists: per stage, the (partition, stream)
+// items sorted by the mapper's cost estimate are assigned one by one to the
+// least-loaded CTA.  Returns the estimated makespan (sum over stages).
+static double build_worklists(const gem_sim* sim, uint32_t G, std::vector<uint32_t>& off,
+                              std::vector<uint2>& items) {
+  off.assign((size_t)sim->n_stages * (G + 1), 0);
+  items.clear();
+  double makespan = 0;
+  for (uint32_t s = 0; s < sim->n_stages; s++) {
+    const uint32_t pb = sim->h_stage[s], np = sim->h_stage[s + 1] - pb;
+    std::vector<std::pair<uint32_t, uint2>> its;
+    its.reserve((size_t)np * sim->n_streams);
+    for (uint32_t st = 0; st < sim->n_streams; st++)
+      for (uint32_t k = 0; k < np; k++) {
+        const uint32_t p = sim->h_stage[sim->n_stages + 1 + pb + k];
+        its.push_back({sim->h_parts[(size_t)p * GP_WORDS + GP_COST], make_uint2(p, st)});
+      }
+    std::stable_sort(its.begin(), its.end(), [](const std::pair<uint32_t, uint2>& x,
+                                                const std::pair<uint32_t, uint2>& y) { return x.first > y.first; });
+    std::vector<std::vector<uint2>> lists(G);
+    // min-heap of (load, cta)
+    std::vector<std::pair<double, uint32_t>> heap;
+    for (uint32_t b = 0; b < G; b++) heap.push_back({0.0, b});
+    auto cmp = [](const std::pair<double, uint32_t>& x, const std::pair<double, uint32_t>& y) {
+      return x.first > y.first || (x.first == y.first && x.second > y.second);
+    };
+    std::make_heap(heap.begin(), heap.end(), cmp);
+    double mx = 0;
+    for (auto& it : its) {
+      std::pop_heap(heap.begin(), heap.end(), cmp);
+      auto& h = heap.back();
+      lists[h.second].push_back(it.second);
+      h.first += std::max<uint32_t>(it.first, 1);
+      mx = std::max(mx, h.first);
+      std::push_heap(heap.begin(), heap.end(), cmp);
+    }
+    makespan += mx;
+    uint32_t* o = &off[(size_t)s * (G + 1)];
+    for (uint32_t b = 0; b < G; b++) {
+      o[b] = (uint32_t)items.size();
+      items.insert(items.end(), lists[b].begin(), lists[b].end());
+    }
+    o[G] = (uint32_t)items.size();
+  }
+  return makespan;
+}
+
+// Choose CTAs per SM, grid, work lists and the shared-memory program mode.
+// Resident mode (every program a CTA runs copied into its shared memory once
+// per launch) is used when it fits; otherwise programs stream through a TMA
+// ring of >= 2 slots.  Single-stream (latency) runs prefer one CTA per SM so
+// the critical partitions do not share an SM; GEM_BPS=n overrides.
+static int plan_launch(gem_sim* sim, uint32_t max_chunk_words, uint32_t grid_limit) {
+  int sms = 0, coop = 0, optin = 0, per_sm = 0;
+  CK(cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, sim->device));
+  CK(cudaDeviceGetAttribute(&coop, cudaDevAttrCooperativeLaunch, sim->device));
+  CK(cudaDeviceGetAttribute(&optin, cudaDevAttrMaxSharedMemoryPerBlockOptin, sim->device));
+  CK(cudaDeviceGetAttribute(&per_sm, cudaDevAttrMaxSharedMemoryPerMultiprocessor, sim->device));
+  if (!coop) return fail(GEM_E_UNSUPPORTED, "device lacks cooperative launch");
+  sim->sm_count = (uint32_t)sms;
+  const uint32_t fixed_words = sim->state_words + GEM_MAX_CHUNKS + 4 * GEM_MAX_RAMS_PER_PART + 16 + 48 + 16;
+  const uint32_t slot = (max_chunk_words + 3u) & ~3u;
+  const char* env = getenv("GEM_NO_RESIDENT");
+  const bool allow_res = !(env && env[0] == '1');
+  const char* benv = getenv("GEM_BPS");
+  const uint32_t force_bps = benv ? (uint32_t)atoi(benv) : 0;
+  struct Choice { uint32_t bps = 0, grid = 0, area = 0, resident = 0, ring = 0; double score = 0; };
+  Choice best;
+  std::vector<uint32_t> best_off, off;
+  std::vector<uint2> best_items, items;
+  double max_cost = 0;
+  for (uint32_t p = 0; p < sim->n_parts; p++)
+    max_cost = std::max<double>(max_cost, sim->h_parts[(size_t)p * GP_WORDS + GP_COST]);
+  for (uint32_t bps = 1; bps <= 4; bps++) {
+    if (force_bps && bps != force_bps) continue;
+    const int64_t budget = std::min<int64_t>(optin, per_sm / (int64_t)bps - 1024);
+    if (budget < (int64_t)(fixed_words * 4 + 2 * slot * 4)) continue;
+    const uint32_t area = (uint32_t)(budget / 4) - fixed_words;
+    uint32_t grid = std::max<uint32_t>(1, std::min<uint32_t>(sim->max_items, bps * (uint32_t)sms));
+    if (grid_limit) grid = std::max<uint32_t>(1, std::min(grid, grid_limit));
+    int occ = 0;
+    CK(cudaFuncSetAttribute(gem_step_kernel, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)budget));
+    CK(cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ, gem_step_kernel, GEM_THREADS, (size_t)budget));
+    if ((uint32_t)occ < bps) continue;
+    const double makespan = build_worklists(sim, grid, off, items);
+    // residency check for every CTA
+    bool res = allow_res;
+    for (uint32_t b = 0; b < grid && res; b++) {
+      std::vector<uint32_t> seen;
+      uint64_t words = 0;
+      for (uint32_t s = 0; s < sim->n_stages && res; s++)
+        for (uint32_t k = off[(size_t)s * (grid + 1) + b]; k < off[(size_t)s * (grid + 1) + b + 1]; k++) {
+          const uint32_t p = items[k].x;
+          if (std::find(seen.begin(), seen.end(), p) != seen.end()) continue;
+          seen.push_back(p);
+          words += (sim->h_parts[(size_t)p * GP_WORDS + GP_PROG_LEN] + 3u) & ~3u;
+          if (seen.size() > GEM_MAX_RESIDENT || words > area) { res = false; break; }
+        }
+    }
+    const uint32_t ring = std::min<uint32_t>(GEM_RING_MAX, area / std::max<uint32_t>(slot, 4));
+    if (!res && ring < 2) continue;
+    // score: estimated makespan, SM sharing slows co-resident CTAs, streaming costs a little
+    double score = makespan * (1.0 + 0.5 * (bps - 1) * std::min(1.0, (double)grid / ((double)bps * sms)))
+                   * (res ? 1.0 : 1.1);
+    if (!best.bps || score < best.score) {
+      best.bps = bps; best.grid = grid; best.area = area; best.resident = res ? 1u : 0u; best.ring = ring;
+      best.score = score;
+      best_off.swap(off);
+      best_items.swap(items);
+    }
+  }
+  (void)max_cost;
+  if (!best.bps) return fail(GEM_E_UNSUPPORTED, "cannot fit the program ring / state in shared memory");
+  sim->blocks_per_sm = best.bps;
+  sim->grid = best.grid;
+  sim->area_words = best.area;
+  sim->resident = best.resident;
+  sim->ring_slots = best.ring;
+  sim->slot_words = slot;
+  sim->smem_bytes = (fixed_words + best.area) * 4;
+  CK(cudaFuncSetAttribute(gem_step_kernel, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)sim->smem_bytes));
+  CK(dalloc(&sim->d_wl_off, best_off.size() * 4));
+  CK(cudaMemcpy(sim->d_wl_off, best_off.data(), best_off.size() * 4, cudaMemcpyHostToDevice));
+  CK(dalloc(&sim->d_wl_items, std::max<size_t>(best_items.size(), 1) * 8));
+  if (!best_items.empty())
+    CK(cudaMemcpy(sim->d_wl_items, best_items.data(), best_items.size() * 8, cudaMemcpyHostToDevice));
+  return GEM_OK;
 }
 
 extern "C" {
@@ -498,20 +930,10 @@ int gem_load_program(const void* blob, size_t nbytes, const gem_config* cfg, gem
     CK(cudaMemset(sim->d_cut, 0, S * std::max<uint32_t>(sim->cut_words, 1) * 4));
     if (sim->n_rams) CK(cudaMemset(sim->d_mem, 0, S * sim->n_rams * (size_t)GEM_RAM_WORDS * 4));
   }
-  // persistent co-resident grid
-  sim->smem_bytes = (sim->state_words + 4 * GEM_MAX_RAMS_PER_PART + GEM_WARPS) * 4;
-  if (sim->smem_bytes > 48 * 1024)
-    CK(cudaFuncSetAttribute(gem_step_kernel, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)sim->smem_bytes));
-  int bps = 0, sms = 0, coop = 0;
-  CK(cudaOccupancyMaxActiveBlocksPerMultiprocessor(&bps, gem_step_kernel, GEM_THREADS, sim->smem_bytes));
-  CK(cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, sim->device));
-  CK(cudaDeviceGetAttribute(&coop, cudaDevAttrCooperativeLaunch, sim->device));
-  if (bps < 1 || !coop) { gem_free(sim); return fail(GEM_E_UNSUPPORTED, "kernel cannot be made co-resident"); }
-  sim->blocks_per_sm = (uint32_t)bps;
-  sim->sm_count = (uint32_t)sms;
-  uint32_t cap = (uint32_t)bps * (uint32_t)sms;
-  sim->grid = std::max<uint32_t>(1, std::min(cap, sim->max_items));
-  if (cfg->grid_limit) sim->grid = std::max<uint32_t>(1, std::min(sim->grid, cfg->grid_limit));
+  // persistent co-resident grid + shared-memory program placement
+  sim->h_parts.assign(parts, parts + (size_t)sim->n_parts * GP_WORDS);
+  sim->h_stage.assign(stages, stages + stage_words);
+  if (int r = plan_launch(sim, w[GH_MAX_CHUNK_WORDS], cfg->grid_limit)) { gem_free(sim); return r; }
   CK(cudaDeviceSynchronize());
   *out = sim;
   return GEM_OK;
@@ -524,6 +946,7 @@ int gem_info_get(const gem_sim* sim, gem_info* out) {
   out->total_layers = sim->total_layers;
   out->pi_words = sim->pi_words; out->po_words = sim->po_words_ext; out->q_words = sim->q_words_ext;
   out->grid = sim->grid; out->blocks_per_sm = sim->blocks_per_sm; out->smem_bytes = sim->smem_bytes;
+  out->resident = sim->resident; out->ring_slots = sim->ring_slots;
   out->n_streams = sim->n_streams;
   out->n_and = sim->n_and; out->n_and_mapped = sim->n_and_mapped; out->program_bytes = sim->program_bytes;
   out->cycle = sim->cycle;
@@ -572,6 +995,22 @@ int gem_step(gem_sim* sim, uint64_t ncycles) {
   kp.q_words = sim->q_words_int; kp.cut_words = sim->cut_words; kp.n_rams = sim->n_rams;
   kp.n_flops = sim->n_flops; kp.q_ext_words = sim->q_words_ext;
   kp.flags = sim->flags & (GEM_F_TRACE_STATE | GEM_F_DIGEST);
+  kp.area_words = sim->area_words; kp.slot_words = sim->slot_words; kp.ring_slots = sim->ring_slots;
+  kp.allow_resident = sim->resident;
+  kp.wl_off = sim->d_wl_off;
+  kp.wl_items = sim->d_wl_items;
+  if (sim->flags & GEM_F_PROFILE) {
+    const uint32_t pc = (uint32_t)std::min<uint64_t>(ncycles, 256);
+    if (!sim->d_prof || sim->prof_cycles < pc) {
+      if (sim->d_prof) cudaFree(sim->d_prof);
+      sim->d_prof = nullptr;
+      CK(dalloc(&sim->d_prof, (size_t)256 * sim->grid * 8 * 8));
+    }
+    sim->prof_cycles = pc;
+    CK(cudaMemsetAsync(sim->d_prof, 0, (size_t)256 * sim->grid * 8 * 8, sim->stream));
+    kp.prof = sim->d_prof;
+    kp.prof_cycles = pc;
+  }
   CK(cudaMemsetAsync(sim->d_bar, 0, 8, sim->stream));
   if (sim->flags & GEM_F_DIGEST)
     CK(cudaMemsetAsync(sim->d_digest, 0, (size_t)sim->n_streams * sim->out_cap * 8, sim->stream));
@@ -706,6 +1145,17 @@ int gem_write_ram(gem_sim* sim, uint32_t ram_id, uint32_t stream, const uint32_t
   return GEM_OK;
 }
 
+int gem_read_profile(gem_sim* sim, uint64_t* dst, uint32_t* n_cycles, uint32_t* grid) {
+  if (int r = check(sim)) return r;
+  if (!(sim->flags & GEM_F_PROFILE) || !sim->d_prof) return fail(GEM_E_INVAL, "GEM_F_PROFILE not set / no step yet");
+  CK(cudaSetDevice(sim->device));
+  CK(cudaStreamSynchronize(sim->stream));
+  if (n_cycles) *n_cycles = sim->prof_cycles;
+  if (grid) *grid = sim->grid;
+  if (dst) CK(cudaMemcpy(dst, sim->d_prof, (size_t)sim->prof_cycles * sim->grid * 8 * 8, cudaMemcpyDeviceToHost));
+  return GEM_OK;
+}
+
 void gem_free(gem_sim* sim) {
   if (!sim) return;
   cudaSetDevice(sim->device);
@@ -713,7 +1163,8 @@ void gem_free(gem_sim* sim) {
   for (void* p : {(void*)sim->d_prog, (void*)sim->d_parts, (void*)sim->d_stage, (void*)sim->d_q_int_of_ext,
                   (void*)sim->d_q_ext_of_int, (void*)sim->d_po_int_of_ext, (void*)sim->d_q, (void*)sim->d_rd,
                   (void*)sim->d_cut, (void*)sim->d_mem, (void*)sim->d_pi, (void*)sim->d_po, (void*)sim->d_qtrace,
-                  (void*)sim->d_scratch, (void*)sim->d_digest, (void*)sim->d_bar, (void*)sim->d_err})
+                  (void*)sim->d_scratch, (void*)sim->d_digest, (void*)sim->d_bar, (void*)sim->d_err,
+                  (void*)sim->d_prof, (void*)sim->d_wl_off, (void*)sim->d_wl_items})
     if (p) cudaFree(p);
   if (sim->ev0) cudaEventDestroy(sim->ev0);
   if (sim->ev1) cudaEventDestroy(sim->ev1);

@@ -18,11 +18,12 @@ from . import _build
 GEM_F_TRACE_STATE = 0x1
 GEM_F_DIGEST = 0x2
 GEM_F_ASYNC = 0x4
+GEM_F_PROFILE = 0x8
 ERRORS = {-1: "GEM_E_INVAL", -2: "GEM_E_FORMAT", -3: "GEM_E_CUDA", -4: "GEM_E_NOMEM", -5: "GEM_E_NOINPUT",
           -6: "GEM_E_UNSUPPORTED"}
 EXPORTS = ["gem_load_program", "gem_info_get", "gem_set_inputs", "gem_step", "gem_read_outputs",
            "gem_read_state", "gem_write_state", "gem_read_state_trace", "gem_read_digests", "gem_read_ram",
-           "gem_write_ram", "gem_last_step_ms", "gem_free", "gem_last_error"]
+           "gem_write_ram", "gem_last_step_ms", "gem_read_profile", "gem_free", "gem_last_error"]
 
 
 class GemConfig(ctypes.Structure):
@@ -33,7 +34,8 @@ class GemConfig(ctypes.Structure):
 class GemInfo(ctypes.Structure):
     _fields_ = [(n, ctypes.c_uint32) for n in
                 ("n_pi", "n_po", "n_flops", "n_rams", "n_parts", "n_stages", "max_layers", "total_layers",
-                 "pi_words", "po_words", "q_words", "grid", "blocks_per_sm", "smem_bytes", "n_streams")] + \
+                 "pi_words", "po_words", "q_words", "grid", "blocks_per_sm", "smem_bytes", "n_streams",
+                 "resident", "ring_slots")] + \
                [(n, ctypes.c_uint64) for n in ("n_and", "n_and_mapped", "program_bytes", "cycle")]
 
     def as_dict(self):
@@ -76,6 +78,7 @@ def load_library(build: bool = True):
             lib.gem_read_ram.argtypes = [P, u32, u32, P]
             lib.gem_write_ram.argtypes = [P, u32, u32, P]
             lib.gem_last_step_ms.argtypes = [P, ctypes.POINTER(ctypes.c_float)]
+            lib.gem_read_profile.argtypes = [P, P, ctypes.POINTER(u32), ctypes.POINTER(u32)]
             lib.gem_free.argtypes = [P]
             lib.gem_free.restype = None
             lib.gem_last_error.restype = ctypes.c_char_p
@@ -183,6 +186,14 @@ class Simulator:
         w = np.ascontiguousarray(words, dtype=np.uint32)
         assert w.shape == (8192,)
         self._check(self.lib.gem_write_ram(self._h, ram, stream, _p(w)))
+
+    def read_profile(self) -> np.ndarray:
+        """uint64 [cycles][grid][8] clock64 phase stamps (GEM_F_PROFILE)."""
+        n, g = ctypes.c_uint32(), ctypes.c_uint32()
+        self._check(self.lib.gem_read_profile(self._h, None, ctypes.byref(n), ctypes.byref(g)))
+        out = np.zeros((n.value, g.value, 8), np.uint64)
+        self._check(self.lib.gem_read_profile(self._h, _p(out), ctypes.byref(n), ctypes.byref(g)))
+        return out
 
     def run(self, pi: np.ndarray) -> np.ndarray:
         """Convenience: set_inputs + step + read_outputs."""

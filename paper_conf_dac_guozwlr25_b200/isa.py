@@ -10,7 +10,9 @@ GH = ["MAGIC", "VERSION", "N_PI", "N_PO", "N_FLOPS", "N_RAMS", "N_PARTS", "N_STA
       "N_AND_LO", "N_AND_HI", "N_AND_MAPPED_LO", "N_AND_MAPPED_HI", "TOTAL_LAYERS",
       "TOTAL_LEAVES_LO", "TOTAL_LEAVES_HI", "OFF_PARTS", "OFF_STAGES", "OFF_FLOP_INIT",
       "OFF_PROG", "PROG_WORDS_LO", "PROG_WORDS_HI", "MAX_LEVELS", "TOTAL_WRITEOUTS",
-      "MAX_OUT", "TOTAL_WORDS_LO", "TOTAL_WORDS_HI", "SLOTS_USED_LO", "SLOTS_USED_HI"]
+      "MAX_OUT", "TOTAL_WORDS_LO", "TOTAL_WORDS_HI", "SLOTS_USED_LO", "SLOTS_USED_HI",
+      "MAX_CHUNK_WORDS", "MAX_PROG_WORDS"]
+GP_WORDS = 12
 GEM_MAGIC = 0x424D4547
 SLOTS_PER_LAYER = 8191
 
@@ -37,6 +39,9 @@ class BlobInfo:
     blob_bytes: int
     slots_used: int
     part_layers: list
+    max_chunk_words: int = 0
+    max_prog_words: int = 0
+    part_cost: list = None
 
     @property
     def replication(self) -> float:
@@ -53,6 +58,7 @@ class BlobInfo:
     def as_dict(self) -> dict:
         d = dataclasses.asdict(self)
         d.pop("part_layers")
+        d.pop("part_cost", None)
         d.update(replication=self.replication, slot_util=self.slot_util, bytes_per_and=self.bytes_per_and,
                  levels_per_layer=self.max_levels / max(1, self.max_layers))
         return d
@@ -65,11 +71,13 @@ def blob_info(blob: bytes) -> BlobInfo:
         raise ValueError("not a .gemb blob")
     u64 = lambda k: h[k + "_LO"] | (h[k + "_HI"] << 32)
     np_ = h["N_PARTS"]
-    pt = w[h["OFF_PARTS"]:h["OFF_PARTS"] + 4 * np_].reshape(np_, 4)
+    pt = w[h["OFF_PARTS"]:h["OFF_PARTS"] + GP_WORDS * np_].reshape(np_, GP_WORDS)
     return BlobInfo(n_pi=h["N_PI"], n_po=h["N_PO"], n_flops=h["N_FLOPS"], n_rams=h["N_RAMS"],
                     n_parts=np_, n_stages=h["N_STAGES"], max_state_words=h["MAX_STATE_WORDS"],
                     max_layers=h["MAX_LAYERS"], total_layers=h["TOTAL_LAYERS"], q_words=h["Q_WORDS"],
                     po_words=h["PO_WORDS"], cut_words=h["CUT_WORDS"], n_and=u64("N_AND"),
                     n_and_mapped=u64("N_AND_MAPPED"), total_leaves=u64("TOTAL_LEAVES"),
                     max_levels=h["MAX_LEVELS"], program_bytes=4 * u64("PROG_WORDS"),
-                    blob_bytes=len(blob), slots_used=u64("SLOTS_USED"), part_layers=pt[:, 3].tolist())
+                    blob_bytes=len(blob), slots_used=u64("SLOTS_USED"), part_layers=pt[:, 3].tolist(),
+                    max_chunk_words=h["MAX_CHUNK_WORDS"], max_prog_words=h["MAX_PROG_WORDS"],
+                    part_cost=pt[:, 8].tolist())

@@ -737,10 +737,23 @@ struct Mapper {
     pr[PH_N_LAYERS] = n_layers;
     pr[PH_N_OUT] = (uint32_t)P.outs.size();
     pr[PH_N_RAM] = (uint32_t)P.rams.size();
+    // chunk table: [chunk0 | layers... | out+ram]
+    pr[PH_OFF_CHUNKS] = (uint32_t)pr.size();
+    pr[PH_N_CHUNKS] = n_layers + 2;
+    for (uint32_t k = 0; k < n_layers + 2; k++) pr.push_back(0);
+    while (pr.size() % 4) pr.push_back(0);
     pr[PH_OFF_GREAD] = (uint32_t)pr.size();
     for (uint32_t k = 0; k < n_gread; k++) { pr.push_back(gread_src[k]); pr.push_back(k + 1); }
     while (pr.size() % 4) pr.push_back(0);
     pr[PH_OFF_LAYERS] = (uint32_t)pr.size();
+    pr[pr[PH_OFF_CHUNKS]] = (uint32_t)pr.size();
+    {
+      size_t off = 0;
+      for (uint32_t l = 0; l < n_layers; l++) {
+        pr[pr[PH_OFF_CHUNKS] + 1 + l] = prog_layers[off + LH_WORDS_];
+        off += prog_layers[off + LH_WORDS_];
+      }
+    }
     pr.insert(pr.end(), prog_layers.begin(), prog_layers.end());
     pr[PH_OFF_OUT] = (uint32_t)pr.size();
     uint32_t n_out = (uint32_t)P.outs.size(), n_out_pad = (n_out + 3) & ~3u;
@@ -754,6 +767,8 @@ struct Mapper {
       }
     pr[PH_OFF_RAM] = (uint32_t)pr.size();
     for (uint32_t r : P.rams) { pr.push_back(r); pr.push_back(0); pr.push_back(0); pr.push_back(0); }
+    while (pr.size() % 4) pr.push_back(0);
+    pr[pr[PH_OFF_CHUNKS] + 1 + n_layers] = (uint32_t)pr.size() - pr[PH_OFF_OUT];
     pr[PH_STATE_WORDS] = max_state;
     pr[PH_N_LEAVES] = total_leaves;
     pr[PH_N_NODES] = n_and;
@@ -771,16 +786,21 @@ struct Mapper {
     for (uint32_t c : cid) (void)c;
   }
 
+  // Layer record encoding (gem_isa.h).  A warp whose fullest lane has more than
+  // kDenseMin leaves uses the DENSE gather (32 entries per lane, entry index =
+  // leaf position, 4 instructions per entry); otherwise SPARSE (explicit
+  // positions, fewer entries).
+  static constexpr uint32_t kDenseMin = 18;
   static void encode_layer(std::vector<uint32_t>& out, std::vector<int32_t>* slot, std::vector<uint8_t>* sxa,
                            std::vector<uint8_t>* sxb, std::vector<uint8_t>* sob,
                            const std::vector<int32_t>& wo_thread, const std::vector<int32_t>& wo_warp,
                            int32_t wo_top) {
     size_t base = out.size();
     out.resize(base + LH_WORDS, 0);
-    // leaves per thread
-    std::vector<std::vector<uint32_t>> leaves(256);
+    // leaves per thread: (state bit, position)
+    std::vector<std::vector<std::pair<uint32_t, uint32_t>>> leaves(256);
     for (uint32_t id = 0; id < 8192; id++)
-      if (slot[0][id] >= 0) leaves[id >> 5].push_back(GEM_LEAF((uint32_t)slot[0][id], id & 31));
+      if (slot[0][id] >= 0) leaves[id >> 5].push_back({(uint32_t)slot[0][id], id & 31});
     uint32_t active = 0;
     uint32_t niter[8] = {0};
     for (uint32_t w = 0; w < 8; w++) {
@@ -804,13 +824,17 @@ struct Mapper {
     out[base + LH_FLAGS] = active | (uses_top ? GEM_LF_USES_TOP : 0u);
     out[base + LH_TOPC] = pack(11, 13, 0, sxa) | (pack(11, 13, 0, sxb) << 8) | (pack(11, 13, 0, sob) << 16);
     out[base + LH_TOPWO] = uses_top ? (uint32_t)wo_top : 0u;
-    for (uint32_t w = 0; w < 8; w++) out[base + LH_NITER0 + w] = (active >> w & 1) ? niter[w] : 0;
     for (uint32_t w = 0; w < 8; w++) {
       if (!(active >> w & 1)) continue;
+      out[base + LH_WOFF0 + w] = (uint32_t)(out.size() - base);
+      const bool dense = niter[w] > kDenseMin;
+      const uint32_t n4 = dense ? 8u : (niter[w] + 3) / 4;
       out.push_back(pack(6, 10, w, sxa));
       out.push_back(pack(6, 10, w, sxb));
       out.push_back(pack(6, 10, w, sob));
       out.push_back(wo_warp[w] >= 0 ? (uint32_t)wo_warp[w] : 0u);
+      out.push_back((dense ? GEM_WM_DENSE : GEM_WM_SPARSE) | (n4 << 8));
+      out.push_back(0); out.push_back(0); out.push_back(0);
       for (uint32_t l = 0; l < 32; l++) {
         uint32_t t = w * 32 + l;
         out.push_back(pack(1, 5, t, sxa));
@@ -818,15 +842,40 @@ struct Mapper {
         out.push_back(pack(1, 5, t, sob));
         out.push_back(wo_thread[t] >= 0 ? (uint32_t)wo_thread[t] : 0u);
       }
-      for (uint32_t i = 0; i < niter[w]; i++)
+      for (uint32_t g = 0; g < n4; g++)
         for (uint32_t l = 0; l < 32; l++) {
           auto& lv = leaves[w * 32 + l];
-          out.push_back(i < lv.size() ? lv[i] : GEM_LEAF(0, 0));
+          for (uint32_t c = 0; c < 4; c++) {
+            uint32_t j = 4 * g + c, e = 0;
+            if (dense) {
+              for (auto& x : lv)
+                if (x.second == j) e = GEM_LEAF_DENSE(x.first >> 5, x.first & 31, j);
+            } else if (j < lv.size()) {
+              e = GEM_LEAF(lv[j].first >> 5, lv[j].first & 31, lv[j].second);
+            }
+            out.push_back(e);
+          }
         }
     }
     out[base + LH_WORDS_] = (uint32_t)(out.size() - base);
   }
 };
+
+// Estimated SM clocks for one cycle of a partition program (cost model fitted to
+// B200 phase measurements: fixed per-layer latency + per-16-byte leaf group).
+static uint32_t part_cost(const uint32_t* pr) {
+  const double kItem = 3000.0, kLayer = 900.0, kGroup = 14.0, kGread = 1.5, kOut = 20.0;
+  double c = kItem + kGread * pr[PH_N_GREAD] + kOut * pr[PH_N_OUT];
+  const uint32_t* L = pr + pr[PH_OFF_LAYERS];
+  for (uint32_t l = 0; l < pr[PH_N_LAYERS]; l++) {
+    uint32_t groups = 0;
+    for (uint32_t w = 0; w < 8; w++)
+      if (L[LH_WOFF0 + w]) groups += L[L[LH_WOFF0 + w] + 4] >> 8;
+    c += kLayer + kGroup * groups;
+    L += L[LH_WORDS_];
+  }
+  return (uint32_t)std::min(c, 4.0e9);
+}
 
 // =========================================================== partitioning
 struct Design {
@@ -1236,16 +1285,31 @@ static Blob compile(const char* data, size_t n, const char* opts) {
   while (w.size() % 4) w.push_back(0);
   w[GH_OFF_PROG] = (uint32_t)w.size();
   uint64_t prog = 0;
+  uint32_t max_chunk = 0, max_prog = 0;
   for (uint32_t i = 0; i < np; i++) {
     auto& P = D.parts[i];
     w[part_tab + i * GP_WORDS + GP_STAGE] = (uint32_t)P.stage;
     w[part_tab + i * GP_WORDS + GP_PROG_OFF] = (uint32_t)prog;
     w[part_tab + i * GP_WORDS + GP_PROG_LEN] = (uint32_t)P.prog.size();
     w[part_tab + i * GP_WORDS + GP_N_LAYERS] = P.n_layers;
+    {
+      const uint32_t* pr = P.prog.data();
+      uint32_t mc = 0;
+      for (uint32_t k = 0; k < pr[PH_N_CHUNKS]; k++) mc = std::max(mc, pr[pr[PH_OFF_CHUNKS] + k]);
+      w[part_tab + i * GP_WORDS + GP_CHUNK0] = pr[pr[PH_OFF_CHUNKS]];
+      w[part_tab + i * GP_WORDS + GP_CHUNK1] = pr[PH_N_CHUNKS] > 1 ? pr[pr[PH_OFF_CHUNKS] + 1] : 0;
+      w[part_tab + i * GP_WORDS + GP_CHUNK2] = pr[PH_N_CHUNKS] > 2 ? pr[pr[PH_OFF_CHUNKS] + 2] : 0;
+      w[part_tab + i * GP_WORDS + GP_MAX_CHUNK] = mc;
+      w[part_tab + i * GP_WORDS + GP_COST] = part_cost(pr);
+      max_chunk = std::max(max_chunk, mc);
+      max_prog = std::max<uint32_t>(max_prog, (uint32_t)P.prog.size());
+    }
     w.insert(w.end(), P.prog.begin(), P.prog.end());
     prog += P.prog.size();
     while (prog % 4) { w.push_back(0); prog++; }
   }
+  w[GH_MAX_CHUNK_WORDS] = max_chunk;
+  w[GH_MAX_PROG_WORDS] = max_prog;
   w[GH_PROG_WORDS_LO] = (uint32_t)prog;
   w[GH_PROG_WORDS_HI] = (uint32_t)(prog >> 32);
   w[GH_TOTAL_WORDS_LO] = (uint32_t)w.size();

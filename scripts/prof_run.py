@@ -15,6 +15,7 @@ ap.add_argument("--cfg", default="c3")
 ap.add_argument("--cycles", type=int, default=50)
 ap.add_argument("--streams", type=int, default=1)
 ap.add_argument("--launches", type=int, default=2)
+ap.add_argument("--phases", action="store_true")
 a = ap.parse_args()
 b = blob(a.cfg)
 sim = gem.Simulator(b, n_streams=a.streams)
@@ -27,3 +28,23 @@ for k in range(a.launches):
     print(f"launch {k}: {sim.last_step_ms():.3f} ms for {a.cycles} cycles "
           f"-> {a.cycles * a.streams / sim.last_step_ms() * 1e3:.0f} stream-cycles/s", flush=True)
 print(sim.info)
+
+if a.phases:
+    psim = gem.Simulator(b, n_streams=a.streams, flags=gem.GEM_F_PROFILE)
+    psim.set_inputs(st[:, :200])
+    psim.step(200)
+    pr = psim.read_profile().astype(np.int64)[20:]     # skip warm-up cycles
+    d = lambda a_, b_: (pr[:, :, b_] - pr[:, :, a_])
+    gread, layers, out = d(0, 1), d(1, 2), d(2, 3)
+    items, bar = d(0, 4), d(4, 5)
+    tot = d(0, 5)
+    nl = pr[:, :, 6]
+    crit = np.argmax(items.mean(0))
+    print(f"phases (SM clocks, mean over cycles): cycle total {tot.mean():.0f}")
+    print(f"  critical CTA {crit}: layers={nl[0, crit]} gread={gread[:, crit].mean():.0f} "
+          f"layers={layers[:, crit].mean():.0f} ({layers[:, crit].mean() / max(1, nl[0, crit]):.0f}/layer) "
+          f"out+ram={out[:, crit].mean():.0f} items={items[:, crit].mean():.0f} barrier={bar[:, crit].mean():.0f}")
+    per_layer = layers.mean(0) / np.maximum(1, nl[0])
+    print(f"  all CTAs: items mean {items.mean():.0f} max {items.mean(0).max():.0f}; per-layer clocks "
+          f"mean {per_layer.mean():.0f} min {per_layer.min():.0f} max {per_layer.max():.0f}; "
+          f"gread mean {gread.mean():.0f}; out mean {out.mean():.0f}; barrier min {bar.mean(0).min():.0f}")

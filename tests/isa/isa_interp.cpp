@@ -71,25 +71,27 @@ int run_part(Interp& I, uint32_t p, uint64_t t, const uint32_t* stim, uint32_t* 
     std::memset(warp_c, 0, sizeof(warp_c));
     for (int k = 0; k <= 13; k++) std::fill(val[k].begin(), val[k].end(), 0);
     std::vector<uint8_t> read(GEM_MAX_STATE_WORDS, 0);
-    const uint32_t* rec = L + LH_WORDS;
     for (uint32_t wp = 0; wp < 8; wp++) {
       if (!((flags >> wp) & 1)) continue;
-      uint32_t niter = L[LH_NITER0 + wp];
+      const uint32_t* rec = L + L[LH_WOFF0 + wp];
+      uint32_t mode = rec[4] & 0xFF, n4 = rec[4] >> 8;
       for (int c = 0; c < 4; c++) warp_c[wp][c] = rec[c];
       for (uint32_t ln = 0; ln < 32; ln++)
-        for (int c = 0; c < 4; c++) lane_c[wp * 32 + ln][c] = rec[4 + ln * 4 + c];
-      const uint32_t* lv = rec + 4 + 128;
-      for (uint32_t i = 0; i < niter; i++)
-        for (uint32_t ln = 0; ln < 32; ln++) {
-          uint32_t e = lv[i * 32 + ln];
-          uint32_t src = e & 0xFFFF, pos = (e >> 16) & 31;
-          read[src >> 5] = 1;
-          uint32_t bit = (S[src >> 5] >> (src & 31)) & 1u;
-          val[0][(wp * 32 + ln) * 32 + pos] |= (uint8_t)bit;
-        }
-      rec += GEM_WARP_REC_WORDS(niter);
+        for (int c = 0; c < 4; c++) lane_c[wp * 32 + ln][c] = rec[GEM_WREC_HDR + ln * 4 + c];
+      const uint32_t* lv = rec + GEM_WREC_HDR + 128;
+      for (uint32_t g = 0; g < n4; g++)
+        for (uint32_t ln = 0; ln < 32; ln++)
+          for (uint32_t c = 0; c < 4; c++) {
+            uint32_t e = lv[(g * 32 + ln) * 4 + c];
+            uint32_t word = GEM_LEAF_WORD(e), rot = GEM_LEAF_ROT(e);
+            uint32_t pos = mode == GEM_WM_DENSE ? 4 * g + c : GEM_LEAF_POS(e);
+            if (word >= GEM_MAX_STATE_WORDS) { g_err = "leaf word out of range"; return -1; }
+            read[word] = 1;
+            uint32_t s = S[word];
+            uint32_t rs = rot ? ((s << rot) | (s >> (32 - rot))) : s;   // rotl: bit b -> (b+rot)%32
+            val[0][(wp * 32 + ln) * 32 + pos] |= (uint8_t)((rs >> pos) & 1u);
+          }
     }
-    if ((uint32_t)(rec - L) != L[LH_WORDS_]) { g_err = "layer size mismatch"; return -1; }
     for (int k = 1; k <= 13; k++) {
       uint32_t g = gw(k);
       for (uint32_t id = 0; id < (8192u >> k); id++) {
@@ -133,7 +135,7 @@ int run_part(Interp& I, uint32_t p, uint64_t t, const uint32_t* stim, uint32_t* 
     uint32_t v = 0;
     for (int b = 0; b < 32; b++) {
       uint32_t e = os[j * 32 + b];
-      uint32_t src = e & 0xFFFF;
+      uint32_t src = e & 0x7FFFFFFFu;
       v |= (((S[src >> 5] >> (src & 31)) & 1u) ^ (e >> 31)) << b;
     }
     uint32_t reg = GEM_GID_REGION(od[j]), idx = GEM_GID_INDEX(od[j]);
