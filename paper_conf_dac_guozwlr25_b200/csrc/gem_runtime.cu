@@ -56,6 +56,7 @@ struct KParams {
   uint32_t area_words, slot_words, ring_slots, allow_resident;
   unsigned long long* prof;   // GEM_F_PROFILE: [prof_cycles][grid][8] clock64 stamps
   uint32_t prof_cycles;
+  uint32_t group;                        // streams per work item (stream states in smem)
   const uint32_t* __restrict__ wl_off;   // [n_stages][grid+1] CSR offsets into wl_items
   const uint2* __restrict__ wl_items;    // {partition, stream} per work item
 };
@@ -309,24 +310,30 @@ __device__ __forceinline__ void exec_layer(const LayerRegs& R, uint32_t s_base, 
   }
 }
 
+// Levels 11-13 for every stream of the item (one thread per stream).
 __device__ __forceinline__ void exec_top(uint32_t flags, uint32_t topc, uint32_t topwo, uint32_t* S,
-                                         const uint32_t* topb) {
+                                         const uint32_t* topb, uint32_t nst, uint32_t state_words) {
   if (flags & GEM_LF_USES_TOP) {
     __syncthreads();
-    if (threadIdx.x == 0) {
+    if (threadIdx.x < nst) {
+      const uint32_t j = threadIdx.x;
       uint32_t t8 = 0;
 #pragma unroll
-      for (uint32_t w = 0; w < GEM_WARPS; w++) t8 |= topb[w] << w;
-      S[topwo] = fold3(t8, topc & 0xFFu, (topc >> 8) & 0xFFu, (topc >> 16) & 0xFFu);
+      for (uint32_t w = 0; w < GEM_WARPS; w++) t8 |= topb[16 * j + w] << w;
+      S[j * state_words + topwo] = fold3(t8, topc & 0xFFu, (topc >> 8) & 0xFFu, (topc >> 16) & 0xFFu);
     }
   }
 }
 
-// One work item = one partition for one stream in one cycle.  In streamed
-// mode the caller has already issued the item's prologue chunks.
+// One work item = one partition for a group of `nst` streams (states S_j =
+// S + j*state_words) in one cycle; every program chunk is loaded once and
+// applied to all streams of the group.  In streamed mode the caller has
+// already issued the item's prologue chunks.
 __device__ void run_partition(const KParams& kp, ProgSrc& ps, uint32_t* S, uint32_t* ramp, uint32_t* topb,
-                              uint32_t p, uint32_t st, uint32_t c, uint32_t cur, uint32_t nxt, bool prof_on) {
+                              uint32_t p, uint32_t st0, uint32_t nst, uint32_t c, uint32_t cur, uint32_t nxt,
+                              bool prof_on) {
   const uint32_t tid = threadIdx.x, lane = tid & 31, warp = tid >> 5;
+  const uint32_t SW = kp.state_words;
   const uint32_t s_base = smem_u32(S);
   const uint32_t* gprog = kp.prog + __ldg(kp.parts + p * GP_WORDS + GP_PROG_OFF);
   const uint32_t* C0;
@@ -366,17 +373,18 @@ __device__ void run_partition(const KParams& kp, ProgSrc& ps, uint32_t* S, uint3
   };
   // ---- a2: global read of input ports (once per cycle)
   const uint32_t* gr = C0 + off_gread;
-  for (uint32_t k = tid; k < n_gread; k += GEM_THREADS) {
-    const uint2 e = *(reinterpret_cast<const uint2*>(gr) + k);
+  for (uint32_t k = tid; k < n_gread * nst; k += GEM_THREADS) {
+    const uint32_t j = k / n_gread, st = st0 + j;
+    const uint2 e = *(reinterpret_cast<const uint2*>(gr) + (k - j * n_gread));
     const uint32_t reg = GEM_GID_REGION(e.x), idx = GEM_GID_INDEX(e.x);
     uint32_t v;
     if (reg == GEM_R_PI) v = __ldg(kp.pi + ((size_t)st * kp.in_cap + kp.in_base + c) * kp.pi_words + idx);
     else if (reg == GEM_R_Q) v = rd_global(kp.q + ((size_t)cur * kp.n_streams + st) * kp.q_words + idx);
     else if (reg == GEM_R_RD) v = rd_global(kp.rd + ((size_t)cur * kp.n_streams + st) * kp.n_rams + idx);
     else v = rd_global(kp.cut + (size_t)st * kp.cut_words + idx);
-    S[e.y] = v;
+    S[j * SW + e.y] = v;
   }
-  if (tid == 0) S[0] = 0u;
+  if (tid < nst) S[tid * SW] = 0u;
   // first layer's records (independent of S) before the barrier
   LayerRegs R;
   const uint32_t* Lres = C0 + off_layers;
@@ -393,7 +401,7 @@ __device__ void run_partition(const KParams& kp, ProgSrc& ps, uint32_t* S, uint3
   // ---- a3-a5: layers, software-pipelined: layer l+1's records are loaded
   // into registers before the barrier that ends layer l
   for (uint32_t l = 0; l < n_layers; l++) {
-    exec_layer(R, s_base, topb);
+    for (uint32_t j = 0; j < nst; j++) exec_layer(R, s_base + 4 * j * SW, topb + 16 * j);
     const uint32_t flags = R.flags, topc = R.topc, topwo = R.topwo;
     if (l + 1 < n_layers) {
       const uint32_t* L;
@@ -401,38 +409,41 @@ __device__ void run_partition(const KParams& kp, ProgSrc& ps, uint32_t* S, uint3
       else L = ring_wait(ps);
       load_layer(L, R);
     }
-    exec_top(flags, topc, topwo, S, topb);
+    exec_top(flags, topc, topwo, S, topb, nst, SW);
     __syncthreads();
     if (!ps.resident && l + 1 < n_layers) ps.seq_free++;
     refill();
   }
   PROF(2);
-  // ---- a6: endpoint commit (warp ballot-gather per output word)
+  // ---- a6: endpoint commit (warp ballot-gather per output word and stream)
   const uint32_t* od = ps.resident ? (C0 + off_out) : ring_wait(ps);
   const uint32_t* os = od + n_out_pad;
-  for (uint32_t j = warp; j < n_out; j += GEM_WARPS) {
-    const uint32_t e = os[j * 32 + lane];
+  for (uint32_t jj = warp; jj < n_out * nst; jj += GEM_WARPS) {
+    const uint32_t j = jj / n_out, o = jj - j * n_out, st = st0 + j;
+    const uint32_t e = os[o * 32 + lane];
     const uint32_t src = e & 0x7FFFFFFFu;
-    const uint32_t bit = ((S[src >> 5] >> (src & 31u)) & 1u) ^ (e >> 31);
+    const uint32_t bit = ((S[j * SW + (src >> 5)] >> (src & 31u)) & 1u) ^ (e >> 31);
     const uint32_t v = __ballot_sync(0xFFFFFFFFu, bit);
     if (lane == 0) {
-      const uint32_t dst = od[j];
+      const uint32_t dst = od[o];
       const uint32_t reg = GEM_GID_REGION(dst), idx = GEM_GID_INDEX(dst);
       if (reg == GEM_R_Q) __stcg(kp.q + ((size_t)nxt * kp.n_streams + st) * kp.q_words + idx, v);
       else if (reg == GEM_R_PO) __stcg(kp.po + ((size_t)st * kp.out_cap + c) * kp.po_words + idx, v);
       else if (reg == GEM_R_CUT) __stcg(kp.cut + (size_t)st * kp.cut_words + idx, v);
-      else ramp[idx] = v;
+      else ramp[j * 4 * GEM_MAX_RAMS_PER_PART + idx] = v;
     }
   }
   // ---- a7: RAM blocks (read-first, then per-bit write; readings U7-U10)
   if (n_ram) {
     __syncthreads();
     const uint32_t* rr = od + (off_ram - off_out);
-    for (uint32_t r = tid; r < n_ram; r += GEM_THREADS) {
+    for (uint32_t jr = tid; jr < n_ram * nst; jr += GEM_THREADS) {
+      const uint32_t j = jr / n_ram, r = jr - j * n_ram, st = st0 + j;
+      const uint32_t* rp = ramp + j * 4 * GEM_MAX_RAMS_PER_PART + 4 * r;
       const uint32_t id = rr[4 * r];
-      const uint32_t ra = ramp[4 * r + GEM_PORT_RADDR] & (GEM_RAM_WORDS - 1);
-      const uint32_t wa = ramp[4 * r + GEM_PORT_WADDR] & (GEM_RAM_WORDS - 1);
-      const uint32_t wd = ramp[4 * r + GEM_PORT_WDATA], be = ramp[4 * r + GEM_PORT_WBE];
+      const uint32_t ra = rp[GEM_PORT_RADDR] & (GEM_RAM_WORDS - 1);
+      const uint32_t wa = rp[GEM_PORT_WADDR] & (GEM_RAM_WORDS - 1);
+      const uint32_t wd = rp[GEM_PORT_WDATA], be = rp[GEM_PORT_WBE];
       uint32_t* M = kp.mem + ((size_t)st * kp.n_rams + id) * GEM_RAM_WORDS;
       const uint32_t old = __ldcg(M + ra);
       const uint32_t cur_w = __ldcg(M + wa);
@@ -471,15 +482,15 @@ __device__ void record_state(const KParams& kp, uint32_t c, uint32_t buf) {
 
 __global__ void __launch_bounds__(GEM_THREADS, 2) gem_step_kernel(const KParams kp) {
   extern __shared__ __align__(16) uint32_t smem[];
-  // layout (words): S[state_words] | area[area_words] | ctab[256] | ramp[128] | topb[16] |
-  //                 res_p[16] | res_off[16] | res_n[16] | mbar[8 x u64]
+  // layout (words): S[group][state_words] | area[area_words] | ctab[256] | ramp[group][128] |
+  //                 topb[group][16] | res_p[16] | res_off[16] | res_n[16] | mbar[8 x u64]
   // S must stay at offset 0 (leaf entries carry byte offsets into it).
   uint32_t* S = smem;
-  uint32_t* area = S + kp.state_words;
+  uint32_t* area = S + kp.group * kp.state_words;
   uint32_t* ctab = area + kp.area_words;
   uint32_t* ramp = ctab + GEM_MAX_CHUNKS;
-  uint32_t* topb = ramp + 4 * GEM_MAX_RAMS_PER_PART;
-  uint32_t* res_p = topb + 16;
+  uint32_t* topb = ramp + kp.group * 4 * GEM_MAX_RAMS_PER_PART;
+  uint32_t* res_p = topb + 16 * kp.group;
   uint32_t* res_off = res_p + GEM_MAX_RESIDENT;
   uint32_t* res_n = res_off + GEM_MAX_RESIDENT;      // [0] = n_res, [1] = resident flag
   uint64_t* mbar = reinterpret_cast<uint64_t*>(res_n + 16);
@@ -557,7 +568,8 @@ __global__ void __launch_bounds__(GEM_THREADS, 2) gem_step_kernel(const KParams 
       const uint32_t kb = wl_begin(s), ke = wl_end(s);
       for (uint32_t k = kb; k < ke; k++) {
         const uint2 it = __ldg(&kp.wl_items[k]);
-        run_partition(kp, ps, S, ramp, topb, it.x, it.y, c, cur, nxt, prof_on && k == kb && s == 0);
+        const uint32_t nst = min(kp.group, kp.n_streams - it.y);
+        run_partition(kp, ps, S, ramp, topb, it.x, it.y, nst, c, cur, nxt, prof_on && k == kb && s == 0);
         if (!ps.resident) {
           // prefetch the next work item's prologue (overlaps the grid barrier)
           uint32_t nk = ~0u;
@@ -634,7 +646,7 @@ struct gem_sim {
   uint32_t po_words_ext = 0, q_words_ext = 0;
   uint64_t n_and = 0, n_and_mapped = 0, program_bytes = 0;
   uint32_t max_items = 0;
-  uint32_t area_words = 0, slot_words = 0, ring_slots = 0, resident = 0;
+  uint32_t area_words = 0, slot_words = 0, ring_slots = 0, resident = 0, group = 1;
   std::vector<uint32_t> h_parts, h_stage;
   // device buffers
   uint32_t *d_prog = nullptr, *d_parts = nullptr, *d_stage = nullptr;
@@ -715,10 +727,12 @@ static double build_worklists(const gem_sim* sim, uint32_t G, std::vector<uint32
     const uint32_t pb = sim->h_stage[s], np = sim->h_stage[s + 1] - pb;
     std::vector<std::pair<uint32_t, uint2>> its;
     its.reserve((size_t)np * sim->n_streams);
-    for (uint32_t st = 0; st < sim->n_streams; st++)
+    for (uint32_t st = 0; st < sim->n_streams; st += sim->group)
       for (uint32_t k = 0; k < np; k++) {
         const uint32_t p = sim->h_stage[sim->n_stages + 1 + pb + k];
-        its.push_back({sim->h_parts[(size_t)p * GP_WORDS + GP_COST], make_uint2(p, st)});
+        const uint32_t nst = std::min(sim->group, sim->n_streams - st);
+        const double c = sim->h_parts[(size_t)p * GP_WORDS + GP_COST] * (1.0 + 0.7 * (nst - 1));
+        its.push_back({(uint32_t)std::min(c, 4.0e9), make_uint2(p, st)});
       }
     std::stable_sort(its.begin(), its.end(), [](const std::pair<uint32_t, uint2>& x,
                                                 const std::pair<uint32_t, uint2>& y) { return x.first > y.first; });
@@ -763,8 +777,24 @@ static int plan_launch(gem_sim* sim, uint32_t max_chunk_words, uint32_t grid_lim
   CK(cudaDeviceGetAttribute(&per_sm, cudaDevAttrMaxSharedMemoryPerMultiprocessor, sim->device));
   if (!coop) return fail(GEM_E_UNSUPPORTED, "device lacks cooperative launch");
   sim->sm_count = (uint32_t)sms;
-  const uint32_t fixed_words = sim->state_words + GEM_MAX_CHUNKS + 4 * GEM_MAX_RAMS_PER_PART + 16 + 48 + 16;
   const uint32_t slot = (max_chunk_words + 3u) & ~3u;
+  // streams per work item: as many stream states as fit beside a 3-slot ring
+  sim->group = 1;
+  if (sim->n_streams > 1) {
+    const char* genv = getenv("GEM_GROUP");
+    uint32_t g = genv ? (uint32_t)atoi(genv) : 16;
+    g = std::max<uint32_t>(1, std::min<uint32_t>(g, sim->n_streams));
+    while (g > 1 && (uint64_t)(g * (sim->state_words + 4 * GEM_MAX_RAMS_PER_PART + 16) + GEM_MAX_CHUNKS + 80 +
+                               3 * slot) * 4 > (uint64_t)optin)
+      g /= 2;
+    sim->group = g;
+  }
+  sim->max_items = 0;
+  for (uint32_t s = 0; s < sim->n_stages; s++)
+    sim->max_items = std::max(sim->max_items, (sim->h_stage[s + 1] - sim->h_stage[s]) *
+                                                  ((sim->n_streams + sim->group - 1) / sim->group));
+  const uint32_t fixed_words =
+      sim->group * (sim->state_words + 4 * GEM_MAX_RAMS_PER_PART + 16) + GEM_MAX_CHUNKS + 48 + 16;
   const char* env = getenv("GEM_NO_RESIDENT");
   const bool allow_res = !(env && env[0] == '1');
   const char* benv = getenv("GEM_BPS");
@@ -946,7 +976,7 @@ int gem_info_get(const gem_sim* sim, gem_info* out) {
   out->total_layers = sim->total_layers;
   out->pi_words = sim->pi_words; out->po_words = sim->po_words_ext; out->q_words = sim->q_words_ext;
   out->grid = sim->grid; out->blocks_per_sm = sim->blocks_per_sm; out->smem_bytes = sim->smem_bytes;
-  out->resident = sim->resident; out->ring_slots = sim->ring_slots;
+  out->resident = sim->resident; out->ring_slots = sim->ring_slots; out->group = sim->group;
   out->n_streams = sim->n_streams;
   out->n_and = sim->n_and; out->n_and_mapped = sim->n_and_mapped; out->program_bytes = sim->program_bytes;
   out->cycle = sim->cycle;
@@ -998,6 +1028,7 @@ int gem_step(gem_sim* sim, uint64_t ncycles) {
   kp.area_words = sim->area_words; kp.slot_words = sim->slot_words; kp.ring_slots = sim->ring_slots;
   kp.allow_resident = sim->resident;
   kp.wl_off = sim->d_wl_off;
+  kp.group = sim->group;
   kp.wl_items = sim->d_wl_items;
   if (sim->flags & GEM_F_PROFILE) {
     const uint32_t pc = (uint32_t)std::min<uint64_t>(ncycles, 256);

@@ -917,10 +917,23 @@ static void partition(Design& D) {
   }
   // ---- units
   std::vector<Unit> units;
-  auto s0 = cone_minhash(G, 1), s1 = cone_minhash(G, 2);
+  // Locality key of a unit: the smallest flop (state) index in its cone --
+  // logic that reads the same registers sits in the same module -- with a
+  // cone min-hash as tie breaker.
+  auto s0 = cone_minhash(G, 1);
+  std::vector<uint32_t> mflop(N, UINT32_MAX);
+  for (size_t i = 0; i < N; i++) {
+    if (G.kind[i] == K_SRC) {
+      uint32_t gb = G.gbit[i];
+      if ((gb >> 27) == GEM_R_Q) mflop[i] = ((gb >> 5) & 0x3FFFFF) * 32 + (gb & 31);
+      else if ((gb >> 27) == GEM_R_RD) mflop[i] = 0x7FFFFFFFu + ((gb >> 5) & 0x3FFFFF);
+    } else if (G.kind[i] == K_AND) {
+      mflop[i] = std::min(mflop[G.a[i] >> 1], mflop[G.b[i] >> 1]);
+    }
+  }
   auto key_of = [&](uint32_t lit) -> uint64_t {
     uint32_t x = lit >> 1;
-    return (uint64_t)((s0[x] & 0xFFFFFFFF00000000ull) | (s1[x] >> 32));
+    return ((uint64_t)mflop[x] << 32) | (s0[x] >> 32);
   };
   std::vector<uint32_t> cut_nodes;            // compact ids that are stage-0 endpoints
   std::vector<int32_t> cut_of(N, -1);
@@ -1013,9 +1026,23 @@ static void partition(Design& D) {
     int target = opt.parts > 0 ? opt.parts : (int)std::max<uint64_t>(1, (G.n_and_live + opt.part_size / 2) / opt.part_size);
     if (opt.stages == 2) target = std::max(1, target / 2);
     target = std::max(1, std::min<int>(target, (int)su.size()));
-    double cap = std::max<double>(64.0, (double)stage_ands / target * opt.cap_slack);
+    // a cap below typical single-unit cones would leave every unit alone (and
+    // re-traverse each full cone): start from >= 3x the median unit cone
+    double med = 0;
+    {
+      std::vector<uint32_t> sz;
+      for (size_t i = 0; i < su.size(); i += std::max<size_t>(1, su.size() / 256)) {
+        cur_stamp++;
+        sz.push_back(add_cone(su[i]));
+      }
+      if (!sz.empty()) {
+        std::nth_element(sz.begin(), sz.begin() + sz.size() / 2, sz.end());
+        med = sz[sz.size() / 2];
+      }
+    }
+    double cap = std::max<double>({64.0, 4.0 * (double)stage_ands / target * opt.cap_slack, 3.0 * med});
     std::vector<std::vector<uint32_t>> groups;   // indices into su
-    for (int iter = 0; iter < 6; iter++) {
+    for (int iter = 0; iter < 4; iter++) {
       groups.clear();
       cur_stamp++;
       uint64_t size = 0;
@@ -1035,7 +1062,10 @@ static void partition(Design& D) {
         }
       }
       double ratio = (double)groups.size() / target;
-      if (ratio > 0.9 && ratio < 1.15) break;
+      if (opt.verbose >= 1)
+        fprintf(stderr, "gem_map: stage %d packing iter %d cap %.0f -> %zu groups (target %d)\n", stage, iter, cap,
+                groups.size(), target);
+      if (ratio > 0.85 && ratio < 1.2) break;
       cap *= std::max(0.5, std::min(2.0, ratio));
     }
     for (auto& grp : groups) {
@@ -1141,10 +1171,22 @@ static Blob compile(const char* data, size_t n, const char* opts) {
   auto t0 = std::chrono::steady_clock::now();
   Design D;
   D.opt = parse_opts(opts);
+  auto tick = [&](const char* what) {
+    if (D.opt.verbose) {
+      static thread_local auto last = std::chrono::steady_clock::now();
+      auto now = std::chrono::steady_clock::now();
+      fprintf(stderr, "gem_map: %-10s %8.0f ms\n", what, std::chrono::duration<double, std::milli>(now - last).count());
+      last = now;
+    }
+  };
+  tick("start");
   Raw raw = read_aiger(data, n);
+  tick("parse");
   D.G = build_graph(raw);
   raw = Raw();
+  tick("strash");
   partition(D);
+  tick("partition");
   // remember which compact nodes are cut nodes (stage-1 leaves) before layout rewrites cut_lit
   std::vector<uint32_t> cut_nodes;
   for (auto& P : D.parts) (void)P;

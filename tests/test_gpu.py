@@ -135,6 +135,39 @@ def test_c5_streams_vs_oracle_lanes(gem):
     assert np.array_equal(dg, r["digest"])
 
 
+def test_c5_ragged_stream_groups(gem):
+    """37 streams (not a multiple of the stream group): every stream matches the oracle lanes."""
+    S, T = 37, 60
+    st = stimulus_streams("c5", 256, T, range(100, 100 + S))
+    sim = gem.Simulator(blob("c5"), n_streams=S, flags=gem.GEM_F_DIGEST)
+    assert sim.info["group"] > 1
+    sim.set_inputs(st)
+    sim.step(T)
+    o = Oracle(eaig("c5"))
+    o.lanes_reset(1)
+    r = o.lanes_run(0, st, digest=True)
+    assert np.array_equal(sim.read_outputs(T), r["po"])
+    assert np.array_equal(sim.read_digests(T), r["digest"])
+
+
+def test_c4_sampled_window(gem):
+    """C4 (~10M ANDs, 2 stages, 24 RAM blocks): full PO trace and per-cycle flop
+    digests for a window the oracle finishes in seconds, plus final state."""
+    T = 60
+    st = stimulus("c4", 512, T)
+    sim = gem.Simulator(blob("c4"), flags=gem.GEM_F_DIGEST)
+    assert sim.info["n_stages"] == 2
+    sim.set_inputs(st)
+    sim.step(T)
+    o = Oracle(eaig("c4"))
+    r = o.run(st, digest=True)
+    assert np.array_equal(sim.read_outputs(T)[0], r["po"])
+    assert np.array_equal(sim.read_digests(T)[0], r["digest"])
+    assert np.array_equal(sim.read_state()[0], o.get_state())
+    for ram in (0, 17, 23):
+        assert np.array_equal(sim.read_ram(ram), o.get_ram(ram))
+
+
 def test_noinput_and_bad_args(gem):
     sim = gem.Simulator(blob("c1"))
     sim.set_inputs(stimulus("c1", 35, 10))
