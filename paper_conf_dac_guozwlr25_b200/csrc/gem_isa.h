@@ -78,6 +78,10 @@
   ((((uint32_t)(pos) - (uint32_t)(bit)) & 31u) | ((uint32_t)(word) << 7) | ((uint32_t)(pos) << 24))
 #define GEM_LEAF_DENSE(word, bit, pos) ((((uint32_t)(pos) - (uint32_t)(bit)) & 31u) | ((uint32_t)(word) << 7))
 #define GEM_LEAF_WORD(e) (((e) >> 7) & 0x1FFFu)
+/* 16-bit dense entry (DENSE16 warps, state words < 2048): rot | word << 5;
+ * u32 k of a lane's group g holds entries 8g+2k (low half) and 8g+2k+1 (high). */
+#define GEM_LEAF16(word, bit, pos) ((((uint32_t)(pos) - (uint32_t)(bit)) & 31u) | ((uint32_t)(word) << 5))
+#define GEM_LEAF16_WORD(h) (((h) >> 5) & 0x7FFu)
 #define GEM_LEAF_ROT(e) ((e) & 31u)
 #define GEM_LEAF_POS(e) (((e) >> 24) & 31u)
 
@@ -139,7 +143,8 @@ enum {
 };
 #define GEM_LF_USES_TOP 0x100u   /* flags bit 8; bits [0,8) = active warp mask */
 #define GEM_WM_SPARSE 0u
-#define GEM_WM_DENSE 1u
+#define GEM_WM_DENSE 1u     /* 32 u32 entries per lane (n4 = 8)                  */
+#define GEM_WM_DENSE16 2u   /* 32 u16 entries per lane (n4 = 4)                  */
 #define GEM_WREC_HDR 8
 #define GEM_WARP_REC_WORDS(n4) (GEM_WREC_HDR + 32 * 4 + 128 * (n4))
 

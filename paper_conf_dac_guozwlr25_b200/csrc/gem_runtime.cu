@@ -57,9 +57,20 @@ struct KParams {
   unsigned long long* prof;   // GEM_F_PROFILE: [prof_cycles][grid][8] clock64 stamps
   uint32_t prof_cycles;
   uint32_t group;                        // streams per work item (stream states in smem)
+  unsigned long long* fprof;             // debug builds (GEM_FINE_PROF) only
   const uint32_t* __restrict__ wl_off;   // [n_stages][grid+1] CSR offsets into wl_items
   const uint2* __restrict__ wl_items;    // {partition, stream} per work item
 };
+#ifdef GEM_FINE_PROF
+// debug build only: per-warp stamps inside the first 8 layers of cycle 5, CTA 0
+#define FPROF(l_, slot_)                                                                      \
+  do {                                                                                        \
+    if (kp.fprof && c == 5 && blockIdx.x == 0 && (l_) < 8 && (threadIdx.x & 31) == 0)        \
+      kp.fprof[((l_) * 8 + (threadIdx.x >> 5)) * 8 + (slot_)] = clock64();                    \
+  } while (0)
+#else
+#define FPROF(l_, slot_) do { } while (0)
+#endif
 #define PROF(slot_)                                                                          \
   do {                                                                                       \
     if (prof_on && threadIdx.x == 0)                                                         \
@@ -103,16 +114,21 @@ __device__ __forceinline__ void grid_sync(const KParams& kp, unsigned long long&
   }
 }
 
-// Levels 1-5 (or 6-10) of the boomerang fold on one 32-bit word; constants are
-// the packed per-unit slot words (gem_isa.h).  Bits above each level's width
-// carry don't-care values that only ever shift toward higher positions.
+// Levels 1-5 (or 6-10) of the boomerang fold on one 32-bit word.  The
+// constants stay in their packed slot positions (gem_isa.h: L1 bits [0,16),
+// L2 [16,24), L3 [24,28), L4 [28,30), L5 [30]); the data of level k is shifted
+// into level k's field instead (2 shifts + 2 LOP3 per level), and the packed
+// result is assembled with bit-selects.  Bits outside each level's field are
+// don't-care.
+__device__ __forceinline__ uint32_t bsel(uint32_t a, uint32_t b, uint32_t m) { return (a & ~m) | (b & m); }
 __device__ __forceinline__ uint32_t fold5(uint32_t v, uint32_t xa, uint32_t xb, uint32_t ob) {
-  uint32_t r1 = (v ^ xa) & (((v >> 16) ^ xb) | ob);
-  uint32_t r2 = (r1 ^ (xa >> 16)) & (((r1 >> 8) ^ (xb >> 16)) | (ob >> 16));
-  uint32_t r3 = (r2 ^ (xa >> 24)) & (((r2 >> 4) ^ (xb >> 24)) | (ob >> 24));
-  uint32_t r4 = (r3 ^ (xa >> 28)) & (((r3 >> 2) ^ (xb >> 28)) | (ob >> 28));
-  uint32_t r5 = (r4 ^ (xa >> 30)) & (((r4 >> 1) ^ (xb >> 30)) | (ob >> 30));
-  return (r1 & 0xFFFFu) | ((r2 & 0xFFu) << 16) | ((r3 & 0xFu) << 24) | ((r4 & 3u) << 28) | ((r5 & 1u) << 30);
+  const uint32_t r1 = (v ^ xa) & (((v >> 16) ^ xb) | ob);                  // [0,16): A=v[q], B=v[q+16]
+  const uint32_t r2 = ((r1 << 16) ^ xa) & (((r1 << 8) ^ xb) | ob);         // [16,24): A=r1[q], B=r1[q+8]
+  const uint32_t r3 = ((r2 << 8) ^ xa) & (((r2 << 4) ^ xb) | ob);          // [24,28): A=r2[16+q], B=r2[20+q]
+  const uint32_t r4 = ((r3 << 4) ^ xa) & (((r3 << 2) ^ xb) | ob);          // [28,30)
+  const uint32_t r5 = ((r4 << 2) ^ xa) & (((r4 << 1) ^ xb) | ob);          // [30]
+  return bsel(bsel(bsel(bsel(r1, r2, 0x00FF0000u), r3, 0x0F000000u), r4, 0x30000000u), r5, 0xC0000000u) &
+         0x7FFFFFFFu;
 }
 
 // Levels 11-13 on the 8 warp bits.
@@ -177,21 +193,22 @@ struct ProgSrc {
   const uint32_t* res_off; // smem [GEM_MAX_RESIDENT] word offsets into area
 };
 
+// ring depth R is a power of two (2 or 4): slot = seq & (R-1), phase = (seq / R) & 1
 __device__ __forceinline__ uint32_t* ring_slot(const ProgSrc& ps, uint32_t seq) {
-  return ps.area + (size_t)(seq % ps.R) * ps.slot_words;
+  return ps.area + (seq & (ps.R - 1)) * ps.slot_words;
 }
 // All threads call this (uniformly); thread 0 issues the copy.
 __device__ __forceinline__ void ring_issue(ProgSrc& ps, const uint32_t* g, uint32_t words) {
   const uint32_t seq = ps.seq_issue++;
   if (threadIdx.x == 0) {
-    uint64_t* bar = ps.mbar + seq % ps.R;
+    uint64_t* bar = ps.mbar + (seq & (ps.R - 1));
     mbar_expect_tx(bar, words * 4);
     tma_load_1d(ring_slot(ps, seq), g, words * 4, bar);
   }
 }
 __device__ __forceinline__ const uint32_t* ring_wait(ProgSrc& ps) {
   const uint32_t seq = ps.seq_wait++;
-  mbar_wait(ps.mbar + seq % ps.R, (seq / ps.R) & 1u);
+  mbar_wait(ps.mbar + (seq & (ps.R - 1)), (seq >> (ps.R == 4 ? 2 : 1)) & 1u);
   return ring_slot(ps, seq);
 }
 
@@ -279,7 +296,20 @@ __device__ __forceinline__ void exec_layer(const LayerRegs& R, uint32_t s_base, 
   if ((R.flags >> warp) & 1u) {
     uint32_t v = 0;
     const uint32_t n4 = R.mode >> 8;
-    if ((R.mode & 0xFFu) == GEM_WM_DENSE) {
+    if ((R.mode & 0xFFu) == GEM_WM_DENSE16) {
+      // two 16-bit entries per u32: entry 8g+2k in the low half, 8g+2k+1 in the high half
+#pragma unroll
+      for (uint32_t g = 0; g < 4; g++) {
+        const uint32_t q[4] = {R.e[g].x, R.e[g].y, R.e[g].z, R.e[g].w};
+#pragma unroll
+        for (uint32_t k = 0; k < 4; k++) {
+          const uint32_t lo = lds(s_base + ((q[k] >> 3) & 0x1FFCu));
+          const uint32_t hi = lds(s_base + ((q[k] >> 19) & 0x1FFCu));
+          v |= __funnelshift_l(lo, lo, q[k]) & (1u << (8 * g + 2 * k));
+          v |= __funnelshift_l(hi, hi, q[k] >> 16) & (1u << (8 * g + 2 * k + 1));
+        }
+      }
+    } else if ((R.mode & 0xFFu) == GEM_WM_DENSE) {
       // entry j of the lane fills leaf position j: rotate + LOP3 with an immediate mask
 #pragma unroll
       for (uint32_t g = 0; g < 8; g++) {
@@ -308,19 +338,16 @@ __device__ __forceinline__ void exec_layer(const LayerRegs& R, uint32_t s_base, 
   } else if (uses_top && lane == 0) {
     topb[warp] = 0u;
   }
-}
-
-// Levels 11-13 for every stream of the item (one thread per stream).
-__device__ __forceinline__ void exec_top(uint32_t flags, uint32_t topc, uint32_t topwo, uint32_t* S,
-                                         const uint32_t* topb, uint32_t nst, uint32_t state_words) {
-  if (flags & GEM_LF_USES_TOP) {
-    __syncthreads();
-    if (threadIdx.x < nst) {
-      const uint32_t j = threadIdx.x;
+  // levels 11-13: the last warp to arrive folds the 8 warp bits (no extra barrier)
+  if (uses_top && lane == 0) {
+    __threadfence_block();
+    if (atomicAdd(&topb[8], 1u) == GEM_WARPS - 1) {
+      __threadfence_block();
       uint32_t t8 = 0;
 #pragma unroll
-      for (uint32_t w = 0; w < GEM_WARPS; w++) t8 |= topb[16 * j + w] << w;
-      S[j * state_words + topwo] = fold3(t8, topc & 0xFFu, (topc >> 8) & 0xFFu, (topc >> 16) & 0xFFu);
+      for (uint32_t w = 0; w < GEM_WARPS; w++) t8 |= *((volatile uint32_t*)topb + w) << w;
+      sts(s_base + 4 * R.topwo, fold3(t8, R.topc & 0xFFu, (R.topc >> 8) & 0xFFu, (R.topc >> 16) & 0xFFu));
+      topb[8] = 0u;
     }
   }
 }
@@ -401,16 +428,22 @@ __device__ void run_partition(const KParams& kp, ProgSrc& ps, uint32_t* S, uint3
   // ---- a3-a5: layers, software-pipelined: layer l+1's records are loaded
   // into registers before the barrier that ends layer l
   for (uint32_t l = 0; l < n_layers; l++) {
+    FPROF(l, 0);
     for (uint32_t j = 0; j < nst; j++) exec_layer(R, s_base + 4 * j * SW, topb + 16 * j);
+    FPROF(l, 1);
     const uint32_t flags = R.flags, topc = R.topc, topwo = R.topwo;
     if (l + 1 < n_layers) {
       const uint32_t* L;
       if (ps.resident) { L = Lres; Lres += ctab[2 + l]; }
       else L = ring_wait(ps);
+      FPROF(l, 2);
       load_layer(L, R);
     }
-    exec_top(flags, topc, topwo, S, topb, nst, SW);
+    FPROF(l, 3);
+    (void)flags; (void)topc; (void)topwo;
+    FPROF(l, 4);
     __syncthreads();
+    FPROF(l, 5);
     if (!ps.resident && l + 1 < n_layers) ps.seq_free++;
     refill();
   }
@@ -498,6 +531,7 @@ __global__ void __launch_bounds__(GEM_THREADS, 2) gem_step_kernel(const KParams 
   const uint32_t G = gridDim.x, B = blockIdx.x;
   auto wl_begin = [&](uint32_t s) { return __ldg(kp.wl_off + s * (G + 1) + B); };
   auto wl_end = [&](uint32_t s) { return __ldg(kp.wl_off + s * (G + 1) + B + 1); };
+  for (uint32_t k = tid; k < 16 * kp.group; k += GEM_THREADS) topb[k] = 0u;
   if (tid == 0) {
     for (uint32_t k = 0; k <= GEM_RING_MAX; k++) mbar_init(mbar + k, 1);
     fence_mbar_init();
@@ -654,7 +688,7 @@ struct gem_sim {
   uint32_t *d_q = nullptr, *d_rd = nullptr, *d_cut = nullptr, *d_mem = nullptr;
   uint32_t *d_pi = nullptr, *d_po = nullptr, *d_qtrace = nullptr, *d_scratch = nullptr, *d_wl_off = nullptr;
   uint2* d_wl_items = nullptr;
-  unsigned long long *d_digest = nullptr, *d_bar = nullptr, *d_prof = nullptr;
+  unsigned long long *d_digest = nullptr, *d_bar = nullptr, *d_prof = nullptr, *d_fprof = nullptr;
   uint32_t prof_cycles = 0;
   int* d_err = nullptr;
   uint32_t in_cap = 0, in_queued = 0, in_head = 0, out_cap = 0, last_cycles = 0;
@@ -832,7 +866,8 @@ static int plan_launch(gem_sim* sim, uint32_t max_chunk_words, uint32_t grid_lim
           if (seen.size() > GEM_MAX_RESIDENT || words > area) { res = false; break; }
         }
     }
-    const uint32_t ring = std::min<uint32_t>(GEM_RING_MAX, area / std::max<uint32_t>(slot, 4));
+    uint32_t ring = std::min<uint32_t>(GEM_RING_MAX, area / std::max<uint32_t>(slot, 4));
+    ring = ring >= 4 ? 4 : ring >= 2 ? 2 : ring;   // power of two (kernel masks instead of dividing)
     if (!res && ring < 2) continue;
     // score: estimated makespan, SM sharing slows co-resident CTAs, streaming costs a little
     double score = makespan * (1.0 + 0.5 * (bps - 1) * std::min(1.0, (double)grid / ((double)bps * sms)))
@@ -1035,12 +1070,16 @@ int gem_step(gem_sim* sim, uint64_t ncycles) {
     if (!sim->d_prof || sim->prof_cycles < pc) {
       if (sim->d_prof) cudaFree(sim->d_prof);
       sim->d_prof = nullptr;
-      CK(dalloc(&sim->d_prof, (size_t)256 * sim->grid * 8 * 8));
+      CK(dalloc(&sim->d_prof, (size_t)256 * sim->grid * 8 * 8 + 8 * 8 * 8 * 8));
+#ifdef GEM_FINE_PROF
+      CK(dalloc(&sim->d_fprof, 8 * 8 * 8 * 8));
+#endif
     }
     sim->prof_cycles = pc;
-    CK(cudaMemsetAsync(sim->d_prof, 0, (size_t)256 * sim->grid * 8 * 8, sim->stream));
+    CK(cudaMemsetAsync(sim->d_prof, 0, (size_t)256 * sim->grid * 8 * 8 + 8 * 8 * 8 * 8, sim->stream));
     kp.prof = sim->d_prof;
     kp.prof_cycles = pc;
+    kp.fprof = sim->d_fprof;
   }
   CK(cudaMemsetAsync(sim->d_bar, 0, 8, sim->stream));
   if (sim->flags & GEM_F_DIGEST)
@@ -1175,6 +1214,14 @@ int gem_write_ram(gem_sim* sim, uint32_t ram_id, uint32_t stream, const uint32_t
                 cudaMemcpyHostToDevice));
   return GEM_OK;
 }
+
+#ifdef GEM_FINE_PROF
+int gem_read_fine(gem_sim* sim, uint64_t* dst) {
+  CK(cudaStreamSynchronize(sim->stream));
+  CK(cudaMemcpy(dst, sim->d_fprof, 8 * 8 * 8 * 8, cudaMemcpyDeviceToHost));
+  return GEM_OK;
+}
+#endif
 
 int gem_read_profile(gem_sim* sim, uint64_t* dst, uint32_t* n_cycles, uint32_t* grid) {
   if (int r = check(sim)) return r;

@@ -57,6 +57,9 @@ struct Options {
   int stages = 1;           // 1 or 2 (multi-stage RepCut)
   int cut_level = 0;        // 0 = auto (middle)
   int merge = 1;            // Algorithm 1 merge pass
+  int refine = 3;           // rounds of splitting the costliest partitions (critical path)
+  double refine_ratio = 1.35;  // split partitions costing more than this x the median
+  int max_parts = 280;      // refinement stops growing the partition count here
   int verbose = 0;
   int max_state_words = GEM_MAX_STATE_WORDS;
   double cap_slack = 1.0;
@@ -81,6 +84,9 @@ static Options parse_opts(const char* s) {
     else if (k == "verbose") o.verbose = std::stoi(v);
     else if (k == "max_state_words") o.max_state_words = std::stoi(v);
     else if (k == "cap_slack") o.cap_slack = std::stod(v);
+    else if (k == "refine") o.refine = std::stoi(v);
+    else if (k == "refine_ratio") o.refine_ratio = std::stod(v);
+    else if (k == "max_parts") o.max_parts = std::stoi(v);
     else throw std::runtime_error("unknown option " + k);
   }
   if (o.stages < 1 || o.stages > 2) throw std::runtime_error("stages must be 1 or 2");
@@ -828,12 +834,16 @@ struct Mapper {
       if (!(active >> w & 1)) continue;
       out[base + LH_WOFF0 + w] = (uint32_t)(out.size() - base);
       const bool dense = niter[w] > kDenseMin;
-      const uint32_t n4 = dense ? 8u : (niter[w] + 3) / 4;
+      bool small_words = true;
+      for (uint32_t l = 0; l < 32; l++)
+        for (auto& x : leaves[w * 32 + l]) small_words = small_words && (x.first >> 5) < 2048;
+      const bool d16 = dense && small_words;
+      const uint32_t n4 = d16 ? 4u : dense ? 8u : (niter[w] + 3) / 4;
       out.push_back(pack(6, 10, w, sxa));
       out.push_back(pack(6, 10, w, sxb));
       out.push_back(pack(6, 10, w, sob));
       out.push_back(wo_warp[w] >= 0 ? (uint32_t)wo_warp[w] : 0u);
-      out.push_back((dense ? GEM_WM_DENSE : GEM_WM_SPARSE) | (n4 << 8));
+      out.push_back((d16 ? GEM_WM_DENSE16 : dense ? GEM_WM_DENSE : GEM_WM_SPARSE) | (n4 << 8));
       out.push_back(0); out.push_back(0); out.push_back(0);
       for (uint32_t l = 0; l < 32; l++) {
         uint32_t t = w * 32 + l;
@@ -847,7 +857,13 @@ struct Mapper {
           auto& lv = leaves[w * 32 + l];
           for (uint32_t c = 0; c < 4; c++) {
             uint32_t j = 4 * g + c, e = 0;
-            if (dense) {
+            if (d16) {
+              for (uint32_t h = 0; h < 2; h++) {
+                uint32_t jj = 8 * g + 2 * c + h;
+                for (auto& x : lv)
+                  if (x.second == jj) e |= GEM_LEAF16(x.first >> 5, x.first & 31, jj) << (16 * h);
+              }
+            } else if (dense) {
               for (auto& x : lv)
                 if (x.second == j) e = GEM_LEAF_DENSE(x.first >> 5, x.first & 31, j);
             } else if (j < lv.size()) {
@@ -864,7 +880,7 @@ struct Mapper {
 // Estimated SM clocks for one cycle of a partition program (cost model fitted to
 // B200 phase measurements: fixed per-layer latency + per-16-byte leaf group).
 static uint32_t part_cost(const uint32_t* pr) {
-  const double kItem = 3000.0, kLayer = 900.0, kGroup = 14.0, kGread = 1.5, kOut = 20.0;
+  const double kItem = 6000.0, kLayer = 1900.0, kGroup = 12.0, kGread = 2.0, kOut = 20.0;
   double c = kItem + kGread * pr[PH_N_GREAD] + kOut * pr[PH_N_OUT];
   const uint32_t* L = pr + pr[PH_OFF_LAYERS];
   for (uint32_t l = 0; l < pr[PH_N_LAYERS]; l++) {
@@ -1197,6 +1213,17 @@ static Blob compile(const char* data, size_t n, const char* opts) {
   std::vector<uint32_t> cut_compact = D.cut_lit;   // compact literals of cut nodes
   auto t1 = std::chrono::steady_clock::now();
   int nth = D.opt.threads > 0 ? D.opt.threads : (int)std::max(1u, std::thread::hardware_concurrency());
+  // deep-cone signature: min-hash over the nodes deeper than a third of the depth
+  std::vector<uint64_t> dsig(D.G.kind.size(), UINT64_MAX);
+  {
+    const uint32_t thr = std::max<uint32_t>(1, D.G.max_level / 3);
+    for (size_t i = 0; i < D.G.kind.size(); i++) {
+      if (D.G.kind[i] != K_AND) continue;
+      uint64_t h = D.G.level[i] >= thr ? mix64(i * 0x9E3779B97F4A7C15ull + 7) : UINT64_MAX;
+      dsig[i] = std::min(h, std::min(dsig[D.G.a[i] >> 1], dsig[D.G.b[i] >> 1]));
+    }
+  }
+  int refine_round = 0;
   for (int attempt = 0;; attempt++) {
     D.cut_lit = cut_compact;
     layout(D);   // cut_lit now holds internal cut bit indices
@@ -1253,6 +1280,53 @@ static Blob compile(const char* data, size_t n, const char* opts) {
         if (X->flops.size() + X->pos.size() + X->rams.size() + X->cuts.size()) next_parts.push_back(std::move(*X));
     }
     D.parts = std::move(next_parts);
+    if (!any_fail && refine_round < D.opt.refine && D.parts.size() > 1) {
+      // critical-path refinement: split the costliest partitions along the
+      // deep-cone signature (units sharing deep logic stay together)
+      std::vector<uint32_t> cost(D.parts.size());
+      for (size_t i = 0; i < D.parts.size(); i++) cost[i] = part_cost(D.parts[i].prog.data());
+      std::vector<uint32_t> sorted = cost;
+      std::sort(sorted.begin(), sorted.end());
+      const double med = sorted[sorted.size() / 2];
+      std::vector<Part> out;
+      size_t n_split = 0;
+      for (size_t i = 0; i < D.parts.size(); i++) {
+        Part& P = D.parts[i];
+        size_t n_units = P.flops.size() + P.pos.size() + P.rams.size() + P.cuts.size();
+        if (cost[i] > D.opt.refine_ratio * med && n_units > 1 &&
+            D.parts.size() + n_split < (size_t)D.opt.max_parts) {
+          // all units ordered by deep signature, then halved
+          std::vector<std::pair<uint64_t, std::pair<int, uint32_t>>> us;
+          for (auto j : P.flops) us.push_back({dsig[D.G.flop_next[j] >> 1], {0, j}});
+          for (auto j : P.pos) us.push_back({dsig[D.G.po[j] >> 1], {1, j}});
+          for (auto j : P.rams) us.push_back({dsig[D.G.rams[j].port[3][0] >> 1], {2, j}});
+          for (auto j : P.cuts) us.push_back({dsig[cut_compact[j] >> 1], {3, j}});
+          std::stable_sort(us.begin(), us.end(), [](auto& a, auto& b) { return a.first < b.first; });
+          Part A, B;
+          A.stage = B.stage = P.stage;
+          for (size_t k = 0; k < us.size(); k++) {
+            Part& X = k < (us.size() + 1) / 2 ? A : B;
+            auto u = us[k].second;
+            (u.first == 0 ? X.flops : u.first == 1 ? X.pos : u.first == 2 ? X.rams : X.cuts).push_back(u.second);
+          }
+          out.push_back(std::move(A));
+          out.push_back(std::move(B));
+          n_split++;
+        } else {
+          out.push_back(std::move(P));
+        }
+      }
+      refine_round++;
+      if (n_split) {
+        D.parts = std::move(out);
+        for (auto& P : D.parts) { P.prog.clear(); P.ok = false; }
+        if (D.opt.verbose)
+          fprintf(stderr, "gem_map: refine %d: split %zu partitions (median cost %.0f) -> %zu\n", refine_round,
+                  n_split, med, D.parts.size());
+        continue;
+      }
+      D.parts = std::move(out);
+    }
     if (!any_fail) break;
     for (auto& P : D.parts) { P.prog.clear(); P.ok = false; }
     if (D.opt.verbose) fprintf(stderr, "gem_map: retry %d with %zu partitions\n", attempt + 1, D.parts.size());

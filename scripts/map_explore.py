@@ -7,24 +7,9 @@ from paper_conf_dac_guozwlr25_b200.isa import blob_info, GP_WORDS
 from tests.common import eaig
 
 
-def part_costs(b, a=150.0, c=12.0):
-    """est. cycles per partition-cycle: sum over layers of a + c * sum_w niter_w / 4 (issue-bound)."""
-    w = np.frombuffer(b, np.uint32)
+def part_costs(b):
     i = blob_info(b)
-    op, opr = int(w[21]), int(w[24])
-    costs, layers = [], []
-    for p in range(i.n_parts):
-        po = opr + int(w[op + p * GP_WORDS + 1])
-        nl = int(w[po + 2])
-        L = po + int(w[po + 7])
-        t = 0.0
-        for l in range(nl):
-            niter = w[L + 4:L + 12].astype(np.int64)
-            t += a + c * max(niter.max(), niter.sum() / 4)
-            L += int(w[L])
-        costs.append(t)
-        layers.append(nl)
-    return np.array(costs), np.array(layers)
+    return np.array(i.part_cost, dtype=np.float64), np.array(i.part_layers)
 
 
 if __name__ == "__main__":

@@ -83,6 +83,17 @@ int run_part(Interp& I, uint32_t p, uint64_t t, const uint32_t* stim, uint32_t* 
         for (uint32_t ln = 0; ln < 32; ln++)
           for (uint32_t c = 0; c < 4; c++) {
             uint32_t e = lv[(g * 32 + ln) * 4 + c];
+            if (mode == GEM_WM_DENSE16) {
+              for (uint32_t h = 0; h < 2; h++) {
+                uint32_t x = (e >> (16 * h)) & 0xFFFFu, word = GEM_LEAF16_WORD(x), rot = x & 31u;
+                uint32_t pos = 8 * g + 2 * c + h;
+                read[word] = 1;
+                uint32_t s = S[word];
+                uint32_t rs = rot ? ((s << rot) | (s >> (32 - rot))) : s;
+                val[0][(wp * 32 + ln) * 32 + pos] |= (uint8_t)((rs >> pos) & 1u);
+              }
+              continue;
+            }
             uint32_t word = GEM_LEAF_WORD(e), rot = GEM_LEAF_ROT(e);
             uint32_t pos = mode == GEM_WM_DENSE ? 4 * g + c : GEM_LEAF_POS(e);
             if (word >= GEM_MAX_STATE_WORDS) { g_err = "leaf word out of range"; return -1; }
