@@ -117,10 +117,38 @@ def workload_inputs(cfg: str, n_pi: int, cycles: int, streams, step: int):
     return np.stack(out)
 
 
+def cpu_baseline_lanes(eaig_path: str, n_pi: int, target_s: float = 12.0) -> dict:
+    """C5: the oracle's 64-lane batched mode, one 64-stream group per host thread."""
+    from concurrent.futures import ThreadPoolExecutor
+    from gen import stimulus_streams
+    from oracle import Oracle
+    o = Oracle(eaig_path)
+    nth = max(1, os.cpu_count() or 1)
+    o.lanes_reset(nth)
+    probe = 5
+    st = stimulus_streams("c5", n_pi, probe, range(64))
+    o.lanes_run(0, st, po=True)
+    rate = probe / max(o.last_seconds, 1e-9)           # cycles/s of one 64-lane group
+    cycles = int(max(probe, min(5000, rate * target_s)))
+    stims = [stimulus_streams("c5", n_pi, cycles, range(64 * g, 64 * g + 64)) for g in range(nth)]
+    o.lanes_reset(nth)
+    t0 = time.perf_counter()
+    with ThreadPoolExecutor(nth) as ex:
+        list(ex.map(lambda g: o.lanes_run(g, stims[g], po=True), range(nth)))
+    dt = time.perf_counter() - t0
+    v = 64 * nth * cycles / dt
+    return {"value": v, "unit": UNIT, "cores": nth, "kind": "oracle",
+            "sample": f"{64 * nth} of the 4096 C5 streams x {cycles} cycles (64-lane uint64 oracle, "
+                      f"{nth} threads, one 64-stream group each)",
+            "gate_evals_per_s": v * o.n_ands, "host_nproc": os.cpu_count(), "seconds": dt}
+
+
 def cpu_baseline(eaig_path: str, n_pi: int, cfg: str, target_s: float = 12.0) -> dict:
     """The oracle as it stands, single-threaded, on a bounded sample (host cores)."""
     from gen import stimulus
     from oracle import Oracle
+    if cfg == "c5":
+        return cpu_baseline_lanes(eaig_path, n_pi, target_s)
     o = Oracle(eaig_path)
     probe = 50
     st = stimulus("c3" if cfg == "c5" else cfg, n_pi, probe)
@@ -153,7 +181,7 @@ def run_reference(args):
     probe = 20
     o.run(stimulus("c3" if cfg == "c5" else cfg, n_pi, probe))
     rate = probe / max(o.last_seconds, 1e-9)
-    per_step = int(max(5, min(args.cycles, rate * 120.0 / max(1, args.steps + args.warmup))))
+    per_step = int(max(5, min(args.cycles or 1000, rate * 120.0 / max(1, args.steps + args.warmup))))
     o.reset()
     tot_c, tot_s = 0, 0.0
     for k in range(args.warmup + args.steps):
@@ -182,8 +210,10 @@ def main():
     ap.add_argument("--warmup", type=int, default=3)
     ap.add_argument("--impl", default="gem", choices=["gem", "reference"])
     ap.add_argument("--workload", default="c3", choices=["c1", "c2", "c3", "c4", "c5"])
-    ap.add_argument("--streams", type=int, default=0, help="streams per GPU (0 = 1, or 4096/N for c5)")
-    ap.add_argument("--cycles", type=int, default=1000, help="simulated cycles per step")
+    ap.add_argument("--streams", type=int, default=0,
+                    help="TOTAL stimulus streams over all GPUs (0 = 1 per GPU, or 4096 for c5)")
+    ap.add_argument("--cycles", type=int, default=0,
+                    help="simulated cycles per step (0 = 1000; 200 for c4; 20 for c5)")
     ap.add_argument("--no-cpu-baseline", action="store_true")
     ap.add_argument("--no-flush", action="store_true")
     ap.add_argument("--map-opts", default=None)
@@ -207,8 +237,11 @@ def main():
     from paper_conf_dac_guozwlr25_b200.isa import blob_info
     from tests.common import blob, eaig, MAP_OPTS
 
+    from paper_conf_dac_guozwlr25_b200.dist import gather_traces, shard_streams
     cfg = args.workload
-    S = args.streams or (max(1, 4096 // ws) if cfg == "c5" else 1)
+    total_streams = args.streams or (4096 if cfg == "c5" else ws)
+    s_start, S = shard_streams(total_streams, ws, rank)
+    scaling = "strong" if (args.streams or cfg == "c5") else "weak"
     opts = MAP_OPTS[cfg] if args.map_opts is None else args.map_opts
     # rank 0 maps (cached on disk), others wait
     if rank == 0:
@@ -220,15 +253,14 @@ def main():
     info = blob_info(b)
     stream = torch.cuda.current_stream(dev)
     sim = gem.Simulator(b, device=dev.index, n_streams=S, cuda_stream=stream.cuda_stream, flags=gem.GEM_F_ASYNC)
-    C = args.cycles
-    gstreams = list(range(rank * S, rank * S + S))
+    C = args.cycles or {"c4": 200, "c5": 20}.get(cfg, 1000)
+    gstreams = list(range(s_start, s_start + S))
     # inputs for (warmup + steps), pre-generated on the host, uploaded per step
     n_steps = args.warmup + args.steps
     host_in = [workload_inputs(cfg, info.n_pi, C, gstreams, k) for k in range(min(n_steps, 4))]
     pi_words = sim.pi_words
     dev_in = [torch.from_numpy(x.view(np.int32)).to(dev) for x in host_in]
     po_dev = torch.empty((S, C, sim.po_words), dtype=torch.int32, device=dev)
-    gather_buf = [torch.empty_like(po_dev) for _ in range(ws)] if (ws > 1 and rank == 0) else None
     flush = torch.empty(512 * 1024 * 1024 // 4, dtype=torch.int32, device=dev)
 
     def one_step(k, timed_events=None):
@@ -238,7 +270,7 @@ def main():
         sim.step(C)
         sim.read_outputs_device(po_dev, C)
         if ws > 1:
-            dist.gather(po_dev, gather_buf, dst=0)
+            gather_traces(po_dev, total_streams)   # NCCL gather of the PO traces to rank 0
         if timed_events is not None:
             timed_events[1].record(stream)
 
@@ -271,7 +303,7 @@ def main():
     if ws > 1:
         dist.all_reduce(t, op=dist.ReduceOp.MAX)
     tot_ms = float(t.item())
-    total_stream_cycles = ws * S * C * args.steps
+    total_stream_cycles = total_streams * C * args.steps
     value = total_stream_cycles / (tot_ms / 1e3)
 
     # ---- e2e through the public API with HOST buffers (pinned), copies inside the timed region
@@ -295,7 +327,7 @@ def main():
     if ws > 1:
         dist.all_reduce(te, op=dist.ReduceOp.MAX)
     e2e_s = float(te.item())
-    e2e = {"value": ws * S * C * e2e_steps / e2e_s, "unit": UNIT,
+    e2e = {"value": total_streams * C * e2e_steps / e2e_s, "unit": UNIT,
            "h2d_bytes_per_step": int(S * C * pi_words * 4), "d2h_bytes_per_step": int(S * C * sim.po_words * 4),
            "api": "gem_set_inputs(host) + gem_step + gem_read_outputs(host), synchronous C ABI"}
     sim_h.close()
@@ -307,7 +339,7 @@ def main():
         n_sms = torch.cuda.get_device_properties(dev).multi_processor_count
         peak_lop3 = n_sms * 64 * float(peaks.get("sm_max_mhz", 1965.0)) * 1e6
         hz_kernel = C / (kern_last / 1e3)
-        achieved_lop3 = info.n_and / 16.0 * hz_kernel * S
+        achieved_lop3 = info.n_and / 16.0 * hz_kernel * S   # this rank's kernel (per GPU)
         roof = {"bound": "alu", "achieved": achieved_lop3 / 1e12, "peak": peak_lop3 / 1e12, "unit": "TLOP3/s",
                 "frac": achieved_lop3 / peak_lop3, "traffic": None,
                 "kernel": "gem_step_kernel", "kernel_ms_per_step": kern_last,
@@ -321,10 +353,11 @@ def main():
             cpu = cpu_baseline(eaig(cfg), info.n_pi, cfg)
         line = {"metric": METRIC, "value": value, "unit": UNIT, "n_gpus": ws, "steps": args.steps,
                 "warmup": args.warmup, "ms_per_step": tot_ms / args.steps, "higher_is_better": True,
-                "scaling": "weak", "vs_baseline": None, "dtype": "u32", "data": "synthetic",
+                "scaling": scaling, "vs_baseline": None, "dtype": "u32", "data": "synthetic",
                 "config": {"workload": f"{cfg}: synthetic CPU-core-shaped netlist, {info.n_and} live ANDs, "
                                        f"{info.n_flops} flops, {info.n_rams} RAM blocks" if cfg == "c3" else cfg,
-                           "streams_per_gpu": S, "cycles_per_step": C, "parts": info.n_parts,
+                           "streams_total": total_streams, "streams_per_gpu": S, "cycles_per_step": C,
+                           "parts": info.n_parts, "stream_group": sim.info["group"],
                            "stages": info.n_stages, "max_layers": info.max_layers, "levels": info.max_levels,
                            "replication": round(info.replication, 3), "program_bytes": info.program_bytes,
                            "grid": sim.info["grid"], "l2": "flushed between timed steps (512 MB write)"
