@@ -66,6 +66,7 @@ typedef struct {
   uint32_t resident;     /* 1 = every CTA's programs live in its shared memory */
   uint32_t ring_slots;   /* else: TMA ring depth used to stream program chunks */
   uint32_t group;        /* streams per work item (program chunks reused across them) */
+  uint32_t lanes;        /* 1 = stream-sliced lane mode (32 streams per lane word)  */
   uint64_t n_and;                          /* live 2-input ANDs (gate evals/cycle) */
   uint64_t n_and_mapped;                   /* with RepCut replication              */
   uint64_t program_bytes;

@@ -101,13 +101,16 @@ enum {
   GH_OFF_PROG, GH_PROG_WORDS_LO, GH_PROG_WORDS_HI, GH_MAX_LEVELS, GH_TOTAL_WRITEOUTS,
   GH_MAX_OUT, GH_TOTAL_WORDS_LO, GH_TOTAL_WORDS_HI, GH_SLOTS_USED_LO, GH_SLOTS_USED_HI,
   GH_MAX_CHUNK_WORDS, GH_MAX_PROG_WORDS,
+  GH_HAS_LANES, GH_OFF_LANE_PROG, GH_LANE_PROG_WORDS_LO, GH_LANE_PROG_WORDS_HI, GH_LANE_MAX_CHUNK_WORDS,
+  GH_LANE_MAX_WORDS, GH_MAX_RAMS_PART,
   GH_N_WORDS = 64
 };
 
-/* part table entry (8 words) */
+/* part table entry */
 enum {
   GP_STAGE = 0, GP_PROG_OFF, GP_PROG_LEN, GP_N_LAYERS, GP_CHUNK0, GP_MAX_CHUNK, GP_CHUNK1, GP_CHUNK2,
-  GP_COST, GP_R9, GP_R10, GP_R11, GP_WORDS = 12
+  GP_COST, GP_LANE_OFF, GP_LANE_LEN, GP_LANE_CHUNK0, GP_LANE_CHUNK1, GP_LANE_CHUNK2, GP_LANE_WORDS, GP_R15,
+  GP_WORDS = 16
 };
 /* GP_COST: mapper's estimate of one cycle of the partition in SM clocks (used by
  * the runtime's longest-processing-time work-list scheduling). */
@@ -151,3 +154,47 @@ enum {
 /* output section: dst gid [n_out_pad] then src [n_out][32]
  * RAM section: per owned RAM 4 words {ram_id, 0, 0, 0}; its ports are staged by
  * outputs with region GEM_R_RAMP index = local*4 + port.                       */
+
+/* ---------------------------------------------------------------------------
+ * Lane mode (stream-sliced execution of the same placement, optional: mapper
+ * option lanes=1).  For a group of 32 independent stimulus streams every
+ * signal is one 32-bit "lane word" (bit s = stream s), so one pass over a
+ * layer evaluates it for 32 streams: leaves are whole lane words (no bit
+ * extraction) and each gate slot is two LOP3 on words.  Same layers, same
+ * slots, same packed constants as the bit-packed program; only signal storage
+ * differs (one lane word per live signal, allocated by liveness).
+ *
+ * Global lane layout (per 32-stream group g, n_groups words per row):
+ *   Q_lane[2][q_words*32][G], RD_lane[2][n_rams*32][G], CUT_lane[cut_words*32][G],
+ *   PI_lane[cycle][pi_words*32][G], PO_lane[cycle][po_words*32][G]
+ * gid_l = region << 24 | bit index (RAMP: (ram_local*4 + port)*32 + bit).
+ *
+ * Lane partition program: header (16) | chunk table | layers | out+ram | gread
+ *   (chunks: 0 = header + table, 1..L = layers, L+1 = out+ram; the gread list
+ *   is read from global memory)
+ *   gread: uint2 {gid_l, dst lane word}
+ *   layer: header (16 words) {size, flags, topc, top_mask | top_base << 8, woff[8], 0...}
+ *          warp record (GEM_LWREC_WORDS words):
+ *            [0..5)    wxa, wxb, wob, wmask, wbase       (levels 6-10)
+ *            [8..136)  lane constants uint4 {xa, xb, ob, mask}  (levels 1-5)
+ *            [136..648) leaves: [4 groups][32 lanes] uint4 (32 u16 lane words
+ *                       per lane, entry 8g+2k low half, 8g+2k+1 high half)
+ *            [648..680) per-lane write-out base word
+ *   Write-outs: a unit (thread / warp / top) stores the slots whose bits are set
+ *   in its mask, in slot-bit order, to consecutive lane words from its base:
+ *   slot b -> base + popc(mask & ((1 << b) - 1)).
+ *   out:   uint2 {dst gid_l, src lane word | GEM_OUT_INV}
+ *   ram:   4 words per owned RAM {ram_id, 0, 0, 0}
+ * Lane word 0 is the constant 0.                                            */
+#define GEM_LANE_MAGIC 0x454E414Cu  /* "LANE" */
+#define GEM_LANE_STREAMS 32
+enum {
+  LPH_MAGIC = 0, LPH_N_GREAD, LPH_N_LAYERS, LPH_N_OUT, LPH_N_RAM, LPH_LANE_WORDS, LPH_OFF_GREAD,
+  LPH_OFF_LAYERS, LPH_OFF_OUT, LPH_OFF_RAM, LPH_OFF_CHUNKS, LPH_N_CHUNKS, LPH_R12, LPH_R13, LPH_R14,
+  LPH_R15, LPH_WORDS = 16
+};
+enum { LLH_WORDS_ = 0, LLH_FLAGS, LLH_TOPC, LLH_TOPWO, LLH_WOFF0 /* ..+7 */, LLH_WORDS = 16 };
+#define GEM_LWREC_HDR 8
+#define GEM_LWREC_LEAVES (GEM_LWREC_HDR + 128)
+#define GEM_LWREC_BASE (GEM_LWREC_HDR + 128 + 512)
+#define GEM_LWREC_WORDS (GEM_LWREC_BASE + 32)

@@ -1,0 +1,386 @@
+// gem_lanes.cuh -- lane mode: stream-sliced execution of the same VLIW
+// placement for batched stimulus streams.
+// Included by gem_runtime.cu (shares KParams, the TMA ring and mbarriers).
+//
+// Every signal of a 32-stream group is one 32-bit lane word (bit s = stream s),
+// so one pass over a boomerang layer evaluates it for 32
+// streams: a leaf is one shared-memory load of a whole word (no bit
+// extraction) and each gate slot is (A ^ XA) & ((B ^ XB) | OB) on words, with
+// XA/XB/OB the slot's constants sign-extended to masks.  The program
+// (gem_isa.h "Lane mode") comes from the same placement as the bit-packed one.
+
+// lane global-state indexing, group-major rows (a work item's signals are
+// contiguous): X[buf][group][bit]
+struct LaneIdx {
+  uint32_t G;
+  __device__ __forceinline__ size_t q(uint32_t buf, uint32_t bits, uint32_t b, uint32_t g) const {
+    return ((size_t)buf * G + g) * bits + b;
+  }
+};
+
+// one lane layer's per-thread records (loaded before the previous layer's barrier)
+struct LaneRegs {
+  uint4 e[4];                 // 32 u16 leaf lane words
+  uint4 lc;                   // xa, xb, ob, write mask (levels 1-5)
+  uint32_t base;              // write-out base lane word
+  uint4 wc;                   // wxa, wxb, wob, wmask (levels 6-10)
+  uint32_t wbase;
+  uint32_t flags, topc, topwo;
+};
+
+__device__ __forceinline__ void load_lane_layer(const uint32_t* L, LaneRegs& R) {
+  const uint32_t lane = threadIdx.x & 31, warp = threadIdx.x >> 5;
+  const uint4 h = *reinterpret_cast<const uint4*>(L);
+  R.flags = h.y;
+  R.topc = h.z;
+  R.topwo = h.w;
+  if ((R.flags >> warp) & 1u) {
+    const uint32_t* rec = L + L[LLH_WOFF0 + warp];
+    R.wc = *reinterpret_cast<const uint4*>(rec);
+    R.wbase = rec[4];
+    R.lc = *(reinterpret_cast<const uint4*>(rec + GEM_LWREC_HDR) + lane);
+    const uint4* lv = reinterpret_cast<const uint4*>(rec + GEM_LWREC_LEAVES) + lane;
+#pragma unroll
+    for (uint32_t g = 0; g < 4; g++) R.e[g] = lv[g * 32];
+    R.base = rec[GEM_LWREC_BASE + lane];
+  }
+}
+
+// slot (A ^ XA) & ((B ^ XB) | OB) with the masks taken from bit b of the constants
+__device__ __forceinline__ uint32_t lslot(uint32_t A, uint32_t B, uint32_t xa, uint32_t xb, uint32_t ob, uint32_t b) {
+  const uint32_t XA = (uint32_t)((int32_t)(xa << (31u - b)) >> 31);
+  const uint32_t XB = (uint32_t)((int32_t)(xb << (31u - b)) >> 31);
+  const uint32_t OB = (uint32_t)((int32_t)(ob << (31u - b)) >> 31);
+  return (A ^ XA) & ((B ^ XB) | OB);
+}
+
+__device__ __forceinline__ void lane_wo(uint32_t s_base, uint32_t mask, uint32_t base, uint32_t b, uint32_t v) {
+  if ((mask >> b) & 1u) sts(s_base + 4u * (base + __popc(mask & ((1u << b) - 1u))), v);
+}
+
+// Rows a3-a5 of one layer for one 32-stream group.  topv: 8 warp results + counter.
+__device__ __forceinline__ void exec_lane_layer(const LaneRegs& R, uint32_t s_base, uint32_t* topv) {
+  const uint32_t lane = threadIdx.x & 31, warp = threadIdx.x >> 5;
+  const bool uses_top = (R.flags & GEM_LF_USES_TOP) != 0;
+  if ((R.flags >> warp) & 1u) {
+    const uint32_t xa = R.lc.x, xb = R.lc.y, ob = R.lc.z, mask = R.lc.w;
+    uint32_t v[32];
+    const uint32_t q8[4][4] = {{R.e[0].x, R.e[0].y, R.e[0].z, R.e[0].w}, {R.e[1].x, R.e[1].y, R.e[1].z, R.e[1].w},
+                               {R.e[2].x, R.e[2].y, R.e[2].z, R.e[2].w}, {R.e[3].x, R.e[3].y, R.e[3].z, R.e[3].w}};
+#pragma unroll
+    for (uint32_t g = 0; g < 4; g++)
+#pragma unroll
+      for (uint32_t k = 0; k < 4; k++) {
+        v[8 * g + 2 * k] = lds(s_base + 4u * (q8[g][k] & 0xFFFFu));
+        v[8 * g + 2 * k + 1] = lds(s_base + 4u * (q8[g][k] >> 16));
+      }
+    // levels 1-5 inside the thread; write-outs as each level completes
+#pragma unroll
+    for (uint32_t q = 0; q < 16; q++) {
+      v[q] = lslot(v[q], v[q + 16], xa, xb, ob, q);
+      lane_wo(s_base, mask, R.base, q, v[q]);
+    }
+#pragma unroll
+    for (uint32_t q = 0; q < 8; q++) {
+      v[q] = lslot(v[q], v[q + 8], xa, xb, ob, 16 + q);
+      lane_wo(s_base, mask, R.base, 16 + q, v[q]);
+    }
+#pragma unroll
+    for (uint32_t q = 0; q < 4; q++) {
+      v[q] = lslot(v[q], v[q + 4], xa, xb, ob, 24 + q);
+      lane_wo(s_base, mask, R.base, 24 + q, v[q]);
+    }
+#pragma unroll
+    for (uint32_t q = 0; q < 2; q++) {
+      v[q] = lslot(v[q], v[q + 2], xa, xb, ob, 28 + q);
+      lane_wo(s_base, mask, R.base, 28 + q, v[q]);
+    }
+    uint32_t x = lslot(v[0], v[1], xa, xb, ob, 30);
+    lane_wo(s_base, mask, R.base, 30, x);
+    // levels 6-10 across the warp: slot q of a level lives in lane q
+    const uint32_t wxa = R.wc.x, wxb = R.wc.y, wob = R.wc.z, wmask = R.wc.w;
+    const uint32_t offs[5] = {0, 16, 24, 28, 30};
+#pragma unroll
+    for (uint32_t k = 0; k < 5; k++) {
+      const uint32_t half = 16u >> k;
+      const uint32_t y = __shfl_down_sync(0xFFFFFFFFu, x, half);
+      const uint32_t b = offs[k] + (lane & (half - 1u));
+      x = lslot(x, y, wxa, wxb, wob, b);
+      if (lane < half) lane_wo(s_base, wmask, R.wbase, b, x);
+    }
+    if (uses_top && lane == 0) topv[warp] = x;
+  } else if (uses_top && lane == 0) {
+    topv[warp] = 0u;
+  }
+  // levels 11-13: the last warp to arrive folds the 8 warp words
+  if (uses_top && lane == 0) {
+    __threadfence_block();
+    if (atomicAdd(&topv[8], 1u) == GEM_WARPS - 1) {
+      __threadfence_block();
+      volatile uint32_t* tv = topv;
+      const uint32_t xa = R.topc & 0xFFu, xb = (R.topc >> 8) & 0xFFu, ob = (R.topc >> 16) & 0xFFu;
+      const uint32_t tm = R.topwo & 0x7Fu, tb = R.topwo >> 8;
+      uint32_t t11[4];
+#pragma unroll
+      for (uint32_t q = 0; q < 4; q++) {
+        t11[q] = lslot(tv[q], tv[q + 4], xa, xb, ob, q);
+        lane_wo(s_base, tm, tb, q, t11[q]);
+      }
+      uint32_t t12[2];
+#pragma unroll
+      for (uint32_t q = 0; q < 2; q++) {
+        t12[q] = lslot(t11[q], t11[q + 2], xa, xb, ob, 4 + q);
+        lane_wo(s_base, tm, tb, 4 + q, t12[q]);
+      }
+      lane_wo(s_base, tm, tb, 6, lslot(t12[0], t12[1], xa, xb, ob, 6));
+      topv[8] = 0u;
+    }
+  }
+}
+
+// One work item: partition p for 32-stream group g (streams 32g .. 32g+nvalid-1).
+__device__ void run_lane_partition(const KParams& kp, ProgSrc& ps, uint32_t* S, uint32_t* ramp, uint32_t* topv,
+                                   uint32_t p, uint32_t g0, uint32_t ng, uint32_t c, uint32_t cur, uint32_t nxt) {
+  const uint32_t tid = threadIdx.x;
+  const uint32_t s_base = smem_u32(S);
+  const uint32_t LW = kp.state_words;   // lane words per group
+  const LaneIdx X{kp.n_groups};
+  const uint32_t* gprog = kp.lprog + __ldg(kp.parts + p * GP_WORDS + GP_LANE_OFF);
+  uint32_t next_chunk = prologue_count_lane(kp, ps, p), next_off = 0;
+  next_off = __ldg(kp.parts + p * GP_WORDS + GP_LANE_CHUNK0);
+  if (next_chunk > 1) next_off += __ldg(kp.parts + p * GP_WORDS + GP_LANE_CHUNK1);
+  if (next_chunk > 2) next_off += __ldg(kp.parts + p * GP_WORDS + GP_LANE_CHUNK2);
+  const uint32_t* C0 = ring_wait(ps);
+  const uint4 h0 = *reinterpret_cast<const uint4*>(C0);
+  const uint4 h1 = *(reinterpret_cast<const uint4*>(C0) + 1);
+  const uint4 h2 = *(reinterpret_cast<const uint4*>(C0) + 2);
+  const uint32_t n_gread = h0.y, n_layers = h0.z, n_out = h0.w;
+  const uint32_t n_ram = h1.x, off_gread = h1.z, off_layers = h1.w;
+  const uint32_t off_out = h2.x, off_ram = h2.y, off_chunks = h2.z, n_chunks = h2.w;
+  for (uint32_t k = tid; k < n_chunks; k += GEM_THREADS) ps.ctab[k] = C0[off_chunks + k];
+  // chunk 0 = header + chunk table; the gread list (after the last chunk) is
+  // read straight from global memory
+  auto refill = [&]() {
+    while (next_chunk < n_chunks && ps.seq_issue - ps.seq_free < ps.R) {
+      const uint32_t words = ps.ctab[next_chunk];
+      ring_issue(ps, gprog + next_off, words);
+      next_off += words;
+      next_chunk++;
+    }
+  };
+  // ---- a2: input ports (once per cycle) for the 32 streams of the group
+  const uint2* gr = reinterpret_cast<const uint2*>(gprog + off_gread);
+#pragma unroll 4
+  for (uint32_t k = tid; k < n_gread; k += GEM_THREADS) {
+    const uint2 e = __ldg(gr + k);
+    const uint32_t reg = e.x >> 24, b = e.x & 0xFFFFFFu;
+    for (uint32_t j = 0; j < ng; j++) {
+      const uint32_t g = g0 + j;
+      uint32_t v;
+      if (reg == GEM_R_PI) v = __ldg(kp.pi_lane + X.q(kp.in_base + c, kp.pi_words * 32, b, g));
+      else if (reg == GEM_R_Q) v = __ldcg(kp.q + X.q(cur, kp.q_words * 32, b, g));
+      else if (reg == GEM_R_RD) v = __ldcg(kp.rd + X.q(cur, kp.n_rams * 32, b, g));
+      else v = __ldcg(kp.cut + X.q(0, kp.cut_words * 32, b, g));
+      sts(s_base + 4u * (j * LW + e.y), v);
+    }
+  }
+  if (tid < ng) S[tid * LW] = 0u;
+  LaneRegs R;
+  if (n_layers) load_lane_layer(ring_wait(ps), R);
+  __syncthreads();
+  ps.seq_free += n_layers ? 2 : 1;
+  refill();
+  for (uint32_t l = 0; l < n_layers; l++) {
+    for (uint32_t j = 0; j < ng; j++) exec_lane_layer(R, s_base + 4u * j * LW, topv + 16 * j);
+    if (l + 1 < n_layers) load_lane_layer(ring_wait(ps), R);
+    __syncthreads();
+    if (l + 1 < n_layers) ps.seq_free++;
+    refill();
+  }
+  // ---- a6: endpoint commit: one lane word per endpoint bit
+  const uint32_t* od = ring_wait(ps);
+  const uint2* oe = reinterpret_cast<const uint2*>(od);
+  for (uint32_t jj = tid; jj < n_out * ng; jj += GEM_THREADS) {
+    const uint32_t j = jj / n_out, o = jj - j * n_out, g = g0 + j;
+    const uint2 e = oe[o];
+    const uint32_t v = lds(s_base + 4u * (j * LW + (e.y & 0xFFFFu))) ^ ((e.y >> 31) ? 0xFFFFFFFFu : 0u);
+    const uint32_t reg = e.x >> 24, b = e.x & 0xFFFFFFu;
+    if (reg == GEM_R_Q) __stcg(kp.q + X.q(nxt, kp.q_words * 32, b, g), v);
+    else if (reg == GEM_R_PO) __stcg(kp.po_lane + X.q(c, kp.po_words * 32, b, g), v);
+    else if (reg == GEM_R_CUT) __stcg(kp.cut + X.q(0, kp.cut_words * 32, b, g), v);
+    else ramp[j * kp.ramp_words + b] = v;
+  }
+  // ---- a7: RAM blocks: one warp per RAM, lane s = stream 32g+s (read-first, per-bit write)
+  if (n_ram) {
+    __syncthreads();
+    const uint32_t* rr = od + (off_ram - off_out);
+    const uint32_t lane = tid & 31;
+    for (uint32_t jr = tid >> 5; jr < n_ram * ng; jr += GEM_WARPS) {
+      const uint32_t j = jr / n_ram, r = jr - j * n_ram, g = g0 + j;
+      const uint32_t nvalid = min(32u, kp.n_streams - 32u * g);
+      const uint32_t id = rr[4 * r];
+      const uint32_t* rp = ramp + j * kp.ramp_words + r * 128;
+      uint32_t ra = 0, wa = 0, wd = 0, be = 0;
+#pragma unroll
+      for (uint32_t k = 0; k < 13; k++) {
+        ra |= ((rp[k] >> lane) & 1u) << k;
+        wa |= ((rp[32 + k] >> lane) & 1u) << k;
+      }
+#pragma unroll 8
+      for (uint32_t k = 0; k < 32; k++) {
+        wd |= ((rp[64 + k] >> lane) & 1u) << k;
+        be |= ((rp[96 + k] >> lane) & 1u) << k;
+      }
+      uint32_t old = 0;
+      if (lane < nvalid) {
+        uint32_t* M = kp.mem + ((size_t)(32u * g + lane) * kp.n_rams + id) * GEM_RAM_WORDS;
+        old = __ldcg(M + ra);
+        const uint32_t cw = __ldcg(M + wa);
+        __stcg(M + wa, (cw & ~be) | (wd & be));
+      }
+      // transpose the 32 read words into 32 lane words
+#pragma unroll 4
+      for (uint32_t k = 0; k < 32; k++) {
+        const uint32_t w = __ballot_sync(0xFFFFFFFFu, (old >> k) & 1u);
+        if (lane == k) __stcg(kp.rd + X.q(nxt, kp.n_rams * 32, id * 32 + k, g), w);
+      }
+    }
+  }
+  __syncthreads();
+  ps.seq_free = ps.seq_issue;
+}
+
+// Parity instruments in lane mode: flop digest / trace from the lane words.
+__device__ void record_state_lane(const KParams& kp, uint32_t c, uint32_t buf) {
+  const LaneIdx X{kp.n_groups};
+  const uint32_t total = kp.n_streams * kp.q_ext_words;
+  for (uint32_t i = blockIdx.x * blockDim.x + threadIdx.x; i < total; i += gridDim.x * blockDim.x) {
+    const uint32_t st = i / kp.q_ext_words, w = i % kp.q_ext_words, g = st >> 5, s = st & 31;
+    uint32_t v = 0;
+    for (uint32_t b = 0; b < 32; b++) {
+      const uint32_t e = w * 32 + b;
+      if (e >= kp.n_flops) break;
+      const uint32_t in = __ldg(kp.q_int_of_ext + e);
+      v |= ((__ldcg(kp.q + X.q(buf, kp.q_words * 32, in, g)) >> s) & 1u) << b;
+    }
+    if (kp.flags & GEM_F_TRACE_STATE) kp.q_trace[((size_t)st * kp.out_cap + c) * kp.q_ext_words + w] = v;
+    if (kp.flags & GEM_F_DIGEST) {
+      const uint32_t r = w & 63u;
+      const unsigned long long x = (unsigned long long)v;
+      const unsigned long long rot = r ? ((x << r) | (x >> (64 - r))) : x;
+      atomicAdd(kp.digest + (size_t)st * kp.out_cap + c, rot * (2ull * w + 1ull));
+    }
+  }
+}
+
+__global__ void __launch_bounds__(GEM_THREADS, 1) gem_lane_kernel(const KParams kp) {
+  extern __shared__ __align__(16) uint32_t smem[];
+  // layout: S[lane_words] | area (ring) | ctab[256] | ramp[ram_words] | topv[16] | mbar[8 x u64]
+  uint32_t* S = smem;                                   // [group][lane words]
+  uint32_t* area = S + kp.group * kp.state_words;
+  uint32_t* ctab = area + kp.area_words;
+  uint32_t* ramp = ctab + GEM_MAX_CHUNKS;               // [group][ramp_words]
+  uint32_t* topv = ramp + kp.group * kp.ramp_words;     // [group][16]
+  uint64_t* mbar = reinterpret_cast<uint64_t*>(topv + 16 * kp.group);
+  const uint32_t tid = threadIdx.x;
+  const uint32_t G = gridDim.x, B = blockIdx.x;
+  auto wl_begin = [&](uint32_t s) { return __ldg(kp.wl_off + s * (G + 1) + B); };
+  auto wl_end = [&](uint32_t s) { return __ldg(kp.wl_off + s * (G + 1) + B + 1); };
+  for (uint32_t k = tid; k < 16 * kp.group; k += GEM_THREADS) topv[k] = 0u;
+  if (tid == 0) {
+    for (uint32_t k = 0; k <= GEM_RING_MAX; k++) mbar_init(mbar + k, 1);
+    fence_mbar_init();
+  }
+  __syncthreads();
+  ProgSrc ps;
+  ps.mbar = mbar;
+  ps.area = area;
+  ps.ctab = ctab;
+  ps.resident = false;
+  ps.n_res = 0;
+  ps.res_p = nullptr;
+  ps.res_off = nullptr;
+  ps.slot_words = kp.slot_words;
+  ps.R = kp.ring_slots;
+  ps.seq_issue = ps.seq_wait = ps.seq_free = 0;
+  auto first_item = [&]() -> uint32_t {
+    for (uint32_t s = 0; s < kp.n_stages; s++)
+      if (wl_begin(s) < wl_end(s)) return wl_begin(s);
+    return ~0u;
+  };
+  if (kp.ncycles) {
+    const uint32_t k0 = first_item();
+    if (k0 != ~0u) issue_prologue_lane(kp, ps, __ldg(&kp.wl_items[k0].x));
+  }
+  unsigned long long bar_target = 0;
+  const bool instr = (kp.flags & (GEM_F_TRACE_STATE | GEM_F_DIGEST)) != 0;
+  for (uint32_t c = 0; c < kp.ncycles; c++) {
+    const uint64_t t = kp.t0 + c;
+    const uint32_t cur = (uint32_t)(t & 1u), nxt = cur ^ 1u;
+    if (instr && c > 0) record_state_lane(kp, c - 1, cur);
+    for (uint32_t s = 0; s < kp.n_stages; s++) {
+      const uint32_t kb = wl_begin(s), ke = wl_end(s);
+      for (uint32_t k = kb; k < ke; k++) {
+        const uint2 it = __ldg(&kp.wl_items[k]);
+        const uint32_t g0 = it.y >> 5;
+        run_lane_partition(kp, ps, S, ramp, topv, it.x, g0, min(kp.group, kp.n_groups - g0), c, cur, nxt);
+        uint32_t nk = ~0u;
+        if (k + 1 < ke) nk = k + 1;
+        for (uint32_t s2 = s + 1; nk == ~0u && s2 < kp.n_stages; s2++)
+          if (wl_begin(s2) < wl_end(s2)) nk = wl_begin(s2);
+        if (nk == ~0u && c + 1 < kp.ncycles) nk = first_item();
+        if (nk != ~0u) issue_prologue_lane(kp, ps, __ldg(&kp.wl_items[nk].x));
+      }
+      grid_sync(kp, bar_target);
+    }
+  }
+  if (instr) record_state_lane(kp, kp.ncycles - 1, (uint32_t)((kp.t0 + kp.ncycles) & 1u));
+}
+
+// ---- 32x32 bit transposes between per-stream words and lane words (one warp per tile)
+// stream-major in[stream][row_stride...]: word w of stream s at in[s * s_stride + row * r_stride + w]
+__global__ void to_lanes_kernel(const uint32_t* __restrict__ in, uint32_t* __restrict__ out, uint32_t n_streams,
+                                uint32_t rows, uint32_t words, uint64_t s_stride, uint64_t r_stride,
+                                uint32_t n_groups, uint64_t out_row_base) {
+  // out[out_row_base + row][g][w*32 + k] = bit k of word w, lane s of group g
+  const uint32_t lane = threadIdx.x & 31;
+  const uint64_t warps = (uint64_t)rows * n_groups * words;
+  for (uint64_t wi = ((uint64_t)blockIdx.x * blockDim.x + threadIdx.x) >> 5; wi < warps;
+       wi += ((uint64_t)gridDim.x * blockDim.x) >> 5) {
+    const uint32_t w = (uint32_t)(wi % words);
+    const uint32_t g = (uint32_t)((wi / words) % n_groups);
+    const uint64_t row = wi / ((uint64_t)words * n_groups);
+    const uint32_t st = g * 32 + lane;
+    const uint32_t x = st < n_streams ? in[st * s_stride + row * r_stride + w] : 0u;
+    uint32_t mine = 0;
+#pragma unroll
+    for (uint32_t k = 0; k < 32; k++) {
+      const uint32_t b = __ballot_sync(0xFFFFFFFFu, (x >> k) & 1u);
+      if (lane == k) mine = b;
+    }
+    out[((out_row_base + row) * n_groups + g) * words * 32 + w * 32 + lane] = mine;
+  }
+}
+
+__global__ void from_lanes_kernel(const uint32_t* __restrict__ in, uint32_t* __restrict__ out, uint32_t n_streams,
+                                  uint32_t rows, uint32_t words, uint64_t s_stride, uint64_t r_stride,
+                                  uint32_t n_groups) {
+  // inverse of to_lanes_kernel (row base 0)
+  const uint32_t lane = threadIdx.x & 31;
+  const uint64_t warps = (uint64_t)rows * n_groups * words;
+  for (uint64_t wi = ((uint64_t)blockIdx.x * blockDim.x + threadIdx.x) >> 5; wi < warps;
+       wi += ((uint64_t)gridDim.x * blockDim.x) >> 5) {
+    const uint32_t w = (uint32_t)(wi % words);
+    const uint32_t g = (uint32_t)((wi / words) % n_groups);
+    const uint64_t row = wi / ((uint64_t)words * n_groups);
+    const uint32_t y = in[(row * n_groups + g) * words * 32 + w * 32 + lane];
+    uint32_t mine = 0;
+#pragma unroll
+    for (uint32_t s = 0; s < 32; s++) {
+      const uint32_t b = __ballot_sync(0xFFFFFFFFu, (y >> s) & 1u);
+      if (lane == s) mine = b;
+    }
+    const uint32_t st = g * 32 + lane;
+    if (st < n_streams) out[st * s_stride + row * r_stride + w] = mine;
+  }
+}

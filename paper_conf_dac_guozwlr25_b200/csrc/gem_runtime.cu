@@ -57,6 +57,11 @@ struct KParams {
   unsigned long long* prof;   // GEM_F_PROFILE: [prof_cycles][grid][8] clock64 stamps
   uint32_t prof_cycles;
   uint32_t group;                        // streams per work item (stream states in smem)
+  // lane mode
+  const uint32_t* __restrict__ lprog;    // lane programs
+  const uint32_t* __restrict__ pi_lane;  // [in_cap][pi_words*32][n_groups]
+  uint32_t* po_lane;                     // [out_cap][po_words*32][n_groups]
+  uint32_t n_groups, ramp_words;
   unsigned long long* fprof;             // debug builds (GEM_FINE_PROF) only
   const uint32_t* __restrict__ wl_off;   // [n_stages][grid+1] CSR offsets into wl_items
   const uint2* __restrict__ wl_items;    // {partition, stream} per work item
@@ -622,6 +627,26 @@ __global__ void __launch_bounds__(GEM_THREADS, 2) gem_step_kernel(const KParams 
   if (instr) record_state(kp, kp.ncycles - 1, (uint32_t)((kp.t0 + kp.ncycles) & 1u));
 }
 
+// ---- lane-mode prologue helpers (same protocol as issue_prologue, lane fields)
+__device__ __forceinline__ uint32_t prologue_count_lane(const KParams& kp, const ProgSrc& ps, uint32_t p) {
+  const uint32_t nch = __ldg(kp.parts + p * GP_WORDS + GP_N_LAYERS) + 2;
+  return min(min(ps.R, 3u), nch);
+}
+__device__ __forceinline__ void issue_prologue_lane(const KParams& kp, ProgSrc& ps, uint32_t p) {
+  const uint32_t* g = kp.lprog + __ldg(kp.parts + p * GP_WORDS + GP_LANE_OFF);
+  const uint32_t k = prologue_count_lane(kp, ps, p);
+  const uint32_t sz[3] = {__ldg(kp.parts + p * GP_WORDS + GP_LANE_CHUNK0),
+                          __ldg(kp.parts + p * GP_WORDS + GP_LANE_CHUNK1),
+                          __ldg(kp.parts + p * GP_WORDS + GP_LANE_CHUNK2)};
+  uint32_t off = 0;
+  for (uint32_t i = 0; i < k; i++) {
+    ring_issue(ps, g + off, sz[i]);
+    off += sz[i];
+  }
+}
+
+#include "gem_lanes.cuh"
+
 // external <-> internal layout conversion kernels
 // out[st][row][ext_w] = gather of 32 internal bits via int_of_ext
 __global__ void unpermute_kernel(const uint32_t* __restrict__ in, uint32_t* __restrict__ out,
@@ -681,6 +706,9 @@ struct gem_sim {
   uint64_t n_and = 0, n_and_mapped = 0, program_bytes = 0;
   uint32_t max_items = 0;
   uint32_t area_words = 0, slot_words = 0, ring_slots = 0, resident = 0, group = 1;
+  // lane mode (stream-sliced, >= 32 streams and a blob with lane programs)
+  uint32_t lanes = 0, n_groups = 0, lane_words = 0, lane_max_chunk = 0, ramp_words = 0, lane_groups = 1;
+  uint32_t *d_lprog = nullptr, *d_pi_lane = nullptr, *d_po_lane = nullptr;
   std::vector<uint32_t> h_parts, h_stage;
   // device buffers
   uint32_t *d_prog = nullptr, *d_parts = nullptr, *d_stage = nullptr;
@@ -737,6 +765,11 @@ static int ensure_out(gem_sim* sim, uint32_t ncycles) {
   sim->d_po = nullptr; sim->d_qtrace = nullptr; sim->d_digest = nullptr;
   sim->out_cap = 0;
   CK(dalloc(&sim->d_po, (size_t)sim->n_streams * cap * sim->po_words_int * 4));
+  if (sim->lanes) {
+    if (sim->d_po_lane) cudaFree(sim->d_po_lane);
+    sim->d_po_lane = nullptr;
+    CK(dalloc(&sim->d_po_lane, (size_t)cap * sim->po_words_int * 32 * sim->n_groups * 4));
+  }
   if (sim->flags & GEM_F_TRACE_STATE) CK(dalloc(&sim->d_qtrace, (size_t)sim->n_streams * cap * sim->q_words_ext * 4));
   if (sim->flags & GEM_F_DIGEST) CK(dalloc(&sim->d_digest, (size_t)sim->n_streams * cap * 8));
   sim->out_cap = cap;
@@ -897,6 +930,61 @@ static int plan_launch(gem_sim* sim, uint32_t max_chunk_words, uint32_t grid_lim
   return GEM_OK;
 }
 
+// Lane mode launch: one CTA per SM (all shared memory for the lane state and
+// the program ring), work items = (partition, 32-stream group), LPT lists.
+static int plan_launch_lanes(gem_sim* sim, uint32_t grid_limit) {
+  int sms = 0, coop = 0, optin = 0;
+  CK(cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, sim->device));
+  CK(cudaDeviceGetAttribute(&coop, cudaDevAttrCooperativeLaunch, sim->device));
+  CK(cudaDeviceGetAttribute(&optin, cudaDevAttrMaxSharedMemoryPerBlockOptin, sim->device));
+  if (!coop) return fail(GEM_E_UNSUPPORTED, "device lacks cooperative launch");
+  sim->sm_count = (uint32_t)sms;
+  const uint32_t slot = (sim->lane_max_chunk + 3u) & ~3u;
+  // 32-stream groups per work item: as many as fit beside a 4-slot ring (GEM_LANE_GROUPS overrides)
+  uint32_t gl = 1;
+  {
+    const char* e = getenv("GEM_LANE_GROUPS");
+    const uint32_t want = e ? (uint32_t)atoi(e) : 4;
+    for (uint32_t k = std::max<uint32_t>(1, std::min(want, sim->n_groups)); k >= 1; k--) {
+      const uint64_t words = (uint64_t)k * (sim->lane_words + sim->ramp_words + 16) + GEM_MAX_CHUNKS + 16 + 4 * slot;
+      if (words * 4 <= (uint64_t)optin || k == 1) { gl = k; break; }
+    }
+  }
+  sim->lane_groups = gl;
+  sim->group = 32 * gl;    // streams per work item
+  sim->max_items = 0;
+  for (uint32_t s = 0; s < sim->n_stages; s++)
+    sim->max_items = std::max(sim->max_items, (sim->h_stage[s + 1] - sim->h_stage[s]) * ((sim->n_groups + gl - 1) / gl));
+  const uint32_t fixed_words = gl * (sim->lane_words + sim->ramp_words + 16) + GEM_MAX_CHUNKS + 16;
+  if ((uint64_t)(fixed_words + 2 * slot) * 4 > (uint64_t)optin)
+    return fail(GEM_E_UNSUPPORTED, "lane state + 2 ring slots exceed shared memory");
+  const uint32_t area = (uint32_t)(optin / 4) - fixed_words;
+  uint32_t ring = std::min<uint32_t>(GEM_RING_MAX, area / std::max<uint32_t>(slot, 4));
+  ring = ring >= 4 ? 4 : 2;
+  uint32_t grid = std::max<uint32_t>(1, std::min<uint32_t>(sim->max_items, (uint32_t)sms));
+  if (grid_limit) grid = std::max<uint32_t>(1, std::min(grid, grid_limit));
+  const uint32_t smem = (fixed_words + ring * slot) * 4;
+  CK(cudaFuncSetAttribute(gem_lane_kernel, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem));
+  int occ = 0;
+  CK(cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ, gem_lane_kernel, GEM_THREADS, smem));
+  if (occ < 1) return fail(GEM_E_UNSUPPORTED, "lane kernel cannot be resident");
+  std::vector<uint32_t> off;
+  std::vector<uint2> items;
+  build_worklists(sim, grid, off, items);
+  sim->blocks_per_sm = 1;
+  sim->grid = grid;
+  sim->area_words = ring * slot;
+  sim->ring_slots = ring;
+  sim->slot_words = slot;
+  sim->resident = 0;
+  sim->smem_bytes = smem;
+  CK(dalloc(&sim->d_wl_off, off.size() * 4));
+  CK(cudaMemcpy(sim->d_wl_off, off.data(), off.size() * 4, cudaMemcpyHostToDevice));
+  CK(dalloc(&sim->d_wl_items, std::max<size_t>(items.size(), 1) * 8));
+  if (!items.empty()) CK(cudaMemcpy(sim->d_wl_items, items.data(), items.size() * 8, cudaMemcpyHostToDevice));
+  return GEM_OK;
+}
+
 extern "C" {
 
 const char* gem_last_error(void) { return g_err.c_str(); }
@@ -963,6 +1051,17 @@ int gem_load_program(const void* blob, size_t nbytes, const gem_config* cfg, gem
   else { CK(cudaStreamCreateWithFlags(&sim->stream, cudaStreamNonBlocking)); sim->own_stream = true; }
   CK(cudaEventCreate(&sim->ev0));
   CK(cudaEventCreate(&sim->ev1));
+  // lane mode: >= 32 streams and lane programs present (GEM_NO_LANES=1 disables)
+  {
+    const char* nl = getenv("GEM_NO_LANES");
+    sim->lanes = (w[GH_HAS_LANES] && cfg->n_streams >= 32 && !(nl && nl[0] == '1')) ? 1u : 0u;
+    if (sim->lanes) {
+      sim->n_groups = (cfg->n_streams + 31) / 32;
+      sim->lane_words = (std::max<uint32_t>(w[GH_LANE_MAX_WORDS], 4) + 3) & ~3u;
+      sim->lane_max_chunk = w[GH_LANE_MAX_CHUNK_WORDS];
+      sim->ramp_words = std::max<uint32_t>(w[GH_MAX_RAMS_PART], 1) * 128;
+    }
+  }
   // uploads
   const size_t S = sim->n_streams;
   CK(dalloc(&sim->d_prog, prog_words * 4));
@@ -978,15 +1077,36 @@ int gem_load_program(const void* blob, size_t nbytes, const gem_config* cfg, gem
   CK(cudaMemcpy(sim->d_q_ext_of_int, q_ext_of_int, (size_t)sim->q_words_int * 32 * 4, cudaMemcpyHostToDevice));
   CK(dalloc(&sim->d_po_int_of_ext, po_int_of_ext.size() * 4));
   CK(cudaMemcpy(sim->d_po_int_of_ext, po_int_of_ext.data(), po_int_of_ext.size() * 4, cudaMemcpyHostToDevice));
-  CK(dalloc(&sim->d_q, 2 * S * sim->q_words_int * 4));
-  CK(dalloc(&sim->d_rd, 2 * S * std::max<uint32_t>(sim->n_rams, 1) * 4));
-  CK(dalloc(&sim->d_cut, S * std::max<uint32_t>(sim->cut_words, 1) * 4));
+  if (sim->lanes) {
+    const uint64_t lp_words = w[GH_LANE_PROG_WORDS_LO] | ((uint64_t)w[GH_LANE_PROG_WORDS_HI] << 32);
+    if (w[GH_OFF_LANE_PROG] + lp_words > nw) { gem_free(sim); return fail(GEM_E_FORMAT, "truncated lane programs"); }
+    CK(dalloc(&sim->d_lprog, lp_words * 4));
+    CK(cudaMemcpy(sim->d_lprog, w + w[GH_OFF_LANE_PROG], lp_words * 4, cudaMemcpyHostToDevice));
+    const size_t G = sim->n_groups, qb = (size_t)sim->q_words_int * 32;
+    CK(dalloc(&sim->d_q, 2 * qb * G * 4));
+    CK(dalloc(&sim->d_rd, 2 * (size_t)std::max<uint32_t>(sim->n_rams, 1) * 32 * G * 4));
+    CK(dalloc(&sim->d_cut, (size_t)std::max<uint32_t>(sim->cut_words, 1) * 32 * G * 4));
+  } else {
+    CK(dalloc(&sim->d_q, 2 * S * sim->q_words_int * 4));
+    CK(dalloc(&sim->d_rd, 2 * S * std::max<uint32_t>(sim->n_rams, 1) * 4));
+    CK(dalloc(&sim->d_cut, S * std::max<uint32_t>(sim->cut_words, 1) * 4));
+  }
   CK(dalloc(&sim->d_mem, S * sim->n_rams * (size_t)GEM_RAM_WORDS * 4));
   CK(dalloc(&sim->d_bar, 64));
   CK(dalloc(&sim->d_err, 64));
   CK(cudaMemset(sim->d_err, 0, 64));
   // initial state: flops = init (U5), RD = 0, RAM = 0 (U10)
-  {
+  if (sim->lanes) {
+    const size_t G = sim->n_groups, qb = (size_t)sim->q_words_int * 32;
+    std::vector<uint32_t> q0(2 * qb * G, 0);
+    for (size_t b = 0; b < qb; b++)
+      if ((finit[b / 32] >> (b % 32)) & 1u)
+        for (size_t g = 0; g < G; g++) q0[g * qb + b] = 0xFFFFFFFFu;
+    CK(cudaMemcpy(sim->d_q, q0.data(), q0.size() * 4, cudaMemcpyHostToDevice));
+    CK(cudaMemset(sim->d_rd, 0, 2 * (size_t)std::max<uint32_t>(sim->n_rams, 1) * 32 * G * 4));
+    CK(cudaMemset(sim->d_cut, 0, (size_t)std::max<uint32_t>(sim->cut_words, 1) * 32 * G * 4));
+    if (sim->n_rams) CK(cudaMemset(sim->d_mem, 0, S * sim->n_rams * (size_t)GEM_RAM_WORDS * 4));
+  } else {
     std::vector<uint32_t> q0(S * sim->q_words_int);
     for (size_t s = 0; s < S; s++) std::memcpy(&q0[s * sim->q_words_int], finit, sim->q_words_int * 4);
     CK(cudaMemcpy(sim->d_q, q0.data(), q0.size() * 4, cudaMemcpyHostToDevice));
@@ -998,7 +1118,12 @@ int gem_load_program(const void* blob, size_t nbytes, const gem_config* cfg, gem
   // persistent co-resident grid + shared-memory program placement
   sim->h_parts.assign(parts, parts + (size_t)sim->n_parts * GP_WORDS);
   sim->h_stage.assign(stages, stages + stage_words);
-  if (int r = plan_launch(sim, w[GH_MAX_CHUNK_WORDS], cfg->grid_limit)) { gem_free(sim); return r; }
+  if (sim->lanes) {
+    if (int r = plan_launch_lanes(sim, cfg->grid_limit)) { gem_free(sim); return r; }
+  } else if (int r = plan_launch(sim, w[GH_MAX_CHUNK_WORDS], cfg->grid_limit)) {
+    gem_free(sim);
+    return r;
+  }
   CK(cudaDeviceSynchronize());
   *out = sim;
   return GEM_OK;
@@ -1012,6 +1137,7 @@ int gem_info_get(const gem_sim* sim, gem_info* out) {
   out->pi_words = sim->pi_words; out->po_words = sim->po_words_ext; out->q_words = sim->q_words_ext;
   out->grid = sim->grid; out->blocks_per_sm = sim->blocks_per_sm; out->smem_bytes = sim->smem_bytes;
   out->resident = sim->resident; out->ring_slots = sim->ring_slots; out->group = sim->group;
+  out->lanes = sim->lanes;
   out->n_streams = sim->n_streams;
   out->n_and = sim->n_and; out->n_and_mapped = sim->n_and_mapped; out->program_bytes = sim->program_bytes;
   out->cycle = sim->cycle;
@@ -1029,12 +1155,24 @@ int gem_set_inputs(gem_sim* sim, const uint32_t* pi, uint64_t ncycles, int src_o
     sim->in_cap = 0;
     uint32_t cap = std::max<uint32_t>((uint32_t)ncycles, 16);
     CK(dalloc(&sim->d_pi, (size_t)sim->n_streams * cap * std::max<uint32_t>(sim->pi_words, 1) * 4));
+    if (sim->lanes) {
+      if (sim->d_pi_lane) cudaFree(sim->d_pi_lane);
+      sim->d_pi_lane = nullptr;
+      CK(dalloc(&sim->d_pi_lane, (size_t)cap * std::max<uint32_t>(sim->pi_words, 1) * 32 * sim->n_groups * 4));
+    }
     sim->in_cap = cap;
   }
   if (ncycles && sim->pi_words) {
     const size_t row = (size_t)ncycles * sim->pi_words * 4;
     CK(cudaMemcpy2DAsync(sim->d_pi, (size_t)sim->in_cap * sim->pi_words * 4, pi, row, row, sim->n_streams,
                          src_on_device ? cudaMemcpyDeviceToDevice : cudaMemcpyHostToDevice, sim->stream));
+    if (sim->lanes) {
+      const uint64_t warps = ncycles * sim->n_groups * sim->pi_words;
+      to_lanes_kernel<<<(unsigned)std::min<uint64_t>(65535, (warps * 32 + 255) / 256), 256, 0, sim->stream>>>(
+          sim->d_pi, sim->d_pi_lane, sim->n_streams, (uint32_t)ncycles, sim->pi_words,
+          (uint64_t)sim->in_cap * sim->pi_words, sim->pi_words, sim->n_groups, 0);
+      CK(cudaGetLastError());
+    }
   }
   sim->in_queued = (uint32_t)ncycles;
   sim->in_head = 0;
@@ -1084,10 +1222,19 @@ int gem_step(gem_sim* sim, uint64_t ncycles) {
   CK(cudaMemsetAsync(sim->d_bar, 0, 8, sim->stream));
   if (sim->flags & GEM_F_DIGEST)
     CK(cudaMemsetAsync(sim->d_digest, 0, (size_t)sim->n_streams * sim->out_cap * 8, sim->stream));
+  if (sim->lanes) {
+    kp.lprog = sim->d_lprog;
+    kp.pi_lane = sim->d_pi_lane;
+    kp.po_lane = sim->d_po_lane;
+    kp.n_groups = sim->n_groups;
+    kp.ramp_words = sim->ramp_words;
+    kp.state_words = sim->lane_words;
+    kp.group = sim->lane_groups;
+  }
   void* args[] = {&kp};
   CK(cudaEventRecord(sim->ev0, sim->stream));
-  CK(cudaLaunchCooperativeKernel((const void*)gem_step_kernel, dim3(sim->grid), dim3(GEM_THREADS), args,
-                                 sim->smem_bytes, sim->stream));
+  CK(cudaLaunchCooperativeKernel(sim->lanes ? (const void*)gem_lane_kernel : (const void*)gem_step_kernel,
+                                 dim3(sim->grid), dim3(GEM_THREADS), args, sim->smem_bytes, sim->stream));
   CK(cudaEventRecord(sim->ev1, sim->stream));
   sim->in_head += (uint32_t)ncycles;
   sim->cycle += ncycles;
@@ -1119,6 +1266,13 @@ int gem_read_outputs(gem_sim* sim, uint32_t* dst, uint64_t ncycles, int dst_on_d
     if (int r = ensure_scratch(sim, bytes)) return r;
     out = sim->d_scratch;
   }
+  if (sim->lanes) {
+    const uint64_t warps = ncycles * sim->n_groups * sim->po_words_int;
+    from_lanes_kernel<<<(unsigned)std::min<uint64_t>(65535, (warps * 32 + 255) / 256), 256, 0, sim->stream>>>(
+        sim->d_po_lane, sim->d_po, sim->n_streams, (uint32_t)ncycles, sim->po_words_int,
+        (uint64_t)sim->out_cap * sim->po_words_int, sim->po_words_int, sim->n_groups);
+    CK(cudaGetLastError());
+  }
   // rows = stream*ncycles + cycle; in-row stride = po_words_int, with stream stride out_cap
   for (uint32_t s = 0; s < sim->n_streams; s++) {
     unpermute_kernel<<<std::min<uint64_t>(4096, (ncycles * sim->po_words_ext + 255) / 256 + 1), 256, 0,
@@ -1140,13 +1294,21 @@ int gem_read_state(gem_sim* sim, uint32_t* dst, int dst_on_device) {
   CK(cudaStreamSynchronize(sim->stream));
   const uint32_t buf = (uint32_t)(sim->cycle & 1);
   const size_t bytes = (size_t)sim->n_streams * sim->q_words_ext * 4;
-  uint32_t* out = dst;
-  if (!dst_on_device) {
-    if (int r = ensure_scratch(sim, bytes)) return r;
-    out = sim->d_scratch;
+  const size_t ibytes = (size_t)sim->n_streams * sim->q_words_int * 4;
+  if (int r = ensure_scratch(sim, bytes + ibytes)) return r;
+  uint32_t* out = dst_on_device ? dst : sim->d_scratch;
+  const uint32_t* qin = sim->d_q + (size_t)buf * sim->n_streams * sim->q_words_int;
+  if (sim->lanes) {
+    uint32_t* tmp = sim->d_scratch + bytes / 4;
+    const uint64_t warps = (uint64_t)sim->n_groups * sim->q_words_int;
+    from_lanes_kernel<<<(unsigned)std::min<uint64_t>(65535, (warps * 32 + 255) / 256), 256, 0, sim->stream>>>(
+        sim->d_q + (size_t)buf * sim->q_words_int * 32 * sim->n_groups, tmp, sim->n_streams, 1, sim->q_words_int,
+        sim->q_words_int, 0, sim->n_groups);
+    CK(cudaGetLastError());
+    qin = tmp;
   }
   unpermute_kernel<<<std::min<uint64_t>(4096, ((uint64_t)sim->n_streams * sim->q_words_ext + 255) / 256 + 1), 256,
-                     0, sim->stream>>>(sim->d_q + (size_t)buf * sim->n_streams * sim->q_words_int, out,
+                     0, sim->stream>>>(qin, out,
                                        sim->d_q_int_of_ext, sim->n_flops, sim->q_words_int, sim->q_words_ext,
                                        sim->n_streams, sim->q_words_int, sim->q_words_ext);
   CK(cudaGetLastError());
@@ -1164,10 +1326,24 @@ int gem_write_state(gem_sim* sim, const uint32_t* src, int src_on_device) {
   if (int r = ensure_scratch(sim, bytes)) return r;
   CK(cudaMemcpyAsync(sim->d_scratch, src, bytes, src_on_device ? cudaMemcpyDeviceToDevice : cudaMemcpyHostToDevice,
                      sim->stream));
+  uint32_t* qdst = sim->d_q + (size_t)buf * sim->n_streams * sim->q_words_int;
+  if (sim->lanes) {
+    if (int r = ensure_scratch(sim, bytes + (size_t)sim->n_streams * sim->q_words_int * 4)) return r;
+    CK(cudaMemcpyAsync(sim->d_scratch, src, bytes, src_on_device ? cudaMemcpyDeviceToDevice : cudaMemcpyHostToDevice,
+                       sim->stream));
+    qdst = sim->d_scratch + bytes / 4;
+  }
   permute_kernel<<<std::min<uint64_t>(4096, ((uint64_t)sim->n_streams * sim->q_words_int + 255) / 256 + 1), 256, 0,
-                   sim->stream>>>(sim->d_scratch, sim->d_q + (size_t)buf * sim->n_streams * sim->q_words_int,
-                                  sim->d_q_ext_of_int, sim->q_words_int, sim->q_words_ext, sim->n_streams);
+                   sim->stream>>>(sim->d_scratch, qdst, sim->d_q_ext_of_int, sim->q_words_int, sim->q_words_ext,
+                                  sim->n_streams);
   CK(cudaGetLastError());
+  if (sim->lanes) {
+    const uint64_t warps = (uint64_t)sim->n_groups * sim->q_words_int;
+    to_lanes_kernel<<<(unsigned)std::min<uint64_t>(65535, (warps * 32 + 255) / 256), 256, 0, sim->stream>>>(
+        qdst, sim->d_q + (size_t)buf * sim->q_words_int * 32 * sim->n_groups, sim->n_streams, 1, sim->q_words_int,
+        sim->q_words_int, 0, sim->n_groups, 0);
+    CK(cudaGetLastError());
+  }
   CK(cudaStreamSynchronize(sim->stream));
   return GEM_OK;
 }
@@ -1242,7 +1418,8 @@ void gem_free(gem_sim* sim) {
                   (void*)sim->d_q_ext_of_int, (void*)sim->d_po_int_of_ext, (void*)sim->d_q, (void*)sim->d_rd,
                   (void*)sim->d_cut, (void*)sim->d_mem, (void*)sim->d_pi, (void*)sim->d_po, (void*)sim->d_qtrace,
                   (void*)sim->d_scratch, (void*)sim->d_digest, (void*)sim->d_bar, (void*)sim->d_err,
-                  (void*)sim->d_prof, (void*)sim->d_wl_off, (void*)sim->d_wl_items})
+                  (void*)sim->d_prof, (void*)sim->d_wl_off, (void*)sim->d_wl_items, (void*)sim->d_lprog,
+                  (void*)sim->d_pi_lane, (void*)sim->d_po_lane})
     if (p) cudaFree(p);
   if (sim->ev0) cudaEventDestroy(sim->ev0);
   if (sim->ev1) cudaEventDestroy(sim->ev1);

@@ -35,7 +35,7 @@ class GemInfo(ctypes.Structure):
     _fields_ = [(n, ctypes.c_uint32) for n in
                 ("n_pi", "n_po", "n_flops", "n_rams", "n_parts", "n_stages", "max_layers", "total_layers",
                  "pi_words", "po_words", "q_words", "grid", "blocks_per_sm", "smem_bytes", "n_streams",
-                 "resident", "ring_slots", "group")] + \
+                 "resident", "ring_slots", "group", "lanes")] + \
                [(n, ctypes.c_uint64) for n in ("n_and", "n_and_mapped", "program_bytes", "cycle")]
 
     def as_dict(self):

@@ -25,6 +25,7 @@
 // The mapper shares no code with oracle/.
 
 #include <algorithm>
+#include <array>
 #include <atomic>
 #include <chrono>
 #include <cstdint>
@@ -33,6 +34,7 @@
 #include <cstring>
 #include <fstream>
 #include <functional>
+#include <map>
 #include <mutex>
 #include <numeric>
 #include <sstream>
@@ -60,6 +62,7 @@ struct Options {
   int refine = 3;           // rounds of splitting the costliest partitions (critical path)
   double refine_ratio = 1.35;  // split partitions costing more than this x the median
   int max_parts = 280;      // refinement stops growing the partition count here
+  int lanes = 0;            // also emit stream-sliced lane programs (batched streams)
   int verbose = 0;
   int max_state_words = GEM_MAX_STATE_WORDS;
   double cap_slack = 1.0;
@@ -87,6 +90,7 @@ static Options parse_opts(const char* s) {
     else if (k == "refine") o.refine = std::stoi(v);
     else if (k == "refine_ratio") o.refine_ratio = std::stod(v);
     else if (k == "max_parts") o.max_parts = std::stoi(v);
+    else if (k == "lanes") o.lanes = std::stoi(v);
     else throw std::runtime_error("unknown option " + k);
   }
   if (o.stages < 1 || o.stages > 2) throw std::runtime_error("stages must be 1 or 2");
@@ -403,6 +407,8 @@ struct Part {
   std::vector<OutWord> outs;
   // filled by mapping
   std::vector<uint32_t> prog;
+  std::vector<uint32_t> lane_prog;   // lane-mode program (opt.lanes)
+  uint32_t lane_words = 0;
   uint32_t n_layers = 0, n_nodes = 0, state_words = 0, n_leaves = 0, max_level = 0, n_writeouts = 0;
   uint64_t slots_used = 0;
   bool ok = false;
@@ -429,6 +435,29 @@ static inline uint32_t slot_bit(int k, uint32_t id) {
   int kk = k <= 5 ? k : k - 5;
   return (uint32_t)kOff[kk] + id % group_width(k);
 }
+
+// packed constant word of a unit (thread: levels 1-5, warp: 6-10, top: 11-13)
+static uint32_t pack_unit(int k0, int k1, uint32_t unit, const std::vector<uint8_t>* arr) {
+  uint32_t v = 0;
+  for (int k = k0; k <= k1; k++) {
+    uint32_t g = group_width(k);
+    for (uint32_t q = 0; q < g; q++) {
+      uint32_t id = unit * g + q;
+      if (arr[k][id]) v |= 1u << slot_bit(k, id);
+    }
+  }
+  return v;
+}
+
+// per-layer record for the lane-mode encoding
+struct LaneLayer {
+  std::vector<uint32_t> leaf_sig;                   // 8192 leaves: local signal or UINT32_MAX
+  std::vector<std::array<uint32_t, 3>> two, wwo;    // {thread|warp, slot bit, signal}
+  std::vector<std::array<uint32_t, 2>> top;         // {slot bit, signal}
+  std::vector<uint32_t> cth;                        // 256 x {xa, xb, ob}
+  uint32_t cw[8][3];
+  uint32_t topc;
+};
 
 struct Mapper {
   const Graph& G;
@@ -571,6 +600,8 @@ struct Mapper {
     std::vector<int32_t> comp_k(n, -1), comp_id(n, -1);   // one computed copy per node
     std::vector<uint32_t> computed;
     std::vector<uint32_t> thread_leaves(256, 0);
+    std::vector<LaneLayer> lane_layers;
+    std::vector<uint32_t> lleaf(opt.lanes ? 8192 : 0, UINT32_MAX);
 
     while (true) {
       // any work left?
@@ -612,6 +643,7 @@ struct Mapper {
         std::fill(sob[k].begin(), sob[k].end(), 0);
       }
       std::fill(thread_leaves.begin(), thread_leaves.end(), 0);
+      if (opt.lanes) std::fill(lleaf.begin(), lleaf.end(), UINT32_MAX);
       for (uint32_t i : computed) { comp_k[i] = -1; comp_id[i] = -1; }
       computed.clear();
       uint32_t layer_leaves = 0;
@@ -637,6 +669,7 @@ struct Mapper {
         if (loc[x] >= 0) {
           while (k > 0) { slot[k][id] = -2; sob[k][id] = 1; id = child_a(k, id); k--; }
           slot[0][id] = loc[x];
+          if (opt.lanes) lleaf[id] = x;
           thread_leaves[id >> 5]++;
           layer_leaves++;
         } else {
@@ -709,6 +742,8 @@ struct Mapper {
         if (*tgt < 0) { fail(P, "state overflow"); return; }
         loc[x] = (int32_t)((uint32_t)*tgt * 32 + slot_bit(k, id));
         word_vals[(uint32_t)*tgt].push_back(x);
+        if (getenv("GEM_DBG_X") && x == (uint32_t)atoi(getenv("GEM_DBG_X")))
+          fprintf(stderr, "dbg: x=%u written out in layer %u k=%d id=%u loc=%d\n", x, n_layers, k, id, loc[x]);
       }
       if (opt.verbose >= 2) {
         uint32_t nwo = 0;
@@ -718,6 +753,31 @@ struct Mapper {
         for (uint32_t i = 0; i < n; i++) nmc += mc[i];
         fprintf(stderr, "  layer %u: mc=%u computed=%zu need_wo=%zu wo_words=%u leaves=%u free=%zu\n", n_layers, nmc,
                 computed.size(), need_wo.size(), nwo, layer_leaves, free_words.size());
+      }
+      // ---- lane-mode record of this layer (same placement, signal-level view)
+      if (opt.lanes) {
+        LaneLayer LL;
+        LL.leaf_sig = lleaf;
+        for (uint32_t x : need_wo) {
+          int k = comp_k[x];
+          uint32_t id = (uint32_t)comp_id[x];
+          if (k <= 5) LL.two.push_back({slot_unit(k, id), slot_bit(k, id), x});
+          else if (k <= 10) LL.wwo.push_back({slot_unit(k, id), slot_bit(k, id), x});
+          else LL.top.push_back({slot_bit(k, id), x});
+        }
+        LL.cth.resize(256 * 3);
+        for (uint32_t t = 0; t < 256; t++) {
+          LL.cth[3 * t] = pack_unit(1, 5, t, sxa);
+          LL.cth[3 * t + 1] = pack_unit(1, 5, t, sxb);
+          LL.cth[3 * t + 2] = pack_unit(1, 5, t, sob);
+        }
+        for (uint32_t w = 0; w < 8; w++) {
+          LL.cw[w][0] = pack_unit(6, 10, w, sxa);
+          LL.cw[w][1] = pack_unit(6, 10, w, sxb);
+          LL.cw[w][2] = pack_unit(6, 10, w, sob);
+        }
+        LL.topc = pack_unit(11, 13, 0, sxa) | (pack_unit(11, 13, 0, sxb) << 8) | (pack_unit(11, 13, 0, sob) << 16);
+        lane_layers.push_back(std::move(LL));
       }
       // ---- encode the layer
       encode_layer(prog_layers, slot, sxa, sxb, sob, wo_thread, wo_warp, wo_top);
@@ -783,7 +843,179 @@ struct Mapper {
     P.n_leaves = total_leaves;
     P.n_writeouts = total_wo;
     P.slots_used = slots_used;
+    if (opt.lanes && !encode_lanes(P, lane_layers, gread_src, scratch)) return;
     P.ok = true;
+  }
+
+  // Lane program (gem_isa.h "Lane mode"): allocate one lane word per live signal
+  // (interval allocation over layers) and encode the recorded layers.
+  bool encode_lanes(Part& P, const std::vector<LaneLayer>& LLs, const std::vector<uint32_t>& gread_src,
+                    const std::vector<int32_t>& scratch) {
+    (void)gread_src;
+    const uint32_t n = (uint32_t)cid.size();
+    const int32_t INF = 1 << 30;
+    const uint32_t L = (uint32_t)LLs.size();
+    std::vector<int32_t> last(n, -1);
+    for (uint32_t l = 0; l < L; l++)
+      for (uint32_t x : LLs[l].leaf_sig)
+        if (x != UINT32_MAX) last[x] = std::max<int32_t>(last[x], (int32_t)l);
+    for (uint32_t i = 0; i < n; i++) if (is_ep[i]) last[i] = INF;
+    std::vector<int32_t> word(n, -1);
+    word[0] = 0;   // local node 0 is the constant
+    // free-interval allocator (first fit, coalescing); word 0 reserved
+    std::map<uint32_t, uint32_t> freeiv;   // start -> length
+    const uint32_t kMaxWords = 65535;
+    freeiv[1] = kMaxWords - 1;
+    uint32_t max_word = 1;
+    std::vector<std::vector<uint32_t>> die(L + 1);
+    auto take = [&](uint32_t k) -> int64_t {
+      for (auto it = freeiv.begin(); it != freeiv.end(); ++it)
+        if (it->second >= k) {
+          uint32_t st = it->first, len = it->second;
+          freeiv.erase(it);
+          if (len > k) freeiv[st + k] = len - k;
+          max_word = std::max(max_word, st + k);
+          return st;
+        }
+      return -1;
+    };
+    auto give = [&](uint32_t w) {
+      auto nx = freeiv.lower_bound(w);
+      uint32_t st = w, len = 1;
+      if (nx != freeiv.end() && nx->first == w + 1) { len += nx->second; nx = freeiv.erase(nx); }
+      if (nx != freeiv.begin()) {
+        auto pv = std::prev(nx);
+        if (pv->first + pv->second == w) { st = pv->first; len += pv->second; freeiv.erase(pv); }
+      }
+      freeiv[st] = len;
+    };
+    auto bind = [&](uint32_t x, uint32_t w) {
+      word[x] = (int32_t)w;
+      if (last[x] >= 0 && last[x] < (int32_t)L) die[last[x]].push_back(w);
+    };
+    std::vector<uint32_t> srcs;
+    for (uint32_t i = 1; i < n; i++)
+      if (is_src[i]) {
+        int64_t w = take(1);
+        if (w < 0) { fail(P, "lane state overflow"); return false; }
+        srcs.push_back(i);
+        bind(i, (uint32_t)w);
+      }
+    // per layer: unit -> (mask, base)
+    struct UnitWo { uint32_t mask = 0, base = 0; };
+    std::vector<std::array<UnitWo, 256>> th(L);
+    std::vector<std::array<UnitWo, 8>> wa(L);
+    std::vector<UnitWo> tp(L);
+    for (uint32_t l = 0; l < L; l++) {
+      if (l > 0)
+        for (uint32_t w : die[l - 1]) give(w);
+      // group write-outs by unit, consecutive words in slot-bit order
+      std::map<uint32_t, std::vector<std::pair<uint32_t, uint32_t>>> units;   // key: kind<<16 | unit
+      for (auto& e : LLs[l].two) units[(0u << 16) | e[0]].push_back({e[1], e[2]});
+      for (auto& e : LLs[l].wwo) units[(1u << 16) | e[0]].push_back({e[1], e[2]});
+      for (auto& e : LLs[l].top) units[(2u << 16)].push_back({e[0], e[1]});
+      for (auto& kv : units) {
+        auto& v = kv.second;
+        std::sort(v.begin(), v.end());
+        int64_t base = take((uint32_t)v.size());
+        if (base < 0) { fail(P, "lane state overflow"); return false; }
+        UnitWo u;
+        u.base = (uint32_t)base;
+        for (size_t k = 0; k < v.size(); k++) {
+          u.mask |= 1u << v[k].first;
+          bind(v[k].second, (uint32_t)base + (uint32_t)k);
+        }
+        uint32_t kind = kv.first >> 16, unit = kv.first & 0xFFFF;
+        if (kind == 0) th[l][unit] = u;
+        else if (kind == 1) wa[l][unit] = u;
+        else tp[l] = u;
+      }
+    }
+    if (max_word >= kMaxWords) { fail(P, "lane state overflow"); return false; }
+    auto lw = [&](uint32_t x) -> uint32_t {
+      if (word[x] < 0)
+        throw std::runtime_error("lane: signal without a word (local " + std::to_string(x) + ")");
+      return (uint32_t)word[x];
+    };
+    std::vector<uint32_t>& pr = P.lane_prog;
+    pr.assign(LPH_WORDS, 0);
+    pr[LPH_MAGIC] = GEM_LANE_MAGIC;
+    pr[LPH_N_LAYERS] = L;
+    pr[LPH_N_OUT] = (uint32_t)P.outs.size() * 32;
+    pr[LPH_N_RAM] = (uint32_t)P.rams.size();
+    pr[LPH_LANE_WORDS] = (max_word + 3) & ~3u;
+    pr[LPH_OFF_CHUNKS] = (uint32_t)pr.size();
+    pr[LPH_N_CHUNKS] = L + 2;
+    for (uint32_t k = 0; k < L + 2; k++) pr.push_back(0);
+    while (pr.size() % 4) pr.push_back(0);
+    pr[LPH_OFF_LAYERS] = (uint32_t)pr.size();   // chunk 0 = header + chunk table
+    pr[pr[LPH_OFF_CHUNKS]] = (uint32_t)pr.size();
+    for (uint32_t l = 0; l < L; l++) {
+      const LaneLayer& LL = LLs[l];
+      size_t base = pr.size();
+      pr.resize(base + LLH_WORDS, 0);
+      uint32_t active = 0;
+      for (uint32_t t = 0; t < 256; t++) if (th[l][t].mask) active |= 1u << (t / 32);
+      for (uint32_t w = 0; w < 8; w++) if (wa[l][w].mask) active |= 1u << w;
+      for (uint32_t id = 0; id < 8192; id++) if (LL.leaf_sig[id] != UINT32_MAX) active |= 1u << (id >> 10);
+      const bool uses_top = tp[l].mask != 0;
+      pr[base + LLH_FLAGS] = active | (uses_top ? GEM_LF_USES_TOP : 0u);
+      pr[base + LLH_TOPC] = LL.topc;
+      pr[base + LLH_TOPWO] = tp[l].mask | (tp[l].base << 8);
+      for (uint32_t w = 0; w < 8; w++) {
+        if (!(active >> w & 1)) continue;
+        pr[base + LLH_WOFF0 + w] = (uint32_t)(pr.size() - base);
+        pr.push_back(LL.cw[w][0]); pr.push_back(LL.cw[w][1]); pr.push_back(LL.cw[w][2]);
+        pr.push_back(wa[l][w].mask); pr.push_back(wa[l][w].base);
+        pr.push_back(0); pr.push_back(0); pr.push_back(0);
+        for (uint32_t ln = 0; ln < 32; ln++) {
+          uint32_t t = w * 32 + ln;
+          pr.push_back(LL.cth[3 * t]); pr.push_back(LL.cth[3 * t + 1]); pr.push_back(LL.cth[3 * t + 2]);
+          pr.push_back(th[l][t].mask);
+        }
+        for (uint32_t g = 0; g < 4; g++)
+          for (uint32_t ln = 0; ln < 32; ln++)
+            for (uint32_t k = 0; k < 4; k++) {
+              uint32_t e = 0;
+              for (uint32_t h = 0; h < 2; h++) {
+                uint32_t pos = 8 * g + 2 * k + h, id = (w * 32 + ln) * 32 + pos;
+                uint32_t x = LL.leaf_sig[id];
+                e |= (x == UINT32_MAX ? 0u : lw(x)) << (16 * h);
+              }
+              pr.push_back(e);
+            }
+        for (uint32_t ln = 0; ln < 32; ln++) pr.push_back(th[l][w * 32 + ln].base);
+      }
+      pr[base + LLH_WORDS_] = (uint32_t)(pr.size() - base);
+      pr[pr[LPH_OFF_CHUNKS] + 1 + l] = pr[base + LLH_WORDS_];
+    }
+    pr[LPH_OFF_OUT] = (uint32_t)pr.size();
+    for (auto& ow : P.outs) {
+      uint32_t reg = GEM_GID_REGION(ow.dst), idx = GEM_GID_INDEX(ow.dst);
+      for (int k = 0; k < 32; k++) {
+        uint32_t l = ow.lit[k];
+        uint32_t x = (uint32_t)scratch[l >> 1];
+        pr.push_back((reg << 24) | (idx * 32 + (uint32_t)k));
+        pr.push_back(lw(x) | ((l & 1) ? GEM_OUT_INV : 0u));
+      }
+    }
+    pr[LPH_OFF_RAM] = (uint32_t)pr.size();
+    for (uint32_t r : P.rams) { pr.push_back(r); pr.push_back(0); pr.push_back(0); pr.push_back(0); }
+    while (pr.size() % 4) pr.push_back(0);
+    pr[pr[LPH_OFF_CHUNKS] + 1 + L] = (uint32_t)pr.size() - pr[LPH_OFF_OUT];
+    // input-port list last: read from global memory by the kernel, not streamed
+    pr[LPH_OFF_GREAD] = (uint32_t)pr.size();
+    uint32_t ng = 0;
+    for (uint32_t x : srcs) {
+      uint32_t gb = G.gbit[cid[x]];
+      pr.push_back(((gb >> 27) << 24) | (((gb >> 5) & 0x3FFFFF) * 32 + (gb & 31)));
+      pr.push_back(lw(x));
+      ng++;
+    }
+    pr[LPH_N_GREAD] = ng;
+    while (pr.size() % 4) pr.push_back(0);
+    P.lane_words = pr[LPH_LANE_WORDS];
+    return true;
   }
 
   void fail(Part& P, const char* why) {
@@ -1250,17 +1482,24 @@ static Blob compile(const char* data, size_t n, const char* opts) {
           if (i >= D.parts.size()) break;
           Part& P = D.parts[i];
           Mapper M(P.stage == 1 ? G1 : D.G, D.opt);
-          M.map(P, scratch);
+          try {
+            M.map(P, scratch);
+          } catch (const std::exception& e) {
+            P.ok = false;
+            P.err = e.what();
+          }
         }
       });
     for (auto& x : th) x.join();
     // split partitions that did not fit (state overflow) and retry
     std::vector<Part> next_parts;
     bool any_fail = false;
+    std::string last_err;
     for (size_t i = 0; i < D.parts.size(); i++) {
       Part& P = D.parts[i];
       if (P.ok) { next_parts.push_back(std::move(P)); continue; }
       any_fail = true;
+      last_err = P.err;
       size_t n_units = P.flops.size() + P.pos.size() + P.rams.size() + P.cuts.size();
       if (n_units <= 1 || attempt >= 12)
         throw std::runtime_error("mapping partition " + std::to_string(i) + " failed: " + P.err);
@@ -1329,7 +1568,7 @@ static Blob compile(const char* data, size_t n, const char* opts) {
     }
     if (!any_fail) break;
     for (auto& P : D.parts) { P.prog.clear(); P.ok = false; }
-    if (D.opt.verbose) fprintf(stderr, "gem_map: retry %d with %zu partitions\n", attempt + 1, D.parts.size());
+    if (D.opt.verbose) fprintf(stderr, "gem_map: retry %d with %zu partitions (%s)\n", attempt + 1, D.parts.size(), last_err.c_str());
   }
   // drop partitions with no endpoints (possible after splitting)
   auto t2 = std::chrono::steady_clock::now();
@@ -1426,6 +1665,34 @@ static Blob compile(const char* data, size_t n, const char* opts) {
   }
   w[GH_MAX_CHUNK_WORDS] = max_chunk;
   w[GH_MAX_PROG_WORDS] = max_prog;
+  if (D.opt.lanes) {
+    w[GH_HAS_LANES] = 1;
+    w[GH_OFF_LANE_PROG] = (uint32_t)w.size();
+    uint64_t lp = 0;
+    uint32_t lmc = 0, lmw = 0;
+    for (uint32_t i = 0; i < np; i++) {
+      auto& P = D.parts[i];
+      const uint32_t* pr = P.lane_prog.data();
+      w[part_tab + i * GP_WORDS + GP_LANE_OFF] = (uint32_t)lp;
+      w[part_tab + i * GP_WORDS + GP_LANE_LEN] = (uint32_t)P.lane_prog.size();
+      w[part_tab + i * GP_WORDS + GP_LANE_CHUNK0] = pr[pr[LPH_OFF_CHUNKS]];
+      w[part_tab + i * GP_WORDS + GP_LANE_CHUNK1] = pr[LPH_N_CHUNKS] > 1 ? pr[pr[LPH_OFF_CHUNKS] + 1] : 0;
+      w[part_tab + i * GP_WORDS + GP_LANE_CHUNK2] = pr[LPH_N_CHUNKS] > 2 ? pr[pr[LPH_OFF_CHUNKS] + 2] : 0;
+      w[part_tab + i * GP_WORDS + GP_LANE_WORDS] = P.lane_words;
+      for (uint32_t k = 0; k < pr[LPH_N_CHUNKS]; k++) lmc = std::max(lmc, pr[pr[LPH_OFF_CHUNKS] + k]);
+      lmw = std::max(lmw, P.lane_words);
+      w.insert(w.end(), P.lane_prog.begin(), P.lane_prog.end());
+      lp += P.lane_prog.size();
+      while (lp % 4) { w.push_back(0); lp++; }
+    }
+    w[GH_LANE_PROG_WORDS_LO] = (uint32_t)lp;
+    w[GH_LANE_PROG_WORDS_HI] = (uint32_t)(lp >> 32);
+    w[GH_LANE_MAX_CHUNK_WORDS] = lmc;
+    w[GH_LANE_MAX_WORDS] = lmw;
+    uint32_t mr = 0;
+    for (auto& P : D.parts) mr = std::max<uint32_t>(mr, (uint32_t)P.rams.size());
+    w[GH_MAX_RAMS_PART] = mr;
+  }
   w[GH_PROG_WORDS_LO] = (uint32_t)prog;
   w[GH_PROG_WORDS_HI] = (uint32_t)(prog >> 32);
   w[GH_TOTAL_WORDS_LO] = (uint32_t)w.size();

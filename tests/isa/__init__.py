@@ -25,6 +25,7 @@ def _load():
         lib.isa_load.argtypes = [P, ctypes.c_size_t]
         lib.isa_free.argtypes = [P]
         lib.isa_run.argtypes = [P, P, ctypes.c_uint64, P, P]
+        lib.isa_run_lanes.argtypes = [P, P, ctypes.c_uint64, P, P]
         lib.isa_last_error.restype = ctypes.c_char_p
         _lib = lib
     return _lib
@@ -52,6 +53,18 @@ class IsaInterp:
         q = np.zeros((T, (self.n_flops + 31) // 32), np.uint32)
         rc = self.lib.isa_run(self._h, stim.ctypes.data_as(ctypes.c_void_p), T,
                               po.ctypes.data_as(ctypes.c_void_p), q.ctypes.data_as(ctypes.c_void_p))
+        if rc:
+            raise RuntimeError(self.lib.isa_last_error().decode())
+        return po, q
+
+    def run_lanes(self, stim32):
+        """stim32 uint32 [32][cycles][pi_words] -> (po [32][cycles][..], q [32][cycles][..]) via lane programs."""
+        stim32 = np.ascontiguousarray(stim32, np.uint32)
+        T = stim32.shape[1]
+        po = np.zeros((32, T, (self.n_po + 31) // 32), np.uint32)
+        q = np.zeros((32, T, (self.n_flops + 31) // 32), np.uint32)
+        rc = self.lib.isa_run_lanes(self._h, stim32.ctypes.data_as(ctypes.c_void_p), T,
+                                    po.ctypes.data_as(ctypes.c_void_p), q.ctypes.data_as(ctypes.c_void_p))
         if rc:
             raise RuntimeError(self.lib.isa_last_error().decode())
         return po, q

@@ -167,6 +167,165 @@ int run_part(Interp& I, uint32_t p, uint64_t t, const uint32_t* stim, uint32_t* 
   (void)t;
   return 0;
 }
+
+// ------------------------------------------------------------------ lane mode
+// 32 streams per lane word.  Global lane state: Q_lane[2][q_bits], RD_lane[2][rams*32],
+// CUT_lane[cut_bits]; MEM per stream.
+struct LaneSim {
+  std::vector<uint32_t> Q[2], RD[2], CUT;
+  std::vector<std::vector<uint32_t>> MEM;   // [stream*n_rams + ram][8192]
+};
+
+int run_lane_part(Interp& I, LaneSim& Ls, uint32_t p, const uint32_t* pi_lane /* [pi_bits] */,
+                  uint32_t* po_lane /* [po_bits] */) {
+  const uint32_t* pt = I.parts + p * GP_WORDS;
+  const uint32_t* lane_base = I.w.data() + I.w[GH_OFF_LANE_PROG];
+  const uint32_t* pr = lane_base + pt[GP_LANE_OFF];
+  if (pr[LPH_MAGIC] != GEM_LANE_MAGIC) { g_err = "bad lane magic"; return -1; }
+  uint32_t cur = (uint32_t)(I.cycle & 1), nxt = cur ^ 1;
+  std::vector<uint32_t> S(pr[LPH_LANE_WORDS] + 1, 0);
+  const uint32_t* gr = pr + pr[LPH_OFF_GREAD];
+  for (uint32_t k = 0; k < pr[LPH_N_GREAD]; k++) {
+    uint32_t gid = gr[2 * k], dst = gr[2 * k + 1];
+    uint32_t reg = gid >> 24, b = gid & 0xFFFFFF, v;
+    if (reg == GEM_R_PI) v = pi_lane[b];
+    else if (reg == GEM_R_Q) v = Ls.Q[cur][b];
+    else if (reg == GEM_R_RD) v = Ls.RD[cur][b];
+    else if (reg == GEM_R_CUT) v = Ls.CUT[b];
+    else { g_err = "bad lane gread"; return -1; }
+    if (dst == 0 || dst >= S.size()) { g_err = "bad lane gread dst"; return -1; }
+    S[dst] = v;
+  }
+  const uint32_t* L = pr + pr[LPH_OFF_LAYERS];
+  std::vector<uint32_t> val[14];
+  for (uint32_t l = 0; l < pr[LPH_N_LAYERS]; l++) {
+    for (int k = 0; k <= 13; k++) val[k].assign(8192u >> k, 0);
+    uint32_t flags = L[LLH_FLAGS], topc = L[LLH_TOPC];
+    uint32_t lane_c[256][3];
+    uint32_t warp_c[8][3];
+    std::memset(lane_c, 0, sizeof(lane_c));
+    std::memset(warp_c, 0, sizeof(warp_c));
+    std::vector<std::pair<uint32_t, uint32_t>> wo;   // (slot id global (k<<16|id), word)
+    std::vector<uint8_t> read(S.size(), 0);
+    for (uint32_t wp = 0; wp < 8; wp++) {
+      if (!((flags >> wp) & 1)) continue;
+      const uint32_t* rec = L + L[LLH_WOFF0 + wp];
+      for (int c = 0; c < 3; c++) warp_c[wp][c] = rec[c];
+      for (uint32_t ln = 0; ln < 32; ln++)
+        for (int c = 0; c < 3; c++) lane_c[wp * 32 + ln][c] = rec[GEM_LWREC_HDR + ln * 4 + c];
+      const uint32_t* lv = rec + GEM_LWREC_HDR + 128;
+      for (uint32_t g = 0; g < 4; g++)
+        for (uint32_t ln = 0; ln < 32; ln++)
+          for (uint32_t k = 0; k < 4; k++) {
+            uint32_t e = lv[(g * 32 + ln) * 4 + k];
+            for (uint32_t h = 0; h < 2; h++) {
+              uint32_t word = (e >> (16 * h)) & 0xFFFFu, pos = 8 * g + 2 * k + h;
+              if (word >= S.size()) { g_err = "lane leaf out of range"; return -1; }
+              read[word] = 1;
+              val[0][(wp * 32 + ln) * 32 + pos] = 0;
+              // stash the word in a separate array: val arrays hold bits for packed mode; here words
+            }
+          }
+    }
+    // word-valued slots
+    std::vector<uint32_t> wv[14];
+    for (int k = 0; k <= 13; k++) wv[k].assign(8192u >> k, 0);
+    for (uint32_t wp = 0; wp < 8; wp++) {
+      if (!((flags >> wp) & 1)) continue;
+      const uint32_t* rec = L + L[LLH_WOFF0 + wp];
+      const uint32_t* lv = rec + GEM_LWREC_HDR + 128;
+      for (uint32_t g = 0; g < 4; g++)
+        for (uint32_t ln = 0; ln < 32; ln++)
+          for (uint32_t k = 0; k < 4; k++) {
+            uint32_t e = lv[(g * 32 + ln) * 4 + k];
+            for (uint32_t h = 0; h < 2; h++) {
+              uint32_t word = (e >> (16 * h)) & 0xFFFFu, pos = 8 * g + 2 * k + h;
+              wv[0][(wp * 32 + ln) * 32 + pos] = S[word];
+            }
+          }
+    }
+    for (int k = 1; k <= 13; k++) {
+      uint32_t gwid = gw(k);
+      for (uint32_t id = 0; id < (8192u >> k); id++) {
+        uint32_t ca = (id / gwid) * 2 * gwid + id % gwid, cb = ca + gwid;
+        uint32_t xa, xb, ob, b = sbit(k, id);
+        if (k <= 5) { uint32_t t = id / gwid; xa = lane_c[t][0]; xb = lane_c[t][1]; ob = lane_c[t][2]; }
+        else if (k <= 10) { uint32_t wq = id / gwid; xa = warp_c[wq][0]; xb = warp_c[wq][1]; ob = warp_c[wq][2]; }
+        else { xa = topc & 0xFF; xb = (topc >> 8) & 0xFF; ob = (topc >> 16) & 0xFF; }
+        uint32_t XA = ((xa >> b) & 1u) ? ~0u : 0u, XB = ((xb >> b) & 1u) ? ~0u : 0u, OB = ((ob >> b) & 1u) ? ~0u : 0u;
+        wv[k][id] = (wv[k - 1][ca] ^ XA) & ((wv[k - 1][cb] ^ XB) | OB);
+      }
+    }
+    // write-outs: slot bit -> slot id within the unit
+    auto slot_of = [&](int unit_kind, uint32_t unit, uint32_t bit, int& k_out, uint32_t& id_out) {
+      static const int off[6] = {0, 0, 16, 24, 28, 30};
+      if (unit_kind == 2) {   // top
+        if (bit < 4) { k_out = 11; id_out = bit; } else if (bit < 6) { k_out = 12; id_out = bit - 4; }
+        else { k_out = 13; id_out = 0; }
+        return;
+      }
+      int kk = bit < 16 ? 1 : bit < 24 ? 2 : bit < 28 ? 3 : bit < 30 ? 4 : 5;
+      uint32_t q = bit - (uint32_t)off[kk];
+      k_out = unit_kind == 0 ? kk : kk + 5;
+      id_out = unit * gw(k_out) + q;
+    };
+    auto do_wo = [&](int kind, uint32_t unit, uint32_t mask, uint32_t base) -> int {
+      for (uint32_t bit = 0; bit < 31; bit++) {
+        if (!((mask >> bit) & 1u)) continue;
+        uint32_t word = base + (uint32_t)__builtin_popcount(mask & ((1u << bit) - 1u));
+        if (word == 0 || word >= S.size()) { g_err = "bad lane write-out"; return -1; }
+        if (read[word]) { g_err = "lane write-out target read in the same layer"; return -1; }
+        int k; uint32_t id;
+        slot_of(kind, unit, bit, k, id);
+        wo.push_back({word, wv[k][id]});
+      }
+      return 0;
+    };
+    for (uint32_t wp = 0; wp < 8; wp++) {
+      if (!((flags >> wp) & 1)) continue;
+      const uint32_t* rec = L + L[LLH_WOFF0 + wp];
+      for (uint32_t ln = 0; ln < 32; ln++)
+        if (do_wo(0, wp * 32 + ln, rec[GEM_LWREC_HDR + ln * 4 + 3], rec[GEM_LWREC_BASE + ln])) return -1;
+      if (do_wo(1, wp, rec[3], rec[4])) return -1;
+    }
+    if (do_wo(2, 0, L[LLH_TOPWO] & 0x7F, L[LLH_TOPWO] >> 8)) return -1;
+    for (auto& x : wo) S[x.first] = x.second;
+    L += L[LLH_WORDS_];
+  }
+  // outputs
+  const uint32_t* od = pr + pr[LPH_OFF_OUT];
+  std::vector<uint32_t> ramp(GEM_MAX_RAMS_PER_PART * 4 * 32, 0);
+  for (uint32_t j = 0; j < pr[LPH_N_OUT]; j++) {
+    uint32_t dst = od[2 * j], src = od[2 * j + 1];
+    uint32_t v = S[src & 0xFFFF] ^ ((src >> 31) ? ~0u : 0u);
+    uint32_t reg = dst >> 24, b = dst & 0xFFFFFF;
+    if (reg == GEM_R_Q) Ls.Q[nxt][b] = v;
+    else if (reg == GEM_R_PO) po_lane[b] = v;
+    else if (reg == GEM_R_CUT) Ls.CUT[b] = v;
+    else if (reg == GEM_R_RAMP) ramp[b] = v;
+    else { g_err = "bad lane out"; return -1; }
+  }
+  const uint32_t* rr = pr + pr[LPH_OFF_RAM];
+  for (uint32_t r = 0; r < pr[LPH_N_RAM]; r++) {
+    uint32_t id = rr[4 * r];
+    for (uint32_t st = 0; st < 32; st++) {
+      auto num = [&](uint32_t port, int bits) {
+        uint32_t v = 0;
+        for (int k = 0; k < bits; k++) v |= ((ramp[(r * 4 + port) * 32 + k] >> st) & 1u) << k;
+        return v;
+      };
+      uint32_t ra = num(0, 13), wa = num(1, 13), wd = num(2, 32), be = num(3, 32);
+      auto& M = Ls.MEM[st * I.n_rams + id];
+      uint32_t old = M[ra];
+      M[wa] = (M[wa] & ~be) | (wd & be);
+      for (int k = 0; k < 32; k++) {
+        uint32_t& word = Ls.RD[nxt][id * 32 + k];
+        word = (word & ~(1u << st)) | (((old >> k) & 1u) << st);
+      }
+    }
+  }
+  return 0;
+}
 }  // namespace
 
 extern "C" {
@@ -194,6 +353,56 @@ void* isa_load(const void* blob, size_t nbytes) {
 }
 
 void isa_free(void* h) { delete (Interp*)h; }
+
+// 32 streams in lane mode: stim [32][cycles][pi_words]; po_ext [32][cycles][ceil(n_po/32)];
+// q_ext [32][cycles][ceil(n_flops/32)]
+int isa_run_lanes(void* h, const uint32_t* stim, uint64_t cycles, uint32_t* po_ext, uint32_t* q_ext_tr) {
+  Interp& I = *(Interp*)h;
+  if (!I.w[GH_HAS_LANES]) { g_err = "blob has no lane programs"; return -1; }
+  LaneSim Ls;
+  for (int b = 0; b < 2; b++) { Ls.Q[b].assign(I.q_words * 32, 0); Ls.RD[b].assign(I.n_rams * 32, 0); }
+  for (uint32_t bit = 0; bit < I.q_words * 32; bit++)
+    Ls.Q[0][bit] = ((I.flop_init[bit / 32] >> (bit % 32)) & 1u) ? ~0u : 0u;
+  Ls.CUT.assign(I.cut_words * 32, 0);
+  Ls.MEM.assign((size_t)32 * I.n_rams, std::vector<uint32_t>(GEM_RAM_WORDS, 0));
+  uint32_t pwe = (I.n_po + 31) / 32, qwe = (I.n_flops + 31) / 32;
+  std::vector<uint32_t> pi_lane(I.pi_words * 32), po_lane(I.po_words * 32);
+  uint64_t c0 = I.cycle;
+  for (uint64_t t = 0; t < cycles; t++) {
+    for (uint32_t b = 0; b < I.pi_words * 32; b++) {
+      uint32_t v = 0;
+      for (uint32_t st = 0; st < 32; st++)
+        v |= ((stim[(st * cycles + t) * I.pi_words + b / 32] >> (b % 32)) & 1u) << st;
+      pi_lane[b] = v;
+    }
+    std::fill(po_lane.begin(), po_lane.end(), 0);
+    for (uint32_t s = 0; s < I.n_stages; s++)
+      for (uint32_t k = I.stages[s]; k < I.stages[s + 1]; k++)
+        if (run_lane_part(I, Ls, I.stages[I.n_stages + 1 + k], pi_lane.data(), po_lane.data())) return -1;
+    I.cycle++;
+    uint32_t cur = (uint32_t)(I.cycle & 1);
+    for (uint32_t st = 0; st < 32; st++) {
+      uint32_t* row = po_ext + (st * cycles + t) * pwe;
+      std::memset(row, 0, pwe * 4);
+      for (uint32_t b = 0; b < I.po_words * 32; b++) {
+        uint32_t e = I.po_ext[b];
+        if (e == 0xFFFFFFFFu) continue;
+        row[e / 32] |= ((po_lane[b] >> st) & 1u) << (e % 32);
+      }
+      if (q_ext_tr) {
+        uint32_t* qr = q_ext_tr + (st * cycles + t) * qwe;
+        std::memset(qr, 0, qwe * 4);
+        for (uint32_t b = 0; b < I.q_words * 32; b++) {
+          uint32_t e = I.q_ext[b];
+          if (e == 0xFFFFFFFFu) continue;
+          qr[e / 32] |= ((Ls.Q[cur][b] >> st) & 1u) << (e % 32);
+        }
+      }
+    }
+  }
+  (void)c0;
+  return 0;
+}
 
 // stim [cycles][pi_words] ; po_ext [cycles][ceil(n_po/32)] ; q_ext [cycles][ceil(n_flops/32)] (nullable)
 int isa_run(void* h, const uint32_t* stim, uint64_t cycles, uint32_t* po_ext, uint32_t* q_ext_tr) {

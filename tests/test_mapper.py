@@ -75,3 +75,28 @@ def test_blob_stats_c2():
     assert i.max_layers >= 40 / 13          # cannot beat 13 levels per layer
     assert i.max_layers <= 40               # boomerang layers are fewer than levels
     assert i.max_state_words <= 2048
+
+
+@pytest.mark.parametrize("opts", ["parts=1 lanes=1", "parts=4 lanes=1", "parts=5 stages=2 lanes=1"])
+def test_lane_programs_match_oracle_lanes(tmp_path, opts):
+    """Lane-mode programs (32 streams per lane word) through the CPU ISA
+    interpreter == the oracle's 64-lane batched mode, stream by stream."""
+    net = circuits.small_G(seed=23, n_and=4000, with_ram=True)
+    p = circuits.save(net, str(tmp_path), "g")
+    b = compile_file(p, opts)
+    st = np.stack([stim_random(net.n_pi, 80, 500 + s, reset_pi0_cycles=2) for s in range(32)])
+    po, q = IsaInterp(b).run_lanes(st)
+    o = Oracle(p)
+    o.lanes_reset(1)
+    r = o.lanes_run(0, st)
+    assert np.array_equal(po, r["po"])
+
+
+def test_c5_lane_program_prefix():
+    from gen import stimulus_streams
+    st = stimulus_streams("c5", 256, 6, range(32))
+    po, q = IsaInterp(blob("c5")).run_lanes(st)
+    o = Oracle(eaig("c5"))
+    o.lanes_reset(1)
+    r = o.lanes_run(0, st)
+    assert np.array_equal(po, r["po"])
