@@ -74,29 +74,36 @@ __device__ __forceinline__ void exec_lane_layer(const LaneRegs& R, uint32_t s_ba
         v[8 * g + 2 * k] = lds(s_base + 4u * (q8[g][k] & 0xFFFFu));
         v[8 * g + 2 * k + 1] = lds(s_base + 4u * (q8[g][k] >> 16));
       }
-    // levels 1-5 inside the thread; write-outs as each level completes
+    // levels 1-5 inside the thread.  Written slots go to consecutive lane words
+    // in slot-bit order: a running store pointer advanced per written slot.
+    uint32_t wp = s_base + 4u * R.base;
+#define LWO(b_, v_)                                   \
+  do {                                              \
+    if (mask & (1u << (b_))) { sts(wp, (v_)); wp += 4u; } \
+  } while (0)
 #pragma unroll
-    for (uint32_t q = 0; q < 16; q++) {
-      v[q] = lslot(v[q], v[q + 16], xa, xb, ob, q);
-      lane_wo(s_base, mask, R.base, q, v[q]);
+    for (uint32_t q = 0; q < 16; q++) v[q] = lslot(v[q], v[q + 16], xa, xb, ob, q);
+    if (mask & 0xFFFFu) {
+#pragma unroll
+      for (uint32_t q = 0; q < 16; q++) LWO(q, v[q]);
     }
 #pragma unroll
-    for (uint32_t q = 0; q < 8; q++) {
-      v[q] = lslot(v[q], v[q + 8], xa, xb, ob, 16 + q);
-      lane_wo(s_base, mask, R.base, 16 + q, v[q]);
-    }
+    for (uint32_t q = 0; q < 8; q++) v[q] = lslot(v[q], v[q + 8], xa, xb, ob, 16 + q);
 #pragma unroll
-    for (uint32_t q = 0; q < 4; q++) {
-      v[q] = lslot(v[q], v[q + 4], xa, xb, ob, 24 + q);
-      lane_wo(s_base, mask, R.base, 24 + q, v[q]);
-    }
+    for (uint32_t q = 0; q < 4; q++) v[8 + q] = lslot(v[q], v[q + 4], xa, xb, ob, 24 + q);
 #pragma unroll
-    for (uint32_t q = 0; q < 2; q++) {
-      v[q] = lslot(v[q], v[q + 2], xa, xb, ob, 28 + q);
-      lane_wo(s_base, mask, R.base, 28 + q, v[q]);
+    for (uint32_t q = 0; q < 2; q++) v[12 + q] = lslot(v[8 + q], v[8 + q + 2], xa, xb, ob, 28 + q);
+    uint32_t x = lslot(v[12], v[13], xa, xb, ob, 30);
+    if (mask & 0x7FFF0000u) {
+#pragma unroll
+      for (uint32_t q = 0; q < 8; q++) LWO(16 + q, v[q]);
+#pragma unroll
+      for (uint32_t q = 0; q < 4; q++) LWO(24 + q, v[8 + q]);
+      LWO(28, v[12]);
+      LWO(29, v[13]);
+      LWO(30, x);
     }
-    uint32_t x = lslot(v[0], v[1], xa, xb, ob, 30);
-    lane_wo(s_base, mask, R.base, 30, x);
+#undef LWO
     // levels 6-10 across the warp: slot q of a level lives in lane q
     const uint32_t wxa = R.wc.x, wxb = R.wc.y, wob = R.wc.z, wmask = R.wc.w;
     const uint32_t offs[5] = {0, 16, 24, 28, 30};
@@ -273,7 +280,7 @@ __device__ void record_state_lane(const KParams& kp, uint32_t c, uint32_t buf) {
   }
 }
 
-__global__ void __launch_bounds__(GEM_THREADS, 1) gem_lane_kernel(const KParams kp) {
+__global__ void __launch_bounds__(GEM_THREADS, 2) gem_lane_kernel(const KParams kp) {
   extern __shared__ __align__(16) uint32_t smem[];
   // layout: S[lane_words] | area (ring) | ctab[256] | ramp[ram_words] | topv[16] | mbar[8 x u64]
   uint32_t* S = smem;                                   // [group][lane words]

@@ -933,45 +933,49 @@ static int plan_launch(gem_sim* sim, uint32_t max_chunk_words, uint32_t grid_lim
 // Lane mode launch: one CTA per SM (all shared memory for the lane state and
 // the program ring), work items = (partition, 32-stream group), LPT lists.
 static int plan_launch_lanes(gem_sim* sim, uint32_t grid_limit) {
-  int sms = 0, coop = 0, optin = 0;
+  int sms = 0, coop = 0, optin = 0, per_sm = 0;
   CK(cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, sim->device));
   CK(cudaDeviceGetAttribute(&coop, cudaDevAttrCooperativeLaunch, sim->device));
   CK(cudaDeviceGetAttribute(&optin, cudaDevAttrMaxSharedMemoryPerBlockOptin, sim->device));
+  CK(cudaDeviceGetAttribute(&per_sm, cudaDevAttrMaxSharedMemoryPerMultiprocessor, sim->device));
   if (!coop) return fail(GEM_E_UNSUPPORTED, "device lacks cooperative launch");
   sim->sm_count = (uint32_t)sms;
   const uint32_t slot = (sim->lane_max_chunk + 3u) & ~3u;
-  // 32-stream groups per work item: as many as fit beside a 4-slot ring (GEM_LANE_GROUPS overrides)
-  uint32_t gl = 1;
-  {
-    const char* e = getenv("GEM_LANE_GROUPS");
-    const uint32_t want = e ? (uint32_t)atoi(e) : 4;
-    for (uint32_t k = std::max<uint32_t>(1, std::min(want, sim->n_groups)); k >= 1; k--) {
-      const uint64_t words = (uint64_t)k * (sim->lane_words + sim->ramp_words + 16) + GEM_MAX_CHUNKS + 16 + 4 * slot;
-      if (words * 4 <= (uint64_t)optin || k == 1) { gl = k; break; }
+  const char* ge = getenv("GEM_LANE_GROUPS");
+  const char* be = getenv("GEM_LANE_BPS");
+  const uint32_t want_gl = ge ? (uint32_t)atoi(ge) : 4;
+  // prefer 2 CTAs per SM (16 warps to hide latency), then as many 32-stream
+  // groups per work item as fit beside a >= 2-slot ring
+  uint32_t bps = 0, gl = 0, budget = 0;
+  for (uint32_t b = 2; b >= 1 && !bps; b--) {
+    if (be && (uint32_t)atoi(be) != b) continue;
+    const uint32_t bud = (uint32_t)std::min<int64_t>(optin, per_sm / (int64_t)b - 1024);
+    for (uint32_t k = std::max<uint32_t>(1, std::min(want_gl, sim->n_groups)); k >= 1; k--) {
+      const uint64_t words = (uint64_t)k * (sim->lane_words + sim->ramp_words + 16) + GEM_MAX_CHUNKS + 16 + 2 * slot;
+      if (words * 4 <= bud) { bps = b; gl = k; budget = bud; break; }
     }
   }
+  if (!bps) return fail(GEM_E_UNSUPPORTED, "lane state + 2 ring slots exceed shared memory");
   sim->lane_groups = gl;
   sim->group = 32 * gl;    // streams per work item
   sim->max_items = 0;
   for (uint32_t s = 0; s < sim->n_stages; s++)
     sim->max_items = std::max(sim->max_items, (sim->h_stage[s + 1] - sim->h_stage[s]) * ((sim->n_groups + gl - 1) / gl));
   const uint32_t fixed_words = gl * (sim->lane_words + sim->ramp_words + 16) + GEM_MAX_CHUNKS + 16;
-  if ((uint64_t)(fixed_words + 2 * slot) * 4 > (uint64_t)optin)
-    return fail(GEM_E_UNSUPPORTED, "lane state + 2 ring slots exceed shared memory");
-  const uint32_t area = (uint32_t)(optin / 4) - fixed_words;
+  const uint32_t area = budget / 4 - fixed_words;
   uint32_t ring = std::min<uint32_t>(GEM_RING_MAX, area / std::max<uint32_t>(slot, 4));
   ring = ring >= 4 ? 4 : 2;
-  uint32_t grid = std::max<uint32_t>(1, std::min<uint32_t>(sim->max_items, (uint32_t)sms));
+  uint32_t grid = std::max<uint32_t>(1, std::min<uint32_t>(sim->max_items, bps * (uint32_t)sms));
   if (grid_limit) grid = std::max<uint32_t>(1, std::min(grid, grid_limit));
   const uint32_t smem = (fixed_words + ring * slot) * 4;
   CK(cudaFuncSetAttribute(gem_lane_kernel, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem));
   int occ = 0;
   CK(cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ, gem_lane_kernel, GEM_THREADS, smem));
-  if (occ < 1) return fail(GEM_E_UNSUPPORTED, "lane kernel cannot be resident");
+  if ((uint32_t)occ < bps) return fail(GEM_E_UNSUPPORTED, "lane kernel cannot be co-resident");
   std::vector<uint32_t> off;
   std::vector<uint2> items;
   build_worklists(sim, grid, off, items);
-  sim->blocks_per_sm = 1;
+  sim->blocks_per_sm = bps;
   sim->grid = grid;
   sim->area_words = ring * slot;
   sim->ring_slots = ring;
