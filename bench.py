@@ -213,7 +213,7 @@ def main():
     ap.add_argument("--streams", type=int, default=0,
                     help="TOTAL stimulus streams over all GPUs (0 = 1 per GPU, or 4096 for c5)")
     ap.add_argument("--cycles", type=int, default=0,
-                    help="simulated cycles per step (0 = 1000; 200 for c4; 20 for c5)")
+                    help="simulated cycles per step (0 = 1000; 200 for c4; 100 for c5)")
     ap.add_argument("--no-cpu-baseline", action="store_true")
     ap.add_argument("--no-flush", action="store_true")
     ap.add_argument("--map-opts", default=None)
@@ -253,7 +253,7 @@ def main():
     info = blob_info(b)
     stream = torch.cuda.current_stream(dev)
     sim = gem.Simulator(b, device=dev.index, n_streams=S, cuda_stream=stream.cuda_stream, flags=gem.GEM_F_ASYNC)
-    C = args.cycles or {"c4": 200, "c5": 20}.get(cfg, 1000)
+    C = args.cycles or {"c4": 200, "c5": 100}.get(cfg, 1000)
     gstreams = list(range(s_start, s_start + S))
     # inputs for (warmup + steps), pre-generated on the host, uploaded per step
     n_steps = args.warmup + args.steps
