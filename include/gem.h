@@ -63,7 +63,7 @@ typedef struct {
   uint32_t n_pi, n_po, n_flops, n_rams, n_parts, n_stages, max_layers, total_layers;
   uint32_t pi_words, po_words, q_words;   /* external word counts per cycle/stream */
   uint32_t grid, blocks_per_sm, smem_bytes, n_streams;
-  uint32_t resident;     /* 1 = every CTA's programs live in its shared memory */
+  uint32_t resident;     /* CTAs whose programs all live in their shared memory */
   uint32_t ring_slots;   /* else: TMA ring depth used to stream program chunks */
   uint32_t group;        /* streams per work item (program chunks reused across them) */
   uint32_t lanes;        /* 1 = stream-sliced lane mode (32 streams per lane word)  */

@@ -59,7 +59,7 @@ __device__ __forceinline__ void lane_wo(uint32_t s_base, uint32_t mask, uint32_t
 }
 
 // Rows a3-a5 of one layer for one 32-stream group.  topv: 8 warp results + counter.
-__device__ __forceinline__ void exec_lane_layer(const LaneRegs& R, uint32_t s_base, uint32_t* topv) {
+__device__ __forceinline__ void exec_lane_layer(const LaneRegs& R, uint32_t s_base, uint32_t* topv, uint32_t bid) {
   const uint32_t lane = threadIdx.x & 31, warp = threadIdx.x >> 5;
   const bool uses_top = (R.flags & GEM_LF_USES_TOP) != 0;
   if ((R.flags >> warp) & 1u) {
@@ -119,12 +119,13 @@ __device__ __forceinline__ void exec_lane_layer(const LaneRegs& R, uint32_t s_ba
   } else if (uses_top && lane == 0) {
     topv[warp] = 0u;
   }
-  // levels 11-13: the last warp to arrive folds the 8 warp words
-  if (uses_top && lane == 0) {
-    __threadfence_block();
-    if (atomicAdd(&topv[8], 1u) == GEM_WARPS - 1) {
-      __threadfence_block();
-      volatile uint32_t* tv = topv;
+  // levels 11-13: warps 1-7 arrive on named barrier `bid`; warp 0 waits and
+  // folds the 8 warp words (the layer's closing barrier orders the write-outs)
+  if (uses_top && warp != 0) asm volatile("bar.arrive %0, %1;" ::"r"(bid), "r"(GEM_THREADS) : "memory");
+  if (uses_top && warp == 0) {
+    asm volatile("bar.sync %0, %1;" ::"r"(bid), "r"(GEM_THREADS) : "memory");
+    if (lane == 0) {
+      const uint32_t* tv = topv;
       const uint32_t xa = R.topc & 0xFFu, xb = (R.topc >> 8) & 0xFFu, ob = (R.topc >> 16) & 0xFFu;
       const uint32_t tm = R.topwo & 0x7Fu, tb = R.topwo >> 8;
       uint32_t t11[4];
@@ -140,7 +141,6 @@ __device__ __forceinline__ void exec_lane_layer(const LaneRegs& R, uint32_t s_ba
         lane_wo(s_base, tm, tb, 4 + q, t12[q]);
       }
       lane_wo(s_base, tm, tb, 6, lslot(t12[0], t12[1], xa, xb, ob, 6));
-      topv[8] = 0u;
     }
   }
 }
@@ -198,7 +198,10 @@ __device__ void run_lane_partition(const KParams& kp, ProgSrc& ps, uint32_t* S, 
   ps.seq_free += n_layers ? 2 : 1;
   refill();
   for (uint32_t l = 0; l < n_layers; l++) {
-    for (uint32_t j = 0; j < ng; j++) exec_lane_layer(R, s_base + 4u * j * LW, topv + 16 * j);
+    for (uint32_t j = 0; j < ng; j++) {   // named barrier ids as in run_partition
+      exec_lane_layer(R, s_base + 4u * j * LW, topv + 16 * j, 1 + j % 15);
+      if (j % 15 == 14 && j + 1 < ng) __syncthreads();
+    }
     if (l + 1 < n_layers) load_lane_layer(ring_wait(ps), R);
     __syncthreads();
     if (l + 1 < n_layers) ps.seq_free++;

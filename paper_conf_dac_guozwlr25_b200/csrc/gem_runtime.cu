@@ -67,6 +67,17 @@ struct KParams {
   const uint2* __restrict__ wl_items;    // {partition, stream} per work item
 };
 #ifdef GEM_FINE_PROF
+__device__ unsigned long long* g_fine_sub;   // [layer 8][warp 8][4] sub-stamps inside exec_layer
+__device__ uint32_t g_fine_on;
+#define FSUB(l_, k_)                                                                          \
+  do {                                                                                        \
+    if (g_fine_on && (threadIdx.x & 31) == 0 && (l_) < 8)                                     \
+      g_fine_sub[((l_) * 8 + (threadIdx.x >> 5)) * 4 + (k_)] = clock64();                     \
+  } while (0)
+#else
+#define FSUB(l_, k_) do { } while (0)
+#endif
+#ifdef GEM_FINE_PROF
 // debug build only: per-warp stamps inside the first 8 layers of cycle 5, CTA 0
 #define FPROF(l_, slot_)                                                                      \
   do {                                                                                        \
@@ -256,15 +267,16 @@ __device__ __forceinline__ uint32_t leaf_rot(uint32_t s_base, uint32_t e, uint32
 }
 template <int N4>
 __device__ __forceinline__ uint32_t gather_sparse(uint32_t s_base, const uint4* e) {
-  uint32_t v = 0;
+  // four independent accumulators keep the OR chain short
+  uint32_t v0 = 0, v1 = 0, v2 = 0, v3 = 0;
 #pragma unroll
   for (int g = 0; g < N4; g++) {
-    v |= leaf_rot(s_base, e[g].x, 0x7FFFu) & (1u << GEM_LEAF_POS(e[g].x));
-    v |= leaf_rot(s_base, e[g].y, 0x7FFFu) & (1u << GEM_LEAF_POS(e[g].y));
-    v |= leaf_rot(s_base, e[g].z, 0x7FFFu) & (1u << GEM_LEAF_POS(e[g].z));
-    v |= leaf_rot(s_base, e[g].w, 0x7FFFu) & (1u << GEM_LEAF_POS(e[g].w));
+    v0 |= leaf_rot(s_base, e[g].x, 0x7FFFu) & (1u << GEM_LEAF_POS(e[g].x));
+    v1 |= leaf_rot(s_base, e[g].y, 0x7FFFu) & (1u << GEM_LEAF_POS(e[g].y));
+    v2 |= leaf_rot(s_base, e[g].z, 0x7FFFu) & (1u << GEM_LEAF_POS(e[g].z));
+    v3 |= leaf_rot(s_base, e[g].w, 0x7FFFu) & (1u << GEM_LEAF_POS(e[g].w));
   }
-  return v;
+  return (v0 | v1) | (v2 | v3);
 }
 
 // Per-thread registers of one layer record: everything that does not depend
@@ -295,14 +307,17 @@ __device__ __forceinline__ void load_layer(const uint32_t* L, LayerRegs& R) {
 
 // Rows a3-a5 of one layer with pre-loaded records: gather (bit permutation),
 // 13-level boomerang fold, write-outs.  No trailing barrier.
-__device__ __forceinline__ void exec_layer(const LayerRegs& R, uint32_t s_base, uint32_t* topb) {
+__device__ __forceinline__ void exec_layer(const LayerRegs& R, uint32_t s_base, uint32_t* topb, uint32_t bid,
+                                           uint32_t fl = 99) {
   const uint32_t lane = threadIdx.x & 31, warp = threadIdx.x >> 5;
+  (void)fl;
   const bool uses_top = (R.flags & GEM_LF_USES_TOP) != 0;
   if ((R.flags >> warp) & 1u) {
     uint32_t v = 0;
     const uint32_t n4 = R.mode >> 8;
     if ((R.mode & 0xFFu) == GEM_WM_DENSE16) {
       // two 16-bit entries per u32: entry 8g+2k in the low half, 8g+2k+1 in the high half
+      uint32_t acc[4] = {0u, 0u, 0u, 0u};
 #pragma unroll
       for (uint32_t g = 0; g < 4; g++) {
         const uint32_t q[4] = {R.e[g].x, R.e[g].y, R.e[g].z, R.e[g].w};
@@ -310,10 +325,11 @@ __device__ __forceinline__ void exec_layer(const LayerRegs& R, uint32_t s_base, 
         for (uint32_t k = 0; k < 4; k++) {
           const uint32_t lo = lds(s_base + ((q[k] >> 3) & 0x1FFCu));
           const uint32_t hi = lds(s_base + ((q[k] >> 19) & 0x1FFCu));
-          v |= __funnelshift_l(lo, lo, q[k]) & (1u << (8 * g + 2 * k));
-          v |= __funnelshift_l(hi, hi, q[k] >> 16) & (1u << (8 * g + 2 * k + 1));
+          acc[k] |= (__funnelshift_l(lo, lo, q[k]) & (1u << (8 * g + 2 * k))) |
+                    (__funnelshift_l(hi, hi, q[k] >> 16) & (1u << (8 * g + 2 * k + 1)));
         }
       }
+      v = (acc[0] | acc[1]) | (acc[2] | acc[3]);
     } else if ((R.mode & 0xFFu) == GEM_WM_DENSE) {
       // entry j of the lane fills leaf position j: rotate + LOP3 with an immediate mask
 #pragma unroll
@@ -332,10 +348,13 @@ __device__ __forceinline__ void exec_layer(const LayerRegs& R, uint32_t s_base, 
     } else {
       v = gather_sparse<8>(s_base, R.e);
     }
+    FSUB(fl, 0);
     const uint32_t P = fold5(v, R.lc.x, R.lc.y, R.lc.z);
     if (R.lc.w) sts(s_base + 4 * R.lc.w, P);
+    FSUB(fl, 1);
     const uint32_t u = __ballot_sync(0xFFFFFFFFu, (P >> 30) & 1u);
     const uint32_t Pw = fold5(u, R.wc.x, R.wc.y, R.wc.z);
+    FSUB(fl, 2);
     if (lane == 0) {
       if (R.wc.w) sts(s_base + 4 * R.wc.w, Pw);
       if (uses_top) topb[warp] = (Pw >> 30) & 1u;
@@ -343,18 +362,23 @@ __device__ __forceinline__ void exec_layer(const LayerRegs& R, uint32_t s_base, 
   } else if (uses_top && lane == 0) {
     topb[warp] = 0u;
   }
-  // levels 11-13: the last warp to arrive folds the 8 warp bits (no extra barrier)
-  if (uses_top && lane == 0) {
-    __threadfence_block();
-    if (atomicAdd(&topb[8], 1u) == GEM_WARPS - 1) {
-      __threadfence_block();
-      uint32_t t8 = 0;
+  // levels 11-13: warps 1-7 arrive (non-blocking) on named barrier `bid` after
+  // publishing their level-10 bit; warp 0 waits there and folds the 8 bits.
+  // The layer's closing __syncthreads orders the write-out before the next gather.
+  if (uses_top) {
+    if (warp == 0) {
+      asm volatile("bar.sync %0, %1;" ::"r"(bid), "r"(GEM_THREADS) : "memory");
+      if (lane == 0) {
+        uint32_t t8 = 0;
 #pragma unroll
-      for (uint32_t w = 0; w < GEM_WARPS; w++) t8 |= *((volatile uint32_t*)topb + w) << w;
-      sts(s_base + 4 * R.topwo, fold3(t8, R.topc & 0xFFu, (R.topc >> 8) & 0xFFu, (R.topc >> 16) & 0xFFu));
-      topb[8] = 0u;
+        for (uint32_t w = 0; w < GEM_WARPS; w++) t8 |= topb[w] << w;
+        sts(s_base + 4 * R.topwo, fold3(t8, R.topc & 0xFFu, (R.topc >> 8) & 0xFFu, (R.topc >> 16) & 0xFFu));
+      }
+    } else {
+      asm volatile("bar.arrive %0, %1;" ::"r"(bid), "r"(GEM_THREADS) : "memory");
     }
   }
+  FSUB(fl, 3);
 }
 
 // One work item = one partition for a group of `nst` streams (states S_j =
@@ -434,7 +458,16 @@ __device__ void run_partition(const KParams& kp, ProgSrc& ps, uint32_t* S, uint3
   // into registers before the barrier that ends layer l
   for (uint32_t l = 0; l < n_layers; l++) {
     FPROF(l, 0);
-    for (uint32_t j = 0; j < nst; j++) exec_layer(R, s_base + 4 * j * SW, topb + 16 * j);
+#ifdef GEM_FINE_PROF
+    if (threadIdx.x == 0) g_fine_on = (kp.fprof && c == 5 && blockIdx.x == 0) ? 1u : 0u;
+    __syncwarp();
+#endif
+    // stream j uses named barrier 1 + j % 15; a full barrier every 15 streams
+    // keeps warps 1-7 from lapping warp 0 on a barrier id
+    for (uint32_t j = 0; j < nst; j++) {
+      exec_layer(R, s_base + 4 * j * SW, topb + 16 * j, 1 + j % 15, l);
+      if (j % 15 == 14 && j + 1 < nst) __syncthreads();
+    }
     FPROF(l, 1);
     const uint32_t flags = R.flags, topc = R.topc, topwo = R.topwo;
     if (l + 1 < n_layers) {
@@ -885,28 +918,31 @@ static int plan_launch(gem_sim* sim, uint32_t max_chunk_words, uint32_t grid_lim
     CK(cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ, gem_step_kernel, GEM_THREADS, (size_t)budget));
     if ((uint32_t)occ < bps) continue;
     const double makespan = build_worklists(sim, grid, off, items);
-    // residency check for every CTA
-    bool res = allow_res;
-    for (uint32_t b = 0; b < grid && res; b++) {
+    // residency is decided per CTA (its work list's distinct programs fit in the area)
+    uint32_t n_res = 0;
+    for (uint32_t b = 0; b < grid && allow_res; b++) {
       std::vector<uint32_t> seen;
       uint64_t words = 0;
-      for (uint32_t s = 0; s < sim->n_stages && res; s++)
+      bool ok = true;
+      for (uint32_t s = 0; s < sim->n_stages && ok; s++)
         for (uint32_t k = off[(size_t)s * (grid + 1) + b]; k < off[(size_t)s * (grid + 1) + b + 1]; k++) {
           const uint32_t p = items[k].x;
           if (std::find(seen.begin(), seen.end(), p) != seen.end()) continue;
           seen.push_back(p);
           words += (sim->h_parts[(size_t)p * GP_WORDS + GP_PROG_LEN] + 3u) & ~3u;
-          if (seen.size() > GEM_MAX_RESIDENT || words > area) { res = false; break; }
+          if (seen.size() > GEM_MAX_RESIDENT || words > area) { ok = false; break; }
         }
+      n_res += ok;
     }
+    const bool res = n_res == grid;
     uint32_t ring = std::min<uint32_t>(GEM_RING_MAX, area / std::max<uint32_t>(slot, 4));
     ring = ring >= 4 ? 4 : ring >= 2 ? 2 : ring;   // power of two (kernel masks instead of dividing)
     if (!res && ring < 2) continue;
     // score: estimated makespan, SM sharing slows co-resident CTAs, streaming costs a little
     double score = makespan * (1.0 + 0.5 * (bps - 1) * std::min(1.0, (double)grid / ((double)bps * sms)))
-                   * (res ? 1.0 : 1.1);
+                   * (1.0 + 0.1 * (double)(grid - n_res) / grid);
     if (!best.bps || score < best.score) {
-      best.bps = bps; best.grid = grid; best.area = area; best.resident = res ? 1u : 0u; best.ring = ring;
+      best.bps = bps; best.grid = grid; best.area = area; best.resident = n_res; best.ring = ring;
       best.score = score;
       best_off.swap(off);
       best_items.swap(items);
@@ -1203,7 +1239,7 @@ int gem_step(gem_sim* sim, uint64_t ncycles) {
   kp.n_flops = sim->n_flops; kp.q_ext_words = sim->q_words_ext;
   kp.flags = sim->flags & (GEM_F_TRACE_STATE | GEM_F_DIGEST);
   kp.area_words = sim->area_words; kp.slot_words = sim->slot_words; kp.ring_slots = sim->ring_slots;
-  kp.allow_resident = sim->resident;
+  kp.allow_resident = sim->resident ? 1u : 0u;   // per-CTA decision in the kernel
   kp.wl_off = sim->d_wl_off;
   kp.group = sim->group;
   kp.wl_items = sim->d_wl_items;
@@ -1214,7 +1250,11 @@ int gem_step(gem_sim* sim, uint64_t ncycles) {
       sim->d_prof = nullptr;
       CK(dalloc(&sim->d_prof, (size_t)256 * sim->grid * 8 * 8 + 8 * 8 * 8 * 8));
 #ifdef GEM_FINE_PROF
-      CK(dalloc(&sim->d_fprof, 8 * 8 * 8 * 8));
+      CK(dalloc(&sim->d_fprof, 8 * 8 * 8 * 8 + 8 * 8 * 4 * 8));
+      {
+        unsigned long long* sub = sim->d_fprof + 8 * 8 * 8;
+        CK(cudaMemcpyToSymbol(g_fine_sub, &sub, sizeof(sub)));
+      }
 #endif
     }
     sim->prof_cycles = pc;
@@ -1398,7 +1438,7 @@ int gem_write_ram(gem_sim* sim, uint32_t ram_id, uint32_t stream, const uint32_t
 #ifdef GEM_FINE_PROF
 int gem_read_fine(gem_sim* sim, uint64_t* dst) {
   CK(cudaStreamSynchronize(sim->stream));
-  CK(cudaMemcpy(dst, sim->d_fprof, 8 * 8 * 8 * 8, cudaMemcpyDeviceToHost));
+  CK(cudaMemcpy(dst, sim->d_fprof, 8 * 8 * 8 * 8 + 8 * 8 * 4 * 8, cudaMemcpyDeviceToHost));
   return GEM_OK;
 }
 #endif

@@ -22,10 +22,11 @@ for cfg in sys.argv[1:] or ["c1"]:
     st = stimulus("c3" if cfg == "c5" else cfg, sim.info["n_pi"], 50)
     sim.set_inputs(st)
     sim.step(50)
-    out = np.zeros(8 * 8 * 8, np.uint64)
+    out = np.zeros(8 * 8 * 8 + 8 * 8 * 4, np.uint64)
     sim.lib.gem_read_fine.argtypes = [ctypes.c_void_p, ctypes.c_void_p]
     sim.lib.gem_read_fine(sim._h, out.ctypes.data_as(ctypes.c_void_p))
-    f = out.reshape(8, 8, 8).astype(np.int64)    # [layer][warp][slot]
+    f = out[:512].reshape(8, 8, 8).astype(np.int64)    # [layer][warp][slot]
+    sub = out[512:].reshape(8, 8, 4).astype(np.int64)  # [layer][warp][gather|fold5|ballot+fold5|wo+top]
     print(f"== {cfg}: per-layer, per-warp deltas (clocks): exec | wait_next | load_next | top | barrier")
     for l in range(8):
         if f[l, :, 0].max() == 0:
@@ -35,3 +36,11 @@ for cfg in sys.argv[1:] or ["c1"]:
         tot = f[l, :, 5].max() - f[l, :, 0].min()
         print(f"  L{l}: total {tot:5d}  exec {ex.min():4d}-{ex.max():4d}  wait {wt.max():4d}  load {ld.max():4d}  "
               f"top {tp.max():4d}  bar {br.min():4d}-{br.max():4d}")
+        act = sub[l, :, 0] > 0
+        if act.any():
+            g_ = sub[l, act, 0] - f[l, act, 0]
+            f1 = sub[l, act, 1] - sub[l, act, 0]
+            f2 = sub[l, act, 2] - sub[l, act, 1]
+            f3 = sub[l, act, 3] - sub[l, act, 2]
+            print(f"        active warps {act.sum()}: gather {g_.min()}-{g_.max()}  fold1 {f1.min()}-{f1.max()}  "
+                  f"ballot+fold2 {f2.min()}-{f2.max()}  wo+top {f3.min()}-{f3.max()}")
