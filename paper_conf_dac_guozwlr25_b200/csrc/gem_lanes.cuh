@@ -119,30 +119,29 @@ __device__ __forceinline__ void exec_lane_layer(const LaneRegs& R, uint32_t s_ba
   } else if (uses_top && lane == 0) {
     topv[warp] = 0u;
   }
-  // levels 11-13: warps 1-7 arrive on named barrier `bid`; warp 0 waits and
-  // folds the 8 warp words (the layer's closing barrier orders the write-outs)
+  // levels 11-13: warps 1-7 arrive on named barrier `bid`; warp 0 folds in
+  // top_lane_layer after loading the next layer's records
   if (uses_top && warp != 0) asm volatile("bar.arrive %0, %1;" ::"r"(bid), "r"(GEM_THREADS) : "memory");
-  if (uses_top && warp == 0) {
-    asm volatile("bar.sync %0, %1;" ::"r"(bid), "r"(GEM_THREADS) : "memory");
-    if (lane == 0) {
-      const uint32_t* tv = topv;
-      const uint32_t xa = R.topc & 0xFFu, xb = (R.topc >> 8) & 0xFFu, ob = (R.topc >> 16) & 0xFFu;
-      const uint32_t tm = R.topwo & 0x7Fu, tb = R.topwo >> 8;
-      uint32_t t11[4];
-#pragma unroll
-      for (uint32_t q = 0; q < 4; q++) {
-        t11[q] = lslot(tv[q], tv[q + 4], xa, xb, ob, q);
-        lane_wo(s_base, tm, tb, q, t11[q]);
-      }
-      uint32_t t12[2];
-#pragma unroll
-      for (uint32_t q = 0; q < 2; q++) {
-        t12[q] = lslot(t11[q], t11[q + 2], xa, xb, ob, 4 + q);
-        lane_wo(s_base, tm, tb, 4 + q, t12[q]);
-      }
-      lane_wo(s_base, tm, tb, 6, lslot(t12[0], t12[1], xa, xb, ob, 6));
-    }
-  }
+}
+
+// Levels 11-13 (warp 0): wait for the 8 warp words on named barrier `bid`;
+// lanes 0-7 hold them and three shuffle levels fold them.
+__device__ __forceinline__ void top_lane_layer(uint32_t topc, uint32_t topwo, uint32_t s_base, const uint32_t* topv,
+                                               uint32_t bid) {
+  asm volatile("bar.sync %0, %1;" ::"r"(bid), "r"(GEM_THREADS) : "memory");
+  const uint32_t lane = threadIdx.x & 31;
+  const uint32_t xa = topc & 0xFFu, xb = (topc >> 8) & 0xFFu, ob = (topc >> 16) & 0xFFu;
+  const uint32_t tm = topwo & 0x7Fu, tb = topwo >> 8;
+  uint32_t x = lds(smem_u32(topv) + 4u * (lane & 7u));
+  uint32_t y = __shfl_down_sync(0xFFFFFFFFu, x, 4);
+  x = lslot(x, y, xa, xb, ob, lane & 3u);                 // level 11: slots 0-3
+  if (lane < 4) lane_wo(s_base, tm, tb, lane, x);
+  y = __shfl_down_sync(0xFFFFFFFFu, x, 2);
+  x = lslot(x, y, xa, xb, ob, 4u + (lane & 1u));          // level 12: slots 4-5
+  if (lane < 2) lane_wo(s_base, tm, tb, 4u + lane, x);
+  y = __shfl_down_sync(0xFFFFFFFFu, x, 1);
+  x = lslot(x, y, xa, xb, ob, 6u);                        // level 13: slot 6
+  if (lane == 0) lane_wo(s_base, tm, tb, 6u, x);
 }
 
 // One work item: partition p for 32-stream group g (streams 32g .. 32g+nvalid-1).
@@ -176,20 +175,31 @@ __device__ void run_lane_partition(const KParams& kp, ProgSrc& ps, uint32_t* S, 
     }
   };
   // ---- a2: input ports (once per cycle) for the 32 streams of the group
+  // loads of 4 (entry, group) pairs per thread are issued before their stores
   const uint2* gr = reinterpret_cast<const uint2*>(gprog + off_gread);
-#pragma unroll 4
-  for (uint32_t k = tid; k < n_gread; k += GEM_THREADS) {
-    const uint2 e = __ldg(gr + k);
-    const uint32_t reg = e.x >> 24, b = e.x & 0xFFFFFFu;
-    for (uint32_t j = 0; j < ng; j++) {
-      const uint32_t g = g0 + j;
-      uint32_t v;
-      if (reg == GEM_R_PI) v = __ldg(kp.pi_lane + X.q(kp.in_base + c, kp.pi_words * 32, b, g));
-      else if (reg == GEM_R_Q) v = __ldcg(kp.q + X.q(cur, kp.q_words * 32, b, g));
-      else if (reg == GEM_R_RD) v = __ldcg(kp.rd + X.q(cur, kp.n_rams * 32, b, g));
-      else v = __ldcg(kp.cut + X.q(0, kp.cut_words * 32, b, g));
-      sts(s_base + 4u * (j * LW + e.y), v);
+  const uint32_t n_gr = n_gread * ng;
+  for (uint32_t k0 = 0; k0 < n_gr; k0 += 4 * GEM_THREADS) {
+    uint32_t v[4], dst[4];
+#pragma unroll
+    for (uint32_t u = 0; u < 4; u++) {
+      const uint32_t k = k0 + u * GEM_THREADS + tid;
+      dst[u] = ~0u;
+      if (k < n_gr) {
+        const uint32_t j = k / n_gread, g = g0 + j;
+        const uint2 e = __ldg(gr + (k - j * n_gread));
+        const uint32_t reg = e.x >> 24, b = e.x & 0xFFFFFFu;
+        const uint32_t* a;
+        if (reg == GEM_R_PI) a = kp.pi_lane + X.q(kp.in_base + c, kp.pi_words * 32, b, g);
+        else if (reg == GEM_R_Q) a = kp.q + X.q(cur, kp.q_words * 32, b, g);
+        else if (reg == GEM_R_RD) a = kp.rd + X.q(cur, kp.n_rams * 32, b, g);
+        else a = kp.cut + X.q(0, kp.cut_words * 32, b, g);
+        v[u] = __ldcg(a);
+        dst[u] = j * LW + e.y;
+      }
     }
+#pragma unroll
+    for (uint32_t u = 0; u < 4; u++)
+      if (dst[u] != ~0u) sts(s_base + 4u * dst[u], v[u]);
   }
   if (tid < ng) S[tid * LW] = 0u;
   LaneRegs R;
@@ -198,11 +208,13 @@ __device__ void run_lane_partition(const KParams& kp, ProgSrc& ps, uint32_t* S, 
   ps.seq_free += n_layers ? 2 : 1;
   refill();
   for (uint32_t l = 0; l < n_layers; l++) {
-    for (uint32_t j = 0; j < ng; j++) {   // named barrier ids as in run_partition
-      exec_lane_layer(R, s_base + 4u * j * LW, topv + 16 * j, 1 + j % 15);
-      if (j % 15 == 14 && j + 1 < ng) __syncthreads();
-    }
+    for (uint32_t j = 0; j < ng; j++)   // named barrier 1 + j, as in run_partition
+      exec_lane_layer(R, s_base + 4u * j * LW, topv + 16 * j, 1 + j);
+    const bool ptop = (R.flags & GEM_LF_USES_TOP) != 0;
+    const uint32_t ptopc = R.topc, ptopwo = R.topwo;
     if (l + 1 < n_layers) load_lane_layer(ring_wait(ps), R);
+    if (ptop && (threadIdx.x >> 5) == 0)
+      for (uint32_t j = 0; j < ng; j++) top_lane_layer(ptopc, ptopwo, s_base + 4u * j * LW, topv + 16 * j, 1 + j);
     __syncthreads();
     if (l + 1 < n_layers) ps.seq_free++;
     refill();

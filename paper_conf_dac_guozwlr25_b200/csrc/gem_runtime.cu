@@ -33,6 +33,10 @@ namespace {
 
 thread_local std::string g_err;
 
+// streams (packed) or 32-stream groups (lanes) per work item: each uses its own
+// named barrier 1..15 for the top levels (barrier 0 = __syncthreads)
+#define GEM_MAX_GROUP 15u
+
 struct KParams {
   const uint32_t* __restrict__ prog;
   const uint32_t* __restrict__ parts;       // part table [n_parts][4]
@@ -67,12 +71,12 @@ struct KParams {
   const uint2* __restrict__ wl_items;    // {partition, stream} per work item
 };
 #ifdef GEM_FINE_PROF
-__device__ unsigned long long* g_fine_sub;   // [layer 8][warp 8][4] sub-stamps inside exec_layer
-__device__ uint32_t g_fine_on;
+// sub-stamps inside exec_layer: fl = layer index when stamping, >= 8 otherwise;
+// fsub = kp.fprof + 512 ([layer 8][warp 8][4])
 #define FSUB(l_, k_)                                                                          \
   do {                                                                                        \
-    if (g_fine_on && (threadIdx.x & 31) == 0 && (l_) < 8)                                     \
-      g_fine_sub[((l_) * 8 + (threadIdx.x >> 5)) * 4 + (k_)] = clock64();                     \
+    if ((l_) < 8 && (threadIdx.x & 31) == 0)                                                  \
+      fsub[((l_) * 8 + (threadIdx.x >> 5)) * 4 + (k_)] = clock64();                           \
   } while (0)
 #else
 #define FSUB(l_, k_) do { } while (0)
@@ -106,7 +110,7 @@ __device__ __forceinline__ uint64_t globaltimer_ns() {
 }
 
 // Grid-wide barrier on a monotonically increasing 64-bit counter (reset to 0
-// before each launch).  Release: bar.sync + gpu-scope fence + atomic arrive.
+// before each launch).  Release: bar.sync + red.release.gpu arrive.
 // Acquire: ld.acquire.gpu spin, then bar.sync.  A 10 s spin limit turns a
 // deadlock (e.g. broken co-residency) into a trapped kernel instead of a hang.
 __device__ __forceinline__ void grid_sync(const KParams& kp, unsigned long long& target) {
@@ -114,8 +118,9 @@ __device__ __forceinline__ void grid_sync(const KParams& kp, unsigned long long&
   if (gridDim.x > 1) {
     if (threadIdx.x == 0) {
       target += gridDim.x;
-      __threadfence();
-      atomicAdd(kp.bar, 1ull);
+      // release at gpu scope, cumulative over the CTA's writes ordered before
+      // it by the bar.sync above (replaces fence.sc + returning atomic)
+      asm volatile("red.release.gpu.global.add.u64 [%0], 1;" ::"l"(kp.bar) : "memory");
       uint32_t spins = 0;
       uint64_t start = 0;
       while (ld_acquire_u64(kp.bar) < target) {
@@ -308,13 +313,15 @@ __device__ __forceinline__ void load_layer(const uint32_t* L, LayerRegs& R) {
 // Rows a3-a5 of one layer with pre-loaded records: gather (bit permutation),
 // 13-level boomerang fold, write-outs.  No trailing barrier.
 __device__ __forceinline__ void exec_layer(const LayerRegs& R, uint32_t s_base, uint32_t* topb, uint32_t bid,
-                                           uint32_t fl = 99) {
+                                           uint32_t fl = 99, unsigned long long* fsub = nullptr) {
   const uint32_t lane = threadIdx.x & 31, warp = threadIdx.x >> 5;
   (void)fl;
+  (void)fsub;
   const bool uses_top = (R.flags & GEM_LF_USES_TOP) != 0;
   if ((R.flags >> warp) & 1u) {
     uint32_t v = 0;
     const uint32_t n4 = R.mode >> 8;
+#ifndef EXP_NO_GATHER
     if ((R.mode & 0xFFu) == GEM_WM_DENSE16) {
       // two 16-bit entries per u32: entry 8g+2k in the low half, 8g+2k+1 in the high half
       uint32_t acc[4] = {0u, 0u, 0u, 0u};
@@ -348,12 +355,24 @@ __device__ __forceinline__ void exec_layer(const LayerRegs& R, uint32_t s_base, 
     } else {
       v = gather_sparse<8>(s_base, R.e);
     }
+#else   // timing experiment only (wrong results)
+    v = R.e[0].x ^ R.e[1].y ^ R.lc.w;
+    (void)n4;
+#endif
     FSUB(fl, 0);
+#ifndef EXP_NO_FOLD
     const uint32_t P = fold5(v, R.lc.x, R.lc.y, R.lc.z);
+#else
+    const uint32_t P = v ^ R.lc.x;
+#endif
     if (R.lc.w) sts(s_base + 4 * R.lc.w, P);
     FSUB(fl, 1);
     const uint32_t u = __ballot_sync(0xFFFFFFFFu, (P >> 30) & 1u);
+#ifndef EXP_NO_FOLD
     const uint32_t Pw = fold5(u, R.wc.x, R.wc.y, R.wc.z);
+#else
+    const uint32_t Pw = u ^ R.wc.x;
+#endif
     FSUB(fl, 2);
     if (lane == 0) {
       if (R.wc.w) sts(s_base + 4 * R.wc.w, Pw);
@@ -362,23 +381,29 @@ __device__ __forceinline__ void exec_layer(const LayerRegs& R, uint32_t s_base, 
   } else if (uses_top && lane == 0) {
     topb[warp] = 0u;
   }
-  // levels 11-13: warps 1-7 arrive (non-blocking) on named barrier `bid` after
-  // publishing their level-10 bit; warp 0 waits there and folds the 8 bits.
-  // The layer's closing __syncthreads orders the write-out before the next gather.
-  if (uses_top) {
-    if (warp == 0) {
-      asm volatile("bar.sync %0, %1;" ::"r"(bid), "r"(GEM_THREADS) : "memory");
-      if (lane == 0) {
-        uint32_t t8 = 0;
-#pragma unroll
-        for (uint32_t w = 0; w < GEM_WARPS; w++) t8 |= topb[w] << w;
-        sts(s_base + 4 * R.topwo, fold3(t8, R.topc & 0xFFu, (R.topc >> 8) & 0xFFu, (R.topc >> 16) & 0xFFu));
-      }
-    } else {
-      asm volatile("bar.arrive %0, %1;" ::"r"(bid), "r"(GEM_THREADS) : "memory");
-    }
-  }
+  // levels 11-13: warps 1-7 arrive (non-blocking) on named barrier `bid`
+  // after publishing their level-10 bit; warp 0 folds later (top_layer).
+#ifndef EXP_NO_TOP
+  if (uses_top && warp != 0) asm volatile("bar.arrive %0, %1;" ::"r"(bid), "r"(GEM_THREADS) : "memory");
+#endif
   FSUB(fl, 3);
+}
+
+// Levels 11-13 of a layer (warp 0 only): wait on named barrier `bid` for the
+// 8 level-10 bits, fold them and write the top word.  Called after warp 0 has
+// loaded the next layer's records; the layer's closing __syncthreads orders
+// the write-out before the next gather.  (Measured alternatives: a smem
+// atomic "last warp folds" costs ~2x; every warp folding redundantly after the
+// barrier costs ~+170 clocks per layer.)
+__device__ __forceinline__ void top_layer(uint32_t topc, uint32_t topwo, uint32_t s_base, const uint32_t* topb,
+                                          uint32_t bid) {
+  asm volatile("bar.sync %0, %1;" ::"r"(bid), "r"(GEM_THREADS) : "memory");
+  if ((threadIdx.x & 31) == 0) {
+    uint32_t t8 = 0;
+#pragma unroll
+    for (uint32_t w = 0; w < GEM_WARPS; w++) t8 |= topb[w] << w;
+    sts(s_base + 4 * topwo, fold3(t8, topc & 0xFFu, (topc >> 8) & 0xFFu, (topc >> 16) & 0xFFu));
+  }
 }
 
 // One work item = one partition for a group of `nst` streams (states S_j =
@@ -428,17 +453,32 @@ __device__ void run_partition(const KParams& kp, ProgSrc& ps, uint32_t* S, uint3
       }
   };
   // ---- a2: global read of input ports (once per cycle)
-  const uint32_t* gr = C0 + off_gread;
-  for (uint32_t k = tid; k < n_gread * nst; k += GEM_THREADS) {
-    const uint32_t j = k / n_gread, st = st0 + j;
-    const uint2 e = *(reinterpret_cast<const uint2*>(gr) + (k - j * n_gread));
-    const uint32_t reg = GEM_GID_REGION(e.x), idx = GEM_GID_INDEX(e.x);
-    uint32_t v;
-    if (reg == GEM_R_PI) v = __ldg(kp.pi + ((size_t)st * kp.in_cap + kp.in_base + c) * kp.pi_words + idx);
-    else if (reg == GEM_R_Q) v = rd_global(kp.q + ((size_t)cur * kp.n_streams + st) * kp.q_words + idx);
-    else if (reg == GEM_R_RD) v = rd_global(kp.rd + ((size_t)cur * kp.n_streams + st) * kp.n_rams + idx);
-    else v = rd_global(kp.cut + (size_t)st * kp.cut_words + idx);
-    S[j * SW + e.y] = v;
+  // 4 entries per thread per round: all loads are issued before the stores so
+  // their L2 latencies overlap
+  const uint2* gr = reinterpret_cast<const uint2*>(C0 + off_gread);
+  const uint32_t n_gr = n_gread * nst;
+  for (uint32_t k0 = 0; k0 < n_gr; k0 += 4 * GEM_THREADS) {
+    uint32_t v[4], dst[4];
+#pragma unroll
+    for (uint32_t u = 0; u < 4; u++) {
+      const uint32_t k = k0 + u * GEM_THREADS + tid;
+      dst[u] = ~0u;
+      if (k < n_gr) {
+        const uint32_t j = k / n_gread, st = st0 + j;
+        const uint2 e = gr[k - j * n_gread];
+        const uint32_t reg = GEM_GID_REGION(e.x), idx = GEM_GID_INDEX(e.x);
+        const uint32_t* a;
+        if (reg == GEM_R_PI) a = kp.pi + ((size_t)st * kp.in_cap + kp.in_base + c) * kp.pi_words + idx;
+        else if (reg == GEM_R_Q) a = kp.q + ((size_t)cur * kp.n_streams + st) * kp.q_words + idx;
+        else if (reg == GEM_R_RD) a = kp.rd + ((size_t)cur * kp.n_streams + st) * kp.n_rams + idx;
+        else a = kp.cut + (size_t)st * kp.cut_words + idx;
+        v[u] = rd_global(a);
+        dst[u] = j * SW + e.y;
+      }
+    }
+#pragma unroll
+    for (uint32_t u = 0; u < 4; u++)
+      if (dst[u] != ~0u) sts(s_base + 4 * dst[u], v[u]);
   }
   if (tid < nst) S[tid * SW] = 0u;
   // first layer's records (independent of S) before the barrier
@@ -452,33 +492,42 @@ __device__ void run_partition(const KParams& kp, ProgSrc& ps, uint32_t* S, uint3
   }
   __syncthreads();   // S ready; chunk 0 and layer 0's chunk consumed
   if (!ps.resident) ps.seq_free += n_layers ? 2 : 1;
-  PROF(1);
+  // (the S[0] read makes the stamp wait for the barrier release, which
+  // BAR.SYNC.DEFER_BLOCKING otherwise defers to the first dependent access)
+  if (prof_on && tid == 0 && lds(s_base) == 0u) PROF(1);
   refill();
   // ---- a3-a5: layers, software-pipelined: layer l+1's records are loaded
   // into registers before the barrier that ends layer l
   for (uint32_t l = 0; l < n_layers; l++) {
     FPROF(l, 0);
 #ifdef GEM_FINE_PROF
-    if (threadIdx.x == 0) g_fine_on = (kp.fprof && c == 5 && blockIdx.x == 0) ? 1u : 0u;
-    __syncwarp();
+    const uint32_t fl = (kp.fprof && c == 5 && blockIdx.x == 0) ? l : 99u;
+    unsigned long long* fsub = kp.fprof ? kp.fprof + 512 : nullptr;
+#else
+    const uint32_t fl = 99u;
+    unsigned long long* fsub = nullptr;
 #endif
-    // stream j uses named barrier 1 + j % 15; a full barrier every 15 streams
-    // keeps warps 1-7 from lapping warp 0 on a barrier id
-    for (uint32_t j = 0; j < nst; j++) {
-      exec_layer(R, s_base + 4 * j * SW, topb + 16 * j, 1 + j % 15, l);
-      if (j % 15 == 14 && j + 1 < nst) __syncthreads();
-    }
+    // stream j uses named barrier 1 + j (group <= GEM_MAX_GROUP < 16)
+    for (uint32_t j = 0; j < nst; j++) exec_layer(R, s_base + 4 * j * SW, topb + 16 * j, 1 + j, fl, fsub);
     FPROF(l, 1);
-    const uint32_t flags = R.flags, topc = R.topc, topwo = R.topwo;
+    const bool ptop = (R.flags & GEM_LF_USES_TOP) != 0;
+    const uint32_t ptopc = R.topc, ptopwo = R.topwo;
     if (l + 1 < n_layers) {
       const uint32_t* L;
       if (ps.resident) { L = Lres; Lres += ctab[2 + l]; }
       else L = ring_wait(ps);
       FPROF(l, 2);
+#ifndef EXP_NO_LOAD
       load_layer(L, R);
+#else
+      if (l == 0) load_layer(L, R);
+#endif
     }
     FPROF(l, 3);
-    (void)flags; (void)topc; (void)topwo;
+#ifndef EXP_NO_TOP
+    if (ptop && warp == 0)
+      for (uint32_t j = 0; j < nst; j++) top_layer(ptopc, ptopwo, s_base + 4 * j * SW, topb + 16 * j, 1 + j);
+#endif
     FPROF(l, 4);
     __syncthreads();
     FPROF(l, 5);
@@ -882,8 +931,8 @@ static int plan_launch(gem_sim* sim, uint32_t max_chunk_words, uint32_t grid_lim
   sim->group = 1;
   if (sim->n_streams > 1) {
     const char* genv = getenv("GEM_GROUP");
-    uint32_t g = genv ? (uint32_t)atoi(genv) : 16;
-    g = std::max<uint32_t>(1, std::min<uint32_t>(g, sim->n_streams));
+    uint32_t g = genv ? (uint32_t)atoi(genv) : GEM_MAX_GROUP;
+    g = std::max<uint32_t>(1, std::min<uint32_t>(std::min<uint32_t>(g, GEM_MAX_GROUP), sim->n_streams));
     while (g > 1 && (uint64_t)(g * (sim->state_words + 4 * GEM_MAX_RAMS_PER_PART + 16) + GEM_MAX_CHUNKS + 80 +
                                3 * slot) * 4 > (uint64_t)optin)
       g /= 2;
@@ -979,7 +1028,7 @@ static int plan_launch_lanes(gem_sim* sim, uint32_t grid_limit) {
   const uint32_t slot = (sim->lane_max_chunk + 3u) & ~3u;
   const char* ge = getenv("GEM_LANE_GROUPS");
   const char* be = getenv("GEM_LANE_BPS");
-  const uint32_t want_gl = ge ? (uint32_t)atoi(ge) : 4;
+  const uint32_t want_gl = std::min<uint32_t>(ge ? (uint32_t)atoi(ge) : 4, GEM_MAX_GROUP);
   // prefer 2 CTAs per SM (16 warps to hide latency), then as many 32-stream
   // groups per work item as fit beside a >= 2-slot ring
   uint32_t bps = 0, gl = 0, budget = 0;
@@ -1251,10 +1300,6 @@ int gem_step(gem_sim* sim, uint64_t ncycles) {
       CK(dalloc(&sim->d_prof, (size_t)256 * sim->grid * 8 * 8 + 8 * 8 * 8 * 8));
 #ifdef GEM_FINE_PROF
       CK(dalloc(&sim->d_fprof, 8 * 8 * 8 * 8 + 8 * 8 * 4 * 8));
-      {
-        unsigned long long* sub = sim->d_fprof + 8 * 8 * 8;
-        CK(cudaMemcpyToSymbol(g_fine_sub, &sub, sizeof(sub)));
-      }
 #endif
     }
     sim->prof_cycles = pc;

@@ -12,7 +12,7 @@ GH = ["MAGIC", "VERSION", "N_PI", "N_PO", "N_FLOPS", "N_RAMS", "N_PARTS", "N_STA
       "OFF_PROG", "PROG_WORDS_LO", "PROG_WORDS_HI", "MAX_LEVELS", "TOTAL_WRITEOUTS",
       "MAX_OUT", "TOTAL_WORDS_LO", "TOTAL_WORDS_HI", "SLOTS_USED_LO", "SLOTS_USED_HI",
       "MAX_CHUNK_WORDS", "MAX_PROG_WORDS"]
-GP_WORDS = 12
+GP_WORDS = 16   # csrc/gem_isa.h GP_WORDS
 GEM_MAGIC = 0x424D4547
 SLOTS_PER_LAYER = 8191
 

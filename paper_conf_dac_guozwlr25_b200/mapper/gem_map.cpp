@@ -56,6 +56,7 @@ struct Options {
   int part_size = 6000;     // auto target ANDs per partition (paper: 5.7-12.9K, Table I)
   int threads = 0;          // 0 = hardware concurrency
   int leafcap = 320;        // max leaves of one placed root (cost filter)
+  int levels = 13;          // deepest boomerang level used per layer (10 = no top levels 11-13)
   int stages = 1;           // 1 or 2 (multi-stage RepCut)
   int cut_level = 0;        // 0 = auto (middle)
   int merge = 1;            // Algorithm 1 merge pass
@@ -81,6 +82,7 @@ static Options parse_opts(const char* s) {
     else if (k == "part_size") o.part_size = std::stoi(v);
     else if (k == "threads") o.threads = std::stoi(v);
     else if (k == "leafcap") o.leafcap = std::stoi(v);
+    else if (k == "levels") o.levels = std::max(5, std::min(13, std::stoi(v)));
     else if (k == "stages") o.stages = std::stoi(v);
     else if (k == "cut_level") o.cut_level = std::stoi(v);
     else if (k == "merge") o.merge = std::stoi(v);
@@ -628,7 +630,7 @@ struct Mapper {
       // candidates per level
       std::vector<uint32_t> cand[14];
       for (uint32_t i = 0; i < n; i++)
-        if (mc[i] && d[i] <= 13) cand[d[i]].push_back(i);
+        if (mc[i] && d[i] <= (uint32_t)opt.levels) cand[d[i]].push_back(i);
       for (int k = 1; k <= 13; k++)
         std::sort(cand[k].begin(), cand[k].end(), [&](uint32_t x, uint32_t y) {
           if (rd[x] != rd[y]) return rd[x] > rd[y];
@@ -677,7 +679,7 @@ struct Mapper {
         }
       };
       // bottom (tip, level 13) to top (leaf side)
-      for (int k = 13; k >= 1; k--) {
+      for (int k = opt.levels; k >= 1; k--) {
         if (cand[k].empty()) continue;
         // free slots at level k, interleaved over units to spread leaves
         std::vector<uint32_t> fs;

@@ -27,7 +27,7 @@ for cfg in sys.argv[1:] or ["c1"]:
     sim.lib.gem_read_fine(sim._h, out.ctypes.data_as(ctypes.c_void_p))
     f = out[:512].reshape(8, 8, 8).astype(np.int64)    # [layer][warp][slot]
     sub = out[512:].reshape(8, 8, 4).astype(np.int64)  # [layer][warp][gather|fold5|ballot+fold5|wo+top]
-    print(f"== {cfg}: per-layer, per-warp deltas (clocks): exec | wait_next | load_next | top | barrier")
+    print(f"== {cfg} (resident={sim.info.get('resident')}): per-layer, per-warp deltas (clocks): exec | wait_next | load_next | top | barrier")
     for l in range(8):
         if f[l, :, 0].max() == 0:
             break

@@ -7,6 +7,10 @@ sys.path.insert(0, os.path.dirname(os.path.dirname(os.path.abspath(__file__))))
 import numpy as np  # noqa: E402
 
 from gen import stimulus  # noqa: E402
+from paper_conf_dac_guozwlr25_b200 import _build  # noqa: E402
+if os.environ.get("GEM_EXP_LIB"):   # timing experiments (scripts/experiment.py)
+    _build.LIBGEM = os.environ["GEM_EXP_LIB"]
+    _build.build_libgem = lambda force=False, extra=(): _build.LIBGEM
 from paper_conf_dac_guozwlr25_b200 import gem  # noqa: E402
 from tests.common import blob  # noqa: E402
 
@@ -16,8 +20,9 @@ ap.add_argument("--cycles", type=int, default=50)
 ap.add_argument("--streams", type=int, default=1)
 ap.add_argument("--launches", type=int, default=2)
 ap.add_argument("--phases", action="store_true")
+ap.add_argument("--map-opts", default=None)
 a = ap.parse_args()
-b = blob(a.cfg)
+b = blob(a.cfg, a.map_opts)
 sim = gem.Simulator(b, n_streams=a.streams)
 n_pi = sim.info["n_pi"]
 st = np.stack([stimulus("c3" if a.cfg == "c5" else a.cfg, n_pi, a.cycles * a.launches, seed=100 + s)

@@ -75,6 +75,10 @@ def test_blob_stats_c2():
     assert i.max_layers >= 40 / 13          # cannot beat 13 levels per layer
     assert i.max_layers <= 40               # boomerang layers are fewer than levels
     assert i.max_state_words <= 2048
+    # part table decoded with the header's stride: per-part layer counts add up
+    assert sum(i.part_layers) == i.total_layers
+    assert max(i.part_layers) == i.max_layers
+    assert all(c > 0 for c in i.part_cost)
 
 
 @pytest.mark.parametrize("opts", ["parts=1 lanes=1", "parts=4 lanes=1", "parts=5 stages=2 lanes=1"])
