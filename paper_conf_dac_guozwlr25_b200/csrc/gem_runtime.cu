@@ -50,7 +50,7 @@ struct KParams {
   uint32_t* q_trace;                        // [stream][out_cap][q_ext_words]
   unsigned long long* digest;               // [stream][out_cap]
   const uint32_t* __restrict__ q_int_of_ext;  // [n_flops] internal bit
-  unsigned long long* bar;                  // grid barrier counter
+  unsigned long long* bar;                  // grid barrier: per-CTA arrival flags
   int* err;
   uint64_t t0;
   uint32_t ncycles, in_base, in_cap, out_cap;
@@ -58,7 +58,7 @@ struct KParams {
   uint32_t pi_words, po_words, q_words, cut_words, n_rams, n_flops, q_ext_words;
   uint32_t flags;
   uint32_t area_words, slot_words, ring_slots, allow_resident;
-  unsigned long long* prof;   // GEM_F_PROFILE: [prof_cycles][grid][8] clock64 stamps
+  unsigned long long* prof;   // GEM_F_PROFILE: [prof_cycles][grid][GEM_PROF_SLOTS] clock64 stamps
   uint32_t prof_cycles;
   uint32_t group;                        // streams per work item (stream states in smem)
   // lane mode
@@ -94,7 +94,7 @@ struct KParams {
 #define PROF(slot_)                                                                          \
   do {                                                                                       \
     if (prof_on && threadIdx.x == 0)                                                         \
-      kp.prof[((size_t)c * gridDim.x + blockIdx.x) * 8 + (slot_)] = (unsigned long long)clock64(); \
+      kp.prof[((size_t)c * gridDim.x + blockIdx.x) * GEM_PROF_SLOTS + (slot_)] = (unsigned long long)clock64(); \
   } while (0)
 
 __device__ __forceinline__ unsigned long long ld_acquire_u64(const unsigned long long* p) {
@@ -109,21 +109,26 @@ __device__ __forceinline__ uint64_t globaltimer_ns() {
   return t;
 }
 
-// Grid-wide barrier on a monotonically increasing 64-bit counter (reset to 0
-// before each launch).  Release: bar.sync + red.release.gpu arrive.
-// Acquire: ld.acquire.gpu spin, then bar.sync.  A 10 s spin limit turns a
-// deadlock (e.g. broken co-residency) into a trapped kernel instead of a hang.
-__device__ __forceinline__ void grid_sync(const KParams& kp, unsigned long long& target) {
+// Grid-wide barrier on per-CTA arrival flags (one 128-byte line each, reset to
+// 0 before each launch).  Arrive: bar.sync, then thread 0 stores the barrier
+// epoch with st.release.gpu (cumulative over the CTA's writes ordered before it
+// by the bar.sync).  Wait: thread f polls CTA f's flag with ld.acquire.gpu (all
+// flags in parallel, no single contended counter), then bar.sync.  A 10 s spin
+// limit turns a deadlock (e.g. broken co-residency) into a trapped kernel.
+#define GEM_BAR_STRIDE 16   /* u64 words between flags (128 bytes) */
+#define GEM_BAR_MAX_CTAS 1024
+__device__ __forceinline__ void st_release_u64(unsigned long long* p, unsigned long long v) {
+  asm volatile("st.release.gpu.global.u64 [%0], %1;" ::"l"(p), "l"(v) : "memory");
+}
+__device__ __forceinline__ void grid_sync(const KParams& kp, unsigned long long& epoch) {
   __syncthreads();
   if (gridDim.x > 1) {
-    if (threadIdx.x == 0) {
-      target += gridDim.x;
-      // release at gpu scope, cumulative over the CTA's writes ordered before
-      // it by the bar.sync above (replaces fence.sc + returning atomic)
-      asm volatile("red.release.gpu.global.add.u64 [%0], 1;" ::"l"(kp.bar) : "memory");
+    epoch++;
+    if (threadIdx.x == 0) st_release_u64(kp.bar + (size_t)blockIdx.x * GEM_BAR_STRIDE, epoch);
+    for (uint32_t f = threadIdx.x; f < gridDim.x; f += blockDim.x) {
       uint32_t spins = 0;
       uint64_t start = 0;
-      while (ld_acquire_u64(kp.bar) < target) {
+      while (ld_acquire_u64(kp.bar + (size_t)f * GEM_BAR_STRIDE) < epoch) {
         if (++spins == 4096) start = globaltimer_ns();
         if (spins > 4096 && (spins & 4095) == 0 && globaltimer_ns() - start > 10000000000ull) {
           atomicExch(kp.err, 2);
@@ -199,6 +204,9 @@ __device__ __forceinline__ void fence_mbar_init() {
 #define GEM_RING_MAX 4
 #define GEM_MAX_CHUNKS 256
 #define GEM_MAX_RESIDENT 16
+#define GEM_WL_MAX_STAGES 8
+#define GEM_WL_CACHE 64                              // work items cached in smem per CTA
+#define GEM_WL_CACHE_WORDS (32 + 2 * GEM_WL_CACHE)
 
 // Shared-memory program source: either every program of this CTA resident
 // (copied once per launch) or a ring of R slots fed chunk by chunk by TMA.
@@ -209,6 +217,11 @@ struct ProgSrc {
   uint32_t slot_words, R;
   uint32_t seq_issue, seq_wait, seq_free;   // chunk sequence numbers (uniform across the CTA)
   bool resident;
+  // pinned prefix (single-partition CTAs whose program does not fit): chunks
+  // [0, pin_chunks) stay in `pin` for the launch, the rest stream through the
+  // ring placed after them; pro_chunk/pro_off = next chunk after the prologue
+  uint32_t pin_chunks, pin_off, pro_chunk, pro_off;
+  const uint32_t* pin;
   uint32_t n_res;
   const uint32_t* res_p;   // smem [GEM_MAX_RESIDENT] partition ids
   const uint32_t* res_off; // smem [GEM_MAX_RESIDENT] word offsets into area
@@ -250,6 +263,22 @@ __device__ __forceinline__ void issue_prologue(const KParams& kp, ProgSrc& ps, u
     ring_issue(ps, g + off, sz[i]);
     off += sz[i];
   }
+}
+
+// Prologue in pinned-prefix mode: the first streamed chunks of partition p
+// (sizes from the pinned chunk table); records where refilling resumes.
+__device__ __forceinline__ void issue_prologue_pinned(const KParams& kp, ProgSrc& ps, uint32_t p) {
+  const uint32_t* g = kp.prog + __ldg(kp.parts + p * GP_WORDS + GP_PROG_OFF);
+  const uint32_t* ct = ps.pin + ps.pin[PH_OFF_CHUNKS];
+  const uint32_t nch = ps.pin[PH_N_CHUNKS];
+  uint32_t k = ps.pin_chunks, off = ps.pin_off;
+  while (k < nch && k < ps.pin_chunks + ps.R) {
+    ring_issue(ps, g + off, ct[k]);
+    off += ct[k];
+    k++;
+  }
+  ps.pro_chunk = k;
+  ps.pro_off = off;
 }
 
 // Explicit shared-window accesses (32-bit addresses): avoids generic->shared
@@ -418,23 +447,34 @@ __device__ void run_partition(const KParams& kp, ProgSrc& ps, uint32_t* S, uint3
   const uint32_t s_base = smem_u32(S);
   const uint32_t* gprog = kp.prog + __ldg(kp.parts + p * GP_WORDS + GP_PROG_OFF);
   const uint32_t* C0;
-  const uint32_t* ctab;
+  const uint32_t* ctab;    // chunk sizes (smem)
   uint32_t next_chunk = 0, next_off = 0;
+  uint32_t n_pin = 0;      // leading chunks served from smem without the ring
   if (ps.resident) {
     uint32_t off = 0;
     for (uint32_t k = 0; k < ps.n_res; k++) if (ps.res_p[k] == p) off = ps.res_off[k];
     C0 = ps.area + off;
     ctab = C0 + C0[PH_OFF_CHUNKS];
+    n_pin = ~0u;
+  } else if (ps.pin_chunks) {
+    C0 = ps.pin;
+    ctab = C0 + C0[PH_OFF_CHUNKS];
+    n_pin = ps.pin_chunks;
+    next_chunk = ps.pro_chunk;
+    next_off = ps.pro_off;
+    PROF(7);
   } else {
     next_chunk = prologue_count(kp, ps, p);
     next_off = __ldg(kp.parts + p * GP_WORDS + GP_CHUNK0);
     if (next_chunk > 1) next_off += __ldg(kp.parts + p * GP_WORDS + GP_CHUNK1);
     if (next_chunk > 2) next_off += __ldg(kp.parts + p * GP_WORDS + GP_CHUNK2);
     C0 = ring_wait(ps);
+    PROF(7);
     // keep the chunk table: chunk 0's slot is recycled
     const uint32_t nch = C0[PH_N_CHUNKS];
     for (uint32_t k = tid; k < nch; k += GEM_THREADS) ps.ctab[k] = C0[C0[PH_OFF_CHUNKS] + k];
-    ctab = C0 + C0[PH_OFF_CHUNKS];
+    ctab = ps.ctab;
+    n_pin = 0;
   }
   const uint4 h0 = *reinterpret_cast<const uint4*>(C0);
   const uint4 h1 = *(reinterpret_cast<const uint4*>(C0) + 1);
@@ -446,7 +486,7 @@ __device__ void run_partition(const KParams& kp, ProgSrc& ps, uint32_t* S, uint3
   auto refill = [&]() {   // issue chunks into free ring slots
     if (!ps.resident)
       while (next_chunk < n_chunks && ps.seq_issue - ps.seq_free < ps.R) {
-        const uint32_t words = ps.ctab[next_chunk];
+        const uint32_t words = ctab[next_chunk];
         ring_issue(ps, gprog + next_off, words);
         next_off += words;
         next_chunk++;
@@ -480,18 +520,20 @@ __device__ void run_partition(const KParams& kp, ProgSrc& ps, uint32_t* S, uint3
     for (uint32_t u = 0; u < 4; u++)
       if (dst[u] != ~0u) sts(s_base + 4 * dst[u], v[u]);
   }
+  PROF(8);
   if (tid < nst) S[tid * SW] = 0u;
   // first layer's records (independent of S) before the barrier
   LayerRegs R;
   const uint32_t* Lres = C0 + off_layers;
   if (n_layers) {
     const uint32_t* L;
-    if (ps.resident) { L = Lres; Lres += ctab[1]; }
+    if (1 < n_pin) { L = Lres; Lres += ctab[1]; }
     else L = ring_wait(ps);
     load_layer(L, R);
   }
+  PROF(9);
   __syncthreads();   // S ready; chunk 0 and layer 0's chunk consumed
-  if (!ps.resident) ps.seq_free += n_layers ? 2 : 1;
+  ps.seq_free = ps.seq_wait;   // records are in registers; waited slots are free
   // (the S[0] read makes the stamp wait for the barrier release, which
   // BAR.SYNC.DEFER_BLOCKING otherwise defers to the first dependent access)
   if (prof_on && tid == 0 && lds(s_base) == 0u) PROF(1);
@@ -514,7 +556,7 @@ __device__ void run_partition(const KParams& kp, ProgSrc& ps, uint32_t* S, uint3
     const uint32_t ptopc = R.topc, ptopwo = R.topwo;
     if (l + 1 < n_layers) {
       const uint32_t* L;
-      if (ps.resident) { L = Lres; Lres += ctab[2 + l]; }
+      if (2 + l < n_pin) { L = Lres; Lres += ctab[2 + l]; }
       else L = ring_wait(ps);
       FPROF(l, 2);
 #ifndef EXP_NO_LOAD
@@ -531,12 +573,12 @@ __device__ void run_partition(const KParams& kp, ProgSrc& ps, uint32_t* S, uint3
     FPROF(l, 4);
     __syncthreads();
     FPROF(l, 5);
-    if (!ps.resident && l + 1 < n_layers) ps.seq_free++;
+    ps.seq_free = ps.seq_wait;
     refill();
   }
   PROF(2);
   // ---- a6: endpoint commit (warp ballot-gather per output word and stream)
-  const uint32_t* od = ps.resident ? (C0 + off_out) : ring_wait(ps);
+  const uint32_t* od = n_layers + 1 < n_pin ? (C0 + off_out) : ring_wait(ps);
   const uint32_t* os = od + n_out_pad;
   for (uint32_t jj = warp; jj < n_out * nst; jj += GEM_WARPS) {
     const uint32_t j = jj / n_out, o = jj - j * n_out, st = st0 + j;
@@ -572,9 +614,9 @@ __device__ void run_partition(const KParams& kp, ProgSrc& ps, uint32_t* S, uint3
     }
   }
   __syncthreads();  // S / ramp / ring slots reused by the next work item
-  if (!ps.resident) ps.seq_free = ps.seq_issue;   // every chunk of this item consumed
+  ps.seq_free = ps.seq_issue;   // every chunk of this item consumed
   PROF(3);
-  if (prof_on && tid == 0) kp.prof[((size_t)c * gridDim.x + blockIdx.x) * 8 + 6] = n_layers;
+  if (prof_on && tid == 0) kp.prof[((size_t)c * gridDim.x + blockIdx.x) * GEM_PROF_SLOTS + 6] = n_layers;
 }
 
 // Parity instruments: trace / digest of Q(t+1) in external (AIGER) order.
@@ -603,7 +645,7 @@ __device__ void record_state(const KParams& kp, uint32_t c, uint32_t buf) {
 __global__ void __launch_bounds__(GEM_THREADS, 2) gem_step_kernel(const KParams kp) {
   extern __shared__ __align__(16) uint32_t smem[];
   // layout (words): S[group][state_words] | area[area_words] | ctab[256] | ramp[group][128] |
-  //                 topb[group][16] | res_p[16] | res_off[16] | res_n[16] | mbar[8 x u64]
+  //                 topb[group][16] | res_p[16] | res_off[16] | res_n[16] | wl cache | mbar[8 x u64]
   // S must stay at offset 0 (leaf entries carry byte offsets into it).
   uint32_t* S = smem;
   uint32_t* area = S + kp.group * kp.state_words;
@@ -612,12 +654,35 @@ __global__ void __launch_bounds__(GEM_THREADS, 2) gem_step_kernel(const KParams 
   uint32_t* topb = ramp + kp.group * 4 * GEM_MAX_RAMS_PER_PART;
   uint32_t* res_p = topb + 16 * kp.group;
   uint32_t* res_off = res_p + GEM_MAX_RESIDENT;
-  uint32_t* res_n = res_off + GEM_MAX_RESIDENT;      // [0] = n_res, [1] = resident flag
-  uint64_t* mbar = reinterpret_cast<uint64_t*>(res_n + 16);
+  uint32_t* res_n = res_off + GEM_MAX_RESIDENT;      // [0] n_res, [1] resident, [2..4] pinned chunks/words, ring R
+  // work-list cache: [0,8) stage begins, [8,16) stage ends, [16,24) cache base
+  // per stage, [24] cached flag, [32, 32 + 2*GEM_WL_CACHE) items (uint2)
+  uint32_t* wlc = res_n + 16;
+  uint64_t* mbar = reinterpret_cast<uint64_t*>(wlc + GEM_WL_CACHE_WORDS);
   const uint32_t tid = threadIdx.x;
   const uint32_t G = gridDim.x, B = blockIdx.x;
-  auto wl_begin = [&](uint32_t s) { return __ldg(kp.wl_off + s * (G + 1) + B); };
-  auto wl_end = [&](uint32_t s) { return __ldg(kp.wl_off + s * (G + 1) + B + 1); };
+  if (tid == 0) {
+    // the CTA's work list is fixed for the launch: keep it in shared memory
+    // (saves two dependent global loads at the start of every cycle)
+    uint32_t n = 0;
+    bool ok = kp.n_stages <= GEM_WL_MAX_STAGES;
+    for (uint32_t s = 0; s < kp.n_stages && ok; s++) {
+      const uint32_t b = __ldg(kp.wl_off + s * (G + 1) + B), e = __ldg(kp.wl_off + s * (G + 1) + B + 1);
+      wlc[s] = b;
+      wlc[8 + s] = e;
+      wlc[16 + s] = n;
+      if (n + (e - b) > GEM_WL_CACHE) { ok = false; break; }
+      for (uint32_t k = b; k < e; k++) reinterpret_cast<uint2*>(wlc + 32)[n++] = __ldg(&kp.wl_items[k]);
+    }
+    wlc[24] = ok ? 1u : 0u;
+  }
+  __syncthreads();
+  const bool wl_cached = wlc[24] != 0;
+  auto wl_begin = [&](uint32_t s) { return wl_cached ? wlc[s] : __ldg(kp.wl_off + s * (G + 1) + B); };
+  auto wl_end = [&](uint32_t s) { return wl_cached ? wlc[8 + s] : __ldg(kp.wl_off + s * (G + 1) + B + 1); };
+  auto wl_item = [&](uint32_t s, uint32_t k) -> uint2 {
+    return wl_cached ? reinterpret_cast<const uint2*>(wlc + 32)[wlc[16 + s] + (k - wlc[s])] : __ldg(&kp.wl_items[k]);
+  };
   for (uint32_t k = tid; k < 16 * kp.group; k += GEM_THREADS) topb[k] = 0u;
   if (tid == 0) {
     for (uint32_t k = 0; k <= GEM_RING_MAX; k++) mbar_init(mbar + k, 1);
@@ -627,7 +692,7 @@ __global__ void __launch_bounds__(GEM_THREADS, 2) gem_step_kernel(const KParams 
     bool ok = kp.allow_resident != 0;
     for (uint32_t s = 0; s < kp.n_stages && ok; s++) {
       for (uint32_t k = wl_begin(s); k < wl_end(s); k++) {
-        const uint32_t p = __ldg(&kp.wl_items[k].x);
+        const uint32_t p = wl_item(s, k).x;
         bool seen = false;
         for (uint32_t j = 0; j < n; j++) seen |= res_p[j] == p;
         if (seen) continue;
@@ -641,6 +706,40 @@ __global__ void __launch_bounds__(GEM_THREADS, 2) gem_step_kernel(const KParams 
     }
     res_n[0] = n;
     res_n[1] = ok ? 1u : 0u;
+    res_n[2] = 0u;               // pinned chunks
+    res_n[3] = 0u;               // pinned words
+    res_n[4] = kp.ring_slots;    // ring depth
+    if (!ok && kp.allow_resident) {
+      // pinned prefix: a CTA that runs a single partition whose program does
+      // not fit keeps its leading chunks (header, gread list, first layers)
+      // for the whole launch and streams only the rest through a ring
+      uint32_t p1 = ~0u;
+      bool single = true;
+      for (uint32_t s = 0; s < kp.n_stages; s++)
+        for (uint32_t k = wl_begin(s); k < wl_end(s); k++) {
+          const uint32_t p = wl_item(s, k).x;
+          if (p1 == ~0u) p1 = p;
+          else single &= p == p1;
+        }
+      if (single && p1 != ~0u) {
+        const uint32_t* g = kp.prog + __ldg(kp.parts + p1 * GP_WORDS + GP_PROG_OFF);
+        const uint32_t nch = __ldg(g + PH_N_CHUNKS), offc = __ldg(g + PH_OFF_CHUNKS);
+        uint32_t P = 0, pw = 0;
+        while (P < nch) {
+          const uint32_t sz = __ldg(g + offc + P);
+          if (pw + sz + 2 * kp.slot_words > kp.area_words) break;
+          pw += sz;
+          P++;
+        }
+        if (P >= 2) {
+          res_n[2] = P;
+          res_n[3] = pw;
+          res_n[4] = pw + 4 * kp.slot_words <= kp.area_words ? 4u : 2u;
+          mbar_expect_tx(mbar + GEM_RING_MAX, pw * 4);
+          tma_load_1d(area, g, pw * 4, mbar + GEM_RING_MAX);
+        }
+      }
+    }
     if (ok && words) {
       mbar_expect_tx(mbar + GEM_RING_MAX, words * 4);
       for (uint32_t k = 0; k < n; k++) {
@@ -665,16 +764,28 @@ __global__ void __launch_bounds__(GEM_THREADS, 2) gem_step_kernel(const KParams 
   ps.seq_issue = 0;
   ps.seq_wait = 0;
   ps.seq_free = 0;
-  if (ps.resident && ps.n_res) mbar_wait(mbar + GEM_RING_MAX, 0);
-  // first work item of this CTA in a cycle (index into wl_items), or ~0u
-  auto first_item = [&]() -> uint32_t {
+  ps.pin_chunks = res_n[2];
+  ps.pin_off = res_n[3];
+  ps.pin = area;
+  ps.pro_chunk = ps.pro_off = 0;
+  if (ps.pin_chunks) {
+    ps.area = area + ps.pin_off;   // ring after the pinned prefix
+    ps.R = res_n[4];
+  }
+  if ((ps.resident && ps.n_res) || ps.pin_chunks) mbar_wait(mbar + GEM_RING_MAX, 0);
+  // first work item of this CTA in a cycle: partition id, or ~0u
+  auto first_part = [&]() -> uint32_t {
     for (uint32_t s = 0; s < kp.n_stages; s++)
-      if (wl_begin(s) < wl_end(s)) return wl_begin(s);
+      if (wl_begin(s) < wl_end(s)) return wl_item(s, wl_begin(s)).x;
     return ~0u;
   };
+  auto prologue = [&](uint32_t p) {
+    if (ps.pin_chunks) issue_prologue_pinned(kp, ps, p);
+    else issue_prologue(kp, ps, p);
+  };
   if (!ps.resident && kp.ncycles) {
-    const uint32_t k0 = first_item();
-    if (k0 != ~0u) issue_prologue(kp, ps, __ldg(&kp.wl_items[k0].x));
+    const uint32_t p0 = first_part();
+    if (p0 != ~0u) prologue(p0);
   }
 
   unsigned long long bar_target = 0;
@@ -688,17 +799,17 @@ __global__ void __launch_bounds__(GEM_THREADS, 2) gem_step_kernel(const KParams 
     for (uint32_t s = 0; s < kp.n_stages; s++) {
       const uint32_t kb = wl_begin(s), ke = wl_end(s);
       for (uint32_t k = kb; k < ke; k++) {
-        const uint2 it = __ldg(&kp.wl_items[k]);
+        const uint2 it = wl_item(s, k);
         const uint32_t nst = min(kp.group, kp.n_streams - it.y);
         run_partition(kp, ps, S, ramp, topb, it.x, it.y, nst, c, cur, nxt, prof_on && k == kb && s == 0);
         if (!ps.resident) {
           // prefetch the next work item's prologue (overlaps the grid barrier)
-          uint32_t nk = ~0u;
-          if (k + 1 < ke) nk = k + 1;
-          for (uint32_t s2 = s + 1; nk == ~0u && s2 < kp.n_stages; s2++)
-            if (wl_begin(s2) < wl_end(s2)) nk = wl_begin(s2);
-          if (nk == ~0u && c + 1 < kp.ncycles) nk = first_item();
-          if (nk != ~0u) issue_prologue(kp, ps, __ldg(&kp.wl_items[nk].x));
+          uint32_t np = ~0u;
+          if (k + 1 < ke) np = wl_item(s, k + 1).x;
+          for (uint32_t s2 = s + 1; np == ~0u && s2 < kp.n_stages; s2++)
+            if (wl_begin(s2) < wl_end(s2)) np = wl_item(s2, wl_begin(s2)).x;
+          if (np == ~0u && c + 1 < kp.ncycles) np = first_part();
+          if (np != ~0u) prologue(np);
         }
       }
       if (s == 0) PROF(4);
@@ -933,7 +1044,7 @@ static int plan_launch(gem_sim* sim, uint32_t max_chunk_words, uint32_t grid_lim
     const char* genv = getenv("GEM_GROUP");
     uint32_t g = genv ? (uint32_t)atoi(genv) : GEM_MAX_GROUP;
     g = std::max<uint32_t>(1, std::min<uint32_t>(std::min<uint32_t>(g, GEM_MAX_GROUP), sim->n_streams));
-    while (g > 1 && (uint64_t)(g * (sim->state_words + 4 * GEM_MAX_RAMS_PER_PART + 16) + GEM_MAX_CHUNKS + 80 +
+    while (g > 1 && (uint64_t)(g * (sim->state_words + 4 * GEM_MAX_RAMS_PER_PART + 16) + GEM_MAX_CHUNKS + 80 + GEM_WL_CACHE_WORDS +
                                3 * slot) * 4 > (uint64_t)optin)
       g /= 2;
     sim->group = g;
@@ -943,7 +1054,7 @@ static int plan_launch(gem_sim* sim, uint32_t max_chunk_words, uint32_t grid_lim
     sim->max_items = std::max(sim->max_items, (sim->h_stage[s + 1] - sim->h_stage[s]) *
                                                   ((sim->n_streams + sim->group - 1) / sim->group));
   const uint32_t fixed_words =
-      sim->group * (sim->state_words + 4 * GEM_MAX_RAMS_PER_PART + 16) + GEM_MAX_CHUNKS + 48 + 16;
+      sim->group * (sim->state_words + 4 * GEM_MAX_RAMS_PER_PART + 16) + GEM_MAX_CHUNKS + 48 + GEM_WL_CACHE_WORDS + 16;
   const char* env = getenv("GEM_NO_RESIDENT");
   const bool allow_res = !(env && env[0] == '1');
   const char* benv = getenv("GEM_BPS");
@@ -962,6 +1073,7 @@ static int plan_launch(gem_sim* sim, uint32_t max_chunk_words, uint32_t grid_lim
     const uint32_t area = (uint32_t)(budget / 4) - fixed_words;
     uint32_t grid = std::max<uint32_t>(1, std::min<uint32_t>(sim->max_items, bps * (uint32_t)sms));
     if (grid_limit) grid = std::max<uint32_t>(1, std::min(grid, grid_limit));
+    grid = std::min<uint32_t>(grid, GEM_BAR_MAX_CTAS);
     int occ = 0;
     CK(cudaFuncSetAttribute(gem_step_kernel, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)budget));
     CK(cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ, gem_step_kernel, GEM_THREADS, (size_t)budget));
@@ -1052,6 +1164,7 @@ static int plan_launch_lanes(gem_sim* sim, uint32_t grid_limit) {
   ring = ring >= 4 ? 4 : 2;
   uint32_t grid = std::max<uint32_t>(1, std::min<uint32_t>(sim->max_items, bps * (uint32_t)sms));
   if (grid_limit) grid = std::max<uint32_t>(1, std::min(grid, grid_limit));
+  grid = std::min<uint32_t>(grid, GEM_BAR_MAX_CTAS);
   const uint32_t smem = (fixed_words + ring * slot) * 4;
   CK(cudaFuncSetAttribute(gem_lane_kernel, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem));
   int occ = 0;
@@ -1181,7 +1294,7 @@ int gem_load_program(const void* blob, size_t nbytes, const gem_config* cfg, gem
     CK(dalloc(&sim->d_cut, S * std::max<uint32_t>(sim->cut_words, 1) * 4));
   }
   CK(dalloc(&sim->d_mem, S * sim->n_rams * (size_t)GEM_RAM_WORDS * 4));
-  CK(dalloc(&sim->d_bar, 64));
+  CK(dalloc(&sim->d_bar, (size_t)GEM_BAR_MAX_CTAS * GEM_BAR_STRIDE * 8));
   CK(dalloc(&sim->d_err, 64));
   CK(cudaMemset(sim->d_err, 0, 64));
   // initial state: flops = init (U5), RD = 0, RAM = 0 (U10)
@@ -1297,18 +1410,18 @@ int gem_step(gem_sim* sim, uint64_t ncycles) {
     if (!sim->d_prof || sim->prof_cycles < pc) {
       if (sim->d_prof) cudaFree(sim->d_prof);
       sim->d_prof = nullptr;
-      CK(dalloc(&sim->d_prof, (size_t)256 * sim->grid * 8 * 8 + 8 * 8 * 8 * 8));
+      CK(dalloc(&sim->d_prof, (size_t)256 * sim->grid * GEM_PROF_SLOTS * 8));
 #ifdef GEM_FINE_PROF
       CK(dalloc(&sim->d_fprof, 8 * 8 * 8 * 8 + 8 * 8 * 4 * 8));
 #endif
     }
     sim->prof_cycles = pc;
-    CK(cudaMemsetAsync(sim->d_prof, 0, (size_t)256 * sim->grid * 8 * 8 + 8 * 8 * 8 * 8, sim->stream));
+    CK(cudaMemsetAsync(sim->d_prof, 0, (size_t)256 * sim->grid * GEM_PROF_SLOTS * 8, sim->stream));
     kp.prof = sim->d_prof;
     kp.prof_cycles = pc;
     kp.fprof = sim->d_fprof;
   }
-  CK(cudaMemsetAsync(sim->d_bar, 0, 8, sim->stream));
+  CK(cudaMemsetAsync(sim->d_bar, 0, (size_t)GEM_BAR_MAX_CTAS * GEM_BAR_STRIDE * 8, sim->stream));
   if (sim->flags & GEM_F_DIGEST)
     CK(cudaMemsetAsync(sim->d_digest, 0, (size_t)sim->n_streams * sim->out_cap * 8, sim->stream));
   if (sim->lanes) {
@@ -1495,7 +1608,7 @@ int gem_read_profile(gem_sim* sim, uint64_t* dst, uint32_t* n_cycles, uint32_t* 
   CK(cudaStreamSynchronize(sim->stream));
   if (n_cycles) *n_cycles = sim->prof_cycles;
   if (grid) *grid = sim->grid;
-  if (dst) CK(cudaMemcpy(dst, sim->d_prof, (size_t)sim->prof_cycles * sim->grid * 8 * 8, cudaMemcpyDeviceToHost));
+  if (dst) CK(cudaMemcpy(dst, sim->d_prof, (size_t)sim->prof_cycles * sim->grid * GEM_PROF_SLOTS * 8, cudaMemcpyDeviceToHost));
   return GEM_OK;
 }
 

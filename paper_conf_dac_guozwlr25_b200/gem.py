@@ -188,10 +188,10 @@ class Simulator:
         self._check(self.lib.gem_write_ram(self._h, ram, stream, _p(w)))
 
     def read_profile(self) -> np.ndarray:
-        """uint64 [cycles][grid][8] clock64 phase stamps (GEM_F_PROFILE)."""
+        """uint64 [cycles][grid][16] clock64 phase stamps (GEM_F_PROFILE; slots in include/gem.h)."""
         n, g = ctypes.c_uint32(), ctypes.c_uint32()
         self._check(self.lib.gem_read_profile(self._h, None, ctypes.byref(n), ctypes.byref(g)))
-        out = np.zeros((n.value, g.value, 8), np.uint64)
+        out = np.zeros((n.value, g.value, 16), np.uint64)
         self._check(self.lib.gem_read_profile(self._h, _p(out), ctypes.byref(n), ctypes.byref(g)))
         return out
 

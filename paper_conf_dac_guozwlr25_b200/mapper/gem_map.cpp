@@ -523,7 +523,8 @@ struct Mapper {
     for (auto& ow : P.outs) for (int k = 0; k < 32; k++) is_ep[(uint32_t)scratch[ow.lit[k] >> 1]] = 1;
     P.n_nodes = n_and;
 
-    // ---- state: word 0 = const 0; gread words next
+    // ---- state: word 0 = const 0; gread words next, in ascending global word
+    // order so that a warp's 32 port loads fall into few L2 sectors (a2)
     std::vector<uint32_t> gread_src;     // gid per gread
     std::unordered_map<uint32_t, uint32_t> gword;   // gid -> state word
     uint32_t sw_next = 1;
@@ -531,17 +532,20 @@ struct Mapper {
     for (uint32_t i = 0; i < n; i++) {
       if (!is_src[i]) continue;
       uint32_t c = nodes[i];
+      if (G.kind[c] == K_CONST) continue;
+      uint32_t gb = G.gbit[c];
+      uint32_t gid = GEM_GID(gb >> 27, (gb >> 5) & 0x3FFFFF);
+      if (gword.emplace(gid, 0u).second) gread_src.push_back(gid);
+    }
+    std::sort(gread_src.begin(), gread_src.end());
+    for (uint32_t gid : gread_src) gword[gid] = sw_next++;
+    for (uint32_t i = 0; i < n; i++) {
+      if (!is_src[i]) continue;
+      uint32_t c = nodes[i];
       if (G.kind[c] == K_CONST) { loc[i] = 0; continue; }
       uint32_t gb = G.gbit[c];
       uint32_t gid = GEM_GID(gb >> 27, (gb >> 5) & 0x3FFFFF);
-      auto it = gword.find(gid);
-      uint32_t sw;
-      if (it == gword.end()) {
-        sw = sw_next++;
-        gword.emplace(gid, sw);
-        gread_src.push_back(gid);
-      } else sw = it->second;
-      loc[i] = (int32_t)(sw * 32 + (gb & 31));
+      loc[i] = (int32_t)(gword[gid] * 32 + (gb & 31));
     }
     uint32_t n_gread = sw_next - 1;
     if (sw_next > (uint32_t)opt.max_state_words) { fail(P, "too many gread words"); return; }
