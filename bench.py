@@ -342,12 +342,31 @@ def main():
         achieved_lop3 = info.n_and / 16.0 * hz_kernel * S   # this rank's kernel (per GPU)
         roof = {"bound": "alu", "achieved": achieved_lop3 / 1e12, "peak": peak_lop3 / 1e12, "unit": "TLOP3/s",
                 "frac": achieved_lop3 / peak_lop3, "traffic": None,
-                "kernel": "gem_step_kernel", "kernel_ms_per_step": kern_last,
+                "kernel": "gem_lane_kernel" if sim.info["lanes"] else "gem_step_kernel", "kernel_ms_per_step": kern_last,
                 "algorithmic": "N_and/16 LOP3 per stream-cycle (2 LOP3 per 32 gate evals, P:81)",
                 "peak_source": f"{n_sms} SMs x 64 LOP3/clk x sm_max_mhz ({peaks['_source']})",
                 "hbm_program_bytes_per_cycle": info.program_bytes,
                 "hbm_frac_if_streamed": info.program_bytes * hz_kernel / (float(peaks.get("hbm_gbs", 6650)) * 1e9),
                 "us_per_layer_critical": 1e6 / hz_kernel / max(1, info.max_layers)}
+        if S == 1:
+            # single design: the cycle is a chain of dependent layers and grid
+            # barriers, so the binding roofline is latency; floor =
+            # critical layers x minimal-layer latency + stages x barrier latency,
+            # both measured on this GPU by gem_bench_floor
+            lay_clk, bar_clk = gem.bench_floor(dev.index, sim.info["grid"])
+            crit = sum(info.stage_max_layers())
+            f_hz = float(sm_mhz) * 1e6
+            floor_hz = f_hz / (crit * lay_clk + info.n_stages * bar_clk)
+            roof["binding"] = "latency"
+            roof["latency_floor"] = {
+                "layer_clk": lay_clk, "barrier_clk": bar_clk, "critical_layers": crit, "stages": info.n_stages,
+                "floor_cycles_per_s": floor_hz, "achieved_cycles_per_s": hz_kernel, "frac": hz_kernel / floor_hz,
+                "achieved_clk_per_cycle": f_hz / hz_kernel,
+                "definition": "floor = sm_clock / (sum over stages of the deepest partition's layers x minimal-layer "
+                              "clocks + stages x grid-barrier clocks); minimal layer = one dependent gathered load "
+                              "per thread + 13 fold levels + write-out + block barrier (gem_bench_floor)"}
+        else:
+            roof["binding"] = "alu/smem throughput (independent streams)"
         cpu = None
         if ws == 1 and not args.no_cpu_baseline:
             cpu = cpu_baseline(eaig(cfg), info.n_pi, cfg)
@@ -365,8 +384,10 @@ def main():
                            "parallelism": f"streams sharded over {ws} GPU(s), NCCL gather of PO traces"
                            if ws > 1 else "1 GPU"},
                 "gate_evals_per_s": value * info.n_and,
-                "clocks": clk, "gpu_launches": args.steps * 2,
-                "gpu_launches_detail": "per step: 1 gem_step_kernel (persistent, all cycles) + 1 unpermute_kernel",
+                "clocks": clk, "gpu_launches": args.steps * (3 if sim.info["lanes"] else 2),
+                "gpu_launches_detail": "per step: 1 gem_lane_kernel (persistent, all cycles) + from_lanes_kernel + "
+                                       "unpermute_kernel" if sim.info["lanes"] else
+                                       "per step: 1 gem_step_kernel (persistent, all cycles) + 1 unpermute_kernel",
                 "e2e": e2e, "roofline": roof, "cpu_baseline": cpu,
                 "step_ms": {"min": min(step_ms), "median": float(np.median(step_ms)), "max": max(step_ms)}}
         print(json.dumps(line), flush=True)

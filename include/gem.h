@@ -109,6 +109,14 @@ int gem_read_digests(gem_sim* sim, uint64_t* dst, uint64_t ncycles);
 int gem_read_ram(gem_sim* sim, uint32_t ram_id, uint32_t stream, uint32_t* words8192);
 int gem_write_ram(gem_sim* sim, uint32_t ram_id, uint32_t stream, const uint32_t* words8192);
 
+/* Latency-floor microbenchmarks (measurement helper for the roofline; not part
+ * of the simulation path): *layer_clk = SM clocks of a minimal boomerang layer
+ * (one dependent gathered load per thread, levels 1-13, write-out, block
+ * barrier) on one CTA; *barrier_clk = SM clocks of one grid barrier round trip
+ * among `grid` co-resident CTAs (grid <= 1024).  Allocates and frees its own
+ * device memory on `device`. */
+int gem_bench_floor(int device, uint32_t grid, uint32_t iters, double* layer_clk, double* barrier_clk);
+
 /* Device time (CUDA events on the launch stream) of the last gem_step kernel. */
 int gem_last_step_ms(gem_sim* sim, float* ms);
 

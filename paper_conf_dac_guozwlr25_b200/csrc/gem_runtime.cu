@@ -359,8 +359,16 @@ __device__ __forceinline__ void exec_layer(const LayerRegs& R, uint32_t s_base, 
         const uint32_t q[4] = {R.e[g].x, R.e[g].y, R.e[g].z, R.e[g].w};
 #pragma unroll
         for (uint32_t k = 0; k < 4; k++) {
+#ifdef EXP_GATHER_HALF
+          if (g >= 2) continue;
+#endif
+#ifdef EXP_NO_CONFLICT   // timing experiment: same instructions, words 0..31 only (conflict-free)
+          const uint32_t lo = lds(s_base + ((q[k] >> 3) & 0x7Cu));
+          const uint32_t hi = lds(s_base + ((q[k] >> 19) & 0x7Cu));
+#else
           const uint32_t lo = lds(s_base + ((q[k] >> 3) & 0x1FFCu));
           const uint32_t hi = lds(s_base + ((q[k] >> 19) & 0x1FFCu));
+#endif
           acc[k] |= (__funnelshift_l(lo, lo, q[k]) & (1u << (8 * g + 2 * k))) |
                     (__funnelshift_l(hi, hi, q[k] >> 16) & (1u << (8 * g + 2 * k + 1)));
         }
@@ -412,7 +420,22 @@ __device__ __forceinline__ void exec_layer(const LayerRegs& R, uint32_t s_base, 
   }
   // levels 11-13: warps 1-7 arrive (non-blocking) on named barrier `bid`
   // after publishing their level-10 bit; warp 0 folds later (top_layer).
-#ifndef EXP_NO_TOP
+#if defined(GEM_TOP_ATOMIC)
+  // variant: the last warp to arrive (acq_rel counter in topb[8]) folds
+  if (uses_top && lane == 0) {
+    uint32_t old;
+    asm volatile("atom.acq_rel.cta.shared::cta.add.u32 %0, [%1], 1;"
+                 : "=r"(old) : "r"(smem_u32(topb + 8)) : "memory");
+    if (old == GEM_WARPS - 1) {
+      uint32_t t8 = 0;
+#pragma unroll
+      for (uint32_t w = 0; w < GEM_WARPS; w++) t8 |= lds(smem_u32(topb + w)) << w;
+      sts(s_base + 4 * R.topwo, fold3(t8, R.topc & 0xFFu, (R.topc >> 8) & 0xFFu, (R.topc >> 16) & 0xFFu));
+      sts(smem_u32(topb + 8), 0u);
+    }
+  }
+  (void)bid;
+#elif !defined(EXP_NO_TOP)
   if (uses_top && warp != 0) asm volatile("bar.arrive %0, %1;" ::"r"(bid), "r"(GEM_THREADS) : "memory");
 #endif
   FSUB(fl, 3);
@@ -566,7 +589,7 @@ __device__ void run_partition(const KParams& kp, ProgSrc& ps, uint32_t* S, uint3
 #endif
     }
     FPROF(l, 3);
-#ifndef EXP_NO_TOP
+#if !defined(EXP_NO_TOP) && !defined(GEM_TOP_ATOMIC)
     if (ptop && warp == 0)
       for (uint32_t j = 0; j < nst; j++) top_layer(ptopc, ptopwo, s_base + 4 * j * SW, topb + 16 * j, 1 + j);
 #endif
@@ -839,6 +862,55 @@ __device__ __forceinline__ void issue_prologue_lane(const KParams& kp, ProgSrc& 
 }
 
 #include "gem_lanes.cuh"
+
+
+// ---- latency-floor microbenchmarks (bench.py roofline; not on the hot path)
+// Minimal layer: the dependent chain every layer must traverse even with one
+// leaf per thread: one gathered LDS, levels 1-5 in-thread, warp ballot, levels
+// 6-10, named-barrier hand-off of levels 11-13 to warp 0, write-out, barrier.
+__global__ void __launch_bounds__(GEM_THREADS, 1) floor_layer_kernel(unsigned long long* out, uint32_t iters) {
+  __shared__ uint32_t S[2048];
+  __shared__ uint32_t topb[8];
+  const uint32_t tid = threadIdx.x, lane = tid & 31, warp = tid >> 5;
+  for (uint32_t i = tid; i < 2048; i += GEM_THREADS) S[i] = i * 2654435761u;
+  __syncthreads();
+  const uint32_t base = smem_u32(S);
+  uint32_t x = tid;
+  const unsigned long long t0 = clock64();
+  for (uint32_t it = 0; it < iters; it++) {
+    const uint32_t v = lds(base + 4 * ((x ^ it) & 2047u));
+    const uint32_t P = fold5(v, 0x1234567u, 0x89ABCDEu, 0x5555u);
+    const uint32_t u = __ballot_sync(0xFFFFFFFFu, (P >> 30) & 1u);
+    const uint32_t Pw = fold5(u, 0x7654321u, 0x0FEDCBAu, 0x3333u);
+    if (lane == 0) topb[warp] = (Pw >> 30) & 1u;
+    if (warp != 0) {
+      asm volatile("bar.arrive 1, %0;" ::"r"(GEM_THREADS) : "memory");
+    } else {
+      asm volatile("bar.sync 1, %0;" ::"r"(GEM_THREADS) : "memory");
+      if (lane == 0) {
+        uint32_t t8 = 0;
+        for (uint32_t w = 0; w < GEM_WARPS; w++) t8 |= topb[w] << w;
+        sts(base + 4 * (1024 + (it & 1023)), fold3(t8, 0x55u, 0x33u, 0x0Fu));
+      }
+    }
+    __syncthreads();
+    x = P ^ Pw ^ lds(base + 4 * (1024 + (it & 1023)));
+  }
+  const unsigned long long t1 = clock64();
+  if (tid == 0) out[0] = (t1 - t0) / iters;
+  if (x == 0x9E3779B9u) out[1] = x;   // keep the chain live
+}
+
+// Grid barrier round trip at a given grid size (same grid_sync as the kernels).
+__global__ void __launch_bounds__(GEM_THREADS, 1) floor_barrier_kernel(const KParams kp, unsigned long long* out,
+                                                                       uint32_t iters) {
+  unsigned long long epoch = 0;
+  grid_sync(kp, epoch);
+  const unsigned long long t0 = clock64();
+  for (uint32_t it = 0; it < iters; it++) grid_sync(kp, epoch);
+  const unsigned long long t1 = clock64();
+  if (blockIdx.x == 0 && threadIdx.x == 0) out[0] = (t1 - t0) / iters;
+}
 
 // external <-> internal layout conversion kernels
 // out[st][row][ext_w] = gather of 32 internal bits via int_of_ext
@@ -1445,6 +1517,36 @@ int gem_step(gem_sim* sim, uint64_t ncycles) {
     CK(cudaStreamSynchronize(sim->stream));
     CK(cudaEventElapsedTime(&sim->last_ms, sim->ev0, sim->ev1));
   }
+  return GEM_OK;
+}
+
+int gem_bench_floor(int device, uint32_t grid, uint32_t iters, double* layer_clk, double* barrier_clk) {
+  gem_sim* sim = nullptr;
+  if (!layer_clk || !barrier_clk || !grid || grid > GEM_BAR_MAX_CTAS || !iters) return fail(GEM_E_INVAL, "bad floor request");
+  CK(cudaSetDevice(device));
+  unsigned long long *d_out = nullptr, *d_bar = nullptr;
+  int* d_err = nullptr;
+  CK(dalloc(&d_out, 64));
+  CK(dalloc(&d_bar, (size_t)GEM_BAR_MAX_CTAS * GEM_BAR_STRIDE * 8));
+  CK(dalloc(&d_err, 64));
+  CK(cudaMemset(d_bar, 0, (size_t)GEM_BAR_MAX_CTAS * GEM_BAR_STRIDE * 8));
+  unsigned long long h[2] = {0, 0};
+  floor_layer_kernel<<<1, GEM_THREADS>>>(d_out, 64);
+  floor_layer_kernel<<<1, GEM_THREADS>>>(d_out, iters);
+  CK(cudaGetLastError());
+  CK(cudaMemcpy(h, d_out, 16, cudaMemcpyDeviceToHost));
+  *layer_clk = (double)h[0];
+  KParams kp;
+  memset(&kp, 0, sizeof(kp));
+  kp.bar = d_bar;
+  kp.err = d_err;
+  void* args[] = {(void*)&kp, (void*)&d_out, (void*)&iters};
+  CK(cudaLaunchCooperativeKernel((const void*)floor_barrier_kernel, dim3(grid), dim3(GEM_THREADS), args, 0, 0));
+  CK(cudaMemcpy(h, d_out, 16, cudaMemcpyDeviceToHost));
+  *barrier_clk = (double)h[0];
+  cudaFree(d_out);
+  cudaFree(d_bar);
+  cudaFree(d_err);
   return GEM_OK;
 }
 

@@ -23,7 +23,7 @@ ERRORS = {-1: "GEM_E_INVAL", -2: "GEM_E_FORMAT", -3: "GEM_E_CUDA", -4: "GEM_E_NO
           -6: "GEM_E_UNSUPPORTED"}
 EXPORTS = ["gem_load_program", "gem_info_get", "gem_set_inputs", "gem_step", "gem_read_outputs",
            "gem_read_state", "gem_write_state", "gem_read_state_trace", "gem_read_digests", "gem_read_ram",
-           "gem_write_ram", "gem_last_step_ms", "gem_read_profile", "gem_free", "gem_last_error"]
+           "gem_write_ram", "gem_last_step_ms", "gem_read_profile", "gem_bench_floor", "gem_free", "gem_last_error"]
 
 
 class GemConfig(ctypes.Structure):
@@ -92,6 +92,18 @@ def _p(a: Optional[np.ndarray]):
 
 def _dev_ptr(t) -> ctypes.c_void_p:
     return ctypes.c_void_p(int(t.data_ptr()))
+
+
+def bench_floor(device: int = 0, grid: int = 148, iters: int = 2000):
+    """Latency-floor microbenchmarks (gem_bench_floor): (minimal-layer clocks,
+    grid-barrier clocks) measured on `device` with `grid` co-resident CTAs."""
+    lib = load_library()
+    lib.gem_bench_floor.argtypes = [ctypes.c_int, ctypes.c_uint32, ctypes.c_uint32,
+                                    ctypes.POINTER(ctypes.c_double), ctypes.POINTER(ctypes.c_double)]
+    a, b = ctypes.c_double(), ctypes.c_double()
+    if lib.gem_bench_floor(device, grid, iters, ctypes.byref(a), ctypes.byref(b)) != 0:
+        raise GemError(lib.gem_last_error().decode())
+    return a.value, b.value
 
 
 class Simulator:

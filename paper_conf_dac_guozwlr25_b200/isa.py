@@ -42,6 +42,15 @@ class BlobInfo:
     max_chunk_words: int = 0
     max_prog_words: int = 0
     part_cost: list = None
+    part_stage: list = None
+
+    def stage_max_layers(self) -> list:
+        """Deepest partition (layers) of each stage: a lower bound on the layers
+        a cycle's critical path executes."""
+        out = [0] * max(1, self.n_stages)
+        for st, nl in zip(self.part_stage or [], self.part_layers):
+            out[st] = max(out[st], nl)
+        return out
 
     @property
     def replication(self) -> float:
@@ -59,6 +68,7 @@ class BlobInfo:
         d = dataclasses.asdict(self)
         d.pop("part_layers")
         d.pop("part_cost", None)
+        d.pop("part_stage", None)
         d.update(replication=self.replication, slot_util=self.slot_util, bytes_per_and=self.bytes_per_and,
                  levels_per_layer=self.max_levels / max(1, self.max_layers))
         return d
@@ -80,4 +90,4 @@ def blob_info(blob: bytes) -> BlobInfo:
                     max_levels=h["MAX_LEVELS"], program_bytes=4 * u64("PROG_WORDS"),
                     blob_bytes=len(blob), slots_used=u64("SLOTS_USED"), part_layers=pt[:, 3].tolist(),
                     max_chunk_words=h["MAX_CHUNK_WORDS"], max_prog_words=h["MAX_PROG_WORDS"],
-                    part_cost=pt[:, 8].tolist())
+                    part_cost=pt[:, 8].tolist(), part_stage=pt[:, 0].tolist())

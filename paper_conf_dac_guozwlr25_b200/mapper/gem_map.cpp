@@ -757,8 +757,13 @@ struct Mapper {
         for (auto x : wo_warp) nwo += x >= 0;
         uint32_t nmc = 0;
         for (uint32_t i = 0; i < n; i++) nmc += mc[i];
-        fprintf(stderr, "  layer %u: mc=%u computed=%zu need_wo=%zu wo_words=%u leaves=%u free=%zu\n", n_layers, nmc,
-                computed.size(), need_wo.size(), nwo, layer_leaves, free_words.size());
+        int topk = 0;
+        for (int k = 13; k >= 1 && !topk; k--) for (auto v : slot[k]) if (v >= 0) { topk = k; break; }
+        uint32_t maxrd = 0, maxd = 0;
+        for (uint32_t i = 0; i < n; i++) if (mc[i]) { maxrd = std::max(maxrd, rd[i]); maxd = std::max(maxd, d[i]); }
+        fprintf(stderr, "  part %p layer %u: mc=%u computed=%zu need_wo=%zu wo_words=%u leaves=%u free=%zu top_level=%d "
+                "max_rd=%u max_d=%u\n", (void*)&P, n_layers, nmc, computed.size(), need_wo.size(), nwo, layer_leaves,
+                free_words.size(), topk, maxrd, maxd);
       }
       // ---- lane-mode record of this layer (same placement, signal-level view)
       if (opt.lanes) {

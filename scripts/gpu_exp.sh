@@ -1,2 +1,1 @@
-python -c "import __graft_entry__ as g; g.build()" 2>&1 | tail -1
-python scripts/experiment.py "" "-DEXP_NO_GATHER" "-DEXP_NO_FOLD" "-DEXP_NO_LOAD" "-DEXP_NO_TOP" "-DEXP_NO_GATHER -DEXP_NO_FOLD -DEXP_NO_LOAD -DEXP_NO_TOP"
+EXP_CFGS="c1 c3" python scripts/experiment.py "" "-DGEM_TOP_ATOMIC" 2>&1 | grep -v "warning\|Remark\|^\s*$\|\^\|declared but\|const uint32_t\|__attribute"
