@@ -120,22 +120,65 @@ __device__ __forceinline__ uint64_t globaltimer_ns() {
 __device__ __forceinline__ void st_release_u64(unsigned long long* p, unsigned long long v) {
   asm volatile("st.release.gpu.global.u64 [%0], %1;" ::"l"(p), "l"(v) : "memory");
 }
+__device__ __forceinline__ unsigned long long ld_relaxed_u64(const unsigned long long* p) {
+  unsigned long long v;
+  asm volatile("ld.relaxed.gpu.global.u64 %0, [%1];" : "=l"(v) : "l"(p) : "memory");
+  return v;
+}
+__device__ __forceinline__ void spin_check(uint32_t& spins, uint64_t& start, const KParams& kp) {
+  if (++spins == 4096) start = globaltimer_ns();
+  if (spins > 4096 && (spins & 4095) == 0 && globaltimer_ns() - start > 10000000000ull) {
+    atomicExch(kp.err, 2);
+    asm volatile("trap;");
+  }
+}
+#ifndef GEM_BAR_VARIANT
+#define GEM_BAR_VARIANT 0
+#endif
 __device__ __forceinline__ void grid_sync(const KParams& kp, unsigned long long& epoch) {
   __syncthreads();
   if (gridDim.x > 1) {
     epoch++;
+#if GEM_BAR_VARIANT == 0 || GEM_BAR_VARIANT == 1
     if (threadIdx.x == 0) st_release_u64(kp.bar + (size_t)blockIdx.x * GEM_BAR_STRIDE, epoch);
     for (uint32_t f = threadIdx.x; f < gridDim.x; f += blockDim.x) {
       uint32_t spins = 0;
       uint64_t start = 0;
-      while (ld_acquire_u64(kp.bar + (size_t)f * GEM_BAR_STRIDE) < epoch) {
-        if (++spins == 4096) start = globaltimer_ns();
-        if (spins > 4096 && (spins & 4095) == 0 && globaltimer_ns() - start > 10000000000ull) {
-          atomicExch(kp.err, 2);
-          asm volatile("trap;");
-        }
+#if GEM_BAR_VARIANT == 0
+      while (ld_acquire_u64(kp.bar + (size_t)f * GEM_BAR_STRIDE) < epoch) spin_check(spins, start, kp);
+#else   // relaxed polling, one acquire fence after the flag is seen
+      while (ld_relaxed_u64(kp.bar + (size_t)f * GEM_BAR_STRIDE) < epoch) spin_check(spins, start, kp);
+      asm volatile("fence.acq_rel.gpu;" ::: "memory");
+#endif
+    }
+#elif GEM_BAR_VARIANT == 2
+    // two-phase: CTA 0 gathers the arrival flags and publishes one release word
+    unsigned long long* rel = kp.bar + (size_t)GEM_BAR_MAX_CTAS * GEM_BAR_STRIDE;
+    if (blockIdx.x == 0) {
+      for (uint32_t f = threadIdx.x + 1; f < gridDim.x; f += blockDim.x) {
+        uint32_t spins = 0;
+        uint64_t start = 0;
+        while (ld_acquire_u64(kp.bar + (size_t)f * GEM_BAR_STRIDE) < epoch) spin_check(spins, start, kp);
+      }
+      __syncthreads();
+      if (threadIdx.x == 0) st_release_u64(rel, epoch);
+    } else {
+      if (threadIdx.x == 0) {
+        st_release_u64(kp.bar + (size_t)blockIdx.x * GEM_BAR_STRIDE, epoch);
+        uint32_t spins = 0;
+        uint64_t start = 0;
+        while (ld_acquire_u64(rel) < epoch) spin_check(spins, start, kp);
       }
     }
+#else   // single counter: red.release arrive, acquire polling by thread 0
+    if (threadIdx.x == 0) {
+      asm volatile("red.release.gpu.global.add.u64 [%0], 1;" ::"l"(kp.bar + (size_t)(GEM_BAR_MAX_CTAS + 1) * GEM_BAR_STRIDE) : "memory");
+      uint32_t spins = 0;
+      uint64_t start = 0;
+      while (ld_acquire_u64(kp.bar + (size_t)(GEM_BAR_MAX_CTAS + 1) * GEM_BAR_STRIDE) < epoch * gridDim.x)
+        spin_check(spins, start, kp);
+    }
+#endif
     __syncthreads();
   }
 }
@@ -295,20 +338,42 @@ __device__ __forceinline__ void sts(uint32_t addr, uint32_t v) {
 // Gather of one leaf entry: rotate the source state word so bit b lands on
 // leaf position p (gem_isa.h).  S sits at the start of dynamic shared memory,
 // so the entry's byte-offset field plus the window base addresses it.
-__device__ __forceinline__ uint32_t leaf_rot(uint32_t s_base, uint32_t e, uint32_t byte_mask) {
-  const uint32_t s = lds(s_base + ((e >> 5) & byte_mask));
+// Dynamic shared memory of both kernels; the partition state S is at offset 0.
+extern __shared__ __align__(16) uint32_t g_smem[];
+
+// Gather loads are plain C++ loads from the shared-memory state (the compiler
+// keeps the per-stream base in a uniform register: LDS [R + UR], no per-leaf add).
+__device__ __forceinline__ uint32_t ldsb(const uint32_t* S, uint32_t byteoff) {
+  return *reinterpret_cast<const uint32_t*>(reinterpret_cast<const char*>(S) + byteoff);
+}
+// Single-stream fast path: the state sits at the start of dynamic shared
+// memory, shared-window address GEM_S0_ADDR (checked at kernel start), so the
+// base is an LDS immediate and a leaf's address is just its byte offset.
+#define GEM_S0_ADDR 1024
+template <bool kS0>
+__device__ __forceinline__ uint32_t ldst(const uint32_t* S, uint32_t byteoff) {
+  if (kS0) {
+    uint32_t v;
+    asm volatile("ld.shared.u32 %0, [%1+1024];" : "=r"(v) : "r"(byteoff));
+    return v;
+  }
+  return ldsb(S, byteoff);
+}
+template <bool kS0 = false>
+__device__ __forceinline__ uint32_t leaf_rot(const uint32_t* S, uint32_t e, uint32_t byte_mask) {
+  const uint32_t s = ldst<kS0>(S, (e >> 5) & byte_mask);
   return __funnelshift_l(s, s, e);   // rotl(s, e & 31)
 }
-template <int N4>
-__device__ __forceinline__ uint32_t gather_sparse(uint32_t s_base, const uint4* e) {
+template <int N4, bool kS0>
+__device__ __forceinline__ uint32_t gather_sparse(const uint32_t* S, const uint4* e) {
   // four independent accumulators keep the OR chain short
   uint32_t v0 = 0, v1 = 0, v2 = 0, v3 = 0;
 #pragma unroll
   for (int g = 0; g < N4; g++) {
-    v0 |= leaf_rot(s_base, e[g].x, 0x7FFFu) & (1u << GEM_LEAF_POS(e[g].x));
-    v1 |= leaf_rot(s_base, e[g].y, 0x7FFFu) & (1u << GEM_LEAF_POS(e[g].y));
-    v2 |= leaf_rot(s_base, e[g].z, 0x7FFFu) & (1u << GEM_LEAF_POS(e[g].z));
-    v3 |= leaf_rot(s_base, e[g].w, 0x7FFFu) & (1u << GEM_LEAF_POS(e[g].w));
+    v0 |= leaf_rot<kS0>(S, e[g].x, 0x7FFFu) & (1u << GEM_LEAF_POS(e[g].x));
+    v1 |= leaf_rot<kS0>(S, e[g].y, 0x7FFFu) & (1u << GEM_LEAF_POS(e[g].y));
+    v2 |= leaf_rot<kS0>(S, e[g].z, 0x7FFFu) & (1u << GEM_LEAF_POS(e[g].z));
+    v3 |= leaf_rot<kS0>(S, e[g].w, 0x7FFFu) & (1u << GEM_LEAF_POS(e[g].w));
   }
   return (v0 | v1) | (v2 | v3);
 }
@@ -341,7 +406,9 @@ __device__ __forceinline__ void load_layer(const uint32_t* L, LayerRegs& R) {
 
 // Rows a3-a5 of one layer with pre-loaded records: gather (bit permutation),
 // 13-level boomerang fold, write-outs.  No trailing barrier.
-__device__ __forceinline__ void exec_layer(const LayerRegs& R, uint32_t s_base, uint32_t* topb, uint32_t bid,
+template <bool kS0>
+__device__ __forceinline__ void exec_layer(const LayerRegs& R, uint32_t s_base, const uint32_t* Sj, uint32_t* topb,
+                                           uint32_t bid,
                                            uint32_t fl = 99, unsigned long long* fsub = nullptr) {
   const uint32_t lane = threadIdx.x & 31, warp = threadIdx.x >> 5;
   (void)fl;
@@ -363,11 +430,11 @@ __device__ __forceinline__ void exec_layer(const LayerRegs& R, uint32_t s_base, 
           if (g >= 2) continue;
 #endif
 #ifdef EXP_NO_CONFLICT   // timing experiment: same instructions, words 0..31 only (conflict-free)
-          const uint32_t lo = lds(s_base + ((q[k] >> 3) & 0x7Cu));
-          const uint32_t hi = lds(s_base + ((q[k] >> 19) & 0x7Cu));
+          const uint32_t lo = ldst<kS0>(Sj, (q[k] >> 3) & 0x7Cu);
+          const uint32_t hi = ldst<kS0>(Sj, (q[k] >> 19) & 0x7Cu);
 #else
-          const uint32_t lo = lds(s_base + ((q[k] >> 3) & 0x1FFCu));
-          const uint32_t hi = lds(s_base + ((q[k] >> 19) & 0x1FFCu));
+          const uint32_t lo = ldst<kS0>(Sj, (q[k] >> 3) & 0x1FFCu);
+          const uint32_t hi = ldst<kS0>(Sj, (q[k] >> 19) & 0x1FFCu);
 #endif
           acc[k] |= (__funnelshift_l(lo, lo, q[k]) & (1u << (8 * g + 2 * k))) |
                     (__funnelshift_l(hi, hi, q[k] >> 16) & (1u << (8 * g + 2 * k + 1)));
@@ -378,19 +445,19 @@ __device__ __forceinline__ void exec_layer(const LayerRegs& R, uint32_t s_base, 
       // entry j of the lane fills leaf position j: rotate + LOP3 with an immediate mask
 #pragma unroll
       for (uint32_t g = 0; g < 8; g++) {
-        v |= leaf_rot(s_base, R.e[g].x, 0xFFFFFFFFu) & (1u << (4 * g + 0));
-        v |= leaf_rot(s_base, R.e[g].y, 0xFFFFFFFFu) & (1u << (4 * g + 1));
-        v |= leaf_rot(s_base, R.e[g].z, 0xFFFFFFFFu) & (1u << (4 * g + 2));
-        v |= leaf_rot(s_base, R.e[g].w, 0xFFFFFFFFu) & (1u << (4 * g + 3));
+        v |= leaf_rot<kS0>(Sj, R.e[g].x, 0xFFFFFFFFu) & (1u << (4 * g + 0));
+        v |= leaf_rot<kS0>(Sj, R.e[g].y, 0xFFFFFFFFu) & (1u << (4 * g + 1));
+        v |= leaf_rot<kS0>(Sj, R.e[g].z, 0xFFFFFFFFu) & (1u << (4 * g + 2));
+        v |= leaf_rot<kS0>(Sj, R.e[g].w, 0xFFFFFFFFu) & (1u << (4 * g + 3));
       }
     } else if (n4 <= 1) {
-      v = gather_sparse<1>(s_base, R.e);
+      v = gather_sparse<1, kS0>(Sj, R.e);
     } else if (n4 <= 2) {
-      v = gather_sparse<2>(s_base, R.e);
+      v = gather_sparse<2, kS0>(Sj, R.e);
     } else if (n4 <= 4) {
-      v = gather_sparse<4>(s_base, R.e);
+      v = gather_sparse<4, kS0>(Sj, R.e);
     } else {
-      v = gather_sparse<8>(s_base, R.e);
+      v = gather_sparse<8, kS0>(Sj, R.e);
     }
 #else   // timing experiment only (wrong results)
     v = R.e[0].x ^ R.e[1].y ^ R.lc.w;
@@ -573,7 +640,10 @@ __device__ void run_partition(const KParams& kp, ProgSrc& ps, uint32_t* S, uint3
     unsigned long long* fsub = nullptr;
 #endif
     // stream j uses named barrier 1 + j (group <= GEM_MAX_GROUP < 16)
-    for (uint32_t j = 0; j < nst; j++) exec_layer(R, s_base + 4 * j * SW, topb + 16 * j, 1 + j, fl, fsub);
+    if (nst == 1 && s_base == GEM_S0_ADDR) exec_layer<true>(R, s_base, g_smem, topb, 1, fl, fsub);
+    else
+      for (uint32_t j = 0; j < nst; j++)
+        exec_layer<false>(R, s_base + 4 * j * SW, g_smem + j * SW, topb + 16 * j, 1 + j, fl, fsub);
     FPROF(l, 1);
     const bool ptop = (R.flags & GEM_LF_USES_TOP) != 0;
     const uint32_t ptopc = R.topc, ptopwo = R.topwo;
@@ -1366,7 +1436,7 @@ int gem_load_program(const void* blob, size_t nbytes, const gem_config* cfg, gem
     CK(dalloc(&sim->d_cut, S * std::max<uint32_t>(sim->cut_words, 1) * 4));
   }
   CK(dalloc(&sim->d_mem, S * sim->n_rams * (size_t)GEM_RAM_WORDS * 4));
-  CK(dalloc(&sim->d_bar, (size_t)GEM_BAR_MAX_CTAS * GEM_BAR_STRIDE * 8));
+  CK(dalloc(&sim->d_bar, (size_t)(GEM_BAR_MAX_CTAS + 2) * GEM_BAR_STRIDE * 8));
   CK(dalloc(&sim->d_err, 64));
   CK(cudaMemset(sim->d_err, 0, 64));
   // initial state: flops = init (U5), RD = 0, RAM = 0 (U10)
@@ -1493,7 +1563,7 @@ int gem_step(gem_sim* sim, uint64_t ncycles) {
     kp.prof_cycles = pc;
     kp.fprof = sim->d_fprof;
   }
-  CK(cudaMemsetAsync(sim->d_bar, 0, (size_t)GEM_BAR_MAX_CTAS * GEM_BAR_STRIDE * 8, sim->stream));
+  CK(cudaMemsetAsync(sim->d_bar, 0, (size_t)(GEM_BAR_MAX_CTAS + 2) * GEM_BAR_STRIDE * 8, sim->stream));
   if (sim->flags & GEM_F_DIGEST)
     CK(cudaMemsetAsync(sim->d_digest, 0, (size_t)sim->n_streams * sim->out_cap * 8, sim->stream));
   if (sim->lanes) {
@@ -1527,9 +1597,9 @@ int gem_bench_floor(int device, uint32_t grid, uint32_t iters, double* layer_clk
   unsigned long long *d_out = nullptr, *d_bar = nullptr;
   int* d_err = nullptr;
   CK(dalloc(&d_out, 64));
-  CK(dalloc(&d_bar, (size_t)GEM_BAR_MAX_CTAS * GEM_BAR_STRIDE * 8));
+  CK(dalloc(&d_bar, (size_t)(GEM_BAR_MAX_CTAS + 2) * GEM_BAR_STRIDE * 8));
   CK(dalloc(&d_err, 64));
-  CK(cudaMemset(d_bar, 0, (size_t)GEM_BAR_MAX_CTAS * GEM_BAR_STRIDE * 8));
+  CK(cudaMemset(d_bar, 0, (size_t)(GEM_BAR_MAX_CTAS + 2) * GEM_BAR_STRIDE * 8));
   unsigned long long h[2] = {0, 0};
   floor_layer_kernel<<<1, GEM_THREADS>>>(d_out, 64);
   floor_layer_kernel<<<1, GEM_THREADS>>>(d_out, iters);
