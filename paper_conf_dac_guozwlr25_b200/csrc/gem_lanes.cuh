@@ -46,78 +46,110 @@ __device__ __forceinline__ void load_lane_layer(const uint32_t* L, LaneRegs& R) 
   }
 }
 
-// slot (A ^ XA) & ((B ^ XB) | OB) with the masks taken from bit b of the constants
-__device__ __forceinline__ uint32_t lslot(uint32_t A, uint32_t B, uint32_t xa, uint32_t xb, uint32_t ob, uint32_t b) {
-  const uint32_t XA = (uint32_t)((int32_t)(xa << (31u - b)) >> 31);
-  const uint32_t XB = (uint32_t)((int32_t)(xb << (31u - b)) >> 31);
-  const uint32_t OB = (uint32_t)((int32_t)(ob << (31u - b)) >> 31);
-  return (A ^ XA) & ((B ^ XB) | OB);
+// K-word vectors: a work item runs K 32-stream groups together, their lane
+// words interleaved in shared memory (word w of group j at S[w*K + j]) so a
+// leaf is one LDS.K and a write-out one STS.K, and each slot's constants are
+// decoded once for all K groups.
+template <int K>
+__device__ __forceinline__ void ldsK(uint32_t addr, uint32_t (&v)[K]) {
+  if (K == 1) {
+    asm volatile("ld.shared.u32 %0, [%1];" : "=r"(v[0]) : "r"(addr));
+  } else if (K == 2) {
+    asm volatile("ld.shared.v2.u32 {%0, %1}, [%2];" : "=r"(v[0]), "=r"(v[1]) : "r"(addr));
+  } else {
+    asm volatile("ld.shared.v4.u32 {%0, %1, %2, %3}, [%4];"
+                 : "=r"(v[0]), "=r"(v[1]), "=r"(v[2]), "=r"(v[3]) : "r"(addr));
+  }
+}
+template <int K>
+__device__ __forceinline__ void stsK(uint32_t addr, const uint32_t (&v)[K]) {
+  if (K == 1) {
+    asm volatile("st.shared.u32 [%0], %1;" ::"r"(addr), "r"(v[0]) : "memory");
+  } else if (K == 2) {
+    asm volatile("st.shared.v2.u32 [%0], {%1, %2};" ::"r"(addr), "r"(v[0]), "r"(v[1]) : "memory");
+  } else {
+    asm volatile("st.shared.v4.u32 [%0], {%1, %2, %3, %4};" ::"r"(addr), "r"(v[0]), "r"(v[1]), "r"(v[2]),
+                 "r"(v[3]) : "memory");
+  }
+}
+// bit b of a packed constant word as a full mask
+__device__ __forceinline__ uint32_t cmask(uint32_t c, uint32_t b) { return (uint32_t)((int32_t)(c << (31u - b)) >> 31); }
+template <int K>
+__device__ __forceinline__ void kslot(uint32_t (&o)[K], const uint32_t (&A)[K], const uint32_t (&B)[K], uint32_t xa,
+                                      uint32_t xb, uint32_t ob, uint32_t b) {
+  const uint32_t XA = cmask(xa, b), XB = cmask(xb, b), OB = cmask(ob, b);
+#pragma unroll
+  for (int j = 0; j < K; j++) o[j] = (A[j] ^ XA) & ((B[j] ^ XB) | OB);
+}
+template <int K>
+__device__ __forceinline__ void lane_woK(uint32_t s_base, uint32_t mask, uint32_t base, uint32_t b,
+                                         const uint32_t (&v)[K]) {
+  if ((mask >> b) & 1u) stsK<K>(s_base + 4u * K * (base + __popc(mask & ((1u << b) - 1u))), v);
 }
 
-__device__ __forceinline__ void lane_wo(uint32_t s_base, uint32_t mask, uint32_t base, uint32_t b, uint32_t v) {
-  if ((mask >> b) & 1u) sts(s_base + 4u * (base + __popc(mask & ((1u << b) - 1u))), v);
-}
-
-// Rows a3-a5 of one layer for one 32-stream group.  topv: 8 warp results + counter.
+// Rows a3-a5 of one layer for the K groups of a work item.  topv[warp][K].
+template <int K>
 __device__ __forceinline__ void exec_lane_layer(const LaneRegs& R, uint32_t s_base, uint32_t* topv, uint32_t bid) {
   const uint32_t lane = threadIdx.x & 31, warp = threadIdx.x >> 5;
   const bool uses_top = (R.flags & GEM_LF_USES_TOP) != 0;
   if ((R.flags >> warp) & 1u) {
     const uint32_t xa = R.lc.x, xb = R.lc.y, ob = R.lc.z, mask = R.lc.w;
-    uint32_t v[32];
     const uint32_t q8[4][4] = {{R.e[0].x, R.e[0].y, R.e[0].z, R.e[0].w}, {R.e[1].x, R.e[1].y, R.e[1].z, R.e[1].w},
                                {R.e[2].x, R.e[2].y, R.e[2].z, R.e[2].w}, {R.e[3].x, R.e[3].y, R.e[3].z, R.e[3].w}};
+    // leaf i (0..31) = u16 lane word: entry 8g+2k in the low half of q8[g][k], +1 in the high half
+    auto leaf = [&](uint32_t i) -> uint32_t {
+      const uint32_t q = q8[i >> 3][(i & 7) >> 1];
+      return (i & 1) ? (q >> 16) : (q & 0xFFFFu);
+    };
+    // written slots go to consecutive lane words (slot-bit order) from R.base
+    uint32_t wp = s_base + 4u * K * R.base;
+    uint32_t r1[16][K];
 #pragma unroll
-    for (uint32_t g = 0; g < 4; g++)
+    for (uint32_t q = 0; q < 16; q++) {          // level 1: A = leaf q, B = leaf q+16
+      uint32_t a[K], b[K];
+      ldsK<K>(s_base + 4u * K * leaf(q), a);
+      ldsK<K>(s_base + 4u * K * leaf(q + 16), b);
+      kslot<K>(r1[q], a, b, xa, xb, ob, q);
+      if (mask & (1u << q)) { stsK<K>(wp, r1[q]); wp += 4u * K; }
+    }
+    uint32_t r2[8][K], r3[4][K], r4[2][K], x[K];
 #pragma unroll
-      for (uint32_t k = 0; k < 4; k++) {
-        v[8 * g + 2 * k] = lds(s_base + 4u * (q8[g][k] & 0xFFFFu));
-        v[8 * g + 2 * k + 1] = lds(s_base + 4u * (q8[g][k] >> 16));
-      }
-    // levels 1-5 inside the thread.  Written slots go to consecutive lane words
-    // in slot-bit order: a running store pointer advanced per written slot.
-    uint32_t wp = s_base + 4u * R.base;
-#define LWO(b_, v_)                                   \
-  do {                                              \
-    if (mask & (1u << (b_))) { sts(wp, (v_)); wp += 4u; } \
-  } while (0)
-#pragma unroll
-    for (uint32_t q = 0; q < 16; q++) v[q] = lslot(v[q], v[q + 16], xa, xb, ob, q);
-    if (mask & 0xFFFFu) {
-#pragma unroll
-      for (uint32_t q = 0; q < 16; q++) LWO(q, v[q]);
+    for (uint32_t q = 0; q < 8; q++) {
+      kslot<K>(r2[q], r1[q], r1[q + 8], xa, xb, ob, 16 + q);
+      if (mask & (1u << (16 + q))) { stsK<K>(wp, r2[q]); wp += 4u * K; }
     }
 #pragma unroll
-    for (uint32_t q = 0; q < 8; q++) v[q] = lslot(v[q], v[q + 8], xa, xb, ob, 16 + q);
-#pragma unroll
-    for (uint32_t q = 0; q < 4; q++) v[8 + q] = lslot(v[q], v[q + 4], xa, xb, ob, 24 + q);
-#pragma unroll
-    for (uint32_t q = 0; q < 2; q++) v[12 + q] = lslot(v[8 + q], v[8 + q + 2], xa, xb, ob, 28 + q);
-    uint32_t x = lslot(v[12], v[13], xa, xb, ob, 30);
-    if (mask & 0x7FFF0000u) {
-#pragma unroll
-      for (uint32_t q = 0; q < 8; q++) LWO(16 + q, v[q]);
-#pragma unroll
-      for (uint32_t q = 0; q < 4; q++) LWO(24 + q, v[8 + q]);
-      LWO(28, v[12]);
-      LWO(29, v[13]);
-      LWO(30, x);
+    for (uint32_t q = 0; q < 4; q++) {
+      kslot<K>(r3[q], r2[q], r2[q + 4], xa, xb, ob, 24 + q);
+      if (mask & (1u << (24 + q))) { stsK<K>(wp, r3[q]); wp += 4u * K; }
     }
-#undef LWO
+#pragma unroll
+    for (uint32_t q = 0; q < 2; q++) {
+      kslot<K>(r4[q], r3[q], r3[q + 2], xa, xb, ob, 28 + q);
+      if (mask & (1u << (28 + q))) { stsK<K>(wp, r4[q]); wp += 4u * K; }
+    }
+    kslot<K>(x, r4[0], r4[1], xa, xb, ob, 30);
+    if (mask & (1u << 30)) stsK<K>(wp, x);
     // levels 6-10 across the warp: slot q of a level lives in lane q
     const uint32_t wxa = R.wc.x, wxb = R.wc.y, wob = R.wc.z, wmask = R.wc.w;
     const uint32_t offs[5] = {0, 16, 24, 28, 30};
 #pragma unroll
     for (uint32_t k = 0; k < 5; k++) {
       const uint32_t half = 16u >> k;
-      const uint32_t y = __shfl_down_sync(0xFFFFFFFFu, x, half);
+      uint32_t y[K];
+#pragma unroll
+      for (int j = 0; j < K; j++) y[j] = __shfl_down_sync(0xFFFFFFFFu, x[j], half);
       const uint32_t b = offs[k] + (lane & (half - 1u));
-      x = lslot(x, y, wxa, wxb, wob, b);
-      if (lane < half) lane_wo(s_base, wmask, R.wbase, b, x);
+      kslot<K>(x, x, y, wxa, wxb, wob, b);
+      if (lane < half) lane_woK<K>(s_base, wmask, R.wbase, b, x);
     }
-    if (uses_top && lane == 0) topv[warp] = x;
+    if (uses_top && lane == 0) {
+#pragma unroll
+      for (int j = 0; j < K; j++) topv[warp * K + j] = x[j];
+    }
   } else if (uses_top && lane == 0) {
-    topv[warp] = 0u;
+#pragma unroll
+    for (int j = 0; j < K; j++) topv[warp * K + j] = 0u;
   }
   // levels 11-13: warps 1-7 arrive on named barrier `bid`; warp 0 folds in
   // top_lane_layer after loading the next layer's records
@@ -126,30 +158,37 @@ __device__ __forceinline__ void exec_lane_layer(const LaneRegs& R, uint32_t s_ba
 
 // Levels 11-13 (warp 0): wait for the 8 warp words on named barrier `bid`;
 // lanes 0-7 hold them and three shuffle levels fold them.
+template <int K>
 __device__ __forceinline__ void top_lane_layer(uint32_t topc, uint32_t topwo, uint32_t s_base, const uint32_t* topv,
                                                uint32_t bid) {
   asm volatile("bar.sync %0, %1;" ::"r"(bid), "r"(GEM_THREADS) : "memory");
   const uint32_t lane = threadIdx.x & 31;
   const uint32_t xa = topc & 0xFFu, xb = (topc >> 8) & 0xFFu, ob = (topc >> 16) & 0xFFu;
   const uint32_t tm = topwo & 0x7Fu, tb = topwo >> 8;
-  uint32_t x = lds(smem_u32(topv) + 4u * (lane & 7u));
-  uint32_t y = __shfl_down_sync(0xFFFFFFFFu, x, 4);
-  x = lslot(x, y, xa, xb, ob, lane & 3u);                 // level 11: slots 0-3
-  if (lane < 4) lane_wo(s_base, tm, tb, lane, x);
-  y = __shfl_down_sync(0xFFFFFFFFu, x, 2);
-  x = lslot(x, y, xa, xb, ob, 4u + (lane & 1u));          // level 12: slots 4-5
-  if (lane < 2) lane_wo(s_base, tm, tb, 4u + lane, x);
-  y = __shfl_down_sync(0xFFFFFFFFu, x, 1);
-  x = lslot(x, y, xa, xb, ob, 6u);                        // level 13: slot 6
-  if (lane == 0) lane_wo(s_base, tm, tb, 6u, x);
+  uint32_t x[K], y[K];
+#pragma unroll
+  for (int j = 0; j < K; j++) x[j] = topv[(lane & 7u) * K + j];
+#pragma unroll
+  for (int j = 0; j < K; j++) y[j] = __shfl_down_sync(0xFFFFFFFFu, x[j], 4);
+  kslot<K>(x, x, y, xa, xb, ob, lane & 3u);                 // level 11: slots 0-3
+  if (lane < 4) lane_woK<K>(s_base, tm, tb, lane, x);
+#pragma unroll
+  for (int j = 0; j < K; j++) y[j] = __shfl_down_sync(0xFFFFFFFFu, x[j], 2);
+  kslot<K>(x, x, y, xa, xb, ob, 4u + (lane & 1u));          // level 12: slots 4-5
+  if (lane < 2) lane_woK<K>(s_base, tm, tb, 4u + lane, x);
+#pragma unroll
+  for (int j = 0; j < K; j++) y[j] = __shfl_down_sync(0xFFFFFFFFu, x[j], 1);
+  kslot<K>(x, x, y, xa, xb, ob, 6u);                        // level 13: slot 6
+  if (lane == 0) lane_woK<K>(s_base, tm, tb, 6u, x);
 }
 
-// One work item: partition p for 32-stream group g (streams 32g .. 32g+nvalid-1).
+// One work item: partition p for the 32-stream groups g0 .. g0+ng-1 (ng <= K;
+// groups ng..K-1 of the vectors are padding and never committed).
+template <int K>
 __device__ void run_lane_partition(const KParams& kp, ProgSrc& ps, uint32_t* S, uint32_t* ramp, uint32_t* topv,
                                    uint32_t p, uint32_t g0, uint32_t ng, uint32_t c, uint32_t cur, uint32_t nxt) {
   const uint32_t tid = threadIdx.x;
   const uint32_t s_base = smem_u32(S);
-  const uint32_t LW = kp.state_words;   // lane words per group
   const LaneIdx X{kp.n_groups};
   const uint32_t* gprog = kp.lprog + __ldg(kp.parts + p * GP_WORDS + GP_LANE_OFF);
   uint32_t next_chunk = prologue_count_lane(kp, ps, p), next_off = 0;
@@ -161,7 +200,7 @@ __device__ void run_lane_partition(const KParams& kp, ProgSrc& ps, uint32_t* S, 
   const uint4 h1 = *(reinterpret_cast<const uint4*>(C0) + 1);
   const uint4 h2 = *(reinterpret_cast<const uint4*>(C0) + 2);
   const uint32_t n_gread = h0.y, n_layers = h0.z, n_out = h0.w;
-  const uint32_t n_ram = h1.x, off_gread = h1.z, off_layers = h1.w;
+  const uint32_t n_ram = h1.x, off_gread = h1.z;
   const uint32_t off_out = h2.x, off_ram = h2.y, off_chunks = h2.z, n_chunks = h2.w;
   for (uint32_t k = tid; k < n_chunks; k += GEM_THREADS) ps.ctab[k] = C0[off_chunks + k];
   // chunk 0 = header + chunk table; the gread list (after the last chunk) is
@@ -174,7 +213,7 @@ __device__ void run_lane_partition(const KParams& kp, ProgSrc& ps, uint32_t* S, 
       next_chunk++;
     }
   };
-  // ---- a2: input ports (once per cycle) for the 32 streams of the group
+  // ---- a2: input ports (once per cycle) for the groups of the item
   // loads of 4 (entry, group) pairs per thread are issued before their stores
   const uint2* gr = reinterpret_cast<const uint2*>(gprog + off_gread);
   const uint32_t n_gr = n_gread * ng;
@@ -194,29 +233,27 @@ __device__ void run_lane_partition(const KParams& kp, ProgSrc& ps, uint32_t* S, 
         else if (reg == GEM_R_RD) a = kp.rd + X.q(cur, kp.n_rams * 32, b, g);
         else a = kp.cut + X.q(0, kp.cut_words * 32, b, g);
         v[u] = __ldcg(a);
-        dst[u] = j * LW + e.y;
+        dst[u] = e.y * K + j;
       }
     }
 #pragma unroll
     for (uint32_t u = 0; u < 4; u++)
       if (dst[u] != ~0u) sts(s_base + 4u * dst[u], v[u]);
   }
-  if (tid < ng) S[tid * LW] = 0u;
+  if (tid < K) S[tid] = 0u;   // lane word 0 = constant 0 for every group
   LaneRegs R;
   if (n_layers) load_lane_layer(ring_wait(ps), R);
   __syncthreads();
-  ps.seq_free += n_layers ? 2 : 1;
+  ps.seq_free = ps.seq_wait;
   refill();
   for (uint32_t l = 0; l < n_layers; l++) {
-    for (uint32_t j = 0; j < ng; j++)   // named barrier 1 + j, as in run_partition
-      exec_lane_layer(R, s_base + 4u * j * LW, topv + 16 * j, 1 + j);
+    exec_lane_layer<K>(R, s_base, topv, 1);
     const bool ptop = (R.flags & GEM_LF_USES_TOP) != 0;
     const uint32_t ptopc = R.topc, ptopwo = R.topwo;
     if (l + 1 < n_layers) load_lane_layer(ring_wait(ps), R);
-    if (ptop && (threadIdx.x >> 5) == 0)
-      for (uint32_t j = 0; j < ng; j++) top_lane_layer(ptopc, ptopwo, s_base + 4u * j * LW, topv + 16 * j, 1 + j);
+    if (ptop && (threadIdx.x >> 5) == 0) top_lane_layer<K>(ptopc, ptopwo, s_base, topv, 1);
     __syncthreads();
-    if (l + 1 < n_layers) ps.seq_free++;
+    ps.seq_free = ps.seq_wait;
     refill();
   }
   // ---- a6: endpoint commit: one lane word per endpoint bit
@@ -225,7 +262,7 @@ __device__ void run_lane_partition(const KParams& kp, ProgSrc& ps, uint32_t* S, 
   for (uint32_t jj = tid; jj < n_out * ng; jj += GEM_THREADS) {
     const uint32_t j = jj / n_out, o = jj - j * n_out, g = g0 + j;
     const uint2 e = oe[o];
-    const uint32_t v = lds(s_base + 4u * (j * LW + (e.y & 0xFFFFu))) ^ ((e.y >> 31) ? 0xFFFFFFFFu : 0u);
+    const uint32_t v = lds(s_base + 4u * ((e.y & 0xFFFFu) * K + j)) ^ ((e.y >> 31) ? 0xFFFFFFFFu : 0u);
     const uint32_t reg = e.x >> 24, b = e.x & 0xFFFFFFu;
     if (reg == GEM_R_Q) __stcg(kp.q + X.q(nxt, kp.q_words * 32, b, g), v);
     else if (reg == GEM_R_PO) __stcg(kp.po_lane + X.q(c, kp.po_words * 32, b, g), v);
@@ -295,10 +332,11 @@ __device__ void record_state_lane(const KParams& kp, uint32_t c, uint32_t buf) {
   }
 }
 
+template <int K>
 __global__ void __launch_bounds__(GEM_THREADS, 2) gem_lane_kernel(const KParams kp) {
   extern __shared__ __align__(16) uint32_t smem[];
-  // layout: S[lane_words] | area (ring) | ctab[256] | ramp[ram_words] | topv[16] | mbar[8 x u64]
-  uint32_t* S = smem;                                   // [group][lane words]
+  // layout: S[lane_words][K] | area (ring) | ctab[256] | ramp[K][ram_words] | topv[8][K] | mbar[8 x u64]
+  uint32_t* S = smem;                                   // [lane word][group] interleaved
   uint32_t* area = S + kp.group * kp.state_words;
   uint32_t* ctab = area + kp.area_words;
   uint32_t* ramp = ctab + GEM_MAX_CHUNKS;               // [group][ramp_words]
@@ -345,7 +383,7 @@ __global__ void __launch_bounds__(GEM_THREADS, 2) gem_lane_kernel(const KParams 
       for (uint32_t k = kb; k < ke; k++) {
         const uint2 it = __ldg(&kp.wl_items[k]);
         const uint32_t g0 = it.y >> 5;
-        run_lane_partition(kp, ps, S, ramp, topv, it.x, g0, min(kp.group, kp.n_groups - g0), c, cur, nxt);
+        run_lane_partition<K>(kp, ps, S, ramp, topv, it.x, g0, min((uint32_t)K, kp.n_groups - g0), c, cur, nxt);
         uint32_t nk = ~0u;
         if (k + 1 < ke) nk = k + 1;
         for (uint32_t s2 = s + 1; nk == ~0u && s2 < kp.n_stages; s2++)

@@ -1269,6 +1269,10 @@ static int plan_launch(gem_sim* sim, uint32_t max_chunk_words, uint32_t grid_lim
   return GEM_OK;
 }
 
+static const void* lane_kernel_for(uint32_t k) {
+  return k >= 4 ? (const void*)gem_lane_kernel<4> : k == 2 ? (const void*)gem_lane_kernel<2> : (const void*)gem_lane_kernel<1>;
+}
+
 // Lane mode launch: one CTA per SM (all shared memory for the lane state and
 // the program ring), work items = (partition, 32-stream group), LPT lists.
 static int plan_launch_lanes(gem_sim* sim, uint32_t grid_limit) {
@@ -1282,7 +1286,7 @@ static int plan_launch_lanes(gem_sim* sim, uint32_t grid_limit) {
   const uint32_t slot = (sim->lane_max_chunk + 3u) & ~3u;
   const char* ge = getenv("GEM_LANE_GROUPS");
   const char* be = getenv("GEM_LANE_BPS");
-  const uint32_t want_gl = std::min<uint32_t>(ge ? (uint32_t)atoi(ge) : 4, GEM_MAX_GROUP);
+  const uint32_t want_gl = std::min<uint32_t>(ge ? (uint32_t)atoi(ge) : 4, 4);
   // prefer 2 CTAs per SM (16 warps to hide latency), then as many 32-stream
   // groups per work item as fit beside a >= 2-slot ring
   uint32_t bps = 0, gl = 0, budget = 0;
@@ -1290,6 +1294,7 @@ static int plan_launch_lanes(gem_sim* sim, uint32_t grid_limit) {
     if (be && (uint32_t)atoi(be) != b) continue;
     const uint32_t bud = (uint32_t)std::min<int64_t>(optin, per_sm / (int64_t)b - 1024);
     for (uint32_t k = std::max<uint32_t>(1, std::min(want_gl, sim->n_groups)); k >= 1; k--) {
+      if (k == 3) continue;   // the kernel is instantiated for K = 1, 2, 4 interleaved groups
       const uint64_t words = (uint64_t)k * (sim->lane_words + sim->ramp_words + 16) + GEM_MAX_CHUNKS + 16 + 2 * slot;
       if (words * 4 <= bud) { bps = b; gl = k; budget = bud; break; }
     }
@@ -1308,9 +1313,10 @@ static int plan_launch_lanes(gem_sim* sim, uint32_t grid_limit) {
   if (grid_limit) grid = std::max<uint32_t>(1, std::min(grid, grid_limit));
   grid = std::min<uint32_t>(grid, GEM_BAR_MAX_CTAS);
   const uint32_t smem = (fixed_words + ring * slot) * 4;
-  CK(cudaFuncSetAttribute(gem_lane_kernel, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem));
+  const void* lk = lane_kernel_for(gl);
+  CK(cudaFuncSetAttribute(lk, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem));
   int occ = 0;
-  CK(cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ, gem_lane_kernel, GEM_THREADS, smem));
+  CK(cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ, lk, GEM_THREADS, smem));
   if ((uint32_t)occ < bps) return fail(GEM_E_UNSUPPORTED, "lane kernel cannot be co-resident");
   std::vector<uint32_t> off;
   std::vector<uint2> items;
@@ -1577,7 +1583,7 @@ int gem_step(gem_sim* sim, uint64_t ncycles) {
   }
   void* args[] = {&kp};
   CK(cudaEventRecord(sim->ev0, sim->stream));
-  CK(cudaLaunchCooperativeKernel(sim->lanes ? (const void*)gem_lane_kernel : (const void*)gem_step_kernel,
+  CK(cudaLaunchCooperativeKernel(sim->lanes ? lane_kernel_for(sim->lane_groups) : (const void*)gem_step_kernel,
                                  dim3(sim->grid), dim3(GEM_THREADS), args, sim->smem_bytes, sim->stream));
   CK(cudaEventRecord(sim->ev1, sim->stream));
   sim->in_head += (uint32_t)ncycles;

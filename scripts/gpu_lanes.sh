@@ -1,4 +1,3 @@
 python -c "import __graft_entry__ as g; g.build()" 2>&1 | tail -1
-timeout 1200 python -m pytest tests/test_gpu.py -x -q -k "c5" 2>&1 | tail -2
-python scripts/prof_run.py --cfg c5 --cycles 50 --streams 4096 2>&1 | grep "launch 1\|n_pi" | cut -c1-400
-GEM_LANE_BPS=1 python scripts/prof_run.py --cfg c5 --cycles 50 --streams 4096 2>&1 | grep "launch 1"
+timeout 1200 python -m pytest tests -m gpu -x -q 2>&1 | tail -2
+for cfg in "2 1" "2 2" "1 1" "1 2" "1 4"; do set -- $cfg; echo "bps=$1 groups=$2"; GEM_LANE_BPS=$1 GEM_LANE_GROUPS=$2 timeout 300 python bench.py --workload c5 --steps 5 --warmup 3 --no-cpu-baseline 2>&1 | tail -1 | python -c "import json,sys; d=json.loads(sys.stdin.read()); print(round(d['value']), d['config']['stream_group'], d['config']['grid'], d['roofline']['kernel_ms_per_step'])"; done
