@@ -91,6 +91,28 @@ class ClockSampler:
                 "reasons": sorted(reasons), "samples": len(self.rows)}
 
 
+def ncu_traffic(cfg: str, kernel: str, cycles: int):
+    """dram read+write bytes of one launch of `kernel` from the newest committed
+    `--set full` capture summary (profiles/rNN/ncu_<cfg>_*.json, written by
+    scripts/ncu_summary.py) taken at the same cycles per launch; else None."""
+    import glob
+    scale = {"byte": 1.0, "Kbyte": 1e3, "Mbyte": 1e6, "Gbyte": 1e9}
+    best = None
+    for f in glob.glob(os.path.join(ROOT, "profiles", "r*", f"ncu_{cfg}_*.json")):
+        try:
+            d = json.load(open(f))
+            if d.get("capture_cycles") != cycles or kernel not in d.get("kernel", kernel):
+                continue
+            c, u = d["capture"], d["capture_units"]
+            t = sum(float(c[k]) * scale[u[k]] for k in ("dram__bytes_read.sum", "dram__bytes_write.sum"))
+            m = os.path.getmtime(f)
+            if best is None or m > best[0]:
+                best = (m, t, os.path.relpath(f, ROOT))
+        except Exception:
+            continue
+    return (best[1], best[2]) if best else (None, None)
+
+
 def dist_env():
     ws = int(os.environ.get("WORLD_SIZE", "1"))
     rank = int(os.environ.get("RANK", "0"))
@@ -340,33 +362,47 @@ def main():
         peak_lop3 = n_sms * 64 * float(peaks.get("sm_max_mhz", 1965.0)) * 1e6
         hz_kernel = C / (kern_last / 1e3)
         achieved_lop3 = info.n_and / 16.0 * hz_kernel * S   # this rank's kernel (per GPU)
-        roof = {"bound": "alu", "achieved": achieved_lop3 / 1e12, "peak": peak_lop3 / 1e12, "unit": "TLOP3/s",
-                "frac": achieved_lop3 / peak_lop3, "traffic": None,
-                "kernel": "gem_lane_kernel" if sim.info["lanes"] else "gem_step_kernel", "kernel_ms_per_step": kern_last,
-                "algorithmic": "N_and/16 LOP3 per stream-cycle (2 LOP3 per 32 gate evals, P:81)",
-                "peak_source": f"{n_sms} SMs x 64 LOP3/clk x sm_max_mhz ({peaks['_source']})",
-                "hbm_program_bytes_per_cycle": info.program_bytes,
-                "hbm_frac_if_streamed": info.program_bytes * hz_kernel / (float(peaks.get("hbm_gbs", 6650)) * 1e9),
-                "us_per_layer_critical": 1e6 / hz_kernel / max(1, info.max_layers)}
+        kname = "gem_lane_kernel" if sim.info["lanes"] else "gem_step_kernel"
+        traffic, traffic_src = ncu_traffic(cfg, kname, C)
+        alu = {"bound": "alu", "achieved": achieved_lop3 / 1e12, "peak": peak_lop3 / 1e12, "unit": "TLOP3/s",
+               "frac": achieved_lop3 / peak_lop3,
+               "algorithmic": "N_and/16 LOP3 per stream-cycle (2 LOP3 per 32 gate evals, P:81)",
+               "peak_source": f"{n_sms} SMs x 64 LOP3/clk x sm_max_mhz ({peaks['_source']})"}
+        # algorithmic HBM bytes per stream-cycle: flop state read+write,
+        # RAM ports, PI/PO words; the program is read once per launch when resident
+        alg_bytes = (2 * info.n_flops + info.n_pi + info.n_po) / 8.0 + 12.0 * info.n_rams
+        hbm = {"bound": "hbm", "program_bytes_per_cycle_if_streamed": info.program_bytes,
+               "frac_if_streamed": info.program_bytes * hz_kernel / (float(peaks.get("hbm_gbs", 6650)) * 1e9),
+               "algorithmic_bytes_per_stream_cycle": alg_bytes,
+               "algorithmic_bytes_per_launch": alg_bytes * C * S + info.program_bytes,
+               "peak_gbs": float(peaks.get("hbm_gbs", 6650))}
+        roof = dict(alu)
+        roof.update({"traffic": traffic, "traffic_unit": "bytes per launch (dram read+write, ncu --set full)",
+                     "traffic_source": traffic_src, "kernel": kname, "kernel_ms_per_step": kern_last,
+                     "us_per_layer_critical": 1e6 / hz_kernel / max(1, info.max_layers), "alu": alu, "hbm": hbm})
         if S == 1:
             # single design: the cycle is a chain of dependent layers and grid
-            # barriers, so the binding roofline is latency; floor =
+            # barriers, so the binding roofline is latency (north_star
+            # "or the grid-barrier latency floor, whichever binds"); floor =
             # critical layers x minimal-layer latency + stages x barrier latency,
             # both measured on this GPU by gem_bench_floor
             lay_clk, bar_clk = gem.bench_floor(dev.index, sim.info["grid"])
             crit = sum(info.stage_max_layers())
             f_hz = float(sm_mhz) * 1e6
             floor_hz = f_hz / (crit * lay_clk + info.n_stages * bar_clk)
+            lat = {"bound": "latency", "achieved": hz_kernel, "peak": floor_hz, "unit": "cycles/s",
+                   "frac": hz_kernel / floor_hz,
+                   "layer_clk": lay_clk, "barrier_clk": bar_clk, "critical_layers": crit, "stages": info.n_stages,
+                   "achieved_clk_per_cycle": f_hz / hz_kernel,
+                   "definition": "peak = sm_clock / (sum over stages of the deepest partition's layers x minimal-layer "
+                                 "clocks + stages x grid-barrier clocks); minimal layer = one dependent gathered load "
+                                 "per thread + 13 fold levels + write-out + block barrier (gem_bench_floor, measured "
+                                 "on this GPU in this run)"}
+            roof.update({k: lat[k] for k in ("bound", "achieved", "peak", "unit", "frac")})
             roof["binding"] = "latency"
-            roof["latency_floor"] = {
-                "layer_clk": lay_clk, "barrier_clk": bar_clk, "critical_layers": crit, "stages": info.n_stages,
-                "floor_cycles_per_s": floor_hz, "achieved_cycles_per_s": hz_kernel, "frac": hz_kernel / floor_hz,
-                "achieved_clk_per_cycle": f_hz / hz_kernel,
-                "definition": "floor = sm_clock / (sum over stages of the deepest partition's layers x minimal-layer "
-                              "clocks + stages x grid-barrier clocks); minimal layer = one dependent gathered load "
-                              "per thread + 13 fold levels + write-out + block barrier (gem_bench_floor)"}
+            roof["latency_floor"] = lat
         else:
-            roof["binding"] = "alu/smem throughput (independent streams)"
+            roof["binding"] = "alu (independent streams: issue of LOP3/LDS per lane word)"
         cpu = None
         if ws == 1 and not args.no_cpu_baseline:
             cpu = cpu_baseline(eaig(cfg), info.n_pi, cfg)

@@ -39,8 +39,9 @@ def raw(rep):
 def main():
     lc, rep, prefix = sys.argv[1:4]
     cycles = int(sys.argv[4]) if len(sys.argv) > 4 else None
-    L = launches(lc)
+    L = launches(lc) if lc != "-" else []
     d, units = raw(rep)
+    kname = d.get("Kernel Name", "kernel").split("(")[0]
     keys = ["gpu__time_duration.sum", "dram__bytes_read.sum", "dram__bytes_write.sum", "lts__t_sector_hit_rate.pct",
             "sm__inst_executed.avg.per_cycle_active", "smsp__inst_executed.sum", "launch__grid_size",
             "launch__registers_per_thread", "launch__shared_mem_per_block_dynamic",
@@ -56,15 +57,16 @@ def main():
                           capture_output=True, text=True).stdout
     mn = {k: sass.count(k) for k in ["UBLKCP", "SYNCS.ARRIVE", "SYNCS.PHASECHK", "VOTE.ANY", "SHF.L.W", "LDS.128",
                                      "ATOMG", "UTCHMMA", "HMMA"]}
-    res = {"launch_list": L, "capture": {k: v[0] for k, v in m.items()}, "capture_units": {k: v[1] for k, v in m.items()},
+    res = {"kernel": kname, "launch_list": L, "capture": {k: v[0] for k, v in m.items()}, "capture_units": {k: v[1] for k, v in m.items()},
            "stalls_per_issue": stalls, "sass_mnemonics_in_capture": mn, "capture_cycles": cycles}
     json.dump(res, open(prefix + ".json", "w"), indent=1)
     with open(prefix + ".md", "w") as f:
         f.write("# ncu summary\n\n## Launch list (`--metrics gpu__time_duration.sum --clock-control none`)\n\n")
-        f.write("| kernel | launches | mean | share of GPU time |\n|---|---|---|---|\n")
+        f.write("| kernel | launches | mean | share of GPU time |\n|---|---|---|---|\n" if L else
+                "(no launch list for this capture)\n")
         for x in L:
             f.write(f"| `{x['kernel']}` | {x['launches']} | {x['mean_ns'] / 1e6:.3f} ms | {x['share']:.4f} |\n")
-        f.write("\n## `gem_step_kernel`, one `--set full` capture\n\n| metric | value | unit |\n|---|---|---|\n")
+        f.write(f"\n## `{kname}`, one `--set full` capture\n\n| metric | value | unit |\n|---|---|---|\n")
         for k, (v, u) in m.items():
             f.write(f"| `{k}` | {v} | {u} |\n")
         f.write("\nTop stall reasons (warps stalled per issued instruction):\n\n")
