@@ -125,7 +125,8 @@ int gem_last_step_ms(gem_sim* sim, float* ms);
  * read (after the barrier), 2 layers done, 3 endpoints+RAM committed (first
  * work item), 4 stage-0 items done, 5 after the last grid barrier, 6 = layer
  * count of the first item, 7 program chunk 0 ready, 8 input-port loads stored,
- * 9 layer-0 records loaded (before the barrier); 10-15 unused.
+ * 9 layer-0 records loaded (before the barrier), 10 = partition id of the
+ * last work item; 11-15 unused.
  * Call with dst = NULL to query n_cycles / grid. */
 #define GEM_PROF_SLOTS 16
 int gem_read_profile(gem_sim* sim, uint64_t* dst, uint32_t* n_cycles, uint32_t* grid);

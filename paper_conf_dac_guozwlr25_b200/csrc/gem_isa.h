@@ -126,7 +126,7 @@ enum {
 enum {
   PH_MAGIC = 0, PH_N_GREAD, PH_N_LAYERS, PH_N_OUT, PH_N_RAM, PH_STATE_WORDS, PH_OFF_GREAD,
   PH_OFF_LAYERS, PH_OFF_OUT, PH_OFF_RAM, PH_N_LEAVES, PH_N_NODES, PH_N_OUT_PAD, PH_OFF_CHUNKS,
-  PH_N_CHUNKS, PH_R15, PH_WORDS = 16
+  PH_N_CHUNKS, PH_OFF_DIR0, PH_WORDS = 16
 };
 #define GEM_PART_MAGIC 0x54524150u  /* "PART" */
 
@@ -142,8 +142,23 @@ enum {
  *   [136..) leaves: [n4][32 lanes] x uint4 (4 entries per lane per group)
  * DENSE warps have n4 = 8 and entry j of a lane fills leaf position j.        */
 enum {
-  LH_WORDS_ = 0, LH_FLAGS, LH_TOPC, LH_TOPWO, LH_WOFF0 /* ..LH_WOFF0+7 */, LH_WORDS = 16
+  LH_WORDS_ = 0, LH_FLAGS, LH_TOPC, LH_TOPWO, LH_WOFF0 /* ..LH_WOFF0+7 */, LH_NEXTDIR = 12 /* ..15 */,
+  LH_WORDS = 16
 };
+/* Record directory of a layer: 8 u16 entries (warp w in half w&1 of word w>>1),
+ *   bits [0,13)  warp record offset from the layer start / 4 (words)
+ *   bits [13,16) record class GEM_DC_* (0 = warp inactive)
+ * Layer l's header holds the directory of layer l+1 (LH_NEXTDIR, zeros after
+ * the last layer); layer 0's directory sits in chunk 0 at PH_OFF_DIR0.  A warp
+ * therefore knows where its next record lies before that record's layer is
+ * read, and issues all of its record loads at once (no dependent load chain). */
+#define GEM_DC_SPARSE1 1u
+#define GEM_DC_SPARSE2 2u
+#define GEM_DC_SPARSE4 3u
+#define GEM_DC_SPARSE8 4u
+#define GEM_DC_DENSE16 5u
+#define GEM_DC_DENSE 6u
+#define GEM_DIR_ENTRY(woff, cls) ((((uint32_t)(woff) >> 2) & 0x1FFFu) | ((uint32_t)(cls) << 13))
 #define GEM_LF_USES_TOP 0x100u   /* flags bit 8; bits [0,8) = active warp mask */
 #define GEM_WM_SPARSE 0u
 #define GEM_WM_DENSE 1u     /* 32 u32 entries per lane (n4 = 8)                  */

@@ -22,6 +22,7 @@
 #include <algorithm>
 #include <cstdint>
 #include <cstdio>
+#include <cstdlib>
 #include <cstring>
 #include <string>
 #include <vector>
@@ -67,25 +68,28 @@ struct KParams {
   uint32_t* po_lane;                     // [out_cap][po_words*32][n_groups]
   uint32_t n_groups, ramp_words;
   unsigned long long* fprof;             // debug builds (GEM_FINE_PROF) only
+  uint32_t fine_cta;                     // CTA stamped by GEM_FINE_PROF builds (env GEM_FINE_CTA)
   const uint32_t* __restrict__ wl_off;   // [n_stages][grid+1] CSR offsets into wl_items
   const uint2* __restrict__ wl_items;    // {partition, stream} per work item
 };
 #ifdef GEM_FINE_PROF
-// sub-stamps inside exec_layer: fl = layer index when stamping, >= 8 otherwise;
-// fsub = kp.fprof + 512 ([layer 8][warp 8][4])
+// sub-stamps inside exec_layer: fl = layer index when stamping, >= 32 otherwise;
+// fsub = kp.fprof + 2048 ([layer 32][warp 8][4])
+#define GEM_FINE_LAYERS 32
 #define FSUB(l_, k_)                                                                          \
   do {                                                                                        \
-    if ((l_) < 8 && (threadIdx.x & 31) == 0)                                                  \
+    if ((l_) < GEM_FINE_LAYERS && (threadIdx.x & 31) == 0)                                    \
       fsub[((l_) * 8 + (threadIdx.x >> 5)) * 4 + (k_)] = clock64();                           \
   } while (0)
 #else
 #define FSUB(l_, k_) do { } while (0)
 #endif
 #ifdef GEM_FINE_PROF
-// debug build only: per-warp stamps inside the first 8 layers of cycle 5, CTA 0
+// debug build only: per-warp stamps inside the first 32 layers of cycle 5, CTA kp.fine_cta
 #define FPROF(l_, slot_)                                                                      \
   do {                                                                                        \
-    if (kp.fprof && c == 5 && blockIdx.x == 0 && (l_) < 8 && (threadIdx.x & 31) == 0)        \
+    if (kp.fprof && c == 5 && blockIdx.x == kp.fine_cta && (l_) < GEM_FINE_LAYERS &&         \
+        (threadIdx.x & 31) == 0)                                                              \
       kp.fprof[((l_) * 8 + (threadIdx.x >> 5)) * 8 + (slot_)] = clock64();                    \
   } while (0)
 #else
@@ -383,25 +387,39 @@ __device__ __forceinline__ uint32_t gather_sparse(const uint32_t* S, const uint4
 struct LayerRegs {
   uint4 e[8];
   uint4 lc, wc;
-  uint32_t mode, flags, topc, topwo;
+  uint32_t cls, flags, topc, topwo;
+  uint32_t ndir;   // this warp's entry of the next layer's record directory
 };
 
-__device__ __forceinline__ void load_layer(const uint32_t* L, LayerRegs& R) {
+// uint4 leaf groups per lane of a record class (gem_isa.h GEM_DC_*)
+__device__ __forceinline__ uint32_t dc_n4(uint32_t cls) { return (0x8484210u >> (4u * cls)) & 15u; }
+
+// `dir` = this warp's directory entry for layer L (from the previous layer's
+// header, or chunk 0 for layer 0): the record address is known up front, so
+// every load below is independent and issues back to back.
+__device__ __forceinline__ void load_layer(const uint32_t* L, uint32_t dir, LayerRegs& R) {
   const uint32_t lane = threadIdx.x & 31, warp = threadIdx.x >> 5;
   const uint4 lh0 = *reinterpret_cast<const uint4*>(L);
+  const uint32_t nd = L[LH_NEXTDIR + (warp >> 1)];
   R.flags = lh0.y;
   R.topc = lh0.z;
   R.topwo = lh0.w;
-  if ((R.flags >> warp) & 1u) {
-    const uint32_t* rec = L + L[LH_WOFF0 + warp];
+  R.ndir = (nd >> (16u * (warp & 1u))) & 0xFFFFu;
+  R.cls = dir >> 13;
+  if (R.cls) {
+    const uint32_t* rec = L + 4u * (dir & 0x1FFFu);
     R.wc = *reinterpret_cast<const uint4*>(rec);
-    R.mode = rec[4];
     R.lc = *(reinterpret_cast<const uint4*>(rec + GEM_WREC_HDR) + lane);
     const uint4* lv = reinterpret_cast<const uint4*>(rec + GEM_WREC_HDR + 128) + lane;
-    const uint32_t n4 = R.mode >> 8;
+    const uint32_t n4 = dc_n4(R.cls);
 #pragma unroll
     for (uint32_t g = 0; g < 8; g++) R.e[g] = g < n4 ? lv[g * 32] : make_uint4(0u, 0u, 0u, 0u);
   }
+}
+// directory entry of this warp for layer 0 (chunk 0)
+__device__ __forceinline__ uint32_t dir0_entry(const uint32_t* C0, uint32_t off_dir0) {
+  const uint32_t warp = threadIdx.x >> 5;
+  return (C0[off_dir0 + (warp >> 1)] >> (16u * (warp & 1u))) & 0xFFFFu;
 }
 
 // Rows a3-a5 of one layer with pre-loaded records: gather (bit permutation),
@@ -416,9 +434,9 @@ __device__ __forceinline__ void exec_layer(const LayerRegs& R, uint32_t s_base, 
   const bool uses_top = (R.flags & GEM_LF_USES_TOP) != 0;
   if ((R.flags >> warp) & 1u) {
     uint32_t v = 0;
-    const uint32_t n4 = R.mode >> 8;
+    const uint32_t n4 = dc_n4(R.cls);
 #ifndef EXP_NO_GATHER
-    if ((R.mode & 0xFFu) == GEM_WM_DENSE16) {
+    if (R.cls == GEM_DC_DENSE16) {
       // two 16-bit entries per u32: entry 8g+2k in the low half, 8g+2k+1 in the high half
       uint32_t acc[4] = {0u, 0u, 0u, 0u};
 #pragma unroll
@@ -441,7 +459,7 @@ __device__ __forceinline__ void exec_layer(const LayerRegs& R, uint32_t s_base, 
         }
       }
       v = (acc[0] | acc[1]) | (acc[2] | acc[3]);
-    } else if ((R.mode & 0xFFu) == GEM_WM_DENSE) {
+    } else if (R.cls == GEM_DC_DENSE) {
       // entry j of the lane fills leaf position j: rotate + LOP3 with an immediate mask
 #pragma unroll
       for (uint32_t g = 0; g < 8; g++) {
@@ -615,12 +633,15 @@ __device__ void run_partition(const KParams& kp, ProgSrc& ps, uint32_t* S, uint3
   // first layer's records (independent of S) before the barrier
   LayerRegs R;
   const uint32_t* Lres = C0 + off_layers;
+  const uint32_t* L0 = nullptr;
   if (n_layers) {
     const uint32_t* L;
     if (1 < n_pin) { L = Lres; Lres += ctab[1]; }
     else L = ring_wait(ps);
-    load_layer(L, R);
+    load_layer(L, dir0_entry(C0, h3.w), R);
+    L0 = L;
   }
+  (void)L0;
   PROF(9);
   __syncthreads();   // S ready; chunk 0 and layer 0's chunk consumed
   ps.seq_free = ps.seq_wait;   // records are in registers; waited slots are free
@@ -633,8 +654,8 @@ __device__ void run_partition(const KParams& kp, ProgSrc& ps, uint32_t* S, uint3
   for (uint32_t l = 0; l < n_layers; l++) {
     FPROF(l, 0);
 #ifdef GEM_FINE_PROF
-    const uint32_t fl = (kp.fprof && c == 5 && blockIdx.x == 0) ? l : 99u;
-    unsigned long long* fsub = kp.fprof ? kp.fprof + 512 : nullptr;
+    const uint32_t fl = (kp.fprof && c == 5 && blockIdx.x == kp.fine_cta) ? l : 99u;
+    unsigned long long* fsub = kp.fprof ? kp.fprof + GEM_FINE_LAYERS * 64 : nullptr;
 #else
     const uint32_t fl = 99u;
     unsigned long long* fsub = nullptr;
@@ -647,15 +668,25 @@ __device__ void run_partition(const KParams& kp, ProgSrc& ps, uint32_t* S, uint3
     FPROF(l, 1);
     const bool ptop = (R.flags & GEM_LF_USES_TOP) != 0;
     const uint32_t ptopc = R.topc, ptopwo = R.topwo;
+#if defined(EXP_NO_WAIT)   // timing experiment: every layer reuses layer 0's records (no wait, no load)
+    if (false) {
+#elif defined(EXP_SAME_L)  // timing experiment: reload layer 0's records (load chain, no chunk wait)
     if (l + 1 < n_layers) {
+      load_layer(L0, dir0_entry(C0, h3.w), R);
+    }
+    if (false) {
+#else
+    if (l + 1 < n_layers) {
+#endif
       const uint32_t* L;
       if (2 + l < n_pin) { L = Lres; Lres += ctab[2 + l]; }
       else L = ring_wait(ps);
       FPROF(l, 2);
+      const uint32_t nd = R.ndir;
 #ifndef EXP_NO_LOAD
-      load_layer(L, R);
+      load_layer(L, nd, R);
 #else
-      if (l == 0) load_layer(L, R);
+      if (l == 0) load_layer(L, nd, R);
 #endif
     }
     FPROF(l, 3);
@@ -709,7 +740,10 @@ __device__ void run_partition(const KParams& kp, ProgSrc& ps, uint32_t* S, uint3
   __syncthreads();  // S / ramp / ring slots reused by the next work item
   ps.seq_free = ps.seq_issue;   // every chunk of this item consumed
   PROF(3);
-  if (prof_on && tid == 0) kp.prof[((size_t)c * gridDim.x + blockIdx.x) * GEM_PROF_SLOTS + 6] = n_layers;
+  if (prof_on && tid == 0) {
+    kp.prof[((size_t)c * gridDim.x + blockIdx.x) * GEM_PROF_SLOTS + 6] = n_layers;
+    kp.prof[((size_t)c * gridDim.x + blockIdx.x) * GEM_PROF_SLOTS + 10] = p;
+  }
 }
 
 // Parity instruments: trace / digest of Q(t+1) in external (AIGER) order.
@@ -1560,7 +1594,7 @@ int gem_step(gem_sim* sim, uint64_t ncycles) {
       sim->d_prof = nullptr;
       CK(dalloc(&sim->d_prof, (size_t)256 * sim->grid * GEM_PROF_SLOTS * 8));
 #ifdef GEM_FINE_PROF
-      CK(dalloc(&sim->d_fprof, 8 * 8 * 8 * 8 + 8 * 8 * 4 * 8));
+      CK(dalloc(&sim->d_fprof, GEM_FINE_LAYERS * 96 * 8));
 #endif
     }
     sim->prof_cycles = pc;
@@ -1568,6 +1602,7 @@ int gem_step(gem_sim* sim, uint64_t ncycles) {
     kp.prof = sim->d_prof;
     kp.prof_cycles = pc;
     kp.fprof = sim->d_fprof;
+    kp.fine_cta = getenv("GEM_FINE_CTA") ? (uint32_t)atoi(getenv("GEM_FINE_CTA")) : 0u;
   }
   CK(cudaMemsetAsync(sim->d_bar, 0, (size_t)(GEM_BAR_MAX_CTAS + 2) * GEM_BAR_STRIDE * 8, sim->stream));
   if (sim->flags & GEM_F_DIGEST)
@@ -1774,7 +1809,7 @@ int gem_write_ram(gem_sim* sim, uint32_t ram_id, uint32_t stream, const uint32_t
 #ifdef GEM_FINE_PROF
 int gem_read_fine(gem_sim* sim, uint64_t* dst) {
   CK(cudaStreamSynchronize(sim->stream));
-  CK(cudaMemcpy(dst, sim->d_fprof, 8 * 8 * 8 * 8 + 8 * 8 * 4 * 8, cudaMemcpyDeviceToHost));
+  CK(cudaMemcpy(dst, sim->d_fprof, GEM_FINE_LAYERS * 96 * 8, cudaMemcpyDeviceToHost));
   return GEM_OK;
 }
 #endif

@@ -64,6 +64,7 @@ struct Options {
   double refine_ratio = 1.35;  // split partitions costing more than this x the median
   int max_parts = 280;      // refinement stops growing the partition count here
   int lanes = 0;            // also emit stream-sliced lane programs (batched streams)
+  int banks = 1;            // bank-conflict-aware renaming of the state words (rename_state_words)
   int verbose = 0;
   int max_state_words = GEM_MAX_STATE_WORDS;
   double cap_slack = 1.0;
@@ -93,6 +94,7 @@ static Options parse_opts(const char* s) {
     else if (k == "refine_ratio") o.refine_ratio = std::stod(v);
     else if (k == "max_parts") o.max_parts = std::stoi(v);
     else if (k == "lanes") o.lanes = std::stoi(v);
+    else if (k == "banks") o.banks = std::stoi(v);
     else throw std::runtime_error("unknown option " + k);
   }
   if (o.stages < 1 || o.stages > 2) throw std::runtime_error("stages must be 1 or 2");
@@ -831,6 +833,36 @@ struct Mapper {
         off += prog_layers[off + LH_WORDS_];
       }
     }
+    // record directories (gem_isa.h): layer l+1's into layer l's header, layer 0's into chunk 0
+    {
+      std::vector<std::array<uint32_t, 4>> dirs(n_layers);
+      size_t off = 0;
+      for (uint32_t l = 0; l < n_layers; l++) {
+        std::array<uint32_t, 4> d{0, 0, 0, 0};
+        for (uint32_t w = 0; w < 8; w++) {
+          const uint32_t wo = prog_layers[off + LH_WOFF0 + w];
+          if (!wo) continue;
+          const uint32_t mw = prog_layers[off + wo + 4], mode = mw & 0xFFu, n4 = mw >> 8;
+          const uint32_t cls = mode == GEM_WM_DENSE16 ? GEM_DC_DENSE16 : mode == GEM_WM_DENSE ? GEM_DC_DENSE
+                               : n4 <= 1 ? GEM_DC_SPARSE1 : n4 <= 2 ? GEM_DC_SPARSE2 : n4 <= 4 ? GEM_DC_SPARSE4
+                               : GEM_DC_SPARSE8;
+          if (wo % 4 || wo >= (1u << 15)) throw std::runtime_error("warp record offset not encodable");
+          d[w >> 1] |= GEM_DIR_ENTRY(wo, cls) << (16 * (w & 1));
+        }
+        dirs[l] = d;
+        off += prog_layers[off + LH_WORDS_];
+      }
+      off = 0;
+      for (uint32_t l = 0; l + 1 < n_layers; l++) {
+        for (int k = 0; k < 4; k++) prog_layers[off + LH_NEXTDIR + k] = dirs[l + 1][k];
+        off += prog_layers[off + LH_WORDS_];
+      }
+      // chunk 0: the layer-0 directory right before the layer records (after the gread list)
+      pr[PH_OFF_DIR0] = (uint32_t)pr.size();
+      for (int k = 0; k < 4; k++) pr.push_back(n_layers ? dirs[0][k] : 0u);
+      pr[PH_OFF_LAYERS] = (uint32_t)pr.size();
+      pr[pr[PH_OFF_CHUNKS]] = (uint32_t)pr.size();
+    }
     pr.insert(pr.end(), prog_layers.begin(), prog_layers.end());
     pr[PH_OFF_OUT] = (uint32_t)pr.size();
     uint32_t n_out = (uint32_t)P.outs.size(), n_out_pad = (n_out + 3) & ~3u;
@@ -847,6 +879,7 @@ struct Mapper {
     while (pr.size() % 4) pr.push_back(0);
     pr[pr[PH_OFF_CHUNKS] + 1 + n_layers] = (uint32_t)pr.size() - pr[PH_OFF_OUT];
     pr[PH_STATE_WORDS] = max_state;
+    if (opt.banks) max_state = rename_state_words(pr, (uint32_t)opt.max_state_words);
     pr[PH_N_LEAVES] = total_leaves;
     pr[PH_N_NODES] = n_and;
     P.n_layers = n_layers;
@@ -856,6 +889,201 @@ struct Mapper {
     P.slots_used = slots_used;
     if (opt.lanes && !encode_lanes(P, lane_layers, gread_src, scratch)) return;
     P.ok = true;
+  }
+
+  // Bank-conflict-aware bit placement (the paper's placement minimises shared-
+  // memory bank conflicts of the permutation).  A
+  // state word w lives in bank w mod 32, and one gather LDS (entry j of the 32
+  // lanes of a warp) costs as many shared-memory wavefronts as the most
+  // crowded bank holds distinct words.  The mapper allocated words by
+  // liveness only; this pass renames them with a bijection on [1, M)
+  // (M = min(state words, 2048) rounded up to a bank row, so DENSE16 entries
+  // stay valid; word 0, the constant, and words >= 2048 keep their index),
+  // chosen greedily so that words read together fall into different banks.
+  // Renaming a physical word for the whole program is always legal: every
+  // read and write of it moves together.  Returns the new state word count.
+  static uint32_t rename_state_words(std::vector<uint32_t>& pr, uint32_t max_words) {
+    const uint32_t N = pr[PH_STATE_WORDS];
+    const uint32_t M = std::min<uint32_t>(N, 2048u);
+    // two spare rows per bank give the local search room to move words
+    const uint32_t Mp = N <= 2048u ? std::min<uint32_t>({2048u, max_words, ((M + 31u) & ~31u) + 64u}) : 2048u;
+    if (M <= 2) return N;
+    // ---- access groups (one per warp-wide shared-memory instruction)
+    std::vector<std::vector<uint16_t>> groups;
+    std::vector<uint16_t> g;
+    auto close = [&]() {
+      std::sort(g.begin(), g.end());
+      g.erase(std::unique(g.begin(), g.end()), g.end());
+      if (g.size() > 1) groups.push_back(g);
+      g.clear();
+    };
+    auto add = [&](uint32_t w) { g.push_back((uint16_t)(w < M ? w : 0xFFFFu)); };  // >= M: fixed word
+    const uint32_t n_layers = pr[PH_N_LAYERS];
+    const uint32_t* ct = pr.data() + pr[PH_OFF_CHUNKS];
+    uint32_t L = pr[PH_OFF_LAYERS];
+    for (uint32_t l = 0; l < n_layers; l++) {
+      for (uint32_t w = 0; w < 8; w++) {
+        const uint32_t wo = pr[L + LH_WOFF0 + w];
+        if (!wo) continue;
+        const uint32_t rec = L + wo, mode = pr[rec + 4] & 0xFFu, n4 = pr[rec + 4] >> 8;
+        const uint32_t lv = rec + GEM_WREC_HDR + 128;
+        for (uint32_t gg = 0; gg < n4; gg++)
+          for (uint32_t c = 0; c < 4; c++) {
+            if (mode == GEM_WM_DENSE16) {
+              for (uint32_t h = 0; h < 2; h++) {
+                for (uint32_t ln = 0; ln < 32; ln++) add(GEM_LEAF16_WORD(pr[lv + (gg * 32 + ln) * 4 + c] >> (16 * h)));
+                close();
+              }
+            } else {
+              for (uint32_t ln = 0; ln < 32; ln++) add(GEM_LEAF_WORD(pr[lv + (gg * 32 + ln) * 4 + c]));
+              close();
+            }
+          }
+        // thread write-outs (one STS per lane)
+        for (uint32_t ln = 0; ln < 32; ln++) {
+          const uint32_t x = pr[rec + GEM_WREC_HDR + 4 * ln + 3];
+          if (x) add(x);
+        }
+        close();
+      }
+      L += ct[1 + l];
+    }
+    // input ports (32 consecutive entries per STS) and endpoint gathers
+    const uint32_t ng = pr[PH_N_GREAD], og = pr[PH_OFF_GREAD];
+    for (uint32_t k = 0; k < ng; k++) {
+      add(pr[og + 2 * k + 1]);
+      if (k % 32 == 31 || k + 1 == ng) close();
+    }
+    const uint32_t no = pr[PH_N_OUT], oo = pr[PH_OFF_OUT] + pr[PH_N_OUT_PAD];
+    for (uint32_t o = 0; o < no; o++) {
+      for (uint32_t k = 0; k < 32; k++) add((pr[oo + o * 32 + k] & 0x7FFFFFFFu) >> 5);
+      close();
+    }
+    // ---- greedy bank assignment, busiest words first
+    const uint32_t G = (uint32_t)groups.size();
+    std::vector<std::vector<uint32_t>> of(M);   // groups of each word
+    for (uint32_t k = 0; k < G; k++)
+      for (uint16_t w : groups[k])
+        if (w != 0xFFFFu) of[w].push_back(k);
+    std::vector<uint8_t> cnt((size_t)G * 32, 0), mx(G, 0);
+    // word 0 (the constant) is fixed in bank 0; fixed words >= M are ignored
+    for (uint32_t k = 0; k < G; k++)
+      for (uint16_t w : groups[k])
+        if (w == 0) { cnt[(size_t)k * 32] = 1; mx[k] = 1; }
+    std::vector<uint32_t> cap(32, 0);
+    for (uint32_t p = 1; p < Mp; p++) cap[p & 31]++;
+    std::vector<uint32_t> order;
+    for (uint32_t w = 1; w < M; w++) order.push_back(w);
+    std::stable_sort(order.begin(), order.end(), [&](uint32_t a, uint32_t b) { return of[a].size() > of[b].size(); });
+    std::vector<int32_t> bank(M, -1);
+    bank[0] = 0;
+    std::vector<uint32_t> used(32, 0);
+    for (uint32_t w : order) {
+      int best = -1;
+      uint64_t best_key = UINT64_MAX;
+      for (uint32_t b = 0; b < 32; b++) {
+        if (used[b] >= cap[b]) continue;
+        uint32_t delta = 0, load = 0;
+        for (uint32_t k : of[w]) {
+          const uint32_t c = cnt[(size_t)k * 32 + b];
+          if (c + 1u > mx[k]) delta++;
+          load += c;
+        }
+        const uint64_t key = ((uint64_t)delta << 40) | ((uint64_t)load << 16) | used[b];
+        if (key < best_key) { best_key = key; best = (int)b; }
+      }
+      bank[w] = best;
+      used[best]++;
+      for (uint32_t k : of[w]) {
+        uint8_t& c = cnt[(size_t)k * 32 + best];
+        c++;
+        mx[k] = std::max(mx[k], c);
+      }
+    }
+    // ---- local search: move a word to the bank that lowers the wavefront count
+    auto regroup_max = [&](uint32_t k) {
+      uint8_t m = 0;
+      for (uint32_t b = 0; b < 32; b++) m = std::max(m, cnt[(size_t)k * 32 + b]);
+      mx[k] = m;
+    };
+    for (int pass = 0; pass < 4; pass++) {
+      uint32_t moved = 0;
+      for (uint32_t w : order) {
+        const uint32_t a = (uint32_t)bank[w];
+        if (of[w].empty()) continue;
+        for (uint32_t k : of[w]) { cnt[(size_t)k * 32 + a]--; regroup_max(k); }
+        // cost of w's groups with w in bank b = sum of maxima + #groups where b becomes the max
+        auto cost_in = [&](uint32_t b) {
+          int32_t c = 0;
+          for (uint32_t k : of[w]) c += mx[k] + ((cnt[(size_t)k * 32 + b] + 1u > mx[k]) ? 1 : 0);
+          return c;
+        };
+        int best = (int)a;
+        int32_t best_cost = cost_in(a);
+        for (uint32_t b = 0; b < 32; b++) {
+          if (b == a || used[b] >= cap[b]) continue;
+          const int32_t c = cost_in(b);
+          if (c < best_cost) { best_cost = c; best = (int)b; }
+        }
+        for (uint32_t k : of[w]) {
+          uint8_t& c = cnt[(size_t)k * 32 + best];
+          c++;
+          mx[k] = std::max(mx[k], c);
+        }
+        if ((uint32_t)best != a) { used[a]--; used[best]++; bank[w] = best; moved++; }
+      }
+      if (!moved) break;
+    }
+    // ---- physical words: bank b's logical words take the free rows of bank b in order
+    std::vector<uint32_t> next_row(32, 0);
+    for (uint32_t b = 0; b < 32; b++) next_row[b] = b == 0 ? 1u : 0u;
+    std::vector<uint32_t> phys(M, 0);
+    uint32_t hi = 0;
+    for (uint32_t w = 1; w < M; w++) {
+      const uint32_t b = (uint32_t)bank[w];
+      phys[w] = next_row[b]++ * 32 + b;
+      hi = std::max(hi, phys[w]);
+    }
+    auto R = [&](uint32_t w) -> uint32_t { return w < M ? phys[w] : w; };
+    // ---- rewrite every word reference
+    L = pr[PH_OFF_LAYERS];
+    for (uint32_t l = 0; l < n_layers; l++) {
+      if (pr[L + LH_FLAGS] & GEM_LF_USES_TOP) pr[L + LH_TOPWO] = R(pr[L + LH_TOPWO]);
+      for (uint32_t w = 0; w < 8; w++) {
+        const uint32_t wo = pr[L + LH_WOFF0 + w];
+        if (!wo) continue;
+        const uint32_t rec = L + wo, mode = pr[rec + 4] & 0xFFu, n4 = pr[rec + 4] >> 8;
+        if (pr[rec + 3]) pr[rec + 3] = R(pr[rec + 3]);
+        for (uint32_t ln = 0; ln < 32; ln++) {
+          uint32_t& x = pr[rec + GEM_WREC_HDR + 4 * ln + 3];
+          if (x) x = R(x);
+        }
+        const uint32_t lv = rec + GEM_WREC_HDR + 128;
+        for (uint32_t k = 0; k < n4 * 128; k++) {
+          uint32_t& e = pr[lv + k];
+          if (mode == GEM_WM_DENSE16) {
+            uint32_t out = 0;
+            for (uint32_t h = 0; h < 2; h++) {
+              const uint32_t x = (e >> (16 * h)) & 0xFFFFu;
+              out |= ((x & 31u) | (R(GEM_LEAF16_WORD(x)) << 5)) << (16 * h);
+            }
+            e = out;
+          } else {
+            e = (e & ~(0x1FFFu << 7)) | (R(GEM_LEAF_WORD(e)) << 7);
+          }
+        }
+      }
+      L += ct[1 + l];
+    }
+    for (uint32_t k = 0; k < ng; k++) pr[og + 2 * k + 1] = R(pr[og + 2 * k + 1]);
+    for (uint32_t k = 0; k < no * 32; k++) {
+      uint32_t& e = pr[oo + k];
+      const uint32_t src = e & 0x7FFFFFFFu;
+      e = (e & GEM_OUT_INV) | (R(src >> 5) << 5) | (src & 31u);
+    }
+    const uint32_t NS = std::max(N, hi + 1);
+    pr[PH_STATE_WORDS] = NS;
+    return NS;
   }
 
   // Lane program (gem_isa.h "Lane mode"): allocate one lane word per live signal
@@ -1081,7 +1309,10 @@ struct Mapper {
       for (uint32_t l = 0; l < 32; l++)
         for (auto& x : leaves[w * 32 + l]) small_words = small_words && (x.first >> 5) < 2048;
       const bool d16 = dense && small_words;
-      const uint32_t n4 = d16 ? 4u : dense ? 8u : (niter[w] + 3) / 4;
+      // sparse records are padded to n4 in {1, 2, 4, 8} (the directory class fixes n4)
+      uint32_t n4s = 1;
+      while (n4s * 4 < niter[w]) n4s *= 2;
+      const uint32_t n4 = d16 ? 4u : dense ? 8u : n4s;
       out.push_back(pack(6, 10, w, sxa));
       out.push_back(pack(6, 10, w, sxb));
       out.push_back(pack(6, 10, w, sob));
