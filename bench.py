@@ -398,9 +398,20 @@ def main():
                                  "clocks + stages x grid-barrier clocks); minimal layer = one dependent gathered load "
                                  "per thread + 13 fold levels + write-out + block barrier (gem_bench_floor, measured "
                                  "on this GPU in this run)"}
-            roof.update({k: lat[k] for k in ("bound", "achieved", "peak", "unit", "frac")})
-            roof["binding"] = "latency"
             roof["latency_floor"] = lat
+            # a program larger than L2 streams from HBM every cycle: that ceiling may bind first
+            l2_bytes = 126e6
+            hbm_floor = (float(peaks.get("hbm_gbs", 6650)) * 1e9 / info.program_bytes
+                         if info.program_bytes > l2_bytes else float("inf"))
+            hbm["floor_cycles_per_s"] = hbm_floor if hbm_floor != float("inf") else None
+            if hbm_floor < floor_hz:
+                roof.update({"bound": "hbm", "achieved": info.program_bytes * hz_kernel / 1e9,
+                             "peak": float(peaks.get("hbm_gbs", 6650)), "unit": "GB/s",
+                             "frac": hz_kernel / hbm_floor})
+                roof["binding"] = "hbm (program > L2, streamed every cycle)"
+            else:
+                roof.update({k: lat[k] for k in ("bound", "achieved", "peak", "unit", "frac")})
+                roof["binding"] = "latency"
         else:
             roof["binding"] = "alu (independent streams: issue of LOP3/LDS per lane word)"
         cpu = None

@@ -71,19 +71,22 @@
 
 /* leaf entry (gather of one state bit b of word w into leaf position p):
  *   bits [0,5)   rot = (p - b) mod 32   -> rotl(S[w], rot) puts bit b at p
- *   bits [5,20)  byte offset of S[w] (w*4; S sits at shared-memory offset 0)
- *   bits [24,29) p (SPARSE warps only; DENSE warps use entry index = p)
+ *                (a funnel shift uses the low 5 bits of the entry directly)
+ *   bits [8,13)  p (SPARSE warps only; DENSE warps use entry index = p):
+ *                rotl(1, entry >> 8) is the position mask
+ *   bits [16,32) byte offset of S[w] (w*4; S sits at shared-memory offset 0),
+ *                so the load address is entry >> 16
  * Padding entries are 0: they read S[0] == 0.                                  */
 #define GEM_LEAF(word, bit, pos) \
-  ((((uint32_t)(pos) - (uint32_t)(bit)) & 31u) | ((uint32_t)(word) << 7) | ((uint32_t)(pos) << 24))
-#define GEM_LEAF_DENSE(word, bit, pos) ((((uint32_t)(pos) - (uint32_t)(bit)) & 31u) | ((uint32_t)(word) << 7))
-#define GEM_LEAF_WORD(e) (((e) >> 7) & 0x1FFFu)
+  ((((uint32_t)(pos) - (uint32_t)(bit)) & 31u) | ((uint32_t)(pos) << 8) | ((uint32_t)(word) << 18))
+#define GEM_LEAF_DENSE(word, bit, pos) ((((uint32_t)(pos) - (uint32_t)(bit)) & 31u) | ((uint32_t)(word) << 18))
+#define GEM_LEAF_WORD(e) ((uint32_t)(e) >> 18)
 /* 16-bit dense entry (DENSE16 warps, state words < 2048): rot | word << 5;
  * u32 k of a lane's group g holds entries 8g+2k (low half) and 8g+2k+1 (high). */
 #define GEM_LEAF16(word, bit, pos) ((((uint32_t)(pos) - (uint32_t)(bit)) & 31u) | ((uint32_t)(word) << 5))
 #define GEM_LEAF16_WORD(h) (((h) >> 5) & 0x7FFu)
 #define GEM_LEAF_ROT(e) ((e) & 31u)
-#define GEM_LEAF_POS(e) (((e) >> 24) & 31u)
+#define GEM_LEAF_POS(e) (((e) >> 8) & 31u)
 
 /* packed slot-word bit offsets for levels 1..5 of a group */
 #define GEM_OFF_L1 0
@@ -146,19 +149,16 @@ enum {
   LH_WORDS = 16
 };
 /* Record directory of a layer: 8 u16 entries (warp w in half w&1 of word w>>1),
- *   bits [0,13)  warp record offset from the layer start / 4 (words)
- *   bits [13,16) record class GEM_DC_* (0 = warp inactive)
+ *   bits [0,12)  warp record offset from the layer start / 4 (words)
+ *   bits [12,16) record class GEM_DC_* (0 = warp inactive; SPARSE n4 = class)
  * Layer l's header holds the directory of layer l+1 (LH_NEXTDIR, zeros after
  * the last layer); layer 0's directory sits in chunk 0 at PH_OFF_DIR0.  A warp
  * therefore knows where its next record lies before that record's layer is
  * read, and issues all of its record loads at once (no dependent load chain). */
-#define GEM_DC_SPARSE1 1u
-#define GEM_DC_SPARSE2 2u
-#define GEM_DC_SPARSE4 3u
-#define GEM_DC_SPARSE8 4u
-#define GEM_DC_DENSE16 5u
-#define GEM_DC_DENSE 6u
-#define GEM_DIR_ENTRY(woff, cls) ((((uint32_t)(woff) >> 2) & 0x1FFFu) | ((uint32_t)(cls) << 13))
+/* classes 1..8: SPARSE with n4 = class */
+#define GEM_DC_DENSE16 9u
+#define GEM_DC_DENSE 10u
+#define GEM_DIR_ENTRY(woff, cls) ((((uint32_t)(woff) >> 2) & 0xFFFu) | ((uint32_t)(cls) << 12))
 #define GEM_LF_USES_TOP 0x100u   /* flags bit 8; bits [0,8) = active warp mask */
 #define GEM_WM_SPARSE 0u
 #define GEM_WM_DENSE 1u     /* 32 u32 entries per lane (n4 = 8)                  */

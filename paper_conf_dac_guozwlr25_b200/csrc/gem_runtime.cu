@@ -363,21 +363,24 @@ __device__ __forceinline__ uint32_t ldst(const uint32_t* S, uint32_t byteoff) {
   }
   return ldsb(S, byteoff);
 }
+// load address = entry >> 16 (byte offset), rotation = low 5 bits (gem_isa.h)
 template <bool kS0 = false>
-__device__ __forceinline__ uint32_t leaf_rot(const uint32_t* S, uint32_t e, uint32_t byte_mask) {
-  const uint32_t s = ldst<kS0>(S, (e >> 5) & byte_mask);
+__device__ __forceinline__ uint32_t leaf_rot(const uint32_t* S, uint32_t e) {
+  const uint32_t s = ldst<kS0>(S, e >> 16);
   return __funnelshift_l(s, s, e);   // rotl(s, e & 31)
 }
+// SPARSE entry: position mask rotl(1, e >> 8) (low 5 bits = leaf position)
+__device__ __forceinline__ uint32_t leaf_mask(uint32_t e) { return __funnelshift_l(1u, 1u, e >> 8); }
 template <int N4, bool kS0>
 __device__ __forceinline__ uint32_t gather_sparse(const uint32_t* S, const uint4* e) {
   // four independent accumulators keep the OR chain short
   uint32_t v0 = 0, v1 = 0, v2 = 0, v3 = 0;
 #pragma unroll
   for (int g = 0; g < N4; g++) {
-    v0 |= leaf_rot<kS0>(S, e[g].x, 0x7FFFu) & (1u << GEM_LEAF_POS(e[g].x));
-    v1 |= leaf_rot<kS0>(S, e[g].y, 0x7FFFu) & (1u << GEM_LEAF_POS(e[g].y));
-    v2 |= leaf_rot<kS0>(S, e[g].z, 0x7FFFu) & (1u << GEM_LEAF_POS(e[g].z));
-    v3 |= leaf_rot<kS0>(S, e[g].w, 0x7FFFu) & (1u << GEM_LEAF_POS(e[g].w));
+    v0 |= leaf_rot<kS0>(S, e[g].x) & leaf_mask(e[g].x);
+    v1 |= leaf_rot<kS0>(S, e[g].y) & leaf_mask(e[g].y);
+    v2 |= leaf_rot<kS0>(S, e[g].z) & leaf_mask(e[g].z);
+    v3 |= leaf_rot<kS0>(S, e[g].w) & leaf_mask(e[g].w);
   }
   return (v0 | v1) | (v2 | v3);
 }
@@ -392,7 +395,9 @@ struct LayerRegs {
 };
 
 // uint4 leaf groups per lane of a record class (gem_isa.h GEM_DC_*)
-__device__ __forceinline__ uint32_t dc_n4(uint32_t cls) { return (0x8484210u >> (4u * cls)) & 15u; }
+__device__ __forceinline__ uint32_t dc_n4(uint32_t cls) {
+  return cls <= 8u ? cls : (cls == GEM_DC_DENSE16 ? 4u : 8u);
+}
 
 // `dir` = this warp's directory entry for layer L (from the previous layer's
 // header, or chunk 0 for layer 0): the record address is known up front, so
@@ -405,9 +410,9 @@ __device__ __forceinline__ void load_layer(const uint32_t* L, uint32_t dir, Laye
   R.topc = lh0.z;
   R.topwo = lh0.w;
   R.ndir = (nd >> (16u * (warp & 1u))) & 0xFFFFu;
-  R.cls = dir >> 13;
+  R.cls = dir >> 12;
   if (R.cls) {
-    const uint32_t* rec = L + 4u * (dir & 0x1FFFu);
+    const uint32_t* rec = L + 4u * (dir & 0xFFFu);
     R.wc = *reinterpret_cast<const uint4*>(rec);
     R.lc = *(reinterpret_cast<const uint4*>(rec + GEM_WREC_HDR) + lane);
     const uint4* lv = reinterpret_cast<const uint4*>(rec + GEM_WREC_HDR + 128) + lane;
@@ -463,19 +468,22 @@ __device__ __forceinline__ void exec_layer(const LayerRegs& R, uint32_t s_base, 
       // entry j of the lane fills leaf position j: rotate + LOP3 with an immediate mask
 #pragma unroll
       for (uint32_t g = 0; g < 8; g++) {
-        v |= leaf_rot<kS0>(Sj, R.e[g].x, 0xFFFFFFFFu) & (1u << (4 * g + 0));
-        v |= leaf_rot<kS0>(Sj, R.e[g].y, 0xFFFFFFFFu) & (1u << (4 * g + 1));
-        v |= leaf_rot<kS0>(Sj, R.e[g].z, 0xFFFFFFFFu) & (1u << (4 * g + 2));
-        v |= leaf_rot<kS0>(Sj, R.e[g].w, 0xFFFFFFFFu) & (1u << (4 * g + 3));
+        v |= leaf_rot<kS0>(Sj, R.e[g].x) & (1u << (4 * g + 0));
+        v |= leaf_rot<kS0>(Sj, R.e[g].y) & (1u << (4 * g + 1));
+        v |= leaf_rot<kS0>(Sj, R.e[g].z) & (1u << (4 * g + 2));
+        v |= leaf_rot<kS0>(Sj, R.e[g].w) & (1u << (4 * g + 3));
       }
-    } else if (n4 <= 1) {
-      v = gather_sparse<1, kS0>(Sj, R.e);
-    } else if (n4 <= 2) {
-      v = gather_sparse<2, kS0>(Sj, R.e);
-    } else if (n4 <= 4) {
-      v = gather_sparse<4, kS0>(Sj, R.e);
     } else {
-      v = gather_sparse<8, kS0>(Sj, R.e);
+      switch (n4) {
+        case 1: v = gather_sparse<1, kS0>(Sj, R.e); break;
+        case 2: v = gather_sparse<2, kS0>(Sj, R.e); break;
+        case 3: v = gather_sparse<3, kS0>(Sj, R.e); break;
+        case 4: v = gather_sparse<4, kS0>(Sj, R.e); break;
+        case 5: v = gather_sparse<5, kS0>(Sj, R.e); break;
+        case 6: v = gather_sparse<6, kS0>(Sj, R.e); break;
+        case 7: v = gather_sparse<7, kS0>(Sj, R.e); break;
+        default: v = gather_sparse<8, kS0>(Sj, R.e); break;
+      }
     }
 #else   // timing experiment only (wrong results)
     v = R.e[0].x ^ R.e[1].y ^ R.lc.w;

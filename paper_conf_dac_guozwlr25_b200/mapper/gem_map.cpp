@@ -844,9 +844,10 @@ struct Mapper {
           if (!wo) continue;
           const uint32_t mw = prog_layers[off + wo + 4], mode = mw & 0xFFu, n4 = mw >> 8;
           const uint32_t cls = mode == GEM_WM_DENSE16 ? GEM_DC_DENSE16 : mode == GEM_WM_DENSE ? GEM_DC_DENSE
-                               : n4 <= 1 ? GEM_DC_SPARSE1 : n4 <= 2 ? GEM_DC_SPARSE2 : n4 <= 4 ? GEM_DC_SPARSE4
-                               : GEM_DC_SPARSE8;
-          if (wo % 4 || wo >= (1u << 15)) throw std::runtime_error("warp record offset not encodable");
+                               : std::max<uint32_t>(1u, n4);
+          if (cls > GEM_DC_DENSE || (mode == GEM_WM_SPARSE && n4 > 8))
+            throw std::runtime_error("warp record class not encodable");
+          if (wo % 4 || wo >= (1u << 14)) throw std::runtime_error("warp record offset not encodable");
           d[w >> 1] |= GEM_DIR_ENTRY(wo, cls) << (16 * (w & 1));
         }
         dirs[l] = d;
@@ -1069,7 +1070,7 @@ struct Mapper {
             }
             e = out;
           } else {
-            e = (e & ~(0x1FFFu << 7)) | (R(GEM_LEAF_WORD(e)) << 7);
+            e = (e & 0xFFFFu) | (R(GEM_LEAF_WORD(e)) << 18);
           }
         }
       }
@@ -1309,10 +1310,7 @@ struct Mapper {
       for (uint32_t l = 0; l < 32; l++)
         for (auto& x : leaves[w * 32 + l]) small_words = small_words && (x.first >> 5) < 2048;
       const bool d16 = dense && small_words;
-      // sparse records are padded to n4 in {1, 2, 4, 8} (the directory class fixes n4)
-      uint32_t n4s = 1;
-      while (n4s * 4 < niter[w]) n4s *= 2;
-      const uint32_t n4 = d16 ? 4u : dense ? 8u : n4s;
+      const uint32_t n4 = d16 ? 4u : dense ? 8u : std::max<uint32_t>(1u, (niter[w] + 3) / 4);
       out.push_back(pack(6, 10, w, sxa));
       out.push_back(pack(6, 10, w, sxb));
       out.push_back(pack(6, 10, w, sob));

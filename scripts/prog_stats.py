@@ -43,7 +43,7 @@ def layer_lds(w, L):
         else:
             for g in range(n4):
                 for k in range(4):
-                    words = (lv[g, :, k] >> 7) & 0x1FFF
+                    words = lv[g, :, k] >> 18
                     n_lds += 1
                     wf += wavefronts(words)
                     leaves += int((lv[g, :, k] != 0).sum())

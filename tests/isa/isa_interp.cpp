@@ -62,6 +62,10 @@ int run_part(Interp& I, uint32_t p, uint64_t t, const uint32_t* stim, uint32_t* 
   const uint32_t* L = pr + pr[PH_OFF_LAYERS];
   std::vector<uint8_t> val[14];
   for (int k = 0; k <= 13; k++) val[k].assign(8192u >> k, 0);
+  // record directory of the current layer (gem_isa.h): chunk 0 for layer 0,
+  // then the previous layer's LH_NEXTDIR words -- read the way the kernel does
+  uint32_t dir[4];
+  for (int k = 0; k < 4; k++) dir[k] = pr[pr[PH_OFF_DIR0] + k];
   for (uint32_t l = 0; l < pr[PH_N_LAYERS]; l++) {
     uint32_t flags = L[LH_FLAGS];
     uint32_t topc = L[LH_TOPC];
@@ -72,9 +76,14 @@ int run_part(Interp& I, uint32_t p, uint64_t t, const uint32_t* stim, uint32_t* 
     for (int k = 0; k <= 13; k++) std::fill(val[k].begin(), val[k].end(), 0);
     std::vector<uint8_t> read(GEM_MAX_STATE_WORDS, 0);
     for (uint32_t wp = 0; wp < 8; wp++) {
+      const uint32_t de = (dir[wp >> 1] >> (16 * (wp & 1))) & 0xFFFFu, cls = de >> 12;
+      if (((flags >> wp) & 1) != (cls != 0)) { g_err = "directory / active-warp mismatch"; return -1; }
       if (!((flags >> wp) & 1)) continue;
-      const uint32_t* rec = L + L[LH_WOFF0 + wp];
-      uint32_t mode = rec[4] & 0xFF, n4 = rec[4] >> 8;
+      const uint32_t* rec = L + 4 * (de & 0xFFFu);
+      if (rec != L + L[LH_WOFF0 + wp]) { g_err = "directory offset mismatch"; return -1; }
+      const uint32_t mode = cls == GEM_DC_DENSE16 ? GEM_WM_DENSE16 : cls == GEM_DC_DENSE ? GEM_WM_DENSE : GEM_WM_SPARSE;
+      const uint32_t n4 = cls == GEM_DC_DENSE16 ? 4u : cls == GEM_DC_DENSE ? 8u : cls;
+      if (rec[4] != (mode | (n4 << 8))) { g_err = "directory class / record mode mismatch"; return -1; }
       for (int c = 0; c < 4; c++) warp_c[wp][c] = rec[c];
       for (uint32_t ln = 0; ln < 32; ln++)
         for (int c = 0; c < 4; c++) lane_c[wp * 32 + ln][c] = rec[GEM_WREC_HDR + ln * 4 + c];
@@ -135,6 +144,7 @@ int run_part(Interp& I, uint32_t p, uint64_t t, const uint32_t* stim, uint32_t* 
     for (uint32_t wq = 0; wq < 8; wq++) if (wo(warp_c[wq][3], 6, 10, wq)) return -1;
     if (flags & GEM_LF_USES_TOP) if (wo(L[LH_TOPWO], 11, 13, 0)) return -1;
     for (auto& x : written) if (x == 2) x = 1;
+    for (int k = 0; k < 4; k++) dir[k] = L[LH_NEXTDIR + k];
     L += L[LH_WORDS_];
   }
   // outputs
