@@ -192,7 +192,7 @@ enum {
  *          warp record (GEM_LWREC_WORDS words):
  *            [0..5)    wxa, wxb, wob, wmask, wbase       (levels 6-10)
  *            [8..136)  lane constants uint4 {xa, xb, ob, mask}  (levels 1-5)
- *            [136..648) leaves: [4 groups][32 lanes] uint4 (32 u16 lane words
+ *            [136..648) leaves: [4 groups][32 lanes] uint4 (32 u16 lane-word byte offsets w*4
  *                       per lane, entry 8g+2k low half, 8g+2k+1 high half)
  *            [648..680) per-lane write-out base word
  *   Write-outs: a unit (thread / warp / top) stores the slots whose bits are set

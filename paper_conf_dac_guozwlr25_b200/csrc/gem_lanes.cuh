@@ -62,6 +62,11 @@ __device__ __forceinline__ void ldsK(uint32_t addr, uint32_t (&v)[K]) {
   }
 }
 template <int K>
+__device__ __forceinline__ void lds_leaf(uint32_t s_base, uint32_t off, uint32_t (&v)[K]) {
+  if (K == 1) v[0] = *reinterpret_cast<const uint32_t*>(reinterpret_cast<const char*>(g_smem) + off);
+  else ldsK<K>(s_base + K * off, v);
+}
+template <int K>
 __device__ __forceinline__ void stsK(uint32_t addr, const uint32_t (&v)[K]) {
   if (K == 1) {
     asm volatile("st.shared.u32 [%0], %1;" ::"r"(addr), "r"(v[0]) : "memory");
@@ -96,9 +101,15 @@ __device__ __forceinline__ void exec_lane_layer(const LaneRegs& R, uint32_t s_ba
     const uint32_t xa = R.lc.x, xb = R.lc.y, ob = R.lc.z, mask = R.lc.w;
     const uint32_t q8[4][4] = {{R.e[0].x, R.e[0].y, R.e[0].z, R.e[0].w}, {R.e[1].x, R.e[1].y, R.e[1].z, R.e[1].w},
                                {R.e[2].x, R.e[2].y, R.e[2].z, R.e[2].w}, {R.e[3].x, R.e[3].y, R.e[3].z, R.e[3].w}};
-    // leaf i (0..31) = u16 lane word: entry 8g+2k in the low half of q8[g][k], +1 in the high half
+    // leaf i (0..31) = u16 byte offset (lane word * 4): entry 8g+2k in the low
+    // half of q8[g][k], +1 in the high half; with K interleaved groups the
+    // word's address is K * offset, for K = 1 a plain shared load off the base
+    // pointer (LDS [R + UR]: one extract per leaf, no address arithmetic)
     auto leaf = [&](uint32_t i) -> uint32_t {
       const uint32_t q = q8[i >> 3][(i & 7) >> 1];
+#ifdef EXP_LANE_NOCONFLICT   // timing experiment only: conflict-free leaf reads (wrong results)
+      return ((q & 0x3E0u) | lane) * 4u;
+#endif
       return (i & 1) ? (q >> 16) : (q & 0xFFFFu);
     };
     // written slots go to consecutive lane words (slot-bit order) from R.base
@@ -107,8 +118,8 @@ __device__ __forceinline__ void exec_lane_layer(const LaneRegs& R, uint32_t s_ba
 #pragma unroll
     for (uint32_t q = 0; q < 16; q++) {          // level 1: A = leaf q, B = leaf q+16
       uint32_t a[K], b[K];
-      ldsK<K>(s_base + 4u * K * leaf(q), a);
-      ldsK<K>(s_base + 4u * K * leaf(q + 16), b);
+      lds_leaf<K>(s_base, leaf(q), a);
+      lds_leaf<K>(s_base, leaf(q + 16), b);
       kslot<K>(r1[q], a, b, xa, xb, ob, q);
       if (mask & (1u << q)) { stsK<K>(wp, r1[q]); wp += 4u * K; }
     }
@@ -186,8 +197,18 @@ __device__ __forceinline__ void top_lane_layer(uint32_t topc, uint32_t topwo, ui
 // groups ng..K-1 of the vectors are padding and never committed).
 template <int K>
 __device__ void run_lane_partition(const KParams& kp, ProgSrc& ps, uint32_t* S, uint32_t* ramp, uint32_t* topv,
-                                   uint32_t p, uint32_t g0, uint32_t ng, uint32_t c, uint32_t cur, uint32_t nxt) {
+                                   uint32_t p, uint32_t g0, uint32_t ng, uint32_t c, uint32_t cur, uint32_t nxt,
+                                   unsigned long long* pacc) {
   const uint32_t tid = threadIdx.x;
+  // GEM_F_PROFILE: thread 0 accumulates per-phase clocks over the CTA's items
+  unsigned long long t_ph = (pacc && tid == 0) ? clock64() : 0ull;
+  auto phase = [&](int k) {
+    if (pacc && tid == 0) {
+      const unsigned long long t = clock64();
+      pacc[k] += t - t_ph;
+      t_ph = t;
+    }
+  };
   const uint32_t s_base = smem_u32(S);
   const LaneIdx X{kp.n_groups};
   const uint32_t* gprog = kp.lprog + __ldg(kp.parts + p * GP_WORDS + GP_LANE_OFF);
@@ -200,6 +221,8 @@ __device__ void run_lane_partition(const KParams& kp, ProgSrc& ps, uint32_t* S, 
   const uint4 h1 = *(reinterpret_cast<const uint4*>(C0) + 1);
   const uint4 h2 = *(reinterpret_cast<const uint4*>(C0) + 2);
   const uint32_t n_gread = h0.y, n_layers = h0.z, n_out = h0.w;
+  if (pacc && tid == 0 && h0.x == 0u) pacc[7]++;   // (keeps the header read before the stamp)
+  phase(0);
   const uint32_t n_ram = h1.x, off_gread = h1.z;
   const uint32_t off_out = h2.x, off_ram = h2.y, off_chunks = h2.z, n_chunks = h2.w;
   for (uint32_t k = tid; k < n_chunks; k += GEM_THREADS) ps.ctab[k] = C0[off_chunks + k];
@@ -241,9 +264,11 @@ __device__ void run_lane_partition(const KParams& kp, ProgSrc& ps, uint32_t* S, 
       if (dst[u] != ~0u) sts(s_base + 4u * dst[u], v[u]);
   }
   if (tid < K) S[tid] = 0u;   // lane word 0 = constant 0 for every group
+  phase(1);
   LaneRegs R;
   if (n_layers) load_lane_layer(ring_wait(ps), R);
   __syncthreads();
+  phase(2);
   ps.seq_free = ps.seq_wait;
   refill();
   for (uint32_t l = 0; l < n_layers; l++) {
@@ -256,6 +281,7 @@ __device__ void run_lane_partition(const KParams& kp, ProgSrc& ps, uint32_t* S, 
     ps.seq_free = ps.seq_wait;
     refill();
   }
+  phase(3);
   // ---- a6: endpoint commit: one lane word per endpoint bit
   const uint32_t* od = ring_wait(ps);
   const uint2* oe = reinterpret_cast<const uint2*>(od);
@@ -306,6 +332,7 @@ __device__ void run_lane_partition(const KParams& kp, ProgSrc& ps, uint32_t* S, 
     }
   }
   __syncthreads();
+  phase(4);
   ps.seq_free = ps.seq_issue;
 }
 
@@ -374,16 +401,22 @@ __global__ void __launch_bounds__(GEM_THREADS, 2) gem_lane_kernel(const KParams 
   }
   unsigned long long bar_target = 0;
   const bool instr = (kp.flags & (GEM_F_TRACE_STATE | GEM_F_DIGEST)) != 0;
+  __shared__ unsigned long long pacc[8];   // GEM_F_PROFILE phase sums (thread 0)
   for (uint32_t c = 0; c < kp.ncycles; c++) {
     const uint64_t t = kp.t0 + c;
     const uint32_t cur = (uint32_t)(t & 1u), nxt = cur ^ 1u;
+    const bool prof_on = kp.prof && c < kp.prof_cycles;
+    if (prof_on && threadIdx.x == 0)
+      for (int k = 0; k < 8; k++) pacc[k] = 0ull;
+    PROF(0);
     if (instr && c > 0) record_state_lane(kp, c - 1, cur);
     for (uint32_t s = 0; s < kp.n_stages; s++) {
       const uint32_t kb = wl_begin(s), ke = wl_end(s);
       for (uint32_t k = kb; k < ke; k++) {
         const uint2 it = __ldg(&kp.wl_items[k]);
         const uint32_t g0 = it.y >> 5;
-        run_lane_partition<K>(kp, ps, S, ramp, topv, it.x, g0, min((uint32_t)K, kp.n_groups - g0), c, cur, nxt);
+        run_lane_partition<K>(kp, ps, S, ramp, topv, it.x, g0, min((uint32_t)K, kp.n_groups - g0), c, cur, nxt,
+                              prof_on ? pacc : nullptr);
         uint32_t nk = ~0u;
         if (k + 1 < ke) nk = k + 1;
         for (uint32_t s2 = s + 1; nk == ~0u && s2 < kp.n_stages; s2++)
@@ -391,8 +424,12 @@ __global__ void __launch_bounds__(GEM_THREADS, 2) gem_lane_kernel(const KParams 
         if (nk == ~0u && c + 1 < kp.ncycles) nk = first_item();
         if (nk != ~0u) issue_prologue_lane(kp, ps, __ldg(&kp.wl_items[nk].x));
       }
+      if (s == 0) PROF(4);
       grid_sync(kp, bar_target);
     }
+    PROF(5);
+    if (prof_on && threadIdx.x == 0)
+      for (int k = 0; k < 5; k++) kp.prof[((size_t)c * gridDim.x + blockIdx.x) * GEM_PROF_SLOTS + 11 + k] = pacc[k];
   }
   if (instr) record_state_lane(kp, kp.ncycles - 1, (uint32_t)((kp.t0 + kp.ncycles) & 1u));
 }

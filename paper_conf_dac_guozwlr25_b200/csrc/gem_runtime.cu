@@ -1169,13 +1169,20 @@ static double build_worklists(const gem_sim* sim, uint32_t G, std::vector<uint32
   double makespan = 0;
   for (uint32_t s = 0; s < sim->n_stages; s++) {
     const uint32_t pb = sim->h_stage[s], np = sim->h_stage[s + 1] - pb;
+    // a scheduling unit = `run` consecutive stream groups of one partition, kept
+    // together on one CTA (lane mode: consecutive items then share the
+    // partition's input-port list and program in L1/L2)
+    const uint32_t run = sim->lanes ? (uint32_t)std::max(1, getenv("GEM_LANE_RUN") ? atoi(getenv("GEM_LANE_RUN")) : 4)
+                                    : 1u;
     std::vector<std::pair<uint32_t, uint2>> its;
     its.reserve((size_t)np * sim->n_streams);
-    for (uint32_t st = 0; st < sim->n_streams; st += sim->group)
+    for (uint32_t st = 0; st < sim->n_streams; st += sim->group * run)
       for (uint32_t k = 0; k < np; k++) {
         const uint32_t p = sim->h_stage[sim->n_stages + 1 + pb + k];
-        const uint32_t nst = std::min(sim->group, sim->n_streams - st);
-        const double c = sim->h_parts[(size_t)p * GP_WORDS + GP_COST] * (1.0 + 0.7 * (nst - 1));
+        const uint32_t nst = std::min(sim->group * run, sim->n_streams - st);
+        const uint32_t n_items = (nst + sim->group - 1) / sim->group;
+        const double c = sim->h_parts[(size_t)p * GP_WORDS + GP_COST] *
+                         (run > 1 ? (double)n_items : (1.0 + 0.7 * (nst - 1)));
         its.push_back({(uint32_t)std::min(c, 4.0e9), make_uint2(p, st)});
       }
     std::stable_sort(its.begin(), its.end(), [](const std::pair<uint32_t, uint2>& x,
@@ -1192,7 +1199,11 @@ static double build_worklists(const gem_sim* sim, uint32_t G, std::vector<uint32
     for (auto& it : its) {
       std::pop_heap(heap.begin(), heap.end(), cmp);
       auto& h = heap.back();
-      lists[h.second].push_back(it.second);
+      for (uint32_t r = 0; r < run; r++) {
+        const uint32_t st = it.second.y + r * sim->group;
+        if (st >= sim->n_streams) break;
+        lists[h.second].push_back(make_uint2(it.second.x, st));
+      }
       h.first += std::max<uint32_t>(it.first, 1);
       mx = std::max(mx, h.first);
       std::push_heap(heap.begin(), heap.end(), cmp);

@@ -1104,7 +1104,7 @@ struct Mapper {
     word[0] = 0;   // local node 0 is the constant
     // free-interval allocator (first fit, coalescing); word 0 reserved
     std::map<uint32_t, uint32_t> freeiv;   // start -> length
-    const uint32_t kMaxWords = 65535;
+    const uint32_t kMaxWords = 16383;   // leaf entries hold byte offsets (word * 4) in 16 bits
     freeiv[1] = kMaxWords - 1;
     uint32_t max_word = 1;
     std::vector<std::vector<uint32_t>> die(L + 1);
@@ -1220,7 +1220,7 @@ struct Mapper {
               for (uint32_t h = 0; h < 2; h++) {
                 uint32_t pos = 8 * g + 2 * k + h, id = (w * 32 + ln) * 32 + pos;
                 uint32_t x = LL.leaf_sig[id];
-                e |= (x == UINT32_MAX ? 0u : lw(x)) << (16 * h);
+                e |= (x == UINT32_MAX ? 0u : 4u * lw(x)) << (16 * h);
               }
               pr.push_back(e);
             }

@@ -56,3 +56,13 @@ if a.phases:
     print(f"  all CTAs: items mean {items.mean():.0f} max {items.mean(0).max():.0f}; per-layer clocks "
           f"mean {per_layer.mean():.0f} min {per_layer.min():.0f} max {per_layer.max():.0f}; "
           f"gread mean {gread.mean():.0f}; out mean {out.mean():.0f}; barrier min {bar.mean(0).min():.0f}")
+
+if a.phases and sim.info.get("lanes"):
+    # lane mode: per-CTA sums over its work items of gread / layers / out / ram clocks (slots 11-14)
+    acc = pr[:, :, 11:16].astype(np.float64)
+    items_t = (pr[:, :, 4] - pr[:, :, 0]).astype(np.float64)
+    bar_t = (pr[:, :, 5] - pr[:, :, 4]).astype(np.float64)
+    print(f"lane phases per cycle (mean over CTAs): items {items_t.mean():.0f} clk = chunk0 {acc[:, :, 0].mean():.0f} + "
+          f"gread {acc[:, :, 1].mean():.0f} + layer0/sync {acc[:, :, 2].mean():.0f} + layers {acc[:, :, 3].mean():.0f} + "
+          f"out+ram {acc[:, :, 4].mean():.0f}; "
+          f"barrier {bar_t.mean():.0f}; items max {items_t.mean(0).max():.0f}")

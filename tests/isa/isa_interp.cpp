@@ -229,7 +229,8 @@ int run_lane_part(Interp& I, LaneSim& Ls, uint32_t p, const uint32_t* pi_lane /*
           for (uint32_t k = 0; k < 4; k++) {
             uint32_t e = lv[(g * 32 + ln) * 4 + k];
             for (uint32_t h = 0; h < 2; h++) {
-              uint32_t word = (e >> (16 * h)) & 0xFFFFu, pos = 8 * g + 2 * k + h;
+              uint32_t word = ((e >> (16 * h)) & 0xFFFFu) >> 2, pos = 8 * g + 2 * k + h;
+              if (((e >> (16 * h)) & 3u) != 0) { g_err = "lane leaf offset not word aligned"; return -1; }
               if (word >= S.size()) { g_err = "lane leaf out of range"; return -1; }
               read[word] = 1;
               val[0][(wp * 32 + ln) * 32 + pos] = 0;
@@ -249,7 +250,7 @@ int run_lane_part(Interp& I, LaneSim& Ls, uint32_t p, const uint32_t* pi_lane /*
           for (uint32_t k = 0; k < 4; k++) {
             uint32_t e = lv[(g * 32 + ln) * 4 + k];
             for (uint32_t h = 0; h < 2; h++) {
-              uint32_t word = (e >> (16 * h)) & 0xFFFFu, pos = 8 * g + 2 * k + h;
+              uint32_t word = ((e >> (16 * h)) & 0xFFFFu) >> 2, pos = 8 * g + 2 * k + h;
               wv[0][(wp * 32 + ln) * 32 + pos] = S[word];
             }
           }
