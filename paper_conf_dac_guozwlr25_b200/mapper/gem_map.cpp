@@ -59,7 +59,11 @@ struct Options {
   int levels = 13;          // deepest boomerang level used per layer (10 = no top levels 11-13)
   int stages = 1;           // 1 or 2 (multi-stage RepCut)
   int cut_level = 0;        // 0 = auto (middle)
-  int merge = 1;            // Algorithm 1 merge pass
+  int merge = 1;            // Algorithm 1 merge pass (P:119-125)
+  int key = 0;              // unit order for packing: 0 = min flop index in the cone, 1 = deep-cone
+                            // min-hash, 2 = a register's own index (declaration order = module order)
+  double merge_cap = 0;     // max merged cone size in ANDs (0 = 2.5 x part_size)
+  double merge_ratio = 0.3; // merge only if overlap >= ratio x the smaller cone
   int refine = 3;           // rounds of splitting the costliest partitions (critical path)
   double refine_ratio = 1.35;  // split partitions costing more than this x the median
   int max_parts = 280;      // refinement stops growing the partition count here
@@ -87,6 +91,9 @@ static Options parse_opts(const char* s) {
     else if (k == "stages") o.stages = std::stoi(v);
     else if (k == "cut_level") o.cut_level = std::stoi(v);
     else if (k == "merge") o.merge = std::stoi(v);
+    else if (k == "key") o.key = std::stoi(v);
+    else if (k == "merge_cap") o.merge_cap = std::stod(v);
+    else if (k == "merge_ratio") o.merge_ratio = std::stod(v);
     else if (k == "verbose") o.verbose = std::stoi(v);
     else if (k == "max_state_words") o.max_state_words = std::stoi(v);
     else if (k == "cap_slack") o.cap_slack = std::stod(v);
@@ -1419,8 +1426,23 @@ static void partition(Design& D) {
       mflop[i] = std::min(mflop[G.a[i] >> 1], mflop[G.b[i] >> 1]);
     }
   }
+  // key 1: min-hash over the endpoint's *deep* cone (nodes below a third of the
+  // depth): endpoints whose deep logic coincides -- one module's registers --
+  // sort together, whatever registers of neighbouring modules they also read
+  std::vector<uint64_t> sdeep;
+  if (opt.key == 1) {
+    sdeep.assign(N, UINT64_MAX);
+    const uint32_t thr = std::max<uint32_t>(1, G.max_level / 3);
+    for (size_t i = 0; i < N; i++) {
+      if (G.kind[i] != K_AND) continue;
+      uint64_t h = G.level[i] >= thr ? mix64(i * 0x9E3779B97F4A7C15ull + 11) : UINT64_MAX;
+      sdeep[i] = std::min(h, std::min(sdeep[G.a[i] >> 1], sdeep[G.b[i] >> 1]));
+    }
+  }
   auto key_of = [&](uint32_t lit) -> uint64_t {
     uint32_t x = lit >> 1;
+    if (opt.key == 1 && sdeep[x] != UINT64_MAX) return sdeep[x] >> 1;
+    if (opt.key == 1) return (1ull << 63) | ((uint64_t)mflop[x] << 31) | (s0[x] >> 33);
     return ((uint64_t)mflop[x] << 32) | (s0[x] >> 32);
   };
   std::vector<uint32_t> cut_nodes;            // compact ids that are stage-0 endpoints
@@ -1448,7 +1470,8 @@ static void partition(Design& D) {
     uint32_t x = lit >> 1;
     return (G.kind[x] == K_AND && G.level[x] > cut) ? 1 : 0;
   };
-  for (uint32_t j = 0; j < G.n_flops; j++) units.push_back({0, j, key_of(G.flop_next[j])});
+  for (uint32_t j = 0; j < G.n_flops; j++)
+    units.push_back({0, j, opt.key == 2 ? ((uint64_t)j << 32) : key_of(G.flop_next[j])});
   for (uint32_t j = 0; j < G.n_po; j++) units.push_back({1, j, key_of(G.po[j])});
   for (uint32_t r = 0; r < G.n_rams; r++) {
     uint64_t k = UINT64_MAX;
@@ -1555,6 +1578,93 @@ static void partition(Design& D) {
                 groups.size(), target);
       if (ratio > 0.85 && ratio < 1.2) break;
       cap *= std::max(0.5, std::min(2.0, ratio));
+    }
+    // ---- Algorithm 1: after the excessive partitioning above,
+    // visit partitions largest first; sort the unvisited ones by cone overlap
+    // with p (large to small) and merge q into p if the result stays mappable.
+    // "Mappable" here: the merged cone stays under merge_cap ANDs (the width /
+    // state check proper runs in the mapper, which splits a partition that
+    // does not fit), and the overlap is a real saving (>= merge_ratio of the
+    // smaller cone) -- merging disjoint logic would only lengthen layers.
+    if (opt.merge && groups.size() > 1) {
+      const size_t ng = groups.size();
+      std::vector<std::vector<uint32_t>> cone(ng);
+      for (size_t gi = 0; gi < ng; gi++) {
+        cur_stamp++;
+        for (uint32_t i : groups[gi]) {
+          unit_lits(su[i], lits);
+          for (uint32_t l : lits) {
+            uint32_t x = l >> 1;
+            if (stamp[x] == cur_stamp) continue;
+            stamp[x] = cur_stamp;
+            st.push_back(x);
+            while (!st.empty()) {
+              uint32_t y = st.back(); st.pop_back();
+              if (is_leaf_for(y, stage)) continue;
+              cone[gi].push_back(y);
+              for (uint32_t z : {G.a[y] >> 1, G.b[y] >> 1})
+                if (stamp[z] != cur_stamp) { stamp[z] = cur_stamp; st.push_back(z); }
+            }
+          }
+        }
+        std::sort(cone[gi].begin(), cone[gi].end());
+      }
+      // inverted index node -> groups (CSR)
+      std::vector<uint32_t> cnt(N + 1, 0);
+      for (size_t gi = 0; gi < ng; gi++) for (uint32_t x : cone[gi]) cnt[x + 1]++;
+      for (size_t i = 0; i < N; i++) cnt[i + 1] += cnt[i];
+      std::vector<uint32_t> inv(cnt[N]);
+      {
+        std::vector<uint32_t> f(cnt.begin(), cnt.end() - 1);
+        for (size_t gi = 0; gi < ng; gi++) for (uint32_t x : cone[gi]) inv[f[x]++] = (uint32_t)gi;
+      }
+      const double cap = opt.merge_cap > 0 ? opt.merge_cap : 2.5 * opt.part_size;
+      std::vector<int32_t> owner(ng);          // group -> current merged partition
+      std::iota(owner.begin(), owner.end(), 0);
+      std::vector<uint8_t> visited(ng, 0);
+      std::vector<size_t> order(ng);
+      std::iota(order.begin(), order.end(), 0);
+      std::stable_sort(order.begin(), order.end(), [&](size_t a, size_t b) { return cone[a].size() > cone[b].size(); });
+      std::vector<uint32_t> ov(ng, 0);
+      size_t merges = 0;
+      for (size_t p : order) {
+        if (visited[p]) continue;
+        visited[p] = 1;
+        // overlap of p's (growing) cone with every unvisited original group
+        std::vector<uint32_t> touched;
+        for (uint32_t x : cone[p])
+          for (uint32_t k = cnt[x]; k < cnt[x + 1]; k++) {
+            const uint32_t q = inv[k];
+            if (visited[q]) continue;
+            if (!ov[q]++) touched.push_back(q);
+          }
+        std::sort(touched.begin(), touched.end(), [&](uint32_t a, uint32_t b) {
+          return ov[a] != ov[b] ? ov[a] > ov[b] : a < b;
+        });
+        for (uint32_t q : touched) {
+          const uint32_t o = ov[q];
+          if (visited[q]) continue;
+          const size_t a = cone[p].size(), b = cone[q].size();
+          if (o < opt.merge_ratio * std::min(a, b) || a + b - o > cap) continue;
+          // commit: p absorbs q (units and cone); overlaps with q's new nodes are not re-counted
+          std::vector<uint32_t> u;
+          u.reserve(a + b - o);
+          std::set_union(cone[p].begin(), cone[p].end(), cone[q].begin(), cone[q].end(), std::back_inserter(u));
+          cone[p].swap(u);
+          groups[p].insert(groups[p].end(), groups[q].begin(), groups[q].end());
+          groups[q].clear();
+          cone[q].clear();
+          cone[q].shrink_to_fit();
+          visited[q] = 1;
+          merges++;
+        }
+        for (uint32_t q : touched) ov[q] = 0;
+      }
+      std::vector<std::vector<uint32_t>> kept;
+      for (auto& g : groups) if (!g.empty()) { std::sort(g.begin(), g.end()); kept.push_back(std::move(g)); }
+      groups.swap(kept);
+      if (opt.verbose >= 1)
+        fprintf(stderr, "gem_map: stage %d Algorithm 1 merged %zu pairs -> %zu groups\n", stage, merges, groups.size());
     }
     for (auto& grp : groups) {
       Part P;
