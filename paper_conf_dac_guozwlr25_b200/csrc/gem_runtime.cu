@@ -1029,13 +1029,17 @@ __global__ void __launch_bounds__(GEM_THREADS, 1) floor_barrier_kernel(const KPa
 __global__ void unpermute_kernel(const uint32_t* __restrict__ in, uint32_t* __restrict__ out,
                                  const uint32_t* __restrict__ int_of_ext, uint32_t n_bits, uint32_t in_words,
                                  uint32_t out_words, uint64_t rows, uint64_t in_row_stride,
-                                 uint64_t out_row_stride) {
+                                 uint64_t out_row_stride, uint64_t rows_per_group = ~0ull,
+                                 uint64_t in_group_stride = 0) {
+  // input row r lives at (r / rows_per_group) * in_group_stride + (r % rows_per_group) * in_row_stride
+  // (all streams of a read in one launch: groups = streams, rows = cycles)
   const uint64_t total = rows * out_words;
   for (uint64_t g = (uint64_t)blockIdx.x * blockDim.x + threadIdx.x; g < total;
        g += (uint64_t)gridDim.x * blockDim.x) {
     const uint64_t row = g / out_words;
     const uint32_t w = (uint32_t)(g % out_words);
-    const uint32_t* src = in + row * in_row_stride;
+    const uint64_t grp = row / rows_per_group, rr = row - grp * rows_per_group;
+    const uint32_t* src = in + grp * in_group_stride + rr * in_row_stride;
     uint32_t v = 0;
     for (uint32_t b = 0; b < 32; b++) {
       const uint32_t e = w * 32 + b;
@@ -1708,12 +1712,13 @@ int gem_read_outputs(gem_sim* sim, uint32_t* dst, uint64_t ncycles, int dst_on_d
     CK(cudaGetLastError());
   }
   // rows = stream*ncycles + cycle; in-row stride = po_words_int, with stream stride out_cap
-  for (uint32_t s = 0; s < sim->n_streams; s++) {
-    unpermute_kernel<<<std::min<uint64_t>(4096, (ncycles * sim->po_words_ext + 255) / 256 + 1), 256, 0,
-                       sim->stream>>>(sim->d_po + (size_t)s * sim->out_cap * sim->po_words_int,
-                                      out + (size_t)s * ncycles * sim->po_words_ext, sim->d_po_int_of_ext,
-                                      sim->n_po, sim->po_words_int, sim->po_words_ext, ncycles,
-                                      sim->po_words_int, sim->po_words_ext);
+  // (one launch for all streams)
+  {
+    const uint64_t rows = (uint64_t)sim->n_streams * ncycles;
+    unpermute_kernel<<<(unsigned)std::min<uint64_t>(4096, (rows * sim->po_words_ext + 255) / 256 + 1), 256, 0,
+                       sim->stream>>>(sim->d_po, out, sim->d_po_int_of_ext, sim->n_po, sim->po_words_int,
+                                      sim->po_words_ext, rows, sim->po_words_int, sim->po_words_ext, ncycles,
+                                      (uint64_t)sim->out_cap * sim->po_words_int);
   }
   CK(cudaGetLastError());
   if (!dst_on_device) CK(cudaMemcpyAsync(dst, out, bytes, cudaMemcpyDeviceToHost, sim->stream));
