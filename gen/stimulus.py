@@ -102,3 +102,25 @@ def stimulus(cfg: str, n_pi: int, cycles: int, stream: int = 0, seed: int = None
 def stimulus_streams(cfg: str, n_pi: int, cycles: int, streams, seed: int = None) -> np.ndarray:
     """uint32 [len(streams)][cycles][ceil(n_pi/32)]."""
     return np.stack([stimulus(cfg, n_pi, cycles, int(s), seed) for s in streams])
+
+
+def stim_bursts(n_pi: int, cycles: int, seed: int, period: int = 64, duty: int = 8,
+                aligned: bool = False) -> np.ndarray:
+    """Low-activity stimulus: PI k is 1 only in bursts of `duty` cycles that start
+    every `period` cycles at a per-PI random phase (the same phase for every PI
+    if `aligned`: the whole design idles between bursts), 0 otherwise (an
+    enable per module that is mostly idle).  uint32 [cycles][ceil(n_pi/32)]."""
+    rng = _rng(seed)
+    nw = n_words(n_pi)
+    w = np.zeros((cycles, nw), np.uint32)
+    t = np.arange(cycles)
+    for k in range(n_pi):
+        ph = 0 if aligned else int(rng.integers(period))
+        on = ((t + ph) % period) < duty
+        w[on, k // 32] |= np.uint32(1 << (k % 32))
+    return w
+
+
+def hold(stim: np.ndarray, r: int) -> np.ndarray:
+    """Repeat every input vector r times (inputs that change every r cycles)."""
+    return np.repeat(stim, r, axis=-2)

@@ -48,6 +48,16 @@ extern "C" {
 #define GEM_F_DIGEST 0x2u       /* record the per-cycle flop digest d_t              */
 #define GEM_F_ASYNC 0x4u        /* gem_step returns without synchronising            */
 #define GEM_F_PROFILE 0x8u      /* record per-CTA clock64 phase stamps (first 256 cycles) */
+/* Activity-based pruning (the paper's next step, P:237-241:
+ * "skip partitions whose inputs did not change").  A partition whose input-port
+ * words (PI[t], Q_cur, RD_cur, stage cuts) equal those of the previous cycle
+ * produces the same endpoint words, so its layers are skipped and its last
+ * results are committed again; RAM ports still operate every cycle.  Results
+ * are identical with and without the flag.  Applies to the bit-packed path for
+ * CTAs that run one partition of one stream per stage and cycle (every
+ * single-stream launch whose grid covers the partitions); other CTAs, and lane
+ * mode, always evaluate.  The first cycle of every gem_step evaluates. */
+#define GEM_F_ACTIVITY 0x10u
 
 typedef struct gem_sim gem_sim; /* opaque, owned by the library */
 
@@ -130,6 +140,10 @@ int gem_last_step_ms(gem_sim* sim, float* ms);
  * Call with dst = NULL to query n_cycles / grid. */
 #define GEM_PROF_SLOTS 16
 int gem_read_profile(gem_sim* sim, uint64_t* dst, uint32_t* n_cycles, uint32_t* grid);
+
+/* Needs GEM_F_ACTIVITY: partition-cycles evaluated and skipped since load
+ * (summed over CTAs eligible for pruning; ineligible CTAs are not counted). */
+int gem_read_activity(gem_sim* sim, uint64_t* evaluated, uint64_t* skipped);
 
 void gem_free(gem_sim* sim);
 const char* gem_last_error(void);

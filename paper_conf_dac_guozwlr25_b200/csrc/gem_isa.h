@@ -124,7 +124,9 @@ enum {
  * TMA bulk copies (cp.async.bulk, 16-byte granules): chunk 0 = header + chunk
  * table + gread list, chunks 1..n_layers = one layer record each, chunk
  * n_layers+1 = output + RAM sections.  The chunk table (PH_OFF_CHUNKS) holds
- * the word size of every chunk (all multiples of 4 words).                  */
+ * the word size of every chunk (all multiples of 4 words).  After the last
+ * chunk, the program's final ceil4(n_gread) words hold the used-bit mask of
+ * every gread word (entry order; read only by GEM_F_ACTIVITY, row f3).      */
 /* partition program header (16 words) */
 enum {
   PH_MAGIC = 0, PH_N_GREAD, PH_N_LAYERS, PH_N_OUT, PH_N_RAM, PH_STATE_WORDS, PH_OFF_GREAD,

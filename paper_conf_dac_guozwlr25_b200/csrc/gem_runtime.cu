@@ -71,6 +71,10 @@ struct KParams {
   uint32_t fine_cta;                     // CTA stamped by GEM_FINE_PROF builds (env GEM_FINE_CTA)
   const uint32_t* __restrict__ wl_off;   // [n_stages][grid+1] CSR offsets into wl_items
   const uint2* __restrict__ wl_items;    // {partition, stream} per work item
+  // GEM_F_ACTIVITY (row f3): per-CTA copy of the last input-port words
+  // (act_words >= max n_gread) and {evaluated, skipped} partition-cycle counters
+  unsigned long long* act_cnt;
+  uint32_t act_words;
 };
 #ifdef GEM_FINE_PROF
 // sub-stamps inside exec_layer: fl = layer index when stamping, >= 32 otherwise;
@@ -555,9 +559,14 @@ __device__ __forceinline__ void top_layer(uint32_t topc, uint32_t topwo, uint32_
 // S + j*state_words) in one cycle; every program chunk is loaded once and
 // applied to all streams of the group.  In streamed mode the caller has
 // already issued the item's prologue chunks.
+// act != nullptr (GEM_F_ACTIVITY, CTA runs this one partition of one stream):
+// the input-port words are compared with the previous cycle's copy in `act`
+// before they enter S; if none changed (and !act_first) the layers are skipped
+// -- S still holds the previous evaluation of the same inputs, so the endpoint
+// commit below re-stores the same words (row f3).
 __device__ void run_partition(const KParams& kp, ProgSrc& ps, uint32_t* S, uint32_t* ramp, uint32_t* topb,
                               uint32_t p, uint32_t st0, uint32_t nst, uint32_t c, uint32_t cur, uint32_t nxt,
-                              bool prof_on) {
+                              bool prof_on, uint32_t* act = nullptr, bool act_first = true) {
   const uint32_t tid = threadIdx.x, lane = tid & 31, warp = tid >> 5;
   const uint32_t SW = kp.state_words;
   const uint32_t s_base = smem_u32(S);
@@ -613,6 +622,10 @@ __device__ void run_partition(const KParams& kp, ProgSrc& ps, uint32_t* S, uint3
   // their L2 latencies overlap
   const uint2* gr = reinterpret_cast<const uint2*>(C0 + off_gread);
   const uint32_t n_gr = n_gread * nst;
+  bool changed = act_first;
+  // GEM_F_ACTIVITY: used-bit masks of the gread words (the program's tail)
+  const uint32_t* gmask = act ? gprog + __ldg(kp.parts + p * GP_WORDS + GP_PROG_LEN) - ((n_gread + 3u) & ~3u)
+                              : nullptr;
   for (uint32_t k0 = 0; k0 < n_gr; k0 += 4 * GEM_THREADS) {
     uint32_t v[4], dst[4];
 #pragma unroll
@@ -634,7 +647,22 @@ __device__ void run_partition(const KParams& kp, ProgSrc& ps, uint32_t* S, uint3
     }
 #pragma unroll
     for (uint32_t u = 0; u < 4; u++)
-      if (dst[u] != ~0u) sts(s_base + 4 * dst[u], v[u]);
+      if (dst[u] != ~0u) {
+        if (act) {
+          const uint32_t k = k0 + u * GEM_THREADS + tid;
+          changed |= ((act[k] ^ v[u]) & __ldg(gmask + k)) != 0u;
+          act[k] = v[u];
+        } else {
+          sts(s_base + 4 * dst[u], v[u]);
+        }
+      }
+  }
+  bool skip = false;
+  if (act) {
+    skip = __syncthreads_or(changed ? 1 : 0) == 0;
+    if (!skip)
+      for (uint32_t k = tid; k < n_gr; k += GEM_THREADS) sts(s_base + 4 * gr[k].y, act[k]);
+    if (tid == 0) atomicAdd(kp.act_cnt + (skip ? 1 : 0), 1ull);
   }
   PROF(8);
   if (tid < nst) S[tid * SW] = 0u;
@@ -657,9 +685,12 @@ __device__ void run_partition(const KParams& kp, ProgSrc& ps, uint32_t* S, uint3
   // BAR.SYNC.DEFER_BLOCKING otherwise defers to the first dependent access)
   if (prof_on && tid == 0 && lds(s_base) == 0u) PROF(1);
   refill();
+  // a skipped partition whose chunks are all in shared memory bypasses the
+  // layer loop; one that streams chunks still walks the ring (no evaluation)
+  const uint32_t n_run = (skip && (ps.resident || n_layers + 1 < n_pin)) ? 0u : n_layers;
   // ---- a3-a5: layers, software-pipelined: layer l+1's records are loaded
   // into registers before the barrier that ends layer l
-  for (uint32_t l = 0; l < n_layers; l++) {
+  for (uint32_t l = 0; l < n_run; l++) {
     FPROF(l, 0);
 #ifdef GEM_FINE_PROF
     const uint32_t fl = (kp.fprof && c == 5 && blockIdx.x == kp.fine_cta) ? l : 99u;
@@ -669,7 +700,8 @@ __device__ void run_partition(const KParams& kp, ProgSrc& ps, uint32_t* S, uint3
     unsigned long long* fsub = nullptr;
 #endif
     // stream j uses named barrier 1 + j (group <= GEM_MAX_GROUP < 16)
-    if (nst == 1 && s_base == GEM_S0_ADDR) exec_layer<true>(R, s_base, g_smem, topb, 1, fl, fsub);
+    if (skip) {
+    } else if (nst == 1 && s_base == GEM_S0_ADDR) exec_layer<true>(R, s_base, g_smem, topb, 1, fl, fsub);
     else
       for (uint32_t j = 0; j < nst; j++)
         exec_layer<false>(R, s_base + 4 * j * SW, g_smem + j * SW, topb + 16 * j, 1 + j, fl, fsub);
@@ -699,7 +731,7 @@ __device__ void run_partition(const KParams& kp, ProgSrc& ps, uint32_t* S, uint3
     }
     FPROF(l, 3);
 #if !defined(EXP_NO_TOP) && !defined(GEM_TOP_ATOMIC)
-    if (ptop && warp == 0)
+    if (ptop && warp == 0 && !skip)
       for (uint32_t j = 0; j < nst; j++) top_layer(ptopc, ptopwo, s_base + 4 * j * SW, topb + 16 * j, 1 + j);
 #endif
     FPROF(l, 4);
@@ -710,6 +742,7 @@ __device__ void run_partition(const KParams& kp, ProgSrc& ps, uint32_t* S, uint3
   }
   PROF(2);
   // ---- a6: endpoint commit (warp ballot-gather per output word and stream)
+  if (n_run == 0 && n_layers) __syncthreads();   // bypassed: S / ramp reads below follow the port compare
   const uint32_t* od = n_layers + 1 < n_pin ? (C0 + off_out) : ring_wait(ps);
   const uint32_t* os = od + n_out_pad;
   for (uint32_t jj = warp; jj < n_out * nst; jj += GEM_WARPS) {
@@ -794,6 +827,7 @@ __global__ void __launch_bounds__(GEM_THREADS, 2) gem_step_kernel(const KParams 
   // per stage, [24] cached flag, [32, 32 + 2*GEM_WL_CACHE) items (uint2)
   uint32_t* wlc = res_n + 16;
   uint64_t* mbar = reinterpret_cast<uint64_t*>(wlc + GEM_WL_CACHE_WORDS);
+  uint32_t* act_buf = reinterpret_cast<uint32_t*>(mbar + 8);   // [act_words] (GEM_F_ACTIVITY)
   const uint32_t tid = threadIdx.x;
   const uint32_t G = gridDim.x, B = blockIdx.x;
   if (tid == 0) {
@@ -922,6 +956,14 @@ __global__ void __launch_bounds__(GEM_THREADS, 2) gem_step_kernel(const KParams 
     const uint32_t p0 = first_part();
     if (p0 != ~0u) prologue(p0);
   }
+  // activity pruning: only a CTA with exactly one work item (one partition,
+  // one stream) per cycle keeps S, ramp and the port copy from cycle to cycle
+  uint32_t* act = nullptr;
+  if (kp.act_words && kp.group == 1) {
+    uint32_t n_it = 0;
+    for (uint32_t s = 0; s < kp.n_stages; s++) n_it += wl_end(s) - wl_begin(s);
+    if (n_it == 1) act = act_buf;
+  }
 
   unsigned long long bar_target = 0;
   const bool instr = (kp.flags & (GEM_F_TRACE_STATE | GEM_F_DIGEST)) != 0;
@@ -936,7 +978,8 @@ __global__ void __launch_bounds__(GEM_THREADS, 2) gem_step_kernel(const KParams 
       for (uint32_t k = kb; k < ke; k++) {
         const uint2 it = wl_item(s, k);
         const uint32_t nst = min(kp.group, kp.n_streams - it.y);
-        run_partition(kp, ps, S, ramp, topb, it.x, it.y, nst, c, cur, nxt, prof_on && k == kb && s == 0);
+        run_partition(kp, ps, S, ramp, topb, it.x, it.y, nst, c, cur, nxt, prof_on && k == kb && s == 0, act,
+                      c == 0);
         if (!ps.resident) {
           // prefetch the next work item's prologue (overlaps the grid barrier)
           uint32_t np = ~0u;
@@ -1088,6 +1131,8 @@ struct gem_sim {
   uint32_t max_items = 0;
   uint32_t area_words = 0, slot_words = 0, ring_slots = 0, resident = 0, group = 1;
   // lane mode (stream-sliced, >= 32 streams and a blob with lane programs)
+  uint32_t act_words = 0;                      // GEM_F_ACTIVITY: max n_gread over partitions
+  unsigned long long* d_act = nullptr;         // {evaluated, skipped}
   uint32_t lanes = 0, n_groups = 0, lane_words = 0, lane_max_chunk = 0, ramp_words = 0, lane_groups = 1;
   uint32_t *d_lprog = nullptr, *d_pi_lane = nullptr, *d_po_lane = nullptr;
   std::vector<uint32_t> h_parts, h_stage;
@@ -1252,8 +1297,9 @@ static int plan_launch(gem_sim* sim, uint32_t max_chunk_words, uint32_t grid_lim
   for (uint32_t s = 0; s < sim->n_stages; s++)
     sim->max_items = std::max(sim->max_items, (sim->h_stage[s + 1] - sim->h_stage[s]) *
                                                   ((sim->n_streams + sim->group - 1) / sim->group));
-  const uint32_t fixed_words =
-      sim->group * (sim->state_words + 4 * GEM_MAX_RAMS_PER_PART + 16) + GEM_MAX_CHUNKS + 48 + GEM_WL_CACHE_WORDS + 16;
+  if (sim->group != 1) sim->act_words = 0;   // activity pruning needs one stream per work item
+  const uint32_t fixed_words = sim->group * (sim->state_words + 4 * GEM_MAX_RAMS_PER_PART + 16) + GEM_MAX_CHUNKS +
+                               48 + GEM_WL_CACHE_WORDS + 16 + sim->act_words;
   const char* env = getenv("GEM_NO_RESIDENT");
   const bool allow_res = !(env && env[0] == '1');
   const char* benv = getenv("GEM_BPS");
@@ -1445,6 +1491,7 @@ int gem_load_program(const void* blob, size_t nbytes, const gem_config* cfg, gem
       delete sim;
       return fail(GEM_E_FORMAT, "bad partition program");
     }
+    if (cfg->flags & GEM_F_ACTIVITY) sim->act_words = std::max(sim->act_words, (pr[PH_N_GREAD] + 3u) & ~3u);
   }
   // inverse permutation tables
   std::vector<uint32_t> q_int_of_ext(std::max<uint32_t>(sim->n_flops, 1), 0),
@@ -1502,6 +1549,8 @@ int gem_load_program(const void* blob, size_t nbytes, const gem_config* cfg, gem
   CK(dalloc(&sim->d_bar, (size_t)(GEM_BAR_MAX_CTAS + 2) * GEM_BAR_STRIDE * 8));
   CK(dalloc(&sim->d_err, 64));
   CK(cudaMemset(sim->d_err, 0, 64));
+  CK(dalloc(&sim->d_act, 16));
+  CK(cudaMemset(sim->d_act, 0, 16));
   // initial state: flops = init (U5), RD = 0, RAM = 0 (U10)
   if (sim->lanes) {
     const size_t G = sim->n_groups, qb = (size_t)sim->q_words_int * 32;
@@ -1610,6 +1659,8 @@ int gem_step(gem_sim* sim, uint64_t ncycles) {
   kp.wl_off = sim->d_wl_off;
   kp.group = sim->group;
   kp.wl_items = sim->d_wl_items;
+  kp.act_cnt = sim->d_act;
+  kp.act_words = sim->lanes ? 0u : sim->act_words;
   if (sim->flags & GEM_F_PROFILE) {
     const uint32_t pc = (uint32_t)std::min<uint64_t>(ncycles, 256);
     if (!sim->d_prof || sim->prof_cycles < pc) {
@@ -1849,6 +1900,19 @@ int gem_read_profile(gem_sim* sim, uint64_t* dst, uint32_t* n_cycles, uint32_t* 
   return GEM_OK;
 }
 
+int gem_read_activity(gem_sim* sim, uint64_t* evaluated, uint64_t* skipped) {
+  if (int r = check(sim)) return r;
+  if (!evaluated || !skipped) return fail(GEM_E_INVAL, "null argument");
+  if (!(sim->flags & GEM_F_ACTIVITY)) return fail(GEM_E_INVAL, "GEM_F_ACTIVITY not set");
+  CK(cudaSetDevice(sim->device));
+  CK(cudaStreamSynchronize(sim->stream));
+  unsigned long long h[2] = {0, 0};
+  CK(cudaMemcpy(h, sim->d_act, 16, cudaMemcpyDeviceToHost));
+  *evaluated = h[0];
+  *skipped = h[1];
+  return GEM_OK;
+}
+
 void gem_free(gem_sim* sim) {
   if (!sim) return;
   cudaSetDevice(sim->device);
@@ -1858,7 +1922,7 @@ void gem_free(gem_sim* sim) {
                   (void*)sim->d_cut, (void*)sim->d_mem, (void*)sim->d_pi, (void*)sim->d_po, (void*)sim->d_qtrace,
                   (void*)sim->d_scratch, (void*)sim->d_digest, (void*)sim->d_bar, (void*)sim->d_err,
                   (void*)sim->d_prof, (void*)sim->d_wl_off, (void*)sim->d_wl_items, (void*)sim->d_lprog,
-                  (void*)sim->d_pi_lane, (void*)sim->d_po_lane})
+                  (void*)sim->d_pi_lane, (void*)sim->d_po_lane, (void*)sim->d_act})
     if (p) cudaFree(p);
   if (sim->ev0) cudaEventDestroy(sim->ev0);
   if (sim->ev1) cudaEventDestroy(sim->ev1);

@@ -19,11 +19,12 @@ GEM_F_TRACE_STATE = 0x1
 GEM_F_DIGEST = 0x2
 GEM_F_ASYNC = 0x4
 GEM_F_PROFILE = 0x8
+GEM_F_ACTIVITY = 0x10
 ERRORS = {-1: "GEM_E_INVAL", -2: "GEM_E_FORMAT", -3: "GEM_E_CUDA", -4: "GEM_E_NOMEM", -5: "GEM_E_NOINPUT",
           -6: "GEM_E_UNSUPPORTED"}
 EXPORTS = ["gem_load_program", "gem_info_get", "gem_set_inputs", "gem_step", "gem_read_outputs",
            "gem_read_state", "gem_write_state", "gem_read_state_trace", "gem_read_digests", "gem_read_ram",
-           "gem_write_ram", "gem_last_step_ms", "gem_read_profile", "gem_bench_floor", "gem_free", "gem_last_error"]
+           "gem_write_ram", "gem_last_step_ms", "gem_read_profile", "gem_read_activity", "gem_bench_floor", "gem_free", "gem_last_error"]
 
 
 class GemConfig(ctypes.Structure):
@@ -79,6 +80,7 @@ def load_library(build: bool = True):
             lib.gem_write_ram.argtypes = [P, u32, u32, P]
             lib.gem_last_step_ms.argtypes = [P, ctypes.POINTER(ctypes.c_float)]
             lib.gem_read_profile.argtypes = [P, P, ctypes.POINTER(u32), ctypes.POINTER(u32)]
+            lib.gem_read_activity.argtypes = [P, ctypes.POINTER(u64), ctypes.POINTER(u64)]
             lib.gem_free.argtypes = [P]
             lib.gem_free.restype = None
             lib.gem_last_error.restype = ctypes.c_char_p
@@ -206,6 +208,12 @@ class Simulator:
         out = np.zeros((n.value, g.value, 16), np.uint64)
         self._check(self.lib.gem_read_profile(self._h, _p(out), ctypes.byref(n), ctypes.byref(g)))
         return out
+
+    def read_activity(self) -> tuple:
+        """(evaluated, skipped) partition-cycles since load (GEM_F_ACTIVITY)."""
+        e, k = ctypes.c_uint64(), ctypes.c_uint64()
+        self._check(self.lib.gem_read_activity(self._h, ctypes.byref(e), ctypes.byref(k)))
+        return int(e.value), int(k.value)
 
     def run(self, pi: np.ndarray) -> np.ndarray:
         """Convenience: set_inputs + step + read_outputs."""

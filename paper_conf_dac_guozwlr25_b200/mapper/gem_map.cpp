@@ -890,6 +890,20 @@ struct Mapper {
     if (opt.banks) max_state = rename_state_words(pr, (uint32_t)opt.max_state_words);
     pr[PH_N_LEAVES] = total_leaves;
     pr[PH_N_NODES] = n_and;
+    // used-bit mask of every gread word (gem_isa.h: the last ceil4(n_gread)
+    // words of the program, outside the chunks; read by GEM_F_ACTIVITY only)
+    {
+      std::vector<uint32_t> gmask(n_gread, 0u);
+      for (uint32_t i = 0; i < n; i++) {
+        if (!is_src[i]) continue;
+        uint32_t c = nodes[i];
+        if (G.kind[c] == K_CONST) continue;
+        uint32_t gb = G.gbit[c];
+        gmask[gword[GEM_GID(gb >> 27, (gb >> 5) & 0x3FFFFF)] - 1] |= 1u << (gb & 31);
+      }
+      pr.insert(pr.end(), gmask.begin(), gmask.end());
+      while (pr.size() % 4) pr.push_back(0);
+    }
     P.n_layers = n_layers;
     P.state_words = max_state;
     P.n_leaves = total_leaves;

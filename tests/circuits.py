@@ -108,3 +108,54 @@ def small_G(seed: int = 7, n_and: int = 3000, with_ram: bool = True, reset: bool
                  pi_per_cluster=8, neighbour_flops=16)
     net, _ = build_G(spec, seed)
     return net
+
+
+def gated_counters(n_blocks: int = 8, width: int = 16) -> Netlist:
+    """n_blocks independent modules with their own enable PI: cnt_k' = cnt_k + en_k,
+    acc_k' = acc_k ^ (cnt_k ^ (cnt_k << 1)) when en_k (a module that is idle while
+    its enable is 0).  PIs: en_0..en_{n-1}; POs: every cnt/acc bit.  Used by the
+    activity-pruning tests (row f3): idle modules' partitions see unchanged inputs."""
+    b = AigBuilder(f"gated{n_blocks}x{width}")
+    ens = b.inputs_n(n_blocks)
+    for k in range(n_blocks):
+        en = ens[k]
+        cnt = [b.latch() for _ in range(width)]
+        acc = [b.latch(init=(k + i) & 1) for i in range(width)]
+        carry = en
+        for i in range(width):
+            b.set_next(cnt[i], b.XOR(cnt[i], carry))
+            carry = b.AND(cnt[i], carry)
+        for i in range(width):
+            mix = b.XOR(cnt[i], cnt[i - 1] if i else AigBuilder.FALSE)
+            b.set_next(acc[i], b.MUX(en, b.XOR(acc[i], mix), acc[i]))
+        for q in cnt + acc:
+            b.output(q)
+    return b.finish()
+
+
+def gated_modules(n_blocks: int = 64, flops: int = 64, width: int = 256, depth: int = 48, seed: int = 1) -> Netlist:
+    """n_blocks modules of random layered logic (depth `depth`, `width` ANDs per
+    level over the module's own flops) whose flops load the logic's outputs only
+    while the module's enable PI is 1 (q' = en ? f(q) : q).  PIs: en_k; POs: the
+    first 8 flops of each module.  The measurement design of row f3."""
+    rng = np.random.default_rng(seed)
+    b = AigBuilder(f"gmods{n_blocks}")
+    ens = b.inputs_n(n_blocks)
+    for k in range(n_blocks):
+        q = [b.latch(init=int(rng.integers(2))) for _ in range(flops)]
+        levels = [q]
+        for _ in range(depth):
+            prev = levels[-1]
+            pool = [x for lv in levels[-3:] for x in lv]
+            cur = []
+            for _ in range(width):
+                x = prev[int(rng.integers(len(prev)))] ^ int(rng.integers(2))
+                y = pool[int(rng.integers(len(pool)))] ^ int(rng.integers(2))
+                cur.append(b.AND(x, y))
+            levels.append(cur)
+        last = levels[-1]
+        for i in range(flops):
+            b.set_next(q[i], b.MUX(ens[k], last[i % len(last)] ^ (i & 1), q[i]))
+        for i in range(8):
+            b.output(q[i])
+    return b.finish()

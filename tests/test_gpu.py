@@ -30,7 +30,8 @@ def gem():
 def _full_parity(gem, path, b, stim, n_streams=1, chunks=(None,), **kw):
     """Run GPU and oracle; compare PO + state trace every cycle."""
     T = stim.shape[-2]
-    sim = gem.Simulator(b, n_streams=n_streams, flags=gem.GEM_F_TRACE_STATE | gem.GEM_F_DIGEST, **kw)
+    flags = gem.GEM_F_TRACE_STATE | gem.GEM_F_DIGEST | kw.pop("extra_flags", 0)
+    sim = gem.Simulator(b, n_streams=n_streams, flags=flags, **kw)
     po_g, st_g, dg_g = [], [], []
     bounds = [0, T] if chunks == (None,) else [0, *chunks, T]
     for a, e in zip(bounds[:-1], bounds[1:]):
@@ -82,6 +83,49 @@ def test_cells_ram_shift(gem, tmp_path):
         if name == "ram":
             st[:, 0] = (st[:, 0] & ~np.uint32(0x3FFFFFF)) | (st[:, 0] & 0x7) | ((st[:, 0] & 0x7) << 13)
         _full_parity(gem, p, compile_file(p), st)
+
+
+def test_activity_pruning_gated_modules(gem, tmp_path):
+    """Row f3 (GEM_F_ACTIVITY): partitions whose input ports did not
+    change are skipped; every PO and flop stays bit-exact, and the idle
+    modules' partition-cycles are actually skipped."""
+    from gen.stimulus import stim_bursts
+    from paper_conf_dac_guozwlr25_b200.mapping import compile_file
+    net = circuits.gated_counters(8, 16)
+    p = circuits.save(net, str(tmp_path), "gated")
+    T = 1000
+    st = stim_bursts(8, T, 11)
+    sim = _full_parity(gem, p, compile_file(p, "parts=8"), st, chunks=(1, 300), extra_flags=gem.GEM_F_ACTIVITY)
+    ev, sk = sim.read_activity()
+    n_parts = sim.info["n_parts"]
+    assert n_parts >= 4 and sim.info["grid"] == n_parts
+    assert ev + sk == n_parts * T          # every CTA runs one partition: all eligible
+    assert sk > 0.5 * (ev + sk), (ev, sk)  # enables are on 8/64 of the cycles
+    # the same design with inputs that change every cycle: nothing to skip
+    rng = np.random.default_rng(3)
+    st2 = rng.integers(0, 256, size=(200, 1)).astype(np.uint32)
+    sim2 = _full_parity(gem, p, compile_file(p, "parts=8"), st2, extra_flags=gem.GEM_F_ACTIVITY)
+    ev2, sk2 = sim2.read_activity()
+    assert ev2 + sk2 == n_parts * 200 and sk2 < ev2
+
+
+def test_activity_pruning_ram_stages_streamed(gem, tmp_path):
+    """GEM_F_ACTIVITY on designs with RAM blocks, two stages, streamed programs
+    (no residency) and multi-item CTAs: results equal the oracle's."""
+    from gen.stimulus import hold
+    from paper_conf_dac_guozwlr25_b200.mapping import compile_file
+    net = circuits.small_G(seed=21, n_and=4000, with_ram=True)
+    p = circuits.save(net, str(tmp_path), "g")
+    st = hold(stim_random(net.n_pi, 100, 3, reset_pi0_cycles=2), 4)
+    for opts, kw in [("parts=5", {}), ("parts=5 stages=2", {}), ("parts=5", {"grid_limit": 2})]:
+        _full_parity(gem, p, compile_file(p, opts), st, chunks=(7, 200), extra_flags=gem.GEM_F_ACTIVITY, **kw)
+    import os
+    os.environ["GEM_NO_RESIDENT"] = "1"
+    try:
+        _full_parity(gem, p, compile_file(p, "parts=5"), st, extra_flags=gem.GEM_F_ACTIVITY)
+    finally:
+        del os.environ["GEM_NO_RESIDENT"]
+    _full_parity(gem, eaig("c1"), blob("c1"), hold(stimulus("c1", 35, 500), 3), extra_flags=gem.GEM_F_ACTIVITY)
 
 
 def test_c2_full_parity(gem):

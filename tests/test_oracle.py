@@ -398,3 +398,22 @@ def test_parser_rejects_double_owned_rdata(tmp_path):
     open(p, "w").write(txt + line.replace("gem-ram 0", "gem-ram 1") + "\n")
     with pytest.raises(ValueError):
         Oracle(p)
+
+
+def test_gated_counters_closed_form(tmp_path):
+    """Closed form for the activity-pruning test design (tests/circuits.py
+    gated_counters): counter k at cycle t = number of cycles u < t with en_k(u)=1,
+    mod 2^16 (flop semantics: 1-cycle delay, PO sampled before the edge, U11)."""
+    from gen.stimulus import stim_bursts
+    net = circuits.gated_counters(8, 16)
+    p = circuits.save(net, str(tmp_path), "gated")
+    st = stim_bursts(8, 700, 11)
+    po = Oracle(p).run(st)["po"].astype(np.int64)
+    en = st[:, 0].astype(np.int64)
+    for k in range(8):
+        want = np.concatenate([[0], np.cumsum((en >> k) & 1)[:-1]]) & 0xFFFF
+        got = (po[:, k] & 0xFFFF)          # module k's POs: cnt (16 bits) then acc (16 bits) = word k
+        assert np.array_equal(got, want), k
+        on = ((en >> k) & 1).astype(bool)
+        acc = po[:, k] >> 16               # acc only changes in cycles after an enabled one
+        assert np.array_equal(acc[1:][~on[:-1]], acc[:-1][~on[:-1]]), k
