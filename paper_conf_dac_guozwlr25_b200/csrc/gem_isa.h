@@ -189,11 +189,14 @@ enum {
  * Lane partition program: header (16) | chunk table | layers | out+ram | gread
  *   (chunks: 0 = header + table, 1..L = layers, L+1 = out+ram; the gread list
  *   is read from global memory)
- *   gread: uint2 {gid_l, dst lane word}
+ *   gread: one u32 gid_l per entry; entry k is stored to lane word k + 1
  *   layer: header (16 words) {size, flags, topc, top_mask | top_base << 8, woff[8], 0...}
  *          warp record (GEM_LWREC_WORDS words):
  *            [0..5)    wxa, wxb, wob, wmask, wbase       (levels 6-10)
- *            [8..136)  lane constants uint4 {xa, xb, ob, mask}  (levels 1-5)
+ *            [8..136)  lane constants uint4 {xa, xb, ob, mask}  (levels 1-5; xa/xb/ob
+ *                      byte-spread: slot bit b at bit 8*(b&3) + 7 - (b>>2), so
+ *                      prmt(c << (b>>2), sign-replicate byte b&3) is its mask;
+ *                      mask keeps slot-bit order)
  *            [136..648) leaves: [4 groups][32 lanes] uint4 (32 u16 lane-word byte offsets w*4
  *                       per lane, entry 8g+2k low half, 8g+2k+1 high half)
  *            [648..680) per-lane write-out base word

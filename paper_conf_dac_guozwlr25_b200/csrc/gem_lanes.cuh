@@ -1,6 +1,6 @@
 // gem_lanes.cuh -- lane mode: stream-sliced execution of the same VLIW
 // placement for batched stimulus streams.
-// Included by gem_runtime.cu (shares KParams, the TMA ring and mbarriers).
+// Included by gem_runtime.cu (shares KParams and the grid barrier).
 //
 // Every signal of a 32-stream group is one 32-bit lane word (bit s = stream s),
 // so one pass over a boomerang layer evaluates it for 32
@@ -25,24 +25,28 @@ struct LaneRegs {
   uint32_t base;              // write-out base lane word
   uint4 wc;                   // wxa, wxb, wob, wmask (levels 6-10)
   uint32_t wbase;
-  uint32_t flags, topc, topwo;
+  uint32_t flags, topc, topwo, size;
 };
 
+// Records come straight from global memory (L2-resident program; no shared
+// memory ring): every warp loads its own record of the layer at L, issued one
+// layer ahead of its use so the L2 latency hides behind the current layer.
 __device__ __forceinline__ void load_lane_layer(const uint32_t* L, LaneRegs& R) {
   const uint32_t lane = threadIdx.x & 31, warp = threadIdx.x >> 5;
-  const uint4 h = *reinterpret_cast<const uint4*>(L);
+  const uint4 h = __ldg(reinterpret_cast<const uint4*>(L));
+  R.size = h.x;
   R.flags = h.y;
   R.topc = h.z;
   R.topwo = h.w;
   if ((R.flags >> warp) & 1u) {
-    const uint32_t* rec = L + L[LLH_WOFF0 + warp];
-    R.wc = *reinterpret_cast<const uint4*>(rec);
-    R.wbase = rec[4];
-    R.lc = *(reinterpret_cast<const uint4*>(rec + GEM_LWREC_HDR) + lane);
+    const uint32_t* rec = L + __ldg(L + LLH_WOFF0 + warp);
+    R.wc = __ldg(reinterpret_cast<const uint4*>(rec));
+    R.wbase = __ldg(rec + 4);
+    R.lc = __ldg(reinterpret_cast<const uint4*>(rec + GEM_LWREC_HDR) + lane);
     const uint4* lv = reinterpret_cast<const uint4*>(rec + GEM_LWREC_LEAVES) + lane;
 #pragma unroll
-    for (uint32_t g = 0; g < 4; g++) R.e[g] = lv[g * 32];
-    R.base = rec[GEM_LWREC_BASE + lane];
+    for (uint32_t g = 0; g < 4; g++) R.e[g] = __ldg(lv + g * 32);
+    R.base = __ldg(rec + GEM_LWREC_BASE + lane);
   }
 }
 
@@ -86,6 +90,20 @@ __device__ __forceinline__ void kslot(uint32_t (&o)[K], const uint32_t (&A)[K], 
 #pragma unroll
   for (int j = 0; j < K; j++) o[j] = (A[j] ^ XA) & ((B[j] ^ XB) | OB);
 }
+// levels 1-5: byte-spread constants (gem_isa.h); b is a compile-time slot bit,
+// so the shift is shared by 4 slots and the mask is one PRMT sign-replicate
+__device__ __forceinline__ uint32_t pmask(uint32_t c, uint32_t b) {
+  uint32_t r;
+  asm("prmt.b32 %0, %1, 0, %2;" : "=r"(r) : "r"(c << (b >> 2)), "r"(0x8888u + (b & 3u) * 0x1111u));
+  return r;
+}
+template <int K>
+__device__ __forceinline__ void kslotp(uint32_t (&o)[K], const uint32_t (&A)[K], const uint32_t (&B)[K], uint32_t xa,
+                                       uint32_t xb, uint32_t ob, uint32_t b) {
+  const uint32_t XA = pmask(xa, b), XB = pmask(xb, b), OB = pmask(ob, b);
+#pragma unroll
+  for (int j = 0; j < K; j++) o[j] = (A[j] ^ XA) & ((B[j] ^ XB) | OB);
+}
 template <int K>
 __device__ __forceinline__ void lane_woK(uint32_t s_base, uint32_t mask, uint32_t base, uint32_t b,
                                          const uint32_t (&v)[K]) {
@@ -96,7 +114,11 @@ __device__ __forceinline__ void lane_woK(uint32_t s_base, uint32_t mask, uint32_
 template <int K>
 __device__ __forceinline__ void exec_lane_layer(const LaneRegs& R, uint32_t s_base, uint32_t* topv, uint32_t bid) {
   const uint32_t lane = threadIdx.x & 31, warp = threadIdx.x >> 5;
+#ifdef EXP_LANE_NOTOP   // timing experiment: no levels 11-13 hand-off
+  const bool uses_top = false;
+#else
   const bool uses_top = (R.flags & GEM_LF_USES_TOP) != 0;
+#endif
   if ((R.flags >> warp) & 1u) {
     const uint32_t xa = R.lc.x, xb = R.lc.y, ob = R.lc.z, mask = R.lc.w;
     const uint32_t q8[4][4] = {{R.e[0].x, R.e[0].y, R.e[0].z, R.e[0].w}, {R.e[1].x, R.e[1].y, R.e[1].z, R.e[1].w},
@@ -118,32 +140,39 @@ __device__ __forceinline__ void exec_lane_layer(const LaneRegs& R, uint32_t s_ba
 #pragma unroll
     for (uint32_t q = 0; q < 16; q++) {          // level 1: A = leaf q, B = leaf q+16
       uint32_t a[K], b[K];
+#ifdef EXP_LANE_NOLEAF   // timing experiment only: leaves from registers (wrong results)
+      for (int j = 0; j < K; j++) { a[j] = leaf(q) ^ lane; b[j] = leaf(q + 16) + lane; }
+#else
       lds_leaf<K>(s_base, leaf(q), a);
       lds_leaf<K>(s_base, leaf(q + 16), b);
-      kslot<K>(r1[q], a, b, xa, xb, ob, q);
+#endif
+      kslotp<K>(r1[q], a, b, xa, xb, ob, q);
+#ifndef EXP_LANE_NOWO   // timing experiment: no write-outs of levels 1-5
       if (mask & (1u << q)) { stsK<K>(wp, r1[q]); wp += 4u * K; }
+#endif
     }
     uint32_t r2[8][K], r3[4][K], r4[2][K], x[K];
 #pragma unroll
     for (uint32_t q = 0; q < 8; q++) {
-      kslot<K>(r2[q], r1[q], r1[q + 8], xa, xb, ob, 16 + q);
+      kslotp<K>(r2[q], r1[q], r1[q + 8], xa, xb, ob, 16 + q);
       if (mask & (1u << (16 + q))) { stsK<K>(wp, r2[q]); wp += 4u * K; }
     }
 #pragma unroll
     for (uint32_t q = 0; q < 4; q++) {
-      kslot<K>(r3[q], r2[q], r2[q + 4], xa, xb, ob, 24 + q);
+      kslotp<K>(r3[q], r2[q], r2[q + 4], xa, xb, ob, 24 + q);
       if (mask & (1u << (24 + q))) { stsK<K>(wp, r3[q]); wp += 4u * K; }
     }
 #pragma unroll
     for (uint32_t q = 0; q < 2; q++) {
-      kslot<K>(r4[q], r3[q], r3[q + 2], xa, xb, ob, 28 + q);
+      kslotp<K>(r4[q], r3[q], r3[q + 2], xa, xb, ob, 28 + q);
       if (mask & (1u << (28 + q))) { stsK<K>(wp, r4[q]); wp += 4u * K; }
     }
-    kslot<K>(x, r4[0], r4[1], xa, xb, ob, 30);
+    kslotp<K>(x, r4[0], r4[1], xa, xb, ob, 30);
     if (mask & (1u << 30)) stsK<K>(wp, x);
     // levels 6-10 across the warp: slot q of a level lives in lane q
     const uint32_t wxa = R.wc.x, wxb = R.wc.y, wob = R.wc.z, wmask = R.wc.w;
     const uint32_t offs[5] = {0, 16, 24, 28, 30};
+#ifndef EXP_LANE_NOWARP   // timing experiment: no levels 6-10
 #pragma unroll
     for (uint32_t k = 0; k < 5; k++) {
       const uint32_t half = 16u >> k;
@@ -154,6 +183,7 @@ __device__ __forceinline__ void exec_lane_layer(const LaneRegs& R, uint32_t s_ba
       kslot<K>(x, x, y, wxa, wxb, wob, b);
       if (lane < half) lane_woK<K>(s_base, wmask, R.wbase, b, x);
     }
+#endif
     if (uses_top && lane == 0) {
 #pragma unroll
       for (int j = 0; j < K; j++) topv[warp * K + j] = x[j];
@@ -196,8 +226,8 @@ __device__ __forceinline__ void top_lane_layer(uint32_t topc, uint32_t topwo, ui
 // One work item: partition p for the 32-stream groups g0 .. g0+ng-1 (ng <= K;
 // groups ng..K-1 of the vectors are padding and never committed).
 template <int K>
-__device__ void run_lane_partition(const KParams& kp, ProgSrc& ps, uint32_t* S, uint32_t* ramp, uint32_t* topv,
-                                   uint32_t p, uint32_t g0, uint32_t ng, uint32_t c, uint32_t cur, uint32_t nxt,
+__device__ void run_lane_partition(const KParams& kp, uint32_t* S, uint32_t* ramp, uint32_t* topv, uint32_t p,
+                                   uint32_t g0, uint32_t ng, uint32_t c, uint32_t cur, uint32_t nxt,
                                    unsigned long long* pacc) {
   const uint32_t tid = threadIdx.x;
   // GEM_F_PROFILE: thread 0 accumulates per-phase clocks over the CTA's items
@@ -212,82 +242,80 @@ __device__ void run_lane_partition(const KParams& kp, ProgSrc& ps, uint32_t* S, 
   const uint32_t s_base = smem_u32(S);
   const LaneIdx X{kp.n_groups};
   const uint32_t* gprog = kp.lprog + __ldg(kp.parts + p * GP_WORDS + GP_LANE_OFF);
-  uint32_t next_chunk = prologue_count_lane(kp, ps, p), next_off = 0;
-  next_off = __ldg(kp.parts + p * GP_WORDS + GP_LANE_CHUNK0);
-  if (next_chunk > 1) next_off += __ldg(kp.parts + p * GP_WORDS + GP_LANE_CHUNK1);
-  if (next_chunk > 2) next_off += __ldg(kp.parts + p * GP_WORDS + GP_LANE_CHUNK2);
-  const uint32_t* C0 = ring_wait(ps);
-  const uint4 h0 = *reinterpret_cast<const uint4*>(C0);
-  const uint4 h1 = *(reinterpret_cast<const uint4*>(C0) + 1);
-  const uint4 h2 = *(reinterpret_cast<const uint4*>(C0) + 2);
+  const uint4 h0 = __ldg(reinterpret_cast<const uint4*>(gprog));
+  const uint4 h1 = __ldg(reinterpret_cast<const uint4*>(gprog) + 1);
+  const uint4 h2 = __ldg(reinterpret_cast<const uint4*>(gprog) + 2);
   const uint32_t n_gread = h0.y, n_layers = h0.z, n_out = h0.w;
+  const uint32_t n_ram = h1.x, off_gread = h1.z, off_layers = h1.w;
+  const uint32_t off_out = h2.x, off_ram = h2.y;
+  // layer 0's records first: independent of S, their latency overlaps the port loads
+  const uint32_t* L = gprog + off_layers;
+  LaneRegs R;
+  if (n_layers) load_lane_layer(L, R);
   if (pacc && tid == 0 && h0.x == 0u) pacc[7]++;   // (keeps the header read before the stamp)
   phase(0);
-  const uint32_t n_ram = h1.x, off_gread = h1.z;
-  const uint32_t off_out = h2.x, off_ram = h2.y, off_chunks = h2.z, n_chunks = h2.w;
-  for (uint32_t k = tid; k < n_chunks; k += GEM_THREADS) ps.ctab[k] = C0[off_chunks + k];
-  // chunk 0 = header + chunk table; the gread list (after the last chunk) is
-  // read straight from global memory
-  auto refill = [&]() {
-    while (next_chunk < n_chunks && ps.seq_issue - ps.seq_free < ps.R) {
-      const uint32_t words = ps.ctab[next_chunk];
-      ring_issue(ps, gprog + next_off, words);
-      next_off += words;
-      next_chunk++;
-    }
-  };
-  // ---- a2: input ports (once per cycle) for the groups of the item
-  // loads of 4 (entry, group) pairs per thread are issued before their stores
-  const uint2* gr = reinterpret_cast<const uint2*>(gprog + off_gread);
-  const uint32_t n_gr = n_gread * ng;
-  for (uint32_t k0 = 0; k0 < n_gr; k0 += 4 * GEM_THREADS) {
-    uint32_t v[4], dst[4];
+  // ---- a2: input ports (once per cycle) for the groups of the item.
+  // Entry k (one u32 gid per entry) goes to lane word k + 1.  A thread takes 4
+  // consecutive entries per uint4 and up to 16 per pass: all entry loads, then
+  // all value loads, then the stores (two L2 round trips per pass, not per entry)
+  const uint4* gr4 = reinterpret_cast<const uint4*>(gprog + off_gread);
+  for (uint32_t j = 0; j < ng; j++) {
+    const uint32_t g = g0 + j;
+    const uint32_t* bpi = kp.pi_lane + X.q(kp.in_base + c, kp.pi_words * 32, 0, g);
+    const uint32_t* bq = kp.q + X.q(cur, kp.q_words * 32, 0, g);
+    const uint32_t* brd = kp.rd + X.q(cur, kp.n_rams * 32, 0, g);
+    const uint32_t* bcut = kp.cut + X.q(0, kp.cut_words * 32, 0, g);
+    for (uint32_t kb = 0; kb < n_gread; kb += 16 * GEM_THREADS) {
+      uint4 e[4];
 #pragma unroll
-    for (uint32_t u = 0; u < 4; u++) {
-      const uint32_t k = k0 + u * GEM_THREADS + tid;
-      dst[u] = ~0u;
-      if (k < n_gr) {
-        const uint32_t j = k / n_gread, g = g0 + j;
-        const uint2 e = __ldg(gr + (k - j * n_gread));
-        const uint32_t reg = e.x >> 24, b = e.x & 0xFFFFFFu;
-        const uint32_t* a;
-        if (reg == GEM_R_PI) a = kp.pi_lane + X.q(kp.in_base + c, kp.pi_words * 32, b, g);
-        else if (reg == GEM_R_Q) a = kp.q + X.q(cur, kp.q_words * 32, b, g);
-        else if (reg == GEM_R_RD) a = kp.rd + X.q(cur, kp.n_rams * 32, b, g);
-        else a = kp.cut + X.q(0, kp.cut_words * 32, b, g);
-        v[u] = __ldcg(a);
-        dst[u] = e.y * K + j;
+      for (uint32_t u = 0; u < 4; u++) {
+        const uint32_t q4 = kb / 4 + u * GEM_THREADS + tid;
+        e[u] = 4 * q4 < n_gread ? __ldg(gr4 + q4) : make_uint4(0, 0, 0, 0);
+      }
+      uint32_t v[16];
+#pragma unroll
+      for (uint32_t u = 0; u < 4; u++) {
+        const uint32_t ev[4] = {e[u].x, e[u].y, e[u].z, e[u].w};
+        const uint32_t k4 = kb + 4 * (u * GEM_THREADS + tid);
+#pragma unroll
+        for (uint32_t h = 0; h < 4; h++) {
+          const uint32_t reg = ev[h] >> 24, b = ev[h] & 0xFFFFFFu;
+          const uint32_t* base = reg == GEM_R_PI ? bpi : reg == GEM_R_Q ? bq : reg == GEM_R_RD ? brd : bcut;
+          v[4 * u + h] = k4 + h < n_gread ? __ldcg(base + b) : 0u;
+        }
+      }
+#pragma unroll
+      for (uint32_t u = 0; u < 4; u++) {
+        const uint32_t k4 = kb + 4 * (u * GEM_THREADS + tid);
+#pragma unroll
+        for (uint32_t h = 0; h < 4; h++)
+          if (k4 + h < n_gread) sts(s_base + 4u * ((k4 + h + 1) * K + j), v[4 * u + h]);
       }
     }
-#pragma unroll
-    for (uint32_t u = 0; u < 4; u++)
-      if (dst[u] != ~0u) sts(s_base + 4u * dst[u], v[u]);
   }
   if (tid < K) S[tid] = 0u;   // lane word 0 = constant 0 for every group
   phase(1);
-  LaneRegs R;
-  if (n_layers) load_lane_layer(ring_wait(ps), R);
   __syncthreads();
   phase(2);
-  ps.seq_free = ps.seq_wait;
-  refill();
   for (uint32_t l = 0; l < n_layers; l++) {
     exec_lane_layer<K>(R, s_base, topv, 1);
+#ifdef EXP_LANE_NOTOP
+    const bool ptop = false;
+#else
     const bool ptop = (R.flags & GEM_LF_USES_TOP) != 0;
+#endif
     const uint32_t ptopc = R.topc, ptopwo = R.topwo;
-    if (l + 1 < n_layers) load_lane_layer(ring_wait(ps), R);
+    L += R.size;
+    if (l + 1 < n_layers) load_lane_layer(L, R);
     if (ptop && (threadIdx.x >> 5) == 0) top_lane_layer<K>(ptopc, ptopwo, s_base, topv, 1);
     __syncthreads();
-    ps.seq_free = ps.seq_wait;
-    refill();
   }
   phase(3);
   // ---- a6: endpoint commit: one lane word per endpoint bit
-  const uint32_t* od = ring_wait(ps);
-  const uint2* oe = reinterpret_cast<const uint2*>(od);
+  const uint2* oe = reinterpret_cast<const uint2*>(gprog + off_out);
   for (uint32_t jj = tid; jj < n_out * ng; jj += GEM_THREADS) {
     const uint32_t j = jj / n_out, o = jj - j * n_out, g = g0 + j;
-    const uint2 e = oe[o];
+    const uint2 e = __ldg(oe + o);
     const uint32_t v = lds(s_base + 4u * ((e.y & 0xFFFFu) * K + j)) ^ ((e.y >> 31) ? 0xFFFFFFFFu : 0u);
     const uint32_t reg = e.x >> 24, b = e.x & 0xFFFFFFu;
     if (reg == GEM_R_Q) __stcg(kp.q + X.q(nxt, kp.q_words * 32, b, g), v);
@@ -298,12 +326,12 @@ __device__ void run_lane_partition(const KParams& kp, ProgSrc& ps, uint32_t* S, 
   // ---- a7: RAM blocks: one warp per RAM, lane s = stream 32g+s (read-first, per-bit write)
   if (n_ram) {
     __syncthreads();
-    const uint32_t* rr = od + (off_ram - off_out);
+    const uint32_t* rr = gprog + off_ram;
     const uint32_t lane = tid & 31;
     for (uint32_t jr = tid >> 5; jr < n_ram * ng; jr += GEM_WARPS) {
       const uint32_t j = jr / n_ram, r = jr - j * n_ram, g = g0 + j;
       const uint32_t nvalid = min(32u, kp.n_streams - 32u * g);
-      const uint32_t id = rr[4 * r];
+      const uint32_t id = __ldg(rr + 4 * r);
       const uint32_t* rp = ramp + j * kp.ramp_words + r * 128;
       uint32_t ra = 0, wa = 0, wd = 0, be = 0;
 #pragma unroll
@@ -333,7 +361,6 @@ __device__ void run_lane_partition(const KParams& kp, ProgSrc& ps, uint32_t* S, 
   }
   __syncthreads();
   phase(4);
-  ps.seq_free = ps.seq_issue;
 }
 
 // Parity instruments in lane mode: flop digest / trace from the lane words.
@@ -362,43 +389,19 @@ __device__ void record_state_lane(const KParams& kp, uint32_t c, uint32_t buf) {
 template <int K>
 __global__ void __launch_bounds__(GEM_THREADS, 2) gem_lane_kernel(const KParams kp) {
   extern __shared__ __align__(16) uint32_t smem[];
-  // layout: S[lane_words][K] | area (ring) | ctab[256] | ramp[K][ram_words] | topv[8][K] | mbar[8 x u64]
+  // layout: S[lane_words][K] | ramp[K][ramp_words] | topv[16][K]  (no program ring:
+  // records are loaded from global memory into registers one layer ahead)
   uint32_t* S = smem;                                   // [lane word][group] interleaved
-  uint32_t* area = S + kp.group * kp.state_words;
-  uint32_t* ctab = area + kp.area_words;
-  uint32_t* ramp = ctab + GEM_MAX_CHUNKS;               // [group][ramp_words]
+  uint32_t* ramp = S + kp.group * kp.state_words;       // [group][ramp_words]
   uint32_t* topv = ramp + kp.group * kp.ramp_words;     // [group][16]
-  uint64_t* mbar = reinterpret_cast<uint64_t*>(topv + 16 * kp.group);
   const uint32_t tid = threadIdx.x;
   const uint32_t G = gridDim.x, B = blockIdx.x;
   auto wl_begin = [&](uint32_t s) { return __ldg(kp.wl_off + s * (G + 1) + B); };
   auto wl_end = [&](uint32_t s) { return __ldg(kp.wl_off + s * (G + 1) + B + 1); };
   for (uint32_t k = tid; k < 16 * kp.group; k += GEM_THREADS) topv[k] = 0u;
-  if (tid == 0) {
-    for (uint32_t k = 0; k <= GEM_RING_MAX; k++) mbar_init(mbar + k, 1);
-    fence_mbar_init();
-  }
   __syncthreads();
-  ProgSrc ps;
-  ps.mbar = mbar;
-  ps.area = area;
-  ps.ctab = ctab;
-  ps.resident = false;
-  ps.n_res = 0;
-  ps.res_p = nullptr;
-  ps.res_off = nullptr;
-  ps.slot_words = kp.slot_words;
-  ps.R = kp.ring_slots;
-  ps.seq_issue = ps.seq_wait = ps.seq_free = 0;
-  auto first_item = [&]() -> uint32_t {
-    for (uint32_t s = 0; s < kp.n_stages; s++)
-      if (wl_begin(s) < wl_end(s)) return wl_begin(s);
-    return ~0u;
-  };
-  if (kp.ncycles) {
-    const uint32_t k0 = first_item();
-    if (k0 != ~0u) issue_prologue_lane(kp, ps, __ldg(&kp.wl_items[k0].x));
-  }
+  const bool dyn = kp.dyn_units != nullptr;
+  __shared__ uint32_t s_next[2];   // dynamic mode: next unit (double-buffered by unit parity)
   unsigned long long bar_target = 0;
   const bool instr = (kp.flags & (GEM_F_TRACE_STATE | GEM_F_DIGEST)) != 0;
   __shared__ unsigned long long pacc[8];   // GEM_F_PROFILE phase sums (thread 0)
@@ -410,22 +413,35 @@ __global__ void __launch_bounds__(GEM_THREADS, 2) gem_lane_kernel(const KParams 
       for (int k = 0; k < 8; k++) pacc[k] = 0ull;
     PROF(0);
     if (instr && c > 0) record_state_lane(kp, c - 1, cur);
-    for (uint32_t s = 0; s < kp.n_stages; s++) {
-      const uint32_t kb = wl_begin(s), ke = wl_end(s);
-      for (uint32_t k = kb; k < ke; k++) {
-        const uint2 it = __ldg(&kp.wl_items[k]);
-        const uint32_t g0 = it.y >> 5;
-        run_lane_partition<K>(kp, ps, S, ramp, topv, it.x, g0, min((uint32_t)K, kp.n_groups - g0), c, cur, nxt,
-                              prof_on ? pacc : nullptr);
-        uint32_t nk = ~0u;
-        if (k + 1 < ke) nk = k + 1;
-        for (uint32_t s2 = s + 1; nk == ~0u && s2 < kp.n_stages; s2++)
-          if (wl_begin(s2) < wl_end(s2)) nk = wl_begin(s2);
-        if (nk == ~0u && c + 1 < kp.ncycles) nk = first_item();
-        if (nk != ~0u) issue_prologue_lane(kp, ps, __ldg(&kp.wl_items[nk].x));
+    if (dyn) {
+      // counter of cycle c+1 was last used in cycle c-1 (all CTAs are past its barrier)
+      if (B == 0 && tid == 0) atomicExch(kp.dyn_ctr + ((c + 1) & 1u), 0u);
+      uint32_t u = B, par = 0;
+      while (u < kp.n_units) {
+        if (tid == 0) s_next[par] = atomicAdd(kp.dyn_ctr + (c & 1u), 1u) + G;
+        const uint4 U = __ldg(&kp.dyn_units[u]);
+        for (uint32_t r = 0; r < U.z; r++) {
+          const uint32_t g0 = (U.y >> 5) + r * K;
+          run_lane_partition<K>(kp, S, ramp, topv, U.x, g0, min((uint32_t)K, kp.n_groups - g0), c, cur, nxt,
+                                prof_on ? pacc : nullptr);
+        }
+        u = s_next[par];   // written before the item's first barrier
+        par ^= 1u;
       }
-      if (s == 0) PROF(4);
+      PROF(4);
       grid_sync(kp, bar_target);
+    } else {
+      for (uint32_t s = 0; s < kp.n_stages; s++) {
+        const uint32_t kb = wl_begin(s), ke = wl_end(s);
+        for (uint32_t k = kb; k < ke; k++) {
+          const uint2 it = __ldg(&kp.wl_items[k]);
+          const uint32_t g0 = it.y >> 5;
+          run_lane_partition<K>(kp, S, ramp, topv, it.x, g0, min((uint32_t)K, kp.n_groups - g0), c, cur, nxt,
+                                prof_on ? pacc : nullptr);
+        }
+        if (s == 0) PROF(4);
+        grid_sync(kp, bar_target);
+      }
     }
     PROF(5);
     if (prof_on && threadIdx.x == 0)

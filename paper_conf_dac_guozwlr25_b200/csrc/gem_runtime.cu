@@ -75,6 +75,12 @@ struct KParams {
   // (act_words >= max n_gread) and {evaluated, skipped} partition-cycle counters
   unsigned long long* act_cnt;
   uint32_t act_words;
+  // lane mode, one stage: dynamic work distribution.  Units {partition, first
+  // stream, items, 0} in LPT order; CTA b starts every cycle with unit b and
+  // then takes tickets from dyn_ctr[cycle & 1] (+ grid).
+  const uint4* __restrict__ dyn_units;
+  uint32_t n_units;
+  uint32_t* dyn_ctr;
 };
 #ifdef GEM_FINE_PROF
 // sub-stamps inside exec_layer: fl = layer index when stamping, >= 32 otherwise;
@@ -999,23 +1005,6 @@ __global__ void __launch_bounds__(GEM_THREADS, 2) gem_step_kernel(const KParams 
 }
 
 // ---- lane-mode prologue helpers (same protocol as issue_prologue, lane fields)
-__device__ __forceinline__ uint32_t prologue_count_lane(const KParams& kp, const ProgSrc& ps, uint32_t p) {
-  const uint32_t nch = __ldg(kp.parts + p * GP_WORDS + GP_N_LAYERS) + 2;
-  return min(min(ps.R, 3u), nch);
-}
-__device__ __forceinline__ void issue_prologue_lane(const KParams& kp, ProgSrc& ps, uint32_t p) {
-  const uint32_t* g = kp.lprog + __ldg(kp.parts + p * GP_WORDS + GP_LANE_OFF);
-  const uint32_t k = prologue_count_lane(kp, ps, p);
-  const uint32_t sz[3] = {__ldg(kp.parts + p * GP_WORDS + GP_LANE_CHUNK0),
-                          __ldg(kp.parts + p * GP_WORDS + GP_LANE_CHUNK1),
-                          __ldg(kp.parts + p * GP_WORDS + GP_LANE_CHUNK2)};
-  uint32_t off = 0;
-  for (uint32_t i = 0; i < k; i++) {
-    ring_issue(ps, g + off, sz[i]);
-    off += sz[i];
-  }
-}
-
 #include "gem_lanes.cuh"
 
 
@@ -1132,6 +1121,8 @@ struct gem_sim {
   uint32_t area_words = 0, slot_words = 0, ring_slots = 0, resident = 0, group = 1;
   // lane mode (stream-sliced, >= 32 streams and a blob with lane programs)
   uint32_t act_words = 0;                      // GEM_F_ACTIVITY: max n_gread over partitions
+  uint4* d_dyn_units = nullptr;                // lane mode dynamic work units
+  uint32_t n_units = 0, *d_dyn_ctr = nullptr;
   unsigned long long* d_act = nullptr;         // {evaluated, skipped}
   uint32_t lanes = 0, n_groups = 0, lane_words = 0, lane_max_chunk = 0, ramp_words = 0, lane_groups = 1;
   uint32_t *d_lprog = nullptr, *d_pi_lane = nullptr, *d_po_lane = nullptr;
@@ -1386,36 +1377,33 @@ static int plan_launch_lanes(gem_sim* sim, uint32_t grid_limit) {
   CK(cudaDeviceGetAttribute(&per_sm, cudaDevAttrMaxSharedMemoryPerMultiprocessor, sim->device));
   if (!coop) return fail(GEM_E_UNSUPPORTED, "device lacks cooperative launch");
   sim->sm_count = (uint32_t)sms;
-  const uint32_t slot = (sim->lane_max_chunk + 3u) & ~3u;
   const char* ge = getenv("GEM_LANE_GROUPS");
   const char* be = getenv("GEM_LANE_BPS");
   const uint32_t want_gl = std::min<uint32_t>(ge ? (uint32_t)atoi(ge) : 4, 4);
   // prefer 2 CTAs per SM (16 warps to hide latency), then as many 32-stream
-  // groups per work item as fit beside a >= 2-slot ring
-  uint32_t bps = 0, gl = 0, budget = 0;
+  // groups per work item as fit (shared memory holds only the lane state:
+  // records stream from global memory into registers)
+  uint32_t bps = 0, gl = 0;
   for (uint32_t b = 2; b >= 1 && !bps; b--) {
     if (be && (uint32_t)atoi(be) != b) continue;
     const uint32_t bud = (uint32_t)std::min<int64_t>(optin, per_sm / (int64_t)b - 1024);
     for (uint32_t k = std::max<uint32_t>(1, std::min(want_gl, sim->n_groups)); k >= 1; k--) {
       if (k == 3) continue;   // the kernel is instantiated for K = 1, 2, 4 interleaved groups
-      const uint64_t words = (uint64_t)k * (sim->lane_words + sim->ramp_words + 16) + GEM_MAX_CHUNKS + 16 + 2 * slot;
-      if (words * 4 <= bud) { bps = b; gl = k; budget = bud; break; }
+      const uint64_t words = (uint64_t)k * (sim->lane_words + sim->ramp_words + 16);
+      if (words * 4 <= bud) { bps = b; gl = k; break; }
     }
   }
-  if (!bps) return fail(GEM_E_UNSUPPORTED, "lane state + 2 ring slots exceed shared memory");
+  if (!bps) return fail(GEM_E_UNSUPPORTED, "lane state exceeds shared memory");
   sim->lane_groups = gl;
   sim->group = 32 * gl;    // streams per work item
   sim->max_items = 0;
   for (uint32_t s = 0; s < sim->n_stages; s++)
     sim->max_items = std::max(sim->max_items, (sim->h_stage[s + 1] - sim->h_stage[s]) * ((sim->n_groups + gl - 1) / gl));
-  const uint32_t fixed_words = gl * (sim->lane_words + sim->ramp_words + 16) + GEM_MAX_CHUNKS + 16;
-  const uint32_t area = budget / 4 - fixed_words;
-  uint32_t ring = std::min<uint32_t>(GEM_RING_MAX, area / std::max<uint32_t>(slot, 4));
-  ring = ring >= 4 ? 4 : 2;
+  const uint32_t fixed_words = gl * (sim->lane_words + sim->ramp_words + 16);
   uint32_t grid = std::max<uint32_t>(1, std::min<uint32_t>(sim->max_items, bps * (uint32_t)sms));
   if (grid_limit) grid = std::max<uint32_t>(1, std::min(grid, grid_limit));
   grid = std::min<uint32_t>(grid, GEM_BAR_MAX_CTAS);
-  const uint32_t smem = (fixed_words + ring * slot) * 4;
+  const uint32_t smem = fixed_words * 4;
   const void* lk = lane_kernel_for(gl);
   CK(cudaFuncSetAttribute(lk, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem));
   int occ = 0;
@@ -1424,11 +1412,39 @@ static int plan_launch_lanes(gem_sim* sim, uint32_t grid_limit) {
   std::vector<uint32_t> off;
   std::vector<uint2> items;
   build_worklists(sim, grid, off, items);
+  // one stage: dynamic distribution of LPT-ordered units (GEM_LANE_DYN=0: static lists)
+  const char* de = getenv("GEM_LANE_DYN");
+  if (sim->n_stages == 1 && !(de && de[0] == '0')) {
+    // unit = `run` consecutive items of one partition (they share its records
+    // in L2 / L1); as long as there are >= 8 units per CTA
+    const uint32_t np1 = sim->h_stage[1] - sim->h_stage[0];
+    const uint64_t items1 = (uint64_t)np1 * ((sim->n_streams + sim->group - 1) / sim->group);
+    uint32_t run = (uint32_t)std::max<uint64_t>(1, std::min<uint64_t>(4, items1 / (8ull * grid)));
+    if (getenv("GEM_LANE_RUN")) run = (uint32_t)std::max(1, atoi(getenv("GEM_LANE_RUN")));
+    std::vector<std::pair<double, uint4>> us;
+    const uint32_t np = sim->h_stage[1] - sim->h_stage[0];
+    for (uint32_t st = 0; st < sim->n_streams; st += sim->group * run)
+      for (uint32_t k = 0; k < np; k++) {
+        const uint32_t p = sim->h_stage[sim->n_stages + 1 + k];
+        const uint32_t n_items = std::min(run, (sim->n_streams - st + sim->group - 1) / sim->group);
+        us.push_back({(double)sim->h_parts[(size_t)p * GP_WORDS + GP_COST] * n_items, make_uint4(p, st, n_items, 0)});
+      }
+    std::stable_sort(us.begin(), us.end(), [](const std::pair<double, uint4>& x, const std::pair<double, uint4>& y) {
+      return x.first > y.first;
+    });
+    std::vector<uint4> hu;
+    for (auto& u : us) hu.push_back(u.second);
+    sim->n_units = (uint32_t)hu.size();
+    CK(dalloc(&sim->d_dyn_units, hu.size() * 16));
+    CK(cudaMemcpy(sim->d_dyn_units, hu.data(), hu.size() * 16, cudaMemcpyHostToDevice));
+    CK(dalloc(&sim->d_dyn_ctr, 16));
+    grid = std::min<uint32_t>(grid, sim->n_units);
+  }
   sim->blocks_per_sm = bps;
   sim->grid = grid;
-  sim->area_words = ring * slot;
-  sim->ring_slots = ring;
-  sim->slot_words = slot;
+  sim->area_words = 0;
+  sim->ring_slots = 0;
+  sim->slot_words = 0;
   sim->resident = 0;
   sim->smem_bytes = smem;
   CK(dalloc(&sim->d_wl_off, off.size() * 4));
@@ -1660,6 +1676,10 @@ int gem_step(gem_sim* sim, uint64_t ncycles) {
   kp.group = sim->group;
   kp.wl_items = sim->d_wl_items;
   kp.act_cnt = sim->d_act;
+  kp.dyn_units = sim->d_dyn_units;
+  kp.n_units = sim->n_units;
+  kp.dyn_ctr = sim->d_dyn_ctr;
+  if (sim->d_dyn_ctr) CK(cudaMemsetAsync(sim->d_dyn_ctr, 0, 16, sim->stream));
   kp.act_words = sim->lanes ? 0u : sim->act_words;
   if (sim->flags & GEM_F_PROFILE) {
     const uint32_t pc = (uint32_t)std::min<uint64_t>(ncycles, 256);
@@ -1922,7 +1942,8 @@ void gem_free(gem_sim* sim) {
                   (void*)sim->d_cut, (void*)sim->d_mem, (void*)sim->d_pi, (void*)sim->d_po, (void*)sim->d_qtrace,
                   (void*)sim->d_scratch, (void*)sim->d_digest, (void*)sim->d_bar, (void*)sim->d_err,
                   (void*)sim->d_prof, (void*)sim->d_wl_off, (void*)sim->d_wl_items, (void*)sim->d_lprog,
-                  (void*)sim->d_pi_lane, (void*)sim->d_po_lane, (void*)sim->d_act})
+                  (void*)sim->d_pi_lane, (void*)sim->d_po_lane, (void*)sim->d_act,
+                  (void*)sim->d_dyn_units, (void*)sim->d_dyn_ctr})
     if (p) cudaFree(p);
   if (sim->ev0) cudaEventDestroy(sim->ev0);
   if (sim->ev1) cudaEventDestroy(sim->ev1);

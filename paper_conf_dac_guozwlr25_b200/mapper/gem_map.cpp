@@ -68,6 +68,7 @@ struct Options {
   double refine_ratio = 1.35;  // split partitions costing more than this x the median
   int max_parts = 280;      // refinement stops growing the partition count here
   int lanes = 0;            // also emit stream-sliced lane programs (batched streams)
+  int lane_words = 16383;   // cap on a lane program's state words (larger partitions are split)
   int banks = 1;            // bank-conflict-aware renaming of the state words (rename_state_words)
   int verbose = 0;
   int max_state_words = GEM_MAX_STATE_WORDS;
@@ -101,6 +102,7 @@ static Options parse_opts(const char* s) {
     else if (k == "refine_ratio") o.refine_ratio = std::stod(v);
     else if (k == "max_parts") o.max_parts = std::stoi(v);
     else if (k == "lanes") o.lanes = std::stoi(v);
+    else if (k == "lane_words") o.lane_words = std::min(16383, std::stoi(v));
     else if (k == "banks") o.banks = std::stoi(v);
     else throw std::runtime_error("unknown option " + k);
   }
@@ -1125,7 +1127,7 @@ struct Mapper {
     word[0] = 0;   // local node 0 is the constant
     // free-interval allocator (first fit, coalescing); word 0 reserved
     std::map<uint32_t, uint32_t> freeiv;   // start -> length
-    const uint32_t kMaxWords = 16383;   // leaf entries hold byte offsets (word * 4) in 16 bits
+    const uint32_t kMaxWords = (uint32_t)opt.lane_words;   // leaf entries hold byte offsets (word * 4) in 16 bits
     freeiv[1] = kMaxWords - 1;
     uint32_t max_word = 1;
     std::vector<std::vector<uint32_t>> die(L + 1);
@@ -1231,7 +1233,15 @@ struct Mapper {
         pr.push_back(0); pr.push_back(0); pr.push_back(0);
         for (uint32_t ln = 0; ln < 32; ln++) {
           uint32_t t = w * 32 + ln;
-          pr.push_back(LL.cth[3 * t]); pr.push_back(LL.cth[3 * t + 1]); pr.push_back(LL.cth[3 * t + 2]);
+          // byte-spread constants (gem_isa.h): slot bit b -> bit 8*(b&3) + 7 - (b>>2), so the
+          // kernel makes each mask with one shift per 4 slots and one PRMT sign-replicate
+          auto spread = [](uint32_t c) {
+            uint32_t r = 0;
+            for (uint32_t q = 0; q < 31; q++) r |= ((c >> q) & 1u) << (8 * (q & 3) + 7 - (q >> 2));
+            return r;
+          };
+          pr.push_back(spread(LL.cth[3 * t])); pr.push_back(spread(LL.cth[3 * t + 1]));
+          pr.push_back(spread(LL.cth[3 * t + 2]));
           pr.push_back(th[l][t].mask);
         }
         for (uint32_t g = 0; g < 4; g++)
@@ -1269,8 +1279,10 @@ struct Mapper {
     uint32_t ng = 0;
     for (uint32_t x : srcs) {
       uint32_t gb = G.gbit[cid[x]];
+      // one word per entry: the destination lane word is implicit (entry k ->
+      // lane word k + 1: the sources took the first words, in this order)
+      if (lw(x) != ng + 1) throw std::runtime_error("lane: source words not consecutive");
       pr.push_back(((gb >> 27) << 24) | (((gb >> 5) & 0x3FFFFF) * 32 + (gb & 31)));
-      pr.push_back(lw(x));
       ng++;
     }
     pr[LPH_N_GREAD] = ng;

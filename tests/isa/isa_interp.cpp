@@ -196,7 +196,7 @@ int run_lane_part(Interp& I, LaneSim& Ls, uint32_t p, const uint32_t* pi_lane /*
   std::vector<uint32_t> S(pr[LPH_LANE_WORDS] + 1, 0);
   const uint32_t* gr = pr + pr[LPH_OFF_GREAD];
   for (uint32_t k = 0; k < pr[LPH_N_GREAD]; k++) {
-    uint32_t gid = gr[2 * k], dst = gr[2 * k + 1];
+    uint32_t gid = gr[k], dst = k + 1;
     uint32_t reg = gid >> 24, b = gid & 0xFFFFFF, v;
     if (reg == GEM_R_PI) v = pi_lane[b];
     else if (reg == GEM_R_Q) v = Ls.Q[cur][b];
@@ -260,7 +260,15 @@ int run_lane_part(Interp& I, LaneSim& Ls, uint32_t p, const uint32_t* pi_lane /*
       for (uint32_t id = 0; id < (8192u >> k); id++) {
         uint32_t ca = (id / gwid) * 2 * gwid + id % gwid, cb = ca + gwid;
         uint32_t xa, xb, ob, b = sbit(k, id);
-        if (k <= 5) { uint32_t t = id / gwid; xa = lane_c[t][0]; xb = lane_c[t][1]; ob = lane_c[t][2]; }
+        if (k <= 5) {
+          // lane-mode levels 1-5: slot bit b sits at bit 8*(b&3) + 7 - (b>>2) (gem_isa.h)
+          auto un = [](uint32_t c) {
+            uint32_t r = 0;
+            for (uint32_t q = 0; q < 31; q++) r |= ((c >> (8 * (q & 3) + 7 - (q >> 2))) & 1u) << q;
+            return r;
+          };
+          uint32_t t = id / gwid; xa = un(lane_c[t][0]); xb = un(lane_c[t][1]); ob = un(lane_c[t][2]);
+        }
         else if (k <= 10) { uint32_t wq = id / gwid; xa = warp_c[wq][0]; xb = warp_c[wq][1]; ob = warp_c[wq][2]; }
         else { xa = topc & 0xFF; xb = (topc >> 8) & 0xFF; ob = (topc >> 16) & 0xFF; }
         uint32_t XA = ((xa >> b) & 1u) ? ~0u : 0u, XB = ((xb >> b) & 1u) ? ~0u : 0u, OB = ((ob >> b) & 1u) ? ~0u : 0u;
