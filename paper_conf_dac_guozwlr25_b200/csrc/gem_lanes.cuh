@@ -259,38 +259,54 @@ __device__ void run_lane_partition(const KParams& kp, uint32_t* S, uint32_t* ram
   // consecutive entries per uint4 and up to 16 per pass: all entry loads, then
   // all value loads, then the stores (two L2 round trips per pass, not per entry)
   const uint4* gr4 = reinterpret_cast<const uint4*>(gprog + off_gread);
-  for (uint32_t j = 0; j < ng; j++) {
-    const uint32_t g = g0 + j;
-    const uint32_t* bpi = kp.pi_lane + X.q(kp.in_base + c, kp.pi_words * 32, 0, g);
-    const uint32_t* bq = kp.q + X.q(cur, kp.q_words * 32, 0, g);
-    const uint32_t* brd = kp.rd + X.q(cur, kp.n_rams * 32, 0, g);
-    const uint32_t* bcut = kp.cut + X.q(0, kp.cut_words * 32, 0, g);
-    for (uint32_t kb = 0; kb < n_gread; kb += 16 * GEM_THREADS) {
-      uint4 e[4];
+  const uint32_t* bpi[K];
+  const uint32_t* bq[K];
+  const uint32_t* brd[K];
+  const uint32_t* bcut[K];
 #pragma unroll
-      for (uint32_t u = 0; u < 4; u++) {
-        const uint32_t q4 = kb / 4 + u * GEM_THREADS + tid;
-        e[u] = 4 * q4 < n_gread ? __ldg(gr4 + q4) : make_uint4(0, 0, 0, 0);
-      }
-      uint32_t v[16];
+  for (int j = 0; j < K; j++) {
+    const uint32_t g = g0 + min((uint32_t)j, ng - 1u);
+    bpi[j] = kp.pi_lane + X.q(kp.in_base + c, kp.pi_words * 32, 0, g);
+    bq[j] = kp.q + X.q(cur, kp.q_words * 32, 0, g);
+    brd[j] = kp.rd + X.q(cur, kp.n_rams * 32, 0, g);
+    bcut[j] = kp.cut + X.q(0, kp.cut_words * 32, 0, g);
+  }
+  constexpr uint32_t NU = K >= 4 ? 1u : 4u / K;   // uint4 entry groups per thread and pass (K * 4 * NU loads in flight)
+  for (uint32_t kb = 0; kb < n_gread; kb += 4 * NU * GEM_THREADS) {
+    uint4 e[NU];
 #pragma unroll
-      for (uint32_t u = 0; u < 4; u++) {
-        const uint32_t ev[4] = {e[u].x, e[u].y, e[u].z, e[u].w};
-        const uint32_t k4 = kb + 4 * (u * GEM_THREADS + tid);
+    for (uint32_t u = 0; u < NU; u++) {
+      const uint32_t q4 = kb / 4 + u * GEM_THREADS + tid;
+      e[u] = 4 * q4 < n_gread ? __ldg(gr4 + q4) : make_uint4(0, 0, 0, 0);
+    }
+    // the K groups' values of the same entries are loaded together (K * 16 in flight)
+    uint32_t v[K][4 * NU];
 #pragma unroll
-        for (uint32_t h = 0; h < 4; h++) {
-          const uint32_t reg = ev[h] >> 24, b = ev[h] & 0xFFFFFFu;
-          const uint32_t* base = reg == GEM_R_PI ? bpi : reg == GEM_R_Q ? bq : reg == GEM_R_RD ? brd : bcut;
-          v[4 * u + h] = k4 + h < n_gread ? __ldcg(base + b) : 0u;
+    for (uint32_t u = 0; u < NU; u++) {
+      const uint32_t ev[4] = {e[u].x, e[u].y, e[u].z, e[u].w};
+      const uint32_t k4 = kb + 4 * (u * GEM_THREADS + tid);
+#pragma unroll
+      for (uint32_t h = 0; h < 4; h++) {
+        const uint32_t reg = ev[h] >> 24, b = ev[h] & 0xFFFFFFu;
+        const bool ok = k4 + h < n_gread;
+#pragma unroll
+        for (int j = 0; j < K; j++) {
+          const uint32_t* base = reg == GEM_R_PI ? bpi[j] : reg == GEM_R_Q ? bq[j] : reg == GEM_R_RD ? brd[j] : bcut[j];
+          v[j][4 * u + h] = ok ? __ldcg(base + b) : 0u;
         }
       }
+    }
 #pragma unroll
-      for (uint32_t u = 0; u < 4; u++) {
-        const uint32_t k4 = kb + 4 * (u * GEM_THREADS + tid);
+    for (uint32_t u = 0; u < NU; u++) {
+      const uint32_t k4 = kb + 4 * (u * GEM_THREADS + tid);
 #pragma unroll
-        for (uint32_t h = 0; h < 4; h++)
-          if (k4 + h < n_gread) sts(s_base + 4u * ((k4 + h + 1) * K + j), v[4 * u + h]);
-      }
+      for (uint32_t h = 0; h < 4; h++)
+        if (k4 + h < n_gread) {
+          uint32_t w[K];
+#pragma unroll
+          for (int j = 0; j < K; j++) w[j] = v[j][4 * u + h];
+          stsK<K>(s_base + 4u * K * (k4 + h + 1), w);   // padding groups (j >= ng) are never committed
+        }
     }
   }
   if (tid < K) S[tid] = 0u;   // lane word 0 = constant 0 for every group
@@ -312,16 +328,33 @@ __device__ void run_lane_partition(const KParams& kp, uint32_t* S, uint32_t* ram
   }
   phase(3);
   // ---- a6: endpoint commit: one lane word per endpoint bit
+  // entries of 4 endpoints per thread are loaded before use; one LDS.K gives
+  // the source word of all K groups
   const uint2* oe = reinterpret_cast<const uint2*>(gprog + off_out);
-  for (uint32_t jj = tid; jj < n_out * ng; jj += GEM_THREADS) {
-    const uint32_t j = jj / n_out, o = jj - j * n_out, g = g0 + j;
-    const uint2 e = __ldg(oe + o);
-    const uint32_t v = lds(s_base + 4u * ((e.y & 0xFFFFu) * K + j)) ^ ((e.y >> 31) ? 0xFFFFFFFFu : 0u);
-    const uint32_t reg = e.x >> 24, b = e.x & 0xFFFFFFu;
-    if (reg == GEM_R_Q) __stcg(kp.q + X.q(nxt, kp.q_words * 32, b, g), v);
-    else if (reg == GEM_R_PO) __stcg(kp.po_lane + X.q(c, kp.po_words * 32, b, g), v);
-    else if (reg == GEM_R_CUT) __stcg(kp.cut + X.q(0, kp.cut_words * 32, b, g), v);
-    else ramp[j * kp.ramp_words + b] = v;
+  for (uint32_t o0 = 0; o0 < n_out; o0 += 4 * GEM_THREADS) {
+    uint2 e[4];
+#pragma unroll
+    for (uint32_t u = 0; u < 4; u++) {
+      const uint32_t o = o0 + u * GEM_THREADS + tid;
+      e[u] = o < n_out ? __ldg(oe + o) : make_uint2(0, 0);
+    }
+#pragma unroll
+    for (uint32_t u = 0; u < 4; u++) {
+      if (o0 + u * GEM_THREADS + tid >= n_out) continue;
+      uint32_t v[K];
+      ldsK<K>(s_base + 4u * K * (e[u].y & 0xFFFFu), v);
+      const uint32_t inv = (e[u].y >> 31) ? 0xFFFFFFFFu : 0u;
+      const uint32_t reg = e[u].x >> 24, b = e[u].x & 0xFFFFFFu;
+#pragma unroll
+      for (int j = 0; j < K; j++) {
+        if ((uint32_t)j >= ng) break;
+        const uint32_t g = g0 + j, x = v[j] ^ inv;
+        if (reg == GEM_R_Q) __stcg(kp.q + X.q(nxt, kp.q_words * 32, b, g), x);
+        else if (reg == GEM_R_PO) __stcg(kp.po_lane + X.q(c, kp.po_words * 32, b, g), x);
+        else if (reg == GEM_R_CUT) __stcg(kp.cut + X.q(0, kp.cut_words * 32, b, g), x);
+        else ramp[j * kp.ramp_words + b] = x;
+      }
+    }
   }
   // ---- a7: RAM blocks: one warp per RAM, lane s = stream 32g+s (read-first, per-bit write)
   if (n_ram) {

@@ -1123,7 +1123,7 @@ struct Mapper {
       for (uint32_t x : LLs[l].leaf_sig)
         if (x != UINT32_MAX) last[x] = std::max<int32_t>(last[x], (int32_t)l);
     for (uint32_t i = 0; i < n; i++) if (is_ep[i]) last[i] = INF;
-    std::vector<int32_t> word(n, -1);
+    std::vector<int32_t> word(n, -1), birth(n, 0);
     word[0] = 0;   // local node 0 is the constant
     // free-interval allocator (first fit, coalescing); word 0 reserved
     std::map<uint32_t, uint32_t> freeiv;   // start -> length
@@ -1131,16 +1131,23 @@ struct Mapper {
     freeiv[1] = kMaxWords - 1;
     uint32_t max_word = 1;
     std::vector<std::vector<uint32_t>> die(L + 1);
+    // best fit among the holes below the allocated extent; the open tail
+    // (the interval reaching kMaxWords) only when no hole is large enough
     auto take = [&](uint32_t k) -> int64_t {
-      for (auto it = freeiv.begin(); it != freeiv.end(); ++it)
-        if (it->second >= k) {
-          uint32_t st = it->first, len = it->second;
-          freeiv.erase(it);
-          if (len > k) freeiv[st + k] = len - k;
-          max_word = std::max(max_word, st + k);
-          return st;
-        }
-      return -1;
+      auto best = freeiv.end();
+      for (auto it = freeiv.begin(); it != freeiv.end(); ++it) {
+        if (it->second < k) continue;
+        const bool tail = it->first + it->second >= kMaxWords;
+        if (best == freeiv.end()) { best = it; continue; }
+        const bool btail = best->first + best->second >= kMaxWords;
+        if ((btail && !tail) || (btail == tail && it->second < best->second)) best = it;
+      }
+      if (best == freeiv.end()) return -1;
+      uint32_t st = best->first, len = best->second;
+      freeiv.erase(best);
+      if (len > k) freeiv[st + k] = len - k;
+      max_word = std::max(max_word, st + k);
+      return st;
     };
     auto give = [&](uint32_t w) {
       auto nx = freeiv.lower_bound(w);
@@ -1177,7 +1184,12 @@ struct Mapper {
       for (auto& e : LLs[l].two) units[(0u << 16) | e[0]].push_back({e[1], e[2]});
       for (auto& e : LLs[l].wwo) units[(1u << 16) | e[0]].push_back({e[1], e[2]});
       for (auto& e : LLs[l].top) units[(2u << 16)].push_back({e[0], e[1]});
-      for (auto& kv : units) {
+      // larger runs first (they are the hardest to place in holes)
+      std::vector<std::pair<const uint32_t, std::vector<std::pair<uint32_t, uint32_t>>>*> order;
+      for (auto& kv : units) order.push_back(&kv);
+      std::stable_sort(order.begin(), order.end(), [](auto* x, auto* y) { return x->second.size() > y->second.size(); });
+      for (auto* kvp : order) {
+        auto& kv = *kvp;
         auto& v = kv.second;
         std::sort(v.begin(), v.end());
         int64_t base = take((uint32_t)v.size());
@@ -1187,12 +1199,25 @@ struct Mapper {
         for (size_t k = 0; k < v.size(); k++) {
           u.mask |= 1u << v[k].first;
           bind(v[k].second, (uint32_t)base + (uint32_t)k);
+          birth[v[k].second] = (int32_t)l;
         }
         uint32_t kind = kv.first >> 16, unit = kv.first & 0xFFFF;
         if (kind == 0) th[l][unit] = u;
         else if (kind == 1) wa[l][unit] = u;
         else tp[l] = u;
       }
+    }
+    if (opt.verbose >= 3) {
+      // peak number of simultaneously live lane words vs the allocated extent
+      uint32_t peak = 0;
+      for (uint32_t l = 0; l < L; l++) {
+        uint32_t live = 0;
+        for (uint32_t i = 0; i < n; i++)
+          if (word[i] > 0 && birth[i] <= (int32_t)l && last[i] >= (int32_t)l) live++;
+        peak = std::max(peak, live);
+      }
+      fprintf(stderr, "lane part: n=%u srcs=%zu layers=%u max_word=%u peak_live=%u\n", n, srcs.size(), L, max_word,
+              peak);
     }
     if (max_word >= kMaxWords) { fail(P, "lane state overflow"); return false; }
     auto lw = [&](uint32_t x) -> uint32_t {
