@@ -92,7 +92,7 @@ class ClockSampler:
 
 
 def ncu_traffic(cfg: str, kernel: str, cycles: int):
-    """dram read+write bytes of one launch of `kernel` from the newest committed
+    """dram read+write bytes of one launch of `kernel` from the newest (highest _vNN) committed
     `--set full` capture summary (profiles/rNN/ncu_<cfg>_*.json, written by
     scripts/ncu_summary.py) taken at the same cycles per launch; else None."""
     import glob
@@ -105,7 +105,9 @@ def ncu_traffic(cfg: str, kernel: str, cycles: int):
                 continue
             c, u = d["capture"], d["capture_units"]
             t = sum(float(c[k]) * scale[u[k]] for k in ("dram__bytes_read.sum", "dram__bytes_write.sum"))
-            m = os.path.getmtime(f)
+            import re
+            mv = re.search(r"_v(\d+)\.json$", f)
+            m = (int(mv.group(1)) if mv else -1, os.path.getmtime(f))   # newest version tag, then mtime
             if best is None or m > best[0]:
                 best = (m, t, os.path.relpath(f, ROOT))
         except Exception:
