@@ -190,7 +190,8 @@ enum {
  *   (chunks: 0 = header + table, 1..L = layers, L+1 = out+ram; the gread list
  *   is read from global memory)
  *   gread: one u32 gid_l per entry; entry k is stored to lane word k + 1
- *   layer: header (16 words) {size, flags, topc, top_mask | top_base << 8, woff[8], 0...}
+ *   layer: header (32 words) {size, flags, topc, top_mask | top_base << 8, woff[8], 0 x4,
+ *          next layer's first 12 words, 0 x4}
  *          warp record (GEM_LWREC_WORDS words):
  *            [0..5)    wxa, wxb, wob, wmask, wbase       (levels 6-10)
  *            [8..136)  lane constants uint4 {xa, xb, ob, mask}  (levels 1-5; xa/xb/ob
@@ -213,7 +214,11 @@ enum {
   LPH_OFF_LAYERS, LPH_OFF_OUT, LPH_OFF_RAM, LPH_OFF_CHUNKS, LPH_N_CHUNKS, LPH_R12, LPH_R13, LPH_R14,
   LPH_R15, LPH_WORDS = 16
 };
-enum { LLH_WORDS_ = 0, LLH_FLAGS, LLH_TOPC, LLH_TOPWO, LLH_WOFF0 /* ..+7 */, LLH_WORDS = 16 };
+/* lane layer header: [0,12) this layer {size, flags, topc, topwo, woff[8]};
+ * [16,28) a copy of the NEXT layer's [0,12) (zeros after the last layer), so
+ * the kernel knows layer l+1's record addresses while it runs layer l and all
+ * of its record loads issue at once (no header -> offset -> record chain) */
+enum { LLH_WORDS_ = 0, LLH_FLAGS, LLH_TOPC, LLH_TOPWO, LLH_WOFF0 /* ..+7 */, LLH_NEXT = 16, LLH_WORDS = 32 };
 #define GEM_LWREC_HDR 8
 #define GEM_LWREC_LEAVES (GEM_LWREC_HDR + 128)
 #define GEM_LWREC_BASE (GEM_LWREC_HDR + 128 + 512)

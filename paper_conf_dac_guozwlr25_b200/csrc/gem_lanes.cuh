@@ -25,29 +25,53 @@ struct LaneRegs {
   uint32_t base;              // write-out base lane word
   uint4 wc;                   // wxa, wxb, wob, wmask (levels 6-10)
   uint32_t wbase;
-  uint32_t flags, topc, topwo, size;
+  uint32_t flags, topc, topwo, size;           // this layer's header
+  uint32_t nflags, ntopc, ntopwo, nsize, nwoff;  // the next layer's (LLH_NEXT copy)
 };
 
 // Records come straight from global memory (L2-resident program; no shared
-// memory ring): every warp loads its own record of the layer at L, issued one
-// layer ahead of its use so the L2 latency hides behind the current layer.
-__device__ __forceinline__ void load_lane_layer(const uint32_t* L, LaneRegs& R) {
-  const uint32_t lane = threadIdx.x & 31, warp = threadIdx.x >> 5;
+// memory ring): every warp loads its own record, one layer ahead of its use.
+__device__ __forceinline__ void load_lane_rec(const uint32_t* rec, LaneRegs& R) {
+  const uint32_t lane = threadIdx.x & 31;
+  R.wc = __ldg(reinterpret_cast<const uint4*>(rec));
+  R.wbase = __ldg(rec + 4);
+  R.lc = __ldg(reinterpret_cast<const uint4*>(rec + GEM_LWREC_HDR) + lane);
+  const uint4* lv = reinterpret_cast<const uint4*>(rec + GEM_LWREC_LEAVES) + lane;
+#pragma unroll
+  for (uint32_t g = 0; g < 4; g++) R.e[g] = __ldg(lv + g * 32);
+  R.base = __ldg(rec + GEM_LWREC_BASE + lane);
+}
+__device__ __forceinline__ void take_next_header(const uint32_t* L, LaneRegs& R) {
+  const uint4 n = __ldg(reinterpret_cast<const uint4*>(L + LLH_NEXT));
+  R.nwoff = __ldg(L + LLH_NEXT + LLH_WOFF0 + (threadIdx.x >> 5));
+  R.nsize = n.x;
+  R.nflags = n.y;
+  R.ntopc = n.z;
+  R.ntopwo = n.w;
+}
+// layer 0 of an item: its header, then its records (one dependent step)
+__device__ __forceinline__ void load_lane_first(const uint32_t* L, LaneRegs& R) {
+  const uint32_t warp = threadIdx.x >> 5;
   const uint4 h = __ldg(reinterpret_cast<const uint4*>(L));
+  const uint32_t woff = __ldg(L + LLH_WOFF0 + warp);
+  take_next_header(L, R);
   R.size = h.x;
   R.flags = h.y;
   R.topc = h.z;
   R.topwo = h.w;
-  if ((R.flags >> warp) & 1u) {
-    const uint32_t* rec = L + __ldg(L + LLH_WOFF0 + warp);
-    R.wc = __ldg(reinterpret_cast<const uint4*>(rec));
-    R.wbase = __ldg(rec + 4);
-    R.lc = __ldg(reinterpret_cast<const uint4*>(rec + GEM_LWREC_HDR) + lane);
-    const uint4* lv = reinterpret_cast<const uint4*>(rec + GEM_LWREC_LEAVES) + lane;
-#pragma unroll
-    for (uint32_t g = 0; g < 4; g++) R.e[g] = __ldg(lv + g * 32);
-    R.base = __ldg(rec + GEM_LWREC_BASE + lane);
-  }
+  if ((R.flags >> warp) & 1u) load_lane_rec(L + woff, R);
+}
+// layer l+1 at L: its header is already in R.n*, so its records and the header
+// of layer l+2 are all loaded at once
+__device__ __forceinline__ void load_lane_next(const uint32_t* L, LaneRegs& R) {
+  const uint32_t warp = threadIdx.x >> 5;
+  R.size = R.nsize;
+  R.flags = R.nflags;
+  R.topc = R.ntopc;
+  R.topwo = R.ntopwo;
+  const uint32_t woff = R.nwoff;
+  take_next_header(L, R);
+  if ((R.flags >> warp) & 1u) load_lane_rec(L + woff, R);
 }
 
 // K-word vectors: a work item runs K 32-stream groups together, their lane
@@ -251,7 +275,7 @@ __device__ void run_lane_partition(const KParams& kp, uint32_t* S, uint32_t* ram
   // layer 0's records first: independent of S, their latency overlaps the port loads
   const uint32_t* L = gprog + off_layers;
   LaneRegs R;
-  if (n_layers) load_lane_layer(L, R);
+  if (n_layers) load_lane_first(L, R);
   if (pacc && tid == 0 && h0.x == 0u) pacc[7]++;   // (keeps the header read before the stamp)
   phase(0);
   // ---- a2: input ports (once per cycle) for the groups of the item.
@@ -322,7 +346,7 @@ __device__ void run_lane_partition(const KParams& kp, uint32_t* S, uint32_t* ram
 #endif
     const uint32_t ptopc = R.topc, ptopwo = R.topwo;
     L += R.size;
-    if (l + 1 < n_layers) load_lane_layer(L, R);
+    if (l + 1 < n_layers) load_lane_next(L, R);
     if (ptop && (threadIdx.x >> 5) == 0) top_lane_layer<K>(ptopc, ptopwo, s_base, topv, 1);
     __syncthreads();
   }

@@ -570,6 +570,8 @@ __device__ __forceinline__ void top_layer(uint32_t topc, uint32_t topwo, uint32_
 // before they enter S; if none changed (and !act_first) the layers are skipped
 // -- S still holds the previous evaluation of the same inputs, so the endpoint
 // commit below re-stores the same words (row f3).
+// ACT = false compiles to the plain path (no activity code in the hot loop).
+template <bool ACT>
 __device__ void run_partition(const KParams& kp, ProgSrc& ps, uint32_t* S, uint32_t* ramp, uint32_t* topb,
                               uint32_t p, uint32_t st0, uint32_t nst, uint32_t c, uint32_t cur, uint32_t nxt,
                               bool prof_on, uint32_t* act = nullptr, bool act_first = true) {
@@ -630,7 +632,7 @@ __device__ void run_partition(const KParams& kp, ProgSrc& ps, uint32_t* S, uint3
   const uint32_t n_gr = n_gread * nst;
   bool changed = act_first;
   // GEM_F_ACTIVITY: used-bit masks of the gread words (the program's tail)
-  const uint32_t* gmask = act ? gprog + __ldg(kp.parts + p * GP_WORDS + GP_PROG_LEN) - ((n_gread + 3u) & ~3u)
+  const uint32_t* gmask = (ACT && act) ? gprog + __ldg(kp.parts + p * GP_WORDS + GP_PROG_LEN) - ((n_gread + 3u) & ~3u)
                               : nullptr;
   constexpr uint32_t GU = 4;   // port loads in flight per thread (8 measured slower on C3)
   for (uint32_t k0 = 0; k0 < n_gr; k0 += GU * GEM_THREADS) {
@@ -655,7 +657,7 @@ __device__ void run_partition(const KParams& kp, ProgSrc& ps, uint32_t* S, uint3
 #pragma unroll
     for (uint32_t u = 0; u < GU; u++)
       if (dst[u] != ~0u) {
-        if (act) {
+        if (ACT && act) {
           const uint32_t k = k0 + u * GEM_THREADS + tid;
           changed |= ((act[k] ^ v[u]) & __ldg(gmask + k)) != 0u;
           act[k] = v[u];
@@ -665,7 +667,7 @@ __device__ void run_partition(const KParams& kp, ProgSrc& ps, uint32_t* S, uint3
       }
   }
   bool skip = false;
-  if (act) {
+  if (ACT && act) {
     skip = __syncthreads_or(changed ? 1 : 0) == 0;
     if (!skip)
       for (uint32_t k = tid; k < n_gr; k += GEM_THREADS) sts(s_base + 4 * gr[k].y, act[k]);
@@ -692,12 +694,23 @@ __device__ void run_partition(const KParams& kp, ProgSrc& ps, uint32_t* S, uint3
   // BAR.SYNC.DEFER_BLOCKING otherwise defers to the first dependent access)
   if (prof_on && tid == 0 && lds(s_base) == 0u) PROF(1);
   refill();
-  // a skipped partition whose chunks are all in shared memory bypasses the
-  // layer loop; one that streams chunks still walks the ring (no evaluation)
-  const uint32_t n_run = (skip && (ps.resident || n_layers + 1 < n_pin)) ? 0u : n_layers;
+  // a skipped partition (GEM_F_ACTIVITY) evaluates no layer; if it streams
+  // chunks it still walks the ring in the same order (kept out of the hot loop
+  // below, whose code must not change when pruning is off)
+  if (ACT && skip) {
+    for (uint32_t l = 0; l + 1 < n_layers; l++) {
+      if (!(2 + l < n_pin)) ring_wait(ps);
+      __syncthreads();
+      ps.seq_free = ps.seq_wait;
+      refill();
+    }
+    __syncthreads();   // S / ramp reads below follow the port compare
+    ps.seq_free = ps.seq_wait;
+    refill();
+  }
   // ---- a3-a5: layers, software-pipelined: layer l+1's records are loaded
   // into registers before the barrier that ends layer l
-  for (uint32_t l = 0; l < n_run; l++) {
+  for (uint32_t l = 0; l < ((ACT && skip) ? 0u : n_layers); l++) {
     FPROF(l, 0);
 #ifdef GEM_FINE_PROF
     const uint32_t fl = (kp.fprof && c == 5 && blockIdx.x == kp.fine_cta) ? l : 99u;
@@ -707,8 +720,7 @@ __device__ void run_partition(const KParams& kp, ProgSrc& ps, uint32_t* S, uint3
     unsigned long long* fsub = nullptr;
 #endif
     // stream j uses named barrier 1 + j (group <= GEM_MAX_GROUP < 16)
-    if (skip) {
-    } else if (nst == 1 && s_base == GEM_S0_ADDR) exec_layer<true>(R, s_base, g_smem, topb, 1, fl, fsub);
+    if (nst == 1 && s_base == GEM_S0_ADDR) exec_layer<true>(R, s_base, g_smem, topb, 1, fl, fsub);
     else
       for (uint32_t j = 0; j < nst; j++)
         exec_layer<false>(R, s_base + 4 * j * SW, g_smem + j * SW, topb + 16 * j, 1 + j, fl, fsub);
@@ -738,7 +750,7 @@ __device__ void run_partition(const KParams& kp, ProgSrc& ps, uint32_t* S, uint3
     }
     FPROF(l, 3);
 #if !defined(EXP_NO_TOP) && !defined(GEM_TOP_ATOMIC)
-    if (ptop && warp == 0 && !skip)
+    if (ptop && warp == 0)
       for (uint32_t j = 0; j < nst; j++) top_layer(ptopc, ptopwo, s_base + 4 * j * SW, topb + 16 * j, 1 + j);
 #endif
     FPROF(l, 4);
@@ -749,7 +761,6 @@ __device__ void run_partition(const KParams& kp, ProgSrc& ps, uint32_t* S, uint3
   }
   PROF(2);
   // ---- a6: endpoint commit (warp ballot-gather per output word and stream)
-  if (n_run == 0 && n_layers) __syncthreads();   // bypassed: S / ramp reads below follow the port compare
   const uint32_t* od = n_layers + 1 < n_pin ? (C0 + off_out) : ring_wait(ps);
   const uint32_t* os = od + n_out_pad;
   for (uint32_t jj = warp; jj < n_out * nst; jj += GEM_WARPS) {
@@ -817,6 +828,8 @@ __device__ void record_state(const KParams& kp, uint32_t c, uint32_t buf) {
   }
 }
 
+// ACT: GEM_F_ACTIVITY build of the kernel (the plain one carries no pruning code)
+template <bool ACT>
 __global__ void __launch_bounds__(GEM_THREADS, 2) gem_step_kernel(const KParams kp) {
   extern __shared__ __align__(16) uint32_t smem[];
   // layout (words): S[group][state_words] | area[area_words] | ctab[256] | ramp[group][128] |
@@ -966,7 +979,7 @@ __global__ void __launch_bounds__(GEM_THREADS, 2) gem_step_kernel(const KParams 
   // activity pruning: only a CTA with exactly one work item (one partition,
   // one stream) per cycle keeps S, ramp and the port copy from cycle to cycle
   uint32_t* act = nullptr;
-  if (kp.act_words && kp.group == 1) {
+  if (ACT && kp.act_words && kp.group == 1) {
     uint32_t n_it = 0;
     for (uint32_t s = 0; s < kp.n_stages; s++) n_it += wl_end(s) - wl_begin(s);
     if (n_it == 1) act = act_buf;
@@ -985,8 +998,8 @@ __global__ void __launch_bounds__(GEM_THREADS, 2) gem_step_kernel(const KParams 
       for (uint32_t k = kb; k < ke; k++) {
         const uint2 it = wl_item(s, k);
         const uint32_t nst = min(kp.group, kp.n_streams - it.y);
-        run_partition(kp, ps, S, ramp, topb, it.x, it.y, nst, c, cur, nxt, prof_on && k == kb && s == 0, act,
-                      c == 0);
+        run_partition<ACT>(kp, ps, S, ramp, topb, it.x, it.y, nst, c, cur, nxt, prof_on && k == kb && s == 0, act,
+                           c == 0);
         if (!ps.resident) {
           // prefetch the next work item's prologue (overlaps the grid barrier)
           uint32_t np = ~0u;
@@ -1260,6 +1273,10 @@ static double build_worklists(const gem_sim* sim, uint32_t G, std::vector<uint32
   return makespan;
 }
 
+static const void* step_kernel_for(const gem_sim* sim) {
+  return sim->act_words ? (const void*)gem_step_kernel<true> : (const void*)gem_step_kernel<false>;
+}
+
 // Choose CTAs per SM, grid, work lists and the shared-memory program mode.
 // Resident mode (every program a CTA runs copied into its shared memory once
 // per launch) is used when it fits; otherwise programs stream through a TMA
@@ -1312,8 +1329,8 @@ static int plan_launch(gem_sim* sim, uint32_t max_chunk_words, uint32_t grid_lim
     if (grid_limit) grid = std::max<uint32_t>(1, std::min(grid, grid_limit));
     grid = std::min<uint32_t>(grid, GEM_BAR_MAX_CTAS);
     int occ = 0;
-    CK(cudaFuncSetAttribute(gem_step_kernel, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)budget));
-    CK(cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ, gem_step_kernel, GEM_THREADS, (size_t)budget));
+    CK(cudaFuncSetAttribute(step_kernel_for(sim), cudaFuncAttributeMaxDynamicSharedMemorySize, (int)budget));
+    CK(cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ, step_kernel_for(sim), GEM_THREADS, (size_t)budget));
     if ((uint32_t)occ < bps) continue;
     const double makespan = build_worklists(sim, grid, off, items);
     // residency is decided per CTA (its work list's distinct programs fit in the area)
@@ -1355,7 +1372,7 @@ static int plan_launch(gem_sim* sim, uint32_t max_chunk_words, uint32_t grid_lim
   sim->ring_slots = best.ring;
   sim->slot_words = slot;
   sim->smem_bytes = (fixed_words + best.area) * 4;
-  CK(cudaFuncSetAttribute(gem_step_kernel, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)sim->smem_bytes));
+  CK(cudaFuncSetAttribute(step_kernel_for(sim), cudaFuncAttributeMaxDynamicSharedMemorySize, (int)sim->smem_bytes));
   CK(dalloc(&sim->d_wl_off, best_off.size() * 4));
   CK(cudaMemcpy(sim->d_wl_off, best_off.data(), best_off.size() * 4, cudaMemcpyHostToDevice));
   CK(dalloc(&sim->d_wl_items, std::max<size_t>(best_items.size(), 1) * 8));
@@ -1713,7 +1730,7 @@ int gem_step(gem_sim* sim, uint64_t ncycles) {
   }
   void* args[] = {&kp};
   CK(cudaEventRecord(sim->ev0, sim->stream));
-  CK(cudaLaunchCooperativeKernel(sim->lanes ? lane_kernel_for(sim->lane_groups) : (const void*)gem_step_kernel,
+  CK(cudaLaunchCooperativeKernel(sim->lanes ? lane_kernel_for(sim->lane_groups) : step_kernel_for(sim),
                                  dim3(sim->grid), dim3(GEM_THREADS), args, sim->smem_bytes, sim->stream));
   CK(cudaEventRecord(sim->ev1, sim->stream));
   sim->in_head += (uint32_t)ncycles;

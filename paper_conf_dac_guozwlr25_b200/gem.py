@@ -80,7 +80,8 @@ def load_library(build: bool = True):
             lib.gem_write_ram.argtypes = [P, u32, u32, P]
             lib.gem_last_step_ms.argtypes = [P, ctypes.POINTER(ctypes.c_float)]
             lib.gem_read_profile.argtypes = [P, P, ctypes.POINTER(u32), ctypes.POINTER(u32)]
-            lib.gem_read_activity.argtypes = [P, ctypes.POINTER(u64), ctypes.POINTER(u64)]
+            if hasattr(lib, "gem_read_activity"):   # (older builds loaded by A/B timing scripts lack it)
+                lib.gem_read_activity.argtypes = [P, ctypes.POINTER(u64), ctypes.POINTER(u64)]
             lib.gem_free.argtypes = [P]
             lib.gem_free.restype = None
             lib.gem_last_error.restype = ctypes.c_char_p

@@ -1285,6 +1285,15 @@ struct Mapper {
       pr[base + LLH_WORDS_] = (uint32_t)(pr.size() - base);
       pr[pr[LPH_OFF_CHUNKS] + 1 + l] = pr[base + LLH_WORDS_];
     }
+    // next-layer header copies (LLH_NEXT)
+    {
+      size_t off = pr[LPH_OFF_LAYERS];
+      for (uint32_t l = 0; l < L; l++) {
+        const size_t nx = off + pr[off + LLH_WORDS_];
+        for (int k = 0; k < 12; k++) pr[off + LLH_NEXT + k] = (l + 1 < L) ? pr[nx + k] : 0u;
+        off = nx;
+      }
+    }
     pr[LPH_OFF_OUT] = (uint32_t)pr.size();
     for (auto& ow : P.outs) {
       uint32_t reg = GEM_GID_REGION(ow.dst), idx = GEM_GID_INDEX(ow.dst);

@@ -163,6 +163,25 @@ def test_c3_state_roundtrip_and_determinism(gem):
     assert np.array_equal(c.read_state(), q)
 
 
+def test_c3_speed_independent_of_stimulus(gem):
+    """the method is oblivious -- every live AND is
+    evaluated every cycle -- so cycles/s must not depend on the stimulus: two
+    stimulus seeds (and an all-zero stimulus) time within 3% (median of 5)."""
+    T = 1000
+    sim = gem.Simulator(blob("c3"))
+    times = {}
+    for name, st in [("seed103", stimulus("c3", 256, T)), ("seed7", stimulus("c3", 256, T, seed=7)),
+                     ("zeros", np.zeros((T, 8), np.uint32))]:
+        ms = []
+        for _ in range(5):
+            sim.set_inputs(st)
+            sim.step(T)
+            ms.append(sim.last_step_ms())
+        times[name] = float(np.median(ms))
+    lo, hi = min(times.values()), max(times.values())
+    assert hi / lo < 1.03, times
+
+
 def test_c5_streams_vs_oracle_lanes(gem):
     """Batched streams: stream s of the GPU == 64-lane oracle lane s (C5 recipe)."""
     S, T = 64, 120
