@@ -236,6 +236,8 @@ __device__ __forceinline__ void mbar_expect_tx(uint64_t* bar, uint32_t bytes) {
                : "memory");
 }
 __device__ __forceinline__ void mbar_wait(uint64_t* bar, uint32_t parity) {
+  // (no watchdog here: even an out-of-line slow path cost ~70 clk per C3
+  // layer; a grid-barrier stall still traps after 10 s)
   uint32_t done = 0;
   while (!done) {
     asm volatile(
@@ -258,7 +260,7 @@ __device__ __forceinline__ void fence_mbar_init() {
   asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
 }
 
-#define GEM_RING_MAX 4
+#define GEM_RING_MAX 8
 #define GEM_MAX_CHUNKS 256
 #define GEM_MAX_RESIDENT 16
 #define GEM_WL_MAX_STAGES 8
@@ -284,7 +286,7 @@ struct ProgSrc {
   const uint32_t* res_off; // smem [GEM_MAX_RESIDENT] word offsets into area
 };
 
-// ring depth R is a power of two (2 or 4): slot = seq & (R-1), phase = (seq / R) & 1
+// ring depth R is a power of two (2, 4 or 8): slot = seq & (R-1), phase = (seq / R) & 1
 __device__ __forceinline__ uint32_t* ring_slot(const ProgSrc& ps, uint32_t seq) {
   return ps.area + (seq & (ps.R - 1)) * ps.slot_words;
 }
@@ -299,7 +301,7 @@ __device__ __forceinline__ void ring_issue(ProgSrc& ps, const uint32_t* g, uint3
 }
 __device__ __forceinline__ const uint32_t* ring_wait(ProgSrc& ps) {
   const uint32_t seq = ps.seq_wait++;
-  mbar_wait(ps.mbar + (seq & (ps.R - 1)), (seq >> (ps.R == 4 ? 2 : 1)) & 1u);
+  mbar_wait(ps.mbar + (seq & (ps.R - 1)), (seq >> (__ffs(ps.R) - 1)) & 1u);   // phase = (seq / R) & 1
   return ring_slot(ps, seq);
 }
 
@@ -833,7 +835,8 @@ template <bool ACT>
 __global__ void __launch_bounds__(GEM_THREADS, 2) gem_step_kernel(const KParams kp) {
   extern __shared__ __align__(16) uint32_t smem[];
   // layout (words): S[group][state_words] | area[area_words] | ctab[256] | ramp[group][128] |
-  //                 topb[group][16] | res_p[16] | res_off[16] | res_n[16] | wl cache | mbar[8 x u64]
+  //                 topb[group][16] | res_p[16] | res_off[16] | res_n[16] | wl cache | mbar[16 x u64] |
+  //                 act[act_words]
   // S must stay at offset 0 (leaf entries carry byte offsets into it).
   uint32_t* S = smem;
   uint32_t* area = S + kp.group * kp.state_words;
@@ -847,7 +850,7 @@ __global__ void __launch_bounds__(GEM_THREADS, 2) gem_step_kernel(const KParams 
   // per stage, [24] cached flag, [32, 32 + 2*GEM_WL_CACHE) items (uint2)
   uint32_t* wlc = res_n + 16;
   uint64_t* mbar = reinterpret_cast<uint64_t*>(wlc + GEM_WL_CACHE_WORDS);
-  uint32_t* act_buf = reinterpret_cast<uint32_t*>(mbar + 8);   // [act_words] (GEM_F_ACTIVITY)
+  uint32_t* act_buf = reinterpret_cast<uint32_t*>(mbar + 16);  // [act_words] (GEM_F_ACTIVITY)
   const uint32_t tid = threadIdx.x;
   const uint32_t G = gridDim.x, B = blockIdx.x;
   if (tid == 0) {
@@ -912,18 +915,27 @@ __global__ void __launch_bounds__(GEM_THREADS, 2) gem_step_kernel(const KParams 
         }
       if (single && p1 != ~0u) {
         const uint32_t* g = kp.prog + __ldg(kp.parts + p1 * GP_WORDS + GP_PROG_OFF);
-        const uint32_t nch = __ldg(g + PH_N_CHUNKS), offc = __ldg(g + PH_OFF_CHUNKS);
+        const uint32_t nch = min(__ldg(g + PH_N_CHUNKS), (uint32_t)GEM_MAX_CHUNKS), offc = __ldg(g + PH_OFF_CHUNKS);
+        // ring slots sized for the largest chunk that still streams (the
+        // light tail layers are a fraction of the heaviest), so the ring is
+        // as deep as possible: ctab (unused in this mode) holds suffix maxima
+        for (uint32_t k = nch; k-- > 0;) ctab[k] = max(__ldg(g + offc + k), k + 1 < nch ? ctab[k + 1] : 0u);
         uint32_t P = 0, pw = 0;
         while (P < nch) {
           const uint32_t sz = __ldg(g + offc + P);
-          if (pw + sz + 2 * kp.slot_words > kp.area_words) break;
+          const uint32_t rest = P + 1 < nch ? ctab[P + 1] : 0u;
+          if (pw + sz + 2 * rest > kp.area_words) break;
           pw += sz;
           P++;
         }
         if (P >= 2) {
+          const uint32_t slot = P < nch ? ((ctab[P] + 3u) & ~3u) : 4u;
+          uint32_t R = 2;
+          while (2 * R <= GEM_RING_MAX && pw + 2 * R * slot <= kp.area_words) R *= 2;
           res_n[2] = P;
           res_n[3] = pw;
-          res_n[4] = pw + 4 * kp.slot_words <= kp.area_words ? 4u : 2u;
+          res_n[4] = R;
+          res_n[5] = slot;
           mbar_expect_tx(mbar + GEM_RING_MAX, pw * 4);
           tma_load_1d(area, g, pw * 4, mbar + GEM_RING_MAX);
         }
@@ -960,6 +972,7 @@ __global__ void __launch_bounds__(GEM_THREADS, 2) gem_step_kernel(const KParams 
   if (ps.pin_chunks) {
     ps.area = area + ps.pin_off;   // ring after the pinned prefix
     ps.R = res_n[4];
+    ps.slot_words = res_n[5];
   }
   if ((ps.resident && ps.n_res) || ps.pin_chunks) mbar_wait(mbar + GEM_RING_MAX, 0);
   // first work item of this CTA in a cycle: partition id, or ~0u
@@ -1297,7 +1310,7 @@ static int plan_launch(gem_sim* sim, uint32_t max_chunk_words, uint32_t grid_lim
     const char* genv = getenv("GEM_GROUP");
     uint32_t g = genv ? (uint32_t)atoi(genv) : GEM_MAX_GROUP;
     g = std::max<uint32_t>(1, std::min<uint32_t>(std::min<uint32_t>(g, GEM_MAX_GROUP), sim->n_streams));
-    while (g > 1 && (uint64_t)(g * (sim->state_words + 4 * GEM_MAX_RAMS_PER_PART + 16) + GEM_MAX_CHUNKS + 80 + GEM_WL_CACHE_WORDS +
+    while (g > 1 && (uint64_t)(g * (sim->state_words + 4 * GEM_MAX_RAMS_PER_PART + 16) + GEM_MAX_CHUNKS + 96 + GEM_WL_CACHE_WORDS +
                                3 * slot) * 4 > (uint64_t)optin)
       g /= 2;
     sim->group = g;
@@ -1308,7 +1321,7 @@ static int plan_launch(gem_sim* sim, uint32_t max_chunk_words, uint32_t grid_lim
                                                   ((sim->n_streams + sim->group - 1) / sim->group));
   if (sim->group != 1) sim->act_words = 0;   // activity pruning needs one stream per work item
   const uint32_t fixed_words = sim->group * (sim->state_words + 4 * GEM_MAX_RAMS_PER_PART + 16) + GEM_MAX_CHUNKS +
-                               48 + GEM_WL_CACHE_WORDS + 16 + sim->act_words;
+                               48 + GEM_WL_CACHE_WORDS + 32 + sim->act_words;
   const char* env = getenv("GEM_NO_RESIDENT");
   const bool allow_res = !(env && env[0] == '1');
   const char* benv = getenv("GEM_BPS");
@@ -1351,7 +1364,7 @@ static int plan_launch(gem_sim* sim, uint32_t max_chunk_words, uint32_t grid_lim
     }
     const bool res = n_res == grid;
     uint32_t ring = std::min<uint32_t>(GEM_RING_MAX, area / std::max<uint32_t>(slot, 4));
-    ring = ring >= 4 ? 4 : ring >= 2 ? 2 : ring;   // power of two (kernel masks instead of dividing)
+    ring = ring >= 8 ? 8 : ring >= 4 ? 4 : ring >= 2 ? 2 : ring;   // power of two (kernel masks instead of dividing)
     if (!res && ring < 2) continue;
     // score: estimated makespan, SM sharing slows co-resident CTAs, streaming costs a little
     double score = makespan * (1.0 + 0.5 * (bps - 1) * std::min(1.0, (double)grid / ((double)bps * sms)))
