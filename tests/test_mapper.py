@@ -104,3 +104,50 @@ def test_c5_lane_program_prefix():
     o.lanes_reset(1)
     r = o.lanes_run(0, st)
     assert np.array_equal(po, r["po"])
+
+
+def _lane_programs(b):
+    """(partition id, lane program words) for every partition of a blob."""
+    w = np.frombuffer(b, np.uint32)
+    n_parts, off_parts, off_lane = int(w[6]), int(w[21]), int(w[37])
+    for p in range(n_parts):
+        pt = w[off_parts + 16 * p: off_parts + 16 * p + 16]
+        yield p, w[off_lane + int(pt[9]): off_lane + int(pt[9]) + int(pt[10])]
+
+
+def test_lane_layer_headers_carry_next_layer():
+    """gem_isa.h LLH_NEXT: layer l's header words [16, 28) equal layer l+1's
+    words [0, 12) (zeros after the last layer) -- the kernel issues layer l+1's
+    record loads from them without reading its header first."""
+    LPH_N_LAYERS, LPH_OFF_LAYERS = 2, 7
+    n_checked = 0
+    for _, pr in _lane_programs(blob("c5")):
+        L = int(pr[LPH_OFF_LAYERS])
+        for l in range(int(pr[LPH_N_LAYERS])):
+            nxt = L + int(pr[L])
+            want = pr[nxt:nxt + 12] if l + 1 < int(pr[LPH_N_LAYERS]) else np.zeros(12, np.uint32)
+            assert np.array_equal(pr[L + 16:L + 28], want), l
+            L = nxt
+            n_checked += 1
+    assert n_checked > 100
+
+
+def test_program_tail_holds_gread_used_bit_masks(tmp_path):
+    """Row f3 (GEM_F_ACTIVITY): the last ceil4(n_gread) words of a partition
+    program are the used-bit masks of its gread words: every mask is non-zero,
+    and together they cover exactly the sources the partition reads."""
+    net = circuits.gated_counters(8, 16)
+    p = circuits.save(net, str(tmp_path), "gated")
+    b = compile_file(p, "parts=8")
+    w = np.frombuffer(b, np.uint32)
+    n_parts, off_parts, off_prog = int(w[6]), int(w[21]), int(w[24])
+    total_bits = 0
+    for q in range(n_parts):
+        pt = w[off_parts + 16 * q: off_parts + 16 * q + 16]
+        pr = w[off_prog + int(pt[1]): off_prog + int(pt[1]) + int(pt[2])]
+        n_gread = int(pr[1])
+        masks = pr[len(pr) - ((n_gread + 3) & ~3):][:n_gread]
+        assert n_gread > 0 and (masks != 0).all()
+        total_bits += sum(bin(int(m)).count("1") for m in masks)
+    # each module reads its enable and its 32 flops: 8 partitions x 33 sources
+    assert total_bits == 8 * 33, total_bits
