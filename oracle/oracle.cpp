@@ -45,6 +45,8 @@
 #include <stdexcept>
 #include <string>
 #include <vector>
+#include <thread>
+#include <atomic>
 
 namespace {
 
@@ -388,6 +390,112 @@ void run_cycles(Oracle& o, const uint32_t* stim, uint64_t cycles, uint32_t* po, 
   }
 }
 
+// ---------------------------------------------------------------- multi-threaded baseline
+// SURVEY §8(d) "also time an nproc-thread variant (OpenMP over the ANDs of each
+// level)": the same cycle as run_cycles, with step 2 evaluated level by level
+// (level = 1 + max level of the AND's AND fan-ins; every AND of a level depends
+// only on earlier levels, so a level is any-order).  Runs of consecutive levels
+// too small to share (< kParMin ANDs) are evaluated by thread 0 alone, so
+// threads meet at a barrier only around the wide levels.  Steps 1 and 3-7 are
+// thread 0's.  Test infrastructure / CPU baseline only, like the rest of oracle/.
+struct SpinBarrier {
+  std::atomic<uint32_t> count{0}, gen{0};
+  uint32_t n;
+  explicit SpinBarrier(uint32_t n_) : n(n_) {}
+  void wait() {
+    const uint32_t g = gen.load(std::memory_order_acquire);
+    if (count.fetch_add(1, std::memory_order_acq_rel) + 1 == n) {
+      count.store(0, std::memory_order_relaxed);
+      gen.store(g + 1, std::memory_order_release);
+    } else {
+      while (gen.load(std::memory_order_acquire) == g) std::this_thread::yield();
+    }
+  }
+};
+
+void run_cycles_mt(Oracle& o, const uint32_t* stim, uint64_t cycles, uint32_t* po, uint32_t nth) {
+  const uint64_t kParMin = 4096;
+  // levels
+  std::vector<uint32_t> lvl_of_var(o.M + 1, 0), lvl(o.A, 0);
+  uint32_t max_lvl = 0;
+  for (uint64_t k : o.topo) {
+    const uint32_t la = lvl_of_var[o.and_a[k] >> 1], lb = lvl_of_var[o.and_b[k] >> 1];
+    lvl[k] = 1 + std::max(la, lb);
+    lvl_of_var[o.and_lhs[k] >> 1] = lvl[k];
+    max_lvl = std::max(max_lvl, lvl[k]);
+  }
+  std::vector<std::vector<uint64_t>> by_lvl(max_lvl + 1);
+  for (uint64_t k : o.topo) by_lvl[lvl[k]].push_back(k);
+  // segments: {parallel?, ANDs in evaluation order}
+  std::vector<std::pair<bool, std::vector<uint64_t>>> seg;
+  for (uint32_t l = 1; l <= max_lvl; l++) {
+    const bool par = by_lvl[l].size() >= kParMin && nth > 1;
+    if (seg.empty() || par || seg.back().first)
+      seg.push_back({par, {}});
+    auto& v = seg.back().second;
+    v.insert(v.end(), by_lvl[l].begin(), by_lvl[l].end());
+  }
+  const uint64_t piw = (o.n_pi + 31) / 32, pow_ = (o.O + 31) / 32;
+  std::vector<uint8_t> Qn(o.L);
+  std::vector<uint32_t> RDn(o.rams.size());
+  SpinBarrier bar(nth);
+  auto worker = [&](uint32_t tid) {
+    for (uint64_t t = 0; t < cycles; t++) {
+      if (tid == 0) {
+        o.v[0] = 0;
+        for (uint64_t i = 0; i < o.I; i++) {
+          uint8_t b;
+          if (o.input_pi[i] >= 0) {
+            uint64_t p = (uint64_t)o.input_pi[i];
+            b = (uint8_t)((stim[t * piw + p / 32] >> (p % 32)) & 1u);
+          } else {
+            b = (uint8_t)((o.RD[(uint64_t)o.input_ram[i]] >> o.input_rambit[i]) & 1u);
+          }
+          o.v[1 + i] = b;
+        }
+        for (uint64_t j = 0; j < o.L; j++) o.v[1 + o.I + j] = o.Q[j];
+      }
+      for (auto& sg : seg) {
+        if (sg.first) {
+          bar.wait();
+          const uint64_t n = sg.second.size(), a = n * tid / nth, b = n * (tid + 1) / nth;
+          for (uint64_t q = a; q < b; q++) {
+            const uint64_t k = sg.second[q];
+            o.v[o.and_lhs[k] >> 1] = (uint8_t)(val(o, o.and_a[k]) & val(o, o.and_b[k]));
+          }
+          bar.wait();
+        } else if (tid == 0) {
+          for (uint64_t k : sg.second) o.v[o.and_lhs[k] >> 1] = (uint8_t)(val(o, o.and_a[k]) & val(o, o.and_b[k]));
+        }
+      }
+      if (tid == 0) {
+        if (po) {
+          uint32_t* row = po + t * pow_;
+          for (uint64_t w = 0; w < pow_; w++) row[w] = 0;
+          for (uint64_t k = 0; k < o.O; k++) row[k / 32] |= (uint32_t)val(o, o.outputs[k]) << (k % 32);
+        }
+        for (uint64_t j = 0; j < o.L; j++) Qn[j] = val(o, o.latch_next[j]);
+        for (size_t r = 0; r < o.rams.size(); r++) {
+          const Ram& ram = o.rams[r];
+          uint32_t ra = 0, wa = 0, wd = 0, be = 0;
+          for (int k = 0; k < kAddrBits; k++) ra |= (uint32_t)val(o, ram.raddr[k]) << k;
+          for (int k = 0; k < kAddrBits; k++) wa |= (uint32_t)val(o, ram.waddr[k]) << k;
+          for (int k = 0; k < kDataBits; k++) wd |= (uint32_t)val(o, ram.wdata[k]) << k;
+          for (int k = 0; k < kDataBits; k++) be |= (uint32_t)val(o, ram.wbe[k]) << k;
+          RDn[r] = o.MEM[r][ra];
+          o.MEM[r][wa] = (o.MEM[r][wa] & ~be) | (wd & be);
+        }
+        o.Q = Qn;
+        for (size_t r = 0; r < o.rams.size(); r++) o.RD[r] = RDn[r];
+      }
+    }
+  };
+  std::vector<std::thread> th;
+  for (uint32_t i = 1; i < nth; i++) th.emplace_back(worker, i);
+  worker(0);
+  for (auto& x : th) x.join();
+}
+
 // ---------------------------------------------------------------- 64-lane batches
 inline uint64_t lval(const std::vector<uint64_t>& v, uint64_t lit) {
   return v[lit >> 1] ^ ((lit & 1) ? ~0ull : 0ull);
@@ -543,6 +651,20 @@ int orc_run(void* h, const uint32_t* stim, uint64_t cycles, uint32_t* po, uint32
     Oracle* o = (Oracle*)h;
     auto t0 = std::chrono::steady_clock::now();
     run_cycles(*o, stim, cycles, po, st, dig);
+    auto t1 = std::chrono::steady_clock::now();
+    if (seconds) *seconds = std::chrono::duration<double>(t1 - t0).count();
+    return 0;
+  } catch (const std::exception& e) {
+    g_err = e.what();
+    return -1;
+  }
+}
+
+int orc_run_mt(void* h, const uint32_t* stim, uint64_t cycles, uint32_t* po, uint32_t threads, double* seconds) {
+  try {
+    Oracle* o = (Oracle*)h;
+    auto t0 = std::chrono::steady_clock::now();
+    run_cycles_mt(*o, stim, cycles, po, std::max<uint32_t>(1, threads));
     auto t1 = std::chrono::steady_clock::now();
     if (seconds) *seconds = std::chrono::duration<double>(t1 - t0).count();
     return 0;

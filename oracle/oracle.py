@@ -45,6 +45,7 @@ def _load():
             lib.orc_set_ram.argtypes = [P, ctypes.c_uint32, P]
             lib.orc_get_rd.argtypes = [P, P]
             lib.orc_run.argtypes = [P, P, u64, P, P, P, P]
+            lib.orc_run_mt.argtypes = [P, P, u64, P, ctypes.c_uint32, P]
             lib.orc_lanes_reset.argtypes = [P, u64]
             lib.orc_lanes_run.argtypes = [P, u64, u64, P, u64, P, P, P]
             lib.orc_lanes_get_state.argtypes = [P, u64, u64, P]
@@ -140,6 +141,19 @@ class Oracle:
         if digest:
             out["digest"] = dg_a
         return out
+
+    def run_mt(self, stim: np.ndarray, threads: int) -> np.ndarray:
+        """Level-parallel variant of run() on `threads` host threads (CPU baseline,
+        SURVEY §8(d)); same results.  Returns po [cycles][po_words]."""
+        stim = np.ascontiguousarray(stim, dtype=np.uint32)
+        cycles = stim.shape[0]
+        assert stim.shape[1] == self.pi_words
+        po_a = np.zeros((cycles, self.po_words), np.uint32)
+        secs = ctypes.c_double(0)
+        if self._lib.orc_run_mt(self._h, _ptr(stim), cycles, _ptr(po_a), threads, ctypes.byref(secs)):
+            raise RuntimeError(self._lib.orc_last_error().decode())
+        self.last_seconds = secs.value
+        return po_a
 
     # ---- 64-lane batched streams -------------------------------------------
     def lanes_reset(self, groups: int):

@@ -417,3 +417,21 @@ def test_gated_counters_closed_form(tmp_path):
         on = ((en >> k) & 1).astype(bool)
         acc = po[:, k] >> 16               # acc only changes in cycles after an enabled one
         assert np.array_equal(acc[1:][~on[:-1]], acc[:-1][~on[:-1]]), k
+
+
+@pytest.mark.parametrize("threads", [1, 3, 8])
+def test_level_parallel_variant_equals_oracle(tmp_path, threads):
+    """The level-parallel CPU baseline (SURVEY §8(d) nproc-thread variant) gives
+    the oracle's PO trace and final state on a design with RAM, resets and
+    long tails (small levels evaluated serially, wide ones split)."""
+    net = circuits.small_G(seed=21, n_and=20000, with_ram=True, clusters=4, flops=256, d_max=40)
+    p = circuits.save(net, str(tmp_path), "g")
+    st = stim_random(net.n_pi, 300, 5, reset_pi0_cycles=2)
+    a = Oracle(p)
+    ref = a.run(st)["po"]
+    b = Oracle(p)
+    got = b.run_mt(st, threads)
+    assert np.array_equal(got, ref)
+    assert np.array_equal(b.get_state(), a.get_state())
+    for r in range(len(net.rams)):
+        assert np.array_equal(b.get_ram(r), a.get_ram(r))
