@@ -69,6 +69,8 @@ struct Options {
   int max_parts = 280;      // refinement stops growing the partition count here
   int lanes = 0;            // also emit stream-sliced lane programs (batched streams)
   int lane_words = 16383;   // cap on a lane program's state words (larger partitions are split)
+  int lane_banks = 1;       // bank-aware placement of lane write-out runs (2: also interior offsets)
+  int lane_holes = 32;      // best-fitting holes considered per run
   int banks = 1;            // bank-conflict-aware renaming of the state words (rename_state_words)
   int verbose = 0;
   int max_state_words = GEM_MAX_STATE_WORDS;
@@ -103,6 +105,8 @@ static Options parse_opts(const char* s) {
     else if (k == "max_parts") o.max_parts = std::stoi(v);
     else if (k == "lanes") o.lanes = std::stoi(v);
     else if (k == "lane_words") o.lane_words = std::min(16383, std::stoi(v));
+    else if (k == "lane_banks") o.lane_banks = std::stoi(v);
+    else if (k == "lane_holes") o.lane_holes = std::max(1, std::stoi(v));
     else if (k == "banks") o.banks = std::stoi(v);
     else throw std::runtime_error("unknown option " + k);
   }
@@ -1159,9 +1163,78 @@ struct Mapper {
       }
       freeiv[st] = len;
     };
+    // Bank-aware placement (lane_banks=1): a leaf load of the lane kernel is one
+    // LDS.K per (layer, warp, leaf position) over the 32 lanes; with K = 2
+    // each half-warp's 16 lanes read 8-byte words, conflict-free when their
+    // lane words differ mod 16.  reads[x] lists the (instruction, half-warp)
+    // groups that read signal x; occ counts the words already placed per group
+    // and residue.  Runs are placed at the offset (within the few best-fitting
+    // holes, or the tail) that adds the fewest same-residue readers.
+    const bool banks = opt.lane_banks != 0;
+    std::vector<std::vector<uint32_t>> reads(banks ? n : 0);
+    std::vector<uint8_t> occ;
+    if (banks) {
+      for (uint32_t l = 0; l < L; l++)
+        for (uint32_t id = 0; id < 8192; id++) {
+          const uint32_t x = LLs[l].leaf_sig[id];
+          if (x == UINT32_MAX || x == 0) continue;
+          const uint32_t warp = id >> 10, lane = (id >> 5) & 31, pos = id & 31;
+          reads[x].push_back(((l * 8 + warp) * 32 + pos) * 2 + (lane >> 4));
+        }
+      occ.assign((size_t)L * 8 * 32 * 2 * 16, 0);
+    }
     auto bind = [&](uint32_t x, uint32_t w) {
       word[x] = (int32_t)w;
       if (last[x] >= 0 && last[x] < (int32_t)L) die[last[x]].push_back(w);
+      if (banks)
+        for (uint32_t g : reads[x]) { uint8_t& o = occ[(size_t)g * 16 + (w & 15)]; if (o < 255) o++; }
+    };
+    auto run_cost = [&](const std::vector<std::pair<uint32_t, uint32_t>>& v, uint32_t b) {
+      uint32_t c = 0;
+      for (size_t k = 0; k < v.size(); k++)
+        for (uint32_t g : reads[v[k].second]) c += occ[(size_t)g * 16 + ((b + k) & 15)];
+      return c;
+    };
+    // place a run: best (cost, hole size, address) over the lane_holes best-fitting holes
+    // (all 16 residues each) and the tail; only holes, if any fits
+    auto take_banked = [&](const std::vector<std::pair<uint32_t, uint32_t>>& v) -> int64_t {
+      const uint32_t k = (uint32_t)v.size();
+      std::vector<std::pair<uint32_t, uint32_t>> holes;   // (len, start)
+      uint32_t tail_st = 0, tail_len = 0;
+      for (auto& iv : freeiv) {
+        if (iv.second < k) continue;
+        if (iv.first + iv.second >= kMaxWords) { tail_st = iv.first; tail_len = iv.second; continue; }
+        holes.push_back({iv.second, iv.first});
+      }
+      std::vector<std::pair<uint32_t, uint32_t>> cands;
+      if (!holes.empty()) {
+        const size_t nh = std::min<size_t>((size_t)opt.lane_holes, holes.size());
+        std::partial_sort(holes.begin(), holes.begin() + nh, holes.end());
+        holes.resize(nh);
+        cands = holes;
+      } else if (tail_len >= k) {
+        cands.push_back({tail_len, tail_st});
+      } else {
+        return -1;
+      }
+      uint64_t best = UINT64_MAX;
+      uint32_t bst = 0, bb = 0;
+      for (auto& c : cands) {
+        // interior offsets fragment the hole: only where it is large (mode 2)
+        // or never (mode 1: choose among holes only)
+        const uint32_t nb = opt.lane_banks == 1 ? 1u : std::min<uint32_t>(16, c.first - k + 1);
+        for (uint32_t o = 0; o < nb; o++) {
+          const uint64_t key = ((uint64_t)run_cost(v, c.second + o) << 40) | ((uint64_t)c.first << 16) | o;
+          if (key < best) { best = key; bst = c.second; bb = c.second + o; }
+        }
+      }
+      // split the interval [bst, bst+len) around [bb, bb+k)
+      const uint32_t len = freeiv[bst];
+      freeiv.erase(bst);
+      if (bb > bst) freeiv[bst] = bb - bst;
+      if (bb + k < bst + len) freeiv[bb + k] = bst + len - (bb + k);
+      max_word = std::max(max_word, bb + k);
+      return bb;
     };
     std::vector<uint32_t> srcs;
     for (uint32_t i = 1; i < n; i++)
@@ -1192,7 +1265,7 @@ struct Mapper {
         auto& kv = *kvp;
         auto& v = kv.second;
         std::sort(v.begin(), v.end());
-        int64_t base = take((uint32_t)v.size());
+        int64_t base = banks ? take_banked(v) : take((uint32_t)v.size());
         if (base < 0) { fail(P, "lane state overflow"); return false; }
         UnitWo u;
         u.base = (uint32_t)base;
