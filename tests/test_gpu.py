@@ -213,6 +213,33 @@ def test_c5_ragged_stream_groups(gem):
     assert np.array_equal(sim.read_digests(T), r["digest"])
 
 
+@pytest.mark.parametrize("opts,dyn", [("parts=5 stages=2 lanes=1", "1"), ("parts=4 lanes=1", "0"),
+                                      ("parts=4 lanes=1", "1")])
+def test_lane_mode_stages_and_work_distribution(gem, monkeypatch, tmp_path, opts, dyn):
+    """Lane mode with two stages (static work lists, cut words between stages)
+    and one stage with static (GEM_LANE_DYN=0) or dynamic ticketed work
+    distribution: 96 streams match the 64-lane oracle bit-exactly."""
+    from paper_conf_dac_guozwlr25_b200.mapping import compile_file
+    S, T = 96, 50
+    net = circuits.small_G(seed=41, n_and=4000, with_ram=True)
+    path = circuits.save(net, str(tmp_path), "g")
+    b = compile_file(path, opts)
+    st = np.stack([stim_random(net.n_pi, T, 2000 + s, reset_pi0_cycles=2) for s in range(S)])
+    monkeypatch.setenv("GEM_LANE_DYN", dyn)
+    sim = gem.Simulator(b, n_streams=S, flags=gem.GEM_F_DIGEST, grid_limit=3)
+    assert sim.info["lanes"] == 1
+    sim.set_inputs(st)
+    sim.step(T)
+    po, dg = sim.read_outputs(T), sim.read_digests(T)
+    o = Oracle(path)
+    o.lanes_reset(2)
+    for g in range(2):
+        lo, hi = 64 * g, min(S, 64 * g + 64)
+        r = o.lanes_run(g, st[lo:hi], digest=True)
+        assert np.array_equal(po[lo:hi], r["po"]), g
+        assert np.array_equal(dg[lo:hi], r["digest"]), g
+
+
 @pytest.mark.parametrize("k", [4, 2])
 def test_lane_interleaved_groups_ragged(gem, monkeypatch, tmp_path, k):
     """150 streams = 5 lane groups: work items of K interleaved 32-stream groups
