@@ -1236,14 +1236,48 @@ struct Mapper {
       max_word = std::max(max_word, bb + k);
       return bb;
     };
+    // sources take the first lane words in port-list order (entry k -> word
+    // k + 1).  The list is sorted by global bit (a warp's port loads stay
+    // coalesced); with lane_banks, each aligned block of 16 entries -- the same
+    // addresses whichever lane loads them -- is permuted so its sources get
+    // the word residues that add the fewest same-residue readers.
     std::vector<uint32_t> srcs;
     for (uint32_t i = 1; i < n; i++)
-      if (is_src[i]) {
-        int64_t w = take(1);
-        if (w < 0) { fail(P, "lane state overflow"); return false; }
-        srcs.push_back(i);
-        bind(i, (uint32_t)w);
+      if (is_src[i]) srcs.push_back(i);
+    std::stable_sort(srcs.begin(), srcs.end(), [&](uint32_t x, uint32_t y) {
+      const uint32_t gx = G.gbit[cid[x]], gy = G.gbit[cid[y]];
+      const uint64_t kx = ((uint64_t)(gx >> 27) << 32) | (((gx >> 5) & 0x3FFFFF) * 32 + (gx & 31));
+      const uint64_t ky = ((uint64_t)(gy >> 27) << 32) | (((gy >> 5) & 0x3FFFFF) * 32 + (gy & 31));
+      return kx < ky;
+    });
+    if (banks) {
+      for (size_t b0 = 0; b0 < srcs.size(); b0 += 16) {
+        const size_t b1 = std::min(srcs.size(), b0 + 16);
+        std::vector<uint32_t> blk(srcs.begin() + b0, srcs.begin() + b1), out(b1 - b0, UINT32_MAX);
+        std::stable_sort(blk.begin(), blk.end(), [&](uint32_t x, uint32_t y) { return reads[x].size() > reads[y].size(); });
+        for (uint32_t x : blk) {
+          size_t best = SIZE_MAX;
+          uint32_t bc = UINT32_MAX;
+          for (size_t j = 0; j < out.size(); j++) {
+            if (out[j] != UINT32_MAX) continue;
+            const uint32_t wj = (uint32_t)(b0 + j + 1);
+            uint32_t c = 0;
+            for (uint32_t g : reads[x]) c += occ[(size_t)g * 16 + (wj & 15)];
+            if (c < bc) { bc = c; best = j; }
+          }
+          out[best] = x;
+          const uint32_t wb = (uint32_t)(b0 + best + 1);
+          for (uint32_t g : reads[x]) { uint8_t& o = occ[(size_t)g * 16 + (wb & 15)]; if (o < 255) o++; }
+        }
+        std::copy(out.begin(), out.end(), srcs.begin() + b0);
       }
+      std::fill(occ.begin(), occ.end(), 0);   // rebuilt by bind below
+    }
+    for (uint32_t x : srcs) {
+      int64_t w = take(1);
+      if (w < 0) { fail(P, "lane state overflow"); return false; }
+      bind(x, (uint32_t)w);
+    }
     // per layer: unit -> (mask, base)
     struct UnitWo { uint32_t mask = 0, base = 0; };
     std::vector<std::array<UnitWo, 256>> th(L);
