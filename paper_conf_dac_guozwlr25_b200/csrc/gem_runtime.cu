@@ -75,6 +75,7 @@ struct KParams {
   // (act_words >= max n_gread) and {evaluated, skipped} partition-cycle counters
   unsigned long long* act_cnt;
   uint32_t act_words;
+  float l2_frac;           // > 0: streamed program chunks keep this fraction evict_last in L2
   // lane mode, one stage: dynamic work distribution.  Units {partition, first
   // stream, items, 0} in LPT order; CTA b starts every cycle with unit b and
   // then takes tickets from dyn_ctr[cycle & 1] (+ grid).
@@ -256,6 +257,27 @@ __device__ __forceinline__ void tma_load_1d(void* dst, const void* src, uint32_t
       "l"(src), "r"(bytes), "r"(smem_u32(bar))
       : "memory");
 }
+// The same copy with an L2 cache-eviction policy (createpolicy): programs larger
+// than the L2 stream every cycle; keeping a fraction of their lines evict_last
+// (the rest evict_first) lets that fraction stay L2-resident across cycles.
+__device__ __forceinline__ void tma_load_1d_hint(void* dst, const void* src, uint32_t bytes, uint64_t* bar,
+                                                 uint64_t pol) {
+  asm volatile(
+      "cp.async.bulk.shared::cluster.global.mbarrier::complete_tx::bytes.L2::cache_hint [%0], [%1], %2, [%3], %4;" ::"r"(
+          smem_u32(dst)),
+      "l"(src), "r"(bytes), "r"(smem_u32(bar)), "l"(pol)
+      : "memory");
+}
+__device__ __forceinline__ uint64_t l2_policy(float frac) {
+  uint64_t pol;
+  asm volatile("createpolicy.fractional.L2::evict_last.L2::evict_first.b64 %0, %1;" : "=l"(pol) : "f"(frac));
+  return pol;
+}
+__device__ __forceinline__ uint64_t l2_policy_unchanged() {
+  uint64_t pol;
+  asm volatile("createpolicy.fractional.L2::evict_unchanged.b64 %0, 1.0;" : "=l"(pol));
+  return pol;
+}
 __device__ __forceinline__ void fence_mbar_init() {
   asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
 }
@@ -281,6 +303,7 @@ struct ProgSrc {
   // ring placed after them; pro_chunk/pro_off = next chunk after the prologue
   uint32_t pin_chunks, pin_off, pro_chunk, pro_off;
   const uint32_t* pin;
+  uint64_t l2pol;          // L2 policy of streamed chunks (KParams::l2_frac)
   uint32_t n_res;
   const uint32_t* res_p;   // smem [GEM_MAX_RESIDENT] partition ids
   const uint32_t* res_off; // smem [GEM_MAX_RESIDENT] word offsets into area
@@ -296,7 +319,7 @@ __device__ __forceinline__ void ring_issue(ProgSrc& ps, const uint32_t* g, uint3
   if (threadIdx.x == 0) {
     uint64_t* bar = ps.mbar + (seq & (ps.R - 1));
     mbar_expect_tx(bar, words * 4);
-    tma_load_1d(ring_slot(ps, seq), g, words * 4, bar);
+    tma_load_1d_hint(ring_slot(ps, seq), g, words * 4, bar, ps.l2pol);
   }
 }
 __device__ __forceinline__ const uint32_t* ring_wait(ProgSrc& ps) {
@@ -967,6 +990,7 @@ __global__ void __launch_bounds__(GEM_THREADS, 2) gem_step_kernel(const KParams 
   ps.seq_free = 0;
   ps.pin_chunks = res_n[2];
   ps.pin_off = res_n[3];
+  ps.l2pol = kp.l2_frac > 0.f ? l2_policy(kp.l2_frac) : l2_policy_unchanged();
   ps.pin = area;
   ps.pro_chunk = ps.pro_off = 0;
   if (ps.pin_chunks) {
@@ -1707,6 +1731,17 @@ int gem_step(gem_sim* sim, uint64_t ncycles) {
   kp.group = sim->group;
   kp.wl_items = sim->d_wl_items;
   kp.act_cnt = sim->d_act;
+  {
+    // programs larger than the L2 (C4): keep a fraction L2-resident (GEM_L2_FRAC overrides)
+    const char* fe = getenv("GEM_L2_FRAC");
+    int l2 = 0;
+    cudaDeviceGetAttribute(&l2, cudaDevAttrL2CacheSize, sim->device);
+    float f = 0.f;
+    if (!sim->lanes && sim->program_bytes > (uint64_t)l2)
+      f = std::min(0.9f, 0.6f * (float)l2 / (float)sim->program_bytes);
+    if (fe) f = (float)atof(fe);
+    kp.l2_frac = std::max(0.f, std::min(1.f, f));
+  }
   kp.dyn_units = sim->d_dyn_units;
   kp.n_units = sim->n_units;
   kp.dyn_ctr = sim->d_dyn_ctr;
