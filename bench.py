@@ -115,6 +115,37 @@ def ncu_traffic(cfg: str, kernel: str, cycles: int):
     return (best[1], best[2]) if best else (None, None)
 
 
+def ncu_pipes(cfg: str, kernel: str, cycles: int, n_sms: int, sm_mhz: float):
+    """Pipe utilisation of the same committed `--set full` capture as ncu_traffic:
+    shared-memory wavefronts per SM clock (peak 1), alu-pipe busy fraction and
+    issue IPC of the captured launch; None if no matching summary."""
+    import glob
+    import re
+    best = None
+    for f in glob.glob(os.path.join(ROOT, "profiles", "r*", f"ncu_{cfg}_*.json")):
+        try:
+            d = json.load(open(f))
+            if d.get("capture_cycles") != cycles or kernel not in d.get("kernel", kernel):
+                continue
+            mv = re.search(r"_v(\d+)\.json$", f)
+            key = (int(mv.group(1)) if mv else -1, os.path.getmtime(f))
+            if best is None or key > best[0]:
+                best = (key, d, os.path.relpath(f, ROOT))
+        except Exception:
+            continue
+    if best is None:
+        return None
+    c = best[1]["capture"]
+    dur_s = float(c["gpu__time_duration.sum"]) * {"ms": 1e-3, "us": 1e-6, "usecond": 1e-6, "msecond": 1e-3}.get(
+        best[1]["capture_units"].get("gpu__time_duration.sum", "ms"), 1e-3)
+    wf = float(c["l1tex__data_pipe_lsu_wavefronts_mem_shared.sum"])
+    return {"smem_wavefronts_per_launch": wf,
+            "smem_frac": wf / (dur_s * n_sms * sm_mhz * 1e6),
+            "smem_peak": "1 wavefront (128 B) per SM clock",
+            "alu_pipe_busy_frac": float(c["sm__pipe_alu_cycles_active.avg.pct_of_peak_sustained_active"]) / 100.0,
+            "ipc_per_sm": float(c["sm__inst_executed.avg.per_cycle_active"]), "source": best[2]}
+
+
 def dist_env():
     ws = int(os.environ.get("WORLD_SIZE", "1"))
     rank = int(os.environ.get("RANK", "0"))
@@ -398,6 +429,7 @@ def main():
                "algorithmic_bytes_per_launch": alg_bytes * C * S + info.program_bytes,
                "peak_gbs": float(peaks.get("hbm_gbs", 6650))}
         roof = dict(alu)
+        roof["pipes_ncu"] = ncu_pipes(cfg, kname, C, n_sms, float(peaks.get("sm_max_mhz", 1965.0)))
         roof.update({"traffic": traffic, "traffic_unit": "bytes per launch (dram read+write, ncu --set full)",
                      "traffic_source": traffic_src, "kernel": kname, "kernel_ms_per_step": kern_last,
                      "us_per_layer_critical": 1e6 / hz_kernel / max(1, info.max_layers), "alu": alu, "hbm": hbm})
