@@ -200,10 +200,12 @@ enum {
  *                      mask keeps slot-bit order)
  *            [136..648) leaves: [4 groups][32 lanes] uint4 (32 u16 lane-word byte offsets w*4
  *                       per lane, entry 8g+2k low half, 8g+2k+1 high half)
- *            [648..680) per-lane write-out base word
+ *            [648..680) per-lane write-out base words: level-1 slots (bits 0-15) from the
+ *                       low 16 bits, levels 2-5 (bits 16-30) from the high 16 bits
  *   Write-outs: a unit (thread / warp / top) stores the slots whose bits are set
  *   in its mask, in slot-bit order, to consecutive lane words from its base:
- *   slot b -> base + popc(mask & ((1 << b) - 1)).
+ *   slot b -> base + popc(mask & ((1 << b) - 1)); thread units write two such
+ *   runs (levels 1 and 2-5, bases in the low / high half of the base word).
  *   out:   uint2 {dst gid_l, src lane word | GEM_OUT_INV}
  *   ram:   4 words per owned RAM {ram_id, 0, 0, 0}
  * Lane word 0 is the constant 0.                                            */

@@ -159,7 +159,7 @@ __device__ __forceinline__ void exec_lane_layer(const LaneRegs& R, uint32_t s_ba
       return (i & 1) ? (q >> 16) : (q & 0xFFFFu);
     };
     // written slots go to consecutive lane words (slot-bit order) from R.base
-    uint32_t wp = s_base + 4u * K * R.base;
+    uint32_t wp = s_base + 4u * K * (R.base & 0xFFFFu);   // level-1 run
     uint32_t r1[16][K];
 #pragma unroll
     for (uint32_t q = 0; q < 16; q++) {          // level 1: A = leaf q, B = leaf q+16
@@ -176,6 +176,7 @@ __device__ __forceinline__ void exec_lane_layer(const LaneRegs& R, uint32_t s_ba
 #endif
     }
     uint32_t r2[8][K], r3[4][K], r4[2][K], x[K];
+    wp = s_base + 4u * K * (R.base >> 16);                // levels 2-5 run
 #pragma unroll
     for (uint32_t q = 0; q < 8; q++) {
       kslotp<K>(r2[q], r1[q], r1[q + 8], xa, xb, ob, 16 + q);

@@ -1299,16 +1299,29 @@ struct Mapper {
         auto& kv = *kvp;
         auto& v = kv.second;
         std::sort(v.begin(), v.end());
-        int64_t base = banks ? take_banked(v) : take((uint32_t)v.size());
-        if (base < 0) { fail(P, "lane state overflow"); return false; }
-        UnitWo u;
-        u.base = (uint32_t)base;
-        for (size_t k = 0; k < v.size(); k++) {
-          u.mask |= 1u << v[k].first;
-          bind(v[k].second, (uint32_t)base + (uint32_t)k);
-          birth[v[k].second] = (int32_t)l;
-        }
         uint32_t kind = kv.first >> 16, unit = kv.first & 0xFFFF;
+        UnitWo u;
+        // thread units write two runs (gem_isa.h): level-1 slots (bits < 16)
+        // and levels 2-5 (bits >= 16), so shorter runs fit the holes
+        const size_t split = kind == 0 ? (size_t)(std::lower_bound(v.begin(), v.end(), std::make_pair(16u, 0u)) - v.begin())
+                                       : v.size();
+        for (int part = 0; part < (kind == 0 ? 2 : 1); part++) {
+          std::vector<std::pair<uint32_t, uint32_t>> r(part == 0 ? v.begin() : v.begin() + split,
+                                                       part == 0 ? v.begin() + split : v.end());
+          uint32_t b0 = 0;
+          if (!r.empty()) {
+            int64_t base = banks ? take_banked(r) : take((uint32_t)r.size());
+            if (base < 0) { fail(P, "lane state overflow"); return false; }
+            b0 = (uint32_t)base;
+            for (size_t k = 0; k < r.size(); k++) {
+              u.mask |= 1u << r[k].first;
+              bind(r[k].second, b0 + (uint32_t)k);
+              birth[r[k].second] = (int32_t)l;
+            }
+          }
+          if (kind == 0) u.base |= b0 << (16 * part);
+          else u.base = b0;
+        }
         if (kind == 0) th[l][unit] = u;
         else if (kind == 1) wa[l][unit] = u;
         else tp[l] = u;

@@ -288,10 +288,15 @@ int run_lane_part(Interp& I, LaneSim& Ls, uint32_t p, const uint32_t* pi_lane /*
       k_out = unit_kind == 0 ? kk : kk + 5;
       id_out = unit * gw(k_out) + q;
     };
+    // thread units (kind 0) write two runs: level-1 slots (bits 0-15) from the
+    // low 16 bits of base, levels 2-5 (bits 16-30) from the high 16 bits
     auto do_wo = [&](int kind, uint32_t unit, uint32_t mask, uint32_t base) -> int {
       for (uint32_t bit = 0; bit < 31; bit++) {
         if (!((mask >> bit) & 1u)) continue;
         uint32_t word = base + (uint32_t)__builtin_popcount(mask & ((1u << bit) - 1u));
+        if (kind == 0)
+          word = bit < 16 ? (base & 0xFFFFu) + (uint32_t)__builtin_popcount(mask & ((1u << bit) - 1u))
+                          : (base >> 16) + (uint32_t)__builtin_popcount(mask & ((1u << bit) - 1u) & 0xFFFF0000u);
         if (word == 0 || word >= S.size()) { g_err = "bad lane write-out"; return -1; }
         if (read[word]) { g_err = "lane write-out target read in the same layer"; return -1; }
         int k; uint32_t id;
