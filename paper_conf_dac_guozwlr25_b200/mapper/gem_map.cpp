@@ -69,6 +69,7 @@ struct Options {
   int max_parts = 280;      // refinement stops growing the partition count here
   int lanes = 0;            // also emit stream-sliced lane programs (batched streams)
   int lane_words = 16383;   // cap on a lane program's state words (larger partitions are split)
+  int max_warps = 8;        // warps that may hold placed roots (8 = all)
   int lane_banks = 1;       // bank-aware placement of lane write-out runs (2: also interior offsets)
   int lane_holes = 32;      // best-fitting holes considered per run
   int banks = 1;            // bank-conflict-aware renaming of the state words (rename_state_words)
@@ -106,6 +107,7 @@ static Options parse_opts(const char* s) {
     else if (k == "lanes") o.lanes = std::stoi(v);
     else if (k == "lane_words") o.lane_words = std::min(16383, std::stoi(v));
     else if (k == "lane_banks") o.lane_banks = std::stoi(v);
+    else if (k == "max_warps") o.max_warps = std::max(1, std::min(8, std::stoi(v)));
     else if (k == "lane_holes") o.lane_holes = std::max(1, std::stoi(v));
     else if (k == "banks") o.banks = std::stoi(v);
     else throw std::runtime_error("unknown option " + k);
@@ -712,6 +714,14 @@ struct Mapper {
             uint32_t ka = (a % 32) * 8 + a / 32, kb = (b % 32) * 8 + b / 32;
             return ka < kb;
           });
+        }
+        // max_warps < 8: roots only in the first max_warps warps (a small
+        // design's layers then run in one warp: no cross-warp wait per layer)
+        if (opt.max_warps < 8) {
+          auto warp_of = [&](uint32_t u) { return k <= 5 ? u / 32 : k <= 10 ? u : 0u; };
+          unit_order.erase(std::remove_if(unit_order.begin(), unit_order.end(),
+                                          [&](uint32_t u) { return k > 10 || warp_of(u) >= (uint32_t)opt.max_warps; }),
+                           unit_order.end());
         }
         for (uint32_t q = 0; q < g; q++)
           for (uint32_t u : unit_order)
