@@ -1736,12 +1736,12 @@ int gem_step(gem_sim* sim, uint64_t ncycles) {
   kp.wl_items = sim->d_wl_items;
   kp.act_cnt = sim->d_act;
   {
-    // programs larger than the L2 (C4): keep a fraction L2-resident (GEM_L2_FRAC overrides)
+    // programs larger than half the L2 (C4): keep a fraction L2-resident (GEM_L2_FRAC overrides)
     const char* fe = getenv("GEM_L2_FRAC");
     int l2 = 0;
     cudaDeviceGetAttribute(&l2, cudaDevAttrL2CacheSize, sim->device);
     float f = 0.f;
-    if (!sim->lanes && sim->program_bytes > (uint64_t)l2)
+    if (!sim->lanes && 2 * sim->program_bytes > (uint64_t)l2)   // does not stay resident by itself
       f = std::min(0.9f, 0.6f * (float)l2 / (float)sim->program_bytes);
     if (fe) f = (float)atof(fe);
     kp.l2_frac = std::max(0.f, std::min(1.f, f));

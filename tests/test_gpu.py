@@ -291,13 +291,15 @@ def test_c5_lane_mode_equals_packed_mode(gem, monkeypatch):
     assert np.array_equal(lane.read_state(), q)
 
 
-def test_c4_sampled_window(gem):
-    """C4 (~10M ANDs, 2 stages, 24 RAM blocks): full PO trace and per-cycle flop
-    digests for a window the oracle finishes in seconds, plus final state."""
+@pytest.mark.parametrize("opts,stages", [(None, 1), ("stages=2 levels=10 key=2 part_size=20000", 2)])
+def test_c4_sampled_window(gem, opts, stages):
+    """C4 (~10M ANDs, 24 RAM blocks) as bench.py maps it (one stage) and with a
+    two-stage RepCut mapping: full PO trace and per-cycle flop digests
+    for a window the oracle finishes in seconds, plus final state and RAMs."""
     T = 60
     st = stimulus("c4", 512, T)
-    sim = gem.Simulator(blob("c4"), flags=gem.GEM_F_DIGEST)
-    assert sim.info["n_stages"] == 2
+    sim = gem.Simulator(blob("c4", opts), flags=gem.GEM_F_DIGEST)
+    assert sim.info["n_stages"] == stages
     sim.set_inputs(st)
     sim.step(T)
     o = Oracle(eaig("c4"))
