@@ -480,10 +480,14 @@ def main():
             if hz_kernel / hbm_floor > hz_kernel / floor_hz:
                 roof.update({"bound": "hbm", "achieved": info.program_bytes * hz_kernel / 1e9,
                              "peak": float(peaks.get("hbm_gbs", 6650)), "unit": "GB/s",
-                             "frac": hz_kernel / hbm_floor})
+                             "frac": hz_kernel / hbm_floor,
+                             "algorithmic": "program bytes per cycle (the whole program streamed from HBM)",
+                             "peak_source": f"MEASURED_PEAKS.json hbm_gbs ({peaks['_source']})"})
                 roof["binding"] = "hbm (program not L2-resident, streamed every cycle)"
             else:
                 roof.update({k: lat[k] for k in ("bound", "achieved", "peak", "unit", "frac")})
+                roof.update({"algorithmic": "simulated cycles per second of one stream",
+                             "peak_source": "latency floor (gem_bench_floor, measured in this run)"})
                 roof["binding"] = "latency"
         else:
             roof["binding"] = "alu (independent streams: issue of LOP3/LDS per lane word)"
