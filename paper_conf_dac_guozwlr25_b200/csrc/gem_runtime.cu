@@ -1189,6 +1189,7 @@ struct gem_sim {
   uint32_t *d_pi = nullptr, *d_po = nullptr, *d_qtrace = nullptr, *d_scratch = nullptr, *d_wl_off = nullptr;
   uint2* d_wl_items = nullptr;
   unsigned long long *d_digest = nullptr, *d_bar = nullptr, *d_prof = nullptr, *d_fprof = nullptr;
+  size_t bar_off = 0;  // experiment (GEM_EXP_BAR_SHIFT_KB): barrier flags placed this many u64 into d_bar
   uint32_t prof_cycles = 0;
   int* d_err = nullptr;
   uint32_t in_cap = 0, in_queued = 0, in_head = 0, out_cap = 0, last_cycles = 0;
@@ -1621,7 +1622,8 @@ int gem_load_program(const void* blob, size_t nbytes, const gem_config* cfg, gem
     CK(dalloc(&sim->d_cut, S * std::max<uint32_t>(sim->cut_words, 1) * 4));
   }
   CK(dalloc(&sim->d_mem, S * sim->n_rams * (size_t)GEM_RAM_WORDS * 4));
-  CK(dalloc(&sim->d_bar, (size_t)(GEM_BAR_MAX_CTAS + 2) * GEM_BAR_STRIDE * 8));
+  if (const char* e = getenv("GEM_EXP_BAR_SHIFT_KB")) sim->bar_off = (size_t)atoi(e) * 128;
+  CK(dalloc(&sim->d_bar, (size_t)(GEM_BAR_MAX_CTAS + 2) * GEM_BAR_STRIDE * 8 + sim->bar_off * 8));
   CK(dalloc(&sim->d_err, 64));
   CK(cudaMemset(sim->d_err, 0, 64));
   CK(dalloc(&sim->d_act, 16));
@@ -1722,7 +1724,7 @@ int gem_step(gem_sim* sim, uint64_t ncycles) {
   kp.prog = sim->d_prog; kp.parts = sim->d_parts; kp.stage_list = sim->d_stage;
   kp.pi = sim->d_pi; kp.po = sim->d_po; kp.q = sim->d_q; kp.rd = sim->d_rd; kp.cut = sim->d_cut;
   kp.mem = sim->d_mem; kp.q_trace = sim->d_qtrace; kp.digest = sim->d_digest;
-  kp.q_int_of_ext = sim->d_q_int_of_ext; kp.bar = sim->d_bar; kp.err = sim->d_err;
+  kp.q_int_of_ext = sim->d_q_int_of_ext; kp.bar = sim->d_bar + sim->bar_off; kp.err = sim->d_err;
   kp.t0 = sim->cycle; kp.ncycles = (uint32_t)ncycles; kp.in_base = sim->in_head; kp.in_cap = sim->in_cap;
   kp.out_cap = sim->out_cap; kp.n_stages = sim->n_stages; kp.n_streams = sim->n_streams;
   kp.state_words = sim->state_words; kp.pi_words = sim->pi_words; kp.po_words = sim->po_words_int;
@@ -1768,7 +1770,7 @@ int gem_step(gem_sim* sim, uint64_t ncycles) {
     kp.fprof = sim->d_fprof;
     kp.fine_cta = getenv("GEM_FINE_CTA") ? (uint32_t)atoi(getenv("GEM_FINE_CTA")) : 0u;
   }
-  CK(cudaMemsetAsync(sim->d_bar, 0, (size_t)(GEM_BAR_MAX_CTAS + 2) * GEM_BAR_STRIDE * 8, sim->stream));
+  CK(cudaMemsetAsync(sim->d_bar + sim->bar_off, 0, (size_t)(GEM_BAR_MAX_CTAS + 2) * GEM_BAR_STRIDE * 8, sim->stream));
   if (sim->flags & GEM_F_DIGEST)
     CK(cudaMemsetAsync(sim->d_digest, 0, (size_t)sim->n_streams * sim->out_cap * 8, sim->stream));
   if (sim->lanes) {
