@@ -58,6 +58,15 @@ extern "C" {
  * single-stream launch whose grid covers the partitions); other CTAs, and lane
  * mode, always evaluate.  The first cycle of every gem_step evaluates. */
 #define GEM_F_ACTIVITY 0x10u
+/* Launch-mode overrides (tests and measurements; results are identical):
+ *   GEM_F_NO_RESIDENT  stream every program chunk through the TMA ring (no
+ *                      shared-memory residency, no pinned prefix);
+ *   GEM_F_NO_LANES     batched streams on the bit-packed path (no lane mode);
+ *   GEM_F_STATIC_LANES lane mode with static LPT work lists instead of the
+ *                      dynamic (ticketed) distribution. */
+#define GEM_F_NO_RESIDENT 0x20u
+#define GEM_F_NO_LANES 0x40u
+#define GEM_F_STATIC_LANES 0x80u
 
 typedef struct gem_sim gem_sim; /* opaque, owned by the library */
 
@@ -67,6 +76,18 @@ typedef struct {
   void* cuda_stream;    /* cudaStream_t to launch on, or NULL for a private stream */
   uint32_t flags;       /* GEM_F_*                                                 */
   uint32_t grid_limit;  /* 0 = auto (co-resident persistent grid); else max CTAs   */
+  /* Launch tuning (0 = automatic; none of these changes results, only speed).
+   * Bit-packed path: */
+  uint32_t ctas_per_sm;      /* CTAs per SM (1..4)                                   */
+  uint32_t max_group;        /* max streams sharing one work item (1..15)            */
+  /* Lane mode (batched streams): */
+  uint32_t lane_groups;      /* 32-stream groups per work item K (1, 2 or 4)          */
+  uint32_t lane_ctas_per_sm; /* CTAs per SM (1 or 2)                                  */
+  uint32_t lane_run;         /* work items per scheduling unit                        */
+  /* L2 residency of streamed program chunks: fraction kept evict_last
+   * (0 = automatic: a share of the L2 for programs larger than half of it;
+   * > 0 = that fraction; < 0 = no eviction policy). */
+  float l2_evict_last;
 } gem_config;
 
 typedef struct {
@@ -83,39 +104,75 @@ typedef struct {
   uint64_t cycle;                          /* cycles simulated so far              */
 } gem_info;
 
-/* Load a .gemb program blob (mapper output), allocate device state for
- * cfg->n_streams streams; flops start at their AIGER init values, RAMs at 0
- * (readings U5, U10).  blob: host memory, nbytes bytes; copied. */
+/* Compile step's output -> executable simulator (§II P:41 "compile
+ * [the netlist] into an executable simulator"; §III-E P:178-196 the bitstream).
+ * blob: host memory, nbytes bytes, the .gemb of gem_map.h; copied, not retained.
+ * Allocates device state for cfg->n_streams independent streams: flops start at
+ * their AIGER init values (uninitialised latches at 0, reading U5), RAM read
+ * registers and RAM contents at 0 (U10).  *out receives the handle (NULL on
+ * failure).  Errors: GEM_E_INVAL (null/size/n_streams 0/bad device),
+ * GEM_E_FORMAT (bad magic, version, truncated or inconsistent tables),
+ * GEM_E_UNSUPPORTED (no CUDA device; state or program ring does not fit in
+ * shared memory; a partition with more than GEM_MAX_CHUNKS-2 layers),
+ * GEM_E_NOMEM, GEM_E_CUDA.  On failure nothing is leaked. */
 int gem_load_program(const void* blob, size_t nbytes, const gem_config* cfg, gem_sim** out);
 
+/* Static facts of the loaded program and the chosen launch (host struct). */
 int gem_info_get(const gem_sim* sim, gem_info* out);
 
-/* Queue ncycles of primary-input vectors for every stream:
- * pi_words = uint32 [n_streams][ncycles][pi_words] (host, or device if
- * src_on_device).  Replaces any inputs not yet consumed. */
+/* Input stimuli ("executes it with input stimuli", one PI vector per
+ * cycle applied before that cycle's evaluation, reading U12).
+ * pi_words = uint32 [n_streams][ncycles][pi_words], PI order as above.
+ * Replaces any inputs not yet consumed.  Host buffers: copied before return
+ * (the caller may reuse the buffer, pinned or not, immediately).
+ * src_on_device = 1 (a deviation from SURVEY §8(b), which has host buffers
+ * only): pi_words is a device pointer on the handle's device, copied
+ * asynchronously on the handle's stream (the caller keeps it alive until the
+ * next gem_step has been enqueued).  Errors: GEM_E_INVAL (null with
+ * ncycles > 0, ncycles > 2^32-16), GEM_E_NOMEM, GEM_E_CUDA. */
 int gem_set_inputs(gem_sim* sim, const uint32_t* pi_words, uint64_t ncycles, int src_on_device);
 
-/* Simulate ncycles cycles (consumes ncycles queued input vectors) with one
- * persistent cooperative kernel launch.  After return, state = Q[t0+ncycles]. */
+/* Simulate ncycles clock cycles (cycle by cycle, synchronous,
+ * 2-state; oblivious full-cycle evaluation P:46) with one persistent
+ * cooperative kernel launch: per cycle and stage, every partition reads its
+ * input ports once, runs its boomerang layers, commits flops,
+ * POs and RAM ports, then a grid barrier.  Consumes
+ * ncycles queued input vectors.  After return (or, with GEM_F_ASYNC, after the
+ * stream reaches it) the state is Q[t0+ncycles].  ncycles = 0 is a no-op.
+ * Errors: GEM_E_NOINPUT (fewer than ncycles queued), GEM_E_CUDA (including a
+ * grid-barrier watchdog trap, reported in gem_last_error; handle poisoned). */
 int gem_step(gem_sim* sim, uint64_t ncycles);
 
-/* PO[t0 .. t0+ncycles-1] of the last gem_step, sampled before each clock edge
- * (reading U11): uint32 [n_streams][ncycles][po_words]. */
+/* Outputs ("producing output"): PO[t0 .. t0+ncycles-1] of the last
+ * gem_step, each sampled after the cycle's combinational evaluation and before
+ * its clock edge (reading U11): uint32 [n_streams][ncycles][po_words], AIGER
+ * output order.  dst: host memory, or a device pointer if dst_on_device
+ * (the multi-GPU gather reads straight into a torch CUDA tensor).  Synchronous.
+ * Errors: GEM_E_INVAL (null dst, ncycles > cycles of the last step). */
 int gem_read_outputs(gem_sim* sim, uint32_t* po_words, uint64_t ncycles, int dst_on_device);
 
-/* Current flop vector: uint32 [n_streams][q_words], AIGER latch order. */
+/* Flop state Q (the only state besides RAMs): uint32 [n_streams][q_words],
+ * AIGER latch order; read after the last step, written before the next one
+ * (checkpoint / resume).  Host or device buffers as flagged.
+ * Synchronous.  Errors: GEM_E_INVAL (null). */
 int gem_read_state(gem_sim* sim, uint32_t* flop_words, int dst_on_device);
 int gem_write_state(gem_sim* sim, const uint32_t* flop_words, int src_on_device);
 
-/* Needs GEM_F_TRACE_STATE: Q(t+1) for every cycle of the last step,
- * uint32 [n_streams][ncycles][q_words] (host). */
+/* Parity instrument (SURVEY §8(c) protocol), needs GEM_F_TRACE_STATE: Q(t+1)
+ * for every cycle of the last step, uint32 [n_streams][ncycles][q_words]
+ * (host).  Errors: GEM_E_INVAL (flag not set, ncycles too large). */
 int gem_read_state_trace(gem_sim* sim, uint32_t* dst, uint64_t ncycles);
 
-/* Needs GEM_F_DIGEST: d_t = sum_w rotl64(zext64(Qw), w mod 64) * (2w+1) mod 2^64
- * over the external flop words of Q(t+1); uint64 [n_streams][ncycles] (host). */
+/* Parity instrument, needs GEM_F_DIGEST: per-cycle flop digest
+ * d_t = sum_w rotl64(zext64(Qw), w mod 64) * (2w+1) mod 2^64 over the external
+ * flop words of Q(t+1); uint64 [n_streams][ncycles] (host). */
 int gem_read_digests(gem_sim* sim, uint64_t* dst, uint64_t ncycles);
 
-/* RAM block contents (8192 x 32-bit words) of one stream (host buffers). */
+/* RAM block contents (8192 x 32-bit words: "13 bits address and 32 bits data",
+ * P:93) of one stream, host buffers of 8192 words.  gem_write_ram preloads a
+ * block before the next step (U10: otherwise 0); the registered read data RD
+ * is not changed (it holds the last read, 0 before the first cycle).
+ * Synchronous.  Errors: GEM_E_INVAL (null, ram_id >= n_rams, stream >= n_streams). */
 int gem_read_ram(gem_sim* sim, uint32_t ram_id, uint32_t stream, uint32_t* words8192);
 int gem_write_ram(gem_sim* sim, uint32_t ram_id, uint32_t stream, const uint32_t* words8192);
 

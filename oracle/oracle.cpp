@@ -702,6 +702,23 @@ int orc_lanes_get_state(void* h, uint64_t g, uint64_t lane, uint32_t* words) {
   return 0;
 }
 
+// RAM block r of lane `lane` in 64-lane group g (state access only, no arithmetic)
+int orc_lanes_get_ram(void* h, uint64_t g, uint64_t lane, uint32_t r, uint32_t* words) {
+  Oracle* o = (Oracle*)h;
+  if (g >= o->n_groups || lane >= 64 || r >= o->rams.size()) { g_err = "bad lane ram"; return -1; }
+  const uint32_t* m = &o->gMEM[g][(r * 64 + lane) * (size_t)kRamWords];
+  for (int k = 0; k < kRamWords; k++) words[k] = m[k];
+  return 0;
+}
+
+int orc_lanes_set_ram(void* h, uint64_t g, uint64_t lane, uint32_t r, const uint32_t* words) {
+  Oracle* o = (Oracle*)h;
+  if (g >= o->n_groups || lane >= 64 || r >= o->rams.size()) { g_err = "bad lane ram"; return -1; }
+  uint32_t* m = &o->gMEM[g][(r * 64 + lane) * (size_t)kRamWords];
+  for (int k = 0; k < kRamWords; k++) m[k] = words[k];
+  return 0;
+}
+
 uint64_t orc_digest(const uint32_t* words, uint64_t nw) { return digest_words(words, nw); }
 
 }  // extern "C"

@@ -49,6 +49,8 @@ def _load():
             lib.orc_lanes_reset.argtypes = [P, u64]
             lib.orc_lanes_run.argtypes = [P, u64, u64, P, u64, P, P, P]
             lib.orc_lanes_get_state.argtypes = [P, u64, u64, P]
+            lib.orc_lanes_get_ram.argtypes = [P, u64, u64, ctypes.c_uint32, P]
+            lib.orc_lanes_set_ram.argtypes = [P, u64, u64, ctypes.c_uint32, P]
             lib.orc_digest.argtypes = [P, u64]
             lib.orc_digest.restype = u64
             _lib = lib
@@ -184,3 +186,15 @@ class Oracle:
         out = np.zeros(self.q_words, np.uint32)
         self._lib.orc_lanes_get_state(self._h, group, lane, _ptr(out))
         return out
+
+    def lanes_get_ram(self, group: int, lane: int, r: int) -> np.ndarray:
+        out = np.zeros(8192, np.uint32)
+        if self._lib.orc_lanes_get_ram(self._h, group, lane, r, _ptr(out)):
+            raise ValueError(self._lib.orc_last_error().decode())
+        return out
+
+    def lanes_set_ram(self, group: int, lane: int, r: int, words: np.ndarray):
+        w = np.ascontiguousarray(words, dtype=np.uint32)
+        assert len(w) == 8192
+        if self._lib.orc_lanes_set_ram(self._h, group, lane, r, _ptr(w)):
+            raise ValueError(self._lib.orc_last_error().decode())

@@ -48,6 +48,7 @@
 #define GEM_RAM_ABITS 13        /* P:93 */
 #define GEM_RAM_WORDS 8192
 #define GEM_MAX_RAMS_PER_PART 32
+#define GEM_MAX_CHUNKS 256      /* chunks per partition program (= layers + 2)      */
 
 /* global word regions (gid = region << 24 | index) */
 #define GEM_R_PI 0u     /* gread source: PI word of the current cycle        */

@@ -138,11 +138,7 @@ __device__ __forceinline__ void lane_woK(uint32_t s_base, uint32_t mask, uint32_
 template <int K>
 __device__ __forceinline__ void exec_lane_layer(const LaneRegs& R, uint32_t s_base, uint32_t* topv, uint32_t bid) {
   const uint32_t lane = threadIdx.x & 31, warp = threadIdx.x >> 5;
-#ifdef EXP_LANE_NOTOP   // timing experiment: no levels 11-13 hand-off
-  const bool uses_top = false;
-#else
   const bool uses_top = (R.flags & GEM_LF_USES_TOP) != 0;
-#endif
   if ((R.flags >> warp) & 1u) {
     const uint32_t xa = R.lc.x, xb = R.lc.y, ob = R.lc.z, mask = R.lc.w;
     const uint32_t q8[4][4] = {{R.e[0].x, R.e[0].y, R.e[0].z, R.e[0].w}, {R.e[1].x, R.e[1].y, R.e[1].z, R.e[1].w},
@@ -153,9 +149,6 @@ __device__ __forceinline__ void exec_lane_layer(const LaneRegs& R, uint32_t s_ba
     // pointer (LDS [R + UR]: one extract per leaf, no address arithmetic)
     auto leaf = [&](uint32_t i) -> uint32_t {
       const uint32_t q = q8[i >> 3][(i & 7) >> 1];
-#ifdef EXP_LANE_NOCONFLICT   // timing experiment only: conflict-free leaf reads (wrong results)
-      return ((q & 0x3E0u) | lane) * 4u;
-#endif
       return (i & 1) ? (q >> 16) : (q & 0xFFFFu);
     };
     // written slots go to consecutive lane words (slot-bit order) from R.base
@@ -164,16 +157,10 @@ __device__ __forceinline__ void exec_lane_layer(const LaneRegs& R, uint32_t s_ba
 #pragma unroll
     for (uint32_t q = 0; q < 16; q++) {          // level 1: A = leaf q, B = leaf q+16
       uint32_t a[K], b[K];
-#ifdef EXP_LANE_NOLEAF   // timing experiment only: leaves from registers (wrong results)
-      for (int j = 0; j < K; j++) { a[j] = leaf(q) ^ lane; b[j] = leaf(q + 16) + lane; }
-#else
       lds_leaf<K>(s_base, leaf(q), a);
       lds_leaf<K>(s_base, leaf(q + 16), b);
-#endif
       kslotp<K>(r1[q], a, b, xa, xb, ob, q);
-#ifndef EXP_LANE_NOWO   // timing experiment: no write-outs of levels 1-5
       if (mask & (1u << q)) { stsK<K>(wp, r1[q]); wp += 4u * K; }
-#endif
     }
     uint32_t r2[8][K], r3[4][K], r4[2][K], x[K];
     wp = s_base + 4u * K * (R.base >> 16);                // levels 2-5 run
@@ -197,7 +184,6 @@ __device__ __forceinline__ void exec_lane_layer(const LaneRegs& R, uint32_t s_ba
     // levels 6-10 across the warp: slot q of a level lives in lane q
     const uint32_t wxa = R.wc.x, wxb = R.wc.y, wob = R.wc.z, wmask = R.wc.w;
     const uint32_t offs[5] = {0, 16, 24, 28, 30};
-#ifndef EXP_LANE_NOWARP   // timing experiment: no levels 6-10
 #pragma unroll
     for (uint32_t k = 0; k < 5; k++) {
       const uint32_t half = 16u >> k;
@@ -208,7 +194,6 @@ __device__ __forceinline__ void exec_lane_layer(const LaneRegs& R, uint32_t s_ba
       kslot<K>(x, x, y, wxa, wxb, wob, b);
       if (lane < half) lane_woK<K>(s_base, wmask, R.wbase, b, x);
     }
-#endif
     if (uses_top && lane == 0) {
 #pragma unroll
       for (int j = 0; j < K; j++) topv[warp * K + j] = x[j];
@@ -340,11 +325,7 @@ __device__ void run_lane_partition(const KParams& kp, uint32_t* S, uint32_t* ram
   phase(2);
   for (uint32_t l = 0; l < n_layers; l++) {
     exec_lane_layer<K>(R, s_base, topv, 1);
-#ifdef EXP_LANE_NOTOP
-    const bool ptop = false;
-#else
     const bool ptop = (R.flags & GEM_LF_USES_TOP) != 0;
-#endif
     const uint32_t ptopc = R.topc, ptopwo = R.topwo;
     L += R.size;
     if (l + 1 < n_layers) load_lane_next(L, R);

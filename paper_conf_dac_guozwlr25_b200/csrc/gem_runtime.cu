@@ -52,7 +52,7 @@ struct KParams {
   unsigned long long* digest;               // [stream][out_cap]
   const uint32_t* __restrict__ q_int_of_ext;  // [n_flops] internal bit
   unsigned long long* bar;                  // grid barrier: per-CTA arrival flags
-  int* err;
+  uint32_t* err;                            // mapped pinned host words {code, cta, flag, epoch}
   uint64_t t0;
   uint32_t ncycles, in_base, in_cap, out_cap;
   uint32_t n_stages, n_streams, state_words;
@@ -67,8 +67,6 @@ struct KParams {
   const uint32_t* __restrict__ pi_lane;  // [in_cap][pi_words*32][n_groups]
   uint32_t* po_lane;                     // [out_cap][po_words*32][n_groups]
   uint32_t n_groups, ramp_words;
-  unsigned long long* fprof;             // debug builds (GEM_FINE_PROF) only
-  uint32_t fine_cta;                     // CTA stamped by GEM_FINE_PROF builds (env GEM_FINE_CTA)
   const uint32_t* __restrict__ wl_off;   // [n_stages][grid+1] CSR offsets into wl_items
   const uint2* __restrict__ wl_items;    // {partition, stream} per work item
   // GEM_F_ACTIVITY (row f3): per-CTA copy of the last input-port words
@@ -83,29 +81,6 @@ struct KParams {
   uint32_t n_units;
   uint32_t* dyn_ctr;
 };
-#ifdef GEM_FINE_PROF
-// sub-stamps inside exec_layer: fl = layer index when stamping, >= 32 otherwise;
-// fsub = kp.fprof + 2048 ([layer 32][warp 8][4])
-#define GEM_FINE_LAYERS 32
-#define FSUB(l_, k_)                                                                          \
-  do {                                                                                        \
-    if ((l_) < GEM_FINE_LAYERS && (threadIdx.x & 31) == 0)                                    \
-      fsub[((l_) * 8 + (threadIdx.x >> 5)) * 4 + (k_)] = clock64();                           \
-  } while (0)
-#else
-#define FSUB(l_, k_) do { } while (0)
-#endif
-#ifdef GEM_FINE_PROF
-// debug build only: per-warp stamps inside the first 32 layers of cycle 5, CTA kp.fine_cta
-#define FPROF(l_, slot_)                                                                      \
-  do {                                                                                        \
-    if (kp.fprof && c == 5 && blockIdx.x == kp.fine_cta && (l_) < GEM_FINE_LAYERS &&         \
-        (threadIdx.x & 31) == 0)                                                              \
-      kp.fprof[((l_) * 8 + (threadIdx.x >> 5)) * 8 + (slot_)] = clock64();                    \
-  } while (0)
-#else
-#define FPROF(l_, slot_) do { } while (0)
-#endif
 #define PROF(slot_)                                                                          \
   do {                                                                                       \
     if (prof_on && threadIdx.x == 0)                                                         \
@@ -129,71 +104,45 @@ __device__ __forceinline__ uint64_t globaltimer_ns() {
 // epoch with st.release.gpu (cumulative over the CTA's writes ordered before it
 // by the bar.sync).  Wait: thread f polls CTA f's flag with ld.acquire.gpu (all
 // flags in parallel, no single contended counter), then bar.sync.  A 10 s spin
-// limit turns a deadlock (e.g. broken co-residency) into a trapped kernel.
+// limit turns a deadlock (e.g. broken co-residency) into a trapped kernel; the
+// watchdog first writes {code, CTA, flag, epoch} to mapped pinned host memory
+// (KParams::err), which the host reads after the failed synchronisation so the
+// error message names the stuck barrier (the context itself is lost).
+// (Measured alternatives: relaxed polling + one fence, a
+// two-phase gather by CTA 0, a single red.release counter: all slower.)
 #define GEM_BAR_STRIDE 16   /* u64 words between flags (128 bytes) */
 #define GEM_BAR_MAX_CTAS 1024
+#define GEM_WATCHDOG_NS 10000000000ull
+#define GEM_ERR_BARRIER 2u
 __device__ __forceinline__ void st_release_u64(unsigned long long* p, unsigned long long v) {
   asm volatile("st.release.gpu.global.u64 [%0], %1;" ::"l"(p), "l"(v) : "memory");
 }
-__device__ __forceinline__ unsigned long long ld_relaxed_u64(const unsigned long long* p) {
-  unsigned long long v;
-  asm volatile("ld.relaxed.gpu.global.u64 %0, [%1];" : "=l"(v) : "l"(p) : "memory");
-  return v;
-}
-__device__ __forceinline__ void spin_check(uint32_t& spins, uint64_t& start, const KParams& kp) {
-  if (++spins == 4096) start = globaltimer_ns();
-  if (spins > 4096 && (spins & 4095) == 0 && globaltimer_ns() - start > 10000000000ull) {
-    atomicExch(kp.err, 2);
-    asm volatile("trap;");
+__device__ __noinline__ void watchdog_trap(const KParams& kp, uint32_t flag, unsigned long long epoch) {
+  volatile uint32_t* e = kp.err;
+  if (atomicCAS(kp.err, 0u, (uint32_t)GEM_ERR_BARRIER) == 0u) {
+    e[1] = blockIdx.x;
+    e[2] = flag;
+    e[3] = (uint32_t)epoch;
+    __threadfence_system();
   }
+  asm volatile("trap;");
 }
-#ifndef GEM_BAR_VARIANT
-#define GEM_BAR_VARIANT 0
-#endif
+__device__ __forceinline__ void spin_check(uint32_t& spins, uint64_t& start, const KParams& kp, uint32_t flag,
+                                           unsigned long long epoch) {
+  if (++spins == 4096) start = globaltimer_ns();
+  if (spins > 4096 && (spins & 4095) == 0 && globaltimer_ns() - start > GEM_WATCHDOG_NS)
+    watchdog_trap(kp, flag, epoch);
+}
 __device__ __forceinline__ void grid_sync(const KParams& kp, unsigned long long& epoch) {
   __syncthreads();
   if (gridDim.x > 1) {
     epoch++;
-#if GEM_BAR_VARIANT == 0 || GEM_BAR_VARIANT == 1
     if (threadIdx.x == 0) st_release_u64(kp.bar + (size_t)blockIdx.x * GEM_BAR_STRIDE, epoch);
     for (uint32_t f = threadIdx.x; f < gridDim.x; f += blockDim.x) {
       uint32_t spins = 0;
       uint64_t start = 0;
-#if GEM_BAR_VARIANT == 0
-      while (ld_acquire_u64(kp.bar + (size_t)f * GEM_BAR_STRIDE) < epoch) spin_check(spins, start, kp);
-#else   // relaxed polling, one acquire fence after the flag is seen
-      while (ld_relaxed_u64(kp.bar + (size_t)f * GEM_BAR_STRIDE) < epoch) spin_check(spins, start, kp);
-      asm volatile("fence.acq_rel.gpu;" ::: "memory");
-#endif
+      while (ld_acquire_u64(kp.bar + (size_t)f * GEM_BAR_STRIDE) < epoch) spin_check(spins, start, kp, f, epoch);
     }
-#elif GEM_BAR_VARIANT == 2
-    // two-phase: CTA 0 gathers the arrival flags and publishes one release word
-    unsigned long long* rel = kp.bar + (size_t)GEM_BAR_MAX_CTAS * GEM_BAR_STRIDE;
-    if (blockIdx.x == 0) {
-      for (uint32_t f = threadIdx.x + 1; f < gridDim.x; f += blockDim.x) {
-        uint32_t spins = 0;
-        uint64_t start = 0;
-        while (ld_acquire_u64(kp.bar + (size_t)f * GEM_BAR_STRIDE) < epoch) spin_check(spins, start, kp);
-      }
-      __syncthreads();
-      if (threadIdx.x == 0) st_release_u64(rel, epoch);
-    } else {
-      if (threadIdx.x == 0) {
-        st_release_u64(kp.bar + (size_t)blockIdx.x * GEM_BAR_STRIDE, epoch);
-        uint32_t spins = 0;
-        uint64_t start = 0;
-        while (ld_acquire_u64(rel) < epoch) spin_check(spins, start, kp);
-      }
-    }
-#else   // single counter: red.release arrive, acquire polling by thread 0
-    if (threadIdx.x == 0) {
-      asm volatile("red.release.gpu.global.add.u64 [%0], 1;" ::"l"(kp.bar + (size_t)(GEM_BAR_MAX_CTAS + 1) * GEM_BAR_STRIDE) : "memory");
-      uint32_t spins = 0;
-      uint64_t start = 0;
-      while (ld_acquire_u64(kp.bar + (size_t)(GEM_BAR_MAX_CTAS + 1) * GEM_BAR_STRIDE) < epoch * gridDim.x)
-        spin_check(spins, start, kp);
-    }
-#endif
     __syncthreads();
   }
 }
@@ -283,7 +232,6 @@ __device__ __forceinline__ void fence_mbar_init() {
 }
 
 #define GEM_RING_MAX 8
-#define GEM_MAX_CHUNKS 256
 #define GEM_MAX_RESIDENT 16
 #define GEM_WL_MAX_STAGES 8
 #define GEM_WL_CACHE 64                              // work items cached in smem per CTA
@@ -466,16 +414,12 @@ __device__ __forceinline__ uint32_t dir0_entry(const uint32_t* C0, uint32_t off_
 // 13-level boomerang fold, write-outs.  No trailing barrier.
 template <bool kS0>
 __device__ __forceinline__ void exec_layer(const LayerRegs& R, uint32_t s_base, const uint32_t* Sj, uint32_t* topb,
-                                           uint32_t bid,
-                                           uint32_t fl = 99, unsigned long long* fsub = nullptr) {
+                                           uint32_t bid) {
   const uint32_t lane = threadIdx.x & 31, warp = threadIdx.x >> 5;
-  (void)fl;
-  (void)fsub;
   const bool uses_top = (R.flags & GEM_LF_USES_TOP) != 0;
   if ((R.flags >> warp) & 1u) {
     uint32_t v = 0;
     const uint32_t n4 = dc_n4(R.cls);
-#ifndef EXP_NO_GATHER
     if (R.cls == GEM_DC_DENSE16) {
       // two 16-bit entries per u32: entry 8g+2k in the low half, 8g+2k+1 in the high half
       uint32_t acc[4] = {0u, 0u, 0u, 0u};
@@ -484,16 +428,8 @@ __device__ __forceinline__ void exec_layer(const LayerRegs& R, uint32_t s_base, 
         const uint32_t q[4] = {R.e[g].x, R.e[g].y, R.e[g].z, R.e[g].w};
 #pragma unroll
         for (uint32_t k = 0; k < 4; k++) {
-#ifdef EXP_GATHER_HALF
-          if (g >= 2) continue;
-#endif
-#ifdef EXP_NO_CONFLICT   // timing experiment: same instructions, words 0..31 only (conflict-free)
-          const uint32_t lo = ldst<kS0>(Sj, (q[k] >> 3) & 0x7Cu);
-          const uint32_t hi = ldst<kS0>(Sj, (q[k] >> 19) & 0x7Cu);
-#else
           const uint32_t lo = ldst<kS0>(Sj, (q[k] >> 3) & 0x1FFCu);
           const uint32_t hi = ldst<kS0>(Sj, (q[k] >> 19) & 0x1FFCu);
-#endif
           acc[k] |= (__funnelshift_l(lo, lo, q[k]) & (1u << (8 * g + 2 * k))) |
                     (__funnelshift_l(hi, hi, q[k] >> 16) & (1u << (8 * g + 2 * k + 1)));
         }
@@ -520,25 +456,10 @@ __device__ __forceinline__ void exec_layer(const LayerRegs& R, uint32_t s_base, 
         default: v = gather_sparse<8, kS0>(Sj, R.e); break;
       }
     }
-#else   // timing experiment only (wrong results)
-    v = R.e[0].x ^ R.e[1].y ^ R.lc.w;
-    (void)n4;
-#endif
-    FSUB(fl, 0);
-#ifndef EXP_NO_FOLD
     const uint32_t P = fold5(v, R.lc.x, R.lc.y, R.lc.z);
-#else
-    const uint32_t P = v ^ R.lc.x;
-#endif
     if (R.lc.w) sts(s_base + 4 * R.lc.w, P);
-    FSUB(fl, 1);
     const uint32_t u = __ballot_sync(0xFFFFFFFFu, (P >> 30) & 1u);
-#ifndef EXP_NO_FOLD
     const uint32_t Pw = fold5(u, R.wc.x, R.wc.y, R.wc.z);
-#else
-    const uint32_t Pw = u ^ R.wc.x;
-#endif
-    FSUB(fl, 2);
     if (lane == 0) {
       if (R.wc.w) sts(s_base + 4 * R.wc.w, Pw);
       if (uses_top) topb[warp] = (Pw >> 30) & 1u;
@@ -548,25 +469,7 @@ __device__ __forceinline__ void exec_layer(const LayerRegs& R, uint32_t s_base, 
   }
   // levels 11-13: warps 1-7 arrive (non-blocking) on named barrier `bid`
   // after publishing their level-10 bit; warp 0 folds later (top_layer).
-#if defined(GEM_TOP_ATOMIC)
-  // variant: the last warp to arrive (acq_rel counter in topb[8]) folds
-  if (uses_top && lane == 0) {
-    uint32_t old;
-    asm volatile("atom.acq_rel.cta.shared::cta.add.u32 %0, [%1], 1;"
-                 : "=r"(old) : "r"(smem_u32(topb + 8)) : "memory");
-    if (old == GEM_WARPS - 1) {
-      uint32_t t8 = 0;
-#pragma unroll
-      for (uint32_t w = 0; w < GEM_WARPS; w++) t8 |= lds(smem_u32(topb + w)) << w;
-      sts(s_base + 4 * R.topwo, fold3(t8, R.topc & 0xFFu, (R.topc >> 8) & 0xFFu, (R.topc >> 16) & 0xFFu));
-      sts(smem_u32(topb + 8), 0u);
-    }
-  }
-  (void)bid;
-#elif !defined(EXP_NO_TOP)
   if (uses_top && warp != 0) asm volatile("bar.arrive %0, %1;" ::"r"(bid), "r"(GEM_THREADS) : "memory");
-#endif
-  FSUB(fl, 3);
 }
 
 // Levels 11-13 of a layer (warp 0 only): wait on named barrier `bid` for the
@@ -703,15 +606,12 @@ __device__ void run_partition(const KParams& kp, ProgSrc& ps, uint32_t* S, uint3
   // first layer's records (independent of S) before the barrier
   LayerRegs R;
   const uint32_t* Lres = C0 + off_layers;
-  const uint32_t* L0 = nullptr;
   if (n_layers) {
     const uint32_t* L;
     if (1 < n_pin) { L = Lres; Lres += ctab[1]; }
     else L = ring_wait(ps);
     load_layer(L, dir0_entry(C0, h3.w), R);
-    L0 = L;
   }
-  (void)L0;
   PROF(9);
   __syncthreads();   // S ready; chunk 0 and layer 0's chunk consumed
   ps.seq_free = ps.seq_wait;   // records are in registers; waited slots are free
@@ -739,51 +639,22 @@ __device__ void run_partition(const KParams& kp, ProgSrc& ps, uint32_t* S, uint3
   // slowed the activity build's layers by ~8%)
   if (ACT && skip) goto commit;
   for (uint32_t l = 0; l < n_layers; l++) {
-    FPROF(l, 0);
-#ifdef GEM_FINE_PROF
-    const uint32_t fl = (kp.fprof && c == 5 && blockIdx.x == kp.fine_cta) ? l : 99u;
-    unsigned long long* fsub = kp.fprof ? kp.fprof + GEM_FINE_LAYERS * 64 : nullptr;
-#else
-    const uint32_t fl = 99u;
-    unsigned long long* fsub = nullptr;
-#endif
     // stream j uses named barrier 1 + j (group <= GEM_MAX_GROUP < 16)
-    if (nst == 1 && s_base == GEM_S0_ADDR) exec_layer<true>(R, s_base, g_smem, topb, 1, fl, fsub);
+    if (nst == 1 && s_base == GEM_S0_ADDR) exec_layer<true>(R, s_base, g_smem, topb, 1);
     else
       for (uint32_t j = 0; j < nst; j++)
-        exec_layer<false>(R, s_base + 4 * j * SW, g_smem + j * SW, topb + 16 * j, 1 + j, fl, fsub);
-    FPROF(l, 1);
+        exec_layer<false>(R, s_base + 4 * j * SW, g_smem + j * SW, topb + 16 * j, 1 + j);
     const bool ptop = (R.flags & GEM_LF_USES_TOP) != 0;
     const uint32_t ptopc = R.topc, ptopwo = R.topwo;
-#if defined(EXP_NO_WAIT)   // timing experiment: every layer reuses layer 0's records (no wait, no load)
-    if (false) {
-#elif defined(EXP_SAME_L)  // timing experiment: reload layer 0's records (load chain, no chunk wait)
     if (l + 1 < n_layers) {
-      load_layer(L0, dir0_entry(C0, h3.w), R);
-    }
-    if (false) {
-#else
-    if (l + 1 < n_layers) {
-#endif
       const uint32_t* L;
       if (2 + l < n_pin) { L = Lres; Lres += ctab[2 + l]; }
       else L = ring_wait(ps);
-      FPROF(l, 2);
-      const uint32_t nd = R.ndir;
-#ifndef EXP_NO_LOAD
-      load_layer(L, nd, R);
-#else
-      if (l == 0) load_layer(L, nd, R);
-#endif
+      load_layer(L, R.ndir, R);
     }
-    FPROF(l, 3);
-#if !defined(EXP_NO_TOP) && !defined(GEM_TOP_ATOMIC)
     if (ptop && warp == 0)
       for (uint32_t j = 0; j < nst; j++) top_layer(ptopc, ptopwo, s_base + 4 * j * SW, topb + 16 * j, 1 + j);
-#endif
-    FPROF(l, 4);
     __syncthreads();
-    FPROF(l, 5);
     ps.seq_free = ps.seq_wait;
     refill();
   }
@@ -1188,14 +1059,15 @@ struct gem_sim {
   uint32_t *d_q = nullptr, *d_rd = nullptr, *d_cut = nullptr, *d_mem = nullptr;
   uint32_t *d_pi = nullptr, *d_po = nullptr, *d_qtrace = nullptr, *d_scratch = nullptr, *d_wl_off = nullptr;
   uint2* d_wl_items = nullptr;
-  unsigned long long *d_digest = nullptr, *d_bar = nullptr, *d_prof = nullptr, *d_fprof = nullptr;
-  size_t bar_off = 0;  // experiment (GEM_EXP_BAR_SHIFT_KB): barrier flags placed this many u64 into d_bar
+  unsigned long long *d_digest = nullptr, *d_bar = nullptr, *d_prof = nullptr;
   uint32_t prof_cycles = 0;
-  int* d_err = nullptr;
+  uint32_t* h_err = nullptr;   // watchdog words {code, cta, flag, epoch}: mapped pinned host memory
+  uint32_t* d_err = nullptr;   // device alias of h_err
+  gem_config cfg{};            // launch tuning (include/gem.h)
   uint32_t in_cap = 0, in_queued = 0, in_head = 0, out_cap = 0, last_cycles = 0;
   size_t scratch_bytes = 0;
   uint64_t cycle = 0;
-  cudaEvent_t ev0 = nullptr, ev1 = nullptr;
+  cudaEvent_t ev0 = nullptr, ev1 = nullptr, ev_in = nullptr;
   float last_ms = 0.f;
 };
 
@@ -1204,13 +1076,22 @@ static int fail(int code, const std::string& msg) {
   return code;
 }
 
+// The grid-barrier watchdog's report (mapped pinned words written before the
+// trap), appended to the CUDA error of the failed call.
+static std::string watchdog_msg(const gem_sim* sim) {
+  if (!sim || !sim->h_err || sim->h_err[0] != GEM_ERR_BARRIER) return "";
+  const volatile uint32_t* e = sim->h_err;
+  return "; grid-barrier watchdog: CTA " + std::to_string(e[1]) + " waited > 10 s for CTA " + std::to_string(e[2]) +
+         " at barrier epoch " + std::to_string(e[3]) + " (persistent grid not co-resident?)";
+}
+
 #define CK(call)                                                                          \
   do {                                                                                    \
     cudaError_t e_ = (call);                                                              \
     if (e_ != cudaSuccess) {                                                              \
       if (sim) sim->poisoned = true;                                                      \
       return fail(e_ == cudaErrorMemoryAllocation ? GEM_E_NOMEM : GEM_E_CUDA,             \
-                  std::string(#call) + ": " + cudaGetErrorString(e_));                    \
+                  std::string(#call) + ": " + cudaGetErrorString(e_) + watchdog_msg(sim)); \
     }                                                                                     \
   } while (0)
 
@@ -1268,8 +1149,7 @@ static double build_worklists(const gem_sim* sim, uint32_t G, std::vector<uint32
     // a scheduling unit = `run` consecutive stream groups of one partition, kept
     // together on one CTA (lane mode: consecutive items then share the
     // partition's input-port list and program in L1/L2)
-    const uint32_t run = sim->lanes ? (uint32_t)std::max(1, getenv("GEM_LANE_RUN") ? atoi(getenv("GEM_LANE_RUN")) : 4)
-                                    : 1u;
+    const uint32_t run = sim->lanes ? (sim->cfg.lane_run ? sim->cfg.lane_run : 4u) : 1u;
     std::vector<std::pair<uint32_t, uint2>> its;
     its.reserve((size_t)np * sim->n_streams);
     for (uint32_t st = 0; st < sim->n_streams; st += sim->group * run)
@@ -1336,8 +1216,7 @@ static int plan_launch(gem_sim* sim, uint32_t max_chunk_words, uint32_t grid_lim
   // streams per work item: as many stream states as fit beside a 3-slot ring
   sim->group = 1;
   if (sim->n_streams > 1) {
-    const char* genv = getenv("GEM_GROUP");
-    uint32_t g = genv ? (uint32_t)atoi(genv) : GEM_MAX_GROUP;
+    uint32_t g = sim->cfg.max_group ? sim->cfg.max_group : GEM_MAX_GROUP;
     g = std::max<uint32_t>(1, std::min<uint32_t>(std::min<uint32_t>(g, GEM_MAX_GROUP), sim->n_streams));
     while (g > 1 && (uint64_t)(g * (sim->state_words + 4 * GEM_MAX_RAMS_PER_PART + 16) + GEM_MAX_CHUNKS + 96 + GEM_WL_CACHE_WORDS +
                                3 * slot) * 4 > (uint64_t)optin)
@@ -1351,10 +1230,8 @@ static int plan_launch(gem_sim* sim, uint32_t max_chunk_words, uint32_t grid_lim
   if (sim->group != 1) sim->act_words = 0;   // activity pruning needs one stream per work item
   const uint32_t fixed_words = sim->group * (sim->state_words + 4 * GEM_MAX_RAMS_PER_PART + 16) + GEM_MAX_CHUNKS +
                                48 + GEM_WL_CACHE_WORDS + 32 + sim->act_words;
-  const char* env = getenv("GEM_NO_RESIDENT");
-  const bool allow_res = !(env && env[0] == '1');
-  const char* benv = getenv("GEM_BPS");
-  const uint32_t force_bps = benv ? (uint32_t)atoi(benv) : 0;
+  const bool allow_res = !(sim->flags & GEM_F_NO_RESIDENT);
+  const uint32_t force_bps = sim->cfg.ctas_per_sm;
   struct Choice { uint32_t bps = 0, grid = 0, area = 0, resident = 0, ring = 0; double score = 0; };
   Choice best;
   std::vector<uint32_t> best_off, off;
@@ -1437,15 +1314,14 @@ static int plan_launch_lanes(gem_sim* sim, uint32_t grid_limit) {
   CK(cudaDeviceGetAttribute(&per_sm, cudaDevAttrMaxSharedMemoryPerMultiprocessor, sim->device));
   if (!coop) return fail(GEM_E_UNSUPPORTED, "device lacks cooperative launch");
   sim->sm_count = (uint32_t)sms;
-  const char* ge = getenv("GEM_LANE_GROUPS");
-  const char* be = getenv("GEM_LANE_BPS");
-  const uint32_t want_gl = std::min<uint32_t>(ge ? (uint32_t)atoi(ge) : 4, 4);
+  const uint32_t want_gl = std::min<uint32_t>(sim->cfg.lane_groups ? sim->cfg.lane_groups : 4u, 4u);
+  const uint32_t force_bps = sim->cfg.lane_ctas_per_sm;
   // prefer 2 CTAs per SM (16 warps to hide latency), then as many 32-stream
   // groups per work item as fit (shared memory holds only the lane state:
   // records stream from global memory into registers)
   uint32_t bps = 0, gl = 0;
   for (uint32_t b = 2; b >= 1 && !bps; b--) {
-    if (be && (uint32_t)atoi(be) != b) continue;
+    if (force_bps && force_bps != b) continue;
     const uint32_t bud = (uint32_t)std::min<int64_t>(optin, per_sm / (int64_t)b - 1024);
     for (uint32_t k = std::max<uint32_t>(1, std::min(want_gl, sim->n_groups)); k >= 1; k--) {
       if (k == 3) continue;   // the kernel is instantiated for K = 1, 2, 4 interleaved groups
@@ -1472,15 +1348,14 @@ static int plan_launch_lanes(gem_sim* sim, uint32_t grid_limit) {
   std::vector<uint32_t> off;
   std::vector<uint2> items;
   build_worklists(sim, grid, off, items);
-  // one stage: dynamic distribution of LPT-ordered units (GEM_LANE_DYN=0: static lists)
-  const char* de = getenv("GEM_LANE_DYN");
-  if (sim->n_stages == 1 && !(de && de[0] == '0')) {
+  // one stage: dynamic distribution of LPT-ordered units (GEM_F_STATIC_LANES: static lists)
+  if (sim->n_stages == 1 && !(sim->flags & GEM_F_STATIC_LANES)) {
     // unit = `run` consecutive items of one partition (they share its records
     // in L2 / L1); as long as there are >= 8 units per CTA
     const uint32_t np1 = sim->h_stage[1] - sim->h_stage[0];
     const uint64_t items1 = (uint64_t)np1 * ((sim->n_streams + sim->group - 1) / sim->group);
     uint32_t run = (uint32_t)std::max<uint64_t>(1, std::min<uint64_t>(4, items1 / (8ull * grid)));
-    if (getenv("GEM_LANE_RUN")) run = (uint32_t)std::max(1, atoi(getenv("GEM_LANE_RUN")));
+    if (sim->cfg.lane_run) run = sim->cfg.lane_run;
     std::vector<std::pair<double, uint4>> us;
     const uint32_t np = sim->h_stage[1] - sim->h_stage[0];
     for (uint32_t st = 0; st < sim->n_streams; st += sim->group * run)
@@ -1518,30 +1393,80 @@ extern "C" {
 
 const char* gem_last_error(void) { return g_err.c_str(); }
 
-int gem_load_program(const void* blob, size_t nbytes, const gem_config* cfg, gem_sim** out) {
-  gem_sim* sim = nullptr;
-  if (!blob || !cfg || !out || nbytes < GH_N_WORDS * 4 || (nbytes & 3)) return fail(GEM_E_INVAL, "bad arguments");
-  const uint32_t* w = (const uint32_t*)blob;
-  const size_t nw = nbytes / 4;
-  if (w[GH_MAGIC] != GEM_MAGIC || w[GH_VERSION] != GEM_VERSION) return fail(GEM_E_FORMAT, "bad blob magic/version");
-  const uint64_t total_words = w[GH_TOTAL_WORDS_LO] | ((uint64_t)w[GH_TOTAL_WORDS_HI] << 32);
+}  // extern "C"
+
+// Structural validation of a program blob (include/gem.h: a malformed or
+// truncated blob is GEM_E_FORMAT, never an out-of-bounds access): every table
+// offset + length inside the blob, permutation entries in range, stage prefix
+// monotone, every partition program inside the program area with a sane
+// header and chunk table (at most GEM_MAX_CHUNKS chunks: the kernel keeps the
+// chunk table in a fixed shared-memory array).
+static int validate_blob(const uint32_t* w, size_t nw) {
+  auto in = [&](uint64_t off, uint64_t len) { return off <= nw && len <= nw - off; };
   const uint64_t prog_words = w[GH_PROG_WORDS_LO] | ((uint64_t)w[GH_PROG_WORDS_HI] << 32);
-  if (total_words != nw || w[GH_OFF_PROG] + prog_words > nw) return fail(GEM_E_FORMAT, "truncated blob");
-  if (cfg->n_streams == 0) return fail(GEM_E_INVAL, "n_streams must be >= 1");
-  if (w[GH_MAX_STATE_WORDS] > GEM_MAX_STATE_WORDS) return fail(GEM_E_FORMAT, "state too large");
-  int ndev = 0;
-  if (cudaGetDeviceCount(&ndev) != cudaSuccess || ndev == 0)
-    return fail(GEM_E_UNSUPPORTED, "no CUDA device (libgem has no CPU fallback)");
-  if (cfg->device < 0 || cfg->device >= ndev) return fail(GEM_E_INVAL, "bad device ordinal");
-  sim = new gem_sim();
-  *out = nullptr;
+  const uint32_t n_parts = w[GH_N_PARTS], n_stages = w[GH_N_STAGES];
+  if (!in(w[GH_OFF_PROG], prog_words)) return fail(GEM_E_FORMAT, "truncated program area");
+  if (n_stages == 0 || n_stages > GEM_WL_MAX_STAGES) return fail(GEM_E_FORMAT, "bad stage count");
+  if (!in(w[GH_OFF_PARTS], (uint64_t)n_parts * GP_WORDS)) return fail(GEM_E_FORMAT, "truncated partition table");
+  if (!in(w[GH_OFF_STAGES], (uint64_t)n_stages + 1 + n_parts)) return fail(GEM_E_FORMAT, "truncated stage list");
+  const uint32_t* st = w + w[GH_OFF_STAGES];
+  if (st[0] != 0 || st[n_stages] > n_parts) return fail(GEM_E_FORMAT, "bad stage prefix");
+  for (uint32_t s = 0; s < n_stages; s++)
+    if (st[s + 1] < st[s]) return fail(GEM_E_FORMAT, "stage prefix not monotone");
+  for (uint32_t k = 0; k < st[n_stages]; k++)
+    if (st[n_stages + 1 + k] >= n_parts) return fail(GEM_E_FORMAT, "bad partition id in stage list");
+  const uint64_t qw = w[GH_Q_WORDS], pw = w[GH_PO_WORDS];
+  if (qw * 32 < w[GH_N_FLOPS] || pw * 32 < w[GH_N_PO] || (uint64_t)w[GH_PI_WORDS] * 32 < w[GH_N_PI])
+    return fail(GEM_E_FORMAT, "word counts too small");
+  if (!in(w[GH_OFF_FLOP_INIT], qw + qw * 32 + pw * 32)) return fail(GEM_E_FORMAT, "truncated permutation tables");
+  const uint32_t* q_ext = w + w[GH_OFF_FLOP_INIT] + qw;
+  const uint32_t* po_ext = q_ext + qw * 32;
+  for (uint64_t b = 0; b < qw * 32; b++)
+    if (q_ext[b] != 0xFFFFFFFFu && q_ext[b] >= w[GH_N_FLOPS]) return fail(GEM_E_FORMAT, "bad flop permutation");
+  for (uint64_t b = 0; b < pw * 32; b++)
+    if (po_ext[b] != 0xFFFFFFFFu && po_ext[b] >= w[GH_N_PO]) return fail(GEM_E_FORMAT, "bad PO permutation");
+  const uint32_t* parts = w + w[GH_OFF_PARTS];
+  const uint32_t* prog = w + w[GH_OFF_PROG];
+  const uint64_t lp_words = w[GH_LANE_PROG_WORDS_LO] | ((uint64_t)w[GH_LANE_PROG_WORDS_HI] << 32);
+  if (w[GH_HAS_LANES] && !in(w[GH_OFF_LANE_PROG], lp_words)) return fail(GEM_E_FORMAT, "truncated lane programs");
+  for (uint32_t p = 0; p < n_parts; p++) {
+    const uint32_t* e = parts + (size_t)p * GP_WORDS;
+    const uint64_t off = e[GP_PROG_OFF], len = e[GP_PROG_LEN];
+    if (off + len > prog_words || len < PH_WORDS) return fail(GEM_E_FORMAT, "partition program out of range");
+    const uint32_t* pr = prog + off;
+    if (pr[PH_MAGIC] != GEM_PART_MAGIC || pr[PH_N_RAM] > GEM_MAX_RAMS_PER_PART || pr[PH_N_LAYERS] != e[GP_N_LAYERS])
+      return fail(GEM_E_FORMAT, "bad partition program header");
+    if (pr[PH_N_CHUNKS] != pr[PH_N_LAYERS] + 2)
+      return fail(GEM_E_FORMAT, "bad chunk count");
+    if (pr[PH_N_CHUNKS] > GEM_MAX_CHUNKS)
+      return fail(GEM_E_UNSUPPORTED, "partition program has more than " + std::to_string(GEM_MAX_CHUNKS - 2) +
+                                         " layers (map with a smaller part_size)");
+    if ((uint64_t)pr[PH_OFF_CHUNKS] + pr[PH_N_CHUNKS] > len) return fail(GEM_E_FORMAT, "bad chunk table");
+    uint64_t sum = 0, mx = 0;
+    for (uint32_t k = 0; k < pr[PH_N_CHUNKS]; k++) {
+      const uint32_t c = pr[pr[PH_OFF_CHUNKS] + k];
+      if (c & 3u) return fail(GEM_E_FORMAT, "chunk not a multiple of 16 bytes");
+      sum += c;
+      mx = std::max<uint64_t>(mx, c);
+    }
+    if (sum > len || mx > w[GH_MAX_CHUNK_WORDS]) return fail(GEM_E_FORMAT, "chunk table exceeds program");
+    if (e[GP_CHUNK0] != pr[pr[PH_OFF_CHUNKS]]) return fail(GEM_E_FORMAT, "partition table / chunk table mismatch");
+    if (pr[PH_OFF_GREAD] + 2ull * pr[PH_N_GREAD] > len || pr[PH_OFF_OUT] + pr[PH_N_OUT_PAD] + 32ull * pr[PH_N_OUT] > len)
+      return fail(GEM_E_FORMAT, "partition sections out of range");
+    if (w[GH_HAS_LANES] && (uint64_t)e[GP_LANE_OFF] + e[GP_LANE_LEN] > lp_words)
+      return fail(GEM_E_FORMAT, "lane program out of range");
+  }
+  return GEM_OK;
+}
+
+// gem_load_program body; on failure the caller frees the partially built handle.
+static int load_impl(gem_sim* sim, const uint32_t* w, size_t nw, const gem_config* cfg) {
   sim->device = cfg->device;
+  sim->cfg = *cfg;
   sim->flags = cfg->flags;
   sim->n_streams = cfg->n_streams;
-  {
-    cudaError_t e = cudaSetDevice(sim->device);
-    if (e != cudaSuccess) { delete sim; return fail(GEM_E_CUDA, cudaGetErrorString(e)); }
-  }
+  CK(cudaSetDevice(sim->device));
+  const uint64_t prog_words = w[GH_PROG_WORDS_LO] | ((uint64_t)w[GH_PROG_WORDS_HI] << 32);
   sim->n_pi = w[GH_N_PI]; sim->n_po = w[GH_N_PO]; sim->n_flops = w[GH_N_FLOPS]; sim->n_rams = w[GH_N_RAMS];
   sim->n_parts = w[GH_N_PARTS]; sim->n_stages = w[GH_N_STAGES]; sim->max_layers = w[GH_MAX_LAYERS];
   sim->total_layers = w[GH_TOTAL_LAYERS];
@@ -1563,10 +1488,6 @@ int gem_load_program(const void* blob, size_t nbytes, const gem_config* cfg, gem
     sim->max_items = std::max(sim->max_items, (stages[s + 1] - stages[s]) * sim->n_streams);
   for (uint32_t p = 0; p < sim->n_parts; p++) {
     const uint32_t* pr = w + w[GH_OFF_PROG] + parts[p * GP_WORDS + GP_PROG_OFF];
-    if (pr[PH_MAGIC] != GEM_PART_MAGIC || pr[PH_N_RAM] > GEM_MAX_RAMS_PER_PART) {
-      delete sim;
-      return fail(GEM_E_FORMAT, "bad partition program");
-    }
     if (cfg->flags & GEM_F_ACTIVITY) sim->act_words = std::max(sim->act_words, (pr[PH_N_GREAD] + 3u) & ~3u);
   }
   // inverse permutation tables
@@ -1576,21 +1497,22 @@ int gem_load_program(const void* blob, size_t nbytes, const gem_config* cfg, gem
     if (q_ext_of_int[b] != 0xFFFFFFFFu) q_int_of_ext[q_ext_of_int[b]] = b;
   for (uint32_t b = 0; b < sim->po_words_int * 32; b++)
     if (po_ext_of_int[b] != 0xFFFFFFFFu) po_int_of_ext[po_ext_of_int[b]] = b;
-  // streams / events
+  // streams / events / watchdog words (mapped pinned host memory)
   if (cfg->cuda_stream) sim->stream = (cudaStream_t)cfg->cuda_stream;
   else { CK(cudaStreamCreateWithFlags(&sim->stream, cudaStreamNonBlocking)); sim->own_stream = true; }
   CK(cudaEventCreate(&sim->ev0));
   CK(cudaEventCreate(&sim->ev1));
-  // lane mode: >= 32 streams and lane programs present (GEM_NO_LANES=1 disables)
-  {
-    const char* nl = getenv("GEM_NO_LANES");
-    sim->lanes = (w[GH_HAS_LANES] && cfg->n_streams >= 32 && !(nl && nl[0] == '1')) ? 1u : 0u;
-    if (sim->lanes) {
-      sim->n_groups = (cfg->n_streams + 31) / 32;
-      sim->lane_words = (std::max<uint32_t>(w[GH_LANE_MAX_WORDS], 4) + 3) & ~3u;
-      sim->lane_max_chunk = w[GH_LANE_MAX_CHUNK_WORDS];
-      sim->ramp_words = std::max<uint32_t>(w[GH_MAX_RAMS_PART], 1) * 128;
-    }
+  CK(cudaEventCreateWithFlags(&sim->ev_in, cudaEventDisableTiming));
+  CK(cudaHostAlloc((void**)&sim->h_err, 64, cudaHostAllocMapped));
+  std::memset(sim->h_err, 0, 64);
+  CK(cudaHostGetDevicePointer((void**)&sim->d_err, sim->h_err, 0));
+  // lane mode: >= 32 streams and lane programs present (GEM_F_NO_LANES disables)
+  sim->lanes = (w[GH_HAS_LANES] && cfg->n_streams >= 32 && !(cfg->flags & GEM_F_NO_LANES)) ? 1u : 0u;
+  if (sim->lanes) {
+    sim->n_groups = (cfg->n_streams + 31) / 32;
+    sim->lane_words = (std::max<uint32_t>(w[GH_LANE_MAX_WORDS], 4) + 3) & ~3u;
+    sim->lane_max_chunk = w[GH_LANE_MAX_CHUNK_WORDS];
+    sim->ramp_words = std::max<uint32_t>(w[GH_MAX_RAMS_PART], 1) * 128;
   }
   // uploads
   const size_t S = sim->n_streams;
@@ -1609,7 +1531,6 @@ int gem_load_program(const void* blob, size_t nbytes, const gem_config* cfg, gem
   CK(cudaMemcpy(sim->d_po_int_of_ext, po_int_of_ext.data(), po_int_of_ext.size() * 4, cudaMemcpyHostToDevice));
   if (sim->lanes) {
     const uint64_t lp_words = w[GH_LANE_PROG_WORDS_LO] | ((uint64_t)w[GH_LANE_PROG_WORDS_HI] << 32);
-    if (w[GH_OFF_LANE_PROG] + lp_words > nw) { gem_free(sim); return fail(GEM_E_FORMAT, "truncated lane programs"); }
     CK(dalloc(&sim->d_lprog, lp_words * 4));
     CK(cudaMemcpy(sim->d_lprog, w + w[GH_OFF_LANE_PROG], lp_words * 4, cudaMemcpyHostToDevice));
     const size_t G = sim->n_groups, qb = (size_t)sim->q_words_int * 32;
@@ -1622,10 +1543,7 @@ int gem_load_program(const void* blob, size_t nbytes, const gem_config* cfg, gem
     CK(dalloc(&sim->d_cut, S * std::max<uint32_t>(sim->cut_words, 1) * 4));
   }
   CK(dalloc(&sim->d_mem, S * sim->n_rams * (size_t)GEM_RAM_WORDS * 4));
-  if (const char* e = getenv("GEM_EXP_BAR_SHIFT_KB")) sim->bar_off = (size_t)atoi(e) * 128;
-  CK(dalloc(&sim->d_bar, (size_t)(GEM_BAR_MAX_CTAS + 2) * GEM_BAR_STRIDE * 8 + sim->bar_off * 8));
-  CK(dalloc(&sim->d_err, 64));
-  CK(cudaMemset(sim->d_err, 0, 64));
+  CK(dalloc(&sim->d_bar, (size_t)(GEM_BAR_MAX_CTAS + 2) * GEM_BAR_STRIDE * 8));
   CK(dalloc(&sim->d_act, 16));
   CK(cudaMemset(sim->d_act, 0, 16));
   // initial state: flops = init (U5), RD = 0, RAM = 0 (U10)
@@ -1638,7 +1556,6 @@ int gem_load_program(const void* blob, size_t nbytes, const gem_config* cfg, gem
     CK(cudaMemcpy(sim->d_q, q0.data(), q0.size() * 4, cudaMemcpyHostToDevice));
     CK(cudaMemset(sim->d_rd, 0, 2 * (size_t)std::max<uint32_t>(sim->n_rams, 1) * 32 * G * 4));
     CK(cudaMemset(sim->d_cut, 0, (size_t)std::max<uint32_t>(sim->cut_words, 1) * 32 * G * 4));
-    if (sim->n_rams) CK(cudaMemset(sim->d_mem, 0, S * sim->n_rams * (size_t)GEM_RAM_WORDS * 4));
   } else {
     std::vector<uint32_t> q0(S * sim->q_words_int);
     for (size_t s = 0; s < S; s++) std::memcpy(&q0[s * sim->q_words_int], finit, sim->q_words_int * 4);
@@ -1646,18 +1563,44 @@ int gem_load_program(const void* blob, size_t nbytes, const gem_config* cfg, gem
     CK(cudaMemset(sim->d_q + S * sim->q_words_int, 0, S * sim->q_words_int * 4));
     CK(cudaMemset(sim->d_rd, 0, 2 * S * std::max<uint32_t>(sim->n_rams, 1) * 4));
     CK(cudaMemset(sim->d_cut, 0, S * std::max<uint32_t>(sim->cut_words, 1) * 4));
-    if (sim->n_rams) CK(cudaMemset(sim->d_mem, 0, S * sim->n_rams * (size_t)GEM_RAM_WORDS * 4));
   }
+  if (sim->n_rams) CK(cudaMemset(sim->d_mem, 0, S * sim->n_rams * (size_t)GEM_RAM_WORDS * 4));
   // persistent co-resident grid + shared-memory program placement
   sim->h_parts.assign(parts, parts + (size_t)sim->n_parts * GP_WORDS);
   sim->h_stage.assign(stages, stages + stage_words);
   if (sim->lanes) {
-    if (int r = plan_launch_lanes(sim, cfg->grid_limit)) { gem_free(sim); return r; }
+    if (int r = plan_launch_lanes(sim, cfg->grid_limit)) return r;
   } else if (int r = plan_launch(sim, w[GH_MAX_CHUNK_WORDS], cfg->grid_limit)) {
-    gem_free(sim);
     return r;
   }
   CK(cudaDeviceSynchronize());
+  return GEM_OK;
+}
+
+extern "C" {
+
+int gem_load_program(const void* blob, size_t nbytes, const gem_config* cfg, gem_sim** out) {
+  if (!blob || !cfg || !out || nbytes < GH_N_WORDS * 4 || (nbytes & 3)) return fail(GEM_E_INVAL, "bad arguments");
+  *out = nullptr;
+  const uint32_t* w = (const uint32_t*)blob;
+  const size_t nw = nbytes / 4;
+  if (w[GH_MAGIC] != GEM_MAGIC || w[GH_VERSION] != GEM_VERSION) return fail(GEM_E_FORMAT, "bad blob magic/version");
+  const uint64_t total_words = w[GH_TOTAL_WORDS_LO] | ((uint64_t)w[GH_TOTAL_WORDS_HI] << 32);
+  if (total_words != nw) return fail(GEM_E_FORMAT, "truncated blob");
+  if (cfg->n_streams == 0) return fail(GEM_E_INVAL, "n_streams must be >= 1");
+  if (w[GH_MAX_STATE_WORDS] > GEM_MAX_STATE_WORDS) return fail(GEM_E_FORMAT, "state too large");
+  if (int r = validate_blob(w, nw)) return r;
+  int ndev = 0;
+  if (cudaGetDeviceCount(&ndev) != cudaSuccess || ndev == 0)
+    return fail(GEM_E_UNSUPPORTED, "no CUDA device (libgem has no CPU fallback)");
+  if (cfg->device < 0 || cfg->device >= ndev) return fail(GEM_E_INVAL, "bad device ordinal");
+  gem_sim* sim = new gem_sim();
+  if (int r = load_impl(sim, w, nw, cfg)) {
+    const std::string msg = g_err;   // gem_free must not clobber the reason
+    gem_free(sim);
+    g_err = msg;
+    return r;
+  }
   *out = sim;
   return GEM_OK;
 }
@@ -1706,6 +1649,11 @@ int gem_set_inputs(gem_sim* sim, const uint32_t* pi, uint64_t ncycles, int src_o
           (uint64_t)sim->in_cap * sim->pi_words, sim->pi_words, sim->n_groups, 0);
       CK(cudaGetLastError());
     }
+    if (!src_on_device) {
+      // the caller may reuse its (possibly pinned) buffer as soon as we return
+      CK(cudaEventRecord(sim->ev_in, sim->stream));
+      CK(cudaEventSynchronize(sim->ev_in));
+    }
   }
   sim->in_queued = (uint32_t)ncycles;
   sim->in_head = 0;
@@ -1724,7 +1672,7 @@ int gem_step(gem_sim* sim, uint64_t ncycles) {
   kp.prog = sim->d_prog; kp.parts = sim->d_parts; kp.stage_list = sim->d_stage;
   kp.pi = sim->d_pi; kp.po = sim->d_po; kp.q = sim->d_q; kp.rd = sim->d_rd; kp.cut = sim->d_cut;
   kp.mem = sim->d_mem; kp.q_trace = sim->d_qtrace; kp.digest = sim->d_digest;
-  kp.q_int_of_ext = sim->d_q_int_of_ext; kp.bar = sim->d_bar + sim->bar_off; kp.err = sim->d_err;
+  kp.q_int_of_ext = sim->d_q_int_of_ext; kp.bar = sim->d_bar; kp.err = sim->d_err;
   kp.t0 = sim->cycle; kp.ncycles = (uint32_t)ncycles; kp.in_base = sim->in_head; kp.in_cap = sim->in_cap;
   kp.out_cap = sim->out_cap; kp.n_stages = sim->n_stages; kp.n_streams = sim->n_streams;
   kp.state_words = sim->state_words; kp.pi_words = sim->pi_words; kp.po_words = sim->po_words_int;
@@ -1738,14 +1686,14 @@ int gem_step(gem_sim* sim, uint64_t ncycles) {
   kp.wl_items = sim->d_wl_items;
   kp.act_cnt = sim->d_act;
   {
-    // programs larger than half the L2 (C4): keep a fraction L2-resident (GEM_L2_FRAC overrides)
-    const char* fe = getenv("GEM_L2_FRAC");
+    // programs larger than half the L2 (C4): keep a fraction L2-resident
+    // (gem_config::l2_evict_last: 0 = this rule, > 0 = that fraction, < 0 = none)
     int l2 = 0;
     cudaDeviceGetAttribute(&l2, cudaDevAttrL2CacheSize, sim->device);
     float f = 0.f;
     if (!sim->lanes && 2 * sim->program_bytes > (uint64_t)l2)   // does not stay resident by itself
       f = std::min(0.9f, 0.6f * (float)l2 / (float)sim->program_bytes);
-    if (fe) f = (float)atof(fe);
+    if (sim->cfg.l2_evict_last != 0.f) f = sim->cfg.l2_evict_last;
     kp.l2_frac = std::max(0.f, std::min(1.f, f));
   }
   kp.dyn_units = sim->d_dyn_units;
@@ -1759,18 +1707,13 @@ int gem_step(gem_sim* sim, uint64_t ncycles) {
       if (sim->d_prof) cudaFree(sim->d_prof);
       sim->d_prof = nullptr;
       CK(dalloc(&sim->d_prof, (size_t)256 * sim->grid * GEM_PROF_SLOTS * 8));
-#ifdef GEM_FINE_PROF
-      CK(dalloc(&sim->d_fprof, GEM_FINE_LAYERS * 96 * 8));
-#endif
     }
     sim->prof_cycles = pc;
     CK(cudaMemsetAsync(sim->d_prof, 0, (size_t)256 * sim->grid * GEM_PROF_SLOTS * 8, sim->stream));
     kp.prof = sim->d_prof;
     kp.prof_cycles = pc;
-    kp.fprof = sim->d_fprof;
-    kp.fine_cta = getenv("GEM_FINE_CTA") ? (uint32_t)atoi(getenv("GEM_FINE_CTA")) : 0u;
   }
-  CK(cudaMemsetAsync(sim->d_bar + sim->bar_off, 0, (size_t)(GEM_BAR_MAX_CTAS + 2) * GEM_BAR_STRIDE * 8, sim->stream));
+  CK(cudaMemsetAsync(sim->d_bar, 0, (size_t)(GEM_BAR_MAX_CTAS + 2) * GEM_BAR_STRIDE * 8, sim->stream));
   if (sim->flags & GEM_F_DIGEST)
     CK(cudaMemsetAsync(sim->d_digest, 0, (size_t)sim->n_streams * sim->out_cap * 8, sim->stream));
   if (sim->lanes) {
@@ -1802,7 +1745,7 @@ int gem_bench_floor(int device, uint32_t grid, uint32_t iters, double* layer_clk
   if (!layer_clk || !barrier_clk || !grid || grid > GEM_BAR_MAX_CTAS || !iters) return fail(GEM_E_INVAL, "bad floor request");
   CK(cudaSetDevice(device));
   unsigned long long *d_out = nullptr, *d_bar = nullptr;
-  int* d_err = nullptr;
+  uint32_t* d_err = nullptr;
   CK(dalloc(&d_out, 64));
   CK(dalloc(&d_bar, (size_t)(GEM_BAR_MAX_CTAS + 2) * GEM_BAR_STRIDE * 8));
   CK(dalloc(&d_err, 64));
@@ -1973,14 +1916,6 @@ int gem_write_ram(gem_sim* sim, uint32_t ram_id, uint32_t stream, const uint32_t
   return GEM_OK;
 }
 
-#ifdef GEM_FINE_PROF
-int gem_read_fine(gem_sim* sim, uint64_t* dst) {
-  CK(cudaStreamSynchronize(sim->stream));
-  CK(cudaMemcpy(dst, sim->d_fprof, GEM_FINE_LAYERS * 96 * 8, cudaMemcpyDeviceToHost));
-  return GEM_OK;
-}
-#endif
-
 int gem_read_profile(gem_sim* sim, uint64_t* dst, uint32_t* n_cycles, uint32_t* grid) {
   if (int r = check(sim)) return r;
   if (!(sim->flags & GEM_F_PROFILE) || !sim->d_prof) return fail(GEM_E_INVAL, "GEM_F_PROFILE not set / no step yet");
@@ -2012,13 +1947,15 @@ void gem_free(gem_sim* sim) {
   for (void* p : {(void*)sim->d_prog, (void*)sim->d_parts, (void*)sim->d_stage, (void*)sim->d_q_int_of_ext,
                   (void*)sim->d_q_ext_of_int, (void*)sim->d_po_int_of_ext, (void*)sim->d_q, (void*)sim->d_rd,
                   (void*)sim->d_cut, (void*)sim->d_mem, (void*)sim->d_pi, (void*)sim->d_po, (void*)sim->d_qtrace,
-                  (void*)sim->d_scratch, (void*)sim->d_digest, (void*)sim->d_bar, (void*)sim->d_err,
+                  (void*)sim->d_scratch, (void*)sim->d_digest, (void*)sim->d_bar,
                   (void*)sim->d_prof, (void*)sim->d_wl_off, (void*)sim->d_wl_items, (void*)sim->d_lprog,
                   (void*)sim->d_pi_lane, (void*)sim->d_po_lane, (void*)sim->d_act,
                   (void*)sim->d_dyn_units, (void*)sim->d_dyn_ctr})
     if (p) cudaFree(p);
   if (sim->ev0) cudaEventDestroy(sim->ev0);
   if (sim->ev1) cudaEventDestroy(sim->ev1);
+  if (sim->ev_in) cudaEventDestroy(sim->ev_in);
+  if (sim->h_err) cudaFreeHost(sim->h_err);
   if (sim->own_stream && sim->stream) cudaStreamDestroy(sim->stream);
   delete sim;
 }

@@ -20,6 +20,9 @@ GEM_F_DIGEST = 0x2
 GEM_F_ASYNC = 0x4
 GEM_F_PROFILE = 0x8
 GEM_F_ACTIVITY = 0x10
+GEM_F_NO_RESIDENT = 0x20
+GEM_F_NO_LANES = 0x40
+GEM_F_STATIC_LANES = 0x80
 ERRORS = {-1: "GEM_E_INVAL", -2: "GEM_E_FORMAT", -3: "GEM_E_CUDA", -4: "GEM_E_NOMEM", -5: "GEM_E_NOINPUT",
           -6: "GEM_E_UNSUPPORTED"}
 EXPORTS = ["gem_load_program", "gem_info_get", "gem_set_inputs", "gem_step", "gem_read_outputs",
@@ -29,7 +32,13 @@ EXPORTS = ["gem_load_program", "gem_info_get", "gem_set_inputs", "gem_step", "ge
 
 class GemConfig(ctypes.Structure):
     _fields_ = [("device", ctypes.c_int), ("n_streams", ctypes.c_uint32), ("cuda_stream", ctypes.c_void_p),
-                ("flags", ctypes.c_uint32), ("grid_limit", ctypes.c_uint32)]
+                ("flags", ctypes.c_uint32), ("grid_limit", ctypes.c_uint32),
+                ("ctas_per_sm", ctypes.c_uint32), ("max_group", ctypes.c_uint32),
+                ("lane_groups", ctypes.c_uint32), ("lane_ctas_per_sm", ctypes.c_uint32),
+                ("lane_run", ctypes.c_uint32), ("l2_evict_last", ctypes.c_float)]
+
+
+TUNING = ("ctas_per_sm", "max_group", "lane_groups", "lane_ctas_per_sm", "lane_run", "l2_evict_last")
 
 
 class GemInfo(ctypes.Structure):
@@ -113,9 +122,15 @@ class Simulator:
     """One loaded program on one GPU, with `n_streams` independent stimulus streams."""
 
     def __init__(self, blob: bytes, device: int = 0, n_streams: int = 1, flags: int = 0,
-                 cuda_stream: int = 0, grid_limit: int = 0):
+                 cuda_stream: int = 0, grid_limit: int = 0, **tuning):
+        """tuning: gem_config launch-tuning fields (TUNING; 0 = automatic)."""
         self.lib = load_library()
+        bad = set(tuning) - set(TUNING)
+        if bad:
+            raise TypeError(f"unknown gem_config fields {sorted(bad)}")
         cfg = GemConfig(device, n_streams, ctypes.c_void_p(cuda_stream or None), flags, grid_limit)
+        for k, v in tuning.items():
+            setattr(cfg, k, v)
         h = ctypes.c_void_p()
         self._blob = ctypes.create_string_buffer(blob, len(blob))
         self._check(self.lib.gem_load_program(self._blob, len(blob), ctypes.byref(cfg), ctypes.byref(h)))

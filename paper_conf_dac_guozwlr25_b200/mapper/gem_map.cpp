@@ -631,7 +631,9 @@ struct Mapper {
       bool any = false;
       for (uint32_t i = 0; i < n; i++) if (mc[i]) { any = true; break; }
       if (!any) break;
-      if (n_layers > 4096) { fail(P, "no progress"); return; }
+      // chunk table limit of the runtime (gem_isa.h GEM_MAX_CHUNKS = layers + 2):
+      // a failing partition is split by the caller
+      if (n_layers + 2 >= GEM_MAX_CHUNKS) { fail(P, "more than GEM_MAX_CHUNKS - 2 layers"); return; }
       // depth over realised set, reverse depth, leaf cost
       for (uint32_t i = 0; i < n; i++) {
         if (!mc[i]) continue;
@@ -773,8 +775,6 @@ struct Mapper {
         if (*tgt < 0) { fail(P, "state overflow"); return; }
         loc[x] = (int32_t)((uint32_t)*tgt * 32 + slot_bit(k, id));
         word_vals[(uint32_t)*tgt].push_back(x);
-        if (getenv("GEM_DBG_X") && x == (uint32_t)atoi(getenv("GEM_DBG_X")))
-          fprintf(stderr, "dbg: x=%u written out in layer %u k=%d id=%u loc=%d\n", x, n_layers, k, id, loc[x]);
       }
       if (opt.verbose >= 2) {
         uint32_t nwo = 0;

@@ -8,9 +8,6 @@ import numpy as np  # noqa: E402
 
 from gen import stimulus  # noqa: E402
 from paper_conf_dac_guozwlr25_b200 import _build  # noqa: E402
-if os.environ.get("GEM_EXP_LIB"):   # timing experiments (scripts/experiment.py)
-    _build.LIBGEM = os.environ["GEM_EXP_LIB"]
-    _build.build_libgem = lambda force=False, extra=(): _build.LIBGEM
 from paper_conf_dac_guozwlr25_b200 import gem  # noqa: E402
 from tests.common import blob  # noqa: E402
 

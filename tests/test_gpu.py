@@ -119,17 +119,14 @@ def test_activity_pruning_ram_stages_streamed(gem, tmp_path):
     st = hold(stim_random(net.n_pi, 100, 3, reset_pi0_cycles=2), 4)
     for opts, kw in [("parts=5", {}), ("parts=5 stages=2", {}), ("parts=5", {"grid_limit": 2})]:
         _full_parity(gem, p, compile_file(p, opts), st, chunks=(7, 200), extra_flags=gem.GEM_F_ACTIVITY, **kw)
-    import os
-    os.environ["GEM_NO_RESIDENT"] = "1"
-    try:
-        _full_parity(gem, p, compile_file(p, "parts=5"), st, extra_flags=gem.GEM_F_ACTIVITY)
-    finally:
-        del os.environ["GEM_NO_RESIDENT"]
+    _full_parity(gem, p, compile_file(p, "parts=5"), st, extra_flags=gem.GEM_F_ACTIVITY | gem.GEM_F_NO_RESIDENT)
     _full_parity(gem, eaig("c1"), blob("c1"), hold(stimulus("c1", 35, 500), 3), extra_flags=gem.GEM_F_ACTIVITY)
 
 
 def test_c2_full_parity(gem):
-    _full_parity(gem, eaig("c2"), blob("c2"), stimulus("c2", 128, 2000))
+    """C2 (100K ANDs, 4K flops): full PO and flop vectors every cycle for 10,000
+    cycles, in ragged gem_step chunks (SURVEY §8(c) protocol for C1-C2)."""
+    _full_parity(gem, eaig("c2"), blob("c2"), stimulus("c2", 128, 10_000), chunks=(3000, 3001, 7777))
 
 
 def test_c3_parity_digests_and_ram(gem):
@@ -217,7 +214,7 @@ def test_c5_ragged_stream_groups(gem):
                                       ("parts=4 lanes=1", "1")])
 def test_lane_mode_stages_and_work_distribution(gem, monkeypatch, tmp_path, opts, dyn):
     """Lane mode with two stages (static work lists, cut words between stages)
-    and one stage with static (GEM_LANE_DYN=0) or dynamic ticketed work
+    and one stage with static (GEM_F_STATIC_LANES) or dynamic ticketed work
     distribution: 96 streams match the 64-lane oracle bit-exactly."""
     from paper_conf_dac_guozwlr25_b200.mapping import compile_file
     S, T = 96, 50
@@ -225,8 +222,8 @@ def test_lane_mode_stages_and_work_distribution(gem, monkeypatch, tmp_path, opts
     path = circuits.save(net, str(tmp_path), "g")
     b = compile_file(path, opts)
     st = np.stack([stim_random(net.n_pi, T, 2000 + s, reset_pi0_cycles=2) for s in range(S)])
-    monkeypatch.setenv("GEM_LANE_DYN", dyn)
-    sim = gem.Simulator(b, n_streams=S, flags=gem.GEM_F_DIGEST, grid_limit=3)
+    flags = gem.GEM_F_DIGEST | (gem.GEM_F_STATIC_LANES if dyn == "0" else 0)
+    sim = gem.Simulator(b, n_streams=S, flags=flags, grid_limit=3)
     assert sim.info["lanes"] == 1
     sim.set_inputs(st)
     sim.step(T)
@@ -256,9 +253,7 @@ def test_lane_interleaved_groups_ragged(gem, monkeypatch, tmp_path, k):
         path = circuits.save(net, str(tmp_path), "g")
         b, n_pi = compile_file(path, "parts=3 lanes=1"), net.n_pi
         st = np.stack([stim_random(n_pi, T, 1000 + s, reset_pi0_cycles=2) for s in range(S)])
-    monkeypatch.setenv("GEM_LANE_BPS", "1")
-    monkeypatch.setenv("GEM_LANE_GROUPS", str(k))
-    sim = gem.Simulator(b, n_streams=S, flags=gem.GEM_F_DIGEST)
+    sim = gem.Simulator(b, n_streams=S, flags=gem.GEM_F_DIGEST, lane_ctas_per_sm=1, lane_groups=k)
     assert sim.info["lanes"] == 1 and sim.info["group"] == 32 * k
     sim.set_inputs(st)
     sim.step(T)
@@ -279,8 +274,7 @@ def test_c5_lane_mode_equals_packed_mode(gem, monkeypatch):
     st = stimulus_streams("c5", 256, T, range(7, 7 + S))
     lane = gem.Simulator(blob("c5"), n_streams=S)
     assert lane.info["lanes"] == 1
-    monkeypatch.setenv("GEM_NO_LANES", "1")
-    packed = gem.Simulator(blob("c5"), n_streams=S)
+    packed = gem.Simulator(blob("c5"), n_streams=S, flags=gem.GEM_F_NO_LANES)
     assert packed.info["lanes"] == 0
     assert np.array_equal(lane.run(st), packed.run(st))
     assert np.array_equal(lane.read_state(), packed.read_state())
@@ -332,7 +326,7 @@ def _golden_rows(name):
     return rows
 
 
-@pytest.mark.parametrize("name", ["half_adder", "toggle", "toggle_init1"])
+@pytest.mark.parametrize("name", ["half_adder", "toggle", "toggle_init1", "toggle_uninit"])
 def test_golden_worked_examples(gem, name):
     """The AIGER-specification worked examples (tests/golden, cited in each
     .expected): a design with no flops (half adder) and designs with no AND
@@ -390,3 +384,143 @@ def test_wires_constants_and_step0(gem, tmp_path):
     assert np.array_equal(np.concatenate([po_a, po_b], 1)[0], r["po"])
     assert np.array_equal(q1[0], r["state"][119])
     assert np.array_equal(sim.read_state()[0], o.get_state())
+
+
+# ------------------------------------------------------------ round-2 parity gaps
+def test_c3_2000_cycles_ten_checkpoints(gem):
+    """C3 as bench.py maps it: 2,000 cycles in 10 steps of 200; full PO trace and
+    per-cycle flop digests, and the full flop vector and both RAM blocks at
+    each of the 10 checkpoints (SURVEY §8(c) protocol for C3-C5)."""
+    T, K = 2000, 10
+    st = stimulus("c3", 256, T)
+    sim = gem.Simulator(blob("c3"), flags=gem.GEM_F_DIGEST)
+    o = Oracle(eaig("c3"))
+    for k in range(K):
+        a, e = k * T // K, (k + 1) * T // K
+        sim.set_inputs(st[a:e])
+        sim.step(e - a)
+        r = o.run(st[a:e], digest=True)
+        assert np.array_equal(sim.read_outputs(e - a)[0], r["po"]), ("PO", k)
+        assert np.array_equal(sim.read_digests(e - a)[0], r["digest"]), ("digest", k)
+        assert np.array_equal(sim.read_state()[0], o.get_state()), ("state", k)
+        for ram in range(o.n_rams):
+            assert np.array_equal(sim.read_ram(ram), o.get_ram(ram)), ("ram", k, ram)
+
+
+def test_c5_bench_size_sampled_shards(gem):
+    """C5 in bench.py's launch configuration (4096 streams on one GPU, lane mode,
+    >= 8 dynamic work units per CTA), 100 cycles: PO trace, per-cycle digests,
+    final flops and RAM contents of 1,024 streams = 16 full 64-lane oracle
+    groups, covering stream 0, stream 4095 and both sides of every boundary of
+    the 2-, 4- and 8-way GPU shards (511|512, 1023|1024, ..., 3583|3584)."""
+    S, T = 4096, 100
+    sim = gem.Simulator(blob("c5"), n_streams=S, flags=gem.GEM_F_DIGEST)
+    info = sim.info
+    assert info["lanes"] == 1 and info["group"] == 64
+    items = info["n_parts"] * (S // info["group"])
+    assert items >= 8 * info["grid"], (items, info["grid"])   # run = 1: >= 8 dynamic units per CTA
+    groups = sorted({0, 63} | {g for b in range(512, 4096, 512) for g in (b // 64 - 1, b // 64)})
+    assert len(groups) == 16
+    streams = [64 * g + l for g in groups for l in range(64)]
+    st_all = np.zeros((S, T, 8), np.uint32)
+    st_sel = stimulus_streams("c5", 256, T, streams)
+    st_all[streams] = st_sel
+    rest = [s for s in range(S) if s not in set(streams)]
+    st_all[rest] = stimulus_streams("c5", 256, T, rest[::97])[np.arange(len(rest)) % len(rest[::97])]
+    sim.set_inputs(st_all)
+    sim.step(T)
+    po, dg, q = sim.read_outputs(T), sim.read_digests(T), sim.read_state()
+    o = Oracle(eaig("c5"))
+    o.lanes_reset(len(groups))
+    for j, g in enumerate(groups):
+        lo = 64 * g
+        r = o.lanes_run(j, st_all[lo:lo + 64], digest=True)
+        assert np.array_equal(po[lo:lo + 64], r["po"]), ("PO", g)
+        assert np.array_equal(dg[lo:lo + 64], r["digest"]), ("digest", g)
+        for lane in range(64):
+            assert np.array_equal(q[lo + lane], o.lanes_get_state(j, lane)), ("state", g, lane)
+        for lane in (0, 31, 32, 63):
+            for ram in range(o.n_rams):
+                assert np.array_equal(sim.read_ram(ram, lo + lane), o.lanes_get_ram(j, lane, ram)), (g, lane, ram)
+
+
+@pytest.mark.parametrize("lanes", [False, True])
+def test_ram_preload(gem, tmp_path, lanes):
+    """gem_write_ram (RAM preload before the first cycle, include/gem.h; oracle
+    side orc_set_ram, pinned in tests/test_oracle.py): random contents per
+    block and stream, then 300 cycles; PO/flop trace, final flops and RAM
+    contents equal the oracle's, on the bit-packed path (3 streams, two stages)
+    and in lane mode (64 streams)."""
+    from paper_conf_dac_guozwlr25_b200.mapping import compile_file
+    net = circuits.small_G(seed=21, n_and=4000, with_ram=True)
+    p = circuits.save(net, str(tmp_path), "g")
+    S = 64 if lanes else 3
+    T = 300 if not lanes else 120
+    rng = np.random.default_rng(77)
+    st = np.stack([stim_random(net.n_pi, T, 500 + s, reset_pi0_cycles=2) for s in range(S)])
+    b = compile_file(p, "parts=4 lanes=1" if lanes else "parts=4 stages=2")
+    sim = gem.Simulator(b, n_streams=S, flags=gem.GEM_F_DIGEST)
+    assert sim.info["lanes"] == int(lanes)
+    o = Oracle(p)
+    assert o.n_rams >= 1
+    pre = rng.integers(0, 1 << 32, size=(S, o.n_rams, 8192), dtype=np.uint64).astype(np.uint32)
+    for s in range(S):
+        for r in range(o.n_rams):
+            sim.write_ram(r, pre[s, r], stream=s)
+    sim.set_inputs(st)
+    sim.step(T)
+    po, dg, q = sim.read_outputs(T), sim.read_digests(T), sim.read_state()
+    if lanes:
+        o.lanes_reset(1)
+        for s in range(S):
+            for r in range(o.n_rams):
+                o.lanes_set_ram(0, s, r, pre[s, r])
+        res = o.lanes_run(0, st, digest=True)
+        assert np.array_equal(po, res["po"]) and np.array_equal(dg, res["digest"])
+        for s in (0, 17, 63):
+            assert np.array_equal(q[s], o.lanes_get_state(0, s))
+            for r in range(o.n_rams):
+                assert np.array_equal(sim.read_ram(r, s), o.lanes_get_ram(0, s, r))
+    else:
+        for s in range(S):
+            os_ = Oracle(p)
+            for r in range(o.n_rams):
+                os_.set_ram(r, pre[s, r])
+            res = os_.run(st[s], digest=True)
+            assert np.array_equal(po[s], res["po"]) and np.array_equal(dg[s], res["digest"]), s
+            assert np.array_equal(q[s], os_.get_state())
+            for r in range(o.n_rams):
+                assert np.array_equal(sim.read_ram(r, s), os_.get_ram(r))
+    # preloading changes the trace (the RAM data reaches the outputs / flops)
+    ref0 = Oracle(p).run(st[0], digest=True)
+    assert not np.array_equal(dg[0], ref0["digest"])
+
+
+def test_uninitialised_latches_read_zero(gem, tmp_path):
+    """Reading U5 on a design with many latches: every latch of a random
+    sequential design declared uninitialised (AIGER "cur next cur") behaves
+    exactly like init 0 on the GPU and in the oracle, and unlike init 1."""
+    from gen.aig import write_eaig
+    from paper_conf_dac_guozwlr25_b200.mapping import compile_file
+    net = circuits.small_G(seed=5, n_and=2000, with_ram=False, reset=False)
+    p0 = circuits.save(net, str(tmp_path), "init0")
+    txt = open(p0).read().split("\n")
+    hdr = txt[0].split()
+    I, L = int(hdr[2]), int(hdr[3])
+    def variant(kind):
+        lines = list(txt)
+        for j in range(L):
+            f = lines[1 + I + j].split()
+            cur = f[0]
+            lines[1 + I + j] = f"{f[0]} {f[1]} " + {"uninit": cur, "one": "1"}[kind]
+        q = str(tmp_path / f"{kind}.aag")
+        open(q, "w").write("\n".join(lines))
+        return q
+    pu, p1 = variant("uninit"), variant("one")
+    st = stim_random(net.n_pi, 200, 9)
+    runs = {}
+    for name, p in (("zero", p0), ("uninit", pu), ("one", p1)):
+        sim = _full_parity(gem, p, compile_file(p), st)
+        runs[name] = sim.read_state()
+    assert np.array_equal(runs["zero"], runs["uninit"])
+    assert Oracle(pu).get_state().sum() == 0 and Oracle(p1).get_state().any()

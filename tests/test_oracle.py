@@ -45,7 +45,7 @@ def test_golden_half_adder():
     assert po.tolist() == [r[1] for r in rows]
 
 
-@pytest.mark.parametrize("name", ["toggle", "toggle_init1"])
+@pytest.mark.parametrize("name", ["toggle", "toggle_init1", "toggle_uninit"])
 def test_golden_toggle(name):
     o = Oracle(os.path.join(GOLD, name + ".aag"))
     rows = _read_expected(name + ".expected")
@@ -280,6 +280,58 @@ def test_ram_write_then_read_latency(tmp_path):
         bits[0, 58 + i] = 1
     po = unpack_bits(o.run(pack_bits(bits))["po"], 32)
     assert [_num(r) for r in po] == [0, 0, k, 0]
+
+
+def test_ram_preload_dict_model(tmp_path):
+    """orc_set_ram (the oracle side of gem_write_ram): a block preloaded with
+    random contents is read first-then-written exactly like the dict model of
+    test_ram_read_first_dict_model started from those contents (U7-U10); the
+    64-lane variant with per-lane preloads gives every lane its own model."""
+    p = circuits.save(circuits.ram_direct(), str(tmp_path), "ram")
+    rng = np.random.default_rng(19)
+    T = 400
+    init = rng.integers(0, 1 << 32, 8192, dtype=np.uint64).astype(np.uint32)
+    ra = rng.integers(0, 64, T)
+    wa = np.where(rng.random(T) < 0.5, ra, rng.integers(0, 64, T))
+    wd = rng.integers(0, 1 << 32, T, dtype=np.uint64)
+    be = np.where(rng.random(T) < 0.4, 0, rng.integers(0, 1 << 32, T, dtype=np.uint64))
+    bits = np.zeros((T, 90), np.uint8)
+    for k in range(13):
+        bits[:, k] = (ra >> k) & 1
+        bits[:, 13 + k] = (wa >> k) & 1
+    for k in range(32):
+        bits[:, 26 + k] = (wd.astype(np.int64) >> k) & 1
+        bits[:, 58 + k] = (be.astype(np.int64) >> k) & 1
+    stim = pack_bits(bits)
+
+    def model(mem0):
+        mem = {a_: int(mem0[a_]) for a_ in range(8192)}
+        rd, out = 0, []
+        for t in range(T):
+            out.append(rd)
+            new_rd = mem[int(ra[t])]
+            m = int(be[t])
+            mem[int(wa[t])] = (mem[int(wa[t])] & ~m & 0xFFFFFFFF) | (int(wd[t]) & m)
+            rd = new_rd
+        return out, np.array([mem[a_] for a_ in range(8192)], np.uint32)
+
+    exp_po, exp_mem = model(init)
+    o = Oracle(p)
+    o.set_ram(0, init)
+    po = unpack_bits(o.run(stim)["po"], 32)
+    assert [_num(r) for r in po] == exp_po
+    assert np.array_equal(o.get_ram(0), exp_mem)
+    # 64-lane group: lane l preloaded with init ^ l, same port traffic
+    o.lanes_reset(1)
+    for lane in (0, 5, 63):
+        o.lanes_set_ram(0, lane, 0, init ^ np.uint32(lane))
+    r = o.lanes_run(0, np.broadcast_to(stim, (64,) + stim.shape))
+    for lane in (0, 5, 63):
+        e_po, e_mem = model(init ^ np.uint32(lane))
+        assert [_num(x) for x in unpack_bits(r["po"][lane], 32)] == e_po, lane
+        assert np.array_equal(o.lanes_get_ram(0, lane, 0), e_mem), lane
+    e_po0, _ = model(np.zeros(8192, np.uint32))
+    assert [_num(x) for x in unpack_bits(r["po"][1], 32)] == e_po0   # not preloaded: U10 zeros
 
 
 # ------------------------------------------------------------------ invariants
