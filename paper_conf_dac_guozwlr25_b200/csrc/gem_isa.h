@@ -107,6 +107,9 @@ enum {
   GH_MAX_CHUNK_WORDS, GH_MAX_PROG_WORDS,
   GH_HAS_LANES, GH_OFF_LANE_PROG, GH_LANE_PROG_WORDS_LO, GH_LANE_PROG_WORDS_HI, GH_LANE_MAX_CHUNK_WORDS,
   GH_LANE_MAX_WORDS, GH_MAX_RAMS_PART,
+  GH_N_AND_SYNTH_LO, GH_N_AND_SYNTH_HI,  /* live ANDs after depth-oriented synthesis (GH_N_AND: before) */
+  GH_LEVELS_IN,                         /* logic depth before synthesis (GH_MAX_LEVELS: after)       */
+  GH_SYNTH_CHAINS,                      /* chains rewritten by the lookahead                          */
   GH_N_WORDS = 64
 };
 

@@ -11,7 +11,9 @@ GH = ["MAGIC", "VERSION", "N_PI", "N_PO", "N_FLOPS", "N_RAMS", "N_PARTS", "N_STA
       "TOTAL_LEAVES_LO", "TOTAL_LEAVES_HI", "OFF_PARTS", "OFF_STAGES", "OFF_FLOP_INIT",
       "OFF_PROG", "PROG_WORDS_LO", "PROG_WORDS_HI", "MAX_LEVELS", "TOTAL_WRITEOUTS",
       "MAX_OUT", "TOTAL_WORDS_LO", "TOTAL_WORDS_HI", "SLOTS_USED_LO", "SLOTS_USED_HI",
-      "MAX_CHUNK_WORDS", "MAX_PROG_WORDS"]
+      "MAX_CHUNK_WORDS", "MAX_PROG_WORDS", "HAS_LANES", "OFF_LANE_PROG", "LANE_PROG_WORDS_LO",
+      "LANE_PROG_WORDS_HI", "LANE_MAX_CHUNK_WORDS", "LANE_MAX_WORDS", "MAX_RAMS_PART",
+      "N_AND_SYNTH_LO", "N_AND_SYNTH_HI", "LEVELS_IN", "SYNTH_CHAINS"]
 GP_WORDS = 16   # csrc/gem_isa.h GP_WORDS
 GEM_MAGIC = 0x424D4547
 SLOTS_PER_LAYER = 8191
@@ -43,6 +45,9 @@ class BlobInfo:
     max_prog_words: int = 0
     part_cost: list = None
     part_stage: list = None
+    n_and_synth: int = 0
+    levels_in: int = 0
+    synth_chains: int = 0
 
     def stage_max_layers(self) -> list:
         """Deepest partition (layers) of each stage: a lower bound on the layers
@@ -54,7 +59,13 @@ class BlobInfo:
 
     @property
     def replication(self) -> float:
-        return self.n_and_mapped / max(1, self.n_and) - 1.0
+        """RepCut replication over the synthesised graph."""
+        return self.n_and_mapped / max(1, self.n_and_synth or self.n_and) - 1.0
+
+    @property
+    def synth_growth(self) -> float:
+        """AND gates added by depth-oriented synthesis, relative."""
+        return (self.n_and_synth or self.n_and) / max(1, self.n_and) - 1.0
 
     @property
     def slot_util(self) -> float:
@@ -69,7 +80,8 @@ class BlobInfo:
         d.pop("part_layers")
         d.pop("part_cost", None)
         d.pop("part_stage", None)
-        d.update(replication=self.replication, slot_util=self.slot_util, bytes_per_and=self.bytes_per_and,
+        d.update(replication=self.replication, synth_growth=self.synth_growth, slot_util=self.slot_util,
+                 bytes_per_and=self.bytes_per_and,
                  levels_per_layer=self.max_levels / max(1, self.max_layers))
         return d
 
@@ -90,4 +102,5 @@ def blob_info(blob: bytes) -> BlobInfo:
                     max_levels=h["MAX_LEVELS"], program_bytes=4 * u64("PROG_WORDS"),
                     blob_bytes=len(blob), slots_used=u64("SLOTS_USED"), part_layers=pt[:, 3].tolist(),
                     max_chunk_words=h["MAX_CHUNK_WORDS"], max_prog_words=h["MAX_PROG_WORDS"],
-                    part_cost=pt[:, 8].tolist(), part_stage=pt[:, 0].tolist())
+                    part_cost=pt[:, 8].tolist(), part_stage=pt[:, 0].tolist(),
+                    n_and_synth=u64("N_AND_SYNTH"), levels_in=h["LEVELS_IN"], synth_chains=h["SYNTH_CHAINS"])

@@ -35,6 +35,7 @@
 #include <fstream>
 #include <functional>
 #include <map>
+#include <memory>
 #include <mutex>
 #include <numeric>
 #include <sstream>
@@ -76,6 +77,10 @@ struct Options {
   int verbose = 0;
   int max_state_words = GEM_MAX_STATE_WORDS;
   double cap_slack = 1.0;
+  int synth = 2;            // depth-oriented synthesis (gem_synth.h): 0 strash only, 1 + AND balancing,
+                            // 2 + chain lookahead
+  int chain_min = 8;        // shortest chain rewritten by the lookahead
+  int chain_slack = 2;      // a link's chain edge arrives >= this many levels after its side input
 };
 
 static Options parse_opts(const char* s) {
@@ -110,6 +115,9 @@ static Options parse_opts(const char* s) {
     else if (k == "max_warps") o.max_warps = std::max(1, std::min(8, std::stoi(v)));
     else if (k == "lane_holes") o.lane_holes = std::max(1, std::stoi(v));
     else if (k == "banks") o.banks = std::stoi(v);
+    else if (k == "synth") o.synth = std::stoi(v);
+    else if (k == "chain_min") o.chain_min = std::max(2, std::stoi(v));
+    else if (k == "chain_slack") o.chain_slack = std::max(1, std::stoi(v));
     else throw std::runtime_error("unknown option " + k);
   }
   if (o.stages < 1 || o.stages > 2) throw std::runtime_error("stages must be 1 or 2");
@@ -405,6 +413,8 @@ static Graph build_graph(const Raw& r) {
     if (live[i] && g.kind[i] == K_AND) { g.n_and_live++; g.max_level = std::max(g.max_level, g.level[i]); }
   return g;
 }
+
+#include "gem_synth.h"
 
 // =========================================================== partition description
 // An output word: destination gid + 32 compact literals (bit k of the word).
@@ -1565,6 +1575,7 @@ static uint32_t part_cost(const uint32_t* pr) {
 // =========================================================== partitioning
 struct Design {
   Graph G;
+  SynthStats synth;                 // depth-oriented synthesis report (gem_synth.h)
   std::vector<uint32_t> ext_gbit;   // source locations before the internal flop layout
   Options opt;
   std::vector<Part> parts;
@@ -1973,6 +1984,13 @@ static Blob compile(const char* data, size_t n, const char* opts) {
   D.G = build_graph(raw);
   raw = Raw();
   tick("strash");
+  D.G = synthesize(D.G, D.opt.synth, D.opt.chain_min, D.opt.chain_slack, D.synth);
+  tick("synth");
+  if (D.opt.verbose)
+    fprintf(stderr, "gem_map: synth ANDs %llu -> %llu (balanced %llu), levels %u -> %u (balanced %u), "
+            "%u chains / %u links / %u taps\n", (unsigned long long)D.synth.and_in, (unsigned long long)D.synth.and_out,
+            (unsigned long long)D.synth.and_balanced, D.synth.level_in, D.synth.level_out, D.synth.level_balanced,
+            D.synth.chains, D.synth.chain_links, D.synth.chain_taps);
   partition(D);
   tick("partition");
   // remember which compact nodes are cut nodes (stage-1 leaves) before layout rewrites cut_lit
@@ -2129,8 +2147,14 @@ static Blob compile(const char* data, size_t n, const char* opts) {
   w[GH_PO_WORDS] = D.po_words;
   w[GH_Q_WORDS] = D.q_words;
   w[GH_CUT_WORDS] = D.cut_words;
-  w[GH_N_AND_LO] = (uint32_t)D.G.n_and_live;
-  w[GH_N_AND_HI] = (uint32_t)(D.G.n_and_live >> 32);
+  // gate evals (reading U14): live ANDs of the design before depth-oriented
+  // synthesis and replication; the synthesised count and depths ride along
+  w[GH_N_AND_LO] = (uint32_t)D.synth.and_in;
+  w[GH_N_AND_HI] = (uint32_t)(D.synth.and_in >> 32);
+  w[GH_N_AND_SYNTH_LO] = (uint32_t)D.G.n_and_live;
+  w[GH_N_AND_SYNTH_HI] = (uint32_t)(D.G.n_and_live >> 32);
+  w[GH_LEVELS_IN] = D.synth.level_in;
+  w[GH_SYNTH_CHAINS] = D.synth.chains;
   uint64_t mapped = 0, leaves = 0, slots = 0;
   uint32_t maxl = 0, maxs = 0, tl = 0, two_ = 0, maxout = 0;
   for (auto& P : D.parts) {
