@@ -330,7 +330,7 @@ static ChainNet<BLD, LEAF> make_net(const Graph& g, const ChainDef& c, BLD& b, L
 
 static Graph chain_lookahead(const Graph& g, int min_len, int slack, SynthStats& st) {
   const size_t N = g.kind.size();
-  const uint32_t kMaxBack = 4, kMaxCone = 16;
+  const uint32_t kMaxBack = 8, kMaxCone = 32;
   std::vector<uint32_t> refs;
   std::vector<uint8_t> comp, ep;
   ref_counts(g, refs, comp, ep);

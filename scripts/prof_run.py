@@ -22,7 +22,7 @@ a = ap.parse_args()
 b = blob(a.cfg, a.map_opts)
 sim = gem.Simulator(b, n_streams=a.streams)
 n_pi = sim.info["n_pi"]
-st = np.stack([stimulus("c3" if a.cfg == "c5" else a.cfg, n_pi, a.cycles * a.launches, seed=100 + s)
+st = np.stack([stimulus("c3" if a.cfg == "c5" else a.cfg, n_pi, max(200, a.cycles * a.launches), seed=100 + s)
                for s in range(a.streams)])
 sim.set_inputs(st)
 for k in range(a.launches):

@@ -159,3 +159,40 @@ def gated_modules(n_blocks: int = 64, flops: int = 64, width: int = 256, depth: 
         for i in range(8):
             b.output(q[i])
     return b.finish()
+
+
+def deep_chains(width: int = 64, chain: int = 120, seed: int = 3) -> Netlist:
+    """Depth-synthesis workload (gem_synth.h): a `width`-bit ripple-carry
+    adder of two PIs words plus a flop word (majority-cell carry chain), a
+    `width`-bit incrementer of a flop word (AND chain), a `chain`-long
+    AND/OR priority chain with random edge inversions (single-AND links), and
+    a linear 48-input AND (a balancing supergate).  POs: every sum bit, the
+    carry out, every priority-chain node, the wide AND."""
+    rng = np.random.default_rng(seed)
+    b = AigBuilder(f"chains{seed}")
+    x = b.inputs_n(width)
+    y = b.inputs_n(width)
+    en = b.input()
+    q = [b.latch() for _ in range(width)]
+    r = [b.latch() for _ in range(width)]
+    c = en
+    for i in range(width):                        # r' = r + 1 (when en): incrementer
+        b.set_next(r[i], b.XOR(r[i], c))
+        c = b.AND(r[i], c)
+    c = b.AND(x[0], en)
+    for i in range(width):                        # s = x + y + q: two ripple adders
+        t, c1 = b.full_adder(x[i], y[i], c)
+        s, c = b.full_adder(t, q[i], c1)
+        b.output(s)
+        b.set_next(q[i], s)
+    b.output(c)
+    side = b.inputs_n(16)
+    n = side[0]
+    for k in range(chain):                        # alternating AND/OR priority chain
+        n = b.AND(n ^ int(rng.integers(0, 2)), side[int(rng.integers(0, 16))] ^ int(rng.integers(0, 2)))
+        b.output(n)
+    a = x[0]
+    for i in range(1, 48):
+        a = b.AND(a, y[i % width])
+    b.output(a)
+    return b.finish()

@@ -60,6 +60,49 @@ def test_random_comb_and_cells(tmp_path, seed):
         _check(p, b, st)
 
 
+@pytest.mark.parametrize("synth", [0, 1, 2])
+def test_depth_synthesis_preserves_function(tmp_path, synth):
+    """Depth-oriented synthesis (gem_synth.h: AND balancing, chain
+    lookahead) is an identity of Boolean algebra: the mapped program of every
+    synthesis level reproduces the oracle, which runs the ORIGINAL netlist."""
+    net = circuits.deep_chains(48, 90, seed=synth + 5)
+    p = circuits.save(net, str(tmp_path), "chains")
+    b = compile_file(p, f"synth={synth} parts=2")
+    n_pi = Oracle(p).n_pi
+    rng = np.random.default_rng(synth)
+    st = rng.integers(0, 1 << 32, size=(300, (n_pi + 31) // 32), dtype=np.uint64).astype(np.uint32)
+    st[:, -1] &= (1 << (n_pi % 32)) - 1
+    _check(p, b, st)
+
+
+def test_depth_synthesis_reduces_levels(tmp_path):
+    """Chains of length n go from O(n) to O(log n) levels: a 64-bit two-adder
+    carry chain (majority cells), a 64-bit incrementer and a 200-link AND/OR
+    priority chain (depth >= 128 before) end below 40 levels; balancing alone
+    turns the 48-input linear AND into a tree; the live AND count is the
+    pre-synthesis one (reading U14) and the synthesised one is reported."""
+    net = circuits.deep_chains(64, 200, seed=1)
+    p = circuits.save(net, str(tmp_path), "chains")
+    i0 = blob_info(compile_file(p, "synth=0"))
+    i1 = blob_info(compile_file(p, "synth=1"))
+    i2 = blob_info(compile_file(p, "synth=2"))
+    assert i0.max_levels == i0.levels_in >= 200
+    assert i1.levels_in == i0.levels_in and i2.levels_in == i0.levels_in
+    assert i2.max_levels <= 40 and i2.synth_chains >= 3, (i2.max_levels, i2.synth_chains)
+    assert i2.max_layers < i0.max_layers
+    assert i0.n_and == i1.n_and == i2.n_and and i2.n_and_synth > i0.n_and
+    assert i1.synth_chains == 0 and i1.n_and_synth <= i0.n_and
+
+
+def test_c3_synthesis_depth():
+    """BASELINE config 3's deep long-tailed paths (carry-chain tails):
+    synthesis cuts the logic depth by > 2x and the critical layers with it."""
+    i = blob_info(blob("c3"))
+    assert i.levels_in == 129 and i.max_levels <= 64, (i.levels_in, i.max_levels)
+    assert sum(i.stage_max_layers()) <= 10
+    assert i.synth_growth < 0.10
+
+
 def test_c2_prefix():
     _check(eaig("c2"), blob("c2"), stimulus("c2", 128, 120))
 
