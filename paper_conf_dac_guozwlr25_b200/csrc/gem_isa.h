@@ -229,3 +229,28 @@ enum { LLH_WORDS_ = 0, LLH_FLAGS, LLH_TOPC, LLH_TOPWO, LLH_WOFF0 /* ..+7 */, LLH
 #define GEM_LWREC_LEAVES (GEM_LWREC_HDR + 128)
 #define GEM_LWREC_BASE (GEM_LWREC_HDR + 128 + 512)
 #define GEM_LWREC_WORDS (GEM_LWREC_BASE + 32)
+
+/* ---------------------------------------------------------------------------
+ * Lane mode, compacted program (magic "LAN2", mapper lane_mode=2, the default).
+ * The boomerang placement evaluates every slot of every layer, 8191 per
+ * layer, of which C5 uses 42% as real ANDs (the rest are pass-throughs, empty
+ * slots and tree-expanded copies); with whole lane words in shared memory a
+ * signal needs no bit permutation and no fan-out duplication, so the lane
+ * program is the partition's AND list itself, list-scheduled into STEPS of at
+ * most 256 independent ANDs (one per thread) separated by a block barrier:
+ *   header (LPH_*, LPH_N_LAYERS = n_steps, LPH_OFF_LAYERS = op array)
+ *   gread:  one u32 gid_l per entry, entry k -> lane word k + 1 (as "LANE")
+ *   ops:    [n_steps][256] uint2 {x, y}, thread t of step s runs op s*256+t:
+ *             x = a | ia << 14 | b << 16 | ib << 30   (lane words < 16384)
+ *             y = destination lane word (0 = no op)
+ *           result(y) = (S[a] ^ -ia) & (S[b] ^ -ib); operands were written in
+ *           earlier steps; a destination is never read in the same step.
+ *   out, ram: as "LANE".
+ * Words are allocated by liveness (free after the last reading step) with
+ * the destination residues of each half-warp chosen apart (LDS.64/STS.64 of
+ * two interleaved 32-stream groups are conflict-free when the 16 lanes of a
+ * half-warp touch different word residues mod 16).                        */
+#define GEM_LANE2_MAGIC 0x324E414Cu  /* "LAN2" */
+#define GEM_LANE2_STEP 256
+#define GEM_LANE2_OP_X(a, ia, b, ib) \
+  ((uint32_t)(a) | ((uint32_t)(ia) << 14) | ((uint32_t)(b) << 16) | ((uint32_t)(ib) << 30))

@@ -233,42 +233,16 @@ __device__ __forceinline__ void top_lane_layer(uint32_t topc, uint32_t topwo, ui
   if (lane == 0) lane_woK<K>(s_base, tm, tb, 6u, x);
 }
 
-// One work item: partition p for the 32-stream groups g0 .. g0+ng-1 (ng <= K;
-// groups ng..K-1 of the vectors are padding and never committed).
+// ---- a2 in lane mode: input ports of an item's groups (once per cycle).
+// Entry k (one u32 gid per entry) goes to lane word k + 1.  A thread takes 4
+// consecutive entries per uint4 and up to 16 per pass: all entry loads, then
+// all value loads, then the stores (two L2 round trips per pass, not per entry)
 template <int K>
-__device__ void run_lane_partition(const KParams& kp, uint32_t* S, uint32_t* ramp, uint32_t* topv, uint32_t p,
-                                   uint32_t g0, uint32_t ng, uint32_t c, uint32_t cur, uint32_t nxt,
-                                   unsigned long long* pacc) {
+__device__ __forceinline__ void lane_ports(const KParams& kp, uint32_t s_base, const uint32_t* gread, uint32_t n_gread,
+                                           uint32_t g0, uint32_t ng, uint32_t c, uint32_t cur) {
   const uint32_t tid = threadIdx.x;
-  // GEM_F_PROFILE: thread 0 accumulates per-phase clocks over the CTA's items
-  unsigned long long t_ph = (pacc && tid == 0) ? clock64() : 0ull;
-  auto phase = [&](int k) {
-    if (pacc && tid == 0) {
-      const unsigned long long t = clock64();
-      pacc[k] += t - t_ph;
-      t_ph = t;
-    }
-  };
-  const uint32_t s_base = smem_u32(S);
   const LaneIdx X{kp.n_groups};
-  const uint32_t* gprog = kp.lprog + __ldg(kp.parts + p * GP_WORDS + GP_LANE_OFF);
-  const uint4 h0 = __ldg(reinterpret_cast<const uint4*>(gprog));
-  const uint4 h1 = __ldg(reinterpret_cast<const uint4*>(gprog) + 1);
-  const uint4 h2 = __ldg(reinterpret_cast<const uint4*>(gprog) + 2);
-  const uint32_t n_gread = h0.y, n_layers = h0.z, n_out = h0.w;
-  const uint32_t n_ram = h1.x, off_gread = h1.z, off_layers = h1.w;
-  const uint32_t off_out = h2.x, off_ram = h2.y;
-  // layer 0's records first: independent of S, their latency overlaps the port loads
-  const uint32_t* L = gprog + off_layers;
-  LaneRegs R;
-  if (n_layers) load_lane_first(L, R);
-  if (pacc && tid == 0 && h0.x == 0u) pacc[7]++;   // (keeps the header read before the stamp)
-  phase(0);
-  // ---- a2: input ports (once per cycle) for the groups of the item.
-  // Entry k (one u32 gid per entry) goes to lane word k + 1.  A thread takes 4
-  // consecutive entries per uint4 and up to 16 per pass: all entry loads, then
-  // all value loads, then the stores (two L2 round trips per pass, not per entry)
-  const uint4* gr4 = reinterpret_cast<const uint4*>(gprog + off_gread);
+  const uint4* gr4 = reinterpret_cast<const uint4*>(gread);
   const uint32_t* bpi[K];
   const uint32_t* bq[K];
   const uint32_t* brd[K];
@@ -319,24 +293,22 @@ __device__ void run_lane_partition(const KParams& kp, uint32_t* S, uint32_t* ram
         }
     }
   }
-  if (tid < K) S[tid] = 0u;   // lane word 0 = constant 0 for every group
-  phase(1);
-  __syncthreads();
-  phase(2);
-  for (uint32_t l = 0; l < n_layers; l++) {
-    exec_lane_layer<K>(R, s_base, topv, 1);
-    const bool ptop = (R.flags & GEM_LF_USES_TOP) != 0;
-    const uint32_t ptopc = R.topc, ptopwo = R.topwo;
-    L += R.size;
-    if (l + 1 < n_layers) load_lane_next(L, R);
-    if (ptop && (threadIdx.x >> 5) == 0) top_lane_layer<K>(ptopc, ptopwo, s_base, topv, 1);
-    __syncthreads();
-  }
-  phase(3);
+}
+
+// ---- a6/a7 in lane mode: endpoint commit (one lane word per endpoint bit,
+// entries of 4 endpoints per thread loaded ahead, one LDS.K for all K groups)
+// and the RAM blocks (one warp per RAM, lane s = stream 32g+s; read-first,
+// per-bit write).
+template <int K>
+__device__ __forceinline__ void lane_commit(const KParams& kp, uint32_t s_base, uint32_t* ramp, const uint32_t* outs,
+                                            uint32_t n_out, const uint32_t* rr, uint32_t n_ram, uint32_t g0,
+                                            uint32_t ng, uint32_t c, uint32_t nxt) {
+  const uint32_t tid = threadIdx.x;
+  const LaneIdx X{kp.n_groups};
   // ---- a6: endpoint commit: one lane word per endpoint bit
   // entries of 4 endpoints per thread are loaded before use; one LDS.K gives
   // the source word of all K groups
-  const uint2* oe = reinterpret_cast<const uint2*>(gprog + off_out);
+  const uint2* oe = reinterpret_cast<const uint2*>(outs);
   for (uint32_t o0 = 0; o0 < n_out; o0 += 4 * GEM_THREADS) {
     uint2 e[4];
 #pragma unroll
@@ -365,7 +337,6 @@ __device__ void run_lane_partition(const KParams& kp, uint32_t* S, uint32_t* ram
   // ---- a7: RAM blocks: one warp per RAM, lane s = stream 32g+s (read-first, per-bit write)
   if (n_ram) {
     __syncthreads();
-    const uint32_t* rr = gprog + off_ram;
     const uint32_t lane = tid & 31;
     for (uint32_t jr = tid >> 5; jr < n_ram * ng; jr += GEM_WARPS) {
       const uint32_t j = jr / n_ram, r = jr - j * n_ram, g = g0 + j;
@@ -398,6 +369,163 @@ __device__ void run_lane_partition(const KParams& kp, uint32_t* S, uint32_t* ram
       }
     }
   }
+}
+
+// One work item: partition p for the 32-stream groups g0 .. g0+ng-1 (ng <= K;
+// groups ng..K-1 of the vectors are padding and never committed).
+template <int K>
+__device__ void run_lane_partition(const KParams& kp, uint32_t* S, uint32_t* ramp, uint32_t* topv, uint32_t p,
+                                   uint32_t g0, uint32_t ng, uint32_t c, uint32_t cur, uint32_t nxt,
+                                   unsigned long long* pacc) {
+  const uint32_t tid = threadIdx.x;
+  // GEM_F_PROFILE: thread 0 accumulates per-phase clocks over the CTA's items
+  unsigned long long t_ph = (pacc && tid == 0) ? clock64() : 0ull;
+  auto phase = [&](int k) {
+    if (pacc && tid == 0) {
+      const unsigned long long t = clock64();
+      pacc[k] += t - t_ph;
+      t_ph = t;
+    }
+  };
+  const uint32_t s_base = smem_u32(S);
+  const LaneIdx X{kp.n_groups};
+  const uint32_t* gprog = kp.lprog + __ldg(kp.parts + p * GP_WORDS + GP_LANE_OFF);
+  const uint4 h0 = __ldg(reinterpret_cast<const uint4*>(gprog));
+  const uint4 h1 = __ldg(reinterpret_cast<const uint4*>(gprog) + 1);
+  const uint4 h2 = __ldg(reinterpret_cast<const uint4*>(gprog) + 2);
+  const uint32_t n_gread = h0.y, n_layers = h0.z, n_out = h0.w;
+  const uint32_t n_ram = h1.x, off_gread = h1.z, off_layers = h1.w;
+  const uint32_t off_out = h2.x, off_ram = h2.y;
+  // layer 0's records first: independent of S, their latency overlaps the port loads
+  const uint32_t* L = gprog + off_layers;
+  LaneRegs R;
+  if (n_layers) load_lane_first(L, R);
+  if (pacc && tid == 0 && h0.x == 0u) pacc[7]++;   // (keeps the header read before the stamp)
+  phase(0);
+  // ---- a2: input ports (once per cycle) for the groups of the item.
+  // Entry k (one u32 gid per entry) goes to lane word k + 1.  A thread takes 4
+  // consecutive entries per uint4 and up to 16 per pass: all entry loads, then
+  // all value loads, then the stores (two L2 round trips per pass, not per entry)
+  lane_ports<K>(kp, s_base, gprog + off_gread, n_gread, g0, ng, c, cur);
+  if (tid < K) S[tid] = 0u;   // lane word 0 = constant 0 for every group
+  phase(1);
+  __syncthreads();
+  phase(2);
+  for (uint32_t l = 0; l < n_layers; l++) {
+    exec_lane_layer<K>(R, s_base, topv, 1);
+    const bool ptop = (R.flags & GEM_LF_USES_TOP) != 0;
+    const uint32_t ptopc = R.topc, ptopwo = R.topwo;
+    L += R.size;
+    if (l + 1 < n_layers) load_lane_next(L, R);
+    if (ptop && (threadIdx.x >> 5) == 0) top_lane_layer<K>(ptopc, ptopwo, s_base, topv, 1);
+    __syncthreads();
+  }
+  phase(3);
+  lane_commit<K>(kp, s_base, ramp, gprog + off_out, n_out, gprog + off_ram, n_ram, g0, ng, c, nxt);
+  __syncthreads();
+  phase(4);
+}
+
+// Input ports of a compacted lane program: entry k (one u32 gid, sorted by
+// global bit) -> lane word k + 1.  Thread t takes entries t, t+256, ... so a
+// warp's 32 consecutive entries -- mostly consecutive bits of one lane row --
+// load as one coalesced line per group, and their STS.K are conflict-free.
+template <int K>
+__device__ __forceinline__ void lane_ports2(const KParams& kp, uint32_t s_base, const uint32_t* gread,
+                                            uint32_t n_gread, uint32_t g0, uint32_t ng, uint32_t c, uint32_t cur) {
+  const uint32_t tid = threadIdx.x;
+  const LaneIdx X{kp.n_groups};
+  const uint32_t* bpi[K];
+  const uint32_t* bq[K];
+  const uint32_t* brd[K];
+  const uint32_t* bcut[K];
+#pragma unroll
+  for (int j = 0; j < K; j++) {
+    const uint32_t g = g0 + min((uint32_t)j, ng - 1u);
+    bpi[j] = kp.pi_lane + X.q(kp.in_base + c, kp.pi_words * 32, 0, g);
+    bq[j] = kp.q + X.q(cur, kp.q_words * 32, 0, g);
+    brd[j] = kp.rd + X.q(cur, kp.n_rams * 32, 0, g);
+    bcut[j] = kp.cut + X.q(0, kp.cut_words * 32, 0, g);
+  }
+  constexpr uint32_t U = K >= 4 ? 4u : 8u / K;   // entries per thread per pass (U * K loads in flight)
+  for (uint32_t kb = 0; kb < n_gread; kb += U * GEM_THREADS) {
+    uint32_t e[U];
+#pragma unroll
+    for (uint32_t u = 0; u < U; u++) {
+      const uint32_t k = kb + u * GEM_THREADS + tid;
+      e[u] = k < n_gread ? __ldg(gread + k) : 0xFFFFFFFFu;
+    }
+    uint32_t v[U][K];
+#pragma unroll
+    for (uint32_t u = 0; u < U; u++) {
+      const uint32_t reg = e[u] >> 24, b = e[u] & 0xFFFFFFu;
+#pragma unroll
+      for (int j = 0; j < K; j++) {
+        const uint32_t* base = reg == GEM_R_PI ? bpi[j] : reg == GEM_R_Q ? bq[j] : reg == GEM_R_RD ? brd[j] : bcut[j];
+        v[u][j] = e[u] != 0xFFFFFFFFu ? __ldcg(base + b) : 0u;
+      }
+    }
+#pragma unroll
+    for (uint32_t u = 0; u < U; u++)
+      if (e[u] != 0xFFFFFFFFu) stsK<K>(s_base + 4u * K * (kb + u * GEM_THREADS + tid + 1), v[u]);
+  }
+}
+
+// One work item of a compacted lane program ("LAN2", gem_isa.h): ports, then
+// the partition's ANDs in barrier-separated steps of <= 256 (thread t runs
+// op s*256+t of step s on all K groups: two LDS.K, 2K LOP3, one STS.K), then
+// endpoints and RAMs.  The op words stream from the L2-resident program into
+// registers kPre steps ahead of their use.
+template <int K>
+__device__ void run_lane_partition2(const KParams& kp, uint32_t* S, uint32_t* ramp, uint32_t p, uint32_t g0,
+                                    uint32_t ng, uint32_t c, uint32_t cur, uint32_t nxt, unsigned long long* pacc) {
+  const uint32_t tid = threadIdx.x;
+  unsigned long long t_ph = (pacc && tid == 0) ? clock64() : 0ull;
+  auto phase = [&](int k) {
+    if (pacc && tid == 0) {
+      const unsigned long long t = clock64();
+      pacc[k] += t - t_ph;
+      t_ph = t;
+    }
+  };
+  const uint32_t s_base = smem_u32(S);
+  const uint32_t* gprog = kp.lprog + __ldg(kp.parts + p * GP_WORDS + GP_LANE_OFF);
+  const uint4 h0 = __ldg(reinterpret_cast<const uint4*>(gprog));
+  const uint4 h1 = __ldg(reinterpret_cast<const uint4*>(gprog) + 1);
+  const uint4 h2 = __ldg(reinterpret_cast<const uint4*>(gprog) + 2);
+  const uint32_t n_gread = h0.y, n_steps = h0.z, n_out = h0.w;
+  const uint32_t n_ram = h1.x, off_gread = h1.z, off_ops = h1.w;
+  const uint32_t off_out = h2.x, off_ram = h2.y;
+  const uint2* ops = reinterpret_cast<const uint2*>(gprog + off_ops) + tid;
+  // the first steps' ops: independent of S, their latency overlaps the port loads
+  constexpr uint32_t kPre = 6;
+  uint2 q[kPre];
+#pragma unroll
+  for (uint32_t i = 0; i < kPre; i++) q[i] = i < n_steps ? __ldg(ops + i * GEM_LANE2_STEP) : make_uint2(0u, 0u);
+  phase(0);
+  lane_ports2<K>(kp, s_base, gprog + off_gread, n_gread, g0, ng, c, cur);
+  if (tid < K) S[tid] = 0u;   // lane word 0 = constant 0 for every group
+  phase(1);
+  __syncthreads();
+  phase(2);
+  for (uint32_t s = 0; s < n_steps; s++) {
+    const uint2 o = q[0];
+#pragma unroll
+    for (uint32_t i = 0; i + 1 < kPre; i++) q[i] = q[i + 1];
+    q[kPre - 1] = s + kPre < n_steps ? __ldg(ops + (s + kPre) * GEM_LANE2_STEP) : make_uint2(0u, 0u);
+    if (o.y) {
+      const uint32_t ia = (uint32_t)((int32_t)(o.x << 17) >> 31), ib = (uint32_t)((int32_t)(o.x << 1) >> 31);
+      uint32_t a[K], b[K], r[K];
+      ldsK<K>(s_base + 4u * K * (o.x & 0x3FFFu), a);
+      ldsK<K>(s_base + 4u * K * ((o.x >> 16) & 0x3FFFu), b);
+#pragma unroll
+      for (int j = 0; j < K; j++) r[j] = (a[j] ^ ia) & (b[j] ^ ib);
+      stsK<K>(s_base + 4u * K * o.y, r);
+    }
+    __syncthreads();
+  }
+  phase(3);
+  lane_commit<K>(kp, s_base, ramp, gprog + off_out, n_out, gprog + off_ram, n_ram, g0, ng, c, nxt);
   __syncthreads();
   phase(4);
 }
@@ -425,7 +553,7 @@ __device__ void record_state_lane(const KParams& kp, uint32_t c, uint32_t buf) {
   }
 }
 
-template <int K>
+template <int K, bool V2>
 __global__ void __launch_bounds__(GEM_THREADS, 2) gem_lane_kernel(const KParams kp) {
   extern __shared__ __align__(16) uint32_t smem[];
   // layout: S[lane_words][K] | ramp[K][ramp_words] | topv[16][K]  (no program ring:
@@ -461,8 +589,12 @@ __global__ void __launch_bounds__(GEM_THREADS, 2) gem_lane_kernel(const KParams 
         const uint4 U = __ldg(&kp.dyn_units[u]);
         for (uint32_t r = 0; r < U.z; r++) {
           const uint32_t g0 = (U.y >> 5) + r * K;
-          run_lane_partition<K>(kp, S, ramp, topv, U.x, g0, min((uint32_t)K, kp.n_groups - g0), c, cur, nxt,
-                                prof_on ? pacc : nullptr);
+          if (V2)
+            run_lane_partition2<K>(kp, S, ramp, U.x, g0, min((uint32_t)K, kp.n_groups - g0), c, cur, nxt,
+                                   prof_on ? pacc : nullptr);
+          else
+            run_lane_partition<K>(kp, S, ramp, topv, U.x, g0, min((uint32_t)K, kp.n_groups - g0), c, cur, nxt,
+                                  prof_on ? pacc : nullptr);
         }
         u = s_next[par];   // written before the item's first barrier
         par ^= 1u;
@@ -475,8 +607,12 @@ __global__ void __launch_bounds__(GEM_THREADS, 2) gem_lane_kernel(const KParams 
         for (uint32_t k = kb; k < ke; k++) {
           const uint2 it = __ldg(&kp.wl_items[k]);
           const uint32_t g0 = it.y >> 5;
-          run_lane_partition<K>(kp, S, ramp, topv, it.x, g0, min((uint32_t)K, kp.n_groups - g0), c, cur, nxt,
-                                prof_on ? pacc : nullptr);
+          if (V2)
+            run_lane_partition2<K>(kp, S, ramp, it.x, g0, min((uint32_t)K, kp.n_groups - g0), c, cur, nxt,
+                                   prof_on ? pacc : nullptr);
+          else
+            run_lane_partition<K>(kp, S, ramp, topv, it.x, g0, min((uint32_t)K, kp.n_groups - g0), c, cur, nxt,
+                                  prof_on ? pacc : nullptr);
         }
         if (s == 0) PROF(4);
         grid_sync(kp, bar_target);

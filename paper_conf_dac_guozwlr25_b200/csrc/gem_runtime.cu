@@ -1044,6 +1044,7 @@ struct gem_sim {
   uint32_t n_units = 0, *d_dyn_ctr = nullptr;
   unsigned long long* d_act = nullptr;         // {evaluated, skipped}
   uint32_t lanes = 0, n_groups = 0, lane_words = 0, lane_max_chunk = 0, ramp_words = 0, lane_groups = 1;
+  bool lane_v2 = false;                        // compacted lane programs ("LAN2")
   uint32_t *d_lprog = nullptr, *d_pi_lane = nullptr, *d_po_lane = nullptr;
   std::vector<uint32_t> h_parts, h_stage;
   // device buffers
@@ -1291,8 +1292,12 @@ static int plan_launch(gem_sim* sim, uint32_t max_chunk_words, uint32_t grid_lim
   return GEM_OK;
 }
 
-static const void* lane_kernel_for(uint32_t k) {
-  return k >= 4 ? (const void*)gem_lane_kernel<4> : k == 2 ? (const void*)gem_lane_kernel<2> : (const void*)gem_lane_kernel<1>;
+static const void* lane_kernel_for(uint32_t k, bool v2) {
+  if (v2)
+    return k >= 4 ? (const void*)gem_lane_kernel<4, true> : k == 2 ? (const void*)gem_lane_kernel<2, true>
+                                                                     : (const void*)gem_lane_kernel<1, true>;
+  return k >= 4 ? (const void*)gem_lane_kernel<4, false> : k == 2 ? (const void*)gem_lane_kernel<2, false>
+                                                                    : (const void*)gem_lane_kernel<1, false>;
 }
 
 // Lane mode launch: one CTA per SM (all shared memory for the lane state and
@@ -1331,7 +1336,7 @@ static int plan_launch_lanes(gem_sim* sim, uint32_t grid_limit) {
   if (grid_limit) grid = std::max<uint32_t>(1, std::min(grid, grid_limit));
   grid = std::min<uint32_t>(grid, GEM_BAR_MAX_CTAS);
   const uint32_t smem = fixed_words * 4;
-  const void* lk = lane_kernel_for(gl);
+  const void* lk = lane_kernel_for(gl, sim->lane_v2);
   CK(cudaFuncSetAttribute(lk, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem));
   int occ = 0;
   CK(cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ, lk, GEM_THREADS, smem));
@@ -1504,6 +1509,12 @@ static int load_impl(gem_sim* sim, const uint32_t* w, size_t nw, const gem_confi
     sim->lane_words = (std::max<uint32_t>(w[GH_LANE_MAX_WORDS], 4) + 3) & ~3u;
     sim->lane_max_chunk = w[GH_LANE_MAX_CHUNK_WORDS];
     sim->ramp_words = std::max<uint32_t>(w[GH_MAX_RAMS_PART], 1) * 128;
+    const uint32_t* lp = w + w[GH_OFF_LANE_PROG];
+    sim->lane_v2 = sim->n_parts && lp[parts[GP_LANE_OFF] + LPH_MAGIC] == GEM_LANE2_MAGIC;
+    for (uint32_t p = 0; p < sim->n_parts; p++) {
+      const uint32_t m = lp[parts[(size_t)p * GP_WORDS + GP_LANE_OFF] + LPH_MAGIC];
+      if (m != (sim->lane_v2 ? GEM_LANE2_MAGIC : GEM_LANE_MAGIC)) return fail(GEM_E_FORMAT, "mixed or bad lane programs");
+    }
   }
   // uploads
   const size_t S = sim->n_streams;
@@ -1718,7 +1729,7 @@ int gem_step(gem_sim* sim, uint64_t ncycles) {
   }
   void* args[] = {&kp};
   CK(cudaEventRecord(sim->ev0, sim->stream));
-  CK(cudaLaunchCooperativeKernel(sim->lanes ? lane_kernel_for(sim->lane_groups) : step_kernel_for(sim),
+  CK(cudaLaunchCooperativeKernel(sim->lanes ? lane_kernel_for(sim->lane_groups, sim->lane_v2) : step_kernel_for(sim),
                                  dim3(sim->grid), dim3(GEM_THREADS), args, sim->smem_bytes, sim->stream));
   CK(cudaEventRecord(sim->ev1, sim->stream));
   sim->in_head += (uint32_t)ncycles;

@@ -36,6 +36,7 @@
 #include <functional>
 #include <map>
 #include <memory>
+#include <set>
 #include <mutex>
 #include <numeric>
 #include <sstream>
@@ -73,6 +74,10 @@ struct Options {
   int max_warps = 8;        // warps that may hold placed roots (8 = all)
   int lane_banks = 1;       // bank-aware placement of lane write-out runs (2: also interior offsets)
   int lane_holes = 32;      // best-fitting holes considered per run
+  int lane_k = 4;           // lane mode 2: bank-conflict model for K interleaved groups (K lanes' words
+                            // per 16 bytes: lanes of 32/K share one wavefront)
+  int lane_mode = 2;        // 1: lane program from the boomerang placement ("LANE"); 2: compacted AND
+                            // list in barrier-separated steps ("LAN2", gem_isa.h)
   int banks = 1;            // bank-conflict-aware renaming of the state words (rename_state_words)
   int verbose = 0;
   int max_state_words = GEM_MAX_STATE_WORDS;
@@ -114,6 +119,8 @@ static Options parse_opts(const char* s) {
     else if (k == "lane_banks") o.lane_banks = std::stoi(v);
     else if (k == "max_warps") o.max_warps = std::max(1, std::min(8, std::stoi(v)));
     else if (k == "lane_holes") o.lane_holes = std::max(1, std::stoi(v));
+    else if (k == "lane_mode") o.lane_mode = std::max(1, std::min(2, std::stoi(v)));
+    else if (k == "lane_k") o.lane_k = std::stoi(v) >= 4 ? 4 : std::stoi(v) >= 2 ? 2 : 1;
     else if (k == "banks") o.banks = std::stoi(v);
     else if (k == "synth") o.synth = std::stoi(v);
     else if (k == "chain_min") o.chain_min = std::max(2, std::stoi(v));
@@ -935,7 +942,8 @@ struct Mapper {
     P.n_leaves = total_leaves;
     P.n_writeouts = total_wo;
     P.slots_used = slots_used;
-    if (opt.lanes && !encode_lanes(P, lane_layers, gread_src, scratch)) return;
+    if (opt.lanes && opt.lane_mode == 1 && !encode_lanes(P, lane_layers, gread_src, scratch)) return;
+    if (opt.lanes && opt.lane_mode == 2 && !encode_lanes2(P, scratch)) return;
     P.ok = true;
   }
 
@@ -1462,6 +1470,186 @@ struct Mapper {
     pr[LPH_N_GREAD] = ng;
     while (pr.size() % 4) pr.push_back(0);
     P.lane_words = pr[LPH_LANE_WORDS];
+    return true;
+  }
+
+  // Compacted lane program ("LAN2", gem_isa.h): the partition's ANDs list-
+  // scheduled into steps of <= 256 (critical path first), lane words
+  // allocated by liveness, ops of a step assigned to threads and destination
+  // words chosen so that each half-warp's 16 operand / destination residues
+  // (mod 16) collide as little as possible.
+  bool encode_lanes2(Part& P, const std::vector<int32_t>& scratch) {
+    const uint32_t n = (uint32_t)cid.size();
+    const uint32_t kMaxWords = (uint32_t)opt.lane_words;
+    // one LDS/STS of K interleaved groups moves 4K bytes per lane: a wavefront
+    // (128 bytes) serves kHalf = 32/K lanes, conflict-free when their words
+    // differ mod kHalf
+    const uint32_t kStep = GEM_LANE2_STEP, kHalf = 32u / (uint32_t)opt.lane_k, kGroups = kStep / kHalf;
+    // sources: port-list order (sorted by global bit: a warp's port loads stay coalesced)
+    std::vector<uint32_t> srcs;
+    for (uint32_t i = 1; i < n; i++)
+      if (is_src[i]) srcs.push_back(i);
+    std::stable_sort(srcs.begin(), srcs.end(), [&](uint32_t x, uint32_t y) {
+      const uint32_t gx = G.gbit[cid[x]], gy = G.gbit[cid[y]];
+      const uint64_t kx = ((uint64_t)(gx >> 27) << 32) | (((gx >> 5) & 0x3FFFFF) * 32 + (gx & 31));
+      const uint64_t ky = ((uint64_t)(gy >> 27) << 32) | (((gy >> 5) & 0x3FFFFF) * 32 + (gy & 31));
+      return kx < ky;
+    });
+    if (srcs.size() + 1 >= kMaxWords) { fail(P, "lane state overflow"); return false; }
+    // ---- list scheduling: an op is ready one step after its last operand
+    std::vector<uint32_t> rd(n, 0), pend(n, 0), step_of(n, 0);
+    for (uint32_t i = n; i-- > 0;)
+      for (uint32_t j = coff[i]; j < coff[i + 1]; j++) rd[i] = std::max(rd[i], rd[cons[j]] + 1);
+    std::vector<uint32_t> ready;   // max-heap on (rd, -id)
+    auto prio = [&](uint32_t x, uint32_t y) { return rd[x] != rd[y] ? rd[x] < rd[y] : x > y; };
+    uint32_t n_ops = 0;
+    for (uint32_t i = 0; i < n; i++) {
+      if (is_src[i]) continue;
+      n_ops++;
+      pend[i] = (uint32_t)(!is_src[la[i] >> 1]) + (uint32_t)(!is_src[lb[i] >> 1]);
+      if ((la[i] >> 1) == (lb[i] >> 1) && !is_src[la[i] >> 1]) pend[i] = 1;
+      if (!pend[i]) ready.push_back(i);
+    }
+    std::make_heap(ready.begin(), ready.end(), prio);
+    std::vector<std::vector<uint32_t>> steps;
+    std::vector<uint32_t> next_ready;
+    uint32_t done = 0;
+    while (done < n_ops) {
+      if (ready.empty()) throw std::runtime_error("lane2: scheduling stalled");
+      steps.emplace_back();
+      auto& st = steps.back();
+      while (!ready.empty() && st.size() < kStep) {
+        std::pop_heap(ready.begin(), ready.end(), prio);
+        st.push_back(ready.back());
+        ready.pop_back();
+      }
+      next_ready.clear();
+      for (uint32_t x : st) {
+        step_of[x] = (uint32_t)steps.size() - 1;
+        done++;
+        for (uint32_t j = coff[x]; j < coff[x + 1]; j++) {
+          const uint32_t c = cons[j];
+          if (j > coff[x] && cons[j - 1] == c) continue;   // both fanins from x: counted once
+          if (--pend[c] == 0) next_ready.push_back(c);
+        }
+      }
+      for (uint32_t c : next_ready) { ready.push_back(c); std::push_heap(ready.begin(), ready.end(), prio); }
+    }
+    const uint32_t S = (uint32_t)steps.size();
+    // ---- last reading step of every value (endpoints: live to the end)
+    const uint32_t INF = UINT32_MAX;
+    std::vector<uint32_t> last(n, 0);
+    for (uint32_t i = 0; i < n; i++) {
+      if (is_ep[i]) { last[i] = INF; continue; }
+      for (uint32_t j = coff[i]; j < coff[i + 1]; j++) last[i] = std::max(last[i], step_of[cons[j]]);
+    }
+    // ---- words: 0 = constant, 1..n_src = ports; free pool per residue mod 16
+    std::vector<int32_t> word(n, -1);
+    word[0] = 0;
+    std::vector<std::set<uint32_t>> freew(kHalf);
+    uint32_t top = 1, max_word = 1;
+    for (uint32_t x : srcs) { word[x] = (int32_t)top++; }
+    max_word = top;
+    std::vector<std::vector<uint32_t>> die(S + 1);
+    for (uint32_t x : srcs)
+      if (last[x] != INF) die[last[x]].push_back((uint32_t)word[x]);
+    auto alloc = [&](uint32_t res) -> uint32_t {   // lowest free word of residue res (or a fresh one)
+      uint32_t best = UINT32_MAX;
+      if (!freew[res].empty()) best = *freew[res].begin();
+      // a fresh word of this residue at the top (may also open lower residues)
+      uint32_t fresh = top + ((res + kHalf - (top % kHalf)) % kHalf);
+      if (best != UINT32_MAX && best < fresh) { freew[res].erase(freew[res].begin()); return best; }
+      for (uint32_t w = top; w < fresh; w++) freew[w % kHalf].insert(w);
+      top = fresh + 1;
+      return fresh;
+    };
+    auto lw = [&](uint32_t l) -> uint32_t {
+      const int32_t w = word[l >> 1];
+      if (w < 0) throw std::runtime_error("lane2: operand without a word");
+      return (uint32_t)w;
+    };
+    std::vector<uint32_t>& pr = P.lane_prog;
+    pr.assign(LPH_WORDS, 0);
+    pr[LPH_MAGIC] = GEM_LANE2_MAGIC;
+    pr[LPH_N_LAYERS] = S;
+    pr[LPH_N_OUT] = (uint32_t)P.outs.size() * 32;
+    pr[LPH_N_RAM] = (uint32_t)P.rams.size();
+    pr[LPH_OFF_CHUNKS] = (uint32_t)pr.size();
+    pr[LPH_N_CHUNKS] = 1;
+    pr.push_back(0);
+    while (pr.size() % 4) pr.push_back(0);
+    pr[LPH_OFF_LAYERS] = (uint32_t)pr.size();
+    pr.resize(pr.size() + (size_t)S * kStep * 2, 0);
+    uint32_t* ops = pr.data() + pr[LPH_OFF_LAYERS];
+    std::vector<std::array<uint8_t, 32>> ca(kGroups), cb(kGroups), cd(kGroups);
+    std::vector<uint32_t> fill(kGroups);
+    for (uint32_t s = 0; s < S; s++) {
+      // words last read before step s are free (the barrier separates the read and the write)
+      if (s > 0)
+        for (uint32_t w : die[s - 1]) freew[w % kHalf].insert(w);
+      for (uint32_t g = 0; g < kGroups; g++) { ca[g].fill(0); cb[g].fill(0); cd[g].fill(0); fill[g] = 0; }
+      auto& st = steps[s];
+      // busiest operands first
+      std::stable_sort(st.begin(), st.end(), [&](uint32_t x, uint32_t y) { return rd[x] > rd[y]; });
+      for (uint32_t x : st) {
+        const uint32_t ra = lw(la[x]) % kHalf, rb = lw(lb[x]) % kHalf;
+        // half-warp group with room and the fewest operand-residue collisions
+        uint32_t bg = 0, bc = UINT32_MAX;
+        for (uint32_t g = 0; g < kGroups; g++) {
+          if (fill[g] == kHalf) continue;
+          const uint32_t c = 4u * (ca[g][ra] + cb[g][rb]) + fill[g] / 8;
+          if (c < bc) { bc = c; bg = g; }
+        }
+        // destination residue: least used in the group, then lowest word
+        uint32_t bres = 0, bcost = UINT32_MAX;
+        for (uint32_t r = 0; r < kHalf; r++) {
+          const uint32_t c = cd[bg][r];
+          if (c < bcost) { bcost = c; bres = r; }
+        }
+        uint32_t w = UINT32_MAX;
+        {
+          // among the least-used residues prefer one with a free word (compact state)
+          uint32_t bw = UINT32_MAX;
+          for (uint32_t r = 0; r < kHalf; r++)
+            if (cd[bg][r] == bcost && !freew[r].empty() && *freew[r].begin() < bw) { bw = *freew[r].begin(); bres = r; }
+          w = alloc(bres);
+        }
+        ca[bg][ra]++; cb[bg][rb]++; cd[bg][w % kHalf]++;
+        const uint32_t t = bg * kHalf + fill[bg]++;
+        word[x] = (int32_t)w;
+        max_word = std::max(max_word, w + 1);
+        if (last[x] != INF) die[std::max(last[x], s)].push_back(w);
+        ops[((size_t)s * kStep + t) * 2] = GEM_LANE2_OP_X(lw(la[x]), la[x] & 1u, lw(lb[x]), lb[x] & 1u);
+        ops[((size_t)s * kStep + t) * 2 + 1] = w;
+      }
+      if (max_word >= kMaxWords) { fail(P, "lane state overflow"); return false; }
+    }
+    pr[LPH_LANE_WORDS] = (max_word + 3) & ~3u;
+    pr[LPH_OFF_OUT] = (uint32_t)pr.size();
+    for (auto& ow : P.outs) {
+      const uint32_t reg = GEM_GID_REGION(ow.dst), idx = GEM_GID_INDEX(ow.dst);
+      for (int k = 0; k < 32; k++) {
+        const uint32_t l = ow.lit[k];
+        const uint32_t x = (uint32_t)scratch[l >> 1];
+        pr.push_back((reg << 24) | (idx * 32 + (uint32_t)k));
+        pr.push_back(lw(2 * x) | ((l & 1) ? GEM_OUT_INV : 0u));
+      }
+    }
+    pr[LPH_OFF_RAM] = (uint32_t)pr.size();
+    for (uint32_t r : P.rams) { pr.push_back(r); pr.push_back(0); pr.push_back(0); pr.push_back(0); }
+    while (pr.size() % 4) pr.push_back(0);
+    pr[LPH_OFF_GREAD] = (uint32_t)pr.size();
+    for (uint32_t x : srcs) {
+      const uint32_t gb = G.gbit[cid[x]];
+      pr.push_back(((gb >> 27) << 24) | (((gb >> 5) & 0x3FFFFF) * 32 + (gb & 31)));
+    }
+    pr[LPH_N_GREAD] = (uint32_t)srcs.size();
+    while (pr.size() % 4) pr.push_back(0);
+    pr[pr[LPH_OFF_CHUNKS]] = (uint32_t)pr.size();
+    P.lane_words = pr[LPH_LANE_WORDS];
+    if (opt.verbose >= 3)
+      fprintf(stderr, "lane2 part: ops=%u steps=%u (fill %.2f) srcs=%zu words=%u\n", n_ops, S,
+              n_ops / (double)(S * kStep), srcs.size(), max_word);
     return true;
   }
 

@@ -17,6 +17,7 @@ ap.add_argument("--cycles", type=int, default=1000)
 ap.add_argument("--steps", type=int, default=10)
 ap.add_argument("--streams", type=int, default=1)
 ap.add_argument("--map-opts", default=None)
+ap.add_argument("--tune", default="", help="gem_config tuning, e.g. lane_groups=2,lane_ctas_per_sm=2")
 a = ap.parse_args()
 from paper_conf_dac_guozwlr25_b200 import _build  # noqa: E402
 _build.LIBGEM = os.path.abspath(a.lib)
@@ -27,7 +28,8 @@ from paper_conf_dac_guozwlr25_b200 import gem  # noqa: E402
 from tests.common import blob  # noqa: E402
 
 b = blob(a.cfg, a.map_opts)
-sim = gem.Simulator(b, n_streams=a.streams)
+tune = {k: (float(v) if k == "l2_evict_last" else int(v)) for k, v in (x.split("=") for x in a.tune.split(",") if x)}
+sim = gem.Simulator(b, n_streams=a.streams, **tune)
 n_pi = sim.info["n_pi"]
 st = stimulus_streams("c5" if a.cfg == "c5" else a.cfg, n_pi, a.cycles, range(a.streams))
 flush = torch.empty(512 * 1024 * 1024 // 4, dtype=torch.int32, device="cuda")
@@ -42,4 +44,4 @@ for k in range(a.steps + 2):
 med = float(np.median(ms))
 print(f"{os.path.basename(a.lib)} {a.cfg} {a.map_opts or ''}: median {med:.3f} ms / {a.cycles} cycles = "
       f"{a.cycles * a.streams / med * 1e3:.0f} stream-cycles/s (min {min(ms):.3f}, max {max(ms):.3f}) "
-      f"grid {sim.info['grid']} layers {sim.info['max_layers']}", flush=True)
+      f"grid {sim.info['grid']} layers {sim.info['max_layers']} group {sim.info['group']} {a.tune}", flush=True)

@@ -191,7 +191,8 @@ int run_lane_part(Interp& I, LaneSim& Ls, uint32_t p, const uint32_t* pi_lane /*
   const uint32_t* pt = I.parts + p * GP_WORDS;
   const uint32_t* lane_base = I.w.data() + I.w[GH_OFF_LANE_PROG];
   const uint32_t* pr = lane_base + pt[GP_LANE_OFF];
-  if (pr[LPH_MAGIC] != GEM_LANE_MAGIC) { g_err = "bad lane magic"; return -1; }
+  const bool v2 = pr[LPH_MAGIC] == GEM_LANE2_MAGIC;
+  if (pr[LPH_MAGIC] != GEM_LANE_MAGIC && !v2) { g_err = "bad lane magic"; return -1; }
   uint32_t cur = (uint32_t)(I.cycle & 1), nxt = cur ^ 1;
   std::vector<uint32_t> S(pr[LPH_LANE_WORDS] + 1, 0);
   const uint32_t* gr = pr + pr[LPH_OFF_GREAD];
@@ -207,8 +208,41 @@ int run_lane_part(Interp& I, LaneSim& Ls, uint32_t p, const uint32_t* pi_lane /*
     S[dst] = v;
   }
   const uint32_t* L = pr + pr[LPH_OFF_LAYERS];
+  if (v2) {
+    // compacted program (gem_isa.h "LAN2"): every op of a step reads the state
+    // as it was before the step; a step's destinations are written after all
+    // of its reads (and must not be read within the step)
+    std::vector<std::pair<uint32_t, uint32_t>> wr;
+    std::vector<uint8_t> written(S.size(), 0);
+    for (uint32_t st = 0; st < pr[LPH_N_LAYERS]; st++) {
+      wr.clear();
+      const uint32_t* ops = L + (size_t)st * GEM_LANE2_STEP * 2;
+      for (uint32_t t = 0; t < GEM_LANE2_STEP; t++) {
+        const uint32_t x = ops[2 * t], y = ops[2 * t + 1];
+        if (!y) continue;
+        const uint32_t a = x & 0x3FFFu, b = (x >> 16) & 0x3FFFu;
+        if (a >= S.size() || b >= S.size() || y >= S.size()) { g_err = "lane2 op word out of range"; return -1; }
+        const uint32_t va = S[a] ^ (((x >> 14) & 1u) ? ~0u : 0u), vb = S[b] ^ (((x >> 30) & 1u) ? ~0u : 0u);
+        wr.push_back({y, va & vb});
+      }
+      for (auto& e : wr) {
+        if (written[e.first] == 1 + (st & 1) ) { g_err = "lane2 destination written twice in a step"; return -1; }
+        written[e.first] = (uint8_t)(1 + (st & 1));
+      }
+      for (uint32_t t = 0; t < GEM_LANE2_STEP; t++) {
+        const uint32_t x = ops[2 * t];
+        if (!ops[2 * t + 1]) continue;
+        if (written[x & 0x3FFFu] == 1 + (st & 1) || written[(x >> 16) & 0x3FFFu] == 1 + (st & 1)) {
+          g_err = "lane2 op reads a word written in the same step";
+          return -1;
+        }
+      }
+      for (auto& e : wr) S[e.first] = e.second;
+      for (auto& e : wr) written[e.first] = 0;
+    }
+  }
   std::vector<uint32_t> val[14];
-  for (uint32_t l = 0; l < pr[LPH_N_LAYERS]; l++) {
+  for (uint32_t l = 0; !v2 && l < pr[LPH_N_LAYERS]; l++) {
     for (int k = 0; k <= 13; k++) val[k].assign(8192u >> k, 0);
     uint32_t flags = L[LLH_FLAGS], topc = L[LLH_TOPC];
     uint32_t lane_c[256][3];

@@ -164,7 +164,8 @@ def test_lane_layer_headers_carry_next_layer():
     record loads from them without reading its header first."""
     LPH_N_LAYERS, LPH_OFF_LAYERS = 2, 7
     n_checked = 0
-    for _, pr in _lane_programs(blob("c5")):
+    from tests.common import MAP_OPTS
+    for _, pr in _lane_programs(blob("c5", MAP_OPTS["c5"] + " lane_mode=1")):
         L = int(pr[LPH_OFF_LAYERS])
         for l in range(int(pr[LPH_N_LAYERS])):
             nxt = L + int(pr[L])
