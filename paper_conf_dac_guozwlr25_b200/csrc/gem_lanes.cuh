@@ -554,7 +554,7 @@ __device__ void record_state_lane(const KParams& kp, uint32_t c, uint32_t buf) {
 }
 
 template <int K, bool V2>
-__global__ void __launch_bounds__(GEM_THREADS, 2) gem_lane_kernel(const KParams kp) {
+__global__ void __launch_bounds__(GEM_THREADS, (V2 && K <= 2) ? 4 : 2) gem_lane_kernel(const KParams kp) {
   extern __shared__ __align__(16) uint32_t smem[];
   // layout: S[lane_words][K] | ramp[K][ramp_words] | topv[16][K]  (no program ring:
   // records are loaded from global memory into registers one layer ahead)

@@ -1316,11 +1316,14 @@ static int plan_launch_lanes(gem_sim* sim, uint32_t grid_limit) {
   // groups per work item as fit (shared memory holds only the lane state:
   // records stream from global memory into registers)
   uint32_t bps = 0, gl = 0;
-  for (uint32_t b = 2; b >= 1 && !bps; b--) {
+  // (compacted programs: the K <= 2 kernels are built for up to 4 CTAs per SM)
+  const uint32_t max_bps = sim->lane_v2 ? 4u : 2u;
+  for (uint32_t b = force_bps ? std::min(force_bps, max_bps) : 2u; b >= 1 && !bps; b--) {
     if (force_bps && force_bps != b) continue;
     const uint32_t bud = (uint32_t)std::min<int64_t>(optin, per_sm / (int64_t)b - 1024);
     for (uint32_t k = std::max<uint32_t>(1, std::min(want_gl, sim->n_groups)); k >= 1; k--) {
       if (k == 3) continue;   // the kernel is instantiated for K = 1, 2, 4 interleaved groups
+      if (b > 2 && k > 2) continue;   // K = 4 kernels are built for <= 2 CTAs per SM
       const uint64_t words = (uint64_t)k * (sim->lane_words + sim->ramp_words + 16);
       if (words * 4 <= bud) { bps = b; gl = k; break; }
     }

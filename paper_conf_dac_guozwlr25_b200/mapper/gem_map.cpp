@@ -62,6 +62,9 @@ struct Options {
   int stages = 1;           // 1 or 2 (multi-stage RepCut)
   int cut_level = 0;        // 0 = auto (middle)
   int merge = 1;            // Algorithm 1 merge pass
+  int km1 = 8;              // passes of k-way min-cut refinement of the RepCut hypergraph (0 = off)
+  int km1_pins = 64;        // hyperedges (shared AND nodes) with more users are left out of the gains
+  double km1_slack = 1.1;   // refinement keeps every partition under this x the packing cap
   int key = 0;              // unit order for packing: 0 = min flop index in the cone, 1 = deep-cone
                             // min-hash, 2 = a register's own index (declaration order = module order)
   double merge_cap = 0;     // max merged cone size in ANDs (0 = 2.5 x part_size)
@@ -105,6 +108,9 @@ static Options parse_opts(const char* s) {
     else if (k == "stages") o.stages = std::stoi(v);
     else if (k == "cut_level") o.cut_level = std::stoi(v);
     else if (k == "merge") o.merge = std::stoi(v);
+    else if (k == "km1") o.km1 = std::stoi(v);
+    else if (k == "km1_pins") o.km1_pins = std::max(2, std::stoi(v));
+    else if (k == "km1_slack") o.km1_slack = std::stod(v);
     else if (k == "key") o.key = std::stoi(v);
     else if (k == "merge_cap") o.merge_cap = std::stod(v);
     else if (k == "merge_ratio") o.merge_ratio = std::stod(v);
@@ -1967,6 +1973,162 @@ static void partition(Design& D) {
                 groups.size(), target);
       if (ratio > 0.85 && ratio < 1.2) break;
       cap *= std::max(0.5, std::min(2.0, ratio));
+    }
+    // ---- min-cut refinement (the partitioner of P:105/P:117, RepCut [17]):
+    // the RepCut hypergraph has one vertex per unit (endpoint) and one
+    // hyperedge per AND node, spanning the units whose cone contains it; a
+    // node is replicated in every partition that holds one of its units, so
+    // the replication cost is the connectivity-minus-one (km1) metric
+    // sum_x (lambda(x) - 1).  k-way FM-style passes move single units to the
+    // partition that lowers km1 most (gain = the unit's shared nodes that leave
+    // its partition minus those new to the target), keeping every partition's
+    // cone under km1_slack x the packing cap.  Nodes with one user move with
+    // their unit; nodes with more than km1_pins users (shallow, wide logic that
+    // every partition needs anyway) are left out of the gains.
+    if (opt.km1 > 0 && groups.size() > 1) {
+      const uint32_t nu = (uint32_t)su.size();
+      std::vector<uint32_t> uoff(nu + 1, 0), unodes;
+      for (uint32_t i = 0; i < nu; i++) {
+        cur_stamp++;
+        unit_lits(su[i], lits);
+        for (uint32_t l : lits) {
+          uint32_t x = l >> 1;
+          if (stamp[x] == cur_stamp) continue;
+          stamp[x] = cur_stamp;
+          st.push_back(x);
+          while (!st.empty()) {
+            uint32_t y = st.back(); st.pop_back();
+            if (is_leaf_for(y, stage)) continue;
+            unodes.push_back(y);
+            for (uint32_t z : {G.a[y] >> 1, G.b[y] >> 1})
+              if (stamp[z] != cur_stamp) { stamp[z] = cur_stamp; st.push_back(z); }
+          }
+        }
+        uoff[i + 1] = (uint32_t)unodes.size();
+      }
+      std::vector<uint32_t> users(N, 0);
+      for (uint32_t x : unodes) users[x]++;
+      // per shared node: (partition, count) slots, at most `users` of them
+      std::vector<uint32_t> noff(N + 1, 0);
+      for (size_t x = 0; x < N; x++) noff[x + 1] = noff[x] + ((users[x] >= 2 && users[x] <= (uint32_t)opt.km1_pins) ? users[x] : 0);
+      std::vector<uint32_t> npart(noff[N], UINT32_MAX), ncnt(noff[N], 0);
+      std::vector<uint8_t> nlen(N, 0);
+      std::vector<uint32_t> part_of(nu, 0);
+      const uint32_t ng = (uint32_t)groups.size();
+      for (uint32_t g = 0; g < ng; g++) for (uint32_t i : groups[g]) part_of[i] = g;
+      auto slot = [&](uint32_t x, uint32_t P) -> int64_t {
+        for (uint32_t k = 0; k < nlen[x]; k++) if (npart[noff[x] + k] == P) return noff[x] + k;
+        return -1;
+      };
+      auto add = [&](uint32_t x, uint32_t P) {
+        int64_t k = slot(x, P);
+        if (k < 0) { k = noff[x] + nlen[x]++; npart[k] = P; ncnt[k] = 0; }
+        ncnt[k]++;
+      };
+      auto remove = [&](uint32_t x, uint32_t P) {
+        const int64_t k = slot(x, P);
+        if (--ncnt[k] == 0) {
+          const uint32_t last = noff[x] + --nlen[x];
+          npart[k] = npart[last]; ncnt[k] = ncnt[last];
+        }
+      };
+      auto shared = [&](uint32_t x) { return users[x] >= 2 && users[x] <= (uint32_t)opt.km1_pins; };
+      // partition sizes: exact cones (private + shared + wide nodes)
+      std::vector<uint64_t> psize(ng, 0);
+      {
+        std::vector<uint32_t> mark(N, UINT32_MAX);
+        for (uint32_t g = 0; g < ng; g++)
+          for (uint32_t i : groups[g])
+            for (uint32_t k = uoff[i]; k < uoff[i + 1]; k++) {
+              const uint32_t x = unodes[k];
+              if (mark[x] != g) { mark[x] = g; psize[g]++; }
+            }
+      }
+      for (uint32_t i = 0; i < nu; i++)
+        for (uint32_t k = uoff[i]; k < uoff[i + 1]; k++)
+          if (shared(unodes[k])) add(unodes[k], part_of[i]);
+      // from here on a unit needs only its shared nodes and its private count
+      std::vector<uint32_t> upriv(nu, 0);
+      {
+        std::vector<uint32_t> off2(nu + 1, 0), sh;
+        for (uint32_t i = 0; i < nu; i++) {
+          for (uint32_t k = uoff[i]; k < uoff[i + 1]; k++) {
+            const uint32_t x = unodes[k];
+            if (users[x] == 1) upriv[i]++;
+            else if (shared(x)) sh.push_back(x);
+          }
+          off2[i + 1] = (uint32_t)sh.size();
+        }
+        uoff.swap(off2);
+        unodes.swap(sh);
+      }
+      auto km1_cost = [&]() {
+        uint64_t c = 0;
+        for (size_t x = 0; x < N; x++) if (nlen[x]) c += nlen[x] - 1;
+        return c;
+      };
+      const uint64_t before = km1_cost();
+      uint64_t rep_before = 0;
+      for (uint32_t g = 0; g < ng; g++) rep_before += psize[g];
+      const double pcap = cap * opt.km1_slack;
+      std::vector<uint32_t> have(ng, 0), touched;
+      std::vector<uint32_t> order(nu);
+      std::iota(order.begin(), order.end(), 0);
+      uint64_t moves_total = 0;
+      for (int pass = 0; pass < opt.km1; pass++) {
+        uint64_t moves = 0;
+        // deterministic shuffle per pass
+        for (uint32_t i = nu; i > 1; i--) std::swap(order[i - 1], order[mix64(pass * 1000003ull + i) % i]);
+        for (uint32_t i : order) {
+          const uint32_t A = part_of[i];
+          if (groups[A].size() <= 1) continue;
+          uint32_t n_sh = 0, loss = 0;
+          const uint32_t priv = upriv[i];
+          touched.clear();
+          for (uint32_t k = uoff[i]; k < uoff[i + 1]; k++) {
+            const uint32_t x = unodes[k];
+            n_sh++;
+            for (uint32_t q = 0; q < nlen[x]; q++) {
+              const uint32_t P = npart[noff[x] + q];
+              if (P == A) { if (ncnt[noff[x] + q] == 1) loss++; continue; }
+              if (!have[P]++) touched.push_back(P);
+            }
+          }
+          int64_t best_gain = 0;
+          uint32_t best = UINT32_MAX;
+          for (uint32_t P : touched) {
+            const int64_t gain = (int64_t)loss - (int64_t)(n_sh - have[P]);
+            const double new_size = (double)psize[P] + priv + (n_sh - have[P]);
+            if (new_size > pcap) continue;
+            if (gain > best_gain || (gain == best_gain && gain > 0 && P < best)) { best_gain = gain; best = P; }
+          }
+          for (uint32_t P : touched) have[P] = 0;
+          if (best == UINT32_MAX) continue;
+          // commit the move A -> best (sizes: wide nodes are assumed present in both)
+          psize[A] -= priv + loss;
+          psize[best] += priv + (uint64_t)((int64_t)loss - best_gain);   // = shared nodes new to `best`
+          for (uint32_t k = uoff[i]; k < uoff[i + 1]; k++) { remove(unodes[k], A); add(unodes[k], best); }
+          part_of[i] = best;
+          auto& ga = groups[A];
+          ga.erase(std::find(ga.begin(), ga.end(), i));
+          groups[best].push_back(i);
+          moves++;
+        }
+        moves_total += moves;
+        if (moves * 200 < nu) break;   // converged (< 0.5% of the units moved)
+      }
+      for (auto& g : groups) std::sort(g.begin(), g.end());
+      std::vector<std::vector<uint32_t>> kept;
+      for (auto& g : groups) if (!g.empty()) kept.push_back(std::move(g));
+      groups.swap(kept);
+      if (opt.verbose >= 1) {
+        uint64_t pins = 0;
+        for (size_t x = 0; x < N; x++) if (shared((uint32_t)x)) pins += users[x];
+        fprintf(stderr, "gem_map: stage %d km1 refinement: %llu moves, km1 %llu -> %llu (%llu pins, %zu groups)\n",
+                stage, (unsigned long long)moves_total, (unsigned long long)before, (unsigned long long)km1_cost(),
+                (unsigned long long)pins, groups.size());
+      }
+      (void)rep_before;
     }
     // ---- Algorithm 1: after the excessive partitioning above,
     // visit partitions largest first; sort the unvisited ones by cone overlap
