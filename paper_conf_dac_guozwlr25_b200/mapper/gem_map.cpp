@@ -31,6 +31,7 @@
 #include <cstdint>
 #include <cstdio>
 #include <cstdlib>
+#include <cmath>
 #include <cstring>
 #include <fstream>
 #include <functional>
@@ -1947,47 +1948,12 @@ static void partition(Design& D) {
       }
     }
     double cap = std::max<double>({64.0, 4.0 * (double)stage_ands / target * opt.cap_slack, 3.0 * med});
-    std::vector<std::vector<uint32_t>> groups;   // indices into su
-    for (int iter = 0; iter < 4; iter++) {
-      groups.clear();
-      cur_stamp++;
-      uint64_t size = 0;
-      for (uint32_t i = 0; i < su.size(); i++) {
-        // try adding to the current group
-        if (groups.empty()) groups.emplace_back();
-        uint32_t add = add_cone(su[i]);
-        if (!groups.back().empty() && size + add > cap) {
-          // start a new group containing unit i
-          groups.emplace_back();
-          cur_stamp++;
-          size = add_cone(su[i]);
-          groups.back().push_back(i);
-        } else {
-          size += add;
-          groups.back().push_back(i);
-        }
-      }
-      double ratio = (double)groups.size() / target;
-      if (opt.verbose >= 1)
-        fprintf(stderr, "gem_map: stage %d packing iter %d cap %.0f -> %zu groups (target %d)\n", stage, iter, cap,
-                groups.size(), target);
-      if (ratio > 0.85 && ratio < 1.2) break;
-      cap *= std::max(0.5, std::min(2.0, ratio));
-    }
-    // ---- min-cut refinement (the partitioner of P:105/P:117, RepCut [17]):
-    // the RepCut hypergraph has one vertex per unit (endpoint) and one
-    // hyperedge per AND node, spanning the units whose cone contains it; a
-    // node is replicated in every partition that holds one of its units, so
-    // the replication cost is the connectivity-minus-one (km1) metric
-    // sum_x (lambda(x) - 1).  k-way FM-style passes move single units to the
-    // partition that lowers km1 most (gain = the unit's shared nodes that leave
-    // its partition minus those new to the target), keeping every partition's
-    // cone under km1_slack x the packing cap.  Nodes with one user move with
-    // their unit; nodes with more than km1_pins users (shallow, wide logic that
-    // every partition needs anyway) are left out of the gains.
-    if (opt.km1 > 0 && groups.size() > 1) {
-      const uint32_t nu = (uint32_t)su.size();
-      std::vector<uint32_t> uoff(nu + 1, 0), unodes;
+    // unit cones (CSR over su) and node users: the RepCut hypergraph (one
+    // hyperedge per AND node over the units whose cone contains it)
+    const uint32_t nu = (uint32_t)su.size();
+    std::vector<uint32_t> uoff(nu + 1, 0), unodes, users;
+    const bool need_cones = opt.km1 > 0;
+    if (need_cones) {
       for (uint32_t i = 0; i < nu; i++) {
         cur_stamp++;
         unit_lits(su[i], lits);
@@ -2006,8 +1972,60 @@ static void partition(Design& D) {
         }
         uoff[i + 1] = (uint32_t)unodes.size();
       }
-      std::vector<uint32_t> users(N, 0);
+      users.assign(N, 0);
       for (uint32_t x : unodes) users[x]++;
+    }
+    auto shared = [&](uint32_t x) { return users[x] >= 2 && users[x] <= (uint32_t)opt.km1_pins; };
+    auto pack = [&](double pcap, std::vector<std::vector<uint32_t>>& out) {
+      out.clear();
+      cur_stamp++;
+      uint64_t size = 0;
+      for (uint32_t i = 0; i < su.size(); i++) {
+        // try adding to the current group
+        if (out.empty()) out.emplace_back();
+        uint32_t add = add_cone(su[i]);
+        if (!out.back().empty() && size + add > pcap) {
+          // start a new group containing unit i
+          out.emplace_back();
+          cur_stamp++;
+          size = add_cone(su[i]);
+          out.back().push_back(i);
+        } else {
+          size += add;
+          out.back().push_back(i);
+        }
+      }
+    };
+    // cap search: the group count as a function of the cap is not monotone
+    // (below the size of typical shared cones every unit ends up alone), so
+    // keep the iteration whose count is closest to the target
+    std::vector<std::vector<uint32_t>> groups, best_groups;   // indices into su
+    double best_err = 1e300, best_cap = cap;
+    for (int iter = 0; iter < 6; iter++) {
+      pack(cap, groups);
+      const double ratio = (double)groups.size() / target;
+      if (opt.verbose >= 1)
+        fprintf(stderr, "gem_map: stage %d packing iter %d cap %.0f -> %zu groups (target %d)\\n", stage, iter, cap,
+                groups.size(), target);
+      const double err = std::fabs(std::log(ratio));
+      if (err < best_err) { best_err = err; best_cap = cap; best_groups = groups; }
+      if (ratio > 0.85 && ratio < 1.2) break;
+      cap *= std::max(0.5, std::min(2.0, ratio > 3.0 ? 1.5 : ratio));
+    }
+    groups.swap(best_groups);
+    cap = best_cap;
+    // ---- min-cut refinement (the partitioner of P:105/P:117, RepCut [17]):
+    // the RepCut hypergraph has one vertex per unit (endpoint) and one
+    // hyperedge per AND node, spanning the units whose cone contains it; a
+    // node is replicated in every partition that holds one of its units, so
+    // the replication cost is the connectivity-minus-one (km1) metric
+    // sum_x (lambda(x) - 1).  k-way FM-style passes move single units to the
+    // partition that lowers km1 most (gain = the unit's shared nodes that leave
+    // its partition minus those new to the target), keeping every partition's
+    // cone under km1_slack x the packing cap.  Nodes with one user move with
+    // their unit; nodes with more than km1_pins users (shallow, wide logic that
+    // every partition needs anyway) are left out of the gains.
+    if (opt.km1 > 0 && groups.size() > 1) {
       // per shared node: (partition, count) slots, at most `users` of them
       std::vector<uint32_t> noff(N + 1, 0);
       for (size_t x = 0; x < N; x++) noff[x + 1] = noff[x] + ((users[x] >= 2 && users[x] <= (uint32_t)opt.km1_pins) ? users[x] : 0);
@@ -2032,7 +2050,6 @@ static void partition(Design& D) {
           npart[k] = npart[last]; ncnt[k] = ncnt[last];
         }
       };
-      auto shared = [&](uint32_t x) { return users[x] >= 2 && users[x] <= (uint32_t)opt.km1_pins; };
       // partition sizes: exact cones (private + shared + wide nodes)
       std::vector<uint64_t> psize(ng, 0);
       {
@@ -2051,6 +2068,7 @@ static void partition(Design& D) {
       std::vector<uint32_t> upriv(nu, 0);
       {
         std::vector<uint32_t> off2(nu + 1, 0), sh;
+        sh.reserve(unodes.size() / 4);
         for (uint32_t i = 0; i < nu; i++) {
           for (uint32_t k = uoff[i]; k < uoff[i + 1]; k++) {
             const uint32_t x = unodes[k];
