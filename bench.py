@@ -558,8 +558,18 @@ def roofline(res, peaks, dev):
                              "per thread + 13 fold levels + write-out + block barrier (gem_bench_floor, measured "
                              "on this GPU in this run)"}
         roof["latency_floor"] = lat
+        # does the program stream from HBM every cycle?  The committed ncu
+        # capture at the same cycles per launch decides (DRAM bytes per cycle
+        # vs program bytes); without one, a program larger than half the L2
+        # (126 MB) is assumed to stream
         l2_bytes = 126e6
-        hbm_floor = hbm_peak * 1e9 / info.program_bytes if info.program_bytes > 0.5 * l2_bytes else float("inf")
+        if traffic is not None:
+            streamed = traffic / C > 0.5 * info.program_bytes
+            hbm["dram_bytes_per_cycle_ncu"] = traffic / C
+        else:
+            streamed = info.program_bytes > 0.5 * l2_bytes
+        hbm["program_streamed"] = streamed
+        hbm_floor = hbm_peak * 1e9 / info.program_bytes if streamed else float("inf")
         hbm["floor_cycles_per_s"] = hbm_floor if hbm_floor != float("inf") else None
         if hz_kernel / hbm_floor > hz_kernel / floor_hz:
             roof.update({"bound": "hbm", "achieved": info.program_bytes * hz_kernel / 1e9,
