@@ -674,6 +674,13 @@ struct Mapper {
           if (mc[cons[j]]) r = std::max(r, rd[cons[j]] + 1);
         rd[i] = r;
       }
+      if (opt.verbose >= 4) {
+        uint32_t rem = 0, left = 0, lv1 = 0;
+        for (uint32_t i = 0; i < n; i++)
+          if (mc[i]) { rem = std::max(rem, d[i] + rd[i]); left++; lv1 += d[i] <= (uint32_t)opt.levels; }
+        fprintf(stderr, "gem_map: part %p layer %u: remaining depth %u, %u nodes left (%u within reach)\n",
+                (void*)&P, n_layers, rem, left, lv1);
+      }
       // candidates per level
       std::vector<uint32_t> cand[14];
       for (uint32_t i = 0; i < n; i++)
