@@ -73,6 +73,9 @@ struct KParams {
   // (act_words >= max n_gread) and {evaluated, skipped} partition-cycle counters
   unsigned long long* act_cnt;
   uint32_t act_words;
+  // single-CTA launches (LOC kernels): the flop / RAM-read words live in shared
+  // memory across cycles, [2][loc_words] with loc_words = q_words + n_rams
+  uint32_t loc_words;
   float l2_frac;           // > 0: streamed program chunks keep this fraction evict_last in L2
   // lane mode, one stage: dynamic work distribution.  Units {partition, first
   // stream, items, 0} in LPT order; CTA b starts every cycle with unit b and
@@ -492,10 +495,16 @@ __device__ __forceinline__ void top_layer(uint32_t topc, uint32_t topwo, uint32_
 // -- S still holds the previous evaluation of the same inputs, so the endpoint
 // commit below re-stores the same words (row f3).
 // ACT = false compiles to the plain path (no activity code in the hot loop).
-template <bool ACT>
+// LOC (single-CTA launch of one partition and one stream, gem_step_kernel<.., true>):
+// every flop and RAM-read word this partition reads was written by itself in
+// the previous cycle, so they come from the shared-memory copy `loc` (no L2
+// round trip), and the PI words of cycle c+1 are loaded into `pv` during
+// cycle c (their latency hides behind the layers).
+template <bool ACT, bool LOC>
 __device__ void run_partition(const KParams& kp, ProgSrc& ps, uint32_t* S, uint32_t* ramp, uint32_t* topb,
                               uint32_t p, uint32_t st0, uint32_t nst, uint32_t c, uint32_t cur, uint32_t nxt,
-                              bool prof_on, uint32_t* act = nullptr, bool act_first = true) {
+                              bool prof_on, uint32_t* act = nullptr, bool act_first = true,
+                              uint32_t* loc = nullptr, uint32_t (*pv)[4] = nullptr) {
   const uint32_t tid = threadIdx.x, lane = tid & 31, warp = tid >> 5;
   const uint32_t SW = kp.state_words;
   const uint32_t s_base = smem_u32(S);
@@ -571,7 +580,20 @@ __device__ void run_partition(const KParams& kp, ProgSrc& ps, uint32_t* S, uint3
         else if (reg == GEM_R_Q) a = kp.q + ((size_t)cur * kp.n_streams + st) * kp.q_words + idx;
         else if (reg == GEM_R_RD) a = kp.rd + ((size_t)cur * kp.n_streams + st) * kp.n_rams + idx;
         else a = kp.cut + (size_t)st * kp.cut_words + idx;
-        v[u] = rd_global(a);
+        if (LOC) {
+          if (reg == GEM_R_PI) {
+            v[u] = c ? (*pv)[u] : rd_global(a);
+            if (c + 1 < kp.ncycles) (*pv)[u] = rd_global(a + kp.pi_words);   // cycle c+1's word
+          } else if (reg == GEM_R_Q) {
+            v[u] = loc[cur * kp.loc_words + idx];
+          } else if (reg == GEM_R_RD) {
+            v[u] = loc[cur * kp.loc_words + kp.q_words + idx];
+          } else {
+            v[u] = rd_global(a);
+          }
+        } else {
+          v[u] = rd_global(a);
+        }
         dst[u] = j * SW + e.y;
       }
     }
@@ -665,7 +687,10 @@ commit:
     if (lane == 0) {
       const uint32_t dst = od[o];
       const uint32_t reg = GEM_GID_REGION(dst), idx = GEM_GID_INDEX(dst);
-      if (reg == GEM_R_Q) __stcg(kp.q + ((size_t)nxt * kp.n_streams + st) * kp.q_words + idx, v);
+      if (reg == GEM_R_Q) {
+        __stcg(kp.q + ((size_t)nxt * kp.n_streams + st) * kp.q_words + idx, v);
+        if (LOC) loc[nxt * kp.loc_words + idx] = v;
+      }
       else if (reg == GEM_R_PO) __stcg(kp.po + ((size_t)st * kp.out_cap + c) * kp.po_words + idx, v);
       else if (reg == GEM_R_CUT) __stcg(kp.cut + (size_t)st * kp.cut_words + idx, v);
       else ramp[j * 4 * GEM_MAX_RAMS_PER_PART + idx] = v;
@@ -687,6 +712,7 @@ commit:
       const uint32_t cur_w = __ldcg(M + wa);
       __stcg(M + wa, (cur_w & ~be) | (wd & be));
       __stcg(kp.rd + ((size_t)nxt * kp.n_streams + st) * kp.n_rams + id, old);
+      if (LOC) loc[nxt * kp.loc_words + kp.q_words + id] = old;
     }
   }
   __syncthreads();  // S / ramp / ring slots reused by the next work item
@@ -722,7 +748,7 @@ __device__ void record_state(const KParams& kp, uint32_t c, uint32_t buf) {
 }
 
 // ACT: GEM_F_ACTIVITY build of the kernel (the plain one carries no pruning code)
-template <bool ACT>
+template <bool ACT, bool LOC>
 __global__ void __launch_bounds__(GEM_THREADS, 2) gem_step_kernel(const KParams kp) {
   extern __shared__ __align__(16) uint32_t smem[];
   // layout (words): S[group][state_words] | area[area_words] | ctab[256] | ramp[group][128] |
@@ -742,6 +768,7 @@ __global__ void __launch_bounds__(GEM_THREADS, 2) gem_step_kernel(const KParams 
   uint32_t* wlc = res_n + 16;
   uint64_t* mbar = reinterpret_cast<uint64_t*>(wlc + GEM_WL_CACHE_WORDS);
   uint32_t* act_buf = reinterpret_cast<uint32_t*>(mbar + 16);  // [act_words] (GEM_F_ACTIVITY)
+  uint32_t* loc = act_buf + kp.act_words;                        // [2][loc_words] (LOC kernels)
   const uint32_t tid = threadIdx.x;
   const uint32_t G = gridDim.x, B = blockIdx.x;
   if (tid == 0) {
@@ -892,6 +919,15 @@ __global__ void __launch_bounds__(GEM_THREADS, 2) gem_step_kernel(const KParams 
 
   unsigned long long bar_target = 0;
   const bool instr = (kp.flags & (GEM_F_TRACE_STATE | GEM_F_DIGEST)) != 0;
+  uint32_t pv[4] = {0u, 0u, 0u, 0u};   // LOC: prefetched PI words of the next cycle
+  if (LOC) {
+    // the state of cycle t0 into shared memory (Q[cur] and RD[cur] of the launch's first cycle)
+    const uint32_t c0 = (uint32_t)(kp.t0 & 1u);
+    for (uint32_t k = tid; k < kp.loc_words; k += GEM_THREADS)
+      loc[c0 * kp.loc_words + k] = k < kp.q_words ? __ldcg(kp.q + (size_t)c0 * kp.n_streams * kp.q_words + k)
+                                                  : __ldcg(kp.rd + (size_t)c0 * kp.n_streams * kp.n_rams + (k - kp.q_words));
+    __syncthreads();
+  }
   for (uint32_t c = 0; c < kp.ncycles; c++) {
     const uint64_t t = kp.t0 + c;
     const uint32_t cur = (uint32_t)(t & 1u), nxt = cur ^ 1u;
@@ -903,8 +939,8 @@ __global__ void __launch_bounds__(GEM_THREADS, 2) gem_step_kernel(const KParams 
       for (uint32_t k = kb; k < ke; k++) {
         const uint2 it = wl_item(s, k);
         const uint32_t nst = min(kp.group, kp.n_streams - it.y);
-        run_partition<ACT>(kp, ps, S, ramp, topb, it.x, it.y, nst, c, cur, nxt, prof_on && k == kb && s == 0, act,
-                           c == 0);
+        run_partition<ACT, LOC>(kp, ps, S, ramp, topb, it.x, it.y, nst, c, cur, nxt, prof_on && k == kb && s == 0,
+                                act, c == 0, loc, &pv);
         if (!ps.resident) {
           // prefetch the next work item's prologue (overlaps the grid barrier)
           uint32_t np = ~0u;
@@ -1040,6 +1076,8 @@ struct gem_sim {
   uint32_t area_words = 0, slot_words = 0, ring_slots = 0, resident = 0, group = 1;
   // lane mode (stream-sliced, >= 32 streams and a blob with lane programs)
   uint32_t act_words = 0;                      // GEM_F_ACTIVITY: max n_gread over partitions
+  bool local = false;                          // single-CTA launch: LOC kernel (flops in shared memory)
+  uint32_t loc_words = 0, max_gread = 0;
   uint4* d_dyn_units = nullptr;                // lane mode dynamic work units
   uint32_t n_units = 0, *d_dyn_ctr = nullptr;
   unsigned long long* d_act = nullptr;         // {evaluated, skipped}
@@ -1188,7 +1226,8 @@ static double build_worklists(const gem_sim* sim, uint32_t G, std::vector<uint32
 }
 
 static const void* step_kernel_for(const gem_sim* sim) {
-  return sim->act_words ? (const void*)gem_step_kernel<true> : (const void*)gem_step_kernel<false>;
+  if (sim->act_words) return (const void*)gem_step_kernel<true, false>;
+  return sim->local ? (const void*)gem_step_kernel<false, true> : (const void*)gem_step_kernel<false, false>;
 }
 
 // Choose CTAs per SM, grid, work lists and the shared-memory program mode.
@@ -1220,8 +1259,13 @@ static int plan_launch(gem_sim* sim, uint32_t max_chunk_words, uint32_t grid_lim
     sim->max_items = std::max(sim->max_items, (sim->h_stage[s + 1] - sim->h_stage[s]) *
                                                   ((sim->n_streams + sim->group - 1) / sim->group));
   if (sim->group != 1) sim->act_words = 0;   // activity pruning needs one stream per work item
+  // one partition, one stream, one stage: a single CTA owns every flop and RAM,
+  // so the LOC kernel keeps them in shared memory across cycles
+  sim->loc_words = sim->q_words_int + sim->n_rams;
+  sim->local = sim->n_parts == 1 && sim->n_streams == 1 && sim->n_stages == 1 && !sim->act_words &&
+               sim->max_gread <= 4 * GEM_THREADS && sim->loc_words <= 4096 && !sim->cfg.grid_limit;
   const uint32_t fixed_words = sim->group * (sim->state_words + 4 * GEM_MAX_RAMS_PER_PART + 16) + GEM_MAX_CHUNKS +
-                               48 + GEM_WL_CACHE_WORDS + 32 + sim->act_words;
+                               48 + GEM_WL_CACHE_WORDS + 32 + sim->act_words + (sim->local ? 2 * sim->loc_words : 0u);
   const bool allow_res = !(sim->flags & GEM_F_NO_RESIDENT);
   const uint32_t force_bps = sim->cfg.ctas_per_sm;
   struct Choice { uint32_t bps = 0, grid = 0, area = 0, resident = 0, ring = 0; double score = 0; };
@@ -1488,6 +1532,7 @@ static int load_impl(gem_sim* sim, const uint32_t* w, size_t nw, const gem_confi
   for (uint32_t p = 0; p < sim->n_parts; p++) {
     const uint32_t* pr = w + w[GH_OFF_PROG] + parts[p * GP_WORDS + GP_PROG_OFF];
     if (cfg->flags & GEM_F_ACTIVITY) sim->act_words = std::max(sim->act_words, (pr[PH_N_GREAD] + 3u) & ~3u);
+    sim->max_gread = std::max(sim->max_gread, pr[PH_N_GREAD]);
   }
   // inverse permutation tables
   std::vector<uint32_t> q_int_of_ext(std::max<uint32_t>(sim->n_flops, 1), 0),
@@ -1706,6 +1751,7 @@ int gem_step(gem_sim* sim, uint64_t ncycles) {
   kp.dyn_ctr = sim->d_dyn_ctr;
   if (sim->d_dyn_ctr) CK(cudaMemsetAsync(sim->d_dyn_ctr, 0, 16, sim->stream));
   kp.act_words = sim->lanes ? 0u : sim->act_words;
+  kp.loc_words = sim->local ? sim->loc_words : 0u;
   if (sim->flags & GEM_F_PROFILE) {
     const uint32_t pc = (uint32_t)std::min<uint64_t>(ncycles, 256);
     if (!sim->d_prof || sim->prof_cycles < pc) {
