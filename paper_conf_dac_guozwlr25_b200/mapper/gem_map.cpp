@@ -1557,7 +1557,46 @@ struct Mapper {
       if (is_ep[i]) { last[i] = INF; continue; }
       for (uint32_t j = coff[i]; j < coff[i + 1]; j++) last[i] = std::max(last[i], step_of[cons[j]]);
     }
-    // ---- words: 0 = constant, 1..n_src = ports; free pool per residue mod 16
+    // ---- future-read residue budgets: bud[(s * 2 + side) * kHalf + r] = operands of
+    // step s (side 0 = A, 1 = B) already placed at word residue r.  A value's word
+    // residue is chosen where its future readers' steps have the fewest, so the
+    // operands of every step spread over the residues (conflict-free groups).
+    std::vector<uint16_t> bud((size_t)S * 2 * kHalf, 0);
+    auto readers_cost = [&](uint32_t x, uint32_t r) {
+      uint32_t c = 0;
+      for (uint32_t j = coff[x]; j < coff[x + 1]; j++) {
+        const uint32_t y = cons[j];
+        c += bud[((size_t)step_of[y] * 2 + ((la[y] >> 1) == x ? 0u : 1u)) * kHalf + r];
+      }
+      return c;
+    };
+    auto add_readers = [&](uint32_t x, uint32_t r) {
+      for (uint32_t j = coff[x]; j < coff[x + 1]; j++) {
+        const uint32_t y = cons[j];
+        bud[((size_t)step_of[y] * 2 + ((la[y] >> 1) == x ? 0u : 1u)) * kHalf + r]++;
+      }
+    };
+    // ---- words: 0 = constant, 1..n_src = ports (entry k -> word k+1); within each
+    // aligned block of kHalf entries (the same lines whichever lane loads them,
+    // and consecutive words for the port stores) the sources are permuted onto
+    // the residues their readers need most
+    for (size_t b0 = 0; b0 < srcs.size(); b0 += kHalf) {
+      const size_t b1 = std::min(srcs.size(), b0 + kHalf);
+      std::vector<uint32_t> blk(srcs.begin() + b0, srcs.begin() + b1), out(b1 - b0, UINT32_MAX);
+      std::stable_sort(blk.begin(), blk.end(), [&](uint32_t x, uint32_t y) { return coff[x + 1] - coff[x] > coff[y + 1] - coff[y]; });
+      for (uint32_t x : blk) {
+        size_t best = 0;
+        uint32_t bc = UINT32_MAX;
+        for (size_t j = 0; j < out.size(); j++) {
+          if (out[j] != UINT32_MAX) continue;
+          const uint32_t c = readers_cost(x, (uint32_t)(b0 + j + 1) % kHalf);
+          if (c < bc) { bc = c; best = j; }
+        }
+        out[best] = x;
+        add_readers(x, (uint32_t)(b0 + best + 1) % kHalf);
+      }
+      std::copy(out.begin(), out.end(), srcs.begin() + b0);
+    }
     std::vector<int32_t> word(n, -1);
     word[0] = 0;
     std::vector<std::set<uint32_t>> freew(kHalf);
@@ -1603,31 +1642,104 @@ struct Mapper {
         for (uint32_t w : die[s - 1]) freew[w % kHalf].insert(w);
       for (uint32_t g = 0; g < kGroups; g++) { ca[g].fill(0); cb[g].fill(0); cd[g].fill(0); fill[g] = 0; }
       auto& st = steps[s];
-      // busiest operands first
+      // critical ops first
       std::stable_sort(st.begin(), st.end(), [&](uint32_t x, uint32_t y) { return rd[x] > rd[y]; });
-      for (uint32_t x : st) {
-        const uint32_t ra = lw(la[x]) % kHalf, rb = lw(lb[x]) % kHalf;
-        // half-warp group with room and the fewest operand-residue collisions
+      // Operand residues: an op is an edge (A residue, B residue) of a bipartite
+      // multigraph; a proper edge colouring puts ops of distinct A and distinct
+      // B residues in each colour class, i.e. conflict-free wavefronts.  König:
+      // max-degree colours suffice (alternating-path recolouring); colour c ->
+      // group c when there are at most kGroups colours, the rest fall back to
+      // the greedy choice below.
+      std::vector<int32_t> pref(st.size(), -1);
+      {
+        const uint32_t n_e = (uint32_t)st.size();
+        std::array<uint32_t, 64> deg{};
+        for (uint32_t x : st) { deg[lw(la[x]) % kHalf]++; deg[kHalf + lw(lb[x]) % kHalf]++; }
+        uint32_t C = 0;
+        for (uint32_t v = 0; v < 2 * kHalf; v++) C = std::max(C, deg[v]);
+        std::vector<int32_t> at((size_t)2 * kHalf * C, -1), col(n_e, -1);   // at[v*C + c] = edge
+        auto U = [&](uint32_t e) { return lw(la[st[e]]) % kHalf; };
+        auto V = [&](uint32_t e) { return kHalf + lw(lb[st[e]]) % kHalf; };
+        for (uint32_t e = 0; e < n_e; e++) {
+          const uint32_t u = U(e), v = V(e);
+          uint32_t a = 0, bcol = 0;
+          while (at[(size_t)u * C + a] >= 0) a++;
+          while (at[(size_t)v * C + bcol] >= 0) bcol++;
+          if (at[(size_t)v * C + a] >= 0) {
+            // flip the a/b alternating path from v (a bipartite path never returns to u)
+            std::vector<uint32_t> path;
+            uint32_t w = v, cc = a;
+            while (at[(size_t)w * C + cc] >= 0) {
+              const uint32_t f = (uint32_t)at[(size_t)w * C + cc];
+              path.push_back(f);
+              w = (U(f) == w) ? V(f) : U(f);
+              cc = (cc == a) ? bcol : a;
+            }
+            for (uint32_t f : path) { at[(size_t)U(f) * C + col[f]] = -1; at[(size_t)V(f) * C + col[f]] = -1; }
+            for (uint32_t f : path) {
+              col[f] = col[f] == (int32_t)a ? (int32_t)bcol : (int32_t)a;
+              at[(size_t)U(f) * C + col[f]] = (int32_t)f;
+              at[(size_t)V(f) * C + col[f]] = (int32_t)f;
+            }
+          }
+          col[e] = (int32_t)a;
+          at[(size_t)u * C + a] = (int32_t)e;
+          at[(size_t)v * C + a] = (int32_t)e;
+        }
+        if (C <= kGroups)
+          for (uint32_t e = 0; e < n_e; e++) pref[e] = col[e];
+        else {
+          // the kGroups largest colour classes keep their group
+          std::vector<std::pair<uint32_t, uint32_t>> sz(C);
+          for (uint32_t c = 0; c < C; c++) sz[c] = {0u, c};
+          for (uint32_t e = 0; e < n_e; e++) sz[col[e]].first++;
+          std::sort(sz.begin(), sz.end(), std::greater<std::pair<uint32_t, uint32_t>>());
+          std::vector<int32_t> gmap(C, -1);
+          for (uint32_t k = 0; k < kGroups; k++) gmap[sz[k].second] = (int32_t)k;
+          for (uint32_t e = 0; e < n_e; e++) pref[e] = gmap[col[e]];
+        }
+      }
+      // operand words already read by each group (a repeated word is a broadcast, no conflict)
+      std::vector<std::array<uint32_t, 32>> gwa(kGroups), gwb(kGroups);
+      for (uint32_t ei = 0; ei < st.size(); ei++) {
+        const uint32_t x = st[ei];
+        const uint32_t wa = lw(la[x]), wb = lw(lb[x]);
+        const uint32_t ra = wa % kHalf, rb = wb % kHalf;
+        // group (kHalf lanes = one wavefront) with room and the fewest distinct
+        // same-residue operand words (the colouring's group when it has room)
         uint32_t bg = 0, bc = UINT32_MAX;
-        for (uint32_t g = 0; g < kGroups; g++) {
+        if (pref[ei] >= 0 && fill[pref[ei]] < kHalf) { bg = (uint32_t)pref[ei]; bc = 0; }
+        for (uint32_t g = 0; g < kGroups && bc; g++) {
           if (fill[g] == kHalf) continue;
-          const uint32_t c = 4u * (ca[g][ra] + cb[g][rb]) + fill[g] / 8;
+          uint32_t xa = 0, xb = 0;
+          bool da = false, db = false;
+          for (uint32_t k = 0; k < fill[g]; k++) {
+            da |= gwa[g][k] == wa; db |= gwb[g][k] == wb;
+          }
+          if (!da) xa = ca[g][ra];
+          if (!db) xb = cb[g][rb];
+          const uint32_t c = 4u * (xa + xb) + fill[g] / 8;
           if (c < bc) { bc = c; bg = g; }
         }
-        // destination residue: least used in the group, then lowest word
-        uint32_t bres = 0, bcost = UINT32_MAX;
-        for (uint32_t r = 0; r < kHalf; r++) {
-          const uint32_t c = cd[bg][r];
-          if (c < bcost) { bcost = c; bres = r; }
-        }
-        uint32_t w = UINT32_MAX;
         {
-          // among the least-used residues prefer one with a free word (compact state)
-          uint32_t bw = UINT32_MAX;
-          for (uint32_t r = 0; r < kHalf; r++)
-            if (cd[bg][r] == bcost && !freew[r].empty() && *freew[r].begin() < bw) { bw = *freew[r].begin(); bres = r; }
-          w = alloc(bres);
+          bool da = false, db = false;
+          for (uint32_t k = 0; k < fill[bg]; k++) { da |= gwa[bg][k] == wa; db |= gwb[bg][k] == wb; }
+          gwa[bg][fill[bg]] = wa;
+          gwb[bg][fill[bg]] = wb;
+          if (da) ca[bg][ra]--;   // (undone by the increment below: a repeated word adds no wavefront)
+          if (db) cb[bg][rb]--;
         }
+        // destination residue: least used by the group's stores, then the fewest
+        // future readers' operands at that residue, then a free (low) word
+        uint32_t bres = 0;
+        uint64_t bkey = UINT64_MAX;
+        for (uint32_t r = 0; r < kHalf; r++) {
+          const uint64_t fw = freew[r].empty() ? 0xFFFFFFull : *freew[r].begin();
+          const uint64_t key = ((uint64_t)cd[bg][r] << 56) | ((uint64_t)std::min<uint32_t>(readers_cost(x, r), 0xFFFFFF) << 24) | fw;
+          if (key < bkey) { bkey = key; bres = r; }
+        }
+        const uint32_t w = alloc(bres);
+        add_readers(x, w % kHalf);
         ca[bg][ra]++; cb[bg][rb]++; cd[bg][w % kHalf]++;
         const uint32_t t = bg * kHalf + fill[bg]++;
         word[x] = (int32_t)w;
