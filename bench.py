@@ -582,6 +582,22 @@ def roofline(res, peaks, dev):
             roof.update({"algorithmic": "simulated cycles per second of one stream",
                          "peak_source": "latency floor (gem_bench_floor, measured in this run)"})
             roof["binding"] = "latency"
+    elif info.lane_ops:
+        # LAN2 lane programs: every AND op moves three 4-byte lane
+        # words per 32-stream group through shared memory (two operand loads, one
+        # result store); the shared-memory pipe (128 B per SM clock) binds before
+        # the LOP3 issue does
+        smem_bytes = info.lane_ops * 12.0 / 32.0          # per stream-cycle
+        peak_smem = n_sms * 128.0 * float(peaks.get("sm_max_mhz", 1965.0)) * 1e6
+        ach = smem_bytes * hz_kernel * S
+        smem = {"bound": "smem", "achieved": ach / 1e9, "peak": peak_smem / 1e9, "unit": "GB/s",
+                "frac": ach / peak_smem,
+                "algorithmic": f"{info.lane_ops} AND ops x 3 lane words x 4 B per 32 streams per cycle "
+                               f"({smem_bytes:.0f} B per stream-cycle)",
+                "peak_source": f"{n_sms} SMs x 128 B/clk x sm_max_mhz ({peaks['_source']})"}
+        roof["smem"] = smem
+        roof.update({k: smem[k] for k in ("bound", "achieved", "peak", "unit", "frac", "algorithmic", "peak_source")})
+        roof["binding"] = "shared-memory traffic of the step ops (ALU fraction alongside)"
     else:
         roof["binding"] = "alu (independent streams: issue of LOP3/LDS per lane word)"
     return roof
@@ -595,7 +611,10 @@ def mapping_stats(info) -> dict:
             "levels": info.max_levels, "total_layers": info.total_layers,
             "replication": round(info.replication, 4), "program_bytes": info.program_bytes,
             "bytes_per_and": round(info.bytes_per_and, 3), "slot_util": round(info.slot_util, 4),
-            "levels_per_layer": round(info.max_levels / max(1, info.max_layers), 3)}
+            "levels_per_layer": round(info.max_levels / max(1, info.max_layers), 3),
+            "n_and_synth": info.n_and_synth, "levels_in": info.levels_in,
+            "leaf_util": round(info.total_leaves / max(1, info.total_layers * 8192), 4),
+            "lane_ops": info.lane_ops, "lane_steps": info.lane_steps}
 
 
 def main():

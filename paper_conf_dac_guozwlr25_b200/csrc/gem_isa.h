@@ -217,8 +217,8 @@ enum {
 #define GEM_LANE_STREAMS 32
 enum {
   LPH_MAGIC = 0, LPH_N_GREAD, LPH_N_LAYERS, LPH_N_OUT, LPH_N_RAM, LPH_LANE_WORDS, LPH_OFF_GREAD,
-  LPH_OFF_LAYERS, LPH_OFF_OUT, LPH_OFF_RAM, LPH_OFF_CHUNKS, LPH_N_CHUNKS, LPH_R12, LPH_R13, LPH_R14,
-  LPH_R15, LPH_WORDS = 16
+  LPH_OFF_LAYERS, LPH_OFF_OUT, LPH_OFF_RAM, LPH_OFF_CHUNKS, LPH_N_CHUNKS, LPH_N_OPS /* LAN2: AND ops */,
+  LPH_R13, LPH_R14, LPH_R15, LPH_WORDS = 16
 };
 /* lane layer header: [0,12) this layer {size, flags, topc, topwo, woff[8]};
  * [16,28) a copy of the NEXT layer's [0,12) (zeros after the last layer), so

@@ -48,6 +48,8 @@ class BlobInfo:
     n_and_synth: int = 0
     levels_in: int = 0
     synth_chains: int = 0
+    lane_ops: int = 0          # LAN2 lane programs: AND ops over all partitions (0 otherwise)
+    lane_steps: int = 0
 
     def stage_max_layers(self) -> list:
         """Deepest partition (layers) of each stage: a lower bound on the layers
@@ -94,6 +96,13 @@ def blob_info(blob: bytes) -> BlobInfo:
     u64 = lambda k: h[k + "_LO"] | (h[k + "_HI"] << 32)
     np_ = h["N_PARTS"]
     pt = w[h["OFF_PARTS"]:h["OFF_PARTS"] + GP_WORDS * np_].reshape(np_, GP_WORDS)
+    lane_ops = lane_steps = 0
+    if h["HAS_LANES"]:
+        for p in range(np_):
+            lp = h["OFF_LANE_PROG"] + int(pt[p, 9])
+            if int(w[lp]) == 0x324E414C:   # "LAN2"
+                lane_steps += int(w[lp + 2])
+                lane_ops += int(w[lp + 12])
     return BlobInfo(n_pi=h["N_PI"], n_po=h["N_PO"], n_flops=h["N_FLOPS"], n_rams=h["N_RAMS"],
                     n_parts=np_, n_stages=h["N_STAGES"], max_state_words=h["MAX_STATE_WORDS"],
                     max_layers=h["MAX_LAYERS"], total_layers=h["TOTAL_LAYERS"], q_words=h["Q_WORDS"],
@@ -103,4 +112,5 @@ def blob_info(blob: bytes) -> BlobInfo:
                     blob_bytes=len(blob), slots_used=u64("SLOTS_USED"), part_layers=pt[:, 3].tolist(),
                     max_chunk_words=h["MAX_CHUNK_WORDS"], max_prog_words=h["MAX_PROG_WORDS"],
                     part_cost=pt[:, 8].tolist(), part_stage=pt[:, 0].tolist(),
-                    n_and_synth=u64("N_AND_SYNTH"), levels_in=h["LEVELS_IN"], synth_chains=h["SYNTH_CHAINS"])
+                    n_and_synth=u64("N_AND_SYNTH"), levels_in=h["LEVELS_IN"], synth_chains=h["SYNTH_CHAINS"],
+                    lane_ops=lane_ops, lane_steps=lane_steps)

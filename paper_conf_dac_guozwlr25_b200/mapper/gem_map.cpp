@@ -1625,6 +1625,7 @@ struct Mapper {
     pr.assign(LPH_WORDS, 0);
     pr[LPH_MAGIC] = GEM_LANE2_MAGIC;
     pr[LPH_N_LAYERS] = S;
+    pr[LPH_N_OPS] = n_ops;
     pr[LPH_N_OUT] = (uint32_t)P.outs.size() * 32;
     pr[LPH_N_RAM] = (uint32_t)P.rams.size();
     pr[LPH_OFF_CHUNKS] = (uint32_t)pr.size();
