@@ -218,7 +218,7 @@ enum {
 enum {
   LPH_MAGIC = 0, LPH_N_GREAD, LPH_N_LAYERS, LPH_N_OUT, LPH_N_RAM, LPH_LANE_WORDS, LPH_OFF_GREAD,
   LPH_OFF_LAYERS, LPH_OFF_OUT, LPH_OFF_RAM, LPH_OFF_CHUNKS, LPH_N_CHUNKS, LPH_N_OPS /* LAN2: AND ops */,
-  LPH_R13, LPH_R14, LPH_R15, LPH_WORDS = 16
+  LPH_OPS_PER_THREAD /* LAN2: M ops per thread and step (0 = 1) */, LPH_R14, LPH_R15, LPH_WORDS = 16
 };
 /* lane layer header: [0,12) this layer {size, flags, topc, topwo, woff[8]};
  * [16,28) a copy of the NEXT layer's [0,12) (zeros after the last layer), so
@@ -240,7 +240,8 @@ enum { LLH_WORDS_ = 0, LLH_FLAGS, LLH_TOPC, LLH_TOPWO, LLH_WOFF0 /* ..+7 */, LLH
  * most 256 independent ANDs (one per thread) separated by a block barrier:
  *   header (LPH_*, LPH_N_LAYERS = n_steps, LPH_OFF_LAYERS = op array)
  *   gread:  one u32 gid_l per entry, entry k -> lane word k + 1 (as "LANE")
- *   ops:    [n_steps][256] uint2 {x, y}, thread t of step s runs op s*256+t:
+ *   ops:    [n_steps][M][256] uint2 {x, y} (M = LPH_OPS_PER_THREAD, 1 or 2), thread
+ *           t of step s runs ops (s*M + j)*256 + t, j < M:
  *             x = a | ia << 14 | b << 16 | ib << 30   (lane words < 16384)
  *             y = destination lane word (0 = no op)
  *           result(y) = (S[a] ^ -ia) & (S[b] ^ -ib); operands were written in

@@ -447,7 +447,7 @@ __device__ __forceinline__ void lane_ports2(const KParams& kp, uint32_t s_base, 
     brd[j] = kp.rd + X.q(cur, kp.n_rams * 32, 0, g);
     bcut[j] = kp.cut + X.q(0, kp.cut_words * 32, 0, g);
   }
-  constexpr uint32_t U = K >= 4 ? 4u : 8u / K;   // entries per thread per pass (U * K loads in flight)
+  constexpr uint32_t U = K >= 4 ? 4u : 8u / K;   // entries per thread per pass (U * K loads in flight; 8 for K = 4 measured slower)
   for (uint32_t kb = 0; kb < n_gread; kb += U * GEM_THREADS) {
     uint32_t e[U];
 #pragma unroll
@@ -472,11 +472,12 @@ __device__ __forceinline__ void lane_ports2(const KParams& kp, uint32_t s_base, 
 }
 
 // One work item of a compacted lane program ("LAN2", gem_isa.h): ports, then
-// the partition's ANDs in barrier-separated steps of <= 256 (thread t runs
-// op s*256+t of step s on all K groups: two LDS.K, 2K LOP3, one STS.K), then
-// endpoints and RAMs.  The op words stream from the L2-resident program into
-// registers kPre steps ahead of their use.
-template <int K>
+// the partition's ANDs in barrier-separated steps of <= 256*M (thread t runs
+// ops (s*M + j)*256 + t, j < M, of step s on all K groups: per op two LDS.K,
+// 2K LOP3, one STS.K; the M ops of a thread are independent, so their loads
+// overlap), then endpoints and RAMs.  The op words stream from the
+// L2-resident program into registers kPre steps ahead of their use.
+template <int K, int M>
 __device__ void run_lane_partition2(const KParams& kp, uint32_t* S, uint32_t* ramp, uint32_t p, uint32_t g0,
                                     uint32_t ng, uint32_t c, uint32_t cur, uint32_t nxt, unsigned long long* pacc) {
   const uint32_t tid = threadIdx.x;
@@ -498,10 +499,13 @@ __device__ void run_lane_partition2(const KParams& kp, uint32_t* S, uint32_t* ra
   const uint32_t off_out = h2.x, off_ram = h2.y;
   const uint2* ops = reinterpret_cast<const uint2*>(gprog + off_ops) + tid;
   // the first steps' ops: independent of S, their latency overlaps the port loads
-  constexpr uint32_t kPre = 6;
-  uint2 q[kPre];
+  constexpr uint32_t kPre = M == 1 ? 6 : 4;
+  uint2 q[kPre][M];
 #pragma unroll
-  for (uint32_t i = 0; i < kPre; i++) q[i] = i < n_steps ? __ldg(ops + i * GEM_LANE2_STEP) : make_uint2(0u, 0u);
+  for (uint32_t i = 0; i < kPre; i++)
+#pragma unroll
+    for (int j = 0; j < M; j++)
+      q[i][j] = i < n_steps ? __ldg(ops + (i * M + j) * GEM_LANE2_STEP) : make_uint2(0u, 0u);
   phase(0);
   lane_ports2<K>(kp, s_base, gprog + off_gread, n_gread, g0, ng, c, cur);
   if (tid < K) S[tid] = 0u;   // lane word 0 = constant 0 for every group
@@ -509,19 +513,32 @@ __device__ void run_lane_partition2(const KParams& kp, uint32_t* S, uint32_t* ra
   __syncthreads();
   phase(2);
   for (uint32_t s = 0; s < n_steps; s++) {
-    const uint2 o = q[0];
+    uint2 o[M];
 #pragma unroll
-    for (uint32_t i = 0; i + 1 < kPre; i++) q[i] = q[i + 1];
-    q[kPre - 1] = s + kPre < n_steps ? __ldg(ops + (s + kPre) * GEM_LANE2_STEP) : make_uint2(0u, 0u);
-    if (o.y) {
-      const uint32_t ia = (uint32_t)((int32_t)(o.x << 17) >> 31), ib = (uint32_t)((int32_t)(o.x << 1) >> 31);
-      uint32_t a[K], b[K], r[K];
-      ldsK<K>(s_base + 4u * K * (o.x & 0x3FFFu), a);
-      ldsK<K>(s_base + 4u * K * ((o.x >> 16) & 0x3FFFu), b);
+    for (int j = 0; j < M; j++) o[j] = q[0][j];
 #pragma unroll
-      for (int j = 0; j < K; j++) r[j] = (a[j] ^ ia) & (b[j] ^ ib);
-      stsK<K>(s_base + 4u * K * o.y, r);
-    }
+    for (uint32_t i = 0; i + 1 < kPre; i++)
+#pragma unroll
+      for (int j = 0; j < M; j++) q[i][j] = q[i + 1][j];
+#pragma unroll
+    for (int j = 0; j < M; j++)
+      q[kPre - 1][j] = s + kPre < n_steps ? __ldg(ops + ((s + kPre) * M + j) * GEM_LANE2_STEP) : make_uint2(0u, 0u);
+    uint32_t a[M][K], b[M][K];
+#pragma unroll
+    for (int j = 0; j < M; j++)
+      if (o[j].y) {
+        ldsK<K>(s_base + 4u * K * (o[j].x & 0x3FFFu), a[j]);
+        ldsK<K>(s_base + 4u * K * ((o[j].x >> 16) & 0x3FFFu), b[j]);
+      }
+#pragma unroll
+    for (int j = 0; j < M; j++)
+      if (o[j].y) {
+        const uint32_t ia = (uint32_t)((int32_t)(o[j].x << 17) >> 31), ib = (uint32_t)((int32_t)(o[j].x << 1) >> 31);
+        uint32_t r[K];
+#pragma unroll
+        for (int g = 0; g < K; g++) r[g] = (a[j][g] ^ ia) & (b[j][g] ^ ib);
+        stsK<K>(s_base + 4u * K * o[j].y, r);
+      }
     __syncthreads();
   }
   phase(3);
@@ -553,7 +570,7 @@ __device__ void record_state_lane(const KParams& kp, uint32_t c, uint32_t buf) {
   }
 }
 
-template <int K, bool V2>
+template <int K, bool V2, int M>
 __global__ void __launch_bounds__(GEM_THREADS, (V2 && K <= 2) ? 4 : 2) gem_lane_kernel(const KParams kp) {
   extern __shared__ __align__(16) uint32_t smem[];
   // layout: S[lane_words][K] | ramp[K][ramp_words] | topv[16][K]  (no program ring:
@@ -590,8 +607,8 @@ __global__ void __launch_bounds__(GEM_THREADS, (V2 && K <= 2) ? 4 : 2) gem_lane_
         for (uint32_t r = 0; r < U.z; r++) {
           const uint32_t g0 = (U.y >> 5) + r * K;
           if (V2)
-            run_lane_partition2<K>(kp, S, ramp, U.x, g0, min((uint32_t)K, kp.n_groups - g0), c, cur, nxt,
-                                   prof_on ? pacc : nullptr);
+            run_lane_partition2<K, M>(kp, S, ramp, U.x, g0, min((uint32_t)K, kp.n_groups - g0), c, cur, nxt,
+                                      prof_on ? pacc : nullptr);
           else
             run_lane_partition<K>(kp, S, ramp, topv, U.x, g0, min((uint32_t)K, kp.n_groups - g0), c, cur, nxt,
                                   prof_on ? pacc : nullptr);
@@ -608,8 +625,8 @@ __global__ void __launch_bounds__(GEM_THREADS, (V2 && K <= 2) ? 4 : 2) gem_lane_
           const uint2 it = __ldg(&kp.wl_items[k]);
           const uint32_t g0 = it.y >> 5;
           if (V2)
-            run_lane_partition2<K>(kp, S, ramp, it.x, g0, min((uint32_t)K, kp.n_groups - g0), c, cur, nxt,
-                                   prof_on ? pacc : nullptr);
+            run_lane_partition2<K, M>(kp, S, ramp, it.x, g0, min((uint32_t)K, kp.n_groups - g0), c, cur, nxt,
+                                      prof_on ? pacc : nullptr);
           else
             run_lane_partition<K>(kp, S, ramp, topv, it.x, g0, min((uint32_t)K, kp.n_groups - g0), c, cur, nxt,
                                   prof_on ? pacc : nullptr);

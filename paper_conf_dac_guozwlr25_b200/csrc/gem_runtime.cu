@@ -1083,6 +1083,7 @@ struct gem_sim {
   unsigned long long* d_act = nullptr;         // {evaluated, skipped}
   uint32_t lanes = 0, n_groups = 0, lane_words = 0, lane_max_chunk = 0, ramp_words = 0, lane_groups = 1;
   bool lane_v2 = false;                        // compacted lane programs ("LAN2")
+  uint32_t lane_m = 1;                         // LAN2: ops per thread and step
   uint32_t *d_lprog = nullptr, *d_pi_lane = nullptr, *d_po_lane = nullptr;
   std::vector<uint32_t> h_parts, h_stage;
   // device buffers
@@ -1336,12 +1337,15 @@ static int plan_launch(gem_sim* sim, uint32_t max_chunk_words, uint32_t grid_lim
   return GEM_OK;
 }
 
-static const void* lane_kernel_for(uint32_t k, bool v2) {
+static const void* lane_kernel_for(uint32_t k, bool v2, uint32_t m) {
+  if (v2 && m == 2)
+    return k >= 4 ? (const void*)gem_lane_kernel<4, true, 2> : k == 2 ? (const void*)gem_lane_kernel<2, true, 2>
+                                                                        : (const void*)gem_lane_kernel<1, true, 2>;
   if (v2)
-    return k >= 4 ? (const void*)gem_lane_kernel<4, true> : k == 2 ? (const void*)gem_lane_kernel<2, true>
-                                                                     : (const void*)gem_lane_kernel<1, true>;
-  return k >= 4 ? (const void*)gem_lane_kernel<4, false> : k == 2 ? (const void*)gem_lane_kernel<2, false>
-                                                                    : (const void*)gem_lane_kernel<1, false>;
+    return k >= 4 ? (const void*)gem_lane_kernel<4, true, 1> : k == 2 ? (const void*)gem_lane_kernel<2, true, 1>
+                                                                        : (const void*)gem_lane_kernel<1, true, 1>;
+  return k >= 4 ? (const void*)gem_lane_kernel<4, false, 1> : k == 2 ? (const void*)gem_lane_kernel<2, false, 1>
+                                                                       : (const void*)gem_lane_kernel<1, false, 1>;
 }
 
 // Lane mode launch: one CTA per SM (all shared memory for the lane state and
@@ -1383,7 +1387,7 @@ static int plan_launch_lanes(gem_sim* sim, uint32_t grid_limit) {
   if (grid_limit) grid = std::max<uint32_t>(1, std::min(grid, grid_limit));
   grid = std::min<uint32_t>(grid, GEM_BAR_MAX_CTAS);
   const uint32_t smem = fixed_words * 4;
-  const void* lk = lane_kernel_for(gl, sim->lane_v2);
+  const void* lk = lane_kernel_for(gl, sim->lane_v2, sim->lane_m);
   CK(cudaFuncSetAttribute(lk, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem));
   int occ = 0;
   CK(cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ, lk, GEM_THREADS, smem));
@@ -1559,9 +1563,12 @@ static int load_impl(gem_sim* sim, const uint32_t* w, size_t nw, const gem_confi
     sim->ramp_words = std::max<uint32_t>(w[GH_MAX_RAMS_PART], 1) * 128;
     const uint32_t* lp = w + w[GH_OFF_LANE_PROG];
     sim->lane_v2 = sim->n_parts && lp[parts[GP_LANE_OFF] + LPH_MAGIC] == GEM_LANE2_MAGIC;
+    sim->lane_m = sim->lane_v2 ? std::max<uint32_t>(1, lp[parts[GP_LANE_OFF] + LPH_OPS_PER_THREAD]) : 1u;
     for (uint32_t p = 0; p < sim->n_parts; p++) {
-      const uint32_t m = lp[parts[(size_t)p * GP_WORDS + GP_LANE_OFF] + LPH_MAGIC];
-      if (m != (sim->lane_v2 ? GEM_LANE2_MAGIC : GEM_LANE_MAGIC)) return fail(GEM_E_FORMAT, "mixed or bad lane programs");
+      const uint32_t* h = lp + parts[(size_t)p * GP_WORDS + GP_LANE_OFF];
+      if (h[LPH_MAGIC] != (sim->lane_v2 ? GEM_LANE2_MAGIC : GEM_LANE_MAGIC) ||
+          (sim->lane_v2 && std::max<uint32_t>(1, h[LPH_OPS_PER_THREAD]) != sim->lane_m) || sim->lane_m > 2)
+        return fail(GEM_E_FORMAT, "mixed or bad lane programs");
     }
   }
   // uploads
@@ -1778,7 +1785,7 @@ int gem_step(gem_sim* sim, uint64_t ncycles) {
   }
   void* args[] = {&kp};
   CK(cudaEventRecord(sim->ev0, sim->stream));
-  CK(cudaLaunchCooperativeKernel(sim->lanes ? lane_kernel_for(sim->lane_groups, sim->lane_v2) : step_kernel_for(sim),
+  CK(cudaLaunchCooperativeKernel(sim->lanes ? lane_kernel_for(sim->lane_groups, sim->lane_v2, sim->lane_m) : step_kernel_for(sim),
                                  dim3(sim->grid), dim3(GEM_THREADS), args, sim->smem_bytes, sim->stream));
   CK(cudaEventRecord(sim->ev1, sim->stream));
   sim->in_head += (uint32_t)ncycles;

@@ -80,6 +80,7 @@ struct Options {
   int lane_holes = 32;      // best-fitting holes considered per run
   int lane_k = 4;           // lane mode 2: bank-conflict model for K interleaved groups (K lanes' words
                             // per 16 bytes: lanes of 32/K share one wavefront)
+  int lane_m = 1;           // lane mode 2: independent ops per thread and step (1 or 2)
   int lane_mode = 2;        // 1: lane program from the boomerang placement ("LANE"); 2: compacted AND
                             // list in barrier-separated steps ("LAN2", gem_isa.h)
   int banks = 1;            // bank-conflict-aware renaming of the state words (rename_state_words)
@@ -127,6 +128,7 @@ static Options parse_opts(const char* s) {
     else if (k == "max_warps") o.max_warps = std::max(1, std::min(8, std::stoi(v)));
     else if (k == "lane_holes") o.lane_holes = std::max(1, std::stoi(v));
     else if (k == "lane_mode") o.lane_mode = std::max(1, std::min(2, std::stoi(v)));
+    else if (k == "lane_m") o.lane_m = std::max(1, std::min(2, std::stoi(v)));
     else if (k == "lane_k") o.lane_k = std::stoi(v) >= 4 ? 4 : std::stoi(v) >= 2 ? 2 : 1;
     else if (k == "banks") o.banks = std::stoi(v);
     else if (k == "synth") o.synth = std::stoi(v);
@@ -1498,7 +1500,8 @@ struct Mapper {
     // one LDS/STS of K interleaved groups moves 4K bytes per lane: a wavefront
     // (128 bytes) serves kHalf = 32/K lanes, conflict-free when their words
     // differ mod kHalf
-    const uint32_t kStep = GEM_LANE2_STEP, kHalf = 32u / (uint32_t)opt.lane_k, kGroups = kStep / kHalf;
+    const uint32_t kStep = GEM_LANE2_STEP * (uint32_t)opt.lane_m, kHalf = 32u / (uint32_t)opt.lane_k,
+                   kGroups = kStep / kHalf;
     // sources: port-list order (sorted by global bit: a warp's port loads stay coalesced)
     std::vector<uint32_t> srcs;
     for (uint32_t i = 1; i < n; i++)
@@ -1626,6 +1629,7 @@ struct Mapper {
     pr[LPH_MAGIC] = GEM_LANE2_MAGIC;
     pr[LPH_N_LAYERS] = S;
     pr[LPH_N_OPS] = n_ops;
+    pr[LPH_OPS_PER_THREAD] = (uint32_t)opt.lane_m;
     pr[LPH_N_OUT] = (uint32_t)P.outs.size() * 32;
     pr[LPH_N_RAM] = (uint32_t)P.rams.size();
     pr[LPH_OFF_CHUNKS] = (uint32_t)pr.size();

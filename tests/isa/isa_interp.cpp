@@ -214,10 +214,11 @@ int run_lane_part(Interp& I, LaneSim& Ls, uint32_t p, const uint32_t* pi_lane /*
     // of its reads (and must not be read within the step)
     std::vector<std::pair<uint32_t, uint32_t>> wr;
     std::vector<uint8_t> written(S.size(), 0);
+    const uint32_t M = pr[LPH_OPS_PER_THREAD] ? pr[LPH_OPS_PER_THREAD] : 1u;
     for (uint32_t st = 0; st < pr[LPH_N_LAYERS]; st++) {
       wr.clear();
-      const uint32_t* ops = L + (size_t)st * GEM_LANE2_STEP * 2;
-      for (uint32_t t = 0; t < GEM_LANE2_STEP; t++) {
+      const uint32_t* ops = L + (size_t)st * GEM_LANE2_STEP * M * 2;
+      for (uint32_t t = 0; t < GEM_LANE2_STEP * M; t++) {
         const uint32_t x = ops[2 * t], y = ops[2 * t + 1];
         if (!y) continue;
         const uint32_t a = x & 0x3FFFu, b = (x >> 16) & 0x3FFFu;
@@ -229,7 +230,7 @@ int run_lane_part(Interp& I, LaneSim& Ls, uint32_t p, const uint32_t* pi_lane /*
         if (written[e.first] == 1 + (st & 1) ) { g_err = "lane2 destination written twice in a step"; return -1; }
         written[e.first] = (uint8_t)(1 + (st & 1));
       }
-      for (uint32_t t = 0; t < GEM_LANE2_STEP; t++) {
+      for (uint32_t t = 0; t < GEM_LANE2_STEP * M; t++) {
         const uint32_t x = ops[2 * t];
         if (!ops[2 * t + 1]) continue;
         if (written[x & 0x3FFFu] == 1 + (st & 1) || written[(x >> 16) & 0x3FFFu] == 1 + (st & 1)) {

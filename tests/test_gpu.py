@@ -211,11 +211,14 @@ def test_c5_ragged_stream_groups(gem):
 
 
 @pytest.mark.parametrize("opts,dyn", [("parts=5 stages=2 lanes=1", "1"), ("parts=4 lanes=1", "0"),
-                                      ("parts=4 lanes=1", "1")])
+                                      ("parts=4 lanes=1", "1"), ("parts=4 lanes=1 lane_m=2", "1"),
+                                      ("parts=4 lanes=1 lane_mode=1", "1")])
 def test_lane_mode_stages_and_work_distribution(gem, monkeypatch, tmp_path, opts, dyn):
     """Lane mode with two stages (static work lists, cut words between stages)
     and one stage with static (GEM_F_STATIC_LANES) or dynamic ticketed work
-    distribution: 96 streams match the 64-lane oracle bit-exactly."""
+    distribution, LAN2 programs with 1 or 2 ops per thread and step, and the
+    round-1 boomerang lane programs ("LANE"): 96 streams match the 64-lane
+    oracle bit-exactly."""
     from paper_conf_dac_guozwlr25_b200.mapping import compile_file
     S, T = 96, 50
     net = circuits.small_G(seed=41, n_and=4000, with_ram=True)
