@@ -43,3 +43,21 @@ def test_workload_inputs_seeded_per_stream_and_step():
     assert (a[:, :4, 0] & 1).all()                 # reset asserted for the first 4 cycles of step 0
     assert not (c[:, :, 0] & 1).any()              # and released afterwards
     assert not (a[:, :, 2] >> 6).any()             # bits above n_pi stay zero
+
+
+def test_gpus_flag_launches_ranks_or_fails_loudly():
+    """`bench.py --gpus N` outside torchrun relaunches itself with N ranks; with
+    fewer than N visible GPUs it exits non-zero with a message (never a silent
+    1-GPU run reporting n_gpus = 1)."""
+    import os
+    import subprocess
+    import sys
+    import torch
+    if torch.cuda.device_count() >= 2:
+        import pytest
+        pytest.skip("needs a host with fewer than 2 GPUs")
+    env = {k: v for k, v in os.environ.items() if k not in ("WORLD_SIZE", "RANK", "LOCAL_RANK")}
+    r = subprocess.run([sys.executable, bench.__file__, "--gpus", "2"], capture_output=True, text=True, env=env,
+                       timeout=300)
+    assert r.returncode == 2, (r.returncode, r.stderr[-500:])
+    assert "--gpus 2" in r.stderr and "CUDA device" in r.stderr
