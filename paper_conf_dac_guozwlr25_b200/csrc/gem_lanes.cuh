@@ -9,12 +9,13 @@
 // XA/XB/OB the slot's constants sign-extended to masks.  The program
 // (gem_isa.h "Lane mode") comes from the same placement as the bit-packed one.
 
-// lane global-state indexing, group-major rows (a work item's signals are
-// contiguous): X[buf][group][bit]
+// lane global-state indexing, group-minor: X[row][bit][group] (row = buffer
+// parity or cycle).  The K groups of a work item are adjacent words, so a port
+// load or an endpoint store of all K groups is one 16-byte access for K = 4.
 struct LaneIdx {
   uint32_t G;
   __device__ __forceinline__ size_t q(uint32_t buf, uint32_t bits, uint32_t b, uint32_t g) const {
-    return ((size_t)buf * G + g) * bits + b;
+    return ((size_t)buf * bits + b) * G + g;
   }
 };
 
@@ -276,7 +277,7 @@ __device__ __forceinline__ void lane_ports(const KParams& kp, uint32_t s_base, c
 #pragma unroll
         for (int j = 0; j < K; j++) {
           const uint32_t* base = reg == GEM_R_PI ? bpi[j] : reg == GEM_R_Q ? bq[j] : reg == GEM_R_RD ? brd[j] : bcut[j];
-          v[j][4 * u + h] = ok ? __ldcg(base + b) : 0u;
+          v[j][4 * u + h] = ok ? __ldcg(base + (size_t)b * X.G) : 0u;
         }
       }
     }
@@ -323,13 +324,19 @@ __device__ __forceinline__ void lane_commit(const KParams& kp, uint32_t s_base, 
       ldsK<K>(s_base + 4u * K * (e[u].y & 0xFFFFu), v);
       const uint32_t inv = (e[u].y >> 31) ? 0xFFFFFFFFu : 0u;
       const uint32_t reg = e[u].x >> 24, b = e[u].x & 0xFFFFFFu;
+      uint32_t* dst = reg == GEM_R_Q ? kp.q + X.q(nxt, kp.q_words * 32, b, g0)
+                    : reg == GEM_R_PO ? kp.po_lane + X.q(c, kp.po_words * 32, b, g0)
+                    : reg == GEM_R_CUT ? kp.cut + X.q(0, kp.cut_words * 32, b, g0) : nullptr;
+      if (dst && K == 4 && ng == 4 && (X.G & 3u) == 0 && (g0 & 3u) == 0) {
+        // the item's 4 groups are one 16-byte word of the group-minor layout
+        __stcg(reinterpret_cast<uint4*>(dst), make_uint4(v[0] ^ inv, v[1 % K] ^ inv, v[2 % K] ^ inv, v[3 % K] ^ inv));
+        continue;
+      }
 #pragma unroll
       for (int j = 0; j < K; j++) {
         if ((uint32_t)j >= ng) break;
-        const uint32_t g = g0 + j, x = v[j] ^ inv;
-        if (reg == GEM_R_Q) __stcg(kp.q + X.q(nxt, kp.q_words * 32, b, g), x);
-        else if (reg == GEM_R_PO) __stcg(kp.po_lane + X.q(c, kp.po_words * 32, b, g), x);
-        else if (reg == GEM_R_CUT) __stcg(kp.cut + X.q(0, kp.cut_words * 32, b, g), x);
+        const uint32_t x = v[j] ^ inv;
+        if (dst) __stcg(dst + j, x);
         else ramp[j * kp.ramp_words + b] = x;
       }
     }
@@ -435,18 +442,13 @@ __device__ __forceinline__ void lane_ports2(const KParams& kp, uint32_t s_base, 
                                             uint32_t n_gread, uint32_t g0, uint32_t ng, uint32_t c, uint32_t cur) {
   const uint32_t tid = threadIdx.x;
   const LaneIdx X{kp.n_groups};
-  const uint32_t* bpi[K];
-  const uint32_t* bq[K];
-  const uint32_t* brd[K];
-  const uint32_t* bcut[K];
-#pragma unroll
-  for (int j = 0; j < K; j++) {
-    const uint32_t g = g0 + min((uint32_t)j, ng - 1u);
-    bpi[j] = kp.pi_lane + X.q(kp.in_base + c, kp.pi_words * 32, 0, g);
-    bq[j] = kp.q + X.q(cur, kp.q_words * 32, 0, g);
-    brd[j] = kp.rd + X.q(cur, kp.n_rams * 32, 0, g);
-    bcut[j] = kp.cut + X.q(0, kp.cut_words * 32, 0, g);
-  }
+  // row bases of group 0 (X[row][bit][group]); a value is row + bit * G + group
+  const uint32_t* rpi = kp.pi_lane + X.q(kp.in_base + c, kp.pi_words * 32, 0, 0);
+  const uint32_t* rq = kp.q + X.q(cur, kp.q_words * 32, 0, 0);
+  const uint32_t* rrd = kp.rd + X.q(cur, kp.n_rams * 32, 0, 0);
+  const uint32_t* rcut = kp.cut;
+  // K = 4 groups of an aligned item are one 16-byte word
+  const bool vec = K == 4 && ng == 4 && (X.G & 3u) == 0 && (g0 & 3u) == 0;
   constexpr uint32_t U = K >= 4 ? 4u : 8u / K;   // entries per thread per pass (U * K loads in flight; 8 for K = 4 measured slower)
   for (uint32_t kb = 0; kb < n_gread; kb += U * GEM_THREADS) {
     uint32_t e[U];
@@ -459,10 +461,17 @@ __device__ __forceinline__ void lane_ports2(const KParams& kp, uint32_t s_base, 
 #pragma unroll
     for (uint32_t u = 0; u < U; u++) {
       const uint32_t reg = e[u] >> 24, b = e[u] & 0xFFFFFFu;
+      const uint32_t* row = reg == GEM_R_PI ? rpi : reg == GEM_R_Q ? rq : reg == GEM_R_RD ? rrd : rcut;
+      const uint32_t* a = row + (size_t)b * X.G + g0;
+      if (e[u] == 0xFFFFFFFFu) {
 #pragma unroll
-      for (int j = 0; j < K; j++) {
-        const uint32_t* base = reg == GEM_R_PI ? bpi[j] : reg == GEM_R_Q ? bq[j] : reg == GEM_R_RD ? brd[j] : bcut[j];
-        v[u][j] = e[u] != 0xFFFFFFFFu ? __ldcg(base + b) : 0u;
+        for (int j = 0; j < K; j++) v[u][j] = 0u;
+      } else if (vec) {
+        const uint4 w4 = __ldcg(reinterpret_cast<const uint4*>(a));
+        v[u][0] = w4.x; v[u][1 % K] = w4.y; v[u][2 % K] = w4.z; v[u][3 % K] = w4.w;
+      } else {
+#pragma unroll
+        for (int j = 0; j < K; j++) v[u][j] = __ldcg(a + min((uint32_t)j, ng - 1u));
       }
     }
 #pragma unroll
@@ -647,7 +656,7 @@ __global__ void __launch_bounds__(GEM_THREADS, (V2 && K <= 2) ? 4 : 2) gem_lane_
 __global__ void to_lanes_kernel(const uint32_t* __restrict__ in, uint32_t* __restrict__ out, uint32_t n_streams,
                                 uint32_t rows, uint32_t words, uint64_t s_stride, uint64_t r_stride,
                                 uint32_t n_groups, uint64_t out_row_base) {
-  // out[out_row_base + row][g][w*32 + k] = bit k of word w, lane s of group g
+  // out[out_row_base + row][w*32 + k][g] = bit k of word w, lane s of group g
   const uint32_t lane = threadIdx.x & 31;
   const uint64_t warps = (uint64_t)rows * n_groups * words;
   for (uint64_t wi = ((uint64_t)blockIdx.x * blockDim.x + threadIdx.x) >> 5; wi < warps;
@@ -663,7 +672,7 @@ __global__ void to_lanes_kernel(const uint32_t* __restrict__ in, uint32_t* __res
       const uint32_t b = __ballot_sync(0xFFFFFFFFu, (x >> k) & 1u);
       if (lane == k) mine = b;
     }
-    out[((out_row_base + row) * n_groups + g) * words * 32 + w * 32 + lane] = mine;
+    out[((out_row_base + row) * words * 32 + w * 32 + lane) * n_groups + g] = mine;   // X[row][bit][group]
   }
 }
 
@@ -678,7 +687,7 @@ __global__ void from_lanes_kernel(const uint32_t* __restrict__ in, uint32_t* __r
     const uint32_t w = (uint32_t)(wi % words);
     const uint32_t g = (uint32_t)((wi / words) % n_groups);
     const uint64_t row = wi / ((uint64_t)words * n_groups);
-    const uint32_t y = in[(row * n_groups + g) * words * 32 + w * 32 + lane];
+    const uint32_t y = in[(row * words * 32 + w * 32 + lane) * n_groups + g];   // X[row][bit][group]
     uint32_t mine = 0;
 #pragma unroll
     for (uint32_t s = 0; s < 32; s++) {

@@ -1609,7 +1609,7 @@ static int load_impl(gem_sim* sim, const uint32_t* w, size_t nw, const gem_confi
     std::vector<uint32_t> q0(2 * qb * G, 0);
     for (size_t b = 0; b < qb; b++)
       if ((finit[b / 32] >> (b % 32)) & 1u)
-        for (size_t g = 0; g < G; g++) q0[g * qb + b] = 0xFFFFFFFFu;
+        for (size_t g = 0; g < G; g++) q0[b * G + g] = 0xFFFFFFFFu;   // X[buf 0][bit][group]
     CK(cudaMemcpy(sim->d_q, q0.data(), q0.size() * 4, cudaMemcpyHostToDevice));
     CK(cudaMemset(sim->d_rd, 0, 2 * (size_t)std::max<uint32_t>(sim->n_rams, 1) * 32 * G * 4));
     CK(cudaMemset(sim->d_cut, 0, (size_t)std::max<uint32_t>(sim->cut_words, 1) * 32 * G * 4));
