@@ -449,7 +449,7 @@ __device__ __forceinline__ void lane_ports2(const KParams& kp, uint32_t s_base, 
   const uint32_t* rcut = kp.cut;
   // K = 4 groups of an aligned item are one 16-byte word
   const bool vec = K == 4 && ng == 4 && (X.G & 3u) == 0 && (g0 & 3u) == 0;
-  constexpr uint32_t U = K >= 4 ? 4u : 8u / K;   // entries per thread per pass (U * K loads in flight; 8 for K = 4 measured slower)
+  constexpr uint32_t U = K >= 4 ? 8u : 8u / K;   // entries per thread per pass (U * K loads in flight)
   for (uint32_t kb = 0; kb < n_gread; kb += U * GEM_THREADS) {
     uint32_t e[U];
 #pragma unroll
@@ -508,7 +508,7 @@ __device__ void run_lane_partition2(const KParams& kp, uint32_t* S, uint32_t* ra
   const uint32_t off_out = h2.x, off_ram = h2.y;
   const uint2* ops = reinterpret_cast<const uint2*>(gprog + off_ops) + tid;
   // the first steps' ops: independent of S, their latency overlaps the port loads
-  constexpr uint32_t kPre = M == 1 ? 6 : 4;
+  constexpr uint32_t kPre = M == 1 ? 8 : 4;
   uint2 q[kPre][M];
 #pragma unroll
   for (uint32_t i = 0; i < kPre; i++)
