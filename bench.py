@@ -603,6 +603,19 @@ def roofline(res, peaks, dev):
     return roof
 
 
+def host_info() -> dict:
+    """The box's host CPU (oracle timings name their cores)."""
+    model = None
+    try:
+        for ln in open("/proc/cpuinfo"):
+            if ln.startswith("model name"):
+                model = ln.split(":", 1)[1].strip()
+                break
+    except OSError:
+        pass
+    return {"nproc": os.cpu_count(), "cpu": model}
+
+
 def mapping_stats(info) -> dict:
     """SURVEY §8(d) mapping fields of the bench line."""
     return {"n_and": info.n_and, "n_and_mapped": info.n_and_mapped, "n_flops": info.n_flops,
@@ -700,6 +713,9 @@ def main():
                 "timed_region": "per step: input staging (D2D copy of the step's PI words"
                                 + (" + lane transpose" if lanes else "") + "), gem_step, PO unpermute",
                 "e2e": main_res.get("e2e"), "roofline": roof, "parity": main_res.get("parity"),
+                "host": host_info(), "seeds": {"netlist": {"c1": None, "c2": 2, "c3": 3, "c4": 4, "c5": 3}[cfg],
+                                               "stimulus": "splitmix64(base ^ stream << 24 ^ step), base "
+                                                           f"{ {'c1': 1, 'c2': 102, 'c3': 103, 'c4': 104, 'c5': 105}[cfg] }"},
                 "cpu_baseline": cpu, "cpu_baseline_mt": cpu_mt,
                 "step_ms": {"min": min(main_res["step_ms"]), "median": float(np.median(main_res["step_ms"])),
                             "max": max(main_res["step_ms"])}}
