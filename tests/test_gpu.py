@@ -528,3 +528,47 @@ def test_uninitialised_latches_read_zero(gem, tmp_path):
         runs[name] = sim.read_state()
     assert np.array_equal(runs["zero"], runs["uninit"])
     assert Oracle(pu).get_state().sum() == 0 and Oracle(p1).get_state().any()
+
+
+def test_single_cta_local_state_resume_and_preload(gem, tmp_path):
+    """Single-partition designs run the LOC kernel (flops and RAM-read words kept
+    in shared memory across cycles, next cycle's PI words prefetched): state
+    written between steps (gem_write_state, checkpoint/resume) and RAM contents
+    preloaded with gem_write_ram are picked up by the next launch, and ragged
+    steps of 1 cycle work (the prefetch never reads past the queued inputs)."""
+    from paper_conf_dac_guozwlr25_b200.mapping import compile_file
+    # C1: resume from a checkpoint taken after 137 cycles, in a fresh simulator
+    T = 400
+    st = stimulus("c1", 35, T)
+    ref = Oracle(eaig("c1")).run(st, state=True)
+    a = gem.Simulator(blob("c1"))
+    assert a.info["grid"] == 1 and a.info["n_parts"] == 1
+    a.set_inputs(st[:137])
+    a.step(137)
+    q = a.read_state()
+    b = gem.Simulator(blob("c1"), flags=gem.GEM_F_TRACE_STATE)
+    b.write_state(q)
+    po = []
+    for a_, e_ in [(137, 138), (138, 139), (139, 250), (250, T)]:
+        b.set_inputs(st[a_:e_])
+        b.step(e_ - a_)
+        po.append(b.read_outputs(e_ - a_)[0])
+        assert np.array_equal(b.read_state_trace(e_ - a_)[0], ref["state"][a_:e_])
+    assert np.array_equal(np.concatenate(po), ref["po"][137:])
+    # a one-partition RAM design: preloaded contents reach the outputs
+    p = circuits.save(circuits.ram_direct(), str(tmp_path), "ram")
+    o = Oracle(p)
+    rng = np.random.default_rng(4)
+    pre = rng.integers(0, 1 << 32, 8192, dtype=np.uint64).astype(np.uint32)
+    n_pi = o.n_pi
+    s2 = rng.integers(0, 1 << 32, size=(200, (n_pi + 31) // 32), dtype=np.uint64).astype(np.uint32)
+    s2[:, -1] &= (1 << (n_pi % 32)) - 1 if n_pi % 32 else 0xFFFFFFFF
+    sim = gem.Simulator(compile_file(p), flags=gem.GEM_F_DIGEST)
+    assert sim.info["grid"] == 1
+    sim.write_ram(0, pre)
+    o.set_ram(0, pre)
+    r = o.run(s2, digest=True)
+    sim.set_inputs(s2)
+    sim.step(200)
+    assert np.array_equal(sim.read_outputs(200)[0], r["po"])
+    assert np.array_equal(sim.read_ram(0), o.get_ram(0))
