@@ -406,15 +406,19 @@ def parity_check(cfg, path, sim_out, stims, C, state=None):
             "oracle": "single-stream oracle, stream 0 of rank 0"}
 
 
-def run_workload(cfg, args, ws, rank, dev, dist, total_streams, scaling, do_e2e=True):
-    """Time `args.steps` gem_step calls of `cfg` (after `args.warmup`), max over ranks."""
+def run_workload(cfg, args, ws, rank, dev, dist, total_streams, scaling, do_e2e=True, split=False):
+    """Time `args.steps` gem_step calls of `cfg` (after `args.warmup`), max over ranks.
+    split: one stream of one design whose partitions are split over the ws
+    ranks (row f4, gem_dist_*: peer stores + cross-device barrier each cycle)."""
     import torch
     from paper_conf_dac_guozwlr25_b200 import gem
     from paper_conf_dac_guozwlr25_b200.dist import gather_traces, shard_streams
     from paper_conf_dac_guozwlr25_b200.isa import blob_info
     from tests.common import blob, eaig, MAP_OPTS
 
-    s_start, S = shard_streams(total_streams, ws, rank)
+    from paper_conf_dac_guozwlr25_b200.dist import connect_split
+    s_start, S = shard_streams(total_streams, ws, rank) if not split else (0, 1)
+    dkw = {"dist_world": ws, "dist_rank": rank} if split else {}
     opts = MAP_OPTS[cfg] if (args.map_opts is None or cfg != args.workload) else args.map_opts
     if rank == 0:
         b = blob(cfg, opts)
@@ -424,8 +428,11 @@ def run_workload(cfg, args, ws, rank, dev, dist, total_streams, scaling, do_e2e=
         b = blob(cfg, opts)
     info = blob_info(b)
     stream = torch.cuda.current_stream(dev)
-    sim = gem.Simulator(b, device=dev.index, n_streams=S, cuda_stream=stream.cuda_stream, flags=gem.GEM_F_ASYNC)
+    sim = gem.Simulator(b, device=dev.index, n_streams=S, cuda_stream=stream.cuda_stream, flags=gem.GEM_F_ASYNC,
+                        **dkw)
     C = (args.cycles if cfg == args.workload else 0) or {"c4": 200, "c5": 100}.get(cfg, 1000)
+    if split:
+        connect_split(sim, C)
     gstreams = list(range(s_start, s_start + S))
     n_steps = args.warmup + args.steps
     host_in = [workload_inputs(cfg, info.n_pi, C, gstreams, k) for k in range(min(n_steps, 4))]
@@ -477,7 +484,9 @@ def run_workload(cfg, args, ws, rank, dev, dist, total_streams, scaling, do_e2e=
     if not do_e2e:
         return res
     # ---- e2e through the public C ABI with HOST buffers (pinned), copies inside the timed region
-    sim_h = gem.Simulator(b, device=dev.index, n_streams=S)
+    sim_h = gem.Simulator(b, device=dev.index, n_streams=S, **dkw)
+    if split:
+        connect_split(sim_h, C)
     host_pinned = [torch.from_numpy(x.view(np.int32)).pin_memory() for x in host_in]
     # first call from reset on step 0's inputs: the parity sample below
     sim_h.set_inputs(host_pinned[0].numpy().view(np.uint32))
@@ -645,6 +654,8 @@ def main():
     ap.add_argument("--no-batched", action="store_true", help="skip the batched C5 (4096-stream) companion run")
     ap.add_argument("--no-flush", action="store_true")
     ap.add_argument("--map-opts", default=None)
+    ap.add_argument("--split", action="store_true",
+                    help="N>1: split the single design's partitions over the N GPUs (row f4) instead of replicas")
     args = ap.parse_args()
     if args.impl == "reference":
         return run_reference(args)
@@ -658,21 +669,33 @@ def main():
     if ws != args.gpus:
         print(f"bench.py: --gpus {args.gpus} but WORLD_SIZE={ws}", file=sys.stderr)
         return 2
+    one_dev = os.environ.get("GEM_BENCH_ONE_DEVICE") == "1"
+    if one_dev:
+        local = 0
     if not torch.cuda.is_available() or torch.cuda.device_count() < (local + 1):
         print("bench.py: no CUDA device for this rank (there is no CPU fallback)", file=sys.stderr)
         return 2
+    # GEM_BENCH_ONE_DEVICE=1 (tests of the N>1 code paths on a 1-GPU box): every
+    # rank on cuda:0, gloo process group (NCCL refuses two ranks on one device)
     if ws > 1:
         os.environ.setdefault("MASTER_ADDR", "127.0.0.1")
         torch.cuda.set_device(local)
-        dist.init_process_group("nccl", device_id=torch.device("cuda", local))
+        if one_dev:
+            dist.init_process_group("gloo")
+        else:
+            dist.init_process_group("nccl", device_id=torch.device("cuda", local))
     else:
         torch.cuda.set_device(0)
     dev = torch.device("cuda", local if ws > 1 else 0)
 
     cfg = args.workload
-    total = args.streams or (4096 if cfg == "c5" else ws)
-    scaling = "strong" if (args.streams or cfg == "c5") else "weak"
-    main_res = run_workload(cfg, args, ws, rank, dev, dist, total, scaling)
+    split = args.split and ws > 1
+    if split and (cfg == "c5" or args.streams):
+        print("bench.py: --split runs one stream of a single design (c1-c4)", file=sys.stderr)
+        return 2
+    total = 1 if split else (args.streams or (4096 if cfg == "c5" else ws))
+    scaling = "strong" if (args.streams or cfg == "c5" or split) else "weak"
+    main_res = run_workload(cfg, args, ws, rank, dev, dist, total, scaling, split=split)
     batched = None
     if cfg != "c5" and not args.no_batched:
         b = run_workload("c5", args, ws, rank, dev, dist, 4096, "strong", do_e2e=False)
@@ -697,7 +720,10 @@ def main():
                 "mapping": mapping_stats(info),
                 "l2": "flushed between timed steps (512 MB write), device-timed and e2e"
                 if not args.no_flush else "not flushed",
-                "parallelism": (f"streams sharded over {ws} GPU(s), NCCL gather of PO traces"
+                "parallelism": (f"one design split over {ws} GPUs: {info.n_parts} partitions by gem_dist_owner, "
+                                "peer stores of committed words + cross-device barrier per stage (row f4)"
+                                if split else
+                                f"streams sharded over {ws} GPU(s), NCCL gather of PO traces"
                                 if (ws > 1 and total > ws) else
                                 f"{ws} independent replicas (single design: replicas only, DESIGN.md §8)"
                                 if ws > 1 else "1 GPU")}

@@ -88,6 +88,12 @@ typedef struct {
    * (0 = automatic: a share of the L2 for programs larger than half of it;
    * > 0 = that fraction; < 0 = no eviction policy). */
   float l2_evict_last;
+  /* Single-design multi-GPU (§V P:247 future work):
+   * the design's partitions are split over dist_world devices (0 or 1 = one
+   * device), this handle runs those owned by dist_rank (gem_dist_owner).  The
+   * handle stays unusable for gem_step until gem_dist_connect. */
+  uint32_t dist_world;
+  uint32_t dist_rank;
 } gem_config;
 
 typedef struct {
@@ -201,6 +207,58 @@ int gem_read_profile(gem_sim* sim, uint64_t* dst, uint32_t* n_cycles, uint32_t* 
 /* Needs GEM_F_ACTIVITY: partition-cycles evaluated and skipped since load
  * (summed over CTAs eligible for pruning; ineligible CTAs are not counted). */
 int gem_read_activity(gem_sim* sim, uint64_t* evaluated, uint64_t* skipped);
+
+/* ---- Single-design multi-GPU (§V P:247 lists
+ * multi-GPU as future work, so the protocol is this library's).
+ * Every rank loads the same blob with the same n_streams and cfg.dist_world,
+ * its own cfg.dist_rank.  A rank evaluates the partitions it owns; at each
+ * endpoint commit the kernel stores the flop (Q), RAM-read (RD),
+ * cut and PO words into its own buffers AND into every peer's (peer memory
+ * over NVLink / PCIe, or the same device), then meets the other ranks at a
+ * cross-device barrier at every stage boundary, plus once at the start of
+ * each launch: every CTA of every rank stores its arrival epoch into its slot
+ * of every rank's flag array (after a system-scope fence) and polls the
+ * slots of its own array.  So Q, RD, cut and PO words are replicated on every rank (gem_read_*
+ * of states, traces and outputs works on any rank); RAM contents (gem_read_ram
+ * / gem_write_ram) live only on the rank that owns the RAM's partition.
+ * Every rank must call gem_set_inputs with the same stimuli and gem_step with
+ * the same cycle counts, concurrently (each call waits for the others in the
+ * kernel; a rank that never comes trips the 10 s barrier watchdog). */
+#define GEM_DIST_MAX 8
+#define GEM_DIST_IPC_BYTES 328   /* 5 cudaIpcMemHandle_t + grid + reserved */
+typedef struct {
+  void* q;      /* device pointers (as seen by the connecting process) of one */
+  void* rd;     /* rank's replicated buffers and its barrier flags            */
+  void* cut;
+  void* po;
+  void* flags;
+  uint32_t grid;       /* CTAs of that rank's launches (its barrier slots) */
+  uint32_t reserved;
+} gem_dist_buffers;
+
+/* Host-only (no CUDA call): owner rank of each partition for a world of
+ * `world` ranks, written to owner[n_parts]: per stage, partitions in
+ * decreasing mapper cost to the least-loaded rank (ties: less work in the
+ * earlier stages, then the lower rank).
+ * Deterministic, so every rank computes the same split.  Errors: GEM_E_INVAL,
+ * GEM_E_FORMAT (as gem_load_program). */
+int gem_dist_owner(const void* blob, size_t nbytes, uint32_t world, uint32_t* owner);
+
+/* This rank's buffers for its peers.  Fixes the output capacity at
+ * max_cycles (a later gem_step of more cycles per call is GEM_E_INVAL) and
+ * allocates the zeroed barrier flags.  Errors: GEM_E_INVAL (not a dist handle,
+ * max_cycles 0 or > 2^32-16), GEM_E_NOMEM, GEM_E_CUDA. */
+int gem_dist_export(gem_sim* sim, uint64_t max_cycles, gem_dist_buffers* out);
+/* The exported buffers as CUDA IPC handles (GEM_DIST_IPC_BYTES host bytes)
+ * for a peer in another process; call after gem_dist_export. */
+int gem_dist_ipc_handles(gem_sim* sim, void* out);
+/* Maps a peer process's handles into this process (closed by gem_free);
+ * *out receives pointers for gem_dist_connect. */
+int gem_dist_ipc_open(gem_sim* sim, const void* handles, gem_dist_buffers* out);
+/* Peer buffers of every rank (peers[dist_world], peers[dist_rank] ignored;
+ * same-process pointers on another device get peer access enabled).
+ * Errors: GEM_E_INVAL (not exported, null entry), GEM_E_CUDA. */
+int gem_dist_connect(gem_sim* sim, const gem_dist_buffers* peers);
 
 void gem_free(gem_sim* sim);
 const char* gem_last_error(void);

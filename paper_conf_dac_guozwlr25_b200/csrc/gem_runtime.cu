@@ -83,6 +83,20 @@ struct KParams {
   const uint4* __restrict__ dyn_units;
   uint32_t n_units;
   uint32_t* dyn_ctr;
+  // single-design multi-GPU (DIST kernels, include/gem.h gem_dist_*): committed
+  // Q / RD / cut / PO words are also stored into every peer's buffers, and the
+  // grid barrier meets the peers' through system-scope flags (epochs continue
+  // across launches: dist_epoch0 = barriers of earlier launches)
+  uint32_t dist_world, dist_rank;
+  unsigned long long dist_epoch0;
+  unsigned long long* dist_flags;              // this rank's flags [world][GEM_BAR_MAX_CTAS] (x stride)
+  unsigned long long* peer_flags[GEM_DIST_MAX];  // every rank's flags (this rank's = dist_flags)
+  uint32_t dist_grid[GEM_DIST_MAX];            // CTAs of each rank's launch
+  uint32_t dist_slots;                         // sum of dist_grid
+  uint32_t* peer_q[GEM_DIST_MAX];
+  uint32_t* peer_rd[GEM_DIST_MAX];
+  uint32_t* peer_cut[GEM_DIST_MAX];
+  uint32_t* peer_po[GEM_DIST_MAX];
 };
 #define PROF(slot_)                                                                          \
   do {                                                                                       \
@@ -129,7 +143,51 @@ __device__ __forceinline__ void spin_check(uint32_t& spins, uint64_t& start, con
     asm volatile("trap;");
   }
 }
+__device__ __forceinline__ unsigned long long ld_acquire_sys_u64(const unsigned long long* p) {
+  unsigned long long v;
+  asm volatile("ld.acquire.sys.global.u64 %0, [%1];" : "=l"(v) : "l"(p) : "memory");
+  return v;
+}
+// DIST: a committed word to every peer's copy of the same buffer (same offset)
+__device__ __forceinline__ void dist_put(const KParams& kp, uint32_t* const* peers, size_t off, uint32_t v) {
+  for (uint32_t r = 0; r < kp.dist_world; r++)
+    if (r != kp.dist_rank) __stcg(peers[r] + off, v);
+}
+template <bool DIST = false>
 __device__ __forceinline__ void grid_sync(const KParams& kp, unsigned long long& epoch) {
+  if (DIST) {
+    // Cross-device barrier, flat like the single-device one: after bar.sync,
+    // thread 0 makes the CTA's stores (local and peer) visible at system scope
+    // (fence.acq_rel.sys, cumulative over the CTA's writes ordered by the
+    // bar.sync) and stores the epoch into this CTA's slot of EVERY rank's flag
+    // array (slot rank * GEM_BAR_MAX_CTAS + cta; its own included); then
+    // thread f polls slot f of its own array (ld.acquire.sys; all ranks' CTAs).
+    // Epochs continue across launches (the flags are never reset).
+    // Measured on one B200 with in-process ranks (scripts/split_bench.py, C3,
+    // 2 ranks): 14.8 us per cycle vs 10.5 single-rank; the system-scope fence
+    // is 3.4 us of it (a gpu-scope one, not valid across devices: 11.4 us);
+    // a fence in every committing thread, or a two-level gather through CTA 0,
+    // was slower (18-22 us, 19.5 us).
+    __syncthreads();
+    epoch++;
+    const unsigned long long de = kp.dist_epoch0 + epoch;
+    if (threadIdx.x == 0) {
+      asm volatile("fence.acq_rel.sys;" ::: "memory");
+      const size_t slot = ((size_t)kp.dist_rank * GEM_BAR_MAX_CTAS + blockIdx.x) * GEM_BAR_STRIDE;
+      for (uint32_t r = 0; r < kp.dist_world; r++)
+        asm volatile("st.relaxed.sys.global.u64 [%0], %1;" ::"l"(kp.peer_flags[r] + slot), "l"(de) : "memory");
+    }
+    for (uint32_t f = threadIdx.x; f < kp.dist_slots; f += blockDim.x) {
+      uint32_t r = 0, b = f;
+      while (b >= kp.dist_grid[r]) b -= kp.dist_grid[r++];
+      const unsigned long long* fl = kp.dist_flags + ((size_t)r * GEM_BAR_MAX_CTAS + b) * GEM_BAR_STRIDE;
+      uint32_t spins = 0;
+      uint64_t start = 0;
+      while (ld_acquire_sys_u64(fl) < de) spin_check(spins, start, kp, f, de);
+    }
+    __syncthreads();
+    return;
+  }
   __syncthreads();
   if (gridDim.x > 1) {
     epoch++;
@@ -500,7 +558,7 @@ __device__ __forceinline__ void top_layer(uint32_t topc, uint32_t topwo, uint32_
 // the previous cycle, so they come from the shared-memory copy `loc` (no L2
 // round trip), and the PI words of cycle c+1 are loaded into `pv` during
 // cycle c (their latency hides behind the layers).
-template <bool ACT, bool LOC>
+template <bool ACT, bool LOC, bool DIST>
 __device__ void run_partition(const KParams& kp, ProgSrc& ps, uint32_t* S, uint32_t* ramp, uint32_t* topb,
                               uint32_t p, uint32_t st0, uint32_t nst, uint32_t c, uint32_t cur, uint32_t nxt,
                               bool prof_on, uint32_t* act = nullptr, bool act_first = true,
@@ -688,12 +746,21 @@ commit:
       const uint32_t dst = od[o];
       const uint32_t reg = GEM_GID_REGION(dst), idx = GEM_GID_INDEX(dst);
       if (reg == GEM_R_Q) {
-        __stcg(kp.q + ((size_t)nxt * kp.n_streams + st) * kp.q_words + idx, v);
+        const size_t o = ((size_t)nxt * kp.n_streams + st) * kp.q_words + idx;
+        __stcg(kp.q + o, v);
         if (LOC) loc[nxt * kp.loc_words + idx] = v;
+        if (DIST) dist_put(kp, kp.peer_q, o, v);
+      } else if (reg == GEM_R_PO) {
+        const size_t o = ((size_t)st * kp.out_cap + c) * kp.po_words + idx;
+        __stcg(kp.po + o, v);
+        if (DIST) dist_put(kp, kp.peer_po, o, v);
+      } else if (reg == GEM_R_CUT) {
+        const size_t o = (size_t)st * kp.cut_words + idx;
+        __stcg(kp.cut + o, v);
+        if (DIST) dist_put(kp, kp.peer_cut, o, v);
+      } else {
+        ramp[j * 4 * GEM_MAX_RAMS_PER_PART + idx] = v;
       }
-      else if (reg == GEM_R_PO) __stcg(kp.po + ((size_t)st * kp.out_cap + c) * kp.po_words + idx, v);
-      else if (reg == GEM_R_CUT) __stcg(kp.cut + (size_t)st * kp.cut_words + idx, v);
-      else ramp[j * 4 * GEM_MAX_RAMS_PER_PART + idx] = v;
     }
   }
   // ---- a7: RAM blocks (read-first, then per-bit write; readings U7-U10)
@@ -711,8 +778,10 @@ commit:
       const uint32_t old = __ldcg(M + ra);
       const uint32_t cur_w = __ldcg(M + wa);
       __stcg(M + wa, (cur_w & ~be) | (wd & be));
-      __stcg(kp.rd + ((size_t)nxt * kp.n_streams + st) * kp.n_rams + id, old);
+      const size_t o = ((size_t)nxt * kp.n_streams + st) * kp.n_rams + id;
+      __stcg(kp.rd + o, old);
       if (LOC) loc[nxt * kp.loc_words + kp.q_words + id] = old;
+      if (DIST) dist_put(kp, kp.peer_rd, o, old);
     }
   }
   __syncthreads();  // S / ramp / ring slots reused by the next work item
@@ -747,8 +816,10 @@ __device__ void record_state(const KParams& kp, uint32_t c, uint32_t buf) {
   }
 }
 
-// ACT: GEM_F_ACTIVITY build of the kernel (the plain one carries no pruning code)
-template <bool ACT, bool LOC>
+// ACT: GEM_F_ACTIVITY build of the kernel (the plain one carries no pruning code);
+// LOC: single-CTA launch, flops / RAM-read words in shared memory; DIST: one
+// rank of a design split over devices (peer stores + cross-device barrier)
+template <bool ACT, bool LOC, bool DIST>
 __global__ void __launch_bounds__(GEM_THREADS, 2) gem_step_kernel(const KParams kp) {
   extern __shared__ __align__(16) uint32_t smem[];
   // layout (words): S[group][state_words] | area[area_words] | ctab[256] | ramp[group][128] |
@@ -928,6 +999,9 @@ __global__ void __launch_bounds__(GEM_THREADS, 2) gem_step_kernel(const KParams 
                                                   : __ldcg(kp.rd + (size_t)c0 * kp.n_streams * kp.n_rams + (k - kp.q_words));
     __syncthreads();
   }
+  // DIST: no rank stores into a peer's buffers before every rank has started
+  // this launch (a peer may still be reading the previous launch's outputs)
+  if (DIST) grid_sync<true>(kp, bar_target);
   for (uint32_t c = 0; c < kp.ncycles; c++) {
     const uint64_t t = kp.t0 + c;
     const uint32_t cur = (uint32_t)(t & 1u), nxt = cur ^ 1u;
@@ -939,7 +1013,7 @@ __global__ void __launch_bounds__(GEM_THREADS, 2) gem_step_kernel(const KParams 
       for (uint32_t k = kb; k < ke; k++) {
         const uint2 it = wl_item(s, k);
         const uint32_t nst = min(kp.group, kp.n_streams - it.y);
-        run_partition<ACT, LOC>(kp, ps, S, ramp, topb, it.x, it.y, nst, c, cur, nxt, prof_on && k == kb && s == 0,
+        run_partition<ACT, LOC, DIST>(kp, ps, S, ramp, topb, it.x, it.y, nst, c, cur, nxt, prof_on && k == kb && s == 0,
                                 act, c == 0, loc, &pv);
         if (!ps.resident) {
           // prefetch the next work item's prologue (overlaps the grid barrier)
@@ -952,7 +1026,7 @@ __global__ void __launch_bounds__(GEM_THREADS, 2) gem_step_kernel(const KParams 
         }
       }
       if (s == 0) PROF(4);
-      grid_sync(kp, bar_target);
+      grid_sync<DIST>(kp, bar_target);
     }
     PROF(5);
   }
@@ -1102,6 +1176,14 @@ struct gem_sim {
   uint64_t cycle = 0;
   cudaEvent_t ev0 = nullptr, ev1 = nullptr, ev_in = nullptr;
   float last_ms = 0.f;
+  // single-design multi-GPU (gem_dist_*)
+  uint32_t dist_world = 1, dist_rank = 0;
+  std::vector<uint32_t> owner;                 // [n_parts] rank of each partition (dist only)
+  bool dist_exported = false, dist_connected = false;
+  unsigned long long* d_dist_flags = nullptr;  // [GEM_DIST_MAX] slots of GEM_BAR_STRIDE u64
+  unsigned long long dist_epoch = 0;           // cross-device barriers completed by earlier launches
+  gem_dist_buffers peers[GEM_DIST_MAX]{};
+  std::vector<void*> ipc_opened;               // peer buffers mapped by gem_dist_ipc_open
 };
 
 static int fail(int code, const std::string& msg) {
@@ -1143,6 +1225,8 @@ static int ensure_scratch(gem_sim* sim, size_t bytes) {
 
 static int ensure_out(gem_sim* sim, uint32_t ncycles) {
   if (sim->out_cap >= ncycles && sim->d_po) return 0;
+  if (sim->dist_exported)   // peers hold pointers into d_po
+    return fail(GEM_E_INVAL, "more cycles per gem_step than gem_dist_export's max_cycles");
   uint32_t cap = std::max<uint32_t>(ncycles, 16);
   if (sim->d_po) cudaFree(sim->d_po);
   if (sim->d_qtrace) cudaFree(sim->d_qtrace);
@@ -1186,6 +1270,7 @@ static double build_worklists(const gem_sim* sim, uint32_t G, std::vector<uint32
     for (uint32_t st = 0; st < sim->n_streams; st += sim->group * run)
       for (uint32_t k = 0; k < np; k++) {
         const uint32_t p = sim->h_stage[sim->n_stages + 1 + pb + k];
+        if (!sim->owner.empty() && sim->owner[p] != sim->dist_rank) continue;   // another rank's
         const uint32_t nst = std::min(sim->group * run, sim->n_streams - st);
         const uint32_t n_items = (nst + sim->group - 1) / sim->group;
         const double c = sim->h_parts[(size_t)p * GP_WORDS + GP_COST] *
@@ -1227,8 +1312,9 @@ static double build_worklists(const gem_sim* sim, uint32_t G, std::vector<uint32
 }
 
 static const void* step_kernel_for(const gem_sim* sim) {
-  if (sim->act_words) return (const void*)gem_step_kernel<true, false>;
-  return sim->local ? (const void*)gem_step_kernel<false, true> : (const void*)gem_step_kernel<false, false>;
+  if (sim->dist_world > 1) return (const void*)gem_step_kernel<false, false, true>;
+  if (sim->act_words) return (const void*)gem_step_kernel<true, false, false>;
+  return sim->local ? (const void*)gem_step_kernel<false, true, false> : (const void*)gem_step_kernel<false, false, false>;
 }
 
 // Choose CTAs per SM, grid, work lists and the shared-memory program mode.
@@ -1256,14 +1342,20 @@ static int plan_launch(gem_sim* sim, uint32_t max_chunk_words, uint32_t grid_lim
     sim->group = g;
   }
   sim->max_items = 0;
-  for (uint32_t s = 0; s < sim->n_stages; s++)
-    sim->max_items = std::max(sim->max_items, (sim->h_stage[s + 1] - sim->h_stage[s]) *
-                                                  ((sim->n_streams + sim->group - 1) / sim->group));
+  for (uint32_t s = 0; s < sim->n_stages; s++) {
+    uint32_t np = sim->h_stage[s + 1] - sim->h_stage[s];
+    if (!sim->owner.empty()) {   // dist: this rank's partitions only
+      np = 0;
+      for (uint32_t k = sim->h_stage[s]; k < sim->h_stage[s + 1]; k++)
+        np += sim->owner[sim->h_stage[sim->n_stages + 1 + k]] == sim->dist_rank;
+    }
+    sim->max_items = std::max(sim->max_items, np * ((sim->n_streams + sim->group - 1) / sim->group));
+  }
   if (sim->group != 1) sim->act_words = 0;   // activity pruning needs one stream per work item
   // one partition, one stream, one stage: a single CTA owns every flop and RAM,
   // so the LOC kernel keeps them in shared memory across cycles
   sim->loc_words = sim->q_words_int + sim->n_rams;
-  sim->local = sim->n_parts == 1 && sim->n_streams == 1 && sim->n_stages == 1 && !sim->act_words &&
+  sim->local = sim->dist_world == 1 && sim->n_parts == 1 && sim->n_streams == 1 && sim->n_stages == 1 && !sim->act_words &&
                sim->max_gread <= 4 * GEM_THREADS && sim->loc_words <= 4096 && !sim->cfg.grid_limit;
   const uint32_t fixed_words = sim->group * (sim->state_words + 4 * GEM_MAX_RAMS_PER_PART + 16) + GEM_MAX_CHUNKS +
                                48 + GEM_WL_CACHE_WORDS + 32 + sim->act_words + (sim->local ? 2 * sim->loc_words : 0u);
@@ -1507,11 +1599,41 @@ static int validate_blob(const uint32_t* w, size_t nw) {
 }
 
 // gem_load_program body; on failure the caller frees the partially built handle.
+// Partition -> rank split of a design over `world` devices (gem_dist_owner):
+// per stage (stages are separated by barriers, so each is balanced on its
+// own), partitions in decreasing mapper cost go to the least-loaded rank
+// (ties: the rank with less work over the earlier stages, then the lower rank).
+static void dist_assign(const uint32_t* parts, const uint32_t* stages, uint32_t n_stages, uint32_t world,
+                        uint32_t* owner) {
+  std::vector<uint64_t> total(world, 0);
+  for (uint32_t s = 0; s < n_stages; s++) {
+    std::vector<std::pair<uint32_t, uint32_t>> ps;   // (cost, partition)
+    for (uint32_t k = stages[s]; k < stages[s + 1]; k++) {
+      const uint32_t p = stages[n_stages + 1 + k];
+      ps.push_back({parts[(size_t)p * GP_WORDS + GP_COST], p});
+    }
+    std::stable_sort(ps.begin(), ps.end(), [](const std::pair<uint32_t, uint32_t>& a,
+                                              const std::pair<uint32_t, uint32_t>& b) { return a.first > b.first; });
+    std::vector<uint64_t> load(world, 0);
+    for (auto& x : ps) {
+      uint32_t r = 0;
+      for (uint32_t q = 1; q < world; q++)
+        if (load[q] < load[r] || (load[q] == load[r] && total[q] < total[r])) r = q;
+      owner[x.second] = r;
+      load[r] += std::max<uint32_t>(x.first, 1);
+    }
+    for (uint32_t q = 0; q < world; q++) total[q] += load[q];
+  }
+}
+
 static int load_impl(gem_sim* sim, const uint32_t* w, size_t nw, const gem_config* cfg) {
   sim->device = cfg->device;
   sim->cfg = *cfg;
   sim->flags = cfg->flags;
   sim->n_streams = cfg->n_streams;
+  sim->dist_world = std::max<uint32_t>(1, cfg->dist_world);
+  sim->dist_rank = cfg->dist_rank;
+  if (sim->dist_world > 1) sim->flags &= ~GEM_F_ACTIVITY;   // the DIST kernel has no pruning build
   CK(cudaSetDevice(sim->device));
   const uint64_t prog_words = w[GH_PROG_WORDS_LO] | ((uint64_t)w[GH_PROG_WORDS_HI] << 32);
   sim->n_pi = w[GH_N_PI]; sim->n_po = w[GH_N_PO]; sim->n_flops = w[GH_N_FLOPS]; sim->n_rams = w[GH_N_RAMS];
@@ -1535,7 +1657,7 @@ static int load_impl(gem_sim* sim, const uint32_t* w, size_t nw, const gem_confi
     sim->max_items = std::max(sim->max_items, (stages[s + 1] - stages[s]) * sim->n_streams);
   for (uint32_t p = 0; p < sim->n_parts; p++) {
     const uint32_t* pr = w + w[GH_OFF_PROG] + parts[p * GP_WORDS + GP_PROG_OFF];
-    if (cfg->flags & GEM_F_ACTIVITY) sim->act_words = std::max(sim->act_words, (pr[PH_N_GREAD] + 3u) & ~3u);
+    if (sim->flags & GEM_F_ACTIVITY) sim->act_words = std::max(sim->act_words, (pr[PH_N_GREAD] + 3u) & ~3u);
     sim->max_gread = std::max(sim->max_gread, pr[PH_N_GREAD]);
   }
   // inverse permutation tables
@@ -1555,7 +1677,8 @@ static int load_impl(gem_sim* sim, const uint32_t* w, size_t nw, const gem_confi
   std::memset(sim->h_err, 0, 64);
   CK(cudaHostGetDevicePointer((void**)&sim->d_err, sim->h_err, 0));
   // lane mode: >= 32 streams and lane programs present (GEM_F_NO_LANES disables)
-  sim->lanes = (w[GH_HAS_LANES] && cfg->n_streams >= 32 && !(cfg->flags & GEM_F_NO_LANES)) ? 1u : 0u;
+  sim->lanes = (w[GH_HAS_LANES] && cfg->n_streams >= 32 && !(cfg->flags & GEM_F_NO_LANES) && sim->dist_world == 1)
+                   ? 1u : 0u;
   if (sim->lanes) {
     sim->n_groups = (cfg->n_streams + 31) / 32;
     sim->lane_words = (std::max<uint32_t>(w[GH_LANE_MAX_WORDS], 4) + 3) & ~3u;
@@ -1625,6 +1748,10 @@ static int load_impl(gem_sim* sim, const uint32_t* w, size_t nw, const gem_confi
   // persistent co-resident grid + shared-memory program placement
   sim->h_parts.assign(parts, parts + (size_t)sim->n_parts * GP_WORDS);
   sim->h_stage.assign(stages, stages + stage_words);
+  if (sim->dist_world > 1) {
+    sim->owner.assign(sim->n_parts, 0);
+    dist_assign(parts, stages, sim->n_stages, sim->dist_world, sim->owner.data());
+  }
   if (sim->lanes) {
     if (int r = plan_launch_lanes(sim, cfg->grid_limit)) return r;
   } else if (int r = plan_launch(sim, w[GH_MAX_CHUNK_WORDS], cfg->grid_limit)) {
@@ -1645,6 +1772,8 @@ int gem_load_program(const void* blob, size_t nbytes, const gem_config* cfg, gem
   const uint64_t total_words = w[GH_TOTAL_WORDS_LO] | ((uint64_t)w[GH_TOTAL_WORDS_HI] << 32);
   if (total_words != nw) return fail(GEM_E_FORMAT, "truncated blob");
   if (cfg->n_streams == 0) return fail(GEM_E_INVAL, "n_streams must be >= 1");
+  if (cfg->dist_world > GEM_DIST_MAX || (cfg->dist_world > 1 && cfg->dist_rank >= cfg->dist_world))
+    return fail(GEM_E_INVAL, "bad dist_world / dist_rank");
   if (w[GH_MAX_STATE_WORDS] > GEM_MAX_STATE_WORDS) return fail(GEM_E_FORMAT, "state too large");
   if (int r = validate_blob(w, nw)) return r;
   int ndev = 0;
@@ -1723,6 +1852,7 @@ int gem_step(gem_sim* sim, uint64_t ncycles) {
   if (ncycles > (uint64_t)(sim->in_queued - sim->in_head))
     return fail(GEM_E_NOINPUT, "gem_step: not enough queued input cycles");
   CK(cudaSetDevice(sim->device));
+  if (sim->dist_world > 1 && !sim->dist_connected) return fail(GEM_E_INVAL, "dist handle: gem_dist_connect first");
   if (int r = ensure_out(sim, (uint32_t)ncycles)) return r;
   KParams kp;
   std::memset(&kp, 0, sizeof(kp));
@@ -1759,6 +1889,24 @@ int gem_step(gem_sim* sim, uint64_t ncycles) {
   if (sim->d_dyn_ctr) CK(cudaMemsetAsync(sim->d_dyn_ctr, 0, 16, sim->stream));
   kp.act_words = sim->lanes ? 0u : sim->act_words;
   kp.loc_words = sim->local ? sim->loc_words : 0u;
+  if (sim->dist_world > 1) {
+    kp.dist_world = sim->dist_world;
+    kp.dist_rank = sim->dist_rank;
+    kp.dist_epoch0 = sim->dist_epoch;
+    kp.dist_flags = sim->d_dist_flags;
+    kp.dist_slots = 0;
+    for (uint32_t r = 0; r < sim->dist_world; r++) {
+      kp.dist_grid[r] = sim->peers[r].grid;
+      kp.dist_slots += sim->peers[r].grid;
+      if (r == sim->dist_rank) continue;   // (dist_put skips the own rank)
+      kp.peer_q[r] = (uint32_t*)sim->peers[r].q;
+      kp.peer_rd[r] = (uint32_t*)sim->peers[r].rd;
+      kp.peer_cut[r] = (uint32_t*)sim->peers[r].cut;
+      kp.peer_po[r] = (uint32_t*)sim->peers[r].po;
+    }
+    for (uint32_t r = 0; r < sim->dist_world; r++) kp.peer_flags[r] = (unsigned long long*)sim->peers[r].flags;
+    sim->dist_epoch += 1 + (unsigned long long)ncycles * sim->n_stages;   // entry + one per stage and cycle
+  }
   if (sim->flags & GEM_F_PROFILE) {
     const uint32_t pc = (uint32_t)std::min<uint64_t>(ncycles, 256);
     if (!sim->d_prof || sim->prof_cycles < pc) {
@@ -1998,6 +2146,101 @@ int gem_read_activity(gem_sim* sim, uint64_t* evaluated, uint64_t* skipped) {
   return GEM_OK;
 }
 
+int gem_dist_owner(const void* blob, size_t nbytes, uint32_t world, uint32_t* owner) {
+  if (!blob || !owner || world == 0 || world > GEM_DIST_MAX || nbytes < GH_N_WORDS * 4 || (nbytes & 3))
+    return fail(GEM_E_INVAL, "bad arguments");
+  const uint32_t* w = (const uint32_t*)blob;
+  const size_t nw = nbytes / 4;
+  if (w[GH_MAGIC] != GEM_MAGIC || w[GH_VERSION] != GEM_VERSION) return fail(GEM_E_FORMAT, "bad blob magic/version");
+  const uint64_t total_words = w[GH_TOTAL_WORDS_LO] | ((uint64_t)w[GH_TOTAL_WORDS_HI] << 32);
+  if (total_words != nw) return fail(GEM_E_FORMAT, "truncated blob");
+  if (int r = validate_blob(w, nw)) return r;
+  dist_assign(w + w[GH_OFF_PARTS], w + w[GH_OFF_STAGES], w[GH_N_STAGES], world, owner);
+  return GEM_OK;
+}
+
+int gem_dist_export(gem_sim* sim, uint64_t max_cycles, gem_dist_buffers* out) {
+  if (int r = check(sim)) return r;
+  if (!out || sim->dist_world < 2) return fail(GEM_E_INVAL, "not a dist handle (gem_config::dist_world < 2)");
+  if (max_cycles == 0 || max_cycles > 0xFFFFFFF0ull) return fail(GEM_E_INVAL, "bad max_cycles");
+  CK(cudaSetDevice(sim->device));
+  if (!sim->dist_exported) {
+    if (int r = ensure_out(sim, (uint32_t)max_cycles)) return r;
+    const size_t fb = (size_t)GEM_DIST_MAX * GEM_BAR_MAX_CTAS * GEM_BAR_STRIDE * 8;
+    CK(dalloc(&sim->d_dist_flags, fb));
+    CK(cudaMemset(sim->d_dist_flags, 0, fb));
+    CK(cudaDeviceSynchronize());
+    sim->dist_exported = true;
+  } else if (max_cycles > sim->out_cap) {
+    return fail(GEM_E_INVAL, "already exported with a smaller max_cycles");
+  }
+  out->q = sim->d_q; out->rd = sim->d_rd; out->cut = sim->d_cut; out->po = sim->d_po; out->flags = sim->d_dist_flags;
+  out->grid = sim->grid;
+  out->reserved = 0;
+  return GEM_OK;
+}
+
+int gem_dist_ipc_handles(gem_sim* sim, void* out) {
+  if (int r = check(sim)) return r;
+  if (!out || !sim->dist_exported) return fail(GEM_E_INVAL, "gem_dist_export first");
+  CK(cudaSetDevice(sim->device));
+  cudaIpcMemHandle_t h[5];
+  void* ptrs[5] = {sim->d_q, sim->d_rd, sim->d_cut, sim->d_po, sim->d_dist_flags};
+  for (int k = 0; k < 5; k++) CK(cudaIpcGetMemHandle(&h[k], ptrs[k]));
+  static_assert(sizeof(h) + 8 == GEM_DIST_IPC_BYTES, "IPC handle size");
+  const uint32_t tail[2] = {sim->grid, 0u};
+  std::memcpy(out, h, sizeof(h));
+  std::memcpy((char*)out + sizeof(h), tail, 8);
+  return GEM_OK;
+}
+
+int gem_dist_ipc_open(gem_sim* sim, const void* handles, gem_dist_buffers* out) {
+  if (int r = check(sim)) return r;
+  if (!handles || !out) return fail(GEM_E_INVAL, "null argument");
+  CK(cudaSetDevice(sim->device));
+  cudaIpcMemHandle_t h[5];
+  std::memcpy(h, handles, sizeof(h));
+  uint32_t tail[2];
+  std::memcpy(tail, (const char*)handles + sizeof(h), 8);
+  void* p[5] = {};
+  for (int k = 0; k < 5; k++) {
+    CK(cudaIpcOpenMemHandle(&p[k], h[k], cudaIpcMemLazyEnablePeerAccess));
+    sim->ipc_opened.push_back(p[k]);
+  }
+  out->q = p[0]; out->rd = p[1]; out->cut = p[2]; out->po = p[3]; out->flags = p[4];
+  out->grid = tail[0];
+  out->reserved = 0;
+  return GEM_OK;
+}
+
+int gem_dist_connect(gem_sim* sim, const gem_dist_buffers* peers) {
+  if (int r = check(sim)) return r;
+  if (!peers || !sim->dist_exported) return fail(GEM_E_INVAL, "gem_dist_export first");
+  CK(cudaSetDevice(sim->device));
+  for (uint32_t r = 0; r < sim->dist_world; r++) {
+    if (r == sim->dist_rank) {   // this rank's own buffers
+      sim->peers[r] = gem_dist_buffers{sim->d_q, sim->d_rd, sim->d_cut, sim->d_po, sim->d_dist_flags, sim->grid, 0};
+      continue;
+    }
+    const gem_dist_buffers& b = peers[r];
+    if (!b.q || !b.rd || !b.cut || !b.po || !b.flags) return fail(GEM_E_INVAL, "null peer buffer");
+    if (b.grid == 0 || b.grid > GEM_BAR_MAX_CTAS) return fail(GEM_E_INVAL, "bad peer grid");
+    cudaPointerAttributes a{};
+    CK(cudaPointerGetAttributes(&a, b.q));
+    if (a.type == cudaMemoryTypeDevice && a.device != sim->device) {   // same process, another device
+      int can = 0;
+      CK(cudaDeviceCanAccessPeer(&can, sim->device, a.device));
+      if (!can) return fail(GEM_E_UNSUPPORTED, "no peer access between the devices");
+      const cudaError_t e = cudaDeviceEnablePeerAccess(a.device, 0);
+      if (e == cudaErrorPeerAccessAlreadyEnabled) (void)cudaGetLastError();
+      else CK(e);
+    }
+    sim->peers[r] = b;
+  }
+  sim->dist_connected = true;
+  return GEM_OK;
+}
+
 void gem_free(gem_sim* sim) {
   if (!sim) return;
   cudaSetDevice(sim->device);
@@ -2008,8 +2251,9 @@ void gem_free(gem_sim* sim) {
                   (void*)sim->d_scratch, (void*)sim->d_digest, (void*)sim->d_bar,
                   (void*)sim->d_prof, (void*)sim->d_wl_off, (void*)sim->d_wl_items, (void*)sim->d_lprog,
                   (void*)sim->d_pi_lane, (void*)sim->d_po_lane, (void*)sim->d_act,
-                  (void*)sim->d_dyn_units, (void*)sim->d_dyn_ctr})
+                  (void*)sim->d_dyn_units, (void*)sim->d_dyn_ctr, (void*)sim->d_dist_flags})
     if (p) cudaFree(p);
+  for (void* p : sim->ipc_opened) cudaIpcCloseMemHandle(p);
   if (sim->ev0) cudaEventDestroy(sim->ev0);
   if (sim->ev1) cudaEventDestroy(sim->ev1);
   if (sim->ev_in) cudaEventDestroy(sim->ev_in);

@@ -1,10 +1,17 @@
-"""Multi-GPU batched-stimulus plumbing.
+"""Multi-GPU plumbing.
 
-Single designs are replicas only (per-cycle partition exchange stays on one
-GPU, PAPER.md P:247 lists multi-GPU as future work).  Independent stimulus
-streams over the same design shard naturally: rank g simulates streams
-[start_g, start_g + count_g) with no per-cycle communication, and after a
-step the PO traces are gathered to rank 0 over NCCL (NVLink/NVSwitch).
+Batched stimuli: independent stimulus streams over the same
+design shard naturally: rank g simulates streams [start_g, start_g + count_g)
+with no per-cycle communication, and after a step the PO traces are gathered
+to rank 0 over NCCL (NVLink/NVSwitch).
+
+Single design split over devices (PAPER.md P:247 lists
+multi-GPU as future work): every rank loads the same blob with dist_world /
+dist_rank, the kernels exchange the committed words over peer memory and meet
+at a cross-device barrier each stage (include/gem.h gem_dist_*).  This module
+only wires the handles: connect_split exchanges CUDA IPC handles of the ranks'
+buffers over torch.distributed (one process per GPU), connect_local connects
+handles of one process (several devices, or one device in tests).
 
 torch.distributed is plumbing only; the simulation runs in libgem.
 """
@@ -51,3 +58,40 @@ def gather_traces(local: torch.Tensor, total_streams: int, dst: int = 0,
     if rank != dst:
         return None
     return torch.cat([b[:c] for b, c in zip(bufs, counts)], 0)
+
+
+# ---- single design split over devices (gem_dist_*) -------------------------
+def connect_split(sim, max_cycles: int, group: Optional[dist.ProcessGroup] = None):
+    """One process per rank: export this rank's buffers, all-gather their CUDA
+    IPC handles, map every peer's and connect.  Collective over `group`; the
+    rank order of `group` must match the handles' dist_rank."""
+    world = dist.get_world_size(group)
+    rank = dist.get_rank(group)
+    sim.dist_export(max_cycles)
+    mine = sim.dist_ipc_handles()
+    handles: List[Optional[bytes]] = [None] * world
+    dist.all_gather_object(handles, mine, group=group)
+    peers = [None if r == rank else sim.dist_ipc_open(handles[r]) for r in range(world)]
+    sim.dist_connect(peers)
+    dist.barrier(group=group)   # nobody steps before every rank is connected
+    return peers
+
+
+def connect_local(sims, max_cycles: int):
+    """Handles of one process (sims[r] = rank r): export all, connect each."""
+    bufs = [s.dist_export(max_cycles) for s in sims]
+    for s in sims:
+        s.dist_connect(bufs)
+    return bufs
+
+
+def step_local(sims, ncycles: int):
+    """Step the ranks of one process together (their kernels meet at the
+    cross-device barrier, so each launch must be asynchronous: GEM_F_ASYNC)."""
+    from .gem import GEM_F_ASYNC
+    for s in sims:
+        if not s.flags & GEM_F_ASYNC:
+            raise ValueError("in-process ranks need GEM_F_ASYNC (the launches must overlap)")
+    for s in sims:
+        s.step(ncycles)
+    return [s.last_step_ms() for s in sims]

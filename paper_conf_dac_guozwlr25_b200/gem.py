@@ -27,7 +27,10 @@ ERRORS = {-1: "GEM_E_INVAL", -2: "GEM_E_FORMAT", -3: "GEM_E_CUDA", -4: "GEM_E_NO
           -6: "GEM_E_UNSUPPORTED"}
 EXPORTS = ["gem_load_program", "gem_info_get", "gem_set_inputs", "gem_step", "gem_read_outputs",
            "gem_read_state", "gem_write_state", "gem_read_state_trace", "gem_read_digests", "gem_read_ram",
-           "gem_write_ram", "gem_last_step_ms", "gem_read_profile", "gem_read_activity", "gem_bench_floor", "gem_free", "gem_last_error"]
+           "gem_write_ram", "gem_last_step_ms", "gem_read_profile", "gem_read_activity", "gem_bench_floor", "gem_free", "gem_last_error",
+           "gem_dist_owner", "gem_dist_export", "gem_dist_ipc_handles", "gem_dist_ipc_open", "gem_dist_connect"]
+GEM_DIST_MAX = 8
+GEM_DIST_IPC_BYTES = 328
 
 
 class GemConfig(ctypes.Structure):
@@ -35,7 +38,13 @@ class GemConfig(ctypes.Structure):
                 ("flags", ctypes.c_uint32), ("grid_limit", ctypes.c_uint32),
                 ("ctas_per_sm", ctypes.c_uint32), ("max_group", ctypes.c_uint32),
                 ("lane_groups", ctypes.c_uint32), ("lane_ctas_per_sm", ctypes.c_uint32),
-                ("lane_run", ctypes.c_uint32), ("l2_evict_last", ctypes.c_float)]
+                ("lane_run", ctypes.c_uint32), ("l2_evict_last", ctypes.c_float),
+                ("dist_world", ctypes.c_uint32), ("dist_rank", ctypes.c_uint32)]
+
+
+class GemDistBuffers(ctypes.Structure):
+    _fields_ = [(n, ctypes.c_void_p) for n in ("q", "rd", "cut", "po", "flags")] + \
+               [("grid", ctypes.c_uint32), ("reserved", ctypes.c_uint32)]
 
 
 TUNING = ("ctas_per_sm", "max_group", "lane_groups", "lane_ctas_per_sm", "lane_run", "l2_evict_last")
@@ -91,6 +100,13 @@ def load_library(build: bool = True):
             lib.gem_read_profile.argtypes = [P, P, ctypes.POINTER(u32), ctypes.POINTER(u32)]
             if hasattr(lib, "gem_read_activity"):   # (older builds loaded by A/B timing scripts lack it)
                 lib.gem_read_activity.argtypes = [P, ctypes.POINTER(u64), ctypes.POINTER(u64)]
+            if hasattr(lib, "gem_dist_connect"):
+                DB = ctypes.POINTER(GemDistBuffers)
+                lib.gem_dist_owner.argtypes = [P, ctypes.c_size_t, u32, P]
+                lib.gem_dist_export.argtypes = [P, u64, DB]
+                lib.gem_dist_ipc_handles.argtypes = [P, P]
+                lib.gem_dist_ipc_open.argtypes = [P, P, DB]
+                lib.gem_dist_connect.argtypes = [P, DB]
             lib.gem_free.argtypes = [P]
             lib.gem_free.restype = None
             lib.gem_last_error.restype = ctypes.c_char_p
@@ -104,6 +120,22 @@ def _p(a: Optional[np.ndarray]):
 
 def _dev_ptr(t) -> ctypes.c_void_p:
     return ctypes.c_void_p(int(t.data_ptr()))
+
+
+def dist_owner(blob: bytes, world: int) -> np.ndarray:
+    """gem_dist_owner: the rank owning each partition when the design is split
+    over `world` devices (host-only, no CUDA call)."""
+    lib = load_library()
+    n_parts = int(np.frombuffer(blob, np.uint32, count=64)[_GH_N_PARTS])
+    out = np.zeros(max(n_parts, 1), np.uint32)
+    buf = ctypes.create_string_buffer(blob, len(blob))
+    rc = lib.gem_dist_owner(buf, len(blob), world, _p(out))
+    if rc != 0:
+        raise GemError(f"{ERRORS.get(rc, rc)}: {lib.gem_last_error().decode()}")
+    return out[:n_parts]
+
+
+_GH_N_PARTS = 6   # csrc/gem_isa.h header word
 
 
 def bench_floor(device: int = 0, grid: int = 148, iters: int = 2000):
@@ -122,13 +154,16 @@ class Simulator:
     """One loaded program on one GPU, with `n_streams` independent stimulus streams."""
 
     def __init__(self, blob: bytes, device: int = 0, n_streams: int = 1, flags: int = 0,
-                 cuda_stream: int = 0, grid_limit: int = 0, **tuning):
-        """tuning: gem_config launch-tuning fields (TUNING; 0 = automatic)."""
+                 cuda_stream: int = 0, grid_limit: int = 0, dist_world: int = 1, dist_rank: int = 0, **tuning):
+        """tuning: gem_config launch-tuning fields (TUNING; 0 = automatic).
+        dist_world > 1: this handle is rank `dist_rank` of a design split over
+        devices (gem_dist_*; see dist.py) and needs dist_connect before step."""
         self.lib = load_library()
         bad = set(tuning) - set(TUNING)
         if bad:
             raise TypeError(f"unknown gem_config fields {sorted(bad)}")
         cfg = GemConfig(device, n_streams, ctypes.c_void_p(cuda_stream or None), flags, grid_limit)
+        cfg.dist_world, cfg.dist_rank = dist_world, dist_rank
         for k, v in tuning.items():
             setattr(cfg, k, v)
         h = ctypes.c_void_p()
@@ -173,6 +208,29 @@ class Simulator:
 
     def step(self, ncycles: int):
         self._check(self.lib.gem_step(self._h, ncycles))
+
+    # ---- single-design multi-GPU (gem_dist_*) -------------------------------
+    def dist_export(self, max_cycles: int) -> GemDistBuffers:
+        out = GemDistBuffers()
+        self._check(self.lib.gem_dist_export(self._h, max_cycles, ctypes.byref(out)))
+        return out
+
+    def dist_ipc_handles(self) -> bytes:
+        buf = ctypes.create_string_buffer(GEM_DIST_IPC_BYTES)
+        self._check(self.lib.gem_dist_ipc_handles(self._h, buf))
+        return buf.raw
+
+    def dist_ipc_open(self, handles: bytes) -> GemDistBuffers:
+        assert len(handles) == GEM_DIST_IPC_BYTES
+        out = GemDistBuffers()
+        buf = ctypes.create_string_buffer(handles, len(handles))
+        self._check(self.lib.gem_dist_ipc_open(self._h, buf, ctypes.byref(out)))
+        return out
+
+    def dist_connect(self, peers):
+        """peers: one GemDistBuffers per rank (this rank's entry is ignored)."""
+        arr = (GemDistBuffers * len(peers))(*[p if p is not None else GemDistBuffers() for p in peers])
+        self._check(self.lib.gem_dist_connect(self._h, arr))
 
     def last_step_ms(self) -> float:
         ms = ctypes.c_float()

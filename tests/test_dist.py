@@ -68,3 +68,82 @@ def test_gather_traces_world_sizes(world, total):
         p.join(timeout=120)
         assert p.exitcode == 0
     assert np.array_equal(got, _trace_of(range(total), T, W))
+
+
+# ---- row f4: handle exchange of a design split over ranks (host logic) -----
+class _FakeSplitSim:
+    """Stands in for gem.Simulator's gem_dist_* calls (no GPU here)."""
+
+    def __init__(self, rank):
+        self.rank, self.calls, self.connected = rank, [], None
+
+    def dist_export(self, max_cycles):
+        self.calls.append(("export", max_cycles))
+
+    def dist_ipc_handles(self):
+        return bytes([self.rank + 1]) * 328
+
+    def dist_ipc_open(self, h):
+        assert len(h) == 328 and len(set(h)) == 1
+        self.calls.append(("open", h[0] - 1))
+        return ("mapped", h[0] - 1)
+
+    def dist_connect(self, peers):
+        self.connected = list(peers)
+
+
+def _split_worker(rank, world, port, q):
+    from paper_conf_dac_guozwlr25_b200.dist import connect_split
+    os.environ["MASTER_ADDR"] = "127.0.0.1"
+    os.environ["MASTER_PORT"] = str(port)
+    dist.init_process_group("gloo", rank=rank, world_size=world)
+    try:
+        s = _FakeSplitSim(rank)
+        connect_split(s, 77)
+        q.put((rank, s.calls, s.connected))
+    finally:
+        dist.destroy_process_group()
+
+
+@pytest.mark.parametrize("world", [2, 3])
+def test_connect_split_exchanges_every_peer(world):
+    """dist.connect_split: each rank exports once, maps every OTHER rank's IPC
+    handles (its own never) and connects with peers in rank order."""
+    ctx = mp.get_context("spawn")
+    q = ctx.Queue()
+    port = _free_port()
+    procs = [ctx.Process(target=_split_worker, args=(r, world, port, q)) for r in range(world)]
+    for p in procs:
+        p.start()
+    got = dict((r, (c, con)) for r, c, con in (q.get(timeout=120) for _ in range(world)))
+    for p in procs:
+        p.join(timeout=120)
+        assert p.exitcode == 0
+    for r in range(world):
+        calls, con = got[r]
+        assert calls[0] == ("export", 77)
+        assert sorted(c[1] for c in calls[1:]) == [x for x in range(world) if x != r]
+        assert con == [None if x == r else ("mapped", x) for x in range(world)]
+
+
+def test_dist_owner_split():
+    """gem_dist_owner (host-only): every partition gets one rank < world, the
+    split is deterministic, world 1 is all rank 0, and per stage the loads
+    differ by at most one partition's cost (LPT)."""
+    from paper_conf_dac_guozwlr25_b200 import gem, isa
+    from tests.common import blob
+    b = blob("c2")
+    info = isa.blob_info(b)
+    stages = [[p for p in range(info.n_parts) if info.part_stage[p] == s] for s in range(info.n_stages)]
+    for world in (1, 2, 3, 8):
+        own = gem.dist_owner(b, world)
+        assert len(own) == info.n_parts and own.max() < world
+        assert np.array_equal(own, gem.dist_owner(b, world))
+        if world == 1:
+            assert not own.any()
+        for st in stages:
+            cost = {p: max(int(info.part_cost[p]), 1) for p in st}
+            load = [sum(cost[p] for p in st if own[p] == r) for r in range(world)]
+            assert max(load) - min(load) <= max(cost.values())
+    with pytest.raises(gem.GemError):
+        gem.dist_owner(b[:-4], 2)
