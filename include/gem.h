@@ -67,6 +67,15 @@ extern "C" {
 #define GEM_F_NO_RESIDENT 0x20u
 #define GEM_F_NO_LANES 0x40u
 #define GEM_F_STATIC_LANES 0x80u
+/* Word mode (blobs mapped with words=1, gem_isa.h "WRD1"): runs with fewer
+ * than 32 streams (or with GEM_F_NO_LANES) execute the partition's AND list
+ * one signal per shared-memory word in barrier-separated steps instead of
+ * bit-packed boomerang layers (the latency path); chosen
+ * when every program a CTA runs fits in its shared memory, else the
+ * bit-packed path runs.  Results are identical.  GEM_F_NO_WORDS keeps the
+ * bit-packed path; GEM_F_ACTIVITY and split designs (dist_world > 1) always
+ * use it. */
+#define GEM_F_NO_WORDS 0x100u
 
 typedef struct gem_sim gem_sim; /* opaque, owned by the library */
 
@@ -104,6 +113,7 @@ typedef struct {
   uint32_t ring_slots;   /* else: TMA ring depth used to stream program chunks */
   uint32_t group;        /* streams per work item (program chunks reused across them) */
   uint32_t lanes;        /* 1 = stream-sliced lane mode (32 streams per lane word)  */
+  uint32_t words;        /* 1 = word mode (single-stream latency path, WRD1)        */
   uint64_t n_and;                          /* live 2-input ANDs (gate evals/cycle) */
   uint64_t n_and_mapped;                   /* with RepCut replication              */
   uint64_t program_bytes;

@@ -110,13 +110,16 @@ enum {
   GH_N_AND_SYNTH_LO, GH_N_AND_SYNTH_HI,  /* live ANDs after depth-oriented synthesis (GH_N_AND: before) */
   GH_LEVELS_IN,                         /* logic depth before synthesis (GH_MAX_LEVELS: after)       */
   GH_SYNTH_CHAINS,                      /* chains rewritten by the lookahead                          */
+  GH_HAS_WORDS, GH_OFF_WORD_PROG, GH_WORD_PROG_WORDS_LO, GH_WORD_PROG_WORDS_HI,   /* word programs (WRD1) */
+  GH_WORD_MAX_STATE, GH_WORD_MAX_PROG, GH_WORD_MAX_STEPS, GH_WORD_OPS_LO, GH_WORD_OPS_HI, GH_WORD_TOTAL_STEPS,
   GH_N_WORDS = 64
 };
 
 /* part table entry */
 enum {
   GP_STAGE = 0, GP_PROG_OFF, GP_PROG_LEN, GP_N_LAYERS, GP_CHUNK0, GP_MAX_CHUNK, GP_CHUNK1, GP_CHUNK2,
-  GP_COST, GP_LANE_OFF, GP_LANE_LEN, GP_LANE_CHUNK0, GP_LANE_CHUNK1, GP_LANE_CHUNK2, GP_LANE_WORDS, GP_R15,
+  GP_COST, GP_LANE_OFF, GP_LANE_LEN, GP_LANE_CHUNK0, GP_LANE_CHUNK1, GP_LANE_CHUNK2, GP_LANE_WORDS,
+  GP_WORD_OFF /* word program offset in the WRD1 section (GH_HAS_WORDS) */,
   GP_WORDS = 16
 };
 /* GP_COST: mapper's estimate of one cycle of the partition in SM clocks (used by
@@ -255,3 +258,37 @@ enum { LLH_WORDS_ = 0, LLH_FLAGS, LLH_TOPC, LLH_TOPWO, LLH_WOFF0 /* ..+7 */, LLH
 #define GEM_LANE2_STEP 256
 #define GEM_LANE2_OP_X(a, ia, b, ib) \
   ((uint32_t)(a) | ((uint32_t)(ia) << 14) | ((uint32_t)(b) << 16) | ((uint32_t)(ib) << 30))
+
+/* ---------------------------------------------------------------------------
+ * Word programs ("WRD1", mapper option words=1): the single-stream latency
+ * path.  One stream, one signal per 32-bit shared-memory word (bit 0 = value,
+ * bits 1-31 don't-care).  The bit-packed boomerang layer buys 32x
+ * gates per instruction, which a batched or throughput-bound run needs; a
+ * single stream is bound by the latency of the partition's logic chain
+ * instead, and a word-level step -- every thread one or
+ * more independent ANDs, one block barrier -- costs ~1/10 of a boomerang
+ * layer while a layer advances the critical path by ~6 levels.  The program
+ * is the partition's AND list list-scheduled (critical path first) into
+ * barrier-separated steps of at most `word_step` ops; steps are stored
+ * compactly (op i of step s at index step_start[s] + i; thread t runs ops
+ * t, t + 256, ... of the step).
+ *   header (WPH_*) | step starts [n_steps + 1] | ops [n_ops] uint2 |
+ *   out dst gid [n_out] | out src [n_out][32] | ram [n_ram][4] | gread [n_gread]
+ *   op: x = (a_byte | ia) | (b_byte | ib) << 16, y = dst_byte
+ *       (a_byte, b_byte, dst_byte: word * 4 < 65536; ia / ib = operand
+ *       inversion in bit 0 of the byte offset, which is 4-aligned)
+ *       S[y] = (S[a] ^ ia) & (S[b] ^ ib)   (bit 0)
+ *   out src: byte offset of the endpoint's word | inv (bit 0); bit k of
+ *       output word o = (S[src[o][k] & ~3] ^ src[o][k]) & 1; a padding bit reads
+ *       word 0 (constant 0)
+ *   gread: region << 24 | global bit (word = bit >> 5); entry k -> word 1 + k
+ *   ram: {ram_id, 0, 0, 0}, ports staged by outputs with region GEM_R_RAMP
+ * Word 0 is the constant 0.  Words are allocated by liveness (a word last
+ * read in step s is rewritten from step s + 1 on, after the barrier).       */
+#define GEM_WORD_MAGIC 0x31445257u  /* "WRD1" */
+#define GEM_WORD_MAX_WORDS 16384    /* byte offsets fit 16 bits */
+enum {
+  WPH_MAGIC = 0, WPH_N_GREAD, WPH_N_STEPS, WPH_N_OPS, WPH_N_OUT, WPH_N_RAM, WPH_STATE_WORDS, WPH_OFF_STEPS,
+  WPH_OFF_OPS, WPH_OFF_OUT, WPH_OFF_RAM, WPH_OFF_GREAD, WPH_PROG_LEN, WPH_MAX_STEP_OPS, WPH_R14, WPH_R15,
+  WPH_WORDS = 16
+};

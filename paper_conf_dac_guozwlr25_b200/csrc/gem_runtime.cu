@@ -577,6 +577,7 @@ __device__ void run_partition(const KParams& kp, ProgSrc& ps, uint32_t* S, uint3
     C0 = ps.area + off;
     ctab = C0 + C0[PH_OFF_CHUNKS];
     n_pin = ~0u;
+    PROF(7);
   } else if (ps.pin_chunks) {
     C0 = ps.pin;
     ctab = C0 + C0[PH_OFF_CHUNKS];
@@ -763,6 +764,7 @@ commit:
       }
     }
   }
+  PROF(11);
   // ---- a7: RAM blocks (read-first, then per-bit write; readings U7-U10)
   if (n_ram) {
     __syncthreads();
@@ -1035,6 +1037,7 @@ __global__ void __launch_bounds__(GEM_THREADS, 2) gem_step_kernel(const KParams 
 
 // ---- lane-mode prologue helpers (same protocol as issue_prologue, lane fields)
 #include "gem_lanes.cuh"
+#include "gem_words.cuh"
 
 
 // ---- latency-floor microbenchmarks (bench.py roofline; not on the hot path)
@@ -1155,6 +1158,10 @@ struct gem_sim {
   uint4* d_dyn_units = nullptr;                // lane mode dynamic work units
   uint32_t n_units = 0, *d_dyn_ctr = nullptr;
   unsigned long long* d_act = nullptr;         // {evaluated, skipped}
+  // word mode (single-stream latency path, WRD1 programs resident in shared memory)
+  bool words = false;
+  uint32_t word_state = 0, *d_wprog = nullptr;
+  std::vector<uint32_t> h_wprog_len;           // [n_parts] word program lengths (words)
   uint32_t lanes = 0, n_groups = 0, lane_words = 0, lane_max_chunk = 0, ramp_words = 0, lane_groups = 1;
   bool lane_v2 = false;                        // compacted lane programs ("LAN2")
   uint32_t lane_m = 1;                         // LAN2: ops per thread and step
@@ -1429,6 +1436,69 @@ static int plan_launch(gem_sim* sim, uint32_t max_chunk_words, uint32_t grid_lim
   return GEM_OK;
 }
 
+static const void* word_kernel_for(const gem_sim* sim) {
+  return sim->local ? (const void*)gem_word_kernel<true> : (const void*)gem_word_kernel<false>;
+}
+
+// Word mode launch: one CTA per SM, LPT work lists of (partition, stream)
+// items; every distinct program of a CTA's list must fit in its shared memory
+// beside the state (else GEM_E_UNSUPPORTED and the bit-packed path runs).
+static int plan_launch_words(gem_sim* sim, uint32_t grid_limit) {
+  int sms = 0, coop = 0, optin = 0;
+  CK(cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, sim->device));
+  CK(cudaDeviceGetAttribute(&coop, cudaDevAttrCooperativeLaunch, sim->device));
+  CK(cudaDeviceGetAttribute(&optin, cudaDevAttrMaxSharedMemoryPerBlockOptin, sim->device));
+  if (!coop) return fail(GEM_E_UNSUPPORTED, "device lacks cooperative launch");
+  if (sim->n_stages > GEM_WL_MAX_STAGES) return fail(GEM_E_UNSUPPORTED, "too many stages for word mode");
+  sim->sm_count = (uint32_t)sms;
+  sim->group = 1;
+  sim->max_items = 0;
+  for (uint32_t s = 0; s < sim->n_stages; s++)
+    sim->max_items = std::max(sim->max_items, (sim->h_stage[s + 1] - sim->h_stage[s]) * sim->n_streams);
+  uint32_t grid = std::max<uint32_t>(1, std::min<uint32_t>(sim->max_items, (uint32_t)sms));
+  if (grid_limit) grid = std::max<uint32_t>(1, std::min(grid, grid_limit));
+  sim->loc_words = sim->q_words_int + sim->n_rams;
+  sim->local = grid == 1 && sim->n_streams == 1 && sim->loc_words <= 8192;
+  std::vector<uint32_t> off;
+  std::vector<uint2> items;
+  build_worklists(sim, grid, off, items);
+  uint32_t area = 0;
+  for (uint32_t b = 0; b < grid; b++) {
+    std::vector<uint32_t> seen;
+    uint32_t words = 0, n_items = 0;
+    for (uint32_t s = 0; s < sim->n_stages; s++)
+      for (uint32_t k = off[(size_t)s * (grid + 1) + b]; k < off[(size_t)s * (grid + 1) + b + 1]; k++) {
+        n_items++;
+        const uint32_t p = items[k].x;
+        if (std::find(seen.begin(), seen.end(), p) != seen.end()) continue;
+        seen.push_back(p);
+        words += sim->h_wprog_len[p];
+      }
+    if (seen.size() > GEM_MAX_RESIDENT || n_items > GEM_WL_CACHE)
+      return fail(GEM_E_UNSUPPORTED, "word mode: too many work items per CTA");
+    area = std::max(area, words);
+  }
+  const uint32_t fixed = sim->word_state + GEM_WORD_RAMP + 3 * 16 + GEM_WL_CACHE_WORDS + 4 + (sim->local ? 2 * sim->loc_words : 0u);
+  const uint64_t bytes = (uint64_t)(fixed + area) * 4;
+  if (bytes > (uint64_t)optin) return fail(GEM_E_UNSUPPORTED, "word programs do not fit in shared memory");
+  CK(cudaFuncSetAttribute(word_kernel_for(sim), cudaFuncAttributeMaxDynamicSharedMemorySize, (int)bytes));
+  int occ = 0;
+  CK(cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ, word_kernel_for(sim), GEM_THREADS, (size_t)bytes));
+  if (occ < 1) return fail(GEM_E_UNSUPPORTED, "word kernel not resident");
+  sim->blocks_per_sm = 1;
+  sim->grid = grid;
+  sim->area_words = area;
+  sim->resident = grid;
+  sim->ring_slots = 0;
+  sim->slot_words = 0;
+  sim->smem_bytes = (uint32_t)bytes;
+  CK(dalloc(&sim->d_wl_off, off.size() * 4));
+  CK(cudaMemcpy(sim->d_wl_off, off.data(), off.size() * 4, cudaMemcpyHostToDevice));
+  CK(dalloc(&sim->d_wl_items, std::max<size_t>(items.size(), 1) * 8));
+  if (!items.empty()) CK(cudaMemcpy(sim->d_wl_items, items.data(), items.size() * 8, cudaMemcpyHostToDevice));
+  return GEM_OK;
+}
+
 static const void* lane_kernel_for(uint32_t k, bool v2, uint32_t m) {
   if (v2 && m == 2)
     return k >= 4 ? (const void*)gem_lane_kernel<4, true, 2> : k == 2 ? (const void*)gem_lane_kernel<2, true, 2>
@@ -1595,6 +1665,59 @@ static int validate_blob(const uint32_t* w, size_t nw) {
     if (w[GH_HAS_LANES] && (uint64_t)e[GP_LANE_OFF] + e[GP_LANE_LEN] > lp_words)
       return fail(GEM_E_FORMAT, "lane program out of range");
   }
+  if (w[GH_HAS_WORDS]) {
+    // word programs (WRD1): every table inside its program, every op / output
+    // byte offset inside the state, every port and output gid inside its region
+    const uint64_t wp_words = w[GH_WORD_PROG_WORDS_LO] | ((uint64_t)w[GH_WORD_PROG_WORDS_HI] << 32);
+    if (!in(w[GH_OFF_WORD_PROG], wp_words) || (w[GH_OFF_WORD_PROG] & 3u)) return fail(GEM_E_FORMAT, "truncated word programs");
+    const uint32_t* wp = w + w[GH_OFF_WORD_PROG];
+    for (uint32_t p = 0; p < n_parts; p++) {
+      const uint64_t off = parts[(size_t)p * GP_WORDS + GP_WORD_OFF];
+      if ((off & 3u) || off + WPH_WORDS > wp_words) return fail(GEM_E_FORMAT, "word program out of range");
+      const uint32_t* h = wp + off;
+      const uint64_t len = h[WPH_PROG_LEN], sw = h[WPH_STATE_WORDS];
+      if (h[WPH_MAGIC] != GEM_WORD_MAGIC || len < WPH_WORDS || (len & 3u) || off + len > wp_words || len > w[GH_WORD_MAX_PROG] ||
+          sw > GEM_WORD_MAX_WORDS || sw > w[GH_WORD_MAX_STATE] || sw < 1 + (uint64_t)h[WPH_N_GREAD] ||
+          h[WPH_N_RAM] > GEM_MAX_RAMS_PER_PART)
+        return fail(GEM_E_FORMAT, "bad word program header");
+      const uint64_t ns = h[WPH_N_STEPS], no = h[WPH_N_OPS], nout = h[WPH_N_OUT], nr = h[WPH_N_RAM], ng = h[WPH_N_GREAD];
+      if (h[WPH_OFF_STEPS] + ns + 1 > len || (h[WPH_OFF_OPS] & 1u) || h[WPH_OFF_OPS] + 2 * no > len ||
+          h[WPH_OFF_OUT] + 33 * nout > len || h[WPH_OFF_RAM] + 4 * nr > len || h[WPH_OFF_GREAD] + ng > len)
+        return fail(GEM_E_FORMAT, "word program sections out of range");
+      const uint32_t* stp = h + h[WPH_OFF_STEPS];
+      if (stp[0] != 0 || stp[ns] != no) return fail(GEM_E_FORMAT, "bad word step table");
+      for (uint64_t k = 0; k < ns; k++)
+        if (stp[k + 1] < stp[k] || stp[k + 1] - stp[k] > 4u * GEM_THREADS)
+          return fail(GEM_E_FORMAT, "word step table not monotone or a step above 1024 ops");
+      const uint32_t lim = (uint32_t)sw * 4;
+      const uint32_t* ops = h + h[WPH_OFF_OPS];
+      for (uint64_t i = 0; i < no; i++) {
+        const uint32_t x = ops[2 * i], y = ops[2 * i + 1];
+        if ((x & 0xFFFCu) >= lim || ((x >> 16) & 0xFFFCu) >= lim || y >= lim || y == 0 || (y & 3u))
+          return fail(GEM_E_FORMAT, "word op outside the state");
+      }
+      const uint32_t* od = h + h[WPH_OFF_OUT];
+      for (uint64_t o = 0; o < nout; o++) {
+        const uint32_t reg = GEM_GID_REGION(od[o]), idx = GEM_GID_INDEX(od[o]);
+        const bool ok = (reg == GEM_R_Q && idx < qw) || (reg == GEM_R_PO && idx < pw) ||
+                        (reg == GEM_R_CUT && idx < w[GH_CUT_WORDS]) || (reg == GEM_R_RAMP && idx < 4 * nr);
+        if (!ok) return fail(GEM_E_FORMAT, "bad word output gid");
+        for (uint32_t k = 0; k < 32; k++)
+          if ((od[nout + o * 32 + k] & 0xFFFCu) >= lim || (od[nout + o * 32 + k] >> 16))
+            return fail(GEM_E_FORMAT, "word output outside the state");
+      }
+      const uint32_t* rr = h + h[WPH_OFF_RAM];
+      for (uint64_t r = 0; r < nr; r++)
+        if (rr[4 * r] >= w[GH_N_RAMS]) return fail(GEM_E_FORMAT, "bad word RAM id");
+      const uint32_t* gr = h + h[WPH_OFF_GREAD];
+      for (uint64_t k = 0; k < ng; k++) {
+        const uint32_t reg = gr[k] >> 24, bit = gr[k] & 0xFFFFFFu;
+        const bool ok = (reg == GEM_R_PI && bit < 32ull * w[GH_PI_WORDS]) || (reg == GEM_R_Q && bit < 32 * qw) ||
+                        (reg == GEM_R_RD && bit < 32ull * w[GH_N_RAMS]) || (reg == GEM_R_CUT && bit < 32ull * w[GH_CUT_WORDS]);
+        if (!ok) return fail(GEM_E_FORMAT, "bad word port gid");
+      }
+    }
+  }
   return GEM_OK;
 }
 
@@ -1694,6 +1817,20 @@ static int load_impl(gem_sim* sim, const uint32_t* w, size_t nw, const gem_confi
         return fail(GEM_E_FORMAT, "mixed or bad lane programs");
     }
   }
+  // word mode: single-stream latency path (GEM_F_NO_WORDS, activity pruning
+  // and split designs keep the bit-packed path); planned below, falls back to
+  // the bit-packed path when the programs do not fit in shared memory
+  sim->words = !sim->lanes && w[GH_HAS_WORDS] && sim->dist_world == 1 &&
+               !(sim->flags & (GEM_F_NO_WORDS | GEM_F_ACTIVITY));
+  if (sim->words) {
+    const uint64_t wp_words = w[GH_WORD_PROG_WORDS_LO] | ((uint64_t)w[GH_WORD_PROG_WORDS_HI] << 32);
+    sim->word_state = (std::max<uint32_t>(w[GH_WORD_MAX_STATE], 4) + 3) & ~3u;
+    CK(dalloc(&sim->d_wprog, wp_words * 4));
+    CK(cudaMemcpy(sim->d_wprog, w + w[GH_OFF_WORD_PROG], wp_words * 4, cudaMemcpyHostToDevice));
+    sim->h_wprog_len.resize(sim->n_parts);
+    for (uint32_t p = 0; p < sim->n_parts; p++)
+      sim->h_wprog_len[p] = w[w[GH_OFF_WORD_PROG] + parts[(size_t)p * GP_WORDS + GP_WORD_OFF] + WPH_PROG_LEN];
+  }
   // uploads
   const size_t S = sim->n_streams;
   CK(dalloc(&sim->d_prog, prog_words * 4));
@@ -1752,10 +1889,14 @@ static int load_impl(gem_sim* sim, const uint32_t* w, size_t nw, const gem_confi
     sim->owner.assign(sim->n_parts, 0);
     dist_assign(parts, stages, sim->n_stages, sim->dist_world, sim->owner.data());
   }
+  if (sim->words && plan_launch_words(sim, cfg->grid_limit) != GEM_OK) {
+    if (sim->poisoned) return GEM_E_CUDA;
+    sim->words = false;   // does not fit: the bit-packed path runs it
+  }
   if (sim->lanes) {
     if (int r = plan_launch_lanes(sim, cfg->grid_limit)) return r;
-  } else if (int r = plan_launch(sim, w[GH_MAX_CHUNK_WORDS], cfg->grid_limit)) {
-    return r;
+  } else if (!sim->words) {
+    if (int r = plan_launch(sim, w[GH_MAX_CHUNK_WORDS], cfg->grid_limit)) return r;
   }
   CK(cudaDeviceSynchronize());
   return GEM_OK;
@@ -1800,6 +1941,7 @@ int gem_info_get(const gem_sim* sim, gem_info* out) {
   out->grid = sim->grid; out->blocks_per_sm = sim->blocks_per_sm; out->smem_bytes = sim->smem_bytes;
   out->resident = sim->resident; out->ring_slots = sim->ring_slots; out->group = sim->group;
   out->lanes = sim->lanes;
+  out->words = sim->words ? 1u : 0u;
   out->n_streams = sim->n_streams;
   out->n_and = sim->n_and; out->n_and_mapped = sim->n_and_mapped; out->program_bytes = sim->program_bytes;
   out->cycle = sim->cycle;
@@ -1931,9 +2073,14 @@ int gem_step(gem_sim* sim, uint64_t ncycles) {
     kp.state_words = sim->lane_words;
     kp.group = sim->lane_groups;
   }
+  if (sim->words) {
+    kp.lprog = sim->d_wprog;
+    kp.state_words = sim->word_state;
+    kp.loc_words = sim->local ? sim->loc_words : 0u;
+  }
   void* args[] = {&kp};
   CK(cudaEventRecord(sim->ev0, sim->stream));
-  CK(cudaLaunchCooperativeKernel(sim->lanes ? lane_kernel_for(sim->lane_groups, sim->lane_v2, sim->lane_m) : step_kernel_for(sim),
+  CK(cudaLaunchCooperativeKernel(sim->words ? word_kernel_for(sim) : sim->lanes ? lane_kernel_for(sim->lane_groups, sim->lane_v2, sim->lane_m) : step_kernel_for(sim),
                                  dim3(sim->grid), dim3(GEM_THREADS), args, sim->smem_bytes, sim->stream));
   CK(cudaEventRecord(sim->ev1, sim->stream));
   sim->in_head += (uint32_t)ncycles;
@@ -2249,7 +2396,7 @@ void gem_free(gem_sim* sim) {
                   (void*)sim->d_q_ext_of_int, (void*)sim->d_po_int_of_ext, (void*)sim->d_q, (void*)sim->d_rd,
                   (void*)sim->d_cut, (void*)sim->d_mem, (void*)sim->d_pi, (void*)sim->d_po, (void*)sim->d_qtrace,
                   (void*)sim->d_scratch, (void*)sim->d_digest, (void*)sim->d_bar,
-                  (void*)sim->d_prof, (void*)sim->d_wl_off, (void*)sim->d_wl_items, (void*)sim->d_lprog,
+                  (void*)sim->d_prof, (void*)sim->d_wl_off, (void*)sim->d_wl_items, (void*)sim->d_lprog, (void*)sim->d_wprog,
                   (void*)sim->d_pi_lane, (void*)sim->d_po_lane, (void*)sim->d_act,
                   (void*)sim->d_dyn_units, (void*)sim->d_dyn_ctr, (void*)sim->d_dist_flags})
     if (p) cudaFree(p);

@@ -23,6 +23,7 @@ GEM_F_ACTIVITY = 0x10
 GEM_F_NO_RESIDENT = 0x20
 GEM_F_NO_LANES = 0x40
 GEM_F_STATIC_LANES = 0x80
+GEM_F_NO_WORDS = 0x100
 ERRORS = {-1: "GEM_E_INVAL", -2: "GEM_E_FORMAT", -3: "GEM_E_CUDA", -4: "GEM_E_NOMEM", -5: "GEM_E_NOINPUT",
           -6: "GEM_E_UNSUPPORTED"}
 EXPORTS = ["gem_load_program", "gem_info_get", "gem_set_inputs", "gem_step", "gem_read_outputs",
@@ -54,7 +55,7 @@ class GemInfo(ctypes.Structure):
     _fields_ = [(n, ctypes.c_uint32) for n in
                 ("n_pi", "n_po", "n_flops", "n_rams", "n_parts", "n_stages", "max_layers", "total_layers",
                  "pi_words", "po_words", "q_words", "grid", "blocks_per_sm", "smem_bytes", "n_streams",
-                 "resident", "ring_slots", "group", "lanes")] + \
+                 "resident", "ring_slots", "group", "lanes", "words")] + \
                [(n, ctypes.c_uint64) for n in ("n_and", "n_and_mapped", "program_bytes", "cycle")]
 
     def as_dict(self):

@@ -13,7 +13,9 @@ GH = ["MAGIC", "VERSION", "N_PI", "N_PO", "N_FLOPS", "N_RAMS", "N_PARTS", "N_STA
       "MAX_OUT", "TOTAL_WORDS_LO", "TOTAL_WORDS_HI", "SLOTS_USED_LO", "SLOTS_USED_HI",
       "MAX_CHUNK_WORDS", "MAX_PROG_WORDS", "HAS_LANES", "OFF_LANE_PROG", "LANE_PROG_WORDS_LO",
       "LANE_PROG_WORDS_HI", "LANE_MAX_CHUNK_WORDS", "LANE_MAX_WORDS", "MAX_RAMS_PART",
-      "N_AND_SYNTH_LO", "N_AND_SYNTH_HI", "LEVELS_IN", "SYNTH_CHAINS"]
+      "N_AND_SYNTH_LO", "N_AND_SYNTH_HI", "LEVELS_IN", "SYNTH_CHAINS",
+      "HAS_WORDS", "OFF_WORD_PROG", "WORD_PROG_WORDS_LO", "WORD_PROG_WORDS_HI", "WORD_MAX_STATE",
+      "WORD_MAX_PROG", "WORD_MAX_STEPS", "WORD_OPS_LO", "WORD_OPS_HI", "WORD_TOTAL_STEPS"]
 GP_WORDS = 16   # csrc/gem_isa.h GP_WORDS
 GEM_MAGIC = 0x424D4547
 SLOTS_PER_LAYER = 8191
@@ -50,6 +52,12 @@ class BlobInfo:
     synth_chains: int = 0
     lane_ops: int = 0          # LAN2 lane programs: AND ops over all partitions (0 otherwise)
     lane_steps: int = 0
+    has_words: bool = False    # word programs (WRD1, the single-stream path)
+    word_max_steps: int = 0    # steps of the deepest word program (the critical step chain)
+    word_total_steps: int = 0
+    word_ops: int = 0
+    word_program_bytes: int = 0
+    word_max_state: int = 0
 
     def stage_max_layers(self) -> list:
         """Deepest partition (layers) of each stage: a lower bound on the layers
@@ -113,4 +121,7 @@ def blob_info(blob: bytes) -> BlobInfo:
                     max_chunk_words=h["MAX_CHUNK_WORDS"], max_prog_words=h["MAX_PROG_WORDS"],
                     part_cost=pt[:, 8].tolist(), part_stage=pt[:, 0].tolist(),
                     n_and_synth=u64("N_AND_SYNTH"), levels_in=h["LEVELS_IN"], synth_chains=h["SYNTH_CHAINS"],
-                    lane_ops=lane_ops, lane_steps=lane_steps)
+                    lane_ops=lane_ops, lane_steps=lane_steps, has_words=bool(h["HAS_WORDS"]),
+                    word_max_steps=h["WORD_MAX_STEPS"], word_total_steps=h["WORD_TOTAL_STEPS"],
+                    word_ops=u64("WORD_OPS"), word_program_bytes=4 * u64("WORD_PROG_WORDS"),
+                    word_max_state=h["WORD_MAX_STATE"])

@@ -81,6 +81,8 @@ struct Options {
   int lane_k = 4;           // lane mode 2: bank-conflict model for K interleaved groups (K lanes' words
                             // per 16 bytes: lanes of 32/K share one wavefront)
   int lane_m = 1;           // lane mode 2: independent ops per thread and step (1 or 2)
+  int words = 0;            // also emit word programs (WRD1, gem_isa.h): the single-stream latency path
+  int word_step = 1024;     // word programs: max ops per barrier-separated step
   int lane_mode = 2;        // 1: lane program from the boomerang placement ("LANE"); 2: compacted AND
                             // list in barrier-separated steps ("LAN2", gem_isa.h)
   int banks = 1;            // bank-conflict-aware renaming of the state words (rename_state_words)
@@ -128,6 +130,8 @@ static Options parse_opts(const char* s) {
     else if (k == "max_warps") o.max_warps = std::max(1, std::min(8, std::stoi(v)));
     else if (k == "lane_holes") o.lane_holes = std::max(1, std::stoi(v));
     else if (k == "lane_mode") o.lane_mode = std::max(1, std::min(2, std::stoi(v)));
+    else if (k == "words") o.words = std::stoi(v);
+    else if (k == "word_step") o.word_step = std::max(32, std::min(4 * GEM_THREADS, std::stoi(v)));
     else if (k == "lane_m") o.lane_m = std::max(1, std::min(2, std::stoi(v)));
     else if (k == "lane_k") o.lane_k = std::stoi(v) >= 4 ? 4 : std::stoi(v) >= 2 ? 2 : 1;
     else if (k == "banks") o.banks = std::stoi(v);
@@ -453,6 +457,8 @@ struct Part {
   // filled by mapping
   std::vector<uint32_t> prog;
   std::vector<uint32_t> lane_prog;   // lane-mode program (opt.lanes)
+  std::vector<uint32_t> word_prog;   // word program (opt.words; empty if it does not fit)
+  uint32_t word_steps = 0, word_ops = 0;
   uint32_t lane_words = 0;
   uint32_t n_layers = 0, n_nodes = 0, state_words = 0, n_leaves = 0, max_level = 0, n_writeouts = 0;
   uint64_t slots_used = 0;
@@ -960,6 +966,7 @@ struct Mapper {
     P.slots_used = slots_used;
     if (opt.lanes && opt.lane_mode == 1 && !encode_lanes(P, lane_layers, gread_src, scratch)) return;
     if (opt.lanes && opt.lane_mode == 2 && !encode_lanes2(P, scratch)) return;
+    if (opt.words) encode_words(P, scratch);
     P.ok = true;
   }
 
@@ -1782,6 +1789,189 @@ struct Mapper {
       fprintf(stderr, "lane2 part: ops=%u steps=%u (fill %.2f) srcs=%zu words=%u\n", n_ops, S,
               n_ops / (double)(S * kStep), srcs.size(), max_word);
     return true;
+  }
+
+  // Word program ("WRD1", gem_isa.h): the single-stream path.  One signal per
+  // shared-memory word; the partition's ANDs list-scheduled (critical path
+  // first, as LAN2) into steps of <= word_step ops separated by one block
+  // barrier, stored compactly.  Within a step, ops are placed in warp-sized
+  // rounds (slot j -> thread j % 256, lane j % 32) so that a round's operand
+  // words fall into distinct banks where the ready list allows it, and each
+  // op's destination word is allocated (by liveness) in bank j % 32, so a
+  // round's 32 stores are conflict-free.  Leaves P.word_prog empty when the
+  // live words exceed GEM_WORD_MAX_WORDS (the blob then has no word programs).
+  void encode_words(Part& P, const std::vector<int32_t>& scratch) {
+    P.word_prog.clear();
+    const uint32_t n = (uint32_t)cid.size();
+    const uint32_t kStep = (uint32_t)opt.word_step;
+    std::vector<uint32_t> srcs;
+    for (uint32_t i = 1; i < n; i++)
+      if (is_src[i]) srcs.push_back(i);
+    std::stable_sort(srcs.begin(), srcs.end(), [&](uint32_t x, uint32_t y) {
+      const uint32_t gx = G.gbit[cid[x]], gy = G.gbit[cid[y]];
+      const uint64_t kx = ((uint64_t)(gx >> 27) << 32) | (((gx >> 5) & 0x3FFFFF) * 32 + (gx & 31));
+      const uint64_t ky = ((uint64_t)(gy >> 27) << 32) | (((gy >> 5) & 0x3FFFFF) * 32 + (gy & 31));
+      return kx < ky;
+    });
+    if (srcs.size() + 1 >= GEM_WORD_MAX_WORDS) return;
+    // ---- list scheduling (an op is ready one step after its last operand)
+    std::vector<uint32_t> rd(n, 0), pend(n, 0), step_of(n, 0);
+    for (uint32_t i = n; i-- > 0;)
+      for (uint32_t j = coff[i]; j < coff[i + 1]; j++) rd[i] = std::max(rd[i], rd[cons[j]] + 1);
+    std::vector<uint32_t> ready;
+    auto prio = [&](uint32_t x, uint32_t y) { return rd[x] != rd[y] ? rd[x] < rd[y] : x > y; };
+    uint32_t n_ops = 0;
+    for (uint32_t i = 0; i < n; i++) {
+      if (is_src[i]) continue;
+      n_ops++;
+      pend[i] = (uint32_t)(!is_src[la[i] >> 1]) + (uint32_t)(!is_src[lb[i] >> 1]);
+      if ((la[i] >> 1) == (lb[i] >> 1) && !is_src[la[i] >> 1]) pend[i] = 1;
+      if (!pend[i]) ready.push_back(i);
+    }
+    std::make_heap(ready.begin(), ready.end(), prio);
+    std::vector<std::vector<uint32_t>> steps;
+    std::vector<uint32_t> next_ready;
+    uint32_t done = 0;
+    while (done < n_ops) {
+      if (ready.empty()) throw std::runtime_error("words: scheduling stalled");
+      steps.emplace_back();
+      auto& st = steps.back();
+      while (!ready.empty() && st.size() < kStep) {
+        std::pop_heap(ready.begin(), ready.end(), prio);
+        st.push_back(ready.back());
+        ready.pop_back();
+      }
+      next_ready.clear();
+      for (uint32_t x : st) {
+        step_of[x] = (uint32_t)steps.size() - 1;
+        done++;
+        for (uint32_t j = coff[x]; j < coff[x + 1]; j++) {
+          const uint32_t c = cons[j];
+          if (j > coff[x] && cons[j - 1] == c) continue;
+          if (--pend[c] == 0) next_ready.push_back(c);
+        }
+      }
+      for (uint32_t c : next_ready) { ready.push_back(c); std::push_heap(ready.begin(), ready.end(), prio); }
+    }
+    const uint32_t S = (uint32_t)steps.size();
+    const uint32_t INF = UINT32_MAX;
+    std::vector<uint32_t> last(n, 0);
+    for (uint32_t i = 0; i < n; i++) {
+      if (is_ep[i]) { last[i] = INF; continue; }
+      for (uint32_t j = coff[i]; j < coff[i + 1]; j++) last[i] = std::max(last[i], step_of[cons[j]]);
+    }
+    // ---- words: 0 = constant, 1..n_src = ports, then by liveness with a bank choice
+    std::vector<int32_t> word(n, -1);
+    word[0] = 0;
+    uint32_t top = 1;
+    for (uint32_t x : srcs) word[x] = (int32_t)top++;
+    std::vector<std::set<uint32_t>> freew(32);
+    std::vector<std::vector<uint32_t>> die(S + 1);
+    for (uint32_t x : srcs)
+      if (last[x] != INF) die[last[x]].push_back((uint32_t)word[x]);
+    auto alloc = [&](uint32_t res) -> uint32_t {
+      if (!freew[res].empty()) {
+        const uint32_t w = *freew[res].begin();
+        freew[res].erase(freew[res].begin());
+        return w;
+      }
+      const uint32_t fresh = top + ((res + 32 - (top % 32)) % 32);
+      for (uint32_t w = top; w < fresh; w++) freew[w % 32].insert(w);
+      top = fresh + 1;
+      return fresh;
+    };
+    auto lw = [&](uint32_t l) -> uint32_t {
+      const int32_t w = word[l >> 1];
+      if (w < 0) throw std::runtime_error("words: operand without a word");
+      return (uint32_t)w;
+    };
+    std::vector<uint32_t> step_start(S + 1, 0), ops;
+    ops.reserve((size_t)n_ops * 2);
+    uint32_t max_step = 0;
+    for (uint32_t s = 0; s < S; s++) {
+      if (s > 0)
+        for (uint32_t w : die[s - 1]) freew[w % 32].insert(w);
+      step_start[s] = (uint32_t)(ops.size() / 2);
+      auto& st = steps[s];
+      max_step = std::max<uint32_t>(max_step, (uint32_t)st.size());
+      std::stable_sort(st.begin(), st.end(), [&](uint32_t x, uint32_t y) { return rd[x] > rd[y]; });
+      // rounds of 32 slots: take, within a window of the remaining ops, the first
+      // whose A and B banks are still unused by the round (else the first)
+      std::vector<uint32_t> rem(st.begin(), st.end()), order;
+      order.reserve(st.size());
+      while (!rem.empty()) {
+        uint32_t usedA = 0, usedB = 0;
+        std::vector<uint32_t> wA, wB;   // words already in the round (repeats broadcast)
+        const size_t take = std::min<size_t>(32, rem.size());
+        for (size_t k = 0; k < take; k++) {
+          size_t pick = 0;
+          const size_t win = std::min<size_t>(rem.size(), 96);
+          for (size_t c = 0; c < win; c++) {
+            const uint32_t x = rem[c], a = lw(la[x]), b = lw(lb[x]);
+            const bool okA = !((usedA >> (a % 32)) & 1u) || std::find(wA.begin(), wA.end(), a) != wA.end();
+            const bool okB = !((usedB >> (b % 32)) & 1u) || std::find(wB.begin(), wB.end(), b) != wB.end();
+            if (okA && okB) { pick = c; break; }
+          }
+          const uint32_t x = rem[pick];
+          rem.erase(rem.begin() + (ptrdiff_t)pick);
+          const uint32_t a = lw(la[x]), b = lw(lb[x]);
+          usedA |= 1u << (a % 32);
+          usedB |= 1u << (b % 32);
+          wA.push_back(a);
+          wB.push_back(b);
+          order.push_back(x);
+        }
+      }
+      for (uint32_t j = 0; j < (uint32_t)order.size(); j++) {
+        const uint32_t x = order[j];
+        const uint32_t a = lw(la[x]), b = lw(lb[x]);
+        const uint32_t w = alloc(j % 32);
+        word[x] = (int32_t)w;
+        if (last[x] != INF) die[std::max(last[x], s)].push_back(w);
+        ops.push_back((a * 4 | (la[x] & 1u)) | ((b * 4 | (lb[x] & 1u)) << 16));
+        ops.push_back(w * 4);
+      }
+      if (top >= GEM_WORD_MAX_WORDS) return;
+    }
+    step_start[S] = (uint32_t)(ops.size() / 2);
+    std::vector<uint32_t>& pr = P.word_prog;
+    pr.assign(WPH_WORDS, 0);
+    pr[WPH_MAGIC] = GEM_WORD_MAGIC;
+    pr[WPH_N_GREAD] = (uint32_t)srcs.size();
+    pr[WPH_N_STEPS] = S;
+    pr[WPH_N_OPS] = n_ops;
+    pr[WPH_N_OUT] = (uint32_t)P.outs.size();
+    pr[WPH_N_RAM] = (uint32_t)P.rams.size();
+    pr[WPH_STATE_WORDS] = (top + 3) & ~3u;
+    pr[WPH_MAX_STEP_OPS] = max_step;
+    pr[WPH_OFF_STEPS] = (uint32_t)pr.size();
+    pr.insert(pr.end(), step_start.begin(), step_start.end());
+    while (pr.size() % 4) pr.push_back(0);
+    pr[WPH_OFF_OPS] = (uint32_t)pr.size();
+    pr.insert(pr.end(), ops.begin(), ops.end());
+    while (pr.size() % 4) pr.push_back(0);
+    pr[WPH_OFF_OUT] = (uint32_t)pr.size();
+    for (auto& ow : P.outs) pr.push_back(ow.dst);
+    for (auto& ow : P.outs)
+      for (int k = 0; k < 32; k++) {
+        const uint32_t l = ow.lit[k];
+        pr.push_back(lw(2 * (uint32_t)scratch[l >> 1]) * 4 | (l & 1u));
+      }
+    while (pr.size() % 4) pr.push_back(0);
+    pr[WPH_OFF_RAM] = (uint32_t)pr.size();
+    for (uint32_t r : P.rams) { pr.push_back(r); pr.push_back(0); pr.push_back(0); pr.push_back(0); }
+    pr[WPH_OFF_GREAD] = (uint32_t)pr.size();
+    for (uint32_t x : srcs) {
+      const uint32_t gb = G.gbit[cid[x]];
+      pr.push_back(((gb >> 27) << 24) | (((gb >> 5) & 0x3FFFFF) * 32 + (gb & 31)));
+    }
+    while (pr.size() % 4) pr.push_back(0);
+    pr[WPH_PROG_LEN] = (uint32_t)pr.size();
+    P.word_steps = S;
+    P.word_ops = n_ops;
+    if (opt.verbose >= 3)
+      fprintf(stderr, "words part: ops=%u steps=%u max_step=%u srcs=%zu words=%u\n", n_ops, S, max_step,
+              srcs.size(), top);
   }
 
   void fail(Part& P, const char* why) {
@@ -2748,6 +2938,39 @@ static Blob compile(const char* data, size_t n, const char* opts) {
     uint32_t mr = 0;
     for (auto& P : D.parts) mr = std::max<uint32_t>(mr, (uint32_t)P.rams.size());
     w[GH_MAX_RAMS_PART] = mr;
+  }
+  // word programs (WRD1): only if every partition has one (else the runtime
+  // stays on the bit-packed path)
+  if (D.opt.words && std::all_of(D.parts.begin(), D.parts.end(), [](const Part& P) { return !P.word_prog.empty(); })) {
+    while (w.size() % 4) w.push_back(0);
+    w[GH_HAS_WORDS] = 1;
+    w[GH_OFF_WORD_PROG] = (uint32_t)w.size();
+    uint64_t wp = 0, wops = 0;
+    uint32_t mst = 0, mpw = 0, msteps = 0, tsteps = 0;
+    for (uint32_t i = 0; i < np; i++) {
+      auto& P = D.parts[i];
+      w[part_tab + i * GP_WORDS + GP_WORD_OFF] = (uint32_t)wp;
+      mst = std::max(mst, P.word_prog[WPH_STATE_WORDS]);
+      mpw = std::max<uint32_t>(mpw, (uint32_t)P.word_prog.size());
+      msteps = std::max(msteps, P.word_steps);
+      tsteps += P.word_steps;
+      wops += P.word_ops;
+      w.insert(w.end(), P.word_prog.begin(), P.word_prog.end());
+      wp += P.word_prog.size();
+    }
+    w[GH_WORD_PROG_WORDS_LO] = (uint32_t)wp;
+    w[GH_WORD_PROG_WORDS_HI] = (uint32_t)(wp >> 32);
+    w[GH_WORD_MAX_STATE] = mst;
+    w[GH_WORD_MAX_PROG] = mpw;
+    w[GH_WORD_MAX_STEPS] = msteps;
+    w[GH_WORD_OPS_LO] = (uint32_t)wops;
+    w[GH_WORD_OPS_HI] = (uint32_t)(wops >> 32);
+    w[GH_WORD_TOTAL_STEPS] = tsteps;
+    uint32_t mr = 0;
+    for (auto& P : D.parts) mr = std::max<uint32_t>(mr, (uint32_t)P.rams.size());
+    w[GH_MAX_RAMS_PART] = std::max(w[GH_MAX_RAMS_PART], mr);
+  } else if (D.opt.words && D.opt.verbose) {
+    fprintf(stderr, "gem_map: no word programs (a partition exceeds %u live words)\n", (unsigned)GEM_WORD_MAX_WORDS);
   }
   w[GH_PROG_WORDS_LO] = (uint32_t)prog;
   w[GH_PROG_WORDS_HI] = (uint32_t)(prog >> 32);

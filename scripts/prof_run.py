@@ -49,6 +49,9 @@ if a.phases:
     c0, grl, l0, gb = d(0, 7), d(7, 8), d(8, 9), d(9, 1)
     print(f"  critical CTA gread split: chunk0 ready {c0[:, crit].mean():.0f}, port loads (thread 0) "
           f"{grl[:, crit].mean():.0f}, layer-0 records {l0[:, crit].mean():.0f}, barrier {gb[:, crit].mean():.0f}")
+    if not sim.info.get("lanes"):
+        e11 = d(2, 11)
+        print(f"  critical CTA commit split: endpoints {e11[:, crit].mean():.0f}, RAM + sync {d(11, 3)[:, crit].mean():.0f}")
     per_layer = layers.mean(0) / np.maximum(1, nl[0])
     print(f"  all CTAs: items mean {items.mean():.0f} max {items.mean(0).max():.0f}; per-layer clocks "
           f"mean {per_layer.mean():.0f} min {per_layer.min():.0f} max {per_layer.max():.0f}; "

@@ -26,6 +26,7 @@ def _load():
         lib.isa_free.argtypes = [P]
         lib.isa_run.argtypes = [P, P, ctypes.c_uint64, P, P]
         lib.isa_run_lanes.argtypes = [P, P, ctypes.c_uint64, P, P]
+        lib.isa_run_words.argtypes = [P, P, ctypes.c_uint64, P, P]
         lib.isa_last_error.restype = ctypes.c_char_p
         _lib = lib
     return _lib
@@ -46,12 +47,13 @@ class IsaInterp:
         if getattr(self, "_h", None):
             self.lib.isa_free(self._h)
 
-    def run(self, stim):
+    def run(self, stim, words: bool = False):
+        """Bit-packed layers (default) or the word programs (WRD1) of the blob."""
         stim = np.ascontiguousarray(stim, np.uint32)
         T = stim.shape[0]
         po = np.zeros((T, (self.n_po + 31) // 32), np.uint32)
         q = np.zeros((T, (self.n_flops + 31) // 32), np.uint32)
-        rc = self.lib.isa_run(self._h, stim.ctypes.data_as(ctypes.c_void_p), T,
+        rc = (self.lib.isa_run_words if words else self.lib.isa_run)(self._h, stim.ctypes.data_as(ctypes.c_void_p), T,
                               po.ctypes.data_as(ctypes.c_void_p), q.ctypes.data_as(ctypes.c_void_p))
         if rc:
             raise RuntimeError(self.lib.isa_last_error().decode())

@@ -385,6 +385,82 @@ int run_lane_part(Interp& I, LaneSim& Ls, uint32_t p, const uint32_t* pi_lane /*
   }
   return 0;
 }
+
+// ------------------------------------------------------------------ word mode
+// gem_isa.h "WRD1": one signal per word (bit 0), steps of independent ops.
+// Hazard checks: an op of step s reads no word written in step s, a word is
+// written at most once per step, word 0 is never written.
+int run_word_part(Interp& I, uint32_t p, const uint32_t* stim, uint32_t* po_row) {
+  const uint32_t* pt = I.parts + p * GP_WORDS;
+  const uint32_t* pr = I.w.data() + I.w[GH_OFF_WORD_PROG] + pt[GP_WORD_OFF];
+  if (pr[WPH_MAGIC] != GEM_WORD_MAGIC) { g_err = "bad word magic"; return -1; }
+  uint32_t cur = (uint32_t)(I.cycle & 1), nxt = cur ^ 1;
+  std::vector<uint32_t> S(pr[WPH_STATE_WORDS], 0);
+  std::vector<uint32_t> wstep(S.size(), 0xFFFFFFFFu);
+  const uint32_t* gr = pr + pr[WPH_OFF_GREAD];
+  for (uint32_t k = 0; k < pr[WPH_N_GREAD]; k++) {
+    const uint32_t reg = gr[k] >> 24, bit = gr[k] & 0xFFFFFFu, wi = bit >> 5;
+    uint32_t v;
+    if (reg == GEM_R_PI) v = stim[wi];
+    else if (reg == GEM_R_Q) v = I.Q[cur][wi];
+    else if (reg == GEM_R_RD) v = I.RD[cur][wi];
+    else if (reg == GEM_R_CUT) v = I.CUT[wi];
+    else { g_err = "bad word gread region"; return -1; }
+    if (1 + k >= S.size()) { g_err = "word gread outside the state"; return -1; }
+    S[1 + k] = (v >> (bit & 31)) & 1u;
+  }
+  const uint32_t* stp = pr + pr[WPH_OFF_STEPS];
+  const uint32_t* ops = pr + pr[WPH_OFF_OPS];
+  std::vector<std::pair<uint32_t, uint32_t>> wr;
+  for (uint32_t s = 0; s < pr[WPH_N_STEPS]; s++) {
+    wr.clear();
+    for (uint32_t i = stp[s]; i < stp[s + 1]; i++) {
+      const uint32_t x = ops[2 * i], y = ops[2 * i + 1];
+      const uint32_t a = (x & 0xFFFCu) >> 2, b = ((x >> 16) & 0xFFFCu) >> 2, d = y >> 2;
+      if (a >= S.size() || b >= S.size() || d >= S.size() || d == 0 || (y & 3u)) { g_err = "word op out of range"; return -1; }
+      if (wstep[a] == s || wstep[b] == s) { g_err = "word op reads a word written in the same step"; return -1; }
+      if (wstep[d] == s) { g_err = "word written twice in a step"; return -1; }
+      wstep[d] = s;
+      wr.push_back({d, ((S[a] ^ x) & (S[b] ^ (x >> 16))) & 1u});
+    }
+    for (uint32_t i = stp[s]; i < stp[s + 1]; i++) {
+      const uint32_t x = ops[2 * i];
+      if (wstep[(x & 0xFFFCu) >> 2] == s || wstep[((x >> 16) & 0xFFFCu) >> 2] == s) {
+        g_err = "word op reads a word written in the same step";
+        return -1;
+      }
+    }
+    for (auto& e : wr) S[e.first] = e.second;
+  }
+  const uint32_t n_out = pr[WPH_N_OUT];
+  const uint32_t* od = pr + pr[WPH_OFF_OUT];
+  const uint32_t* os = od + n_out;
+  uint32_t ramp[GEM_MAX_RAMS_PER_PART * 4];
+  std::memset(ramp, 0, sizeof(ramp));
+  for (uint32_t j = 0; j < n_out; j++) {
+    uint32_t v = 0;
+    for (int b = 0; b < 32; b++) {
+      const uint32_t e = os[j * 32 + b];
+      if (((e & 0xFFFCu) >> 2) >= S.size()) { g_err = "word output out of range"; return -1; }
+      v |= ((S[(e & 0xFFFCu) >> 2] ^ e) & 1u) << b;
+    }
+    uint32_t reg = GEM_GID_REGION(od[j]), idx = GEM_GID_INDEX(od[j]);
+    if (reg == GEM_R_Q) I.Q[nxt][idx] = v;
+    else if (reg == GEM_R_PO) po_row[idx] = v;
+    else if (reg == GEM_R_CUT) I.CUT[idx] = v;
+    else if (reg == GEM_R_RAMP) ramp[idx] = v;
+    else { g_err = "bad word out region"; return -1; }
+  }
+  const uint32_t* rr = pr + pr[WPH_OFF_RAM];
+  for (uint32_t r = 0; r < pr[WPH_N_RAM]; r++) {
+    uint32_t id = rr[4 * r];
+    uint32_t ra = ramp[4 * r + 0] & 0x1FFF, wa = ramp[4 * r + 1] & 0x1FFF;
+    uint32_t wd = ramp[4 * r + 2], be = ramp[4 * r + 3];
+    I.RD[nxt][id] = I.MEM[id][ra];
+    I.MEM[id][wa] = (I.MEM[id][wa] & ~be) | (wd & be);
+  }
+  return 0;
+}
 }  // namespace
 
 extern "C" {
@@ -464,8 +540,10 @@ int isa_run_lanes(void* h, const uint32_t* stim, uint64_t cycles, uint32_t* po_e
 }
 
 // stim [cycles][pi_words] ; po_ext [cycles][ceil(n_po/32)] ; q_ext [cycles][ceil(n_flops/32)] (nullable)
-int isa_run(void* h, const uint32_t* stim, uint64_t cycles, uint32_t* po_ext, uint32_t* q_ext_tr) {
+static int isa_run_impl(void* h, const uint32_t* stim, uint64_t cycles, uint32_t* po_ext, uint32_t* q_ext_tr,
+                        bool words) {
   Interp& I = *(Interp*)h;
+  if (words && !I.w[GH_HAS_WORDS]) { g_err = "blob has no word programs"; return -1; }
   std::vector<uint32_t> po_int(I.po_words);
   uint32_t pwe = (I.n_po + 31) / 32, qwe = (I.n_flops + 31) / 32;
   for (uint64_t t = 0; t < cycles; t++) {
@@ -473,7 +551,9 @@ int isa_run(void* h, const uint32_t* stim, uint64_t cycles, uint32_t* po_ext, ui
     for (uint32_t s = 0; s < I.n_stages; s++)
       for (uint32_t k = I.stages[s]; k < I.stages[s + 1]; k++) {
         uint32_t p = I.stages[I.n_stages + 1 + k];
-        if (run_part(I, p, t, stim + t * I.pi_words, po_int.data())) return -1;
+        if (words ? run_word_part(I, p, stim + t * I.pi_words, po_int.data())
+                  : run_part(I, p, t, stim + t * I.pi_words, po_int.data()))
+          return -1;
       }
     I.cycle++;
     uint32_t cur = (uint32_t)(I.cycle & 1);
@@ -497,5 +577,11 @@ int isa_run(void* h, const uint32_t* stim, uint64_t cycles, uint32_t* po_ext, ui
     }
   }
   return 0;
+}
+int isa_run(void* h, const uint32_t* stim, uint64_t cycles, uint32_t* po_ext, uint32_t* q_ext_tr) {
+  return isa_run_impl(h, stim, cycles, po_ext, q_ext_tr, false);
+}
+int isa_run_words(void* h, const uint32_t* stim, uint64_t cycles, uint32_t* po_ext, uint32_t* q_ext_tr) {
+  return isa_run_impl(h, stim, cycles, po_ext, q_ext_tr, true);
 }
 }

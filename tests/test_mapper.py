@@ -216,3 +216,56 @@ def test_program_tail_holds_gread_used_bit_masks(tmp_path):
         total_bits += sum(bin(int(m)).count("1") for m in masks)
     # each module reads its enable and its 32 flops: 8 partitions x 33 sources
     assert total_bits == 8 * 33, total_bits
+
+
+# ---------------------------------------------------------------- word programs (WRD1)
+def _check_words(path, b, stim):
+    assert blob_info(b).has_words, "mapper emitted no word programs"
+    r = Oracle(path).run(stim, state=True)
+    po, q = IsaInterp(b).run(stim, words=True)
+    assert np.array_equal(po, r["po"]), np.where((po != r["po"]).any(1))[0][:5]
+    assert np.array_equal(q, r["state"]), np.where((q != r["state"]).any(1))[0][:5]
+
+
+def test_c1_word_program_matches_oracle(tmp_path):
+    p = os.path.join(str(tmp_path), "c1.aag")
+    write_eaig(build_c1(), p)
+    b = compile_file(p, "levels=10 words=1")
+    info = blob_info(b)
+    # depth-bound: one step per level of the synthesised C1 (20 levels)
+    assert info.word_max_steps == info.max_levels
+    _check_words(p, b, stimulus("c1", 35, 3000))
+
+
+@pytest.mark.parametrize("opts", ["parts=1", "parts=3 word_step=64", "parts=5 stages=2", "parts=4 stages=2 cut_level=3",
+                                  "parts=2 word_step=32"])
+def test_small_designs_word_programs(tmp_path, opts):
+    net = circuits.small_G(seed=21, n_and=4000, with_ram=True)
+    p = circuits.save(net, str(tmp_path), "g")
+    b = compile_file(p, opts + " words=1")
+    _check_words(p, b, stim_random(net.n_pi, 150, 3, reset_pi0_cycles=2))
+
+
+@pytest.mark.parametrize("seed", [1, 2])
+def test_word_programs_cells(tmp_path, seed):
+    for name, net in [("rc", circuits.random_comb(12, 300, 20, seed)), ("cells", circuits.cells()),
+                      ("sr", circuits.shift_register(40)), ("ram", circuits.ram_direct()),
+                      ("cnt", circuits.counter_with_load())]:
+        p = circuits.save(net, str(tmp_path), name)
+        b = compile_file(p, "words=1")
+        rng = np.random.default_rng(seed)
+        n_pi = Oracle(p).n_pi
+        st = rng.integers(0, 1 << 32, size=(200, (n_pi + 31) // 32), dtype=np.uint64).astype(np.uint32)
+        if n_pi % 32:
+            st[:, -1] &= (1 << (n_pi % 32)) - 1
+        if name == "ram":
+            st[:, 0] = (st[:, 0] & ~np.uint32(0x3FFFFFF)) | (st[:, 0] & 0x7) | ((st[:, 0] & 0x7) << 13)
+        _check_words(p, b, st)
+
+
+def test_c2_word_program_prefix(tmp_path):
+    from tests.common import MAP_OPTS
+    b = blob("c2", MAP_OPTS["c2"] + " words=1")
+    info = blob_info(b)
+    assert info.word_max_steps <= info.max_levels + 1
+    _check_words(eaig("c2"), b, stimulus("c2", 128, 60))
