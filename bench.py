@@ -532,7 +532,8 @@ def roofline(res, peaks, dev):
     peak_lop3 = n_sms * 64 * float(peaks.get("sm_max_mhz", 1965.0)) * 1e6
     hz_kernel = C / (res["kern_ms"] / 1e3)
     achieved_lop3 = info.n_and / 16.0 * hz_kernel * S   # this rank's kernel (per GPU)
-    kname = "gem_lane_kernel" if res["sim_info"]["lanes"] else "gem_step_kernel"
+    words = bool(res["sim_info"].get("words"))
+    kname = "gem_lane_kernel" if res["sim_info"]["lanes"] else "gem_word_kernel" if words else "gem_step_kernel"
     traffic, traffic_src = ncu_traffic(cfg, kname, C)
     alu = {"bound": "alu", "achieved": achieved_lop3 / 1e12, "peak": peak_lop3 / 1e12, "unit": "TLOP3/s",
            "frac": achieved_lop3 / peak_lop3,
@@ -554,18 +555,34 @@ def roofline(res, peaks, dev):
                  "us_per_layer_critical": 1e6 / hz_kernel / max(1, info.max_layers), "alu": alu, "hbm": hbm})
     if S == 1:
         lay_clk, bar_clk = gem.bench_floor(dev.index, res["sim_info"]["grid"])
-        crit = sum(info.stage_max_layers())
         f_hz = float(sm_mhz) * 1e6
-        floor_hz = f_hz / (crit * lay_clk + info.n_stages * bar_clk)
-        lat = {"bound": "latency", "achieved": hz_kernel, "peak": floor_hz, "unit": "cycles/s",
-               "frac": hz_kernel / floor_hz,
-               "layer_clk": lay_clk, "barrier_clk": bar_clk, "critical_layers": crit, "stages": info.n_stages,
-               "achieved_clk_per_cycle": f_hz / hz_kernel,
-               "achieved_clk_per_critical_layer": f_hz / hz_kernel / max(1, crit),
-               "definition": "peak = sm_clock / (sum over stages of the deepest partition's layers x minimal-layer "
-                             "clocks + stages x grid-barrier clocks); minimal layer = one dependent gathered load "
-                             "per thread + 13 fold levels + write-out + block barrier (gem_bench_floor, measured "
-                             "on this GPU in this run)"}
+        if words:
+            # word mode: the chain is the deepest word program's
+            # steps, each at least one minimal step (gem_bench_floor_step)
+            step_clk = gem.bench_floor_step(dev.index)
+            crit = sum(info.stage_max_word_steps())
+            floor_hz = f_hz / (crit * step_clk + info.n_stages * bar_clk)
+            lat = {"bound": "latency", "achieved": hz_kernel, "peak": floor_hz, "unit": "cycles/s",
+                   "frac": hz_kernel / floor_hz, "mode": "words",
+                   "step_clk": step_clk, "barrier_clk": bar_clk, "critical_steps": crit, "stages": info.n_stages,
+                   "achieved_clk_per_cycle": f_hz / hz_kernel,
+                   "achieved_clk_per_critical_step": f_hz / hz_kernel / max(1, crit),
+                   "definition": "peak = sm_clock / (sum over stages of the deepest word program's steps x "
+                                 "minimal-step clocks + stages x grid-barrier clocks); minimal step = block barrier "
+                                 "+ two operand loads + AND + store per thread (gem_bench_floor_step, measured on "
+                                 "this GPU in this run)"}
+        else:
+            crit = sum(info.stage_max_layers())
+            floor_hz = f_hz / (crit * lay_clk + info.n_stages * bar_clk)
+            lat = {"bound": "latency", "achieved": hz_kernel, "peak": floor_hz, "unit": "cycles/s",
+                   "frac": hz_kernel / floor_hz, "mode": "bits",
+                   "layer_clk": lay_clk, "barrier_clk": bar_clk, "critical_layers": crit, "stages": info.n_stages,
+                   "achieved_clk_per_cycle": f_hz / hz_kernel,
+                   "achieved_clk_per_critical_layer": f_hz / hz_kernel / max(1, crit),
+                   "definition": "peak = sm_clock / (sum over stages of the deepest partition's layers x "
+                                 "minimal-layer clocks + stages x grid-barrier clocks); minimal layer = one "
+                                 "dependent gathered load per thread + 13 fold levels + write-out + block barrier "
+                                 "(gem_bench_floor, measured on this GPU in this run)"}
         roof["latency_floor"] = lat
         # does the program stream from HBM every cycle?  The committed ncu
         # capture at the same cycles per launch decides (DRAM bytes per cycle
@@ -577,6 +594,8 @@ def roofline(res, peaks, dev):
             hbm["dram_bytes_per_cycle_ncu"] = traffic / C
         else:
             streamed = info.program_bytes > 0.5 * l2_bytes
+        if words:
+            streamed = False   # word programs are copied into shared memory once per launch
         hbm["program_streamed"] = streamed
         hbm_floor = hbm_peak * 1e9 / info.program_bytes if streamed else float("inf")
         hbm["floor_cycles_per_s"] = hbm_floor if hbm_floor != float("inf") else None
@@ -636,7 +655,12 @@ def mapping_stats(info) -> dict:
             "levels_per_layer": round(info.max_levels / max(1, info.max_layers), 3),
             "n_and_synth": info.n_and_synth, "levels_in": info.levels_in,
             "leaf_util": round(info.total_leaves / max(1, info.total_layers * 8192), 4),
-            "lane_ops": info.lane_ops, "lane_steps": info.lane_steps}
+            "lane_ops": info.lane_ops, "lane_steps": info.lane_steps,
+            "word_programs": info.has_words, "word_ops": info.word_ops,
+            "critical_word_steps": sum(info.stage_max_word_steps()) if info.has_words else None,
+            "word_program_bytes": info.word_program_bytes,
+            "levels_per_critical_step": round(info.max_levels / max(1, sum(info.stage_max_word_steps())), 3)
+            if info.has_words else None}
 
 
 def main():
@@ -735,7 +759,8 @@ def main():
                 "clocks": main_res["clk"], "gpu_launches": args.steps * (n_launch + (1 if lanes else 0)),
                 "gpu_launches_detail": ("per step: to_lanes_kernel (input transpose) + gem_lane_kernel (persistent, "
                                         "all cycles) + from_lanes_kernel + unpermute_kernel") if lanes else
-                                       "per step: 1 gem_step_kernel (persistent, all cycles) + 1 unpermute_kernel",
+                                       ("per step: 1 %s (persistent, all cycles) + 1 unpermute_kernel" %
+                                        ("gem_word_kernel" if main_res["sim_info"].get("words") else "gem_step_kernel")),
                 "timed_region": "per step: input staging (D2D copy of the step's PI words"
                                 + (" + lane transpose" if lanes else "") + "), gem_step, PO unpermute",
                 "e2e": main_res.get("e2e"), "roofline": roof, "parity": main_res.get("parity"),

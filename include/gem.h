@@ -199,6 +199,11 @@ int gem_write_ram(gem_sim* sim, uint32_t ram_id, uint32_t stream, const uint32_t
  * among `grid` co-resident CTAs (grid <= 1024).  Allocates and frees its own
  * device memory on `device`. */
 int gem_bench_floor(int device, uint32_t grid, uint32_t iters, double* layer_clk, double* barrier_clk);
+/* *step_clk = SM clocks of a minimal word-mode step (GEM_F_NO_WORDS off, blobs
+ * mapped with words=1): block barrier, two operand loads per thread, AND with
+ * inversions, result store, on one CTA -- the per-step term of word mode's
+ * latency floor.  Measurement helper, not part of the simulation path. */
+int gem_bench_floor_step(int device, uint32_t iters, double* step_clk);
 
 /* Device time (CUDA events on the launch stream) of the last gem_step kernel. */
 int gem_last_step_ms(gem_sim* sim, float* ms);

@@ -1077,6 +1077,31 @@ __global__ void __launch_bounds__(GEM_THREADS, 1) floor_layer_kernel(unsigned lo
   if (x == 0x9E3779B9u) out[1] = x;   // keep the chain live
 }
 
+// Minimal word-mode step (gem_words.cuh): after the block barrier every thread
+// loads two operand words (bank-conflict-free), computes the AND with its
+// inversions and stores the result, then the next barrier -- the dependent
+// chain every step traverses however few ops it has.  Op words stay in
+// registers (the kernel prefetches them off the chain).
+__global__ void __launch_bounds__(GEM_THREADS, 1) floor_step_kernel(unsigned long long* out, uint32_t iters) {
+  __shared__ uint32_t S[2048];
+  const uint32_t tid = threadIdx.x;
+  for (uint32_t i = tid; i < 2048; i += GEM_THREADS) S[i] = i * 2654435761u;
+  __syncthreads();
+  const uint32_t base = smem_u32(S);
+  uint32_t a_off = 4 * (tid & 1023u), b_off = 4 * (1024 + ((tid + 7) & 1023u));
+  const unsigned long long t0 = clock64();
+  for (uint32_t it = 0; it < iters; it++) {
+    const uint32_t a = lds(base + a_off), b = lds(base + b_off);
+    const uint32_t r = (a ^ it) & (b ^ (it >> 1));
+    sts(base + 4 * (((tid + 32 * (it & 7)) & 1023u) + 1024 * (it & 1)), r);
+    __syncthreads();
+    a_off ^= 4096u;   // next step reads the words this one wrote
+    b_off ^= 4096u;
+  }
+  const unsigned long long t1 = clock64();
+  if (tid == 0) out[0] = (t1 - t0) / iters;
+}
+
 // Grid barrier round trip at a given grid size (same grid_sync as the kernels).
 __global__ void __launch_bounds__(GEM_THREADS, 1) floor_barrier_kernel(const KParams kp, unsigned long long* out,
                                                                        uint32_t iters) {
@@ -2120,6 +2145,22 @@ int gem_bench_floor(int device, uint32_t grid, uint32_t iters, double* layer_clk
   cudaFree(d_out);
   cudaFree(d_bar);
   cudaFree(d_err);
+  return GEM_OK;
+}
+
+int gem_bench_floor_step(int device, uint32_t iters, double* step_clk) {
+  gem_sim* sim = nullptr;
+  if (!step_clk || !iters) return fail(GEM_E_INVAL, "bad floor request");
+  CK(cudaSetDevice(device));
+  unsigned long long* d_out = nullptr;
+  CK(dalloc(&d_out, 64));
+  unsigned long long h = 0;
+  floor_step_kernel<<<1, GEM_THREADS>>>(d_out, 64);
+  floor_step_kernel<<<1, GEM_THREADS>>>(d_out, iters);
+  CK(cudaGetLastError());
+  CK(cudaMemcpy(&h, d_out, 8, cudaMemcpyDeviceToHost));
+  cudaFree(d_out);
+  *step_clk = (double)h;
   return GEM_OK;
 }
 

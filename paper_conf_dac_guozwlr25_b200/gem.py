@@ -28,7 +28,7 @@ ERRORS = {-1: "GEM_E_INVAL", -2: "GEM_E_FORMAT", -3: "GEM_E_CUDA", -4: "GEM_E_NO
           -6: "GEM_E_UNSUPPORTED"}
 EXPORTS = ["gem_load_program", "gem_info_get", "gem_set_inputs", "gem_step", "gem_read_outputs",
            "gem_read_state", "gem_write_state", "gem_read_state_trace", "gem_read_digests", "gem_read_ram",
-           "gem_write_ram", "gem_last_step_ms", "gem_read_profile", "gem_read_activity", "gem_bench_floor", "gem_free", "gem_last_error",
+           "gem_write_ram", "gem_last_step_ms", "gem_read_profile", "gem_read_activity", "gem_bench_floor", "gem_bench_floor_step", "gem_free", "gem_last_error",
            "gem_dist_owner", "gem_dist_export", "gem_dist_ipc_handles", "gem_dist_ipc_open", "gem_dist_connect"]
 GEM_DIST_MAX = 8
 GEM_DIST_IPC_BYTES = 328
@@ -149,6 +149,16 @@ def bench_floor(device: int = 0, grid: int = 148, iters: int = 2000):
     if lib.gem_bench_floor(device, grid, iters, ctypes.byref(a), ctypes.byref(b)) != 0:
         raise GemError(lib.gem_last_error().decode())
     return a.value, b.value
+
+
+def bench_floor_step(device: int = 0, iters: int = 4000) -> float:
+    """Minimal word-mode step clocks (gem_bench_floor_step) measured on `device`."""
+    lib = load_library()
+    lib.gem_bench_floor_step.argtypes = [ctypes.c_int, ctypes.c_uint32, ctypes.POINTER(ctypes.c_double)]
+    a = ctypes.c_double()
+    if lib.gem_bench_floor_step(device, iters, ctypes.byref(a)) != 0:
+        raise GemError(lib.gem_last_error().decode())
+    return a.value
 
 
 class Simulator:

@@ -58,6 +58,14 @@ class BlobInfo:
     word_ops: int = 0
     word_program_bytes: int = 0
     word_max_state: int = 0
+    word_part_steps: list = None   # steps of each partition's word program
+
+    def stage_max_word_steps(self) -> list:
+        """Deepest word program (steps) of each stage: the critical step chain."""
+        out = [0] * max(1, self.n_stages)
+        for st, ns in zip(self.part_stage or [], self.word_part_steps or []):
+            out[st] = max(out[st], ns)
+        return out
 
     def stage_max_layers(self) -> list:
         """Deepest partition (layers) of each stage: a lower bound on the layers
@@ -90,6 +98,7 @@ class BlobInfo:
         d.pop("part_layers")
         d.pop("part_cost", None)
         d.pop("part_stage", None)
+        d.pop("word_part_steps", None)
         d.update(replication=self.replication, synth_growth=self.synth_growth, slot_util=self.slot_util,
                  bytes_per_and=self.bytes_per_and,
                  levels_per_layer=self.max_levels / max(1, self.max_layers))
@@ -104,6 +113,11 @@ def blob_info(blob: bytes) -> BlobInfo:
     u64 = lambda k: h[k + "_LO"] | (h[k + "_HI"] << 32)
     np_ = h["N_PARTS"]
     pt = w[h["OFF_PARTS"]:h["OFF_PARTS"] + GP_WORDS * np_].reshape(np_, GP_WORDS)
+    word_part_steps = []
+    if h["HAS_WORDS"]:
+        for p in range(np_):
+            wp = h["OFF_WORD_PROG"] + int(pt[p, 15])
+            word_part_steps.append(int(w[wp + 2]))
     lane_ops = lane_steps = 0
     if h["HAS_LANES"]:
         for p in range(np_):
@@ -124,4 +138,4 @@ def blob_info(blob: bytes) -> BlobInfo:
                     lane_ops=lane_ops, lane_steps=lane_steps, has_words=bool(h["HAS_WORDS"]),
                     word_max_steps=h["WORD_MAX_STEPS"], word_total_steps=h["WORD_TOTAL_STEPS"],
                     word_ops=u64("WORD_OPS"), word_program_bytes=4 * u64("WORD_PROG_WORDS"),
-                    word_max_state=h["WORD_MAX_STATE"])
+                    word_max_state=h["WORD_MAX_STATE"], word_part_steps=word_part_steps)

@@ -27,8 +27,8 @@ for s in "$@"; do
     ncu) C=${b:-0}; [ "$C" = 0 ] && C=$(python -c "print({'c4':200,'c5':100}.get('$a',1000))")
          timeout 900 ncu --metrics gpu__time_duration.sum --clock-control none -c 400 --csv --log-file $O/${TAG}_launches_$a.csv \
            python bench.py --workload $a --steps 2 --warmup 3 --cycles $C --no-cpu-baseline --no-batched > /dev/null 2>&1
-         K=$(python -c "print('gem_lane_kernel' if '$a'=='c5' else 'gem_step_kernel')")
-         timeout 1500 ncu --set full --clock-control none --import-source on -k regex:$K -s 1 -c 1 -f -o $O/${TAG}_ncu_$a \
+         K=$(python -c "print('gem_lane_kernel' if '$a'=='c5' else 'gem_(step|word)_kernel')")
+         timeout 1500 ncu --set full --clock-control none --import-source on -k "regex:$K" -s 1 -c 1 -f -o $O/${TAG}_ncu_$a \
            python scripts/prof_run.py --cfg $a --cycles $C --streams $( [ "$a" = c5 ] && echo 4096 || echo 1 ) > /dev/null 2>&1
          python scripts/ncu_summary.py $O/${TAG}_launches_$a.csv $O/${TAG}_ncu_$a.ncu-rep $O/${TAG}_ncu_$a $C > /dev/null 2>&1
          head -12 $O/${TAG}_ncu_$a.md ;;
