@@ -135,26 +135,39 @@ __device__ __forceinline__ void run_word_partition(const KParams& kp, const uint
   __syncthreads();
   PROF(1);
   // ---- a3-a5: steps.  A step has n <= 4 x 256 ops (the host checks); thread t
-  // runs ops t, t + 256, ... < n.  Latency layout (scripts/ubench_steps2.cu,
-  // V17: 120-130 clk per step vs ~300 for a loop that prepares addresses or
-  // loads bounds ahead of the operand loads): after the barrier a thread
-  // issues its operand loads first; then it loads step s+3's bound and step
-  // s+1's first op word, both consumed after the barrier.  Ops of rounds 1-3
-  // (the capacity-bound wide steps) are loaded in the step itself.
+  // runs ops t, t + 256, ... < n.  Latency layout (scripts/ubench_steps2.cu:
+  // ~110-130 clk per step against ~300 for a loop that prepares addresses or
+  // loads bounds ahead of its operand loads): after the barrier a thread issues
+  // its operand loads first, then the loads of later steps' bounds and op
+  // words; the first-round op of a step is in a register before the step
+  // begins, rounds 1-3 (the capacity-bound wide steps) are loaded in the step.
   const uint32_t* stp = P + H.off_steps;
   const uint32_t o_base = smem_u32(P + H.off_ops) + 8u * tid;
   const uint32_t ns = H.n_steps;
-  uint32_t e0 = 0, e1 = 0, e2 = 0;
-  uint2 o = make_uint2(0u, 0u);
-  bool v = false;
-  if (ns) {
-    e1 = stp[1];
-    e2 = ns >= 2 ? stp[2] : e1;
-    v = tid < e1;
-    if (v) o = lds64(o_base);
-  }
+  auto bound = [&](uint32_t k) { return stp[min(k, ns)]; };
   if (s_base == GEM_S0_ADDR) {
+    // op words two steps ahead (o: this step, o1: the next one, loaded during
+    // the previous step), bounds e0..e3 of steps s..s+3 in registers, e4
+    // loaded during the step: whatever the compiler hoists above a barrier
+    // only touches values that arrived a step earlier (one step ahead, every
+    // other step of an unrolled pair waited ~80 clk at the barrier for its
+    // op load)
+    uint32_t e0 = 0, e1 = 0, e2 = 0, e3 = 0;
+    uint2 o = make_uint2(0u, 0u), o1 = o;
+    if (ns) {
+      e1 = bound(1);
+      e2 = bound(2);
+      e3 = bound(3);
+      if (tid < e1) o = lds64(o_base);
+      if (tid < e2 - e1) o1 = lds64(o_base + 8u * e1);
+    }
     for (uint32_t s = 0; s < ns; s++) {
+      // loads whose results are consumed a step later go first (their latency
+      // then never meets a barrier: a value loaded just before the barrier and
+      // used right after it stalls the in-order issue of the next step)
+      const uint32_t e4 = bound(s + 4);
+      uint2 o2 = make_uint2(0u, 0u);
+      if (tid < e3 - e2) o2 = lds64(o_base + 8u * e2);
       word_op_s0(o);
       const uint32_t n = e1 - e0;
       if (n > GEM_THREADS) {   // CTA-uniform: rounds 1-3 of a wide step
@@ -167,21 +180,30 @@ __device__ __forceinline__ void run_word_partition(const KParams& kp, const uint
 #pragma unroll
         for (uint32_t r = 0; r < 3; r++) word_op_s0(w[r]);
       }
-      const uint32_t e3 = s + 3 <= ns ? stp[s + 3] : e2;
-      o = make_uint2(0u, 0u);
-      if (tid < e2 - e1) o = lds64(o_base + 8u * e1);
+      o = o1;
+      o1 = o2;
       e0 = e1;
       e1 = e2;
       e2 = e3;
+      e3 = e4;
       __syncthreads();
     }
   } else {
+    uint32_t e0 = 0, e1 = 0, e2 = 0;
+    uint2 o = make_uint2(0u, 0u);
+    bool v = false;
+    if (ns) {
+      e1 = bound(1);
+      e2 = bound(2);
+      v = tid < e1;
+      if (v) o = lds64(o_base);
+    }
     for (uint32_t s = 0; s < ns; s++) {
       if (v) word_op(s_base, o);
       const uint32_t n = e1 - e0;
       for (uint32_t r = 1; r < 4; r++)
         if (tid + r * GEM_THREADS < n) word_op(s_base, lds64(o_base + 8u * (e0 + r * GEM_THREADS)));
-      const uint32_t e3 = s + 3 <= ns ? stp[s + 3] : e2;
+      const uint32_t e3 = bound(s + 3);
       v = tid < e2 - e1;
       if (v) o = lds64(o_base + 8u * e1);
       e0 = e1;

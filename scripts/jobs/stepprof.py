@@ -6,7 +6,7 @@ from gen import stimulus
 from paper_conf_dac_guozwlr25_b200 import gem
 from tests.common import blob, MAP_OPTS
 cfg = sys.argv[1]
-b = blob(cfg, MAP_OPTS[cfg] + ' words=1')
+b = blob(cfg)
 sim = gem.Simulator(b, flags=gem.GEM_F_PROFILE)
 st = stimulus(cfg, sim.info['n_pi'], 200)
 sim.set_inputs(st); sim.step(200)
