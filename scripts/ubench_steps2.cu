@@ -41,7 +41,7 @@ __global__ void __launch_bounds__(NT, 1) k(const uint2* __restrict__ ops, const 
   const uint32_t tid = threadIdx.x;
   for (uint32_t i = tid; i < NW; i += NT) S[i] = i * 2654435761u;
   for (uint32_t i = tid; i < NSTEPS * NT; i += NT) O[i] = ops[i];
-  for (uint32_t i = tid; i <= NSTEPS + 1; i += NT) C[i] = cnt[i];
+  for (uint32_t i = tid; i < 2 * (NSTEPS + 2); i += NT) C[i] = cnt[i];
   __syncthreads();
   const uint32_t sb = (uint32_t)__cvta_generic_to_shared(S);
   const uint32_t ob = (uint32_t)__cvta_generic_to_shared(O) + 8 * tid;
@@ -462,6 +462,88 @@ __global__ void __launch_bounds__(NT, 1) k(const uint2* __restrict__ ops, const 
         t1 = t2;
         __syncthreads();
       }
+    } else if (V == 18) {
+      // V18: the WRD2 loop of gem_words.cuh (uniform 2-level form, table entries
+      // {first, n1 | n2 << 16}, ops two steps ahead, S at shared address 1024)
+      const uint32_t* tab = C;   // host: {first slot, n1} pairs
+      const uint32_t ops_base = (uint32_t)__cvta_generic_to_shared(O);
+      const uint32_t ns = NSTEPS;
+      auto tabe = [&](uint32_t k) { return lds64(cb + 8u * min(k, ns)); };
+      auto op_of = [&](uint2 t) -> uint3 {
+        const uint32_t n1 = t.y & 0xFFFFu, n2 = t.y >> 16;
+        uint3 r = make_uint3(0u, 0u, 0u);
+        if (tid < n1) {
+          const uint2 q = lds64(ops_base + 8u * (t.x + tid));
+          r = make_uint3(q.x, 0x00010001u, q.y);
+        } else if (tid < n1 + n2) {
+          uint4 q;
+          asm volatile("ld.shared.v4.u32 {%0, %1, %2, %3}, [%4];" : "=r"(q.x), "=r"(q.y), "=r"(q.z), "=r"(q.w)
+                       : "r"(ops_base + 8u * (((t.x + n1 + 1u) & ~1u) + 2u * (tid - n1))));
+          r = make_uint3(q.x, q.y, q.z);
+        }
+        return r;
+      };
+      uint2 t0 = tabe(0), t1 = tabe(1), t2 = tabe(2);
+      uint3 o = op_of(t0), o1 = op_of(t1);
+      for (uint32_t s = 0; s < ns; s++) {
+        const uint2 t3 = tabe(s + 3);
+        const uint3 o2 = op_of(t2);
+        {
+          const uint32_t a1 = lds(sb + (o.x & 0xFFFCu)), b1 = lds(sb + ((o.x >> 16) & 0xFFFCu));
+          const uint32_t a2 = lds(sb + (o.y & 0xFFFCu)), b2 = lds(sb + ((o.y >> 16) & 0xFFFCu));
+          const uint32_t u = (a1 ^ o.x) & (b1 ^ (o.x >> 16)), v = (a2 ^ o.y) & (b2 ^ (o.y >> 16));
+          const uint32_t r = (u ^ o.z) & (v ^ (o.z >> 1)), d = o.z & 0xFFFCu;
+          if (d) sts(sb + d, r);
+        }
+        o = o1;
+        o1 = o2;
+        t0 = t1;
+        t1 = t2;
+        t2 = t3;
+        __syncthreads();
+      }
+    } else if (V == 19) {
+      // V18: the WRD2 loop of gem_words.cuh (uniform 2-level form, table entries
+      // {first, n1 | n2 << 16}, ops two steps ahead, S at shared address 1024)
+      const uint32_t* tab = C;   // host: {first slot, n1} pairs
+      const uint32_t ops_base = (uint32_t)__cvta_generic_to_shared(O);
+      const uint32_t ns = NSTEPS;
+      auto tabe = [&](uint32_t k) { return lds64(cb + 8u * min(k, ns)); };
+      const uint32_t wlo = tid & ~31u;
+      auto op_of = [&](uint2 t) -> uint3 {
+        const uint32_t n1 = t.y & 0xFFFFu, n2 = t.y >> 16;
+        uint3 r = make_uint3(0u, 0u, 0u);
+        if (wlo >= n1 + n2) return r;   // warp-uniform: no op for this warp
+        if (tid < n1) {
+          const uint2 q = lds64(ops_base + 8u * (t.x + tid));
+          r = make_uint3(q.x, 0x00010001u, q.y);
+        } else if (tid < n1 + n2) {
+          uint4 q;
+          asm volatile("ld.shared.v4.u32 {%0, %1, %2, %3}, [%4];" : "=r"(q.x), "=r"(q.y), "=r"(q.z), "=r"(q.w)
+                       : "r"(ops_base + 8u * (((t.x + n1 + 1u) & ~1u) + 2u * (tid - n1))));
+          r = make_uint3(q.x, q.y, q.z);
+        }
+        return r;
+      };
+      uint2 t0 = tabe(0), t1 = tabe(1), t2 = tabe(2);
+      uint3 o = op_of(t0), o1 = op_of(t1);
+      for (uint32_t s = 0; s < ns; s++) {
+        const uint2 t3 = tabe(s + 3);
+        const uint3 o2 = op_of(t2);
+        if (wlo < (t0.y & 0xFFFFu) + (t0.y >> 16)) {
+          const uint32_t a1 = lds(sb + (o.x & 0xFFFCu)), b1 = lds(sb + ((o.x >> 16) & 0xFFFCu));
+          const uint32_t a2 = lds(sb + (o.y & 0xFFFCu)), b2 = lds(sb + ((o.y >> 16) & 0xFFFCu));
+          const uint32_t u = (a1 ^ o.x) & (b1 ^ (o.x >> 16)), v = (a2 ^ o.y) & (b2 ^ (o.y >> 16));
+          const uint32_t r = (u ^ o.z) & (v ^ (o.z >> 1)), d = o.z & 0xFFFCu;
+          if (d) sts(sb + d, r);
+        }
+        o = o1;
+        o1 = o2;
+        t0 = t1;
+        t1 = t2;
+        t2 = t3;
+        __syncthreads();
+      }
     } else if (V == 7) {
       // V7: V5 with the loop-carried bound rotated by asm-volatile moves after the stores
       const uint32_t* stp = C;
@@ -519,7 +601,7 @@ __global__ void __launch_bounds__(NT, 1) k(const uint2* __restrict__ ops, const 
 
 template <int V>
 void run(const char* name, const uint2* d_ops, const uint32_t* d_cnt, unsigned long long* d_out, int G) {
-  const size_t smem = NW * 4 + (size_t)(NSTEPS + 1) * NT * 8 + (NSTEPS + 2) * 4;
+  const size_t smem = NW * 4 + (size_t)(NSTEPS + 1) * NT * 8 + 2 * (NSTEPS + 2) * 4;
   cudaFuncSetAttribute(k<V>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
   k<V><<<G, NT, smem>>>(d_ops, d_cnt, d_out, 4);
   k<V><<<G, NT, smem>>>(d_ops, d_cnt, d_out, 40);
@@ -537,7 +619,7 @@ int main() {
     for (int fill : {256, 64}) {
       std::mt19937 rng(3);
       std::vector<uint2> ops((size_t)NSTEPS * NT);
-      std::vector<uint32_t> cnt(NSTEPS + 2, fill);
+      std::vector<uint32_t> cnt(2 * (NSTEPS + 2), fill);
       for (size_t i = 0; i < ops.size(); i++) {
         const uint32_t t = i % NT;
         uint32_t a = 1 + rng() % (NW - 1), b = 1 + rng() % (NW - 1);
@@ -583,6 +665,13 @@ int main() {
         run<15>("V15 V13 unroll 2 (runtime step count)", d_ops, d_cnt, d_out, G);
         run<16>("V16 V13 with operand loads first", d_ops, d_cnt, d_out, G);
         run<17>("V17 packed table, op consumed after barrier", d_ops, d_cnt, d_out, G);
+        {
+          std::vector<uint32_t> t2((NSTEPS + 2) * 2);
+          for (int i = 0; i < NSTEPS + 1; i++) { t2[2 * i] = (uint32_t)(std::min(i, NSTEPS) * fill); t2[2 * i + 1] = i < NSTEPS ? (uint32_t)fill : 0u; }
+          cudaMemcpy(d_cnt, t2.data(), t2.size() * 4, cudaMemcpyHostToDevice);
+        }
+        run<18>("V18 WRD2 loop (uniform 2-level form, 1-level ops)", d_ops, d_cnt, d_out, G);
+        run<19>("V19 V18 + idle warps skip op and prefetch", d_ops, d_cnt, d_out, G);
       }
       cudaFree(d_ops);
       cudaFree(d_cnt);
