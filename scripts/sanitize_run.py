@@ -34,19 +34,23 @@ def check(name, b, path, st, n_streams=1, **kw):
         ok = np.array_equal(po[:64], r["po"])
     else:
         ok = all(np.array_equal(po[s], Oracle(path).run(stims[s])["po"]) for s in range(n_streams))
-    print(f"{name}: {'ok' if ok else 'MISMATCH'} ({sim.info['grid']} CTAs, lanes={sim.info['lanes']})", flush=True)
+    print(f"{name}: {'ok' if ok else 'MISMATCH'} ({sim.info['grid']} CTAs, lanes={sim.info['lanes']}, "
+          f"words={sim.info['words']})", flush=True)
     sim.close()
     return ok
 
 
 ok = True
-ok &= check("c1", blob("c1"), eaig("c1"), stimulus("c1", 35, 60))
+ok &= check("c1 words", blob("c1"), eaig("c1"), stimulus("c1", 35, 60))
+ok &= check("c1 bits", blob("c1"), eaig("c1"), stimulus("c1", 35, 60), flags=gem.GEM_F_NO_WORDS)
 with tempfile.TemporaryDirectory() as d:
     net = circuits.small_G(seed=21, n_and=3000, with_ram=True)
     p = circuits.save(net, d, "g")
     st = stim_random(net.n_pi, 12, 3, reset_pi0_cycles=2)
     for opts, kw in [("parts=4", {}), ("parts=4 stages=2", {}), ("parts=4", {"grid_limit": 2}),
-                     ("parts=4", {"flags": gem.GEM_F_NO_RESIDENT})]:
+                     ("parts=4", {"flags": gem.GEM_F_NO_RESIDENT}), ("parts=4 words=1", {}),
+                     ("parts=4 stages=2 words=1", {}), ("parts=4 words=1", {"grid_limit": 2}),
+                     ("parts=4 words=1", {"grid_limit": 1}), ("parts=1 words=1", {})]:
         ok &= check(f"small {opts} {kw}", compile_file(p, opts), p, st, **kw)
     S = 64
     stl = np.stack([stim_random(net.n_pi, 6, 100 + s, reset_pi0_cycles=2) for s in range(S)])
