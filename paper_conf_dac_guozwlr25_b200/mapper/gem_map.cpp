@@ -1860,7 +1860,46 @@ struct Mapper {
       if (is_ep[i]) { last[i] = INF; continue; }
       for (uint32_t j = coff[i]; j < coff[i + 1]; j++) last[i] = std::max(last[i], step_of[cons[j]]);
     }
-    // ---- words: 0 = constant, 1..n_src = ports, then by liveness with a bank choice
+    // ---- future-read bank budgets (as LAN2): bud[(s * 2 + side) * 32 + r] =
+    // operands of step s (side 0 = A, 1 = B) already placed in bank r.  A
+    // value's bank is chosen where its readers' steps have the fewest, so the
+    // operands of every step spread over the banks (fewer conflict replays).
+    std::vector<uint16_t> bud((size_t)S * 2 * 32, 0);
+    auto readers_cost = [&](uint32_t x, uint32_t r) {
+      uint32_t c = 0;
+      for (uint32_t j = coff[x]; j < coff[x + 1]; j++) {
+        const uint32_t y = cons[j];
+        c += bud[((size_t)step_of[y] * 2 + ((la[y] >> 1) == x ? 0u : 1u)) * 32 + r];
+      }
+      return c;
+    };
+    auto add_readers = [&](uint32_t x, uint32_t r) {
+      for (uint32_t j = coff[x]; j < coff[x + 1]; j++) {
+        const uint32_t y = cons[j];
+        uint16_t& b = bud[((size_t)step_of[y] * 2 + ((la[y] >> 1) == x ? 0u : 1u)) * 32 + r];
+        b = (uint16_t)std::min<uint32_t>(b + 1u, 0xFFFFu);
+      }
+    };
+    // ---- words: 0 = constant, 1..n_src = ports (permuted within aligned blocks
+    // of 32 onto the banks their readers need most; a warp still loads the same
+    // 32 entries), then by liveness with a bank choice
+    for (size_t b0 = 0; b0 < srcs.size(); b0 += 32) {
+      const size_t b1 = std::min(srcs.size(), b0 + 32);
+      std::vector<uint32_t> blk(srcs.begin() + b0, srcs.begin() + b1), out(b1 - b0, UINT32_MAX);
+      std::stable_sort(blk.begin(), blk.end(), [&](uint32_t x, uint32_t y) { return coff[x + 1] - coff[x] > coff[y + 1] - coff[y]; });
+      for (uint32_t x : blk) {
+        size_t best = 0;
+        uint32_t bc = UINT32_MAX;
+        for (size_t j = 0; j < out.size(); j++) {
+          if (out[j] != UINT32_MAX) continue;
+          const uint32_t c = readers_cost(x, (uint32_t)(b0 + j + 1) % 32);
+          if (c < bc) { bc = c; best = j; }
+        }
+        out[best] = x;
+        add_readers(x, (uint32_t)(b0 + best + 1) % 32);
+      }
+      std::copy(out.begin(), out.end(), srcs.begin() + b0);
+    }
     std::vector<int32_t> word(n, -1);
     word[0] = 0;
     uint32_t top = 1;
@@ -1895,37 +1934,53 @@ struct Mapper {
       auto& st = steps[s];
       max_step = std::max<uint32_t>(max_step, (uint32_t)st.size());
       std::stable_sort(st.begin(), st.end(), [&](uint32_t x, uint32_t y) { return rd[x] > rd[y]; });
-      // rounds of 32 slots: take, within a window of the remaining ops, the first
-      // whose A and B banks are still unused by the round (else the first)
+      // rounds of 32 slots (one warp's LDS): take the first remaining op (in
+      // priority order) whose A and B banks the round does not use yet (a word
+      // already in the round is a broadcast, free); if none, the op adding the
+      // fewest same-bank words
       std::vector<uint32_t> rem(st.begin(), st.end()), order;
       order.reserve(st.size());
       while (!rem.empty()) {
-        uint32_t usedA = 0, usedB = 0;
-        std::vector<uint32_t> wA, wB;   // words already in the round (repeats broadcast)
+        uint8_t cntA[32] = {0}, cntB[32] = {0};
+        std::vector<uint32_t> wA, wB;   // words already in the round
         const size_t take = std::min<size_t>(32, rem.size());
         for (size_t k = 0; k < take; k++) {
           size_t pick = 0;
-          const size_t win = std::min<size_t>(rem.size(), 96);
-          for (size_t c = 0; c < win; c++) {
+          uint32_t best = UINT32_MAX;
+          for (size_t c = 0; c < rem.size() && best; c++) {
             const uint32_t x = rem[c], a = lw(la[x]), b = lw(lb[x]);
-            const bool okA = !((usedA >> (a % 32)) & 1u) || std::find(wA.begin(), wA.end(), a) != wA.end();
-            const bool okB = !((usedB >> (b % 32)) & 1u) || std::find(wB.begin(), wB.end(), b) != wB.end();
-            if (okA && okB) { pick = c; break; }
+            const bool inA = std::find(wA.begin(), wA.end(), a) != wA.end();
+            const bool inB = std::find(wB.begin(), wB.end(), b) != wB.end();
+            const uint32_t cost = (inA ? 0u : cntA[a % 32]) + (inB ? 0u : cntB[b % 32]);
+            if (cost < best) { best = cost; pick = c; }
           }
           const uint32_t x = rem[pick];
           rem.erase(rem.begin() + (ptrdiff_t)pick);
           const uint32_t a = lw(la[x]), b = lw(lb[x]);
-          usedA |= 1u << (a % 32);
-          usedB |= 1u << (b % 32);
-          wA.push_back(a);
-          wB.push_back(b);
+          if (std::find(wA.begin(), wA.end(), a) == wA.end()) { wA.push_back(a); cntA[a % 32]++; }
+          if (std::find(wB.begin(), wB.end(), b) == wB.end()) { wB.push_back(b); cntB[b % 32]++; }
           order.push_back(x);
         }
       }
+      uint32_t used = 0;   // banks already stored to by the op's warp (32 slots)
       for (uint32_t j = 0; j < (uint32_t)order.size(); j++) {
         const uint32_t x = order[j];
         const uint32_t a = lw(la[x]), b = lw(lb[x]);
-        const uint32_t w = alloc(j % 32);
+        if (j % 32 == 0) used = 0;
+        // a bank no other op of this warp stores to (conflict-free STS), the
+        // one whose future readers have the fewest operands there, then the
+        // lowest free word
+        uint32_t bres = 0;
+        uint64_t bkey = UINT64_MAX;
+        for (uint32_t r = 0; r < 32; r++) {
+          if ((used >> r) & 1u) continue;
+          const uint64_t fw = freew[r].empty() ? 0xFFFFFFull : *freew[r].begin();
+          const uint64_t key = ((uint64_t)std::min<uint32_t>(readers_cost(x, r), 0xFFFFFF) << 24) | fw;
+          if (key < bkey) { bkey = key; bres = r; }
+        }
+        used |= 1u << bres;
+        add_readers(x, bres);
+        const uint32_t w = alloc(bres);
         word[x] = (int32_t)w;
         if (last[x] != INF) die[std::max(last[x], s)].push_back(w);
         ops.push_back((a * 4 | (la[x] & 1u)) | ((b * 4 | (lb[x] & 1u)) << 16));
