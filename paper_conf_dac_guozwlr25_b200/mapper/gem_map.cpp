@@ -83,6 +83,7 @@ struct Options {
   int lane_m = 1;           // lane mode 2: independent ops per thread and step (1 or 2)
   int words = 0;            // also emit word programs (WRD1, gem_isa.h): the single-stream latency path
   int word_step = 1024;     // word programs: max ops per barrier-separated step
+  int word_chain_probe = 0; // analysis: print step counts with per-thread op chains
   int lane_mode = 2;        // 1: lane program from the boomerang placement ("LANE"); 2: compacted AND
                             // list in barrier-separated steps ("LAN2", gem_isa.h)
   int banks = 1;            // bank-conflict-aware renaming of the state words (rename_state_words)
@@ -131,6 +132,7 @@ static Options parse_opts(const char* s) {
     else if (k == "lane_holes") o.lane_holes = std::max(1, std::stoi(v));
     else if (k == "lane_mode") o.lane_mode = std::max(1, std::min(2, std::stoi(v)));
     else if (k == "words") o.words = std::stoi(v);
+    else if (k == "word_chain_probe") o.word_chain_probe = std::stoi(v);
     else if (k == "word_step") o.word_step = std::max(32, std::min(4 * GEM_THREADS, std::stoi(v)));
     else if (k == "lane_m") o.lane_m = std::max(1, std::min(2, std::stoi(v)));
     else if (k == "lane_k") o.lane_k = std::stoi(v) >= 4 ? 4 : std::stoi(v) >= 2 ? 2 : 1;
@@ -1852,6 +1854,52 @@ struct Mapper {
         }
       }
       for (uint32_t c : next_ready) { ready.push_back(c); std::push_heap(ready.begin(), ready.end(), prio); }
+    }
+    if (opt.word_chain_probe) {
+      // analysis only: steps if a thread could run a chain of up to L ops in one
+      // narrow step (op k+1 takes op k's result from a register, its other
+      // operand from an earlier step)
+      for (uint32_t L : {2u, 4u, 8u}) {
+        std::vector<int32_t> d2(n, -1);
+        std::vector<uint32_t> pend2(n, 0), rdy;
+        uint32_t left = 0;
+        for (uint32_t i = 0; i < n; i++) {
+          if (is_src[i]) continue;
+          d2[i] = INT32_MAX;
+          left++;
+        }
+        auto avail = [&](uint32_t c, int32_t s) { return d2[c] < s; };
+        int32_t s = 0;
+        while (left) {
+          rdy.clear();
+          for (uint32_t i = 0; i < n; i++)
+            if (d2[i] == INT32_MAX && avail(la[i] >> 1, s) && avail(lb[i] >> 1, s)) rdy.push_back(i);
+          std::stable_sort(rdy.begin(), rdy.end(), [&](uint32_t x, uint32_t y) { return rd[x] > rd[y]; });
+          const bool wide = rdy.size() > 256;
+          if (rdy.size() > (wide ? kStep : 256u)) rdy.resize(wide ? kStep : 256u);
+          for (uint32_t x : rdy) { d2[x] = s; left--; }
+          if (!wide)
+            for (uint32_t x : rdy) {
+              uint32_t cur = x;
+              for (uint32_t k = 1; k < L; k++) {
+                uint32_t best = UINT32_MAX;
+                for (uint32_t j = coff[cur]; j < coff[cur + 1]; j++) {
+                  const uint32_t y = cons[j];
+                  if (d2[y] != INT32_MAX) continue;
+                  const uint32_t o = (la[y] >> 1) == cur ? (lb[y] >> 1) : (la[y] >> 1);
+                  if (o != cur && !avail(o, s)) continue;
+                  if (best == UINT32_MAX || rd[y] > rd[best]) best = y;
+                }
+                if (best == UINT32_MAX) break;
+                d2[best] = s;
+                left--;
+                cur = best;
+              }
+            }
+          s++;
+        }
+        fprintf(stderr, "words chain probe: L=%u steps %d (plain %zu)\n", L, s, steps.size());
+      }
     }
     const uint32_t S = (uint32_t)steps.size();
     const uint32_t INF = UINT32_MAX;

@@ -95,3 +95,42 @@ def test_load_program_validates_blob():
     assert bad(lambda x: x.__setitem__(po, 0))[0] == -2                           # partition magic
     cfg0 = _load_rc(b, n_streams=0)[0]
     assert cfg0 == -1                                                             # n_streams = 0
+
+
+def test_load_program_validates_word_programs():
+    """Word programs (gem_isa.h WRD1) are bounds-checked on load: an op, output or
+    port entry outside the state / its region, a broken step table or a step
+    above 1024 ops is GEM_E_FORMAT before any CUDA call."""
+    import numpy as np
+    from tests.common import blob
+    from paper_conf_dac_guozwlr25_b200.isa import GH
+    b = blob("c1")
+    w = np.frombuffer(b, np.uint32).copy()
+    H = {k: i for i, k in enumerate(GH)}
+    assert w[H["HAS_WORDS"]] == 1
+    wp = int(w[H["OFF_WORD_PROG"]] + w[w[H["OFF_PARTS"]] + 15])    # partition 0's word program
+    # WPH_* word indices
+    N_GREAD, N_STEPS, N_OPS, N_OUT, STATE, OFF_STEPS, OFF_OPS, OFF_OUT, OFF_GREAD = 1, 2, 3, 4, 6, 7, 8, 9, 11
+    ops = wp + int(w[wp + OFF_OPS])
+    stp = wp + int(w[wp + OFF_STEPS])
+    out = wp + int(w[wp + OFF_OUT])
+    gr = wp + int(w[wp + OFF_GREAD])
+    lim = int(w[wp + STATE]) * 4
+
+    def rc_of(mut):
+        x = w.copy()
+        mut(x)
+        rc, msg, h = _load_rc(x.tobytes())
+        assert h is None
+        return rc, msg
+
+    assert rc_of(lambda x: x.__setitem__(wp, 0))[0] == -2                         # magic
+    assert rc_of(lambda x: x.__setitem__(ops + 1, lim))[0] == -2                  # op destination
+    assert rc_of(lambda x: x.__setitem__(ops + 1, 0))[0] == -2                    # writes word 0
+    assert rc_of(lambda x: x.__setitem__(ops, (lim & 0xFFFC) | ((lim & 0xFFFC) << 16)))[0] == -2   # operand
+    assert rc_of(lambda x: x.__setitem__(stp + 1, 1 << 20))[0] == -2              # step table
+    n_out = int(w[wp + N_OUT])
+    assert rc_of(lambda x: x.__setitem__(out, (9 << 24) | 0))[0] == -2            # output region
+    assert rc_of(lambda x: x.__setitem__(out + n_out, lim))[0] == -2              # output source
+    assert rc_of(lambda x: x.__setitem__(gr, (1 << 24) | (1 << 23)))[0] == -2     # port beyond Q
+    assert rc_of(lambda x: x.__setitem__(wp + STATE, 1 << 20))[0] == -2           # state size
