@@ -84,6 +84,8 @@ struct Options {
   int words = 0;            // also emit word programs (WRD1, gem_isa.h): the single-stream latency path
   int word_step = 1024;     // word programs: max ops per barrier-separated step
   int word_chain_probe = 0; // analysis: print step counts with per-thread op chains
+  int word_sched = 1;       // word programs: 1 = balanced (slack-aware) steps, 0 = greedy ASAP
+  int word_fill = GEM_THREADS;  // balanced scheduling: ops per step before slack ops wait
   int lane_mode = 2;        // 1: lane program from the boomerang placement ("LANE"); 2: compacted AND
                             // list in barrier-separated steps ("LAN2", gem_isa.h)
   int banks = 1;            // bank-conflict-aware renaming of the state words (rename_state_words)
@@ -132,6 +134,8 @@ static Options parse_opts(const char* s) {
     else if (k == "lane_holes") o.lane_holes = std::max(1, std::stoi(v));
     else if (k == "lane_mode") o.lane_mode = std::max(1, std::min(2, std::stoi(v)));
     else if (k == "words") o.words = std::stoi(v);
+    else if (k == "word_sched") o.word_sched = std::stoi(v);
+    else if (k == "word_fill") o.word_fill = std::max(32, std::min(4 * GEM_THREADS, std::stoi(v)));
     else if (k == "word_chain_probe") o.word_chain_probe = std::stoi(v);
     else if (k == "word_step") o.word_step = std::max(32, std::min(4 * GEM_THREADS, std::stoi(v)));
     else if (k == "lane_m") o.lane_m = std::max(1, std::min(2, std::stoi(v)));
@@ -1834,11 +1838,33 @@ struct Mapper {
     std::vector<std::vector<uint32_t>> steps;
     std::vector<uint32_t> next_ready;
     uint32_t done = 0;
+    // balanced scheduling (word_sched=1): an op with slack need not run in the
+    // first step it is ready in.  Steps are as many as the critical path (Lc =
+    // 1 + max rd over ops); op x must run by step Lc - 1 - rd[x] (its ALAP
+    // step).  Each step takes every ready op at its deadline, then fills up to
+    // one round (256 ops) with the ready ops of least slack; only a step whose
+    // deadlines exceed that goes wide.  Fewer capacity-bound wide steps, same
+    // number of steps.
+    uint32_t Lc = 0;
+    for (uint32_t i = 0; i < n; i++)
+      if (!is_src[i]) Lc = std::max(Lc, rd[i] + 1);
     while (done < n_ops) {
       if (ready.empty()) throw std::runtime_error("words: scheduling stalled");
       steps.emplace_back();
       auto& st = steps.back();
-      while (!ready.empty() && st.size() < kStep) {
+      if (opt.word_sched) {
+        const uint32_t s = (uint32_t)steps.size() - 1;
+        // ready ops by deadline (ALAP step = Lc - 1 - rd), most urgent first
+        std::sort(ready.begin(), ready.end(), [&](uint32_t x, uint32_t y) { return rd[x] != rd[y] ? rd[x] > rd[y] : x < y; });
+        size_t take = 0;
+        while (take < ready.size() && take < kStep && Lc - 1 - rd[ready[take]] <= s) take++;   // due now
+        const size_t fill = std::max<size_t>(take, std::min<size_t>((size_t)opt.word_fill, kStep));
+        while (take < ready.size() && take < fill) take++;
+        st.assign(ready.begin(), ready.begin() + (ptrdiff_t)take);
+        ready.erase(ready.begin(), ready.begin() + (ptrdiff_t)take);
+        std::make_heap(ready.begin(), ready.end(), prio);
+      }
+      while (!opt.word_sched && !ready.empty() && st.size() < kStep) {
         std::pop_heap(ready.begin(), ready.end(), prio);
         st.push_back(ready.back());
         ready.pop_back();
