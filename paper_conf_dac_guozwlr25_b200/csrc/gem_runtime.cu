@@ -1508,7 +1508,7 @@ static int plan_launch_words(gem_sim* sim, uint32_t grid_limit) {
   if (bytes > (uint64_t)optin) return fail(GEM_E_UNSUPPORTED, "word programs do not fit in shared memory");
   CK(cudaFuncSetAttribute(word_kernel_for(sim), cudaFuncAttributeMaxDynamicSharedMemorySize, (int)bytes));
   int occ = 0;
-  CK(cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ, word_kernel_for(sim), GEM_THREADS, (size_t)bytes));
+  CK(cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ, word_kernel_for(sim), GEM_WORD_THREADS, (size_t)bytes));
   if (occ < 1) return fail(GEM_E_UNSUPPORTED, "word kernel not resident");
   sim->blocks_per_sm = 1;
   sim->grid = grid;
@@ -2106,7 +2106,7 @@ int gem_step(gem_sim* sim, uint64_t ncycles) {
   void* args[] = {&kp};
   CK(cudaEventRecord(sim->ev0, sim->stream));
   CK(cudaLaunchCooperativeKernel(sim->words ? word_kernel_for(sim) : sim->lanes ? lane_kernel_for(sim->lane_groups, sim->lane_v2, sim->lane_m) : step_kernel_for(sim),
-                                 dim3(sim->grid), dim3(GEM_THREADS), args, sim->smem_bytes, sim->stream));
+                                 dim3(sim->grid), dim3(sim->words ? GEM_WORD_THREADS : GEM_THREADS), args, sim->smem_bytes, sim->stream));
   CK(cudaEventRecord(sim->ev1, sim->stream));
   sim->in_head += (uint32_t)ncycles;
   sim->cycle += ncycles;

@@ -22,6 +22,10 @@
 // ~6 levels; a step ~0.12K clk advances it by one).
 
 #define GEM_WORD_RAMP (4 * GEM_MAX_RAMS_PER_PART)
+#ifndef GEM_WORD_THREADS
+#define GEM_WORD_THREADS 256   /* threads of a word-mode CTA (a step's round) */
+#endif
+#define GEM_WORD_WARPS (GEM_WORD_THREADS / 32)
 #define GEM_WORD_PORT_REGS 4   /* port entries per thread kept in registers (fast path) */
 
 // Header fields of a word program (loaded once per launch on the fast path).
@@ -101,7 +105,7 @@ __device__ __forceinline__ void run_word_partition(const KParams& kp, const uint
     }
 #pragma unroll
     for (uint32_t u = 0; u < GEM_WORD_PORT_REGS; u++)
-      if (wp.g[u] != ~0u) sts(s_base + 4u * (1u + u * GEM_THREADS + tid), v[u] >> (wp.g[u] & 31u));
+      if (wp.g[u] != ~0u) sts(s_base + 4u * (1u + u * GEM_WORD_THREADS + tid), v[u] >> (wp.g[u] & 31u));
     // next cycle's PI words (consumed at the top of cycle c+1)
 #pragma unroll
     for (uint32_t u = 0; u < GEM_WORD_PORT_REGS; u++)
@@ -110,11 +114,11 @@ __device__ __forceinline__ void run_word_partition(const KParams& kp, const uint
   } else {
     const uint32_t* gr = P + H.off_gread;
     constexpr uint32_t GU = 4;
-    for (uint32_t k0 = 0; k0 < H.n_gread; k0 += GU * GEM_THREADS) {
+    for (uint32_t k0 = 0; k0 < H.n_gread; k0 += GU * GEM_WORD_THREADS) {
       uint32_t v[GU], sh[GU];
 #pragma unroll
       for (uint32_t u = 0; u < GU; u++) {
-        const uint32_t k = k0 + u * GEM_THREADS + tid;
+        const uint32_t k = k0 + u * GEM_WORD_THREADS + tid;
         v[u] = 0u;
         sh[u] = 0u;
         if (k < H.n_gread) {
@@ -125,7 +129,7 @@ __device__ __forceinline__ void run_word_partition(const KParams& kp, const uint
       }
 #pragma unroll
       for (uint32_t u = 0; u < GU; u++) {
-        const uint32_t k = k0 + u * GEM_THREADS + tid;
+        const uint32_t k = k0 + u * GEM_WORD_THREADS + tid;
         if (k < H.n_gread) sts(s_base + 4u * (1u + k), v[u] >> sh[u]);
       }
     }
@@ -174,12 +178,12 @@ __device__ __forceinline__ void run_word_partition(const KParams& kp, const uint
       if (tid < e3 - e2) o2 = lds64(o_base + 8u * e2);
       word_op_s0(o);
       const uint32_t n = e1 - e0;
-      if (n > GEM_THREADS) {   // CTA-uniform: rounds 1-3 of a wide step
+      if (n > GEM_WORD_THREADS) {   // CTA-uniform: rounds 1-3 of a wide step
         uint2 w[3];
 #pragma unroll
         for (uint32_t r = 0; r < 3; r++) {
           w[r] = make_uint2(0u, 0u);
-          if (tid + (r + 1) * GEM_THREADS < n) w[r] = lds64(o_base + 8u * (e0 + (r + 1) * GEM_THREADS));
+          if (tid + (r + 1) * GEM_WORD_THREADS < n) w[r] = lds64(o_base + 8u * (e0 + (r + 1) * GEM_WORD_THREADS));
         }
 #pragma unroll
         for (uint32_t r = 0; r < 3; r++) word_op_s0(w[r]);
@@ -206,7 +210,7 @@ __device__ __forceinline__ void run_word_partition(const KParams& kp, const uint
       if (v) word_op(s_base, o);
       const uint32_t n = e1 - e0;
       for (uint32_t r = 1; r < 4; r++)
-        if (tid + r * GEM_THREADS < n) word_op(s_base, lds64(o_base + 8u * (e0 + r * GEM_THREADS)));
+        if (tid + r * GEM_WORD_THREADS < n) word_op(s_base, lds64(o_base + 8u * (e0 + r * GEM_WORD_THREADS)));
       const uint32_t e3 = bound(s + 3);
       v = tid < e2 - e1;
       if (v) o = lds64(o_base + 8u * e1);
@@ -220,7 +224,7 @@ __device__ __forceinline__ void run_word_partition(const KParams& kp, const uint
   // ---- a6: endpoint commit (one warp ballot per owned output word)
   const uint32_t* od = P + H.off_out;
   const uint32_t* os = od + H.n_out;
-  for (uint32_t o = warp; o < H.n_out; o += GEM_WARPS) {
+  for (uint32_t o = warp; o < H.n_out; o += GEM_WORD_WARPS) {
     const uint32_t e = os[o * 32 + lane];
     const uint32_t bit = (lds(s_base + (e & 0xFFFCu)) ^ e) & 1u;
     const uint32_t v = __ballot_sync(0xFFFFFFFFu, bit);
@@ -243,7 +247,7 @@ __device__ __forceinline__ void run_word_partition(const KParams& kp, const uint
   if (H.n_ram) {
     __syncthreads();
     const uint32_t* rr = P + H.off_ram;
-    for (uint32_t r = tid; r < H.n_ram; r += GEM_THREADS) {
+    for (uint32_t r = tid; r < H.n_ram; r += GEM_WORD_THREADS) {
       const uint32_t* rp = ramp + 4 * r;
       const uint32_t id = rr[4 * r];
       const uint32_t ra = rp[GEM_PORT_RADDR] & (GEM_RAM_WORDS - 1);
@@ -264,7 +268,7 @@ __device__ __forceinline__ void run_word_partition(const KParams& kp, const uint
 // LOC: single-CTA launch of one stream (every flop and RAM-read word is
 // written by this CTA), so Q / RD are read from a shared-memory copy.
 template <bool LOC>
-__global__ void __launch_bounds__(GEM_THREADS, 1) gem_word_kernel(const KParams kp) {
+__global__ void __launch_bounds__(GEM_WORD_THREADS, 1) gem_word_kernel(const KParams kp) {
   extern __shared__ __align__(16) uint32_t smem[];
   // layout (words): S[state_words] | area[area_words] | ramp[GEM_WORD_RAMP] | res_p[16] | res_off[16] |
   //                 res_n[16] | wl cache | mbar[2 x u64] | loc[2][loc_words]
@@ -319,7 +323,7 @@ __global__ void __launch_bounds__(GEM_THREADS, 1) gem_word_kernel(const KParams 
   if (n_res) mbar_wait(mbar, 0);
   if (LOC) {
     const uint32_t c0 = (uint32_t)(kp.t0 & 1u);
-    for (uint32_t k = tid; k < kp.loc_words; k += GEM_THREADS)
+    for (uint32_t k = tid; k < kp.loc_words; k += GEM_WORD_THREADS)
       loc[c0 * kp.loc_words + k] = k < kp.q_words ? __ldcg(kp.q + (size_t)c0 * kp.n_streams * kp.q_words + k)
                                                   : __ldcg(kp.rd + (size_t)c0 * kp.n_streams * kp.n_rams + (k - kp.q_words));
     __syncthreads();
@@ -330,12 +334,12 @@ __global__ void __launch_bounds__(GEM_THREADS, 1) gem_word_kernel(const KParams 
   // fast path: one stage, one work item, <= 1024 ports (every per-cycle constant
   // in registers; C1-C3 single stream)
   const WordHdr H1 = word_hdr(area);
-  const bool fast = kp.n_stages == 1 && n_items == 1 && H1.n_gread <= GEM_WORD_PORT_REGS * GEM_THREADS;
+  const bool fast = kp.n_stages == 1 && n_items == 1 && H1.n_gread <= GEM_WORD_PORT_REGS * GEM_WORD_THREADS;
   if (fast) {
     const uint2 it = reinterpret_cast<const uint2*>(wlc + 32)[0];
 #pragma unroll
     for (uint32_t u = 0; u < GEM_WORD_PORT_REGS; u++) {
-      const uint32_t k = u * GEM_THREADS + tid;
+      const uint32_t k = u * GEM_WORD_THREADS + tid;
       wp.g[u] = k < H1.n_gread ? area[H1.off_gread + k] : ~0u;
       wp.pv[u] = 0u;
     }
