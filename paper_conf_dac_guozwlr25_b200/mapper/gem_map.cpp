@@ -86,6 +86,7 @@ struct Options {
   int word_chain_probe = 0; // analysis: print step counts with per-thread op chains
   int word_sched = 1;       // word programs: 1 = balanced (slack-aware) steps, 0 = greedy ASAP
   int word_fill = GEM_THREADS;  // balanced scheduling: ops per step before slack ops wait
+  int word_spread = 0;      // balanced scheduling: every partition spreads over the design depth (measured slower)
   int lane_mode = 2;        // 1: lane program from the boomerang placement ("LANE"); 2: compacted AND
                             // list in barrier-separated steps ("LAN2", gem_isa.h)
   int banks = 1;            // bank-conflict-aware renaming of the state words (rename_state_words)
@@ -135,6 +136,7 @@ static Options parse_opts(const char* s) {
     else if (k == "lane_mode") o.lane_mode = std::max(1, std::min(2, std::stoi(v)));
     else if (k == "words") o.words = std::stoi(v);
     else if (k == "word_sched") o.word_sched = std::stoi(v);
+    else if (k == "word_spread") o.word_spread = std::stoi(v);
     else if (k == "word_fill") o.word_fill = std::max(32, std::min(4 * GEM_THREADS, std::stoi(v)));
     else if (k == "word_chain_probe") o.word_chain_probe = std::stoi(v);
     else if (k == "word_step") o.word_step = std::max(32, std::min(4 * GEM_THREADS, std::stoi(v)));
@@ -1848,6 +1850,11 @@ struct Mapper {
     uint32_t Lc = 0;
     for (uint32_t i = 0; i < n; i++)
       if (!is_src[i]) Lc = std::max(Lc, rd[i] + 1);
+    // one stage: every partition may use as many steps as the deepest one has
+    // (the design's depth); a shallow partition with many ops then spreads
+    // them thinner instead of running extra rounds in fewer steps -- the cycle
+    // is the slowest partition's, and an extra round costs more than a step
+    if (opt.word_spread && opt.stages == 1) Lc = std::max(Lc, G.max_level + 1);
     while (done < n_ops) {
       if (ready.empty()) throw std::runtime_error("words: scheduling stalled");
       steps.emplace_back();
