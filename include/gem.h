@@ -76,6 +76,8 @@ extern "C" {
  * bit-packed path; GEM_F_ACTIVITY and split designs (dist_world > 1) always
  * use it. */
 #define GEM_F_NO_WORDS 0x100u
+/* (GEM_F_NO_RESIDENT applies to the bit-packed path; word programs are always
+ * resident in shared memory.) */
 
 typedef struct gem_sim gem_sim; /* opaque, owned by the library */
 

@@ -12,8 +12,21 @@
  * gem_load_program().
  *
  * opts: space separated key=value pairs, e.g. "parts=148 stages=2 threads=8":
- *   parts, part_size, threads, leafcap, stages (1|2), cut_level, merge,
- *   max_state_words, cap_slack, verbose.
+ *   partitioning: parts, part_size, max_parts, key, km1, km1_pins, km1_slack,
+ *     merge, merge_cap, merge_ratio, refine, refine_ratio, stages (1|2),
+ *     cut_level;
+ *   synthesis: synth (0 strash, 1 + AND balancing, 2 + chain
+ *     lookahead), chain_min, chain_slack;
+ *   boomerang layers: levels, leafcap, max_warps, banks, max_state_words,
+ *     cap_slack;
+ *   lane programs (batched streams): lanes=1, lane_mode, lane_k, lane_m,
+ *     lane_words, lane_banks, lane_holes;
+ *   word programs (the single-stream path, gem_isa.h WRD1): words=1,
+ *     word_step (ops per step, <= 1024), word_sched (1 balanced, 0 ASAP),
+ *     word_fill, word_spread, word_chain_probe (analysis output only);
+ *   threads, verbose.
+ *   A blob gets word programs only if every partition's fits in 16K state
+ *   words; the runtime then also needs them to fit in shared memory.
  *
  * Ownership: *blob is malloc'ed by the library; release with gem_free_blob().
  * Errors: 0 on success; -1 bad argument / unreadable file, -2 parse or mapping
