@@ -1296,7 +1296,9 @@ static double build_worklists(const gem_sim* sim, uint32_t G, std::vector<uint32
     // a scheduling unit = `run` consecutive stream groups of one partition, kept
     // together on one CTA (lane mode: consecutive items then share the
     // partition's input-port list and program in L1/L2)
-    const uint32_t run = sim->lanes ? (sim->cfg.lane_run ? sim->cfg.lane_run : 4u) : 1u;
+    // (word mode: every stream of a partition on one CTA, so its program is
+    // resident once)
+    const uint32_t run = sim->lanes ? (sim->cfg.lane_run ? sim->cfg.lane_run : 4u) : sim->words ? sim->n_streams : 1u;
     std::vector<std::pair<uint32_t, uint2>> its;
     its.reserve((size_t)np * sim->n_streams);
     for (uint32_t st = 0; st < sim->n_streams; st += sim->group * run)

@@ -136,3 +136,29 @@ def test_c3_word_mode_2000_cycles_checkpoints(gem):
     assert np.array_equal(sim.read_state()[0], o.get_state())
     for ram in range(o.n_rams):
         assert np.array_equal(sim.read_ram(ram), o.get_ram(ram))
+
+
+def test_c2_two_stage_word_mode(gem):
+    """C2 mapped as two stages (P:109 cut words exchanged through the second
+    grid barrier) in word mode: PO and flops every cycle vs the oracle."""
+    from tests.common import MAP_OPTS
+    b = blob("c2", MAP_OPTS["c2"] + " stages=2")
+    sim = _full_parity(gem, eaig("c2"), b, stimulus("c2", 128, 600), chunks=(250,))
+    assert sim.info["words"] == 1 and sim.info["n_stages"] == 2
+
+
+def test_c3_word_mode_four_streams(gem):
+    """Four independent streams of C3 in word mode (several work items per
+    CTA, the generic item loop): every stream's PO trace and final flops equal
+    its own oracle run."""
+    S, T = 4, 120
+    st = np.stack([stimulus("c3", 256, T, seed=300 + s) for s in range(S)])
+    sim = gem.Simulator(blob("c3"), n_streams=S)
+    assert sim.info["words"] == 1
+    po = sim.run(st)
+    q = sim.read_state()
+    for s in range(S):
+        o = Oracle(eaig("c3"))
+        r = o.run(st[s])
+        assert np.array_equal(po[s], r["po"]), s
+        assert np.array_equal(q[s], o.get_state()), s
