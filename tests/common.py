@@ -14,7 +14,7 @@ CACHE = os.environ.get("GEM_CACHE") or os.path.join(ROOT, ".cache")
 
 # mapper options per config (also used by bench.py)
 MAP_OPTS = {"c1": "levels=10 words=1", "c2": "levels=10 key=2 part_size=2000 words=1",
-            "c3": "part_size=8000 max_parts=148 levels=10 key=2 merge_ratio=0.6 merge_cap=12000 words=1",
+            "c3": "part_size=7000 max_parts=148 levels=10 key=2 merge_ratio=0.6 merge_cap=9000 words=1",
             "c4": "stages=1 levels=10 key=2 part_size=22000", "c5": "refine=0 lanes=1 key=2 merge_cap=60000 lane_words=7000 levels=10 merge_ratio=0.5"}
 
 
