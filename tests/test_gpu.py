@@ -342,9 +342,10 @@ def test_golden_worked_examples(gem, name):
     rows = _golden_rows(name + ".expected")
     n_pi = len(rows[0][0])
     st = pack_bits(np.array([r[0] for r in rows], np.uint8)) if n_pi else np.zeros((len(rows), 0), np.uint32)
-    b = compile_file(p)
-    for ns in (1, 3):
+    for opts, ns in [("", 1), ("", 3), ("words=1", 1), ("words=1", 3)]:
+        b = compile_file(p, opts)
         sim = gem.Simulator(b, n_streams=ns)
+        assert sim.info["words"] == (1 if opts else 0)
         if sim.pi_words:
             sim.set_inputs(np.broadcast_to(st, (ns,) + st.shape))
         else:
@@ -371,7 +372,13 @@ def test_wires_constants_and_step0(gem, tmp_path):
         b.output(lit)
     p = circuits.save(b.finish(), str(tmp_path), "wires")
     st = stim_random(5, 200, 11)
-    sim = gem.Simulator(compile_file(p), flags=gem.GEM_F_TRACE_STATE | gem.GEM_F_DIGEST)
+    for opts in ("", "words=1"):
+        _wires_run(gem, p, compile_file(p, opts), st, bool(opts))
+
+
+def _wires_run(gem, p, blob_, st, words):
+    sim = gem.Simulator(blob_, flags=gem.GEM_F_TRACE_STATE | gem.GEM_F_DIGEST)
+    assert sim.info["words"] == int(words)
     sim.set_inputs(st)
     sim.step(0)
     q0 = sim.read_state()
