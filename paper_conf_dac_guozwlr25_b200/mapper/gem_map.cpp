@@ -45,6 +45,7 @@
 #include <string>
 #include <thread>
 #include <unordered_map>
+#include <unordered_set>
 #include <vector>
 
 #include "../csrc/gem_isa.h"
@@ -84,6 +85,7 @@ struct Options {
   int words = 0;            // also emit word programs (WRD1, gem_isa.h): the single-stream latency path
   int word_step = 1024;     // word programs: max ops per barrier-separated step
   int word_chain_probe = 0; // analysis: print step counts with per-thread op chains
+  int word_local_probe = 0; // analysis: print the share of ops computable before the grid barrier
   int word_sched = 1;       // word programs: 1 = balanced (slack-aware) steps, 0 = greedy ASAP
   int word_fill = GEM_THREADS;  // balanced scheduling: ops per step before slack ops wait
   int word_spread = 0;      // balanced scheduling: every partition spreads over the design depth (measured slower)
@@ -138,6 +140,7 @@ static Options parse_opts(const char* s) {
     else if (k == "word_sched") o.word_sched = std::stoi(v);
     else if (k == "word_spread") o.word_spread = std::stoi(v);
     else if (k == "word_fill") o.word_fill = std::max(32, std::min(4 * GEM_THREADS, std::stoi(v)));
+    else if (k == "word_local_probe") o.word_local_probe = std::stoi(v);
     else if (k == "word_chain_probe") o.word_chain_probe = std::stoi(v);
     else if (k == "word_step") o.word_step = std::max(32, std::min(4 * GEM_THREADS, std::stoi(v)));
     else if (k == "lane_m") o.lane_m = std::max(1, std::min(2, std::stoi(v)));
@@ -1887,6 +1890,41 @@ struct Mapper {
         }
       }
       for (uint32_t c : next_ready) { ready.push_back(c); std::push_heap(ready.begin(), ready.end(), prio); }
+    }
+    if (opt.word_local_probe) {
+      // analysis only: ops whose cone reads only this partition's own flop
+      // words, its own RAMs' read data and PIs ("local": computable right after
+      // the partition's own commit, before the grid barrier completes) -- the
+      // work a split-phase barrier (arrive, local steps, wait) could hide
+      std::unordered_set<uint32_t> own_q, own_rd;
+      for (auto& ow : P.outs)
+        if (GEM_GID_REGION(ow.dst) == GEM_R_Q) own_q.insert(GEM_GID_INDEX(ow.dst));
+      for (uint32_t r : P.rams) own_rd.insert(r);
+      std::vector<uint8_t> local(n, 1);
+      uint32_t n_local = 0, n_and_ops = 0, src_local = 0, src_all = 0;
+      for (uint32_t i = 0; i < n; i++) {
+        if (is_src[i]) {
+          if (G.kind[cid[i]] == K_CONST) { local[i] = 1; continue; }
+          const uint32_t gb = G.gbit[cid[i]], reg = gb >> 27, w = (gb >> 5) & 0x3FFFFF;
+          local[i] = reg == GEM_R_PI || (reg == GEM_R_Q && own_q.count(w)) || (reg == GEM_R_RD && own_rd.count(w));
+          src_all++;
+          src_local += local[i];
+          continue;
+        }
+        local[i] = local[la[i] >> 1] && local[lb[i] >> 1];
+        n_and_ops++;
+        n_local += local[i];
+      }
+      // steps of the local sub-schedule (ops only waiting for local ops)
+      uint32_t local_steps = 0;
+      for (uint32_t x = 0; x < n; x++)
+        if (!is_src[x] && local[x]) local_steps = std::max(local_steps, step_of[x] + 1);
+      uint32_t first_remote = UINT32_MAX;
+      for (uint32_t x = 0; x < n; x++)
+        if (!is_src[x] && !local[x]) first_remote = std::min(first_remote, step_of[x]);
+      fprintf(stderr, "words local probe: ops %u local %u (%.2f) ports %u local %u steps %zu first remote-dependent step %u last local step %u\n",
+              n_and_ops, n_local, n_and_ops ? (double)n_local / n_and_ops : 0.0, src_all, src_local, steps.size(),
+              first_remote, local_steps);
     }
     if (opt.word_chain_probe) {
       // analysis only: steps if a thread could run a chain of up to L ops in one
